@@ -101,3 +101,19 @@ ALIASES = {"t": "tiny", "bb": "ee-bert-base", "bl": "ee-bert-large",
 
 def get(name: str) -> ModelConfig:
     return CONFIGS[ALIASES.get(name, name)]
+
+
+def tau_path(cfg: ModelConfig) -> str:
+    import os
+    root = os.path.dirname(os.path.dirname(os.path.abspath(__file__)))
+    return os.path.join(root, "tests", "golden", f"tau_{cfg.name}.json")
+
+
+def tau_for(cfg: ModelConfig):
+    """Per-ramp thresholds: cfg.tau, else the calibrated values committed in
+    tests/golden/tau_<name>.json (written by ``python -m oracle.calibrate``)."""
+    if cfg.tau is not None:
+        return cfg.tau
+    import json
+    with open(tau_path(cfg)) as f:
+        return tuple(json.load(f)["tau"])

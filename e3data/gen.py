@@ -17,6 +17,7 @@ Weight layout is the nn.Linear convention ``[out_features, in_features]``.
 """
 from __future__ import annotations
 
+import os
 import zlib
 from typing import Dict, Iterable
 
@@ -29,10 +30,13 @@ _KIND_INPUT = 0xD47A
 
 
 def bf16_round(x: np.ndarray) -> np.ndarray:
-    """float -> nearest bf16 value (ties to even), returned as float32."""
-    u = np.ascontiguousarray(x, dtype=np.float32).view(np.uint32).astype(np.uint64)
-    u = (u + 0x7FFF + ((u >> 16) & 1)) & 0xFFFF0000
-    return u.astype(np.uint32).view(np.float32)
+    """float -> nearest bf16 value (ties to even), returned as float32.
+
+    uint32 arithmetic cannot wrap for finite inputs (max 0xFF7FFFFF + 0x8000)."""
+    u = np.array(x, dtype=np.float32, copy=True).view(np.uint32)
+    u += np.uint32(0x7FFF) + ((u >> np.uint32(16)) & np.uint32(1))
+    u &= np.uint32(0xFFFF0000)
+    return u.view(np.float32)
 
 
 def bf16_bits(x: np.ndarray) -> np.ndarray:
@@ -111,11 +115,28 @@ def make_weights(cfg: ModelConfig, seed: int = 0):
     }
 
 
-def make_inputs(cfg: ModelConfig, ids: Iterable[int], seed: int = 1) -> np.ndarray:
-    """Embedded inputs X0[i] of shape [n, S, H] (C16: embeddings are upstream)."""
+def make_inputs(cfg: ModelConfig, ids: Iterable[int], seed: int = 1, threads: int = 0) -> np.ndarray:
+    """Embedded inputs X0[i] of shape [n, S, H] (C16: embeddings are upstream).
+
+    Input i is drawn from its own stream (seed, i): any subset regenerates
+    identically.  Large requests are filled by a thread pool (NumPy releases
+    the GIL while filling)."""
     ids = [int(i) for i in ids]
     out = np.empty((len(ids), cfg.seq, cfg.hidden), dtype=np.float32)
-    for k, i in enumerate(ids):
-        g = _rng(seed, _KIND_INPUT, i)
-        out[k] = g.standard_normal(size=(cfg.seq, cfg.hidden), dtype=np.float32)
-    return bf16_round(out)
+
+    def fill(lo, hi):
+        for k in range(lo, hi):
+            g = _rng(seed, _KIND_INPUT, ids[k])
+            g.standard_normal(size=(cfg.seq, cfg.hidden), dtype=np.float32, out=out[k])
+            out[k] = bf16_round(out[k])
+
+    n = len(ids)
+    nt = threads or min(32, len(os.sched_getaffinity(0)))
+    if n * cfg.seq * cfg.hidden < (1 << 22) or nt <= 1:
+        fill(0, n)
+    else:
+        from concurrent.futures import ThreadPoolExecutor
+        step = (n + nt - 1) // nt
+        with ThreadPoolExecutor(nt) as ex:
+            list(ex.map(lambda lo: fill(lo, min(n, lo + step)), range(0, n, step)))
+    return out

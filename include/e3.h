@@ -1,0 +1,239 @@
+/*
+ * e3.h — C ABI of the B200-native E3 early-exit split executor.
+ *
+ * E3 (Iyer et al., SOSP '24) keeps the batch size of an early-exit (EE) DNN
+ * constant by cutting the model into splits at exit ramps, running each split
+ * on full batches and re-batching the survivors of several upstream runs into
+ * one full batch for the next split (§3.2 PAPER.md:755-768,
+ * §3.3).  This library executes that data path on sm_100a:
+ *
+ *   e3_split_run   one split on one constant-size batch: encoder layers
+ *                  (tcgen05 GEMMs + attention), fused exit ramp + threshold
+ *                  test, stable compaction of the surviving rows;
+ *   e3_rebatch     pop exactly B rows FIFO from a survivor queue (top-up);
+ *   e3_pipeline_run  the whole split chain over n inputs with per-split
+ *                  queues, on one GPU or one rank of a multi-GPU plan.
+ *
+ * Conventions (all calls):
+ *   - Every call returns an e3_status and never throws or aborts.  On failure
+ *     e3_last_error() returns a thread-local message.
+ *   - Validation failures return E3_EINVAL / E3_EUNSUPPORTED before any
+ *     launch (no side effects).  A CUDA/NCCL failure poisons the handle; later
+ *     calls on it return E3_ESTATE.
+ *   - "stream" arguments are cudaStream_t passed as void* (NULL = legacy
+ *     default stream).  Calls marked ASYNC enqueue work and do not
+ *     synchronise the host.
+ *   - Activations are bf16, row-major [B, S, H] (token matrix [B*S, H]).
+ *     Weights are bf16 in nn.Linear layout [out_features, in_features];
+ *     biases / norm parameters are bf16 vectors.  Weight pointers are
+ *     BORROWED device pointers that must outlive the handle.
+ *   - Layer / ramp indices are 0-based ("ramp after layer 2" == layer 1).
+ *   - Numerics: bf16 storage with fp32 accumulation at the points listed in
+ *     DESIGN.md "Rounding contract"; ramp math in fp32.
+ */
+#ifndef E3_H_
+#define E3_H_
+
+#include <stddef.h>
+#include <stdint.h>
+
+#ifdef __cplusplus
+extern "C" {
+#endif
+
+#define E3_MAX_RAMPS 64
+#define E3_MAX_SPLITS 64
+#define E3_COMM_ID_BYTES 128
+
+typedef enum {
+  E3_OK = 0,
+  E3_EINVAL = 1,        /* bad argument (checked before any launch)            */
+  E3_EUNSUPPORTED = 2,  /* not sm_100, or dims outside the kernels' tiling     */
+  E3_ECUDA = 3,         /* CUDA runtime / launch failure (handle poisoned)     */
+  E3_ENCCL = 4,         /* NCCL failure or NCCL unavailable                    */
+  E3_ECAPACITY = 5,     /* a queue push would overflow the ring                */
+  E3_ESTATE = 6         /* handle poisoned by an earlier failure               */
+} e3_status;
+
+typedef enum { E3_ARCH_BERT = 0, E3_ARCH_VIT = 1, E3_ARCH_LLAMA_DECODE = 2 } e3_arch;
+typedef enum { E3_DTYPE_BF16 = 0, E3_DTYPE_FP32 = 1 } e3_dtype;
+/* Exit criteria: confidence ("certainty level is higher
+ * than a pre-defined threshold") -> exit iff max softmax > tau; entropy
+ * ("entropy ... smaller than pre-defined threshold") -> exit iff H < tau
+ * (natural log).  Comparisons are strict. */
+typedef enum { E3_TEST_MAXPROB = 0, E3_TEST_ENTROPY = 1 } e3_test;
+/* Ramps inside a split (§3.4 exit-wrapper; §5.8.6):
+ * EXACT evaluates every ramp (plan-independent results; rows that exit at an
+ * inner ramp are recorded there and carried, masked, to the split end);
+ * DISABLED evaluates only the split's last ramp. */
+typedef enum { E3_INNER_EXACT = 0, E3_INNER_DISABLED = 1 } e3_inner;
+
+const char *e3_last_error(void);
+const char *e3_version(void);
+
+/* ------------------------------------------------------------- split --- */
+
+/* One split: layers [layer_begin, layer_end) of the EE model ending in a ramp
+ * ("a contiguous block of encoder layers ending in an exit ramp").
+ * ramp_layer[] lists the model ramps whose layer lies in the split, ascending;
+ * the last must equal layer_end-1.  ramp_index[] are their model-wide ramp
+ * numbers (used for stats).  final_ramp = 1 iff the split's last ramp is the
+ * model's last ramp: "Remaining samples exit" there (Fig. 1). */
+typedef struct e3_split_desc {
+  int32_t arch;        /* e3_arch                                               */
+  int32_t dtype;       /* e3_dtype (only BF16 is implemented)                   */
+  int32_t hidden;      /* H   (multiple of 64)                                  */
+  int32_t heads;       /* nh  (H / nh == 64)                                    */
+  int32_t kv_heads;    /* LLAMA only                                            */
+  int32_t ffn;         /* F   (multiple of 64)                                  */
+  int32_t seq_len;     /* S   (<= 256)                                          */
+  int32_t num_labels;  /* C   (ramp classes)                                    */
+  int32_t ctx_len;     /* LLAMA only                                            */
+  float norm_eps;
+  int32_t layer_begin, layer_end;
+  int32_t n_ramps;
+  int32_t ramp_layer[E3_MAX_RAMPS];
+  int32_t ramp_index[E3_MAX_RAMPS];
+  float tau[E3_MAX_RAMPS];
+  int32_t test;        /* e3_test                                               */
+  int32_t final_ramp;
+  int32_t inner;       /* e3_inner                                              */
+  int32_t batch;       /* constant batch B (rows per run)                       */
+} e3_split_desc;
+
+typedef struct e3_layer_weights {
+  const void *w_qkv, *b_qkv;   /* [3H,H], [3H]  rows: q | k | v, head-major   */
+  const void *w_o, *b_o;       /* [H,H], [H]                                  */
+  const void *ln1_g, *ln1_b;   /* [H]                                         */
+  const void *w_1, *b_1;       /* [F,H], [F]                                  */
+  const void *w_2, *b_2;       /* [H,F], [H]                                  */
+  const void *ln2_g, *ln2_b;   /* [H]                                         */
+} e3_layer_weights;
+
+typedef struct e3_ramp_weights {
+  const void *w_p, *b_p;       /* BERT pooler [H,H], [H]   */
+  const void *w_c, *b_c;       /* classifier [C,H], [C]                       */
+  const void *ln_g, *ln_b;     /* VIT ramp LayerNorm [H] (NULL for BERT)      */
+} e3_ramp_weights;
+
+/* Model weights indexed by model-wide layer / ramp number. */
+typedef struct e3_weights {
+  int32_t n_layers;
+  const e3_layer_weights *layer;
+  int32_t n_ramps;
+  const e3_ramp_weights *ramp;
+} e3_weights;
+
+/* Exit records, written by the ramp kernel for every exiting valid row into
+ * arrays INDEXED BY INPUT ID (ids must lie in [0, capacity)).  All device
+ * memory, caller-owned; any pointer may be NULL to skip that field.
+ * logits is [capacity, C] fp32.  n_exit and ramp_count (indexed by model
+ * ramp number) are device counters that are incremented, never reset. */
+typedef struct e3_exits {
+  int32_t *exit_layer;
+  int32_t *label;      /* argmax, lowest index on ties                        */
+  float *conf;         /* the exit metric (max-prob or entropy)               */
+  float *logits;
+  int64_t capacity;
+  int32_t *n_exit;
+  int32_t *ramp_count;
+} e3_exits;
+
+typedef struct e3_split e3_split;
+
+/* Validates the descriptor, checks the device is sm_100, borrows the weights
+ * (layers [layer_begin, layer_end), the listed ramps) and allocates the
+ * handle-owned workspace for batch B.  E3_EUNSUPPORTED for shapes outside the
+ * kernels' tiling (H % 64, F % 64, head_dim != 64, S > 256, B*S % 128 ...). */
+e3_status e3_split_create(const e3_split_desc *d, const e3_weights *w, int device, e3_split **out);
+e3_status e3_split_destroy(e3_split *s);
+
+/* ASYNC.  Runs the split on one batch.
+ *   x_in     [B,S,H] bf16 device, read-only; must not alias x_out
+ *   id_in    [B] int64 device; rows >= n_valid are padding (never exit, never emitted)
+ *   n_valid_dev  device int32 (NULL: all B rows valid)
+ *   x_out    [B,S,H] bf16 device: survivors in stable (input) order
+ *   id_out   [B] int64 device: survivor ids, same order
+ *   n_surv_dev   device int32: number of survivors
+ *   ex       exit records (may be NULL)
+ * Conservation: exits recorded + n_surv == n_valid. */
+e3_status e3_split_run(e3_split *s, void *stream, const void *x_in, const int64_t *id_in,
+                       const int32_t *n_valid_dev, void *x_out, int64_t *id_out, int32_t *n_surv_dev,
+                       const e3_exits *ex);
+
+/* ------------------------------------------------------ queue / rebatch --- */
+
+/* Device FIFO ring of survivor rows ("a queue that holds the partial
+ * results") of row_bytes each (+ an int64 id per row),
+ * cap_rows rows.  Owned by the handle. */
+typedef struct e3_queue e3_queue;
+e3_status e3_queue_create(int device, int64_t row_bytes, int32_t cap_rows, e3_queue **q);
+e3_status e3_queue_destroy(e3_queue *q);
+/* ASYNC.  Appends *n_dev rows (device count, <= max_rows) of rows[]/ids[] in
+ * order.  If the ring would overflow nothing is written and the queue is
+ * flagged: the next e3_queue_count / e3_rebatch returns E3_ECAPACITY. */
+e3_status e3_queue_push(e3_queue *q, void *stream, const void *rows, const int64_t *ids, const int32_t *n_dev,
+                        int32_t max_rows);
+/* Synchronises `stream`-ordered work already enqueued on the queue's device
+ * and returns the exact row count. */
+e3_status e3_queue_count(e3_queue *q, int32_t *host_count);
+/* Re-batching top-up ("combine the two outputs to obtain a
+ * batch size of 16"; "multiple batches are fused"):
+ * synchronises the stream, then if count >= B pops exactly B rows FIFO into
+ * x_out/id_out, or if flush && count > 0 pops the remainder padded to B
+ * (padding rows zero, id -1).  Never emits more than B rows.
+ * *n_valid_dev (device) receives the valid count; *emitted (host) 1 or 0. */
+e3_status e3_rebatch(e3_queue *q, void *stream, int32_t B, int32_t flush, void *x_out, int64_t *id_out,
+                     int32_t *n_valid_dev, int32_t *emitted);
+
+/* ----------------------------------------------------------- pipeline --- */
+
+/* Split plan ("the apt number of splits ..., the number of resources to place
+ * them, and the batch sizes to run the splits with"). */
+typedef struct e3_plan {
+  int32_t n_splits;
+  e3_split_desc split[E3_MAX_SPLITS];  /* contiguous: split[s+1].layer_begin == split[s].layer_end;
+                                          same model dims and batch in every split */
+  int32_t lag;                         /* host look-behind: 0 serial, 1 (default)   */
+  int32_t queue_cap_batches;           /* ring capacity per split in batches (>= 4) */
+  int32_t trace;                       /* record dispatch order (e3_pipeline_trace) */
+} e3_plan;
+
+typedef struct e3_stats {
+  int64_t runs;
+  int64_t batches[E3_MAX_SPLITS];
+  int64_t valid_rows[E3_MAX_SPLITS];
+  int64_t padded_rows[E3_MAX_SPLITS];
+  int64_t rows_out[E3_MAX_SPLITS];
+  int64_t host_waits;                  /* times the host blocked on a run          */
+} e3_stats;
+
+typedef struct e3_pipeline e3_pipeline;
+/* All splits of the plan on one GPU with local queues (the paper's base
+ * formulation: "each GPU executes the splits sequentially").
+ * Multi-GPU plans (replicas, or splits on different GPUs with survivors sent
+ * over NVLink) are driven one rank per GPU from Python over torch.distributed
+ * (paper_conf_sosp_iyergdpgn24_b200/parallel.py), each rank calling this API. */
+e3_status e3_pipeline_create(const e3_plan *p, const e3_weights *w, int device, e3_pipeline **out);
+e3_status e3_pipeline_destroy(e3_pipeline *pl);
+/* Runs every input through the split chain until it exits.
+ *   x    [n,S,H] bf16, ids [n] int64 (ids in [0, ex->capacity)).  Both may be
+ *        DEVICE or HOST memory; host inputs are staged batch by batch on a
+ *        copy stream (H2D copies overlap compute).
+ *   ex   exit records (device arrays).
+ * Blocks until all of this rank's work is done (returns with the stream idle).
+ * Split 0 takes inputs in order, B at a time; every split runs exactly B rows
+ * per batch; the deepest split holding >= B queued rows runs first; when no
+ * queue is full and nothing upstream is pending, the shallowest non-empty
+ * queue is flushed padded to B. */
+e3_status e3_pipeline_run(e3_pipeline *pl, void *stream, const void *x, const int64_t *ids, int64_t n,
+                          const e3_exits *ex, e3_stats *st);
+/* Dispatch order of the last run (plan.trace = 1): per run its split, valid
+ * count and the B ids (padding = -1) into ids_out[run * B ...]. */
+e3_status e3_pipeline_trace(e3_pipeline *pl, int32_t *split, int32_t *n_valid, int64_t *ids_out,
+                            int64_t max_runs, int64_t *n_runs);
+
+#ifdef __cplusplus
+}
+#endif
+#endif /* E3_H_ */

@@ -96,6 +96,52 @@ def run(cfg, weights, X, ids: Optional[Sequence[int]] = None, tau=None,
     return out  # type: ignore[return-value]
 
 
+def run_split(cfg, weights, X, begin: int, end: int, ids: Optional[Sequence[int]] = None, tau=None,
+              mode: str = "fp64", inner: str = "exact"):
+    """One split (layers [begin, end), ending in a ramp) on the rows X.
+
+    The same per-input definition as ``run`` restricted to the split: apply
+    layers begin..end-1; at each ramp inside the split (all of them for inner
+    EXACT, only the split's last for DISABLED) evaluate the exit test; the
+    model's last ramp exits every row.  Returns (records of the rows that
+    exit inside the split, in input order; ids of the survivors in input
+    order; survivors' hidden states [k, S, H]; {id: min margin over the
+    split's tau-decided ramps}).
+    """
+    X = np.asarray(X, dtype=np.float64)
+    n = X.shape[0]
+    ids = list(range(n)) if ids is None else [int(i) for i in ids]
+    tau = cfg.tau if tau is None else tau
+    last = cfg.n_ramps - 1
+    ramps_in = [r for r, l in enumerate(cfg.ramp_layers) if begin <= l < end]
+    assert ramps_in and cfg.ramp_layers[ramps_in[-1]] == end - 1, "a split must end in a ramp"
+    en = set(ramps_in) if inner == "exact" else {ramps_in[-1]}
+    ramp_at = {cfg.ramp_layers[r]: r for r in ramps_in}
+    exited = {}
+    alive = np.arange(n)
+    margin = np.full(n, np.inf)
+    h = X
+    for l in range(begin, end):
+        h = encoder_layer(cfg, h, _as64(weights["layers"][l]), mode)
+        r = ramp_at.get(l)
+        if r is None or r not in en or alive.size == 0:
+            continue
+        z = ramp_logits(cfg, h, _as64(weights["ramps"][r]))
+        m = metric(cfg.test, z)
+        if r == last:
+            ok = np.ones(alive.size, dtype=bool)
+        else:
+            ok = passes(cfg.test, m, tau[r])
+            margin[alive] = np.minimum(margin[alive], np.abs(m - np.float64(np.float32(tau[r]))))
+        for j in np.nonzero(ok)[0]:
+            i = alive[j]
+            exited[i] = ExitRecord(ids[i], l, r, int(np.argmax(z[j])), float(m[j]), z[j].copy(),
+                                   float(margin[i]))
+        alive, h = alive[~ok], h[~ok]
+    recs = [exited[i] for i in sorted(exited)]
+    return recs, [ids[i] for i in alive], h, {ids[i]: float(margin[i]) for i in range(n)}
+
+
 def run_input(cfg, weights, x, id: int = 0, tau=None, mode="fp64", enabled=None) -> ExitRecord:
     """The EE-DNN run on one input alone."""
     return run(cfg, weights, np.asarray(x)[None], [id], tau, mode, enabled)[0]

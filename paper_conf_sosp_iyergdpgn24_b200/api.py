@@ -1,0 +1,263 @@
+"""Thin Python layer over the C ABI: torch tensors in, C pointers out.
+
+PyTorch provides device memory and streams only; every step of the path
+runs in libe3.so.  Names follow the C ABI (include/e3.h):
+
+    DeviceModel      weights of an EE model resident in HBM (bf16)
+    split_desc       e3_split_desc for layers [begin, end) of a model
+    Split            e3_split_create / e3_split_run
+    Queue            e3_queue_* and e3_rebatch
+    Pipeline         e3_pipeline_create / e3_pipeline_run / e3_pipeline_trace
+    ExitBuffers      device arrays of exit records indexed by input id
+    ops              kernel-level entry points (e3_ops.h)
+"""
+from __future__ import annotations
+
+import ctypes as C
+from typing import List, Optional, Sequence
+
+import numpy as np
+import torch
+
+from . import _lib
+from ._lib import check, lib
+
+_LAYER_KEYS = ("w_qkv", "b_qkv", "w_o", "b_o", "ln1_g", "ln1_b", "w_1", "b_1", "w_2", "b_2",
+               "ln2_g", "ln2_b")
+_RAMP_KEYS = ("w_p", "b_p", "w_c", "b_c", "ln_g", "ln_b")
+
+
+def _ptr(t: Optional[torch.Tensor]):
+    return None if t is None else C.c_void_p(t.data_ptr())
+
+
+def _stream(stream) -> C.c_void_p:
+    if stream is None:
+        stream = torch.cuda.current_stream()
+    return C.c_void_p(stream.cuda_stream)
+
+
+def to_bf16(a, device) -> torch.Tensor:
+    """float32 array holding bf16-representable values -> bf16 tensor (exact)."""
+    t = torch.from_numpy(np.ascontiguousarray(a, dtype=np.float32))
+    return t.to(device=device, dtype=torch.bfloat16)
+
+
+class DeviceModel:
+    """EE-model weights uploaded once to HBM; builds the e3_weights struct."""
+
+    def __init__(self, cfg, weights, device="cuda:0"):
+        self.cfg = cfg
+        self.device = torch.device(device)
+        self.layers = [{k: to_bf16(v, self.device) for k, v in w.items()} for w in weights["layers"]]
+        self.ramps = [{k: to_bf16(v, self.device) for k, v in w.items()} for w in weights["ramps"]]
+        n_l, n_r = len(self.layers), len(self.ramps)
+        self._lw = (_lib.LayerWeights * max(n_l, 1))()
+        for i, w in enumerate(self.layers):
+            for k in _LAYER_KEYS:
+                setattr(self._lw[i], k, w[k].data_ptr() if k in w else None)
+        self._rw = (_lib.RampWeights * max(n_r, 1))()
+        for i, w in enumerate(self.ramps):
+            for k in _RAMP_KEYS:
+                setattr(self._rw[i], k, w[k].data_ptr() if k in w else None)
+        self.c_weights = _lib.Weights(n_l, self._lw, n_r, self._rw)
+
+    def ramp_struct(self, r):
+        return self._rw[r]
+
+
+def split_desc(cfg, begin: int, end: int, tau, batch: Optional[int] = None,
+               inner: str = "exact") -> _lib.SplitDesc:
+    """e3_split_desc for layers [begin, end) of cfg (must end in a ramp)."""
+    d = _lib.SplitDesc()
+    d.arch = _lib.ARCH[cfg.arch]
+    d.dtype = 0
+    d.hidden, d.heads, d.kv_heads, d.ffn = cfg.hidden, cfg.heads, cfg.kv_heads, cfg.ffn
+    d.seq_len, d.num_labels, d.ctx_len = cfg.seq, cfg.classes, cfg.ctx
+    d.norm_eps = cfg.norm_eps
+    d.layer_begin, d.layer_end = begin, end
+    rs = [(r, l) for r, l in enumerate(cfg.ramp_layers) if begin <= l < end]
+    d.n_ramps = len(rs)
+    for j, (r, l) in enumerate(rs):
+        d.ramp_layer[j] = l
+        d.ramp_index[j] = r
+        d.tau[j] = float(tau[r])
+    d.test = _lib.TEST[cfg.test]
+    d.final_ramp = int(bool(rs) and rs[-1][0] == cfg.n_ramps - 1)
+    d.inner = _lib.INNER[inner]
+    d.batch = cfg.batch if batch is None else batch
+    return d
+
+
+class ExitBuffers:
+    """Exit records indexed by input id (e3_exits)."""
+
+    def __init__(self, capacity: int, classes: int, n_ramps: int, device, logits=True):
+        dev = torch.device(device)
+        self.capacity = capacity
+        self.exit_layer = torch.full((capacity,), -1, dtype=torch.int32, device=dev)
+        self.label = torch.full((capacity,), -1, dtype=torch.int32, device=dev)
+        self.conf = torch.full((capacity,), float("nan"), dtype=torch.float32, device=dev)
+        self.logits = torch.zeros((capacity, classes), dtype=torch.float32, device=dev) if logits else None
+        self.n_exit = torch.zeros((1,), dtype=torch.int32, device=dev)
+        self.ramp_count = torch.zeros((max(n_ramps, 1),), dtype=torch.int32, device=dev)
+        self.c = _lib.Exits(self.exit_layer.data_ptr(), self.label.data_ptr(), self.conf.data_ptr(),
+                            None if self.logits is None else self.logits.data_ptr(), capacity,
+                            self.n_exit.data_ptr(), self.ramp_count.data_ptr())
+
+    def reset(self):
+        self.exit_layer.fill_(-1)
+        self.label.fill_(-1)
+        self.conf.fill_(float("nan"))
+        if self.logits is not None:
+            self.logits.zero_()
+        self.n_exit.zero_()
+        self.ramp_count.zero_()
+
+
+class Split:
+    """One split on one constant-size batch (e3_split_create / e3_split_run)."""
+
+    def __init__(self, model: DeviceModel, desc: _lib.SplitDesc):
+        self.model, self.desc = model, desc
+        h = C.c_void_p()
+        check(lib.e3_split_create(C.byref(desc), C.byref(model.c_weights), model.device.index or 0,
+                                  C.byref(h)), "e3_split_create")
+        self.h = h
+
+    def run(self, x, ids, x_out, id_out, n_surv, exits: Optional[ExitBuffers] = None,
+            n_valid: Optional[torch.Tensor] = None, stream=None):
+        check(lib.e3_split_run(self.h, _stream(stream), _ptr(x), _ptr(ids), _ptr(n_valid), _ptr(x_out),
+                               _ptr(id_out), _ptr(n_surv), C.byref(exits.c) if exits else None),
+              "e3_split_run")
+
+    def __del__(self):
+        if getattr(self, "h", None) and _lib.lib is not None:
+            _lib.lib.e3_split_destroy(self.h)
+            self.h = None
+
+
+class Queue:
+    """Device FIFO of survivor rows (e3_queue_*), with e3_rebatch top-up."""
+
+    def __init__(self, device, row_bytes: int, cap_rows: int):
+        h = C.c_void_p()
+        check(lib.e3_queue_create(torch.device(device).index or 0, row_bytes, cap_rows, C.byref(h)),
+              "e3_queue_create")
+        self.h = h
+
+    def push(self, rows, ids, n_dev, max_rows, stream=None):
+        check(lib.e3_queue_push(self.h, _stream(stream), _ptr(rows), _ptr(ids), _ptr(n_dev), max_rows),
+              "e3_queue_push")
+
+    def count(self) -> int:
+        c = C.c_int32()
+        check(lib.e3_queue_count(self.h, C.byref(c)), "e3_queue_count")
+        return c.value
+
+    def rebatch(self, B, flush, x_out, id_out, n_valid_dev, stream=None) -> bool:
+        e = C.c_int32()
+        check(lib.e3_rebatch(self.h, _stream(stream), B, int(flush), _ptr(x_out), _ptr(id_out),
+                             _ptr(n_valid_dev), C.byref(e)), "e3_rebatch")
+        return bool(e.value)
+
+    def __del__(self):
+        if getattr(self, "h", None) and _lib.lib is not None:
+            _lib.lib.e3_queue_destroy(self.h)
+            self.h = None
+
+
+def make_plan(cfg, bounds: Sequence[int], tau, batch=None, inner="exact", lag=1,
+              queue_cap_batches=4, trace=False) -> _lib.Plan:
+    """Plan with split s covering layers [bounds[s], bounds[s+1])."""
+    p = _lib.Plan()
+    p.n_splits = len(bounds) - 1
+    for s in range(p.n_splits):
+        p.split[s] = split_desc(cfg, bounds[s], bounds[s + 1], tau, batch, inner)
+    p.lag = lag
+    p.queue_cap_batches = queue_cap_batches
+    p.trace = int(trace)
+    return p
+
+
+class Pipeline:
+    """All splits of a plan on one GPU (e3_pipeline_*)."""
+
+    def __init__(self, model: DeviceModel, plan: _lib.Plan):
+        self.model, self.plan = model, plan
+        h = C.c_void_p()
+        check(lib.e3_pipeline_create(C.byref(plan), C.byref(model.c_weights), model.device.index or 0,
+                                     C.byref(h)), "e3_pipeline_create")
+        self.h = h
+        self.B = plan.split[0].batch
+
+    def run(self, x, ids, exits: ExitBuffers, stream=None) -> _lib.Stats:
+        """x [n,S,H] bf16 and ids [n] int64, both on the device or both on the host."""
+        st = _lib.Stats()
+        n = int(ids.shape[0])
+        check(lib.e3_pipeline_run(self.h, _stream(stream), _ptr(x) if n else None,
+                                  _ptr(ids) if n else None, n, C.byref(exits.c), C.byref(st)),
+              "e3_pipeline_run")
+        return st
+
+    def trace(self):
+        n = C.c_int64()
+        check(lib.e3_pipeline_trace(self.h, None, None, None, 0, C.byref(n)), "e3_pipeline_trace")
+        k = n.value
+        split = (C.c_int32 * max(k, 1))()
+        nv = (C.c_int32 * max(k, 1))()
+        ids = np.zeros(max(k, 1) * self.B, dtype=np.int64)
+        check(lib.e3_pipeline_trace(self.h, split, nv, ids.ctypes.data_as(C.c_void_p), k, C.byref(n)),
+              "e3_pipeline_trace")
+        ids = ids[:k * self.B].reshape(k, self.B)
+        return [(split[i], nv[i], tuple(int(v) for v in ids[i, :nv[i]])) for i in range(k)]
+
+    def __del__(self):
+        if getattr(self, "h", None) and _lib.lib is not None:
+            _lib.lib.e3_pipeline_destroy(self.h)
+            self.h = None
+
+
+class ops:
+    """Kernel-level entry points (include/e3_ops.h)."""
+
+    @staticmethod
+    def gemm(A, W, bias, epilogue="bias", resid=None, out=None, stream=None):
+        M, K = A.shape
+        N = W.shape[0]
+        out = torch.empty((M, N), dtype=torch.bfloat16, device=A.device) if out is None else out
+        check(lib.e3_op_gemm(_stream(stream), _ptr(A), A.stride(0), _ptr(W), _ptr(bias), _ptr(resid),
+                             _ptr(out), M, N, K, _lib.EPI[epilogue]), "e3_op_gemm")
+        return out
+
+    @staticmethod
+    def attention(qkv, B, S, H, heads, out=None, stream=None):
+        out = torch.empty((B * S, H), dtype=torch.bfloat16, device=qkv.device) if out is None else out
+        check(lib.e3_op_attention(_stream(stream), _ptr(qkv), _ptr(out), B, S, H, heads), "e3_op_attention")
+        return out
+
+    @staticmethod
+    def layernorm(x, g, b, eps, out=None, stream=None):
+        rows, H = x.shape
+        out = torch.empty_like(x) if out is None else out
+        check(lib.e3_op_layernorm(_stream(stream), _ptr(x), _ptr(g), _ptr(b), _ptr(out), rows, H, eps),
+              "e3_op_layernorm")
+        return out
+
+    @staticmethod
+    def ramp(cfg, model: DeviceModel, r, x, ids, tau, alive, exits: ExitBuffers, final=False,
+             layer=None, init_alive=True, n_valid=None, stream=None):
+        B, S, H = x.shape
+        layer = cfg.ramp_layers[r] if layer is None else layer
+        rw = model.ramp_struct(r)
+        check(lib.e3_op_ramp(_stream(stream), _lib.ARCH[cfg.arch], _ptr(x), _ptr(ids), B, S, H, cfg.classes,
+                             C.byref(rw), _lib.TEST[cfg.test], float(tau), int(final), layer, r,
+                             cfg.norm_eps, _ptr(alive), int(init_alive), _ptr(n_valid), C.byref(exits.c)),
+              "e3_op_ramp")
+
+    @staticmethod
+    def compact(x, ids, alive, x_out, id_out, n_surv, stream=None):
+        B = x.shape[0]
+        row_bytes = x[0].numel() * x.element_size()
+        check(lib.e3_op_compact(_stream(stream), _ptr(x), _ptr(ids), _ptr(alive), B, row_bytes, _ptr(x_out),
+                                _ptr(id_out), _ptr(n_surv)), "e3_op_compact")

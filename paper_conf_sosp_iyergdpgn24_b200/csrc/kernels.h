@@ -1,0 +1,83 @@
+// Internal launchers of the split path (host side).  Product code only.
+#pragma once
+
+#include <cuda.h>
+#include <cuda_runtime.h>
+#include <stdint.h>
+
+#include "../../include/e3.h"
+#include "../../include/e3_ops.h"
+
+namespace e3 {
+
+// ---- K1 layer GEMM (gemm_tc.cu)
+struct GemmMaps {
+  CUtensorMap a;
+  CUtensorMap b;
+  int bn;
+};
+int gemm_pick_bn(int M, int N, int sms);
+e3_status gemm_tmaps(GemmMaps *g, const void *A, int64_t lda, const void *W, int M, int N, int K, int bn);
+e3_status gemm_run(const GemmMaps &g, void *C, const void *bias, const void *R, int M, int N, int K, int epi,
+                   int sms, cudaStream_t st);
+
+// ---- K2 attention (attn_tc.cu)
+struct AttnMaps {
+  CUtensorMap q;    // box 64 x 128 x 1
+  CUtensorMap kv;   // box 64 x SKV x 1
+  int skv;
+};
+e3_status attn_tmaps(AttnMaps *m, const void *qkv, int B, int S, int H);
+e3_status attn_run(const AttnMaps &m, void *ctx, int B, int S, int H, int heads, cudaStream_t st);
+
+// ---- K3 LayerNorm (layernorm.cu)
+e3_status layernorm_run(const void *x, const void *g, const void *b, void *y, int rows, int H, float eps,
+                        cudaStream_t st);
+
+// ---- K4 exit ramp (ramp.cu)
+constexpr int kRampRowsPerCta = 16;   // rows per ramp row group (one ticket each)
+struct RampArgs {
+  int arch;
+  const void *x;            // [B,S,H] bf16
+  const int64_t *id;        // [B]
+  int B, S, H, C;
+  e3_ramp_weights w;
+  int test;
+  float tau;
+  int final_ramp;
+  int layer, ramp_index;
+  float eps;
+  uint8_t *alive;           // [B]
+  int init_alive;
+  const int32_t *n_valid_dev;   // NULL: n_valid_host
+  int n_valid_host;
+  e3_exits ex;
+  float *pool_ws;           // [B,H] fp32 workspace
+  unsigned *done_ctr;       // device tickets [ceil(B/kRampRowsPerCta)] (zero between launches)
+};
+e3_status ramp_run(const RampArgs &a, cudaStream_t st);
+
+// ---- K5 compaction (compact.cu)
+struct RingDst {
+  uint8_t *rows;            // [cap, row_bytes]
+  int64_t *ids;             // [cap]
+  int64_t cap;
+  int64_t *tail_dev;        // NULL: contiguous output at row 0
+  int64_t head;             // host-known head (rows) at launch
+  int *overflow_dev;        // may be NULL
+  volatile int *mailbox;    // host-mapped slot for n_surv (may be NULL)
+};
+e3_status compact_run(const void *x, const int64_t *id, const uint8_t *alive, int B, int64_t row_bytes,
+                      const RingDst &dst, int32_t *n_surv_dev, unsigned *done_ctr, int sms, cudaStream_t st);
+
+// ---- K6 queue pop (compact.cu): rows [head, head+n) of a ring -> contiguous
+// dst, zero-padding rows n..B-1 (ids -1).
+e3_status ring_pop_copy(const uint8_t *ring, const int64_t *ring_ids, int64_t cap, int64_t head, int n, int B,
+                        int64_t row_bytes, void *dst, int64_t *dst_ids, int sms, cudaStream_t st);
+// device-count push (e3_queue_push): rows [0, *n_dev) appended at *tail_dev
+e3_status ring_push_copy(const void *rows, const int64_t *ids, const int32_t *n_dev, int max_rows, uint8_t *ring,
+                         int64_t *ring_ids, int64_t cap, int64_t *tail_dev, const int64_t *head_dev,
+                         int *overflow_dev, int64_t row_bytes, cudaStream_t st);
+e3_status fill_valid(int32_t *dst, int value, cudaStream_t st);
+
+}  // namespace e3

@@ -1,0 +1,425 @@
+// Split executor: one split of the early-exit encoder
+// on one constant-size batch, stream-ordered, no host synchronisation.
+//
+// For each layer l of the split (BERT post-LN, R11):
+//   qkv = gemm(x, W_qkv) + b                    [tcgen05 GEMM, bias epilogue]
+//   ctx = attention(qkv)                        [tcgen05 attention]
+//   y   = gemm(ctx, W_o) + b_o + x              [residual epilogue]
+//   x1  = LN1(y)                                [row LayerNorm]
+//   h   = GELU(gemm(x1, W_1) + b_1)             [GELU epilogue]
+//   y   = gemm(h, W_2) + b_2 + x1               [residual epilogue]
+//   x2  = LN2(y)
+//   if a ramp follows l (and is evaluated): fused ramp + threshold test
+// then the stable compaction of the rows still alive.  Rows that exit at an
+// inner ramp (inner = EXACT) are recorded there and carried masked to the end
+// of the split ("mark and carry"; R7), which yields plan-independent
+// results.  Activations ping-pong between two workspace buffers so the caller's
+// x_in is never written.
+#include <cstring>
+#include <new>
+
+#include "common.cuh"
+#include "prof.h"
+#include "split.h"
+
+namespace e3 {
+
+Workspace::~Workspace() {
+  int prev = 0;
+  cudaGetDevice(&prev);
+  cudaSetDevice(device);
+  void *bufs[] = {qkv, ctx, y, x1, h, xa, xb, pool, alive, ctr};
+  for (void *p : bufs)
+    if (p) cudaFree(p);
+  cudaSetDevice(prev);
+}
+
+e3_status Workspace::create(int device, int B, int S, int H, int F, std::shared_ptr<Workspace> *out) {
+  auto ws = std::make_shared<Workspace>();
+  ws->device = device;
+  ws->B = B;
+  ws->S = S;
+  ws->H = H;
+  ws->F = F;
+  const size_t M = (size_t)B * S;
+  E3_CUDA_TRY(cudaMalloc(&ws->qkv, M * 3 * H * 2));
+  E3_CUDA_TRY(cudaMalloc(&ws->ctx, M * H * 2));
+  E3_CUDA_TRY(cudaMalloc(&ws->y, M * H * 2));
+  E3_CUDA_TRY(cudaMalloc(&ws->x1, M * H * 2));
+  E3_CUDA_TRY(cudaMalloc(&ws->h, M * F * 2));
+  E3_CUDA_TRY(cudaMalloc(&ws->xa, M * H * 2));
+  E3_CUDA_TRY(cudaMalloc(&ws->xb, M * H * 2));
+  E3_CUDA_TRY(cudaMalloc(&ws->pool, (size_t)B * H * 4));
+  E3_CUDA_TRY(cudaMalloc(&ws->alive, (size_t)B));
+  E3_CUDA_TRY(cudaMalloc(&ws->ctr, kCtrWords * sizeof(unsigned)));
+  E3_CUDA_TRY(cudaMemset(ws->ctr, 0, kCtrWords * sizeof(unsigned)));
+  E3_CUDA_TRY(cudaMemset(ws->alive, 0, (size_t)B));
+  *out = ws;
+  return E3_OK;
+}
+
+static bool aligned16(const void *p) { return (reinterpret_cast<uintptr_t>(p) & 15) == 0; }
+
+e3_status split_validate(const e3_split_desc *d, const e3_weights *w) {
+  E3_CHECK_ARG(d && w, "null descriptor or weights");
+  if (d->arch != E3_ARCH_BERT) {
+    set_error("e3_split_create: only arch BERT is implemented on the GPU path");
+    return E3_EUNSUPPORTED;
+  }
+  if (d->dtype != E3_DTYPE_BF16) {
+    set_error("e3_split_create: only dtype BF16 is implemented");
+    return E3_EUNSUPPORTED;
+  }
+  E3_CHECK_ARG(d->hidden > 0 && d->heads > 0 && d->ffn > 0 && d->seq_len > 0 && d->batch > 0, "non-positive dims");
+  if (d->hidden % 64 || d->hidden / d->heads != 64 || d->hidden % d->heads || d->ffn % 64 || d->seq_len > 256 ||
+      d->batch > 4096 || d->num_labels < 1 || d->num_labels > 16 || d->hidden > 4096) {
+    set_error("e3_split_create: unsupported shape (need H % 64 == 0, head_dim 64, F % 64 == 0, S <= 256, "
+              "B <= 4096, 1 <= C <= 16, H <= 4096)");
+    return E3_EUNSUPPORTED;
+  }
+  E3_CHECK_ARG(d->layer_begin >= 0 && d->layer_end > d->layer_begin && d->layer_end <= w->n_layers,
+               "layer range outside the model");
+  E3_CHECK_ARG(d->n_ramps >= 1 && d->n_ramps <= E3_MAX_RAMPS, "a split needs 1..64 ramps");
+  for (int r = 0; r < d->n_ramps; ++r) {
+    E3_CHECK_ARG(d->ramp_layer[r] >= d->layer_begin && d->ramp_layer[r] < d->layer_end, "ramp outside split");
+    E3_CHECK_ARG(r == 0 || d->ramp_layer[r] > d->ramp_layer[r - 1], "ramp layers not ascending");
+    E3_CHECK_ARG(d->ramp_index[r] >= 0 && d->ramp_index[r] < w->n_ramps, "ramp index outside the model");
+  }
+  E3_CHECK_ARG(d->ramp_layer[d->n_ramps - 1] == d->layer_end - 1, "a split must end in a ramp");
+  E3_CHECK_ARG(d->test == E3_TEST_MAXPROB || d->test == E3_TEST_ENTROPY, "bad test");
+  E3_CHECK_ARG(d->inner == E3_INNER_EXACT || d->inner == E3_INNER_DISABLED, "bad inner mode");
+  for (int l = d->layer_begin; l < d->layer_end; ++l) {
+    const e3_layer_weights &L = w->layer[l];
+    const void *ps[] = {L.w_qkv, L.b_qkv, L.w_o, L.b_o, L.ln1_g, L.ln1_b, L.w_1, L.b_1, L.w_2, L.b_2, L.ln2_g, L.ln2_b};
+    for (const void *p : ps) E3_CHECK_ARG(p && aligned16(p), "layer weight pointer null or not 16-byte aligned");
+  }
+  for (int r = 0; r < d->n_ramps; ++r) {
+    const e3_ramp_weights &R = w->ramp[d->ramp_index[r]];
+    E3_CHECK_ARG(R.w_p && R.b_p && R.w_c && R.b_c && aligned16(R.w_p), "ramp weight pointer null / misaligned");
+  }
+  return E3_OK;
+}
+
+static e3_status check_device(int device) {
+  cudaDeviceProp p;
+  E3_CUDA_TRY(cudaGetDeviceProperties(&p, device));
+  if (p.major != 10 || p.minor != 0) {
+    set_error("E3 kernels are built for sm_100a (B200); device is sm_" + std::to_string(p.major * 10 + p.minor));
+    return E3_EUNSUPPORTED;
+  }
+  return E3_OK;
+}
+
+e3_status split_create_shared(const e3_split_desc *d, const e3_weights *w, int device, std::shared_ptr<Workspace> ws,
+                              e3_split **out) {
+  E3_CHECK_ARG(out, "null out");
+  e3_status st = split_validate(d, w);
+  if (st != E3_OK) return st;
+  st = check_device(device);
+  if (st != E3_OK) return st;
+  E3_CUDA_TRY(cudaSetDevice(device));
+  e3_split *s = new (std::nothrow) e3_split();
+  if (!s) {
+    set_error("out of host memory");
+    return E3_ECUDA;
+  }
+  s->d = *d;
+  s->device = device;
+  s->sms = num_sms(device);
+  const int B = d->batch, S = d->seq_len, H = d->hidden, F = d->ffn;
+  for (int l = d->layer_begin; l < d->layer_end; ++l) s->L.push_back(w->layer[l]);
+  for (int r = 0; r < d->n_ramps; ++r) s->R.push_back(w->ramp[d->ramp_index[r]]);
+  if (!ws) {
+    st = Workspace::create(device, B, S, H, F, &ws);
+    if (st != E3_OK) {
+      delete s;
+      return st;
+    }
+  } else if (ws->B != B || ws->S != S || ws->H != H || ws->F != F) {
+    delete s;
+    set_error("shared workspace shape mismatch");
+    return E3_EINVAL;
+  }
+  s->ws = ws;
+  const int M = B * S;
+  s->bn_qkv = gemm_pick_bn(M, 3 * H, s->sms);
+  s->bn_o = gemm_pick_bn(M, H, s->sms);
+  s->bn_f1 = gemm_pick_bn(M, F, s->sms);
+  s->bn_f2 = gemm_pick_bn(M, H, s->sms);
+  const int nl = d->layer_end - d->layer_begin;
+  s->maps.resize(nl);
+  for (int i = 0; i < nl && st == E3_OK; ++i) {
+    auto &m = s->maps[i];
+    const void *prev = (i % 2 == 1) ? ws->xa : ws->xb;   // output of layer i-1
+    if (i > 0) st = gemm_tmaps(&m.qkv, prev, H, s->L[i].w_qkv, M, 3 * H, H, s->bn_qkv);
+    if (st == E3_OK) st = gemm_tmaps(&m.o, ws->ctx, H, s->L[i].w_o, M, H, H, s->bn_o);
+    if (st == E3_OK) st = gemm_tmaps(&m.f1, ws->x1, H, s->L[i].w_1, M, F, H, s->bn_f1);
+    if (st == E3_OK) st = gemm_tmaps(&m.f2, ws->h, F, s->L[i].w_2, M, H, F, s->bn_f2);
+  }
+  if (st == E3_OK) st = attn_tmaps(&s->attn, ws->qkv, B, S, H);
+  if (st != E3_OK) {
+    delete s;
+    return st;
+  }
+  *out = s;
+  return E3_OK;
+}
+
+e3_status split_run_to(e3_split *s, cudaStream_t st, const void *x_in, const int64_t *id_in,
+                       const int32_t *n_valid_dev, int n_valid_host, const RingDst &dst, int32_t *n_surv_dev,
+                       const e3_exits *ex) {
+  const e3_split_desc &d = s->d;
+  Workspace &ws = *s->ws;
+  const int B = d.batch, S = d.seq_len, H = d.hidden, F = d.ffn, M = B * S;
+  const int nl = d.layer_end - d.layer_begin;
+  e3_exits exits{};
+  if (ex) exits = *ex;
+  const void *cur = x_in;
+  bool first_ramp = true;
+  int ri = 0;
+  e3_status r = E3_OK;
+#define E3_RUN(expr)              \
+  do {                            \
+    r = (expr);                   \
+    if (r != E3_OK) return r;     \
+  } while (0)
+  // algorithmic work of this run counts valid rows only (padding is overhead)
+  const double nvS = (double)n_valid_host * S;
+  const double f_qkv = 2.0 * nvS * 3 * H * H, f_o = 2.0 * nvS * H * H, f_1 = 2.0 * nvS * F * H;
+  const double f_att = 4.0 * n_valid_host * (double)S * S * H, b_ln = 2.0 * nvS * H * 2;
+  for (int i = 0; i < nl; ++i) {
+    const int l = d.layer_begin + i;
+    const e3_layer_weights &L = s->L[i];
+    auto &m = s->maps[i];
+    void *out = (i % 2 == 0) ? ws.xa : ws.xb;
+    {
+      ProfScope ps(PK_GEMM_QKV, st, f_qkv, 0);
+      if (i == 0) {
+        GemmMaps g0;
+        E3_RUN(gemm_tmaps(&g0, cur, H, L.w_qkv, M, 3 * H, H, s->bn_qkv));
+        E3_RUN(gemm_run(g0, ws.qkv, L.b_qkv, nullptr, M, 3 * H, H, E3_EPI_BIAS, s->sms, st));
+      } else {
+        E3_RUN(gemm_run(m.qkv, ws.qkv, L.b_qkv, nullptr, M, 3 * H, H, E3_EPI_BIAS, s->sms, st));
+      }
+    }
+    {
+      ProfScope ps(PK_ATTN, st, f_att, 0);
+      E3_RUN(attn_run(s->attn, ws.ctx, B, S, H, d.heads, st));
+    }
+    {
+      ProfScope ps(PK_GEMM_O, st, f_o, 0);
+      E3_RUN(gemm_run(m.o, ws.y, L.b_o, cur, M, H, H, E3_EPI_BIAS_RESID, s->sms, st));
+    }
+    {
+      ProfScope ps(PK_LN, st, 0, b_ln);
+      E3_RUN(layernorm_run(ws.y, L.ln1_g, L.ln1_b, ws.x1, M, H, d.norm_eps, st));
+    }
+    {
+      ProfScope ps(PK_GEMM_FFN1, st, f_1, 0);
+      E3_RUN(gemm_run(m.f1, ws.h, L.b_1, nullptr, M, F, H, E3_EPI_BIAS_GELU, s->sms, st));
+    }
+    {
+      ProfScope ps(PK_GEMM_FFN2, st, f_1, 0);
+      E3_RUN(gemm_run(m.f2, ws.y, L.b_2, ws.x1, M, H, F, E3_EPI_BIAS_RESID, s->sms, st));
+    }
+    {
+      ProfScope ps(PK_LN, st, 0, b_ln);
+      E3_RUN(layernorm_run(ws.y, L.ln2_g, L.ln2_b, out, M, H, d.norm_eps, st));
+    }
+    cur = out;
+    while (ri < d.n_ramps && d.ramp_layer[ri] == l) {
+      const bool last = (ri == d.n_ramps - 1);
+      if (last || d.inner == E3_INNER_EXACT) {
+        RampArgs a{};
+        a.arch = d.arch;
+        a.x = cur;
+        a.id = id_in;
+        a.B = B;
+        a.S = S;
+        a.H = H;
+        a.C = d.num_labels;
+        a.w = s->R[ri];
+        a.test = d.test;
+        a.tau = d.tau[ri];
+        a.final_ramp = last && d.final_ramp;
+        a.layer = l;
+        a.ramp_index = d.ramp_index[ri];
+        a.eps = d.norm_eps;
+        a.alive = ws.alive;
+        a.init_alive = first_ramp;
+        a.n_valid_dev = n_valid_dev;
+        a.n_valid_host = n_valid_host;
+        a.ex = exits;
+        a.pool_ws = ws.pool;
+        a.done_ctr = ws.ctr + 1;   // per-row-group tickets
+        {
+          // pooler weights + CLS rows + classifier weights (bytes); 2H^2 + 2HC per row (flops)
+          ProfScope ps(PK_RAMP, st, (double)n_valid_host * (2.0 * H * H + 2.0 * H * d.num_labels),
+                       2.0 * H * H + 2.0 * n_valid_host * H + 2.0 * d.num_labels * H);
+          E3_RUN(ramp_run(a, st));
+        }
+        first_ramp = false;
+      }
+      ++ri;
+    }
+  }
+  {
+    ProfScope ps(PK_COMPACT, st, 0, 0);   // bytes added once n_surv is known (pipeline)
+    E3_RUN(compact_run(cur, id_in, ws.alive, B, (int64_t)S * H * 2, dst, n_surv_dev, ws.ctr, s->sms, st));
+  }
+#undef E3_RUN
+  return E3_OK;
+}
+
+}  // namespace e3
+
+using namespace e3;
+
+extern "C" {
+
+e3_status e3_split_create(const e3_split_desc *d, const e3_weights *w, int device, e3_split **out) {
+  return split_create_shared(d, w, device, nullptr, out);
+}
+
+e3_status e3_split_destroy(e3_split *s) {
+  delete s;
+  return E3_OK;
+}
+
+e3_status e3_split_run(e3_split *s, void *stream, const void *x_in, const int64_t *id_in, const int32_t *n_valid_dev,
+                       void *x_out, int64_t *id_out, int32_t *n_surv_dev, const e3_exits *ex) {
+  E3_CHECK_ARG(s, "null split");
+  if (s->poisoned) {
+    set_error("split handle poisoned by an earlier CUDA failure");
+    return E3_ESTATE;
+  }
+  E3_CHECK_ARG(x_in && id_in && x_out && id_out && n_surv_dev, "null buffer");
+  E3_CHECK_ARG(x_in != x_out, "x_in must not alias x_out");
+  E3_CHECK_ARG(aligned16(x_in) && aligned16(x_out), "activations must be 16-byte aligned");
+  const int B = s->d.batch;
+  RingDst dst{};
+  dst.rows = reinterpret_cast<uint8_t *>(x_out);
+  dst.ids = id_out;
+  dst.cap = B;
+  int dev = 0;
+  E3_CUDA_TRY(cudaGetDevice(&dev));
+  if (dev != s->device) E3_CUDA_TRY(cudaSetDevice(s->device));
+  e3_status r = split_run_to(s, reinterpret_cast<cudaStream_t>(stream), x_in, id_in, n_valid_dev, B, dst, n_surv_dev,
+                             ex);
+  if (r == E3_ECUDA) s->poisoned = true;
+  if (dev != s->device) cudaSetDevice(dev);
+  return r;
+}
+
+// ------------------------------------------------------------- e3_ops.h --
+
+e3_status e3_op_gemm(void *stream, const void *A, int64_t lda, const void *W, const void *bias, const void *resid,
+                     void *C, int32_t M, int32_t N, int32_t K, int32_t epilogue) {
+  E3_CHECK_ARG(A && W && bias && C, "null buffer");
+  E3_CHECK_ARG(epilogue >= 0 && epilogue <= 2, "bad epilogue");
+  E3_CHECK_ARG(epilogue != E3_EPI_BIAS_RESID || resid, "residual epilogue needs resid");
+  E3_CHECK_ARG(M > 0 && N > 0 && K > 0 && lda >= K, "bad dims");
+  if (K % 64 || N % 64 || lda % 8 || !aligned16(A) || !aligned16(W) || !aligned16(C) || !aligned16(bias)) {
+    set_error("e3_op_gemm: need K % 64 == 0, N % 64 == 0, lda % 8 == 0, 16-byte aligned pointers");
+    return E3_EUNSUPPORTED;
+  }
+  int dev = 0;
+  E3_CUDA_TRY(cudaGetDevice(&dev));
+  const int sms = num_sms(dev);
+  GemmMaps g;
+  e3_status r = gemm_tmaps(&g, A, lda, W, M, N, K, gemm_pick_bn(M, N, sms));
+  if (r != E3_OK) return r;
+  return gemm_run(g, C, bias, resid, M, N, K, epilogue, sms, reinterpret_cast<cudaStream_t>(stream));
+}
+
+e3_status e3_op_attention(void *stream, const void *qkv, void *ctx, int32_t B, int32_t S, int32_t H, int32_t heads) {
+  E3_CHECK_ARG(qkv && ctx && B > 0 && S > 0 && H > 0 && heads > 0, "bad arguments");
+  if (H / heads != 64 || H % heads || S > 256 || !aligned16(qkv) || !aligned16(ctx)) {
+    set_error("e3_op_attention: need head_dim 64, S <= 256, aligned buffers");
+    return E3_EUNSUPPORTED;
+  }
+  AttnMaps m;
+  e3_status r = attn_tmaps(&m, qkv, B, S, H);
+  if (r != E3_OK) return r;
+  return attn_run(m, ctx, B, S, H, heads, reinterpret_cast<cudaStream_t>(stream));
+}
+
+e3_status e3_op_layernorm(void *stream, const void *x, const void *g, const void *b, void *y, int32_t rows, int32_t H,
+                          float eps) {
+  E3_CHECK_ARG(x && g && b && y && rows > 0 && H > 0, "bad arguments");
+  if (H % 8 || H > 4096 || !aligned16(x) || !aligned16(y) || !aligned16(g) || !aligned16(b)) {
+    set_error("e3_op_layernorm: need H % 8 == 0, H <= 4096, aligned buffers");
+    return E3_EUNSUPPORTED;
+  }
+  return layernorm_run(x, g, b, y, rows, H, eps, reinterpret_cast<cudaStream_t>(stream));
+}
+
+e3_status e3_op_ramp(void *stream, int32_t arch, const void *x, const int64_t *id, int32_t B, int32_t S, int32_t H,
+                     int32_t C, const e3_ramp_weights *rw, int32_t test, float tau, int32_t final, int32_t layer,
+                     int32_t ramp_index, float norm_eps, uint8_t *alive, int32_t init_alive,
+                     const int32_t *n_valid_dev, const e3_exits *ex) {
+  E3_CHECK_ARG(x && id && rw && alive && B > 0 && S > 0 && H > 0 && C > 0, "bad arguments");
+  E3_CHECK_ARG(B <= 4096, "B > 4096");
+  E3_CHECK_ARG(aligned16(x) && aligned16(rw->w_p), "misaligned");
+  int dev = 0;
+  E3_CUDA_TRY(cudaGetDevice(&dev));
+  // per-call scratch: pooled activations + ticket (freed asynchronously)
+  cudaStream_t st = reinterpret_cast<cudaStream_t>(stream);
+  float *pool = nullptr;
+  unsigned *ctr = nullptr;
+  E3_CUDA_TRY(cudaMallocAsync(reinterpret_cast<void **>(&pool), (size_t)B * H * 4, st));
+  const size_t nctr = (size_t)(B + kRampRowsPerCta - 1) / kRampRowsPerCta * sizeof(unsigned);
+  E3_CUDA_TRY(cudaMallocAsync(reinterpret_cast<void **>(&ctr), nctr, st));
+  E3_CUDA_TRY(cudaMemsetAsync(ctr, 0, nctr, st));
+  RampArgs a{};
+  a.arch = arch;
+  a.x = x;
+  a.id = id;
+  a.B = B;
+  a.S = S;
+  a.H = H;
+  a.C = C;
+  a.w = *rw;
+  a.test = test;
+  a.tau = tau;
+  a.final_ramp = final;
+  a.layer = layer;
+  a.ramp_index = ramp_index;
+  a.eps = norm_eps;
+  a.alive = alive;
+  a.init_alive = init_alive;
+  a.n_valid_dev = n_valid_dev;
+  a.n_valid_host = B;
+  if (ex) a.ex = *ex;
+  a.pool_ws = pool;
+  a.done_ctr = ctr;
+  e3_status r = ramp_run(a, st);
+  cudaFreeAsync(pool, st);
+  cudaFreeAsync(ctr, st);
+  return r;
+}
+
+e3_status e3_op_compact(void *stream, const void *x, const int64_t *id, const uint8_t *alive, int32_t B,
+                        int64_t row_bytes, void *x_out, int64_t *id_out, int32_t *n_surv_dev) {
+  E3_CHECK_ARG(x && id && alive && x_out && id_out && n_surv_dev && B > 0 && row_bytes > 0, "bad arguments");
+  E3_CHECK_ARG(x != x_out, "x must not alias x_out");
+  if (row_bytes % 16 || B > 4096 || !aligned16(x) || !aligned16(x_out)) {
+    set_error("e3_op_compact: need row_bytes % 16 == 0, B <= 4096, aligned buffers");
+    return E3_EUNSUPPORTED;
+  }
+  int dev = 0;
+  E3_CUDA_TRY(cudaGetDevice(&dev));
+  cudaStream_t st = reinterpret_cast<cudaStream_t>(stream);
+  unsigned *ctr = nullptr;
+  E3_CUDA_TRY(cudaMallocAsync(reinterpret_cast<void **>(&ctr), sizeof(unsigned), st));
+  E3_CUDA_TRY(cudaMemsetAsync(ctr, 0, sizeof(unsigned), st));
+  RingDst dst{};
+  dst.rows = reinterpret_cast<uint8_t *>(x_out);
+  dst.ids = id_out;
+  dst.cap = B;
+  e3_status r = compact_run(x, id, alive, B, row_bytes, dst, n_surv_dev, ctr, num_sms(dev), st);
+  cudaFreeAsync(ctr, st);
+  return r;
+}
+
+}  // extern "C"

@@ -1,0 +1,55 @@
+// Split executor internals (shared by split.cu and pipeline.cu).
+#pragma once
+
+#include <memory>
+#include <vector>
+
+#include "kernels.h"
+
+namespace e3 {
+
+// 1 compaction ticket + one ramp ticket per group of kRampRowsPerCta rows (B <= 4096)
+constexpr int kCtrWords = 1 + 4096 / kRampRowsPerCta;
+
+// Activation workspace for one batch of B rows.  Splits that run serially on
+// one stream may share a workspace (the pipeline does).
+struct Workspace {
+  int device = 0;
+  int B = 0, S = 0, H = 0, F = 0;
+  void *qkv = nullptr, *ctx = nullptr, *y = nullptr, *x1 = nullptr, *h = nullptr, *xa = nullptr, *xb = nullptr;
+  float *pool = nullptr;
+  uint8_t *alive = nullptr;
+  unsigned *ctr = nullptr;        // [kCtrWords]: compaction ticket, ramp row-group tickets
+  ~Workspace();
+  static e3_status create(int device, int B, int S, int H, int F, std::shared_ptr<Workspace> *out);
+};
+
+}  // namespace e3
+
+struct e3_split {
+  e3_split_desc d;
+  int device = 0;
+  int sms = 148;
+  bool poisoned = false;
+  std::vector<e3_layer_weights> L;      // layers [begin, end)
+  std::vector<e3_ramp_weights> R;       // ramps listed in d.ramp_layer
+  std::shared_ptr<e3::Workspace> ws;
+  struct LayerMaps {
+    e3::GemmMaps qkv, o, f1, f2;
+  };
+  std::vector<LayerMaps> maps;
+  e3::AttnMaps attn;
+  int bn_qkv = 0, bn_o = 0, bn_f1 = 0, bn_f2 = 0;
+};
+
+namespace e3 {
+
+e3_status split_validate(const e3_split_desc *d, const e3_weights *w);
+e3_status split_create_shared(const e3_split_desc *d, const e3_weights *w, int device,
+                              std::shared_ptr<Workspace> ws, e3_split **out);
+// Runs the split; survivors go to `dst` (contiguous or a queue ring).
+e3_status split_run_to(e3_split *s, cudaStream_t st, const void *x_in, const int64_t *id_in,
+                       const int32_t *n_valid_dev, int n_valid_host, const RingDst &dst, int32_t *n_surv_dev,
+                       const e3_exits *ex);
+
+}  // namespace e3

@@ -1,0 +1,235 @@
+"""-m gpu: e3_split_run / e3_rebatch / e3_pipeline_run vs the oracle.
+
+Per split run (the unit of the hot path): exit layers, labels and survivor
+ids/order exact wherever every ramp margin exceeds 1e-3, logits within 2e-2
+absolute per bf16 layer of the split of the bf16-emulating oracle applied to
+the SAME input rows (north_star; R13).  End to end through many splits bf16 storage
+amplifies one-ulp rounding differences layer after layer, so the chained
+comparison uses the looser bounds of DESIGN.md R13 (decisions exact where
+margin > 1e-2, logits within 0.1).  The dispatch trace of the pipeline equals
+oracle.pipeline_sim with the same lag exactly."""
+import numpy as np
+import pytest
+import torch
+
+import e3data
+import oracle
+from oracle.pipeline_sim import Plan, simulate_pipeline
+from tests.gpu_util import DEV, bf16_tensor, requires_cuda, to64
+
+pytestmark = [pytest.mark.gpu, requires_cuda]
+
+LOGIT_TOL = 2e-2       # per bf16 layer of a split run (R13)
+MARGIN = 1e-3
+E2E_LOGIT_TOL = 0.1    # chained over up to 12 bf16 layers (R13)
+E2E_MARGIN = 1e-2
+
+
+@pytest.fixture(scope="module")
+def api():
+    from paper_conf_sosp_iyergdpgn24_b200 import api as A
+    return A
+
+
+@pytest.fixture(scope="module")
+def tiny(api):
+    cfg = e3data.get("tiny")
+    W = e3data.make_weights(cfg)
+    model = api.DeviceModel(cfg, W, DEV)
+    return cfg, W, model
+
+
+def _compare_records(recs, ex, ids, cfg, margin=MARGIN, logit_tol=LOGIT_TOL):
+    el = ex.exit_layer.cpu().numpy()
+    lab = ex.label.cpu().numpy()
+    conf = ex.conf.cpu().numpy()
+    lg = ex.logits.cpu().numpy()
+    n_checked = 0
+    for i, r in zip(ids, recs):
+        assert el[i] >= 0, f"input {i} never exited"
+        if r.margin > margin:
+            assert el[i] == r.exit_layer, f"input {i}: gpu exit {el[i]} oracle {r.exit_layer} margin {r.margin}"
+            n_checked += 1
+        top2 = np.sort(r.logits)[-2:]
+        if el[i] == r.exit_layer and top2[1] - top2[0] > 2 * logit_tol:   # argmax unique (R12)
+            assert lab[i] == r.label
+        if el[i] == r.exit_layer:
+            assert np.max(np.abs(lg[i] - r.logits)) < logit_tol, (i, lg[i], r.logits)
+            assert abs(conf[i] - r.metric) < logit_tol
+    return n_checked
+
+
+def _split_parity(api, cfg, W, model, X, ids, begin, end, tau, n_valid=None):
+    """GPU split on rows X vs oracle.run_split on the same rows."""
+    from oracle.model import run_split
+    B = cfg.batch
+    n_valid = len(ids) if n_valid is None else n_valid
+    xb = np.zeros((B, cfg.seq, cfg.hidden), np.float32)
+    xb[:len(X)] = X
+    idb = np.full(B, -1, np.int64)
+    idb[:len(ids)] = ids
+    split = api.Split(model, api.split_desc(cfg, begin, end, tau))
+    x = bf16_tensor(xb)
+    id_t = torch.from_numpy(idb).to(DEV)
+    x_out = torch.zeros_like(x)
+    id_out = torch.full((B,), -9, dtype=torch.int64, device=DEV)
+    n_surv = torch.zeros(1, dtype=torch.int32, device=DEV)
+    nv = torch.tensor([n_valid], dtype=torch.int32, device=DEV)
+    cap = int(max(ids)) + 1 if len(ids) else 1
+    ex = api.ExitBuffers(cap, cfg.classes, cfg.n_ramps, DEV)
+    split.run(x, id_t, x_out, id_out, n_surv, ex, n_valid=nv)
+    torch.cuda.synchronize()
+    ns = int(n_surv.item())
+    assert ns + int(ex.n_exit.item()) == n_valid                      # conservation
+    recs, surv_ids, h, margins = run_split(cfg, W, X[:n_valid], begin, end, ids=list(ids[:n_valid]),
+                                           tau=tau, mode="bf16")
+    _compare_records(recs, ex, [r.id for r in recs], cfg, MARGIN, LOGIT_TOL * (end - begin))
+    got_ids = id_out[:ns].cpu().tolist()
+    pos = {int(i): k for k, i in enumerate(ids)}
+    assert [pos[i] for i in got_ids] == sorted(pos[i] for i in got_ids)   # stable order
+    if all(m > MARGIN for m in margins.values()):
+        assert got_ids == surv_ids
+    assert torch.all(id_out[ns:] == -9)                               # nothing beyond n_surv
+    # survivor hidden states: same rows, one bf16 trajectory vs another
+    common = [i for i in got_ids if i in surv_ids]
+    if common:
+        g = to64(x_out[:ns])[[got_ids.index(i) for i in common]]
+        o = h[[surv_ids.index(i) for i in common]]
+        assert np.mean(np.abs(g - o)) < 5e-3 and np.max(np.abs(g - o)) < 0.25
+    return to64(x_out[:ns]).astype(np.float32), got_ids
+
+
+def test_split_run_per_split_parity_chain(api, tiny):
+    """Split [0,2) on a padded batch, then split [2,4) on the GPU's own
+    survivors: each run checked against the oracle on its exact input rows."""
+    cfg, W, model = tiny
+    X = e3data.make_inputs(cfg, range(cfg.batch))
+    rows, ids = _split_parity(api, cfg, W, model, X[:27], list(range(27)), 0, 2, cfg.tau)
+    _split_parity(api, cfg, W, model, rows, ids, 2, 4, cfg.tau)
+
+
+def test_pipeline_tiny_matches_oracle_and_simulator(api, tiny):
+    cfg, W, model = tiny
+    N = 256
+    X = e3data.make_inputs(cfg, range(N))
+    recs = oracle.run(cfg, W, X, mode="bf16")
+    ex = api.ExitBuffers(N, cfg.classes, cfg.n_ramps, DEV)
+    bounds = Plan.per_ramp(cfg.ramp_layers).bounds
+    for lag in (1, 0):
+        ex.reset()
+        pipe = api.Pipeline(model, api.make_plan(cfg, bounds, cfg.tau, lag=lag, trace=True))
+        st = pipe.run(bf16_tensor(X), torch.arange(N, dtype=torch.int64, device=DEV), ex)
+        n_checked = _compare_records(recs, ex, range(N), cfg, E2E_MARGIN, E2E_LOGIT_TOL)
+        assert n_checked >= 0.8 * N
+        assert int(ex.n_exit.item()) == N
+        trace = pipe.trace()
+        # every split batch has exactly B rows; padding only when flushed
+        assert all(0 < nv <= cfg.batch for _, nv, _ in trace)
+        exit_layer = {i: int(v) for i, v in enumerate(ex.exit_layer.cpu().numpy())}
+        sim = simulate_pipeline(exit_layer, list(range(N)), Plan(bounds), cfg.batch, lag=lag)
+        assert [(r.split, r.n_valid, r.ids) for r in sim.runs] == trace
+        for s in range(len(bounds) - 1):
+            assert st.batches[s] == sim.per_split[s]["batches"]
+            assert st.valid_rows[s] == sim.per_split[s]["valid"]
+            assert st.rows_out[s] == sim.per_split[s]["rows_out"]
+
+
+def test_pipeline_plan_invariance_inner_exact(api, tiny):
+    """inner = EXACT: one split holding both ramps == per-ramp splits (bitwise)."""
+    cfg, W, model = tiny
+    N = 100
+    X = bf16_tensor(e3data.make_inputs(cfg, range(N), seed=7))
+    ids = torch.arange(N, dtype=torch.int64, device=DEV)
+    outs = []
+    for bounds in ((0, 2, 4), (0, 4)):
+        ex = api.ExitBuffers(N, cfg.classes, cfg.n_ramps, DEV)
+        api.Pipeline(model, api.make_plan(cfg, bounds, cfg.tau)).run(X, ids, ex)
+        outs.append((ex.exit_layer.cpu(), ex.label.cpu(), ex.logits.cpu()))
+    assert torch.equal(outs[0][0], outs[1][0]) and torch.equal(outs[0][1], outs[1][1])
+    assert torch.equal(outs[0][2], outs[1][2])
+
+
+def test_pipeline_host_inputs_and_edge_sizes(api, tiny):
+    cfg, W, model = tiny
+    pipe = api.Pipeline(model, api.make_plan(cfg, (0, 2, 4), cfg.tau))
+    for N in (0, 1, 31, 33, 95):
+        X = e3data.make_inputs(cfg, range(N), seed=9)
+        ex = api.ExitBuffers(max(N, 1), cfg.classes, cfg.n_ramps, DEV)
+        xh = torch.from_numpy(X).to(torch.bfloat16).pin_memory() if N else torch.empty(0)
+        idh = torch.arange(N, dtype=torch.int64).pin_memory() if N else torch.empty(0, dtype=torch.int64)
+        st = pipe.run(xh, idh, ex)
+        assert int(ex.n_exit.item()) == N
+        if N:
+            recs = oracle.run(cfg, W, X, mode="bf16")
+            _compare_records(recs, ex, range(N), cfg, E2E_MARGIN, E2E_LOGIT_TOL)
+            assert sum(st.valid_rows[s] for s in range(2)) == N + int((ex.exit_layer[:N] > 1).sum())
+
+
+def test_rebatch_fifo_and_flush(api):
+    B, row = 8, 64
+    q = api.Queue(DEV, row * 2, 4 * B)
+    rows = torch.arange(5 * row, dtype=torch.float32, device=DEV).reshape(5, row).to(torch.bfloat16)
+    ids = torch.arange(100, 105, dtype=torch.int64, device=DEV)
+    n5 = torch.tensor([5], dtype=torch.int32, device=DEV)
+    x_out = torch.empty(B, row, dtype=torch.bfloat16, device=DEV)
+    id_out = torch.empty(B, dtype=torch.int64, device=DEV)
+    nv = torch.zeros(1, dtype=torch.int32, device=DEV)
+    q.push(rows, ids, n5, 5)
+    assert q.count() == 5
+    assert not q.rebatch(B, False, x_out, id_out, nv)               # 5 < B: wait
+    q.push(rows, ids, n5, 5)                                        # two partial batches ...
+    assert q.rebatch(B, False, x_out, id_out, nv)                   # ... fused into one of B
+    assert int(nv) == B and q.count() == 2
+    assert id_out.cpu().tolist() == [100, 101, 102, 103, 104, 100, 101, 102]
+    assert torch.equal(x_out[5:], rows[:3])
+    assert q.rebatch(B, True, x_out, id_out, nv)                    # flush: 2 valid + padding
+    assert int(nv) == 2 and id_out.cpu().tolist() == [103, 104] + [-1] * 6
+    assert torch.all(x_out[2:] == 0)
+    assert q.count() == 0 and not q.rebatch(B, True, x_out, id_out, nv)
+    # overflow is reported, never silently truncated
+    big = torch.zeros(40, row, dtype=torch.bfloat16, device=DEV)
+    bid = torch.zeros(40, dtype=torch.int64, device=DEV)
+    n40 = torch.tensor([40], dtype=torch.int32, device=DEV)
+    q.push(big, bid, n40, 40)
+    from paper_conf_sosp_iyergdpgn24_b200._lib import E3Error
+    with pytest.raises(E3Error, match="ECAPACITY"):
+        q.count()
+
+
+@pytest.fixture(scope="module")
+def bert_base(api):
+    from oracle.calibrate import load_tau
+    cfg = e3data.get("bb")
+    tau = load_tau(cfg)
+    W = e3data.make_weights(cfg)
+    model = api.DeviceModel(cfg, W, DEV)
+    return cfg, tau, W, model
+
+
+def test_bert_base_split_parity_full_size(api, bert_base):
+    """EE-BERT-base at the bench shape (B=64, S=128, H=768): split [0,1) on a
+    full batch, then split [1,2) on the GPU's survivors padded to B; every
+    row checked against the oracle on identical input rows."""
+    cfg, tau, W, model = bert_base
+    X = e3data.make_inputs(cfg, range(64))
+    rows, ids = _split_parity(api, cfg, W, model, X, list(range(64)), 0, 1, tau)
+    _split_parity(api, cfg, W, model, rows, ids, 1, 2, tau)
+
+
+def test_bert_base_pipeline_full_size_sampled(api, bert_base):
+    """The bench configuration end to end (12 per-ramp splits, calibrated
+    entropy thresholds): every input exits once, exit histogram ~ the target
+    profile, sampled inputs vs the chained oracle (R13 bounds)."""
+    cfg, tau, W, model = bert_base
+    N = 640
+    X = e3data.make_inputs(cfg, range(N))
+    ex = api.ExitBuffers(N, cfg.classes, cfg.n_ramps, DEV)
+    pipe = api.Pipeline(model, api.make_plan(cfg, Plan.per_ramp(cfg.ramp_layers).bounds, tau))
+    pipe.run(bf16_tensor(X), torch.arange(N, dtype=torch.int64, device=DEV), ex)
+    el = ex.exit_layer.cpu().numpy()
+    assert int(ex.n_exit.item()) == N and np.all(el >= 0)
+    hist = np.bincount(el, minlength=12) / N
+    assert np.all(np.abs(hist - np.array(cfg.exit_profile)) < 0.08), hist
+    sample = [int(i) for i in np.random.default_rng(0).choice(N, 6, replace=False)]
+    recs = oracle.run(cfg, W, X[sample], ids=sample, tau=tau, mode="bf16")
+    _compare_records(recs, ex, sample, cfg, E2E_MARGIN, E2E_LOGIT_TOL)

@@ -146,3 +146,21 @@ def test_calibration_hits_exit_profile():
     recs = run(cfg, W, Xm, tau=tau, mode="bf16")
     frac = np.array([sum(r.ramp == k for r in recs) for k in range(4)]) / 400.0
     assert np.all(np.abs(frac - np.array(cfg.exit_profile)) < 0.08), frac
+
+
+@pytest.mark.parametrize("bounds", [(0, 2, 4), (0, 4)])
+def test_run_split_composes_to_run(tiny, bounds):
+    """Chaining run_split over a plan (inner EXACT) reproduces run (plan invariance)."""
+    from oracle.model import run_split
+    W, X = tiny
+    full = {r.id: r for r in run(TINY, W, X, mode="bf16")}
+    ids = list(range(len(X)))
+    h = X.astype(np.float64)
+    got = {}
+    for b, e in zip(bounds[:-1], bounds[1:]):
+        recs, ids, h, _ = run_split(TINY, W, h, b, e, ids=ids, mode="bf16")
+        got.update({r.id: r for r in recs})
+    assert not ids and set(got) == set(full)
+    for i, r in got.items():
+        assert (r.exit_layer, r.label) == (full[i].exit_layer, full[i].label)
+        assert np.max(np.abs(r.logits - full[i].logits)) < 1e-12
