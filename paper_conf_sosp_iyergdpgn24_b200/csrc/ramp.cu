@@ -6,19 +6,21 @@
 // exit test (R3/R4/R12): max softmax(z) > tau, or
 // entropy(softmax(z)) < tau; the model's last ramp exits every row (R6).
 //
-// One launch, two phases:
-//   phase 1 (all CTAs)  CTA (j, g) computes pooler outputs 8j..8j+7 for rows
-//                       16g..16g+15: warp = one output, lanes split H in
-//                       16-byte vectors, W_p row held in registers, CLS
-//                       vectors of 4 rows in flight at once, dot products
-//                       reduced with __shfl_xor_sync; fp32 result to a [B,H]
-//                       workspace.
-//   phase 2 (last CTA   the CTA of row group g that retires last (threadfence +
-//    of each group)     atomic ticket per group) runs the classifier of its 16
-//                       rows: warp per row, lanes split H in 8-wide vectors,
-//                       per-class warp-shuffle reductions, then softmax /
-//                       max-prob / entropy, argmax (lowest index on ties),
-//                       threshold test, exit record by id, alive flag.
+// One launch; grid (H / 32 pooler-output tiles, ceil(B / 16) row groups),
+// 4 warps per CTA:
+//   stage    cp.async the 16 CLS rows and the 32 W_p rows of the tile into
+//            padded smem (row pitch H + 8 bf16: conflict-free fragments);
+//   pooler   warp w owns outputs 8w..8w+7 of the tile: mma.sync m16n8k16
+//            bf16 -> fp32 over K = H (a 16 x 32 x H GEMM per CTA is far too
+//            small for a tcgen05 tile; the tensor pipe is still the one used);
+//   partial  p = tanh(acc + b_p) stays in registers and is immediately folded
+//            into partial logits sum_{o in tile} p[b,o] W_c[c,o], reduced over
+//            the quad with __shfl_xor_sync and over the 4 warps in smem, and
+//            written to a per-tile slot (deterministic, no float atomics);
+//   decide   the CTA of row group g that retires last (threadfence + atomic
+//            ticket) sums the H/32 partials per (row, class) in fixed order,
+//            then softmax / max-prob / entropy, argmax (lowest index on ties),
+//            threshold test, exit record by input id and the alive flag.
 // All ramp math is fp32, never rounded to bf16 (rounding contract).
 #include "common.cuh"
 #include "kernels.h"
@@ -29,180 +31,205 @@ namespace e3 {
 namespace {
 
 constexpr int kMaxC = 16;
-constexpr int kRowsPerCta = kRampRowsPerCta;
-constexpr int kRowUnroll = 4;   // rows whose CLS vectors are in flight together
+constexpr int kRows = kRampRowsPerCta;   // 16 = mma M
+constexpr int kTileN = 32;               // pooler outputs per CTA (4 warps x n8)
+constexpr int kThreads = 128;
 
-__device__ __forceinline__ float dot8(uint4 c4, uint4 w4, float acc) {
-  const uint32_t cw[4] = {c4.x, c4.y, c4.z, c4.w};
-  const uint32_t ww[4] = {w4.x, w4.y, w4.z, w4.w};
-#pragma unroll
-  for (int e = 0; e < 4; ++e) {
-    acc = fmaf(bf_lo(cw[e]), bf_lo(ww[e]), acc);
-    acc = fmaf(bf_hi(cw[e]), bf_hi(ww[e]), acc);
-  }
-  return acc;
+__device__ __forceinline__ void cp_async16(void *smem, const void *gmem) {
+  asm volatile("cp.async.cg.shared.global [%0], [%1], 16;" ::"r"(smem_u32(smem)), "l"(gmem) : "memory");
+}
+__device__ __forceinline__ void cp_async_wait_all() { asm volatile("cp.async.wait_all;" ::: "memory"); }
+
+__device__ __forceinline__ void mma_bf16_16816(float (&d)[4], const uint32_t (&a)[4], uint32_t b0, uint32_t b1) {
+  asm volatile(
+      "mma.sync.aligned.m16n8k16.row.col.f32.bf16.bf16.f32 {%0, %1, %2, %3}, {%4, %5, %6, %7}, {%8, %9}, "
+      "{%0, %1, %2, %3};"
+      : "+f"(d[0]), "+f"(d[1]), "+f"(d[2]), "+f"(d[3])
+      : "r"(a[0]), "r"(a[1]), "r"(a[2]), "r"(a[3]), "r"(b0), "r"(b1));
 }
 
 __device__ __forceinline__ bool row_alive(const RampArgs &a, int b, int n_valid) {
   return b < a.B && (a.init_alive ? (b < n_valid) : (a.alive[b] != 0));
 }
 
-// grid (H/8 pooler-output groups, ceil(B/16) row groups); 8 warps per CTA
-template <int VPL>
-__global__ void __launch_bounds__(256)
+__global__ void __launch_bounds__(kThreads)
     ramp_bert_kernel(RampArgs a) {
-  const int warp = warp_id(), lane = lane_id();
+  extern __shared__ uint8_t smem_raw[];
   const int H = a.H;
+  const int P = H + 8;                                   // padded pitch (bf16)
+  __nv_bfloat16 *sC = reinterpret_cast<__nv_bfloat16 *>(smem_raw);   // [16][P]
+  __nv_bfloat16 *sW = sC + kRows * P;                                 // [32][P]
+  float *sZ = reinterpret_cast<float *>(sW + kTileN * P);             // [4 warps][16 rows][kMaxC]
+  __shared__ bool is_last;
+  __shared__ bool row_ok[kRows];
+
+  const int warp = warp_id(), lane = lane_id();
+  const int g = lane >> 2, t = lane & 3;
+  const int b0 = blockIdx.y * kRows;
+  const int o0 = blockIdx.x * kTileN;
+  const int C = a.C;
+  const int n_valid = a.n_valid_dev ? *a.n_valid_dev : a.n_valid_host;
   const int nvec = H / 8;
   const __nv_bfloat16 *x = reinterpret_cast<const __nv_bfloat16 *>(a.x);
   const size_t row_stride = (size_t)a.S * H;
-  const int n_valid = a.n_valid_dev ? *a.n_valid_dev : a.n_valid_host;
-  const int b0 = blockIdx.y * kRowsPerCta;
 
-  // ---------------------------------------------------------- phase 1
-  // warp = pooler output o; its W_p row lives in registers; the CLS vectors
-  // of kRowUnroll rows are loaded before any arithmetic (memory parallelism).
+  // ---------------------------------------------------------- stage
+  if (threadIdx.x < kRows) row_ok[threadIdx.x] = row_alive(a, b0 + threadIdx.x, n_valid);
+  __syncthreads();
+  for (int i = threadIdx.x; i < kRows * nvec; i += kThreads) {
+    const int r = i / nvec, k = i - r * nvec;
+    uint4 *dst = reinterpret_cast<uint4 *>(sC + r * P) + k;
+    if (row_ok[r])
+      cp_async16(dst, reinterpret_cast<const uint4 *>(x + (size_t)(b0 + r) * row_stride) + k);
+    else
+      *dst = make_uint4(0, 0, 0, 0);
+  }
+  const uint4 *wp = reinterpret_cast<const uint4 *>(a.w.w_p);
+  for (int i = threadIdx.x; i < kTileN * nvec; i += kThreads) {
+    const int r = i / nvec, k = i - r * nvec;
+    cp_async16(reinterpret_cast<uint4 *>(sW + r * P) + k, wp + (size_t)(o0 + r) * nvec + k);
+  }
+  cp_async_wait_all();
+  __syncthreads();
+
+  // ---------------------------------------------------------- pooler (mma.sync)
+  float acc[4] = {0.f, 0.f, 0.f, 0.f};
   {
-    const int o = blockIdx.x * 8 + warp;
-    const uint4 *wrow = reinterpret_cast<const uint4 *>(a.w.w_p) + (size_t)o * nvec;
-    uint4 w[VPL];
-#pragma unroll
-    for (int i = 0; i < VPL; ++i) {
-      const int k = lane + 32 * i;
-      w[i] = (k < nvec) ? __ldg(wrow + k) : make_uint4(0, 0, 0, 0);
+    const __nv_bfloat16 *a_lo = sC + g * P + 2 * t;           // row g
+    const __nv_bfloat16 *a_hi = sC + (g + 8) * P + 2 * t;     // row g + 8
+    const __nv_bfloat16 *bp = sW + (warp * 8 + g) * P + 2 * t;
+#pragma unroll 4
+    for (int kk = 0; kk < H; kk += 16) {
+      uint32_t af[4];
+      af[0] = *reinterpret_cast<const uint32_t *>(a_lo + kk);
+      af[1] = *reinterpret_cast<const uint32_t *>(a_hi + kk);
+      af[2] = *reinterpret_cast<const uint32_t *>(a_lo + kk + 8);
+      af[3] = *reinterpret_cast<const uint32_t *>(a_hi + kk + 8);
+      const uint32_t bf0 = *reinterpret_cast<const uint32_t *>(bp + kk);
+      const uint32_t bf1 = *reinterpret_cast<const uint32_t *>(bp + kk + 8);
+      mma_bf16_16816(acc, af, bf0, bf1);
     }
-    const float bias = bf2f(reinterpret_cast<const __nv_bfloat16 *>(a.w.b_p)[o]);
-#pragma unroll 1
-    for (int r0 = b0; r0 < b0 + kRowsPerCta; r0 += kRowUnroll) {
-      uint4 c[kRowUnroll][VPL];
-      bool al[kRowUnroll];
+  }
+
+  // ---------------------------------------------------------- partial logits
+  {
+    const __nv_bfloat16 *bpool = reinterpret_cast<const __nv_bfloat16 *>(a.w.b_p);
+    const __nv_bfloat16 *wc = reinterpret_cast<const __nv_bfloat16 *>(a.w.w_c);
+    const int col = o0 + warp * 8 + 2 * t;                  // this lane's two pooler outputs
+    const float bb0 = bf2f(bpool[col]), bb1 = bf2f(bpool[col + 1]);
+    const float p00 = tanhf(acc[0] + bb0), p01 = tanhf(acc[1] + bb1);   // row g
+    const float p10 = tanhf(acc[2] + bb0), p11 = tanhf(acc[3] + bb1);   // row g + 8
 #pragma unroll
-      for (int u = 0; u < kRowUnroll; ++u) {
-        al[u] = row_alive(a, r0 + u, n_valid);
-        const uint4 *cr = reinterpret_cast<const uint4 *>(x + (size_t)(r0 + u) * row_stride);
-#pragma unroll
-        for (int i = 0; i < VPL; ++i) {
-          const int k = lane + 32 * i;
-          c[u][i] = (al[u] && k < nvec) ? __ldg(cr + k) : make_uint4(0, 0, 0, 0);
+    for (int c = 0; c < kMaxC; ++c) {
+      if (c < C) {
+        const float w0 = bf2f(wc[(size_t)c * H + col]), w1 = bf2f(wc[(size_t)c * H + col + 1]);
+        float z0 = fmaf(p00, w0, p01 * w1);
+        float z1 = fmaf(p10, w0, p11 * w1);
+        z0 += __shfl_xor_sync(0xffffffffu, z0, 1);
+        z0 += __shfl_xor_sync(0xffffffffu, z0, 2);
+        z1 += __shfl_xor_sync(0xffffffffu, z1, 1);
+        z1 += __shfl_xor_sync(0xffffffffu, z1, 2);
+        if (t == 0) {
+          sZ[(warp * kRows + g) * kMaxC + c] = z0;
+          sZ[(warp * kRows + g + 8) * kMaxC + c] = z1;
         }
       }
+    }
+  }
+  __syncthreads();
+  float *part = a.pool_ws;   // [gridDim.x tiles][B][C]
+  for (int i = threadIdx.x; i < kRows * C; i += kThreads) {
+    const int r = i / C, c = i - r * C;
+    if (b0 + r < a.B) {
+      float s = sZ[(0 * kRows + r) * kMaxC + c];
 #pragma unroll
-      for (int u = 0; u < kRowUnroll; ++u) {
-        if (!al[u]) continue;   // warp-uniform
-        float acc = 0.f;
-#pragma unroll
-        for (int i = 0; i < VPL; ++i) acc = dot8(c[u][i], w[i], acc);
-#pragma unroll
-        for (int s = 16; s; s >>= 1) acc += __shfl_xor_sync(0xffffffffu, acc, s);
-        if (lane == 0) a.pool_ws[(size_t)(r0 + u) * H + o] = tanhf(acc + bias);
-      }
+      for (int w = 1; w < 4; ++w) s += sZ[(w * kRows + r) * kMaxC + c];
+      part[((size_t)blockIdx.x * a.B + b0 + r) * C + c] = s;
     }
   }
 
   // ---------------------------------------------------------- ticket
-  // the last CTA of this row group (over the H/8 output groups) classifies it
-  __shared__ bool is_last;
   __threadfence();
   __syncthreads();
   if (threadIdx.x == 0) {
-    const unsigned t = atomicAdd(a.done_ctr + blockIdx.y, 1u);
-    is_last = (t == gridDim.x - 1);
+    const unsigned tk = atomicAdd(a.done_ctr + blockIdx.y, 1u);
+    is_last = (tk == gridDim.x - 1);
     if (is_last) a.done_ctr[blockIdx.y] = 0;   // re-arm for the next launch (stream-ordered)
   }
   __syncthreads();
   if (!is_last) return;
   __threadfence();
 
-  // ---------------------------------------------------------- phase 2
-  // warp per row: lanes split H into 8-wide vectors, one warp-shuffle
-  // reduction per class, then softmax / metric / test on lane 0.
-  const int C = a.C;
-  const uint4 *wc = reinterpret_cast<const uint4 *>(a.w.w_c);
+  // ---------------------------------------------------------- decide
+  // gather the group's partials [tiles][16 rows][C] into smem with all loads
+  // independent (one L2 round trip), then one thread per row sums them in
+  // fixed tile order.
+  float *sP = reinterpret_cast<float *>(smem_raw);   // reuse the staging area
+  const int ntiles = gridDim.x;
+  const int per_tile = kRows * C;
+  for (int i = threadIdx.x; i < ntiles * per_tile; i += kThreads) {
+    const int nt = i / per_tile, rc = i - nt * per_tile;
+    const int rr = rc / C;
+    sP[i] = (b0 + rr < a.B) ? __ldcg(part + ((size_t)nt * a.B + b0) * C + rc) : 0.f;
+  }
+  __syncthreads();
+  const int r = threadIdx.x;
+  if (r >= kRows || b0 + r >= a.B) return;
+  const int b = b0 + r;
+  if (!row_ok[r]) {
+    if (a.init_alive) a.alive[b] = 0;
+    return;
+  }
   const __nv_bfloat16 *bc = reinterpret_cast<const __nv_bfloat16 *>(a.w.b_c);
-  const float tau = a.tau;
-  for (int b = b0 + warp; b < b0 + kRowsPerCta && b < a.B; b += 8) {
-    if (!row_alive(a, b, n_valid)) {
-      if (a.init_alive && lane == 0) a.alive[b] = 0;
-      continue;
-    }
-    const float4 *pr = reinterpret_cast<const float4 *>(a.pool_ws + (size_t)b * H);
-    float p[VPL][8];
+  float z[kMaxC];
 #pragma unroll
-    for (int i = 0; i < VPL; ++i) {
-      const int k = lane + 32 * i;
-      const float4 lo = (k < nvec) ? __ldcg(pr + 2 * k) : make_float4(0.f, 0.f, 0.f, 0.f);
-      const float4 hi = (k < nvec) ? __ldcg(pr + 2 * k + 1) : make_float4(0.f, 0.f, 0.f, 0.f);
-      p[i][0] = lo.x; p[i][1] = lo.y; p[i][2] = lo.z; p[i][3] = lo.w;
-      p[i][4] = hi.x; p[i][5] = hi.y; p[i][6] = hi.z; p[i][7] = hi.w;
-    }
-    float z[kMaxC];
-#pragma unroll
-    for (int c = 0; c < kMaxC; ++c) {
-      z[c] = 0.f;
-      if (c < C) {
-        uint4 wv[VPL];
-#pragma unroll
-        for (int i = 0; i < VPL; ++i) {
-          const int k = lane + 32 * i;
-          wv[i] = (k < nvec) ? __ldg(wc + (size_t)c * nvec + k) : make_uint4(0, 0, 0, 0);
-        }
-        float acc = 0.f;
-#pragma unroll
-        for (int i = 0; i < VPL; ++i) {
-          const uint32_t ww[4] = {wv[i].x, wv[i].y, wv[i].z, wv[i].w};
-#pragma unroll
-          for (int e = 0; e < 4; ++e) {
-            acc = fmaf(p[i][2 * e], bf_lo(ww[e]), acc);
-            acc = fmaf(p[i][2 * e + 1], bf_hi(ww[e]), acc);
-          }
-        }
-#pragma unroll
-        for (int s = 16; s; s >>= 1) acc += __shfl_xor_sync(0xffffffffu, acc, s);
-        z[c] = acc + bf2f(bc[c]);
-      }
-    }
-    if (lane == 0) {
-      float m = z[0];
-      int label = 0;
-#pragma unroll
-      for (int c = 1; c < kMaxC; ++c)
-        if (c < C && z[c] > m) { m = z[c]; label = c; }   // lowest index on ties
-      float sum = 0.f, qz = 0.f;
-#pragma unroll
-      for (int c = 0; c < kMaxC; ++c)
-        if (c < C) {
-          const float e = expf(z[c] - m);
-          sum += e;
-          qz += e * (z[c] - m);
-        }
-      float metric;
-      bool pass;
-      if (a.test == E3_TEST_MAXPROB) {
-        metric = 1.0f / sum;                       // max_c softmax(z)_c
-        pass = metric > tau;
-      } else {
-        metric = logf(sum) - qz / sum;             // H = lse - sum_c q_c z_c
-        pass = metric < tau;
-      }
-      const bool exit_now = pass || a.final_ramp;
-      if (exit_now) {
-        const int64_t id = a.id[b];
-        if (id >= 0 && id < a.ex.capacity) {
-          if (a.ex.exit_layer) a.ex.exit_layer[id] = a.layer;
-          if (a.ex.label) a.ex.label[id] = label;
-          if (a.ex.conf) a.ex.conf[id] = metric;
-          if (a.ex.logits) {
-#pragma unroll
-            for (int c = 0; c < kMaxC; ++c)
-              if (c < C) a.ex.logits[id * C + c] = z[c];
-          }
-        }
-        if (a.ex.n_exit) atomicAdd(a.ex.n_exit, 1);
-        if (a.ex.ramp_count) atomicAdd(a.ex.ramp_count + a.ramp_index, 1);
-      }
-      a.alive[b] = exit_now ? 0 : 1;
+  for (int c = 0; c < kMaxC; ++c) {
+    z[c] = 0.f;
+    if (c < C) {
+      float s = 0.f;
+      for (int nt = 0; nt < ntiles; ++nt) s += sP[nt * per_tile + r * C + c];
+      z[c] = s + bf2f(bc[c]);
     }
   }
+  float m = z[0];
+  int label = 0;
+#pragma unroll
+  for (int c = 1; c < kMaxC; ++c)
+    if (c < C && z[c] > m) { m = z[c]; label = c; }   // lowest index on ties
+  float sum = 0.f, qz = 0.f;
+#pragma unroll
+  for (int c = 0; c < kMaxC; ++c)
+    if (c < C) {
+      const float e = expf(z[c] - m);
+      sum += e;
+      qz += e * (z[c] - m);
+    }
+  float metric;
+  bool pass;
+  if (a.test == E3_TEST_MAXPROB) {
+    metric = 1.0f / sum;                       // max_c softmax(z)_c
+    pass = metric > a.tau;
+  } else {
+    metric = logf(sum) - qz / sum;             // H = lse - sum_c q_c z_c
+    pass = metric < a.tau;
+  }
+  const bool exit_now = pass || a.final_ramp;
+  if (exit_now) {
+    const int64_t id = a.id[b];
+    if (id >= 0 && id < a.ex.capacity) {
+      if (a.ex.exit_layer) a.ex.exit_layer[id] = a.layer;
+      if (a.ex.label) a.ex.label[id] = label;
+      if (a.ex.conf) a.ex.conf[id] = metric;
+      if (a.ex.logits) {
+#pragma unroll
+        for (int c = 0; c < kMaxC; ++c)
+          if (c < C) a.ex.logits[id * C + c] = z[c];
+      }
+    }
+    if (a.ex.n_exit) atomicAdd(a.ex.n_exit, 1);
+    if (a.ex.ramp_count) atomicAdd(a.ex.ramp_count + a.ramp_index, 1);
+  }
+  a.alive[b] = exit_now ? 0 : 1;
 }
 
 }  // namespace
@@ -212,17 +239,19 @@ e3_status ramp_run(const RampArgs &a, cudaStream_t st) {
     set_error("ramp: only the BERT (pooler) ramp is implemented");
     return E3_EUNSUPPORTED;
   }
-  if (a.C < 1 || a.C > kMaxC || a.H % 8 || a.H > 4096) {
-    set_error("ramp: need 1 <= C <= 16, H % 8 == 0, H <= 4096");
+  if (a.C < 1 || a.C > kMaxC || a.H % kTileN || a.H > 1024) {
+    set_error("ramp: need 1 <= C <= 16, H % 32 == 0, H <= 1024");
     return E3_EUNSUPPORTED;
   }
-  dim3 grid(a.H / 8, (a.B + kRowsPerCta - 1) / kRowsPerCta);
-  const int vpl = (a.H / 8 + 31) / 32;
-  if (vpl <= 1) ramp_bert_kernel<1><<<grid, 256, 0, st>>>(a);
-  else if (vpl <= 3) ramp_bert_kernel<3><<<grid, 256, 0, st>>>(a);
-  else if (vpl <= 4) ramp_bert_kernel<4><<<grid, 256, 0, st>>>(a);
-  else if (vpl <= 8) ramp_bert_kernel<8><<<grid, 256, 0, st>>>(a);
-  else ramp_bert_kernel<16><<<grid, 256, 0, st>>>(a);
+  const int smem = (kRows + kTileN) * (a.H + 8) * 2 + 4 * kRows * kMaxC * 4;
+  static bool attr_done = false;
+  if (!attr_done) {
+    E3_CUDA_TRY(cudaFuncSetAttribute(ramp_bert_kernel, cudaFuncAttributeMaxDynamicSharedMemorySize,
+                                     (kRows + kTileN) * (1024 + 8) * 2 + 4 * kRows * kMaxC * 4));
+    attr_done = true;
+  }
+  dim3 grid(a.H / kTileN, (a.B + kRows - 1) / kRows);
+  ramp_bert_kernel<<<grid, kThreads, smem, st>>>(a);
   E3_CUDA_TRY(cudaGetLastError());
   count_launch();
   return E3_OK;
