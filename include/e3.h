@@ -144,7 +144,7 @@ typedef struct e3_split e3_split;
 /* Validates the descriptor, checks the device is sm_100, borrows the weights
  * (layers [layer_begin, layer_end), the listed ramps) and allocates the
  * handle-owned workspace for batch B.  E3_EUNSUPPORTED for shapes outside the
- * kernels' tiling (H % 64, F % 64, head_dim != 64, S > 256, B*S % 128 ...). */
+ * kernels' tiling (H % 128, F % 128, head_dim != 64, S > 256, C > 16, B > 4096). */
 e3_status e3_split_create(const e3_split_desc *d, const e3_weights *w, int device, e3_split **out);
 e3_status e3_split_destroy(e3_split *s);
 

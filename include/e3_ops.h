@@ -24,7 +24,7 @@ typedef enum {
 } e3_epilogue;
 
 /* Layer GEMM on tcgen05 tensor cores (a2): C[M,N] = epi(A[M,K] W[N,K]^T).
- * A row pitch lda (elements), C / R row pitch N.  K % 64 == 0, N % 64 == 0,
+ * A row pitch lda (elements), C / R row pitch N.  K % 128 == 0, N % 64 == 0,
  * 16-byte aligned pointers.  fp32 accumulation in TMEM; one rounding to bf16. */
 e3_status e3_op_gemm(void *stream, const void *A, int64_t lda, const void *W, const void *bias,
                      const void *resid, void *C, int32_t M, int32_t N, int32_t K, int32_t epilogue);

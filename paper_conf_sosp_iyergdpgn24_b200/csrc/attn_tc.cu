@@ -1,15 +1,24 @@
 // Self-attention of the split's encoder layers on the
 // sm_100a tensor cores.  S <= 256 fits one KV tile, so there is no online
-// rescaling: one CTA owns (input b, head h, 128-query tile):
+// rescaling.  A work item is (input b, head h, 128-query tile):
 //
 //   TMA   Q [128x64], K [SKVx64], V [SKVx64] (128B swizzle, OOB rows -> 0)
 //   MMA1  S = Q K^T          tcgen05 128 x SKV x 64, fp32 in TMEM
-//   soft  thread r owns query row r (TMEM lane r): row max, p = 2^((s-m)*log2e/8),
-//         l = sum p (fp32, unrounded), bf16(p) -> smem in the K-major SW128
-//         layout the next MMA reads as its A operand
-//   MMA2  O = P V            tcgen05 128 x 64 x SKV, V read MN-major
-//   out   ctx = bf16(O / l)  (rounding contract)
+//   soft  query row r = TMEM lane r is shared by two threads (warps w and
+//         w+4 own lane quarter w and one half of the keys each): row max and
+//         sum l of p = 2^((s-m) log2e / 8) combined through smem; l is fp32 of
+//         the UNROUNDED p; bf16(p) -> smem in the K-major SW128 layout the
+//         next MMA reads as its A operand
+//   MMA2  O = P V            tcgen05 128 x 64 x SKV, V read MN-major; O reuses
+//         the S columns of TMEM (S is dead once the softmax has read it)
+//   out   ctx = bf16(O / l)  (rounding contract), staged in smem
+//         with the 128B swizzle and written by one TMA store of the
+//         [128 q x 64 d] box (rows >= S clipped by the 3-D tensor map)
 //
+// Persistent CTAs (2 per SM for SKV = 128) walk the items with the Q/K/V
+// tiles double buffered: the next item's loads fly while the current item
+// runs.  P overwrites the current item's dead Q|K tiles and the output tile is
+// staged in the dead V tile, so a CTA needs 96 KB of smem and 128 TMEM columns.
 // Keys >= S are masked to -inf; query rows >= S are not stored.
 #include "common.cuh"
 #include "kernels.h"
@@ -20,43 +29,54 @@ namespace e3 {
 namespace {
 
 constexpr int D = 64;          // head dim
-constexpr int QT = 128;        // query rows per CTA
+constexpr int QT = 128;        // query rows per item
+constexpr int kThreads = 256;  // 8 warps: two threads per query row
 
 template <int SKV>
 struct ACfg {
-  static constexpr int kQ = QT * D * 2;          // 16 KB
-  static constexpr int kKV = SKV * D * 2;        // 16 / 32 KB
-  static constexpr int kP = QT * SKV * 2;        // 32 / 64 KB
-  static constexpr int kSmem = kQ + 2 * kKV + kP + 1024 + 64;
-  static constexpr int kTmemCols = (SKV + D <= 256) ? 256 : 512;
+  static constexpr int kQ = QT * D * 2;                  // 16 KB
+  static constexpr int kKV = SKV * D * 2;                // 16 / 32 KB
+  static constexpr int kP = QT * SKV * 2;                // 32 / 64 KB
+  static constexpr int kBuf = kQ + 2 * kKV;              // Q | K | V
+  static constexpr int kNBuf = (SKV == 128) ? 2 : 1;     // double buffer when it fits
+  static constexpr bool kPInQK = (kP <= kQ + kKV);       // P overwrites the dead Q|K tiles
+  static constexpr int kSmem = kNBuf * kBuf + (kPInQK ? 0 : kP) + 1024 + 64 + 2 * 2 * QT * 4;
+  static constexpr int kTmemCols = SKV <= 128 ? 128 : 256;   // S, later O (64 columns)
 };
 
 template <int SKV>
-__global__ void __launch_bounds__(128)
+__global__ void __launch_bounds__(kThreads)
     attn_tc_kernel(const __grid_constant__ CUtensorMap tq, const __grid_constant__ CUtensorMap tkv,
-                   __nv_bfloat16 *__restrict__ ctx, int S, int H, int heads) {
+                   const __grid_constant__ CUtensorMap tctx, int S, int H, int heads, int n_items) {
   using CF = ACfg<SKV>;
+  constexpr int HALF = SKV / 2;     // keys per thread
   extern __shared__ uint8_t smem_raw[];
   uint8_t *smem = reinterpret_cast<uint8_t *>((reinterpret_cast<uintptr_t>(smem_raw) + 1023) & ~uintptr_t(1023));
-  uint8_t *sQ = smem;
-  uint8_t *sK = sQ + CF::kQ;
-  uint8_t *sV = sK + CF::kKV;
-  uint8_t *sP = sV + CF::kKV;
-  uint64_t *bars = reinterpret_cast<uint64_t *>(sP + CF::kP);   // [0] load, [1] S, [2] O
-  uint32_t *tslot = reinterpret_cast<uint32_t *>(bars + 3);
+  uint8_t *pbuf_sep = smem + CF::kNBuf * CF::kBuf;      // only when !kPInQK
+  float *xch = reinterpret_cast<float *>(smem + CF::kNBuf * CF::kBuf + (CF::kPInQK ? 0 : CF::kP));  // [2][2][QT]
+  uint64_t *bars = reinterpret_cast<uint64_t *>(xch + 2 * 2 * QT);
+  uint64_t *bar_load = bars;        // [2]
+  uint64_t *bar_s = bars + 2;
+  uint64_t *bar_o = bars + 3;
+  uint32_t *tslot = reinterpret_cast<uint32_t *>(bars + 4);
 
-  const int bh = blockIdx.x;
-  const int b = bh / heads, h = bh % heads;
-  const int q0 = blockIdx.y * QT;
   const int warp = warp_id(), lane = lane_id();
   const int tid = threadIdx.x;
+  const int qtiles = (S + QT - 1) / QT;
+  const int quarter = warp & 3;
+  const int khalf = warp >> 2;                            // which half of the keys / of D
+  const int row = quarter * 32 + lane;                    // query row within tile == TMEM lane
+  const uint32_t lane_off = (uint32_t)(quarter * 32) << 16;
+  const float sl2 = 1.4426950408889634f * 0.125f;         // log2(e) / sqrt(64)
 
   if (tid == 0) {
     tma_prefetch(&tq);
     tma_prefetch(&tkv);
-    mbar_init(&bars[0], 1);
-    mbar_init(&bars[1], 1);
-    mbar_init(&bars[2], 1);
+    tma_prefetch(&tctx);
+    mbar_init(&bar_load[0], 1);
+    mbar_init(&bar_load[1], 1);
+    mbar_init(bar_s, 1);
+    mbar_init(bar_o, 1);
     fence_barrier_init();
   }
   if (warp == 0) tmem_alloc(tslot, CF::kTmemCols);
@@ -64,139 +84,196 @@ __global__ void __launch_bounds__(128)
   __syncthreads();
   tc_fence_after();
   const uint32_t tbase = *tslot;
-  const uint32_t t_s = tbase;          // S accumulator: columns [0, SKV)
-  const uint32_t t_o = tbase + SKV;    // O accumulator: columns [SKV, SKV+64)
 
-  if (tid == 0) {
-    mbar_expect_tx(&bars[0], CF::kQ + 2 * CF::kKV);
-    tma_load_3d(sQ, &tq, &bars[0], h * D, q0, b);
-    tma_load_3d(sK, &tkv, &bars[0], H + h * D, 0, b);
-    tma_load_3d(sV, &tkv, &bars[0], 2 * H + h * D, 0, b);
-    mbar_wait(&bars[0], 0);
+  auto issue_load = [&](int item, int buf) {
+    const int bh = item / qtiles, qt = item % qtiles;
+    const int b = bh / heads, h = bh % heads;
+    uint8_t *base = smem + buf * CF::kBuf;
+    mbar_expect_tx(&bar_load[buf], CF::kBuf);
+    tma_load_3d(base, &tq, &bar_load[buf], h * D, qt * QT, b);
+    tma_load_3d(base + CF::kQ, &tkv, &bar_load[buf], H + h * D, 0, b);
+    tma_load_3d(base + CF::kQ + CF::kKV, &tkv, &bar_load[buf], 2 * H + h * D, 0, b);
+  };
+
+  int item = blockIdx.x;
+  if (tid == 0 && item < n_items) issue_load(item, 0);
+  uint32_t load_phases = 0;                               // bit i: parity of bar_load[i]
+  uint32_t sphase = 0, ophase = 0;
+
+  for (int j = 0; item < n_items; ++j, item += gridDim.x) {
+    const int buf = (CF::kNBuf == 2) ? (j & 1) : 0;
+    uint8_t *sQ = smem + buf * CF::kBuf;
+    uint8_t *sK = sQ + CF::kQ;
+    uint8_t *sV = sK + CF::kKV;
+    uint8_t *sP = CF::kPInQK ? sQ : pbuf_sep;
+    const int bh = item / qtiles, qt = item % qtiles;
+    const int b = bh / heads, h = bh % heads;
+    const int q0 = qt * QT;
+    const int next = item + gridDim.x;
+
+    if (tid == 0) {
+      mbar_wait(&bar_load[buf], (load_phases >> buf) & 1u);
+      tc_fence_after();
+      const uint32_t idesc = idesc_bf16_f32(QT, SKV, 0);
+      const uint64_t dq = smem_desc_sw128(smem_u32(sQ), 16, 1024);
+      const uint64_t dk = smem_desc_sw128(smem_u32(sK), 16, 1024);
+#pragma unroll
+      for (int k = 0; k < D / 16; ++k) tc_mma_f16(tbase, dq + 2 * k, dk + 2 * k, idesc, k != 0);
+      tc_commit(bar_s);
+      if (CF::kNBuf == 2 && next < n_items) {
+        // the other buffer's last readers: MMA2 of item j-1 (done: waited before
+        // its epilogue) and the TMA store of its output from the V tile
+        bulk_wait_read<0>();
+        issue_load(next, buf ^ 1);
+      }
+    }
+    load_phases ^= 1u << buf;
+    __syncwarp();
+
+    // ------------------------------------------------------------ softmax
+    mbar_wait(bar_s, sphase);
+    sphase ^= 1;
     tc_fence_after();
-    const uint32_t idesc = idesc_bf16_f32(QT, SKV, 0);
-    const uint64_t dq = smem_desc_sw128(smem_u32(sQ), 16, 1024);
-    const uint64_t dk = smem_desc_sw128(smem_u32(sK), 16, 1024);
-#pragma unroll
-    for (int k = 0; k < D / 16; ++k) tc_mma_f16(t_s, dq + 2 * k, dk + 2 * k, idesc, k != 0);
-    tc_commit(&bars[1]);
-  }
-  __syncwarp();
-
-  // ------------------------------------------------------------ softmax
-  mbar_wait(&bars[1], 0);
-  tc_fence_after();
-  const int row = warp * 32 + lane;                       // query row within tile == TMEM lane
-  const uint32_t lane_off = (uint32_t)(warp * 32) << 16;
-  float mx = -INFINITY;
+    const int c_begin = khalf * HALF;
+    float mx = -INFINITY;
 #pragma unroll 1
-  for (int c = 0; c < SKV; c += 32) {
-    uint32_t r[32];
-    tmem_ld32(t_s + lane_off + c, r);
-    tmem_wait_ld();
+    for (int c = c_begin; c < c_begin + HALF; c += 32) {
+      uint32_t r[32];
+      tmem_ld32(tbase + lane_off + c, r);
+      tmem_wait_ld();
+      float m4[4] = {-INFINITY, -INFINITY, -INFINITY, -INFINITY};
 #pragma unroll
-    for (int j = 0; j < 32; ++j)
-      if (c + j < S) mx = fmaxf(mx, __uint_as_float(r[j]));
-  }
-  const float sl2 = 1.4426950408889634f * 0.125f;   // log2(e) / sqrt(64)
-  const float mb = mx * sl2;
-  float l = 0.f;
-  uint8_t *prow = sP + row * 128;
+      for (int jj = 0; jj < 32; ++jj)
+        if (c + jj < S) m4[jj & 3] = fmaxf(m4[jj & 3], __uint_as_float(r[jj]));
+      mx = fmaxf(mx, fmaxf(fmaxf(m4[0], m4[1]), fmaxf(m4[2], m4[3])));
+    }
+    float *xmax = xch + (j & 1) * 2 * QT;                  // double-buffered exchange slots
+    float *xsum = xmax + QT;
+    if (khalf == 1) xmax[row] = mx;
+    __syncthreads();
+    if (khalf == 0) xmax[row] = mx = fmaxf(mx, xmax[row]);
+    __syncthreads();
+    if (khalf == 1) mx = xmax[row];
+    const float mb = mx * sl2;
+    float l4[4] = {0.f, 0.f, 0.f, 0.f};
+    uint8_t *prow = sP + row * 128;
 #pragma unroll 1
-  for (int c = 0; c < SKV; c += 32) {
-    uint32_t r[32];
-    tmem_ld32(t_s + lane_off + c, r);
-    tmem_wait_ld();
-    float p[32];
+    for (int c = c_begin; c < c_begin + HALF; c += 32) {
+      uint32_t r[32];
+      tmem_ld32(tbase + lane_off + c, r);
+      tmem_wait_ld();
+      float p[32];
 #pragma unroll
-    for (int j = 0; j < 32; ++j) {
-      p[j] = (c + j < S) ? exp2f(fmaf(__uint_as_float(r[j]), sl2, -mb)) : 0.f;
-      l += p[j];
-    }
-    // columns c..c+31 -> block c/64, 16-byte chunks (c%64)/8 .. +3, XOR-swizzled by row%8
-    uint8_t *blk = prow + (c / 64) * (QT * 128);
-    const int ch0 = (c % 64) / 8;
+      for (int jj = 0; jj < 32; ++jj) {
+        p[jj] = (c + jj < S) ? ex2_approx(fmaf(__uint_as_float(r[jj]), sl2, -mb)) : 0.f;
+        l4[jj & 3] += p[jj];
+      }
+      // columns c..c+31 -> block c/64, 16-byte chunks (c%64)/8 .. +3, XOR-swizzled by row%8
+      uint8_t *blk = prow + (c / 64) * (QT * 128);
+      const int ch0 = (c % 64) / 8;
 #pragma unroll
-    for (int j = 0; j < 4; ++j) {
-      uint4 o;
-      o.x = pack_bf16(p[8 * j + 0], p[8 * j + 1]);
-      o.y = pack_bf16(p[8 * j + 2], p[8 * j + 3]);
-      o.z = pack_bf16(p[8 * j + 4], p[8 * j + 5]);
-      o.w = pack_bf16(p[8 * j + 6], p[8 * j + 7]);
-      *reinterpret_cast<uint4 *>(blk + (((ch0 + j) ^ (row & 7)) << 4)) = o;
-    }
-  }
-  fence_proxy_async_smem();     // generic-proxy smem writes -> visible to the tensor core
-  tc_fence_before();
-  __syncthreads();
-
-  if (tid == 0) {
-    tc_fence_after();
-    const uint32_t idesc = idesc_bf16_f32(QT, D, 1);   // B (= V) is MN-major
-#pragma unroll
-    for (int kk = 0; kk < SKV / 16; ++kk) {
-      const uint64_t dp = smem_desc_sw128(smem_u32(sP + (kk / 4) * (QT * 128) + (kk % 4) * 32), 16, 1024);
-      const uint64_t dv = smem_desc_sw128(smem_u32(sV + kk * 16 * 128), SKV * 128, 1024);
-      tc_mma_f16(t_o, dp, dv, idesc, kk != 0);
-    }
-    tc_commit(&bars[2]);
-  }
-  __syncwarp();
-  mbar_wait(&bars[2], 0);
-  tc_fence_after();
-  const float inv_l = 1.0f / l;
-  const int q = q0 + row;
-#pragma unroll
-  for (int c = 0; c < D; c += 32) {
-    uint32_t r[32];
-    tmem_ld32(t_o + lane_off + c, r);
-    tmem_wait_ld();
-    if (q < S) {
-      uint4 *dst = reinterpret_cast<uint4 *>(ctx + ((size_t)b * S + q) * H + h * D + c);
-#pragma unroll
-      for (int j = 0; j < 4; ++j) {
+      for (int jj = 0; jj < 4; ++jj) {
         uint4 o;
-        o.x = pack_bf16(__uint_as_float(r[8 * j + 0]) * inv_l, __uint_as_float(r[8 * j + 1]) * inv_l);
-        o.y = pack_bf16(__uint_as_float(r[8 * j + 2]) * inv_l, __uint_as_float(r[8 * j + 3]) * inv_l);
-        o.z = pack_bf16(__uint_as_float(r[8 * j + 4]) * inv_l, __uint_as_float(r[8 * j + 5]) * inv_l);
-        o.w = pack_bf16(__uint_as_float(r[8 * j + 6]) * inv_l, __uint_as_float(r[8 * j + 7]) * inv_l);
-        dst[j] = o;
+        o.x = pack_bf16(p[8 * jj + 0], p[8 * jj + 1]);
+        o.y = pack_bf16(p[8 * jj + 2], p[8 * jj + 3]);
+        o.z = pack_bf16(p[8 * jj + 4], p[8 * jj + 5]);
+        o.w = pack_bf16(p[8 * jj + 6], p[8 * jj + 7]);
+        *reinterpret_cast<uint4 *>(blk + (((ch0 + jj) ^ (row & 7)) << 4)) = o;
+      }
+    }
+    const float lpart = (l4[0] + l4[1]) + (l4[2] + l4[3]);
+    if (khalf == 1) xsum[row] = lpart;
+    fence_proxy_async_smem();     // generic-proxy smem writes -> visible to the tensor core
+    tc_fence_before();            // S fully read before MMA2 overwrites it with O
+    __syncthreads();
+    const float l = (khalf == 0) ? lpart + xsum[row] : 0.f;
+    if (khalf == 0) xsum[row] = l;
+
+    if (tid == 0) {
+      tc_fence_after();
+      const uint32_t idesc = idesc_bf16_f32(QT, D, 1);   // B (= V) is MN-major
+#pragma unroll
+      for (int kk = 0; kk < SKV / 16; ++kk) {
+        const uint64_t dp = smem_desc_sw128(smem_u32(sP + (kk / 4) * (QT * 128) + (kk % 4) * 32), 16, 1024);
+        const uint64_t dv = smem_desc_sw128(smem_u32(sV + kk * 16 * 128), SKV * 128, 1024);
+        tc_mma_f16(tbase, dp, dv, idesc, kk != 0);
+      }
+      tc_commit(bar_o);
+    }
+    __syncwarp();
+    mbar_wait(bar_o, ophase);     // MMA2 done: V tile is dead -> output staging
+    ophase ^= 1;
+    tc_fence_after();
+    __syncthreads();              // xsum[row] written by the khalf-0 thread
+    const float inv_l = 1.0f / xsum[row];
+    {
+      uint32_t r[32];
+      tmem_ld32(tbase + lane_off + khalf * 32, r);        // this thread's 32 of the 64 d columns
+      tmem_wait_ld();
+      uint8_t *orow = sV + row * 128;                     // [128 q x 128 B], 128B swizzle
+#pragma unroll
+      for (int jj = 0; jj < 4; ++jj) {
+        uint4 o;
+        o.x = pack_bf16(__uint_as_float(r[8 * jj + 0]) * inv_l, __uint_as_float(r[8 * jj + 1]) * inv_l);
+        o.y = pack_bf16(__uint_as_float(r[8 * jj + 2]) * inv_l, __uint_as_float(r[8 * jj + 3]) * inv_l);
+        o.z = pack_bf16(__uint_as_float(r[8 * jj + 4]) * inv_l, __uint_as_float(r[8 * jj + 5]) * inv_l);
+        o.w = pack_bf16(__uint_as_float(r[8 * jj + 6]) * inv_l, __uint_as_float(r[8 * jj + 7]) * inv_l);
+        *reinterpret_cast<uint4 *>(orow + (((khalf * 4 + jj) ^ (row & 7)) << 4)) = o;
+      }
+    }
+    fence_proxy_async_smem();
+    tc_fence_before();            // O read before the next MMA1 overwrites TMEM
+    __syncthreads();
+    if (tid == 0) {
+      tma_store_3d(&tctx, sV, h * D, q0, b);
+      bulk_commit();
+      if (CF::kNBuf == 1 && next < n_items) {
+        bulk_wait_read<0>();
+        issue_load(next, 0);
       }
     }
   }
-  tc_fence_before();
+  if (tid == 0) bulk_wait<0>();
   __syncthreads();
   if (warp == 0) tmem_dealloc(tbase, CF::kTmemCols);
 }
 
 template <int SKV>
-e3_status launch_attn(const AttnMaps &m, void *ctx, int B, int S, int H, int heads, cudaStream_t st) {
+e3_status launch_attn(const AttnMaps &m, int B, int S, int H, int heads, cudaStream_t st) {
   auto kern = attn_tc_kernel<SKV>;
   static bool attr_done = false;
+  static int sms = 0;
   if (!attr_done) {
     E3_CUDA_TRY(cudaFuncSetAttribute(kern, cudaFuncAttributeMaxDynamicSharedMemorySize, ACfg<SKV>::kSmem));
+    int dev = 0;
+    E3_CUDA_TRY(cudaGetDevice(&dev));
+    sms = num_sms(dev);
     attr_done = true;
   }
-  dim3 grid(B * heads, (S + QT - 1) / QT);
-  kern<<<grid, 128, ACfg<SKV>::kSmem, st>>>(m.q, m.kv, reinterpret_cast<__nv_bfloat16 *>(ctx), S, H, heads);
-  count_launch();
+  const int n_items = B * heads * ((S + QT - 1) / QT);
+  const int per_sm = (SKV == 128) ? 2 : 1;
+  const int grid = n_items < per_sm * sms ? n_items : per_sm * sms;
+  kern<<<grid, kThreads, ACfg<SKV>::kSmem, st>>>(m.q, m.kv, m.ctx, S, H, heads, n_items);
   E3_CUDA_TRY(cudaGetLastError());
+  count_launch();
   return E3_OK;
 }
 
 }  // namespace
 
-e3_status attn_tmaps(AttnMaps *m, const void *qkv, int B, int S, int H) {
+e3_status attn_tmaps(AttnMaps *m, const void *qkv, const void *ctx, int B, int S, int H) {
   m->skv = S <= 128 ? 128 : 256;
   const uint64_t W3 = 3ull * H;
   e3_status s = make_tmap_3d(&m->q, qkv, W3, (uint64_t)S, (uint64_t)B, W3, W3 * S, D, QT, 1);
-  if (s != E3_OK) return s;
-  return make_tmap_3d(&m->kv, qkv, W3, (uint64_t)S, (uint64_t)B, W3, W3 * S, D, (uint32_t)m->skv, 1);
+  if (s == E3_OK) s = make_tmap_3d(&m->kv, qkv, W3, (uint64_t)S, (uint64_t)B, W3, W3 * S, D, (uint32_t)m->skv, 1);
+  if (s == E3_OK)
+    s = make_tmap_3d(&m->ctx, ctx, (uint64_t)H, (uint64_t)S, (uint64_t)B, (uint64_t)H, (uint64_t)H * S, D, QT, 1);
+  return s;
 }
 
-e3_status attn_run(const AttnMaps &m, void *ctx, int B, int S, int H, int heads, cudaStream_t st) {
-  if (m.skv == 128) return launch_attn<128>(m, ctx, B, S, H, heads, st);
-  return launch_attn<256>(m, ctx, B, S, H, heads, st);
+e3_status attn_run(const AttnMaps &m, int B, int S, int H, int heads, cudaStream_t st) {
+  if (m.skv == 128) return launch_attn<128>(m, B, S, H, heads, st);
+  return launch_attn<256>(m, B, S, H, heads, st);
 }
 
 }  // namespace e3

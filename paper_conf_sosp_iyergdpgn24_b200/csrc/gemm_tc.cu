@@ -2,18 +2,29 @@
 // cores: C[M,N] = epi(A[M,K] . W[N,K]^T), bf16 operands, fp32 accumulation in
 // TMEM, one rounding to bf16 in the epilogue.
 //
-// Design:
-//   * persistent grid (<= #SMs CTAs), static round-robin over 128 x BN tiles,
-//     n-fastest so concurrently running CTAs share the A tile through L2;
-//   * warp 0 = TMA producer (128B-swizzled 128x64 A and BNx64 W boxes into a
-//     STAGES-deep smem ring guarded by full/empty mbarriers);
-//   * warp 1 = MMA issuer: one thread issues tcgen05.mma.cta_group::1.kind::f16
-//     128xBNx16 per 16-wide K step, tcgen05.commit frees the smem stage;
-//   * two TMEM accumulators (2*BN columns) so the epilogue of tile i overlaps
-//     the MMAs of tile i+1;
-//   * warps 4..11 = epilogue: tcgen05.ld 32x32b.x32 -> +bias (+GELU | +residual)
-//     -> bf16 -> 16-byte global stores; each warp owns its TMEM lane quarter
-//     (warp % 4) and one half of the BN columns.
+// Design (DESIGN.md §6 K1): CTA PAIRS (cluster of 2, cta_group::2).
+//   * A pair owns a 256 x BN output tile (BN in {64,128,192,256}); CTA r of the
+//     pair loads A rows [m0 + 128r, +128) and W rows [n0 + r*BN/2, +BN/2) per
+//     64-wide K block by TMA (128-byte swizzle) into its own smem ring; the
+//     completion bytes of both CTAs land on the LEADER's full barrier.  Per CTA
+//     that is (128 + BN/2) x 128 B of smem fill per 128 x BN x 64 of MMA work,
+//     twice the arithmetic intensity of a 1-SM 128 x BN tile (the L2 -> SM
+//     fill rate, ~15 TB/s measured, otherwise caps the tensor pipe).
+//   * the leader's single MMA thread issues tcgen05.mma.cta_group::2.kind::f16
+//     256 x BN x 16; the hardware reads the A/W halves from both CTAs and
+//     writes rows 0-127 of D to the leader's TMEM, rows 128-255 to the peer's;
+//     tcgen05.commit multicasts "stage free" / "accumulator full" to both CTAs.
+//   * persistent: pairs walk the tiles round-robin, n-fastest; two TMEM
+//     accumulators (2*BN columns) so the epilogue of tile i overlaps the MMAs of
+//     tile i+1; both CTAs' epilogue warps arrive on the leader's "accumulator
+//     empty" barrier (remote mbarrier arrive through mapa).
+//   * 8 epilogue warps per CTA; warp w owns TMEM lane quarter w % 4 (32 rows)
+//     and one half of the BN columns, in chunks of 32 columns:
+//     tcgen05.ld 32x32b.x32 -> +bias (+GELU | +residual, prefetched one chunk
+//     ahead) -> bf16 -> 64-byte-swizzled smem staging (double buffered) ->
+//     one TMA store of the 32 x 32 box.  Coalesced full-line writes instead of
+//     32 scattered 16-byte stores per instruction (r01 measurement: the
+//     scattered stores cost 8-25 us per GEMM launch).
 #include "common.cuh"
 #include "kernels.h"
 #include "prof.h"
@@ -22,32 +33,45 @@ namespace e3 {
 
 namespace {
 
-constexpr int BM = 128;
-constexpr int BK = 64;
-constexpr int kThreads = 384;   // 4 control warps + 8 epilogue warps
+constexpr int BM = 128;           // rows per CTA (256 per pair)
+constexpr int BK = 64;            // K width of one 128-byte swizzle atom (TMA box)
+constexpr int KSUB = 2;           // swizzle atoms per pipeline stage: 128-wide K stages
+                                  // halve the per-MMA barrier / commit overhead
+constexpr int kThreads = 384;     // 4 control warps + 8 epilogue warps
+constexpr int kEpiWarps = 8;
+constexpr int kEpiBuf = 32 * 64;  // one 32 x 32 bf16 box
+constexpr int kEpiBytes = kEpiWarps * 2 * kEpiBuf;
+constexpr int kSmemMax = 232448;  // 227 KB opt-in limit
 
 template <int BN>
 struct Cfg {
-  static constexpr int kABytes = BM * BK * 2;
-  static constexpr int kBBytes = BN * BK * 2;
+  static constexpr int kASub = BM * BK * 2;            // 16 KB per swizzle atom column
+  static constexpr int kBSub = (BN / 2) * BK * 2;      // this CTA's half of the W tile
+  static constexpr int kABytes = KSUB * kASub;
+  static constexpr int kBBytes = KSUB * kBSub;
   static constexpr int kStageBytes = kABytes + kBBytes;
-  static constexpr int kStages = (192 * 1024) / kStageBytes;
-  static constexpr int kTmemCols = 2 * BN;   // 128 / 256 / 512: powers of two
-  static constexpr int kSmem = kStages * kStageBytes + 1024 /*align*/ + 256 /*barriers*/;
+  static constexpr int kStages = (kSmemMax - kEpiBytes - 1024 - 256) / kStageBytes;
+  static constexpr int kTmemCols = (2 * BN <= 128) ? 128 : (2 * BN <= 256) ? 256 : 512;
+  static constexpr int kSmem = kStages * kStageBytes + kEpiBytes + 1024 /*align*/ + 256 /*barriers*/;
 };
 
+// 64-byte swizzle of a [32 rows x 64 B] box: 16-byte chunk j of row r
+__device__ __forceinline__ uint32_t sw64(int r, int j) { return r * 64 + ((j ^ ((r >> 1) & 3)) << 4); }
+
 template <int BN, int EPI>
-__global__ void __launch_bounds__(kThreads, 1)
+__global__ void __cluster_dims__(2, 1, 1) __launch_bounds__(kThreads, 1)
     gemm_bf16_tc_kernel(const __grid_constant__ CUtensorMap tmA, const __grid_constant__ CUtensorMap tmB,
-                        __nv_bfloat16 *__restrict__ C, const __nv_bfloat16 *__restrict__ bias,
+                        const __grid_constant__ CUtensorMap tmC, const __nv_bfloat16 *__restrict__ bias,
                         const __nv_bfloat16 *__restrict__ R, int M, int N, int K) {
   using CF = Cfg<BN>;
   constexpr int S = CF::kStages;
   extern __shared__ uint8_t smem_raw[];
+  // identical layout (same offsets) in both CTAs of the pair
   uint8_t *smem = reinterpret_cast<uint8_t *>((reinterpret_cast<uintptr_t>(smem_raw) + 1023) & ~uintptr_t(1023));
-  uint8_t *sA = smem;                                   // S x 16 KB
-  uint8_t *sB = smem + S * CF::kABytes;                 // S x BN*128 B
-  uint64_t *full = reinterpret_cast<uint64_t *>(smem + S * CF::kStageBytes);
+  uint8_t *sA = smem;
+  uint8_t *sB = smem + S * CF::kABytes;
+  uint8_t *sE = smem + S * CF::kStageBytes;              // epilogue staging (1024-aligned)
+  uint64_t *full = reinterpret_cast<uint64_t *>(sE + kEpiBytes);
   uint64_t *empty = full + S;
   uint64_t *tfull = empty + S;        // [2]
   uint64_t *tempty = tfull + 2;       // [2]
@@ -55,175 +79,217 @@ __global__ void __launch_bounds__(kThreads, 1)
 
   const int warp = warp_id();
   const int lane = lane_id();
-  const int num_m = (M + BM - 1) / BM;
+  const uint32_t rank = cluster_ctarank();
+  const bool leader = rank == 0;
+  const int pair = blockIdx.x >> 1;
+  const int num_pairs = gridDim.x >> 1;
+  const int num_m = (M + 2 * BM - 1) / (2 * BM);
   const int num_n = N / BN;
   const int num_tiles = num_m * num_n;
-  const int num_kb = K / BK;
+  const int num_kb = K / (BK * KSUB);
 
   if (warp == 0 && lane == 0) {
     tma_prefetch(&tmA);
     tma_prefetch(&tmB);
+    tma_prefetch(&tmC);
   }
   if (warp == 1 && lane == 0) {
     for (int i = 0; i < S; ++i) {
-      mbar_init(&full[i], 1);
-      mbar_init(&empty[i], 1);
+      mbar_init(&full[i], 1);      // leader's arrive.expect_tx (bytes of both CTAs)
+      mbar_init(&empty[i], 1);     // multicast tcgen05.commit
     }
     for (int i = 0; i < 2; ++i) {
-      mbar_init(&tfull[i], 1);
-      mbar_init(&tempty[i], 8);   // one arrive per epilogue warp
+      mbar_init(&tfull[i], 1);     // multicast tcgen05.commit
+      mbar_init(&tempty[i], 16);   // 8 epilogue warps x 2 CTAs (leader's copy is used)
     }
     fence_barrier_init();
   }
-  if (warp == 2) tmem_alloc(tmem_base_slot, CF::kTmemCols);
+  if (warp == 2) tmem_alloc2(tmem_base_slot, CF::kTmemCols);
   tc_fence_before();
-  __syncthreads();
+  cluster_sync();                  // peer barriers initialised, TMEM allocated in both CTAs
   tc_fence_after();
   const uint32_t tmem_base = *tmem_base_slot;
 
   if (warp == 0) {
-    // ------------------------------------------------ TMA producer
+    // ------------------------------------------------ TMA producer (both CTAs)
     if (lane == 0) {
       int stage = 0;
       uint32_t phase = 0;
-      for (int t = blockIdx.x; t < num_tiles; t += gridDim.x) {
+      for (int t = pair; t < num_tiles; t += num_pairs) {
         const int m_blk = t / num_n, n_blk = t % num_n;
+        const int am = m_blk * 2 * BM + (int)rank * BM;
+        const int bn = n_blk * BN + (int)rank * (BN / 2);
         for (int kb = 0; kb < num_kb; ++kb) {
           mbar_wait(&empty[stage], phase ^ 1);
-          mbar_expect_tx(&full[stage], CF::kStageBytes);
-          tma_load_2d(sA + stage * CF::kABytes, &tmA, &full[stage], kb * BK, m_blk * BM);
-          tma_load_2d(sB + stage * CF::kBBytes, &tmB, &full[stage], kb * BK, n_blk * BN);
+          const uint32_t fb = mapa_shared(smem_u32(&full[stage]), 0);
+          if (leader) mbar_expect_tx(&full[stage], 2 * CF::kStageBytes);
+#pragma unroll
+          for (int ks = 0; ks < KSUB; ++ks) {
+            const int k0 = (kb * KSUB + ks) * BK;
+            tma_load_2d_2sm(sA + stage * CF::kABytes + ks * CF::kASub, &tmA, fb, k0, am);
+            tma_load_2d_2sm(sB + stage * CF::kBBytes + ks * CF::kBSub, &tmB, fb, k0, bn);
+          }
           if (++stage == S) { stage = 0; phase ^= 1; }
         }
       }
     }
   } else if (warp == 1) {
-    // ------------------------------------------------ MMA issuer
-    constexpr uint32_t idesc = idesc_bf16_f32(BM, BN, 0);
-    int stage = 0;
-    uint32_t phase = 0;
-    int acc = 0;
-    uint32_t acc_phase = 0;
-    for (int t = blockIdx.x; t < num_tiles; t += gridDim.x) {
-      mbar_wait(&tempty[acc], acc_phase ^ 1);
-      tc_fence_after();
-      const uint32_t d_tmem = tmem_base + acc * BN;
-      for (int kb = 0; kb < num_kb; ++kb) {
-        mbar_wait(&full[stage], phase);
+    // ------------------------------------------------ MMA issuer (leader, one thread)
+    if (leader && lane == 0) {
+      constexpr uint32_t idesc = idesc_bf16_f32(2 * BM, BN, 0);
+      int stage = 0;
+      uint32_t phase = 0;
+      int acc = 0;
+      uint32_t acc_phase = 0;
+      for (int t = pair; t < num_tiles; t += num_pairs) {
+        mbar_wait(&tempty[acc], acc_phase ^ 1);
         tc_fence_after();
-        if (lane == 0) {
-          const uint64_t da = smem_desc_sw128(smem_u32(sA + stage * CF::kABytes), 16, 1024);
-          const uint64_t db = smem_desc_sw128(smem_u32(sB + stage * CF::kBBytes), 16, 1024);
+        const uint32_t d_tmem = tmem_base + acc * BN;
+        for (int kb = 0; kb < num_kb; ++kb) {
+          mbar_wait(&full[stage], phase);
+          tc_fence_after();
 #pragma unroll
-          for (int k = 0; k < BK / 16; ++k) {
-            // +32 bytes per 16-element K step inside the 128-byte swizzle atom
-            tc_mma_f16(d_tmem, da + (uint64_t)(2 * k), db + (uint64_t)(2 * k), idesc, (kb | k) != 0);
+          for (int ks = 0; ks < KSUB; ++ks) {
+            const uint64_t da = smem_desc_sw128(smem_u32(sA + stage * CF::kABytes + ks * CF::kASub), 16, 1024);
+            const uint64_t db = smem_desc_sw128(smem_u32(sB + stage * CF::kBBytes + ks * CF::kBSub), 16, 1024);
+#pragma unroll
+            for (int k = 0; k < BK / 16; ++k)   // +32 bytes per 16-element K step inside the swizzle atom
+              tc_mma2_f16(d_tmem, da + (uint64_t)(2 * k), db + (uint64_t)(2 * k), idesc, (kb | ks | k) != 0);
           }
-          tc_commit(&empty[stage]);
+          tc_commit2_mc(&empty[stage], 0x3);
+          if (++stage == S) { stage = 0; phase ^= 1; }
         }
-        __syncwarp();
-        if (++stage == S) { stage = 0; phase ^= 1; }
+        tc_commit2_mc(&tfull[acc], 0x3);
+        if (++acc == 2) { acc = 0; acc_phase ^= 1; }
       }
-      if (lane == 0) tc_commit(&tfull[acc]);
-      __syncwarp();
-      if (++acc == 2) { acc = 0; acc_phase ^= 1; }
     }
   } else if (warp >= 4) {
-    // ------------------------------------------------ epilogue
+    // ------------------------------------------------ epilogue (both CTAs)
     const int q = warp & 3;              // TMEM lane quarter this warp may access
     const int half = (warp - 4) >> 2;    // which half of the BN columns
-    const int row = q * 32 + lane;
+    uint8_t *ebuf = sE + (warp - 4) * 2 * kEpiBuf;
+    const uint32_t tempty_leader0 = mapa_shared(smem_u32(&tempty[0]), 0);
+    const uint32_t tempty_leader1 = mapa_shared(smem_u32(&tempty[1]), 0);
     int acc = 0;
     uint32_t acc_phase = 0;
-    for (int t = blockIdx.x; t < num_tiles; t += gridDim.x) {
+    int ci = 0;                          // chunk counter (selects the staging buffer)
+    for (int t = pair; t < num_tiles; t += num_pairs) {
       const int m_blk = t / num_n, n_blk = t % num_n;
+      const int m0 = m_blk * 2 * BM + (int)rank * BM + q * 32;   // this warp's first row
+      const int m = m0 + lane;
+      const uint32_t taddr = tmem_base + ((uint32_t)(q * 32) << 16) + acc * BN;
+      constexpr int kChunks = BN / 64;   // 32-column chunks per warp
+      uint4 rnext[4];
+      if (EPI == E3_EPI_BIAS_RESID) {
+        const uint4 *rp = reinterpret_cast<const uint4 *>(R + (size_t)m * N + n_blk * BN + half * (BN / 2));
+#pragma unroll
+        for (int j = 0; j < 4; ++j) rnext[j] = (m < M) ? __ldg(rp + j) : make_uint4(0, 0, 0, 0);
+      }
       mbar_wait(&tfull[acc], acc_phase);
       tc_fence_after();
-      const int m = m_blk * BM + row;
-      const uint32_t taddr = tmem_base + ((uint32_t)(q * 32) << 16) + acc * BN;
 #pragma unroll 1
-      for (int c = half * (BN / 2); c < (half + 1) * (BN / 2); c += 32) {
+      for (int c = 0; c < kChunks; ++c) {
+        const int col = half * (BN / 2) + c * 32;
+        const int n0 = n_blk * BN + col;
         uint32_t r[32];
-        tmem_ld32(taddr + c, r);
+        tmem_ld32(taddr + col, r);
+        uint4 rcur[4];
+        if (EPI == E3_EPI_BIAS_RESID) {
+#pragma unroll
+          for (int j = 0; j < 4; ++j) rcur[j] = rnext[j];
+          if (c + 1 < kChunks) {          // prefetch the next chunk's residual
+            const uint4 *rp = reinterpret_cast<const uint4 *>(R + (size_t)m * N + n0 + 32);
+#pragma unroll
+            for (int j = 0; j < 4; ++j) rnext[j] = (m < M) ? __ldg(rp + j) : make_uint4(0, 0, 0, 0);
+          }
+        }
         tmem_wait_ld();
-        const int n0 = n_blk * BN + c;
         float v[32];
         const uint4 *bp = reinterpret_cast<const uint4 *>(bias + n0);
 #pragma unroll
         for (int j = 0; j < 4; ++j) {
-          uint4 b4 = __ldg(bp + j);
-          uint32_t bw[4] = {b4.x, b4.y, b4.z, b4.w};
+          const uint4 b4 = __ldg(bp + j);
+          const uint32_t bw[4] = {b4.x, b4.y, b4.z, b4.w};
 #pragma unroll
           for (int e = 0; e < 4; ++e) {
             v[j * 8 + 2 * e] = __uint_as_float(r[j * 8 + 2 * e]) + bf_lo(bw[e]);
             v[j * 8 + 2 * e + 1] = __uint_as_float(r[j * 8 + 2 * e + 1]) + bf_hi(bw[e]);
           }
         }
-        if (m < M) {
-          if (EPI == E3_EPI_BIAS_GELU) {
+        if (EPI == E3_EPI_BIAS_GELU) {
 #pragma unroll
-            for (int j = 0; j < 32; ++j) v[j] = gelu_erf(v[j]);
-          }
-          if (EPI == E3_EPI_BIAS_RESID) {
-            const uint4 *rp = reinterpret_cast<const uint4 *>(R + (size_t)m * N + n0);
-#pragma unroll
-            for (int j = 0; j < 4; ++j) {
-              uint4 r4 = rp[j];
-              uint32_t rw[4] = {r4.x, r4.y, r4.z, r4.w};
-#pragma unroll
-              for (int e = 0; e < 4; ++e) {
-                v[j * 8 + 2 * e] += bf_lo(rw[e]);
-                v[j * 8 + 2 * e + 1] += bf_hi(rw[e]);
-              }
-            }
-          }
-          uint4 *cp = reinterpret_cast<uint4 *>(C + (size_t)m * N + n0);
+          for (int j = 0; j < 32; ++j) v[j] = gelu_fast(v[j]);
+        }
+        if (EPI == E3_EPI_BIAS_RESID) {
 #pragma unroll
           for (int j = 0; j < 4; ++j) {
-            uint4 o;
-            o.x = pack_bf16(v[j * 8 + 0], v[j * 8 + 1]);
-            o.y = pack_bf16(v[j * 8 + 2], v[j * 8 + 3]);
-            o.z = pack_bf16(v[j * 8 + 4], v[j * 8 + 5]);
-            o.w = pack_bf16(v[j * 8 + 6], v[j * 8 + 7]);
-            cp[j] = o;
+            const uint32_t rw[4] = {rcur[j].x, rcur[j].y, rcur[j].z, rcur[j].w};
+#pragma unroll
+            for (int e = 0; e < 4; ++e) {
+              v[j * 8 + 2 * e] += bf_lo(rw[e]);
+              v[j * 8 + 2 * e + 1] += bf_hi(rw[e]);
+            }
           }
         }
+        // stage: buffer (ci & 1) was last used by chunk ci-2; its TMA store must
+        // have finished reading smem
+        uint8_t *buf = ebuf + (ci & 1) * kEpiBuf;
+        if (lane == 0) bulk_wait_read<1>();
+        __syncwarp();
+#pragma unroll
+        for (int j = 0; j < 4; ++j) {
+          uint4 o;
+          o.x = pack_bf16(v[j * 8 + 0], v[j * 8 + 1]);
+          o.y = pack_bf16(v[j * 8 + 2], v[j * 8 + 3]);
+          o.z = pack_bf16(v[j * 8 + 4], v[j * 8 + 5]);
+          o.w = pack_bf16(v[j * 8 + 6], v[j * 8 + 7]);
+          *reinterpret_cast<uint4 *>(buf + sw64(lane, j)) = o;
+        }
+        fence_proxy_async_smem();
+        __syncwarp();
+        if (lane == 0) {
+          tma_store_2d(&tmC, buf, n0, m0);   // rows >= M are clipped by the tensor map
+          bulk_commit();
+        }
+        ++ci;
       }
       tc_fence_before();
       __syncwarp();
-      if (lane == 0) mbar_arrive(&tempty[acc]);
+      if (lane == 0) mbar_arrive_cluster(acc ? tempty_leader1 : tempty_leader0);
       if (++acc == 2) { acc = 0; acc_phase ^= 1; }
     }
+    if (lane == 0) bulk_wait<0>();
   }
-  __syncthreads();
-  if (warp == 2) tmem_dealloc(tmem_base, CF::kTmemCols);
+  tc_fence_before();
+  cluster_sync();                  // no CTA leaves while its peer may still signal it
+  tc_fence_after();
+  if (warp == 2) tmem_dealloc2(tmem_base, CF::kTmemCols);
 }
 
 template <int BN, int EPI>
-e3_status launch(const CUtensorMap &ta, const CUtensorMap &tb, __nv_bfloat16 *C, const __nv_bfloat16 *bias,
-                 const __nv_bfloat16 *R, int M, int N, int K, int sms, cudaStream_t st) {
+e3_status launch(const GemmMaps &g, const __nv_bfloat16 *bias, const __nv_bfloat16 *R, int M, int N, int K, int sms,
+                 cudaStream_t st) {
   auto kern = gemm_bf16_tc_kernel<BN, EPI>;
   static bool attr_done = false;   // per instantiation
   if (!attr_done) {
     E3_CUDA_TRY(cudaFuncSetAttribute(kern, cudaFuncAttributeMaxDynamicSharedMemorySize, Cfg<BN>::kSmem));
     attr_done = true;
   }
-  const int tiles = ((M + BM - 1) / BM) * (N / BN);
-  const int grid = tiles < sms ? tiles : sms;
-  kern<<<grid, kThreads, Cfg<BN>::kSmem, st>>>(ta, tb, C, bias, R, M, N, K);
-  count_launch();
+  const int tiles = ((M + 2 * BM - 1) / (2 * BM)) * (N / BN);
+  const int pairs = tiles < sms / 2 ? tiles : sms / 2;
+  kern<<<2 * pairs, kThreads, Cfg<BN>::kSmem, st>>>(g.a, g.b, g.c, bias, R, M, N, K);
   E3_CUDA_TRY(cudaGetLastError());
+  count_launch();
   return E3_OK;
 }
 
 template <int BN>
-e3_status launch_epi(int epi, const CUtensorMap &ta, const CUtensorMap &tb, __nv_bfloat16 *C,
-                     const __nv_bfloat16 *bias, const __nv_bfloat16 *R, int M, int N, int K, int sms,
-                     cudaStream_t st) {
+e3_status launch_epi(int epi, const GemmMaps &g, const __nv_bfloat16 *bias, const __nv_bfloat16 *R, int M, int N,
+                     int K, int sms, cudaStream_t st) {
   switch (epi) {
-    case E3_EPI_BIAS: return launch<BN, E3_EPI_BIAS>(ta, tb, C, bias, R, M, N, K, sms, st);
-    case E3_EPI_BIAS_GELU: return launch<BN, E3_EPI_BIAS_GELU>(ta, tb, C, bias, R, M, N, K, sms, st);
-    case E3_EPI_BIAS_RESID: return launch<BN, E3_EPI_BIAS_RESID>(ta, tb, C, bias, R, M, N, K, sms, st);
+    case E3_EPI_BIAS: return launch<BN, E3_EPI_BIAS>(g, bias, R, M, N, K, sms, st);
+    case E3_EPI_BIAS_GELU: return launch<BN, E3_EPI_BIAS_GELU>(g, bias, R, M, N, K, sms, st);
+    case E3_EPI_BIAS_RESID: return launch<BN, E3_EPI_BIAS_RESID>(g, bias, R, M, N, K, sms, st);
   }
   set_error("bad epilogue");
   return E3_EINVAL;
@@ -232,39 +298,41 @@ e3_status launch_epi(int epi, const CUtensorMap &ta, const CUtensorMap &tb, __nv
 }  // namespace
 
 int gemm_pick_bn(int M, int N, int sms) {
-  // Minimise (waves x per-tile cost), per-tile cost ~ BN + 16 (fixed
-  // prologue / epilogue overhead in column units).
+  // Minimise waves x per-tile cost over the pair tiles (256 x BN); per-tile
+  // cost ~ BN + 32 (fixed prologue / epilogue overhead in column units).
   int best = 0;
   long best_cost = 0;
-  const int cands[3] = {256, 128, 64};
-  for (int i = 0; i < 3; ++i) {
+  const int cands[4] = {256, 192, 128, 64};
+  const int pairs = sms / 2;
+  for (int i = 0; i < 4; ++i) {
     const int bn = cands[i];
     if (N % bn) continue;
-    const long tiles = (long)((M + BM - 1) / BM) * (N / bn);
-    const long waves = (tiles + sms - 1) / sms;
-    const long cost = waves * (bn + 16);
+    const long tiles = (long)((M + 2 * BM - 1) / (2 * BM)) * (N / bn);
+    const long waves = (tiles + pairs - 1) / pairs;
+    const long cost = waves * (bn + 32);
     if (best == 0 || cost < best_cost) { best = bn; best_cost = cost; }
   }
   return best;
 }
 
-e3_status gemm_tmaps(GemmMaps *g, const void *A, int64_t lda, const void *W, int M, int N, int K, int bn) {
+e3_status gemm_tmaps(GemmMaps *g, const void *A, int64_t lda, const void *W, const void *C, int M, int N, int K,
+                     int bn) {
   e3_status s = make_tmap_2d(&g->a, A, (uint64_t)M, (uint64_t)K, (uint64_t)lda, BM, BK);
-  if (s != E3_OK) return s;
-  s = make_tmap_2d(&g->b, W, (uint64_t)N, (uint64_t)K, (uint64_t)K, (uint32_t)bn, BK);
+  if (s == E3_OK) s = make_tmap_2d(&g->b, W, (uint64_t)N, (uint64_t)K, (uint64_t)K, (uint32_t)(bn / 2), BK);
+  if (s == E3_OK) s = make_tmap_2d_sw64(&g->c, C, (uint64_t)M, (uint64_t)N, (uint64_t)N, 32, 32);
   g->bn = bn;
   return s;
 }
 
-e3_status gemm_run(const GemmMaps &g, void *C, const void *bias, const void *R, int M, int N, int K, int epi,
-                   int sms, cudaStream_t st) {
-  auto *c = reinterpret_cast<__nv_bfloat16 *>(C);
+e3_status gemm_run(const GemmMaps &g, const void *bias, const void *R, int M, int N, int K, int epi, int sms,
+                   cudaStream_t st) {
   auto *b = reinterpret_cast<const __nv_bfloat16 *>(bias);
   auto *r = reinterpret_cast<const __nv_bfloat16 *>(R);
   switch (g.bn) {
-    case 256: return launch_epi<256>(epi, g.a, g.b, c, b, r, M, N, K, sms, st);
-    case 128: return launch_epi<128>(epi, g.a, g.b, c, b, r, M, N, K, sms, st);
-    case 64: return launch_epi<64>(epi, g.a, g.b, c, b, r, M, N, K, sms, st);
+    case 256: return launch_epi<256>(epi, g, b, r, M, N, K, sms, st);
+    case 192: return launch_epi<192>(epi, g, b, r, M, N, K, sms, st);
+    case 128: return launch_epi<128>(epi, g, b, r, M, N, K, sms, st);
+    case 64: return launch_epi<64>(epi, g, b, r, M, N, K, sms, st);
   }
   set_error("unsupported GEMM N tile");
   return E3_EUNSUPPORTED;

@@ -12,23 +12,26 @@ namespace e3 {
 
 // ---- K1 layer GEMM (gemm_tc.cu)
 struct GemmMaps {
-  CUtensorMap a;
-  CUtensorMap b;
+  CUtensorMap a;   // A [M,K], box 128 x 64, 128-B swizzle
+  CUtensorMap b;   // W [N,K], box BN/2 x 64, 128-B swizzle
+  CUtensorMap c;   // C [M,N], box 32 x 32, 64-B swizzle (epilogue TMA store)
   int bn;
 };
 int gemm_pick_bn(int M, int N, int sms);
-e3_status gemm_tmaps(GemmMaps *g, const void *A, int64_t lda, const void *W, int M, int N, int K, int bn);
-e3_status gemm_run(const GemmMaps &g, void *C, const void *bias, const void *R, int M, int N, int K, int epi,
-                   int sms, cudaStream_t st);
+e3_status gemm_tmaps(GemmMaps *g, const void *A, int64_t lda, const void *W, const void *C, int M, int N, int K,
+                     int bn);
+e3_status gemm_run(const GemmMaps &g, const void *bias, const void *R, int M, int N, int K, int epi, int sms,
+                   cudaStream_t st);
 
 // ---- K2 attention (attn_tc.cu)
 struct AttnMaps {
-  CUtensorMap q;    // box 64 x 128 x 1
-  CUtensorMap kv;   // box 64 x SKV x 1
+  CUtensorMap q;    // qkv [B][S][3H], box 64 x 128 x 1
+  CUtensorMap kv;   // qkv [B][S][3H], box 64 x SKV x 1
+  CUtensorMap ctx;  // ctx [B][S][H],  box 64 x 128 x 1 (TMA store)
   int skv;
 };
-e3_status attn_tmaps(AttnMaps *m, const void *qkv, int B, int S, int H);
-e3_status attn_run(const AttnMaps &m, void *ctx, int B, int S, int H, int heads, cudaStream_t st);
+e3_status attn_tmaps(AttnMaps *m, const void *qkv, const void *ctx, int B, int S, int H);
+e3_status attn_run(const AttnMaps &m, int B, int S, int H, int heads, cudaStream_t st);
 
 // ---- K3 LayerNorm (layernorm.cu)
 e3_status layernorm_run(const void *x, const void *g, const void *b, void *y, int rows, int H, float eps,

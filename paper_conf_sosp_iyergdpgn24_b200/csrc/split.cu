@@ -71,9 +71,9 @@ e3_status split_validate(const e3_split_desc *d, const e3_weights *w) {
     return E3_EUNSUPPORTED;
   }
   E3_CHECK_ARG(d->hidden > 0 && d->heads > 0 && d->ffn > 0 && d->seq_len > 0 && d->batch > 0, "non-positive dims");
-  if (d->hidden % 64 || d->hidden / d->heads != 64 || d->hidden % d->heads || d->ffn % 64 || d->seq_len > 256 ||
+  if (d->hidden % 128 || d->hidden / d->heads != 64 || d->hidden % d->heads || d->ffn % 128 || d->seq_len > 256 ||
       d->batch > 4096 || d->num_labels < 1 || d->num_labels > 16 || d->hidden > 4096) {
-    set_error("e3_split_create: unsupported shape (need H % 64 == 0, head_dim 64, F % 64 == 0, S <= 256, "
+    set_error("e3_split_create: unsupported shape (need H % 128 == 0, head_dim 64, F % 128 == 0, S <= 256, "
               "B <= 4096, 1 <= C <= 16, H <= 4096)");
     return E3_EUNSUPPORTED;
   }
@@ -151,12 +151,12 @@ e3_status split_create_shared(const e3_split_desc *d, const e3_weights *w, int d
   for (int i = 0; i < nl && st == E3_OK; ++i) {
     auto &m = s->maps[i];
     const void *prev = (i % 2 == 1) ? ws->xa : ws->xb;   // output of layer i-1
-    if (i > 0) st = gemm_tmaps(&m.qkv, prev, H, s->L[i].w_qkv, M, 3 * H, H, s->bn_qkv);
-    if (st == E3_OK) st = gemm_tmaps(&m.o, ws->ctx, H, s->L[i].w_o, M, H, H, s->bn_o);
-    if (st == E3_OK) st = gemm_tmaps(&m.f1, ws->x1, H, s->L[i].w_1, M, F, H, s->bn_f1);
-    if (st == E3_OK) st = gemm_tmaps(&m.f2, ws->h, F, s->L[i].w_2, M, H, F, s->bn_f2);
+    if (i > 0) st = gemm_tmaps(&m.qkv, prev, H, s->L[i].w_qkv, ws->qkv, M, 3 * H, H, s->bn_qkv);
+    if (st == E3_OK) st = gemm_tmaps(&m.o, ws->ctx, H, s->L[i].w_o, ws->y, M, H, H, s->bn_o);
+    if (st == E3_OK) st = gemm_tmaps(&m.f1, ws->x1, H, s->L[i].w_1, ws->h, M, F, H, s->bn_f1);
+    if (st == E3_OK) st = gemm_tmaps(&m.f2, ws->h, F, s->L[i].w_2, ws->y, M, H, F, s->bn_f2);
   }
-  if (st == E3_OK) st = attn_tmaps(&s->attn, ws->qkv, B, S, H);
+  if (st == E3_OK) st = attn_tmaps(&s->attn, ws->qkv, ws->ctx, B, S, H);
   if (st != E3_OK) {
     delete s;
     return st;
@@ -196,19 +196,19 @@ e3_status split_run_to(e3_split *s, cudaStream_t st, const void *x_in, const int
       ProfScope ps(PK_GEMM_QKV, st, f_qkv, 0);
       if (i == 0) {
         GemmMaps g0;
-        E3_RUN(gemm_tmaps(&g0, cur, H, L.w_qkv, M, 3 * H, H, s->bn_qkv));
-        E3_RUN(gemm_run(g0, ws.qkv, L.b_qkv, nullptr, M, 3 * H, H, E3_EPI_BIAS, s->sms, st));
+        E3_RUN(gemm_tmaps(&g0, cur, H, L.w_qkv, ws.qkv, M, 3 * H, H, s->bn_qkv));
+        E3_RUN(gemm_run(g0, L.b_qkv, nullptr, M, 3 * H, H, E3_EPI_BIAS, s->sms, st));
       } else {
-        E3_RUN(gemm_run(m.qkv, ws.qkv, L.b_qkv, nullptr, M, 3 * H, H, E3_EPI_BIAS, s->sms, st));
+        E3_RUN(gemm_run(m.qkv, L.b_qkv, nullptr, M, 3 * H, H, E3_EPI_BIAS, s->sms, st));
       }
     }
     {
       ProfScope ps(PK_ATTN, st, f_att, 0);
-      E3_RUN(attn_run(s->attn, ws.ctx, B, S, H, d.heads, st));
+      E3_RUN(attn_run(s->attn, B, S, H, d.heads, st));
     }
     {
       ProfScope ps(PK_GEMM_O, st, f_o, 0);
-      E3_RUN(gemm_run(m.o, ws.y, L.b_o, cur, M, H, H, E3_EPI_BIAS_RESID, s->sms, st));
+      E3_RUN(gemm_run(m.o, L.b_o, cur, M, H, H, E3_EPI_BIAS_RESID, s->sms, st));
     }
     {
       ProfScope ps(PK_LN, st, 0, b_ln);
@@ -216,11 +216,11 @@ e3_status split_run_to(e3_split *s, cudaStream_t st, const void *x_in, const int
     }
     {
       ProfScope ps(PK_GEMM_FFN1, st, f_1, 0);
-      E3_RUN(gemm_run(m.f1, ws.h, L.b_1, nullptr, M, F, H, E3_EPI_BIAS_GELU, s->sms, st));
+      E3_RUN(gemm_run(m.f1, L.b_1, nullptr, M, F, H, E3_EPI_BIAS_GELU, s->sms, st));
     }
     {
       ProfScope ps(PK_GEMM_FFN2, st, f_1, 0);
-      E3_RUN(gemm_run(m.f2, ws.y, L.b_2, ws.x1, M, H, F, E3_EPI_BIAS_RESID, s->sms, st));
+      E3_RUN(gemm_run(m.f2, L.b_2, ws.x1, M, H, F, E3_EPI_BIAS_RESID, s->sms, st));
     }
     {
       ProfScope ps(PK_LN, st, 0, b_ln);
@@ -319,17 +319,17 @@ e3_status e3_op_gemm(void *stream, const void *A, int64_t lda, const void *W, co
   E3_CHECK_ARG(epilogue >= 0 && epilogue <= 2, "bad epilogue");
   E3_CHECK_ARG(epilogue != E3_EPI_BIAS_RESID || resid, "residual epilogue needs resid");
   E3_CHECK_ARG(M > 0 && N > 0 && K > 0 && lda >= K, "bad dims");
-  if (K % 64 || N % 64 || lda % 8 || !aligned16(A) || !aligned16(W) || !aligned16(C) || !aligned16(bias)) {
-    set_error("e3_op_gemm: need K % 64 == 0, N % 64 == 0, lda % 8 == 0, 16-byte aligned pointers");
+  if (K % 128 || N % 64 || lda % 8 || !aligned16(A) || !aligned16(W) || !aligned16(C) || !aligned16(bias)) {
+    set_error("e3_op_gemm: need K % 128 == 0, N % 64 == 0, lda % 8 == 0, 16-byte aligned pointers");
     return E3_EUNSUPPORTED;
   }
   int dev = 0;
   E3_CUDA_TRY(cudaGetDevice(&dev));
   const int sms = num_sms(dev);
   GemmMaps g;
-  e3_status r = gemm_tmaps(&g, A, lda, W, M, N, K, gemm_pick_bn(M, N, sms));
+  e3_status r = gemm_tmaps(&g, A, lda, W, C, M, N, K, gemm_pick_bn(M, N, sms));
   if (r != E3_OK) return r;
-  return gemm_run(g, C, bias, resid, M, N, K, epilogue, sms, reinterpret_cast<cudaStream_t>(stream));
+  return gemm_run(g, bias, resid, M, N, K, epilogue, sms, reinterpret_cast<cudaStream_t>(stream));
 }
 
 e3_status e3_op_attention(void *stream, const void *qkv, void *ctx, int32_t B, int32_t S, int32_t H, int32_t heads) {
@@ -339,9 +339,9 @@ e3_status e3_op_attention(void *stream, const void *qkv, void *ctx, int32_t B, i
     return E3_EUNSUPPORTED;
   }
   AttnMaps m;
-  e3_status r = attn_tmaps(&m, qkv, B, S, H);
+  e3_status r = attn_tmaps(&m, qkv, ctx, B, S, H);
   if (r != E3_OK) return r;
-  return attn_run(m, ctx, B, S, H, heads, reinterpret_cast<cudaStream_t>(stream));
+  return attn_run(m, B, S, H, heads, reinterpret_cast<cudaStream_t>(stream));
 }
 
 e3_status e3_op_layernorm(void *stream, const void *x, const void *g, const void *b, void *y, int32_t rows, int32_t H,

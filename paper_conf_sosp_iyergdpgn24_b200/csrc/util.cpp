@@ -33,7 +33,7 @@ PFN_encodeTiled encode_tiled_fn() {
 }
 
 static e3_status encode(CUtensorMap *m, int rank, const void *base, const cuuint64_t *dims, const cuuint64_t *strides,
-                        const cuuint32_t *box) {
+                        const cuuint32_t *box, CUtensorMapSwizzle swz = CU_TENSOR_MAP_SWIZZLE_128B) {
   PFN_encodeTiled fn = encode_tiled_fn();
   if (!fn) {
     set_error("cuTensorMapEncodeTiled unavailable (no CUDA driver?)");
@@ -41,7 +41,7 @@ static e3_status encode(CUtensorMap *m, int rank, const void *base, const cuuint
   }
   cuuint32_t estr[3] = {1, 1, 1};
   CUresult r = fn(m, CU_TENSOR_MAP_DATA_TYPE_BFLOAT16, (cuuint32_t)rank, const_cast<void *>(base), dims, strides, box,
-                  estr, CU_TENSOR_MAP_INTERLEAVE_NONE, CU_TENSOR_MAP_SWIZZLE_128B,
+                  estr, CU_TENSOR_MAP_INTERLEAVE_NONE, swz,
                   CU_TENSOR_MAP_L2_PROMOTION_L2_256B, CU_TENSOR_MAP_FLOAT_OOB_FILL_NONE);
   if (r != CUDA_SUCCESS) {
     char buf[160];
@@ -59,6 +59,14 @@ e3_status make_tmap_2d(CUtensorMap *m, const void *base, uint64_t rows, uint64_t
   cuuint64_t strides[1] = {row_pitch_elems * 2};
   cuuint32_t box[2] = {box_cols, box_rows};
   return encode(m, 2, base, dims, strides, box);
+}
+
+e3_status make_tmap_2d_sw64(CUtensorMap *m, const void *base, uint64_t rows, uint64_t cols, uint64_t row_pitch_elems,
+                            uint32_t box_rows, uint32_t box_cols) {
+  cuuint64_t dims[2] = {cols, rows};
+  cuuint64_t strides[1] = {row_pitch_elems * 2};
+  cuuint32_t box[2] = {box_cols, box_rows};
+  return encode(m, 2, base, dims, strides, box, CU_TENSOR_MAP_SWIZZLE_64B);
 }
 
 e3_status make_tmap_3d(CUtensorMap *m, const void *base, uint64_t d0, uint64_t d1, uint64_t d2, uint64_t pitch1,
