@@ -84,6 +84,8 @@ __global__ void __launch_bounds__(kThreads)
   __syncthreads();
   tc_fence_after();
   const uint32_t tbase = *tslot;
+  pdl_wait();                       // qkv of the previous kernel now visible
+  pdl_trigger();
 
   auto issue_load = [&](int item, int buf) {
     const int bh = item / qtiles, qt = item % qtiles;
@@ -253,7 +255,8 @@ e3_status launch_attn(const AttnMaps &m, int B, int S, int H, int heads, cudaStr
   const int n_items = B * heads * ((S + QT - 1) / QT);
   const int per_sm = (SKV == 128) ? 2 : 1;
   const int grid = n_items < per_sm * sms ? n_items : per_sm * sms;
-  kern<<<grid, kThreads, ACfg<SKV>::kSmem, st>>>(m.q, m.kv, m.ctx, S, H, heads, n_items);
+  E3_CUDA_TRY(launch_k(kern, dim3(grid), dim3(kThreads), ACfg<SKV>::kSmem, st, m.q, m.kv, m.ctx, S, H, heads,
+                       n_items));
   E3_CUDA_TRY(cudaGetLastError());
   count_launch();
   return E3_OK;

@@ -109,6 +109,8 @@ __global__ void __cluster_dims__(2, 1, 1) __launch_bounds__(kThreads, 1)
   cluster_sync();                  // peer barriers initialised, TMEM allocated in both CTAs
   tc_fence_after();
   const uint32_t tmem_base = *tmem_base_slot;
+  pdl_wait();                      // A / residual / C of the previous kernels now visible
+  pdl_trigger();
 
   if (warp == 0) {
     // ------------------------------------------------ TMA producer (both CTAs)
@@ -277,7 +279,7 @@ e3_status launch(const GemmMaps &g, const __nv_bfloat16 *bias, const __nv_bfloat
   }
   const int tiles = ((M + 2 * BM - 1) / (2 * BM)) * (N / BN);
   const int pairs = tiles < sms / 2 ? tiles : sms / 2;
-  kern<<<2 * pairs, kThreads, Cfg<BN>::kSmem, st>>>(g.a, g.b, g.c, bias, R, M, N, K);
+  E3_CUDA_TRY(launch_k(kern, dim3(2 * pairs), dim3(kThreads), Cfg<BN>::kSmem, st, g.a, g.b, g.c, bias, R, M, N, K));
   E3_CUDA_TRY(cudaGetLastError());
   count_launch();
   return E3_OK;

@@ -41,7 +41,8 @@ e3_status layernorm_run(const void *x, const void *g, const void *b, void *y, in
 constexpr int kRampRowsPerCta = 16;   // rows per ramp row group (one ticket each)
 struct RampArgs {
   int arch;
-  const void *x;            // [B,S,H] bf16
+  const void *x;            // [B,S,H] bf16 (pre-LN rows when ln_g != NULL)
+  const void *ln_g, *ln_b;  // optional LayerNorm applied to the CLS rows first
   const int64_t *id;        // [B]
   int B, S, H, C;
   e3_ramp_weights w;
@@ -72,6 +73,12 @@ struct RingDst {
 };
 e3_status compact_run(const void *x, const int64_t *id, const uint8_t *alive, int B, int64_t row_bytes,
                       const RingDst &dst, int32_t *n_surv_dev, unsigned *done_ctr, int sms, cudaStream_t st);
+
+// fused LN2 + compaction: survivors of the PRE-LN rows y [B,S,H] are
+// LayerNorm-ed (g, b, eps) and written to dst
+e3_status ln_compact_run(const void *y, const int64_t *id, const uint8_t *alive, int B, int S, int H, const void *g,
+                         const void *b, float eps, const RingDst &dst, int32_t *n_surv_dev, unsigned *done_ctr,
+                         int sms, cudaStream_t st);
 
 // ---- K6 queue pop (compact.cu): rows [head, head+n) of a ring -> contiguous
 // dst, zero-padding rows n..B-1 (ids -1).

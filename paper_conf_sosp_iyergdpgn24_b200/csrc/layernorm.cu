@@ -1,9 +1,11 @@
 // Row LayerNorm of the post-LN encoder layer:
 // y = bf16((x - mean) / sqrt(var + eps) * g + b), fp32 statistics, biased
-// variance, two passes over registers.  One warp per row, 16-byte loads; the
-// row (H <= 4096 bf16) stays in registers.  HBM-bound: 2 * H * 2 bytes/row.
+// variance, two passes over registers (ln_row.cuh).  One warp per row, 16-byte
+// loads, the row and gamma/beta loaded together (one memory round trip).
+// HBM/L2-bound: 2 * H * 2 bytes per row.
 #include "common.cuh"
 #include "kernels.h"
+#include "ln_row.cuh"
 #include "prof.h"
 
 namespace e3 {
@@ -16,62 +18,16 @@ __global__ void __launch_bounds__(256)
                      const __nv_bfloat16 *__restrict__ bb, __nv_bfloat16 *__restrict__ y, int rows, int H,
                      float eps) {
   const int row = blockIdx.x * 8 + warp_id();
-  if (row >= rows) return;
   const int lane = lane_id();
-  const int nvec = H / 8;
-  const uint4 *xr = reinterpret_cast<const uint4 *>(x + (size_t)row * H);
   uint4 v[VPL];
-  float s = 0.f;
-#pragma unroll
-  for (int i = 0; i < VPL; ++i) {
-    const int k = lane + 32 * i;
-    if (k < nvec) {
-      v[i] = __ldg(xr + k);
-      const uint32_t w[4] = {v[i].x, v[i].y, v[i].z, v[i].w};
-#pragma unroll
-      for (int e = 0; e < 4; ++e) s += bf_lo(w[e]) + bf_hi(w[e]);
-    }
-  }
-#pragma unroll
-  for (int o = 16; o; o >>= 1) s += __shfl_xor_sync(0xffffffffu, s, o);
-  const float mean = s / (float)H;
-  float q = 0.f;
-#pragma unroll
-  for (int i = 0; i < VPL; ++i) {
-    const int k = lane + 32 * i;
-    if (k < nvec) {
-      const uint32_t w[4] = {v[i].x, v[i].y, v[i].z, v[i].w};
-#pragma unroll
-      for (int e = 0; e < 4; ++e) {
-        const float a = bf_lo(w[e]) - mean, c = bf_hi(w[e]) - mean;
-        q += a * a + c * c;
-      }
-    }
-  }
-#pragma unroll
-  for (int o = 16; o; o >>= 1) q += __shfl_xor_sync(0xffffffffu, q, o);
-  const float rstd = 1.0f / sqrtf(q / (float)H + eps);
-  uint4 *yr = reinterpret_cast<uint4 *>(y + (size_t)row * H);
-  const uint4 *gp = reinterpret_cast<const uint4 *>(g);
-  const uint4 *bp = reinterpret_cast<const uint4 *>(bb);
-#pragma unroll
-  for (int i = 0; i < VPL; ++i) {
-    const int k = lane + 32 * i;
-    if (k < nvec) {
-      const uint4 g4 = __ldg(gp + k), b4 = __ldg(bp + k);
-      const uint32_t w[4] = {v[i].x, v[i].y, v[i].z, v[i].w};
-      const uint32_t gw[4] = {g4.x, g4.y, g4.z, g4.w};
-      const uint32_t bw[4] = {b4.x, b4.y, b4.z, b4.w};
-      uint32_t o[4];
-#pragma unroll
-      for (int e = 0; e < 4; ++e) {
-        const float a = (bf_lo(w[e]) - mean) * rstd * bf_lo(gw[e]) + bf_lo(bw[e]);
-        const float c = (bf_hi(w[e]) - mean) * rstd * bf_hi(gw[e]) + bf_hi(bw[e]);
-        o[e] = pack_bf16(a, c);
-      }
-      yr[k] = make_uint4(o[0], o[1], o[2], o[3]);
-    }
-  }
+  LnParams<VPL> p;
+  ln_load_params<VPL>(p, g, bb, H, lane);   // weights: before the dependency wait
+  pdl_wait();
+  pdl_trigger();
+  if (row >= rows) return;
+  ln_load_row<VPL>(v, x + (size_t)row * H, H, lane);
+  ln_apply<VPL>(v, p, H, eps, lane);
+  ln_store_row<VPL>(v, y + (size_t)row * H, H, lane);
 }
 
 }  // namespace
@@ -84,11 +40,11 @@ e3_status layernorm_run(const void *x, const void *g, const void *b, void *y, in
   auto *bp = reinterpret_cast<const __nv_bfloat16 *>(b);
   auto *yp = reinterpret_cast<__nv_bfloat16 *>(y);
   const int vpl = (H / 8 + 31) / 32;
-  if (vpl <= 1) layernorm_kernel<1><<<grid, 256, 0, st>>>(xp, gp, bp, yp, rows, H, eps);
-  else if (vpl <= 3) layernorm_kernel<3><<<grid, 256, 0, st>>>(xp, gp, bp, yp, rows, H, eps);
-  else if (vpl <= 4) layernorm_kernel<4><<<grid, 256, 0, st>>>(xp, gp, bp, yp, rows, H, eps);
-  else if (vpl <= 8) layernorm_kernel<8><<<grid, 256, 0, st>>>(xp, gp, bp, yp, rows, H, eps);
-  else if (vpl <= 16) layernorm_kernel<16><<<grid, 256, 0, st>>>(xp, gp, bp, yp, rows, H, eps);
+  if (vpl <= 1) E3_CUDA_TRY(launch_k(layernorm_kernel<1>, dim3(grid), dim3(256), 0, st, xp, gp, bp, yp, rows, H, eps));
+  else if (vpl <= 3) E3_CUDA_TRY(launch_k(layernorm_kernel<3>, dim3(grid), dim3(256), 0, st, xp, gp, bp, yp, rows, H, eps));
+  else if (vpl <= 4) E3_CUDA_TRY(launch_k(layernorm_kernel<4>, dim3(grid), dim3(256), 0, st, xp, gp, bp, yp, rows, H, eps));
+  else if (vpl <= 8) E3_CUDA_TRY(launch_k(layernorm_kernel<8>, dim3(grid), dim3(256), 0, st, xp, gp, bp, yp, rows, H, eps));
+  else if (vpl <= 16) E3_CUDA_TRY(launch_k(layernorm_kernel<16>, dim3(grid), dim3(256), 0, st, xp, gp, bp, yp, rows, H, eps));
   else {
     set_error("LayerNorm: H > 4096 unsupported");
     return E3_EUNSUPPORTED;

@@ -8,8 +8,12 @@
 //
 // One launch; grid (H / 32 pooler-output tiles, ceil(B / 16) row groups),
 // 4 warps per CTA:
-//   stage    cp.async the 16 CLS rows and the 32 W_p rows of the tile into
-//            padded smem (row pitch H + 8 bf16: conflict-free fragments);
+//   stage    the 32 W_p rows of the tile by cp.async into padded smem (row
+//            pitch H + 8 bf16: conflict-free fragments) and the 16 CLS rows:
+//            either copied (cp.async) or, at a split's last layer, read
+//            PRE-LayerNorm and normalised here by the shared warp-per-row LN
+//            (ln_row.cuh) -- bit-identical to what the fused LN + compaction
+//            writes for the survivors, and no full LN2 pass is needed;
 //   pooler   warp w owns outputs 8w..8w+7 of the tile: mma.sync m16n8k16
 //            bf16 -> fp32 over K = H (a 16 x 32 x H GEMM per CTA is far too
 //            small for a tcgen05 tile; the tensor pipe is still the one used);
@@ -18,12 +22,14 @@
 //            the quad with __shfl_xor_sync and over the 4 warps in smem, and
 //            written to a per-tile slot (deterministic, no float atomics);
 //   decide   the CTA of row group g that retires last (threadfence + atomic
-//            ticket) sums the H/32 partials per (row, class) in fixed order,
-//            then softmax / max-prob / entropy, argmax (lowest index on ties),
-//            threshold test, exit record by input id and the alive flag.
+//            ticket) reduces the H/32 partials per (row, class) with one
+//            warp-shuffle butterfly per row (fixed order), then softmax /
+//            max-prob / entropy, argmax (lowest index on ties), threshold
+//            test, exit record by input id and the alive flag.
 // All ramp math is fp32, never rounded to bf16 (rounding contract).
 #include "common.cuh"
 #include "kernels.h"
+#include "ln_row.cuh"
 #include "prof.h"
 
 namespace e3 {
@@ -52,6 +58,7 @@ __device__ __forceinline__ bool row_alive(const RampArgs &a, int b, int n_valid)
   return b < a.B && (a.init_alive ? (b < n_valid) : (a.alive[b] != 0));
 }
 
+template <int VPL>
 __global__ void __launch_bounds__(kThreads)
     ramp_bert_kernel(RampArgs a) {
   extern __shared__ uint8_t smem_raw[];
@@ -68,26 +75,52 @@ __global__ void __launch_bounds__(kThreads)
   const int b0 = blockIdx.y * kRows;
   const int o0 = blockIdx.x * kTileN;
   const int C = a.C;
-  const int n_valid = a.n_valid_dev ? *a.n_valid_dev : a.n_valid_host;
   const int nvec = H / 8;
   const __nv_bfloat16 *x = reinterpret_cast<const __nv_bfloat16 *>(a.x);
   const size_t row_stride = (size_t)a.S * H;
 
   // ---------------------------------------------------------- stage
-  if (threadIdx.x < kRows) row_ok[threadIdx.x] = row_alive(a, b0 + threadIdx.x, n_valid);
-  __syncthreads();
-  for (int i = threadIdx.x; i < kRows * nvec; i += kThreads) {
-    const int r = i / nvec, k = i - r * nvec;
-    uint4 *dst = reinterpret_cast<uint4 *>(sC + r * P) + k;
-    if (row_ok[r])
-      cp_async16(dst, reinterpret_cast<const uint4 *>(x + (size_t)(b0 + r) * row_stride) + k);
-    else
-      *dst = make_uint4(0, 0, 0, 0);
-  }
   const uint4 *wp = reinterpret_cast<const uint4 *>(a.w.w_p);
-  for (int i = threadIdx.x; i < kTileN * nvec; i += kThreads) {
+  for (int i = threadIdx.x; i < kTileN * nvec; i += kThreads) {   // weights first: no dependency
     const int r = i / nvec, k = i - r * nvec;
     cp_async16(reinterpret_cast<uint4 *>(sW + r * P) + k, wp + (size_t)(o0 + r) * nvec + k);
+  }
+  pdl_wait();                      // CLS rows / alive flags of the previous kernels now visible
+  pdl_trigger();
+  const int n_valid = a.n_valid_dev ? *a.n_valid_dev : a.n_valid_host;
+  if (threadIdx.x < kRows) row_ok[threadIdx.x] = row_alive(a, b0 + threadIdx.x, n_valid);
+  __syncthreads();
+  if (a.ln_g) {
+    LnParams<VPL> lp;
+    ln_load_params<VPL>(lp, reinterpret_cast<const __nv_bfloat16 *>(a.ln_g),
+                        reinterpret_cast<const __nv_bfloat16 *>(a.ln_b), H, lane);
+    constexpr int kPerWarp = kRows / (kThreads / 32);   // 4 CLS rows per warp, loads in flight together
+    uint4 v[kPerWarp][VPL];
+#pragma unroll
+    for (int u = 0; u < kPerWarp; ++u) {
+      const int r = warp + u * (kThreads / 32);
+      if (row_ok[r]) {
+        ln_load_row<VPL>(v[u], x + (size_t)(b0 + r) * row_stride, H, lane);
+      } else {
+#pragma unroll
+        for (int i = 0; i < VPL; ++i) v[u][i] = make_uint4(0, 0, 0, 0);
+      }
+    }
+#pragma unroll
+    for (int u = 0; u < kPerWarp; ++u) {
+      const int r = warp + u * (kThreads / 32);
+      if (row_ok[r]) ln_apply<VPL>(v[u], lp, H, a.eps, lane);
+      ln_store_row<VPL>(v[u], sC + r * P, H, lane);
+    }
+  } else {
+    for (int i = threadIdx.x; i < kRows * nvec; i += kThreads) {
+      const int r = i / nvec, k = i - r * nvec;
+      uint4 *dst = reinterpret_cast<uint4 *>(sC + r * P) + k;
+      if (row_ok[r])
+        cp_async16(dst, reinterpret_cast<const uint4 *>(x + (size_t)(b0 + r) * row_stride) + k);
+      else
+        *dst = make_uint4(0, 0, 0, 0);
+    }
   }
   cp_async_wait_all();
   __syncthreads();
@@ -161,75 +194,70 @@ __global__ void __launch_bounds__(kThreads)
   __threadfence();
 
   // ---------------------------------------------------------- decide
-  // gather the group's partials [tiles][16 rows][C] into smem with all loads
-  // independent (one L2 round trip), then one thread per row sums them in
-  // fixed tile order.
-  float *sP = reinterpret_cast<float *>(smem_raw);   // reuse the staging area
-  const int ntiles = gridDim.x;
-  const int per_tile = kRows * C;
-  for (int i = threadIdx.x; i < ntiles * per_tile; i += kThreads) {
-    const int nt = i / per_tile, rc = i - nt * per_tile;
-    const int rr = rc / C;
-    sP[i] = (b0 + rr < a.B) ? __ldcg(part + ((size_t)nt * a.B + b0) * C + rc) : 0.f;
-  }
-  __syncthreads();
-  const int r = threadIdx.x;
-  if (r >= kRows || b0 + r >= a.B) return;
-  const int b = b0 + r;
-  if (!row_ok[r]) {
-    if (a.init_alive) a.alive[b] = 0;
-    return;
-  }
+  // warp per row; lane l < ntiles holds tile l's partial logits, butterfly sum
+  const int ntiles = gridDim.x;                // <= 32 (H <= 1024)
   const __nv_bfloat16 *bc = reinterpret_cast<const __nv_bfloat16 *>(a.w.b_c);
-  float z[kMaxC];
-#pragma unroll
-  for (int c = 0; c < kMaxC; ++c) {
-    z[c] = 0.f;
-    if (c < C) {
-      float s = 0.f;
-      for (int nt = 0; nt < ntiles; ++nt) s += sP[nt * per_tile + r * C + c];
-      z[c] = s + bf2f(bc[c]);
+  for (int r = warp; r < kRows; r += kThreads / 32) {
+    const int b = b0 + r;
+    if (b >= a.B) break;
+    if (!row_ok[r]) {
+      if (a.init_alive && lane == 0) a.alive[b] = 0;
+      continue;
     }
-  }
-  float m = z[0];
-  int label = 0;
+    float z[kMaxC];
 #pragma unroll
-  for (int c = 1; c < kMaxC; ++c)
-    if (c < C && z[c] > m) { m = z[c]; label = c; }   // lowest index on ties
-  float sum = 0.f, qz = 0.f;
+    for (int c = 0; c < kMaxC; ++c)
+      z[c] = (c < C && lane < ntiles) ? __ldcg(part + ((size_t)lane * a.B + b) * C + c) : 0.f;
 #pragma unroll
-  for (int c = 0; c < kMaxC; ++c)
-    if (c < C) {
-      const float e = expf(z[c] - m);
-      sum += e;
-      qz += e * (z[c] - m);
-    }
-  float metric;
-  bool pass;
-  if (a.test == E3_TEST_MAXPROB) {
-    metric = 1.0f / sum;                       // max_c softmax(z)_c
-    pass = metric > a.tau;
-  } else {
-    metric = logf(sum) - qz / sum;             // H = lse - sum_c q_c z_c
-    pass = metric < a.tau;
-  }
-  const bool exit_now = pass || a.final_ramp;
-  if (exit_now) {
-    const int64_t id = a.id[b];
-    if (id >= 0 && id < a.ex.capacity) {
-      if (a.ex.exit_layer) a.ex.exit_layer[id] = a.layer;
-      if (a.ex.label) a.ex.label[id] = label;
-      if (a.ex.conf) a.ex.conf[id] = metric;
-      if (a.ex.logits) {
+    for (int c = 0; c < kMaxC; ++c) {
+      if (c < C) {
 #pragma unroll
-        for (int c = 0; c < kMaxC; ++c)
-          if (c < C) a.ex.logits[id * C + c] = z[c];
+        for (int o = 16; o; o >>= 1) z[c] += __shfl_xor_sync(0xffffffffu, z[c], o);
+        z[c] += bf2f(bc[c]);
       }
     }
-    if (a.ex.n_exit) atomicAdd(a.ex.n_exit, 1);
-    if (a.ex.ramp_count) atomicAdd(a.ex.ramp_count + a.ramp_index, 1);
+    if (lane == 0) {
+      float m = z[0];
+      int label = 0;
+#pragma unroll
+      for (int c = 1; c < kMaxC; ++c)
+        if (c < C && z[c] > m) { m = z[c]; label = c; }   // lowest index on ties
+      float sum = 0.f, qz = 0.f;
+#pragma unroll
+      for (int c = 0; c < kMaxC; ++c)
+        if (c < C) {
+          const float e = expf(z[c] - m);
+          sum += e;
+          qz += e * (z[c] - m);
+        }
+      float metric;
+      bool pass;
+      if (a.test == E3_TEST_MAXPROB) {
+        metric = 1.0f / sum;                       // max_c softmax(z)_c
+        pass = metric > a.tau;
+      } else {
+        metric = logf(sum) - qz / sum;             // H = lse - sum_c q_c z_c
+        pass = metric < a.tau;
+      }
+      const bool exit_now = pass || a.final_ramp;
+      if (exit_now) {
+        const int64_t id = a.id[b];
+        if (id >= 0 && id < a.ex.capacity) {
+          if (a.ex.exit_layer) a.ex.exit_layer[id] = a.layer;
+          if (a.ex.label) a.ex.label[id] = label;
+          if (a.ex.conf) a.ex.conf[id] = metric;
+          if (a.ex.logits) {
+#pragma unroll
+            for (int c = 0; c < kMaxC; ++c)
+              if (c < C) a.ex.logits[id * C + c] = z[c];
+          }
+        }
+        if (a.ex.n_exit) atomicAdd(a.ex.n_exit, 1);
+        if (a.ex.ramp_count) atomicAdd(a.ex.ramp_count + a.ramp_index, 1);
+      }
+      a.alive[b] = exit_now ? 0 : 1;
+    }
   }
-  a.alive[b] = exit_now ? 0 : 1;
 }
 
 }  // namespace
@@ -244,14 +272,23 @@ e3_status ramp_run(const RampArgs &a, cudaStream_t st) {
     return E3_EUNSUPPORTED;
   }
   const int smem = (kRows + kTileN) * (a.H + 8) * 2 + 4 * kRows * kMaxC * 4;
-  static bool attr_done = false;
-  if (!attr_done) {
-    E3_CUDA_TRY(cudaFuncSetAttribute(ramp_bert_kernel, cudaFuncAttributeMaxDynamicSharedMemorySize,
-                                     (kRows + kTileN) * (1024 + 8) * 2 + 4 * kRows * kMaxC * 4));
-    attr_done = true;
-  }
+  const int smem_max = (kRows + kTileN) * (1024 + 8) * 2 + 4 * kRows * kMaxC * 4;
   dim3 grid(a.H / kTileN, (a.B + kRows - 1) / kRows);
-  ramp_bert_kernel<<<grid, kThreads, smem, st>>>(a);
+  const int vpl = (a.H / 8 + 31) / 32;
+#define E3_RAMP(V)                                                                                        \
+  do {                                                                                                    \
+    static bool attr_done = false;                                                                        \
+    if (!attr_done) {                                                                                     \
+      E3_CUDA_TRY(cudaFuncSetAttribute(ramp_bert_kernel<V>, cudaFuncAttributeMaxDynamicSharedMemorySize, \
+                                       smem_max));                                                        \
+      attr_done = true;                                                                                   \
+    }                                                                                                     \
+    E3_CUDA_TRY(launch_k(ramp_bert_kernel<V>, grid, dim3(kThreads), smem, st, a));                        \
+  } while (0)
+  if (vpl <= 1) E3_RAMP(1);
+  else if (vpl <= 3) E3_RAMP(3);
+  else E3_RAMP(4);
+#undef E3_RAMP
   E3_CUDA_TRY(cudaGetLastError());
   count_launch();
   return E3_OK;

@@ -222,17 +222,23 @@ e3_status split_run_to(e3_split *s, cudaStream_t st, const void *x_in, const int
       ProfScope ps(PK_GEMM_FFN2, st, f_1, 0);
       E3_RUN(gemm_run(m.f2, L.b_2, ws.x1, M, H, F, E3_EPI_BIAS_RESID, s->sms, st));
     }
-    {
+    // The split's last layer never materialises LN2: its ramp normalises the
+    // CLS rows itself and the fused LN2 + compaction normalises only the
+    // survivors, writing them straight to the destination.
+    const bool last_layer = (i == nl - 1);
+    if (!last_layer) {
       ProfScope ps(PK_LN, st, 0, b_ln);
       E3_RUN(layernorm_run(ws.y, L.ln2_g, L.ln2_b, out, M, H, d.norm_eps, st));
+      cur = out;
     }
-    cur = out;
     while (ri < d.n_ramps && d.ramp_layer[ri] == l) {
       const bool last = (ri == d.n_ramps - 1);
       if (last || d.inner == E3_INNER_EXACT) {
         RampArgs a{};
         a.arch = d.arch;
-        a.x = cur;
+        a.x = last_layer ? ws.y : cur;
+        a.ln_g = last_layer ? L.ln2_g : nullptr;
+        a.ln_b = last_layer ? L.ln2_b : nullptr;
         a.id = id_in;
         a.B = B;
         a.S = S;
@@ -264,8 +270,12 @@ e3_status split_run_to(e3_split *s, cudaStream_t st, const void *x_in, const int
     }
   }
   {
-    ProfScope ps(PK_COMPACT, st, 0, 0);   // bytes added once n_surv is known (pipeline)
-    E3_RUN(compact_run(cur, id_in, ws.alive, B, (int64_t)S * H * 2, dst, n_surv_dev, ws.ctr, s->sms, st));
+    // survivors: LN2 of the last layer fused with the stable compaction
+    // (bytes added once n_surv is known, in the pipeline)
+    const e3_layer_weights &L = s->L[nl - 1];
+    ProfScope ps(PK_COMPACT, st, 0, 0);
+    E3_RUN(ln_compact_run(ws.y, id_in, ws.alive, B, S, H, L.ln2_g, L.ln2_b, d.norm_eps, dst, n_surv_dev, ws.ctr,
+                          s->sms, st));
   }
 #undef E3_RUN
   return E3_OK;

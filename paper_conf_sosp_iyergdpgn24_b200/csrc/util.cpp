@@ -3,6 +3,7 @@
 #include <cuda_runtime.h>
 
 #include <cstdio>
+#include <cstdlib>
 #include <mutex>
 #include <string>
 
@@ -75,6 +76,14 @@ e3_status make_tmap_3d(CUtensorMap *m, const void *base, uint64_t d0, uint64_t d
   cuuint64_t strides[2] = {pitch1 * 2, pitch2 * 2};
   cuuint32_t box[3] = {b0, b1, b2};
   return encode(m, 3, base, dims, strides, box);
+}
+
+bool pdl_enabled() {
+  static const bool on = [] {
+    const char *e = getenv("E3_NO_PDL");
+    return !(e && e[0] == '1');
+  }();
+  return on;
 }
 
 int num_sms(int device) {
