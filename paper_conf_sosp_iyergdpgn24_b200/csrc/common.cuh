@@ -313,6 +313,35 @@ __device__ __forceinline__ float gelu_fast(float x) {
   return x * phi;
 }
 
+// gelu_fast on a pair of values with Blackwell's packed fp32x2 FMA/MUL
+// (FFMA2): same arithmetic, same rounding per element, ~35 % fewer issued
+// instructions -- the FFN1 epilogue is issue-bound.
+__device__ __forceinline__ float2 gelu_fast2(float2 x) {
+  const float2 z = __fmul2_rn(make_float2(fabsf(x.x), fabsf(x.y)), make_float2(0.70710678118654752f, 0.70710678118654752f));
+  const float2 d = __ffma2_rn(make_float2(0.5f, 0.5f), z, make_float2(1.0f, 1.0f));
+  float2 t;
+  asm("rcp.approx.ftz.f32 %0, %1;" : "=f"(t.x) : "f"(d.x));
+  asm("rcp.approx.ftz.f32 %0, %1;" : "=f"(t.y) : "f"(d.y));
+  float2 p = make_float2(0.17087277f, 0.17087277f);
+  p = __ffma2_rn(p, t, make_float2(-0.82215223f, -0.82215223f));
+  p = __ffma2_rn(p, t, make_float2(1.48851587f, 1.48851587f));
+  p = __ffma2_rn(p, t, make_float2(-1.13520398f, -1.13520398f));
+  p = __ffma2_rn(p, t, make_float2(0.27886807f, 0.27886807f));
+  p = __ffma2_rn(p, t, make_float2(-0.18628806f, -0.18628806f));
+  p = __ffma2_rn(p, t, make_float2(0.09678418f, 0.09678418f));
+  p = __ffma2_rn(p, t, make_float2(0.37409196f, 0.37409196f));
+  p = __ffma2_rn(p, t, make_float2(1.00002368f, 1.00002368f));
+  p = __ffma2_rn(p, t, make_float2(-1.26551223f, -1.26551223f));
+  const float2 nz = __fmul2_rn(z, make_float2(-1.0f, -1.0f));
+  const float2 arg = __fmul2_rn(__ffma2_rn(nz, z, p), make_float2(1.4426950408889634f, 1.4426950408889634f));
+  float2 e;
+  asm("ex2.approx.ftz.f32 %0, %1;" : "=f"(e.x) : "f"(arg.x));
+  asm("ex2.approx.ftz.f32 %0, %1;" : "=f"(e.y) : "f"(arg.y));
+  const float2 he = __fmul2_rn(__fmul2_rn(t, e), make_float2(0.5f, 0.5f));   // Phi(-|x|)
+  const float2 phi = make_float2(x.x >= 0.f ? 1.0f - he.x : he.x, x.y >= 0.f ? 1.0f - he.y : he.y);
+  return __fmul2_rn(x, phi);
+}
+
 __device__ __forceinline__ int warp_id() { return threadIdx.x >> 5; }
 __device__ __forceinline__ int lane_id() { return threadIdx.x & 31; }
 

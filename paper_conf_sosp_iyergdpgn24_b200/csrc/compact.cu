@@ -174,84 +174,78 @@ __global__ void fill_kernel(int32_t *dst, int v) { *dst = v; }
 // read PRE-LayerNorm (y = residual sum), normalised (ln_row.cuh, bit-identical
 // to layernorm_kernel and to the ramp's CLS rows) and written straight into
 // the destination (next split's queue ring or a contiguous buffer).  Rows that
-// exited are never normalised or written.  One warp per token row, two rows in
-// flight per warp.
+// exited are never normalised or written.  One warp per token row, kRowsInFlight
+// rows' loads in flight per warp.  No grid-wide ticket: every CTA derives the
+// same survivor count from the flags, CTA 0 publishes it (n_surv, host
+// mailbox, overflow flag) and writes the queue's NEXT tail slot (dst.tail_out)
+// while everyone reads the current one (dst.tail_dev) -- the two slots
+// alternate per push, chosen by the host.
+constexpr int kRowsInFlight = 4;
+
 template <int VPL>
 __global__ void __launch_bounds__(kThreads)
     ln_compact_kernel(const __nv_bfloat16 *__restrict__ y, const int64_t *__restrict__ id,
                       const uint8_t *__restrict__ alive, int B, int S, int H, const __nv_bfloat16 *__restrict__ g,
-                      const __nv_bfloat16 *__restrict__ bb, float eps, RingDst dst, int32_t *n_surv_dev,
-                      unsigned *done_ctr) {
+                      const __nv_bfloat16 *__restrict__ bb, float eps, RingDst dst, int32_t *n_surv_dev) {
   __shared__ int16_t src_of[kMaxB];
   __shared__ int word_cnt[kMaxB / 32 + 1];
-  __shared__ bool is_last;
   const int warp = warp_id(), lane = lane_id();
   LnParams<VPL> p;
   ln_load_params<VPL>(p, g, bb, H, lane);   // weights: before the dependency wait
   pdl_wait();
   pdl_trigger();
+  const int64_t tail = dst.tail_dev ? *dst.tail_dev : 0;
   const int n = block_scan_flags(alive, B, src_of, word_cnt);
-  const int64_t tail = dst.tail_dev ? *(volatile int64_t *)dst.tail_dev : 0;
   const bool fits = (tail - dst.head) + n <= dst.cap;
-
-  if (fits && n > 0) {
-    const int units = n * S;
-    const int stride = gridDim.x * (kThreads / 32);
-    __nv_bfloat16 *ring = reinterpret_cast<__nv_bfloat16 *>(dst.rows);
-    const size_t row_elems = (size_t)S * H;
-    for (int u0 = blockIdx.x * (kThreads / 32) + warp; u0 < units; u0 += 2 * stride) {
-      const int u1 = u0 + stride;
-      uint4 v0[VPL], v1[VPL];
-      const int k0 = u0 / S, t0 = u0 - k0 * S;
-      ln_load_row<VPL>(v0, y + (size_t)src_of[k0] * row_elems + (size_t)t0 * H, H, lane);
-      int k1 = 0, t1 = 0;
-      if (u1 < units) {
-        k1 = u1 / S;
-        t1 = u1 - k1 * S;
-        ln_load_row<VPL>(v1, y + (size_t)src_of[k1] * row_elems + (size_t)t1 * H, H, lane);
-      }
-      ln_apply<VPL>(v0, p, H, eps, lane);
-      ln_store_row<VPL>(v0, ring + ((tail + k0) % dst.cap) * row_elems + (size_t)t0 * H, H, lane);
-      if (u1 < units) {
-        ln_apply<VPL>(v1, p, H, eps, lane);
-        ln_store_row<VPL>(v1, ring + ((tail + k1) % dst.cap) * row_elems + (size_t)t1 * H, H, lane);
-      }
-    }
-    if (blockIdx.x == 0)
-      for (int k = threadIdx.x; k < n; k += kThreads) dst.ids[(tail + k) % dst.cap] = id[src_of[k]];
-  }
-
-  __threadfence();
-  __syncthreads();
-  if (threadIdx.x == 0) {
-    const unsigned t = atomicAdd(done_ctr, 1u);
-    is_last = (t == gridDim.x - 1);
-  }
-  __syncthreads();
-  if (is_last && threadIdx.x == 0) {
-    *done_ctr = 0;
+  if (blockIdx.x == 0 && threadIdx.x == 0) {
     const int out = fits ? n : 0;
     if (!fits && dst.overflow_dev) *dst.overflow_dev = 1;
-    if (fits && dst.tail_dev) *(volatile int64_t *)dst.tail_dev = tail + n;
+    if (dst.tail_out) *dst.tail_out = fits ? tail + n : tail;
     if (n_surv_dev) *n_surv_dev = out;
-    if (dst.mailbox) {
-      *dst.mailbox = fits ? out : -1;
-      __threadfence_system();
+    if (dst.mailbox) *dst.mailbox = fits ? out : -1;   // read by the host after the run's event
+  }
+  if (!fits || n == 0) return;
+
+  const int units = n * S;
+  const int stride = gridDim.x * (kThreads / 32);
+  __nv_bfloat16 *ring = reinterpret_cast<__nv_bfloat16 *>(dst.rows);
+  const size_t row_elems = (size_t)S * H;
+  for (int u0 = blockIdx.x * (kThreads / 32) + warp; u0 < units; u0 += kRowsInFlight * stride) {
+    uint4 v[kRowsInFlight][VPL];
+#pragma unroll
+    for (int j = 0; j < kRowsInFlight; ++j) {
+      const int u = u0 + j * stride;
+      if (u < units) {
+        const int k = u / S, t = u - k * S;
+        ln_load_row<VPL>(v[j], y + (size_t)src_of[k] * row_elems + (size_t)t * H, H, lane);
+      }
+    }
+#pragma unroll
+    for (int j = 0; j < kRowsInFlight; ++j) {
+      const int u = u0 + j * stride;
+      if (u < units) {
+        const int k = u / S, t = u - k * S;
+        ln_apply<VPL>(v[j], p, H, eps, lane);
+        ln_store_row<VPL>(v[j], ring + ((tail + k) % dst.cap) * row_elems + (size_t)t * H, H, lane);
+      }
     }
   }
+  if (blockIdx.x == 0)
+    for (int k = threadIdx.x; k < n; k += kThreads) dst.ids[(tail + k) % dst.cap] = id[src_of[k]];
 }
 
 }  // namespace
 
 e3_status ln_compact_run(const void *y, const int64_t *id, const uint8_t *alive, int B, int S, int H, const void *g,
-                         const void *b, float eps, const RingDst &dst, int32_t *n_surv_dev, unsigned *done_ctr,
-                         int sms, cudaStream_t st) {
+                         const void *b, float eps, const RingDst &dst, int32_t *n_surv_dev, int sms,
+                         cudaStream_t st) {
   if (B > kMaxB || H % 8 || H > 4096) {
     set_error("ln_compact: need B <= 4096, H % 8 == 0, H <= 4096");
     return E3_EUNSUPPORTED;
   }
-  int64_t grid = ((int64_t)B * S + 7) / 8;   // one token row per warp on a full batch
-  if (grid > 8 * sms) grid = 8 * sms;
+  // kRowsInFlight token rows per warp on a full batch
+  int64_t grid = ((int64_t)B * S + 8 * kRowsInFlight - 1) / (8 * kRowsInFlight);
+  if (grid > 4 * sms) grid = 4 * sms;
   if (grid < 1) grid = 1;
   auto *yp = reinterpret_cast<const __nv_bfloat16 *>(y);
   auto *gp = reinterpret_cast<const __nv_bfloat16 *>(g);
@@ -259,7 +253,7 @@ e3_status ln_compact_run(const void *y, const int64_t *id, const uint8_t *alive,
   const int vpl = (H / 8 + 31) / 32;
 #define E3_LNC(V) \
   E3_CUDA_TRY(launch_k(ln_compact_kernel<V>, dim3((unsigned)grid), dim3(kThreads), 0, st, yp, id, alive, B, S, H, \
-                       gp, bp, eps, dst, n_surv_dev, done_ctr))
+                       gp, bp, eps, dst, n_surv_dev))
   if (vpl <= 1) E3_LNC(1);
   else if (vpl <= 3) E3_LNC(3);
   else if (vpl <= 4) E3_LNC(4);

@@ -220,7 +220,11 @@ __global__ void __cluster_dims__(2, 1, 1) __launch_bounds__(kThreads, 1)
         }
         if (EPI == E3_EPI_BIAS_GELU) {
 #pragma unroll
-          for (int j = 0; j < 32; ++j) v[j] = gelu_fast(v[j]);
+          for (int j = 0; j < 32; j += 2) {
+            const float2 gv = gelu_fast2(make_float2(v[j], v[j + 1]));
+            v[j] = gv.x;
+            v[j + 1] = gv.y;
+          }
         }
         if (EPI == E3_EPI_BIAS_RESID) {
 #pragma unroll

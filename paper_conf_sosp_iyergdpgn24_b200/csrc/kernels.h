@@ -66,7 +66,8 @@ struct RingDst {
   uint8_t *rows;            // [cap, row_bytes]
   int64_t *ids;             // [cap]
   int64_t cap;
-  int64_t *tail_dev;        // NULL: contiguous output at row 0
+  int64_t *tail_dev;        // current tail (read); NULL: contiguous output at row 0
+  int64_t *tail_out;        // next tail slot (written by ln_compact; NULL: none)
   int64_t head;             // host-known head (rows) at launch
   int *overflow_dev;        // may be NULL
   volatile int *mailbox;    // host-mapped slot for n_surv (may be NULL)
@@ -77,8 +78,8 @@ e3_status compact_run(const void *x, const int64_t *id, const uint8_t *alive, in
 // fused LN2 + compaction: survivors of the PRE-LN rows y [B,S,H] are
 // LayerNorm-ed (g, b, eps) and written to dst
 e3_status ln_compact_run(const void *y, const int64_t *id, const uint8_t *alive, int B, int S, int H, const void *g,
-                         const void *b, float eps, const RingDst &dst, int32_t *n_surv_dev, unsigned *done_ctr,
-                         int sms, cudaStream_t st);
+                         const void *b, float eps, const RingDst &dst, int32_t *n_surv_dev, int sms,
+                         cudaStream_t st);
 
 // ---- K6 queue pop (compact.cu): rows [head, head+n) of a ring -> contiguous
 // dst, zero-padding rows n..B-1 (ids -1).

@@ -39,7 +39,8 @@ struct DevQueue {
   uint8_t *rows = nullptr;
   int64_t *ids = nullptr;
   int64_t cap = 0;
-  int64_t *tail_dev = nullptr;
+  int64_t *tails = nullptr;   // device [2]: the tail alternates between two slots per push
+  int64_t pushes = 0;         // pushes issued (host): push j reads slot j&1, writes slot (j+1)&1
   int64_t head = 0;    // rows popped (host decision, exact)
   int64_t known = 0;   // rows pushed by completed runs (lower bound of tail)
 };
@@ -56,7 +57,7 @@ struct e3_pipeline {
   std::shared_ptr<e3::Workspace> ws;
   std::vector<e3_split *> splits;
   std::vector<DevQueue> q;            // q[s] feeds split s (q[0] unused)
-  int64_t *tails = nullptr;           // device [n_splits]
+  int64_t *tails = nullptr;           // device [2 * n_splits]
   int *overflow = nullptr;            // device flag
   uint8_t *staging = nullptr;         // [B, row] wrapped / flush pops
   int64_t *staging_ids = nullptr;
@@ -230,7 +231,9 @@ struct Runner {
       dst.rows = N.rows;
       dst.ids = N.ids;
       dst.cap = N.cap;
-      dst.tail_dev = N.tail_dev;
+      dst.tail_dev = N.tails + (N.pushes & 1);
+      dst.tail_out = N.tails + ((N.pushes + 1) & 1);
+      ++N.pushes;
       dst.head = N.head;
     } else {
       dst.rows = pl->sink;
@@ -350,14 +353,14 @@ e3_status e3_pipeline_create(const e3_plan *p, const e3_weights *w, int device, 
     return r;
   }
   const int64_t cap = (int64_t)pl->plan.queue_cap_batches * pl->B;
-  cudaError_t e = cudaMalloc(&pl->tails, sizeof(int64_t) * p->n_splits);
-  if (e == cudaSuccess) e = cudaMemset(pl->tails, 0, sizeof(int64_t) * p->n_splits);
+  cudaError_t e = cudaMalloc(&pl->tails, 2 * sizeof(int64_t) * p->n_splits);
+  if (e == cudaSuccess) e = cudaMemset(pl->tails, 0, 2 * sizeof(int64_t) * p->n_splits);
   if (e != cudaSuccess) return fail(e, "alloc tails");
   pl->q.resize(p->n_splits);
   for (int s = 1; s < p->n_splits; ++s) {
     DevQueue &Q = pl->q[s];
     Q.cap = cap;
-    Q.tail_dev = pl->tails + s;
+    Q.tails = pl->tails + 2 * s;
     e = cudaMalloc(&Q.rows, (size_t)cap * pl->row_bytes);
     if (e == cudaSuccess) e = cudaMalloc(&Q.ids, (size_t)cap * 8);
     if (e != cudaSuccess) return fail(e, "alloc queue ring");
@@ -426,8 +429,9 @@ e3_status e3_pipeline_run(e3_pipeline *pl, void *stream, const void *x, const in
   for (int s = 1; s < pl->plan.n_splits; ++s) {
     pl->q[s].head = 0;
     pl->q[s].known = 0;
+    pl->q[s].pushes = 0;
   }
-  E3_CUDA_TRY(cudaMemsetAsync(pl->tails, 0, sizeof(int64_t) * pl->plan.n_splits, R.st));
+  E3_CUDA_TRY(cudaMemsetAsync(pl->tails, 0, 2 * sizeof(int64_t) * pl->plan.n_splits, R.st));
   if (R.host_in) {
     // the copy stream must not overwrite staging slots still read by earlier work
     for (int i = 0; i < kInSlots; ++i) E3_CUDA_TRY(cudaEventRecord(pl->in_free[i], R.st));

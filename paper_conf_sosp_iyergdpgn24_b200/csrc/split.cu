@@ -274,8 +274,8 @@ e3_status split_run_to(e3_split *s, cudaStream_t st, const void *x_in, const int
     // (bytes added once n_surv is known, in the pipeline)
     const e3_layer_weights &L = s->L[nl - 1];
     ProfScope ps(PK_COMPACT, st, 0, 0);
-    E3_RUN(ln_compact_run(ws.y, id_in, ws.alive, B, S, H, L.ln2_g, L.ln2_b, d.norm_eps, dst, n_surv_dev, ws.ctr,
-                          s->sms, st));
+    E3_RUN(ln_compact_run(ws.y, id_in, ws.alive, B, S, H, L.ln2_g, L.ln2_b, d.norm_eps, dst, n_surv_dev, s->sms,
+                          st));
   }
 #undef E3_RUN
   return E3_OK;
