@@ -16,6 +16,9 @@ the timed region.
 
 N > 1 (torchrun): replica mode -- every rank runs the whole split chain on
 its own shard (weak scaling, no data-path collective).
+--mode stage: the chain is cut into stages on different GPUs (parallel.py,
+plan_stages balanced on the calibrated survival profile); survivors travel
+GPU to GPU over NCCL send/recv, chunk by chunk.
 Time = max over ranks of CUDA-event time, barrier + synchronize around it.
 
 --impl reference: the CPU oracle (oracle/, NumPy float64) timed on the host
@@ -53,6 +56,10 @@ def parse():
     ap.add_argument("--no-e2e", action="store_true")
     ap.add_argument("--no-cpu", action="store_true")
     ap.add_argument("--cpu-inputs", type=int, default=32)
+    ap.add_argument("--mode", default="replica", choices=["replica", "stage"],
+                    help="N>1: replicas of the whole chain, or stages on different GPUs (parallel.py)")
+    ap.add_argument("--chunk", type=int, default=1024, help="stage mode: inputs per chunk")
+    ap.add_argument("--stages", type=int, default=2, help="stage mode: number of stages")
     return ap.parse_args()
 
 
@@ -120,6 +127,12 @@ def plan_bounds(cfg, plan):
     return (0, 6, cfg.layers), "cut after layer 6 (2 splits, inner ramps exact)"
 
 
+def survival(cfg, layer):
+    """Expected fraction of inputs entering `layer` (0-based) under the
+    workload's calibrated exit profile (e3data.configs.survival_profile)."""
+    return 1.0 - sum(e for r, e in zip(cfg.ramp_layers, cfg.exit_profile) if r < layer)
+
+
 def cpu_oracle_rate(cfg, tau, n_inputs, seed_offset=0):
     """The oracle as it stands (fp64 NumPy, all host cores) on a bounded sample."""
     import e3data
@@ -181,23 +194,49 @@ def main():
     W = e3data.make_weights(cfg)
     model = api.DeviceModel(cfg, W, dev)
     n = args.inputs_per_gpu
-    first_id = rank * n
-    # synthetic inputs of the paper-shaped workload (seeded; one stream per id)
-    X = e3data.make_inputs(cfg, range(first_id, first_id + n))
-    x_host = torch.from_numpy(X).to(torch.bfloat16).pin_memory()
-    del X
-    x_dev = x_host.to(dev)
-    ids_dev = torch.arange(0, n, dtype=torch.int64, device=dev)   # local ids index the exit arrays
-    ids_host = torch.arange(0, n, dtype=torch.int64).pin_memory()
-    ex = api.ExitBuffers(n, cfg.classes, cfg.n_ramps, dev)
-    pipe = api.Pipeline(model, api.make_plan(cfg, bounds, tau, lag=1))
     stream = torch.cuda.Stream(dev)
+    stage_mode = args.mode == "stage" and world > 1
+    if stage_mode:
+        # stages on different GPUs: chunk c of the job enters at the stage-0
+        # replica owning it; ids are global so exits land at their input's slot
+        from paper_conf_sosp_iyergdpgn24_b200 import parallel as par
+        layout = par.plan_stages(cfg.ramp_layers, lambda l: survival(cfg, l), world,
+                                 n_stages=min(args.stages, world))
+        g_stage, _ = layout.stage_of(rank)
+        total = n * world
+        n_chunks = (total + args.chunk - 1) // args.chunk
+        mine = [c for c in range(n_chunks) if layout.owner(0, c) == rank] if g_stage == 0 else []
+        chunk_ids = {c: range(c * args.chunk, min(total, (c + 1) * args.chunk)) for c in mine}
+        chunk_x = {c: torch.from_numpy(e3data.make_inputs(cfg, r)).to(torch.bfloat16).to(dev)
+                   for c, r in chunk_ids.items()}
+        chunk_id_t = {c: torch.tensor(list(r), dtype=torch.int64, device=dev) for c, r in chunk_ids.items()}
+        ex = api.ExitBuffers(total, cfg.classes, cfg.n_ramps, dev)
+        executor = par.GpuStageExecutor(model, cfg, layout.bounds[g_stage], layout.bounds[g_stage + 1], tau, ex,
+                                        args.chunk)
+        transport = par.Transport(device=True)
+        plan_name = f"stages {list(layout.bounds)} replicas {list(layout.replicas)} (per-ramp splits inside)"
+    else:
+        first_id = rank * n
+        # synthetic inputs of the paper-shaped workload (seeded; one stream per id)
+        X = e3data.make_inputs(cfg, range(first_id, first_id + n))
+        x_host = torch.from_numpy(X).to(torch.bfloat16).pin_memory()
+        del X
+        x_dev = x_host.to(dev)
+        ids_dev = torch.arange(0, n, dtype=torch.int64, device=dev)   # local ids index the exit arrays
+        ids_host = torch.arange(0, n, dtype=torch.int64).pin_memory()
+        ex = api.ExitBuffers(n, cfg.classes, cfg.n_ramps, dev)
+        pipe = api.Pipeline(model, api.make_plan(cfg, bounds, tau, lag=1))
 
     def barrier():
         if world > 1:
             dist.barrier()
 
     def step(host=False, res=None):
+        if stage_mode:
+            with torch.cuda.stream(stream):
+                par.run_stage_pipeline(executor, layout, rank, n_chunks, lambda c: (chunk_x[c], chunk_id_t[c]),
+                                       (cfg.seq, cfg.hidden), torch.bfloat16, dev, transport)
+            return None
         with torch.cuda.stream(stream):
             st = pipe.run(x_host if host else x_dev, ids_host if host else ids_dev, ex, stream=stream)
             if res is not None:   # D2H read of the step's result (exit records)
@@ -239,17 +278,19 @@ def main():
     value = total_inputs / (ms / 1000.0)
 
     # exit histogram + invariants of the last step
+    if stage_mode:
+        par.reduce_exits(ex)
     el = ex.exit_layer.cpu().numpy()
     assert (el >= 0).all(), "an input did not exit"
-    hist = (np.bincount(el, minlength=cfg.layers) / n).round(4).tolist()
+    hist = (np.bincount(el, minlength=cfg.layers) / len(el)).round(4).tolist()
     splits = len(bounds) - 1
-    valid = [int(stats.valid_rows[s]) for s in range(splits)]
-    padded = [int(stats.padded_rows[s]) for s in range(splits)]
-    batches = [int(stats.batches[s]) for s in range(splits)]
+    valid = [int(stats.valid_rows[s]) for s in range(splits)] if stats else None
+    padded = [int(stats.padded_rows[s]) for s in range(splits)] if stats else None
+    batches = [int(stats.batches[s]) for s in range(splits)] if stats else None
 
     # e2e: host-pinned inputs through the same C-ABI call, results read back
     e2e = None
-    if not args.no_e2e:
+    if not args.no_e2e and not stage_mode:
         res = (torch.empty(n, dtype=torch.int32).pin_memory(), torch.empty(n, dtype=torch.int32).pin_memory(),
                torch.empty(n, dtype=torch.float32).pin_memory())
         step(host=True, res=res)
@@ -320,7 +361,8 @@ def main():
             "data": "synthetic (seeded random-init weights and N(0,1) embedded inputs, e3data)",
             "config": {"workload": cfg.name, "layers": cfg.layers, "hidden": cfg.hidden, "batch": cfg.batch,
                        "seq_len": cfg.seq, "ramps": cfg.n_ramps, "test": cfg.test, "plan": plan_name,
-                       "inputs_per_step_per_gpu": n, "parallelism": f"replica x{world}" if world > 1 else "1 GPU",
+                       "inputs_per_step_per_gpu": n,
+                       "parallelism": (f"stage x{world}" if stage_mode else f"replica x{world}") if world > 1 else "1 GPU",
                        "l2": "inputs larger than L2 (%.2f GB per step per GPU)" % (n * cfg.seq * cfg.hidden * 2 / 1e9)},
             "roofline": roof,
             "whole_path_roofline_frac": round(whole, 4),
@@ -331,7 +373,7 @@ def main():
             "clocks": clocks,
             "exit_hist": hist,
             "split_batches": batches, "split_valid_rows": valid, "split_padded_rows": padded,
-            "host_waits": int(stats.host_waits),
+            "host_waits": int(stats.host_waits) if stats else None,
         }
         print(json.dumps(out), flush=True)
     if world > 1:

@@ -228,6 +228,16 @@ e3_status e3_pipeline_destroy(e3_pipeline *pl);
  * queue is flushed padded to B. */
 e3_status e3_pipeline_run(e3_pipeline *pl, void *stream, const void *x, const int64_t *ids, int64_t n,
                           const e3_exits *ex, e3_stats *st);
+/* One STAGE of a multi-GPU stage pipeline: like e3_pipeline_run, for a plan
+ * whose last split does not hold the model's final ramp.  The survivors of
+ * that last split are appended in dispatch order (stable within each run) to
+ * x_out / id_out (device, capacity out_cap rows; E3_ECAPACITY beyond it) and
+ * *n_out (host) receives their number -- the rows the next stage's GPU must
+ * receive ("outputs are then directed to the machines
+ * hosting the next split"). */
+e3_status e3_pipeline_run_out(e3_pipeline *pl, void *stream, const void *x, const int64_t *ids, int64_t n,
+                              const e3_exits *ex, e3_stats *st, void *x_out, int64_t *id_out, int64_t out_cap,
+                              int64_t *n_out);
 /* Dispatch order of the last run (plan.trace = 1): per run its split, valid
  * count and the B ids (padding = -1) into ids_out[run * B ...]. */
 e3_status e3_pipeline_trace(e3_pipeline *pl, int32_t *split, int32_t *n_valid, int64_t *ids_out,

@@ -89,6 +89,8 @@ SIGNATURES = {
     "e3_pipeline_create": (I32, [C.POINTER(Plan), C.POINTER(Weights), C.c_int, C.POINTER(P)]),
     "e3_pipeline_destroy": (I32, [P]),
     "e3_pipeline_run": (I32, [P, P, P, P, I64, C.POINTER(Exits), C.POINTER(Stats)]),
+    "e3_pipeline_run_out": (I32, [P, P, P, P, I64, C.POINTER(Exits), C.POINTER(Stats), P, P, I64,
+                                  C.POINTER(I64)]),
     "e3_pipeline_trace": (I32, [P, P, P, P, I64, C.POINTER(I64)]),
     "e3_op_gemm": (I32, [P, P, I64, P, P, P, P, I32, I32, I32, I32]),
     "e3_op_attention": (I32, [P, P, P, I32, I32, I32, I32]),

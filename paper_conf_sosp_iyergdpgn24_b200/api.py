@@ -200,6 +200,17 @@ class Pipeline:
               "e3_pipeline_run")
         return st
 
+    def run_out(self, x, ids, exits: ExitBuffers, x_out, id_out, stream=None):
+        """Stage of a stage pipeline: survivors of the (non-final) last split are
+        appended to x_out / id_out; returns (stats, number of survivors)."""
+        st = _lib.Stats()
+        n_out = C.c_int64()
+        n = int(ids.shape[0])
+        check(lib.e3_pipeline_run_out(self.h, _stream(stream), _ptr(x) if n else None, _ptr(ids) if n else None,
+                                      n, C.byref(exits.c), C.byref(st), _ptr(x_out), _ptr(id_out),
+                                      int(id_out.shape[0]), C.byref(n_out)), "e3_pipeline_run_out")
+        return st, n_out.value
+
     def trace(self):
         n = C.c_int64()
         check(lib.e3_pipeline_trace(self.h, None, None, None, 0, C.byref(n)), "e3_pipeline_trace")

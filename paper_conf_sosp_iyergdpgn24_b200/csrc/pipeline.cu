@@ -62,6 +62,7 @@ struct e3_pipeline {
   uint8_t *staging = nullptr;         // [B, row] wrapped / flush pops
   int64_t *staging_ids = nullptr;
   uint8_t *sink = nullptr;            // [B, row] output of the last split (empty)
+  int64_t *out_tails = nullptr;       // device [2]: tail slots of the caller's output buffer
   int64_t *sink_ids = nullptr;
   volatile int *mailbox = nullptr;    // host-mapped [kSlots]
   int *mailbox_dev = nullptr;
@@ -88,6 +89,7 @@ struct e3_pipeline {
     cudaFree(staging);
     cudaFree(staging_ids);
     cudaFree(sink);
+    cudaFree(out_tails);
     cudaFree(sink_ids);
     cudaFree(in_rows);
     cudaFree(in_ids);
@@ -124,6 +126,12 @@ struct Runner {
   const uint8_t *x;
   const int64_t *ids;
   int64_t n;
+  // survivors of a non-final last split (stage pipeline): caller's buffer
+  uint8_t *out_rows = nullptr;
+  int64_t *out_ids = nullptr;
+  int64_t out_cap = 0;
+  int64_t out_pushes = 0;
+  int64_t out_known = 0;
   bool host_in;
   int64_t cursor = 0;      // inputs dispatched
   int64_t staged = 0;      // host inputs issued to the copy stream (batches)
@@ -148,6 +156,7 @@ struct Runner {
       return E3_ECAPACITY;
     }
     if (p.split + 1 < pl->plan.n_splits) pl->q[p.split + 1].known += c;
+    else out_known += c;
     prof_add_bytes(PK_COMPACT, 2.0 * c * pl->row_bytes);   // read + write of the survivors
     if (stats) stats->rows_out[p.split] += c;
     return E3_OK;
@@ -235,6 +244,13 @@ struct Runner {
       dst.tail_out = N.tails + ((N.pushes + 1) & 1);
       ++N.pushes;
       dst.head = N.head;
+    } else if (out_rows) {
+      dst.rows = out_rows;
+      dst.ids = out_ids;
+      dst.cap = out_cap;
+      dst.tail_dev = pl->out_tails + (out_pushes & 1);
+      dst.tail_out = pl->out_tails + ((out_pushes + 1) & 1);
+      ++out_pushes;
     } else {
       dst.rows = pl->sink;
       dst.ids = pl->sink_ids;
@@ -323,7 +339,7 @@ e3_status e3_pipeline_create(const e3_plan *p, const e3_weights *w, int device, 
                      d.heads == d0.heads && d.arch == d0.arch,
                  "splits differ in model dims or batch");
     E3_CHECK_ARG(s == 0 || d.layer_begin == p->split[s - 1].layer_end, "splits not contiguous");
-    E3_CHECK_ARG((s == p->n_splits - 1) == (d.final_ramp != 0), "only the last split may (and must) hold the final ramp");
+    E3_CHECK_ARG(s == p->n_splits - 1 || d.final_ramp == 0, "only the last split may hold the final ramp");
   }
   for (int s = 0; s < p->n_splits; ++s) {
     e3_status r = split_validate(&p->split[s], w);
@@ -370,6 +386,7 @@ e3_status e3_pipeline_create(const e3_plan *p, const e3_weights *w, int device, 
   if (e == cudaSuccess) e = cudaMalloc(&pl->staging, (size_t)pl->B * pl->row_bytes);
   if (e == cudaSuccess) e = cudaMalloc(&pl->staging_ids, (size_t)pl->B * 8);
   if (e == cudaSuccess) e = cudaMalloc(&pl->sink, (size_t)pl->B * pl->row_bytes);
+  if (e == cudaSuccess) e = cudaMalloc(&pl->out_tails, 2 * sizeof(int64_t));
   if (e == cudaSuccess) e = cudaMalloc(&pl->sink_ids, (size_t)pl->B * 8);
   if (e == cudaSuccess) e = cudaMalloc(&pl->in_rows, (size_t)kInSlots * pl->B * pl->row_bytes);
   if (e == cudaSuccess) e = cudaMalloc(&pl->in_ids, (size_t)kInSlots * pl->B * 8);
@@ -395,8 +412,9 @@ e3_status e3_pipeline_destroy(e3_pipeline *pl) {
   return E3_OK;
 }
 
-e3_status e3_pipeline_run(e3_pipeline *pl, void *stream, const void *x, const int64_t *ids, int64_t n,
-                          const e3_exits *ex, e3_stats *st) {
+static e3_status pipeline_run_impl(e3_pipeline *pl, void *stream, const void *x, const int64_t *ids, int64_t n,
+                                   const e3_exits *ex, e3_stats *st, void *x_out, int64_t *id_out, int64_t out_cap,
+                                   int64_t *n_out) {
   E3_CHECK_ARG(pl, "null pipeline");
   if (pl->poisoned) {
     set_error("pipeline poisoned by an earlier failure");
@@ -422,6 +440,17 @@ e3_status e3_pipeline_run(e3_pipeline *pl, void *stream, const void *x, const in
     return E3_EINVAL;
   }
   R.host_in = n > 0 && !xd;
+  const bool final_last = pl->plan.split[pl->plan.n_splits - 1].final_ramp != 0;
+  if (!final_last && !x_out) {
+    set_error("the plan's last split is not final: use e3_pipeline_run_out");
+    return E3_EINVAL;
+  }
+  if (!final_last) {
+    R.out_rows = reinterpret_cast<uint8_t *>(x_out);
+    R.out_ids = id_out;
+    R.out_cap = out_cap;
+    E3_CUDA_TRY(cudaMemsetAsync(pl->out_tails, 0, 2 * sizeof(int64_t), R.st));
+  }
   pl->tr_split.clear();
   pl->tr_nvalid.clear();
   pl->tr_ids.clear();
@@ -447,9 +476,27 @@ e3_status e3_pipeline_run(e3_pipeline *pl, void *stream, const void *x, const in
     }
   }
   if (r == E3_ECUDA || r == E3_ECAPACITY) pl->poisoned = true;
+  if (n_out) *n_out = R.out_known;
   cudaSetDevice(prev);
   return r;
 }
+
+e3_status e3_pipeline_run(e3_pipeline *pl, void *stream, const void *x, const int64_t *ids, int64_t n,
+                          const e3_exits *ex, e3_stats *st) {
+  return pipeline_run_impl(pl, stream, x, ids, n, ex, st, nullptr, nullptr, 0, nullptr);
+}
+
+e3_status e3_pipeline_run_out(e3_pipeline *pl, void *stream, const void *x, const int64_t *ids, int64_t n,
+                              const e3_exits *ex, e3_stats *st, void *x_out, int64_t *id_out, int64_t out_cap,
+                              int64_t *n_out) {
+  E3_CHECK_ARG(pl && x_out && id_out && n_out && out_cap >= 0, "bad output buffer");
+  E3_CHECK_ARG(pl->plan.split[pl->plan.n_splits - 1].final_ramp == 0,
+               "e3_pipeline_run_out needs a plan whose last split is not final");
+  E3_CHECK_ARG(((reinterpret_cast<uintptr_t>(x_out)) & 15) == 0, "x_out must be 16-byte aligned");
+  return pipeline_run_impl(pl, stream, x, ids, n, ex, st, x_out, id_out, out_cap, n_out);
+}
+
+
 
 e3_status e3_pipeline_trace(e3_pipeline *pl, int32_t *split, int32_t *n_valid, int64_t *ids_out, int64_t max_runs,
                             int64_t *n_runs) {

@@ -165,6 +165,44 @@ def test_pipeline_host_inputs_and_edge_sizes(api, tiny):
             assert sum(st.valid_rows[s] for s in range(2)) == N + int((ex.exit_layer[:N] > 1).sum())
 
 
+def test_pipeline_run_out_two_stages_equal_single_pipeline(api, tiny):
+    """Stage pipeline on one GPU: stage 0 = layers [0,2) (e3_pipeline_run_out),
+    its survivors -> stage 1 = layers [2,4).  Per input the result is bitwise
+    the single-pipeline result (rows are independent, inner EXACT), the
+    survivors come out in input order, and a too-small output is an error."""
+    cfg, W, model = tiny
+    N = 150
+    X = bf16_tensor(e3data.make_inputs(cfg, range(N), seed=11))
+    ids = torch.arange(N, dtype=torch.int64, device=DEV)
+    ref = api.ExitBuffers(N, cfg.classes, cfg.n_ramps, DEV)
+    api.Pipeline(model, api.make_plan(cfg, (0, 2, 4), cfg.tau)).run(X, ids, ref)
+    ex = api.ExitBuffers(N, cfg.classes, cfg.n_ramps, DEV)
+    s0 = api.Pipeline(model, api.make_plan(cfg, (0, 2), cfg.tau))
+    s1 = api.Pipeline(model, api.make_plan(cfg, (2, 4), cfg.tau))
+    x_out = torch.empty_like(X)
+    id_out = torch.full((N,), -9, dtype=torch.int64, device=DEV)
+    st, n_out = s0.run_out(X, ids, ex, x_out, id_out)
+    torch.cuda.synchronize()
+    exp = torch.nonzero(ref.exit_layer > 1).flatten()
+    assert n_out == exp.numel() and torch.equal(id_out[:n_out], exp)
+    assert torch.all(id_out[n_out:] == -9)
+    assert int(ex.n_exit.item()) == N - n_out
+    s1.run(x_out[:n_out], id_out[:n_out], ex)
+    assert torch.equal(ex.exit_layer.cpu(), ref.exit_layer.cpu())
+    assert torch.equal(ex.label.cpu(), ref.label.cpu())
+    assert torch.equal(ex.logits.cpu(), ref.logits.cpu())
+    # survivors beyond the caller's capacity: reported, never truncated silently
+    from paper_conf_sosp_iyergdpgn24_b200._lib import E3Error
+    small = api.Pipeline(model, api.make_plan(cfg, (0, 2), cfg.tau))
+    with pytest.raises(E3Error):
+        small.run_out(X, ids, api.ExitBuffers(N, cfg.classes, cfg.n_ramps, DEV), x_out[:4], id_out[:4])
+    # the final split cannot be driven through run_out, nor a non-final one through run
+    with pytest.raises(E3Error):
+        s1.run_out(X, ids, ex, x_out, id_out)
+    with pytest.raises(E3Error):
+        s0.run(X, ids, ex)
+
+
 def test_rebatch_fifo_and_flush(api):
     B, row = 8, 64
     q = api.Queue(DEV, row * 2, 4 * B)
