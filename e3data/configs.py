@@ -67,6 +67,14 @@ TINY = ModelConfig(
     tau=(0.9, 0.9),
 )
 
+# ViT-shaped tiny case: pre-LN layers, LN + linear ramp over 10 classes, a
+# token count (37) that leaves a ragged tail in every 128-row tile
+TINY_VIT = ModelConfig(
+    name="tiny-vit", arch="vit", layers=4, hidden=128, heads=2, ffn=512, seq=37,
+    classes=10, norm_eps=1e-6, ramp_layers=(1, 3), batch=32, test="maxprob",
+    tau=(0.77, 0.77),
+)
+
 BERT_BASE = ModelConfig(
     name="ee-bert-base", arch="bert", layers=12, hidden=768, heads=12, ffn=3072,
     seq=128, classes=2, norm_eps=1e-12, ramp_layers=tuple(range(12)), batch=64,
@@ -94,8 +102,8 @@ LLAMA_7B = ModelConfig(
     kv_heads=32, ctx=512,
 )
 
-CONFIGS = {c.name: c for c in (TINY, BERT_BASE, BERT_LARGE, VIT_BASE, LLAMA_7B)}
-ALIASES = {"t": "tiny", "bb": "ee-bert-base", "bl": "ee-bert-large",
+CONFIGS = {c.name: c for c in (TINY, TINY_VIT, BERT_BASE, BERT_LARGE, VIT_BASE, LLAMA_7B)}
+ALIASES = {"t": "tiny", "tv": "tiny-vit", "bb": "ee-bert-base", "bl": "ee-bert-large",
            "vt": "ee-vit-b16", "lm": "ee-llama-7b-decode"}
 
 

@@ -182,7 +182,7 @@ __global__ void fill_kernel(int32_t *dst, int v) { *dst = v; }
 // alternate per push, chosen by the host.
 constexpr int kRowsInFlight = 4;
 
-template <int VPL>
+template <int VPL, bool kLn>
 __global__ void __launch_bounds__(kThreads)
     ln_compact_kernel(const __nv_bfloat16 *__restrict__ y, const int64_t *__restrict__ id,
                       const uint8_t *__restrict__ alive, int B, int S, int H, const __nv_bfloat16 *__restrict__ g,
@@ -191,7 +191,7 @@ __global__ void __launch_bounds__(kThreads)
   __shared__ int word_cnt[kMaxB / 32 + 1];
   const int warp = warp_id(), lane = lane_id();
   LnParams<VPL> p;
-  ln_load_params<VPL>(p, g, bb, H, lane);   // weights: before the dependency wait
+  if (kLn) ln_load_params<VPL>(p, g, bb, H, lane);   // weights: before the dependency wait
   pdl_wait();
   pdl_trigger();
   const int64_t tail = dst.tail_dev ? *dst.tail_dev : 0;
@@ -225,7 +225,7 @@ __global__ void __launch_bounds__(kThreads)
       const int u = u0 + j * stride;
       if (u < units) {
         const int k = u / S, t = u - k * S;
-        ln_apply<VPL>(v[j], p, H, eps, lane);
+        if (kLn) ln_apply<VPL>(v[j], p, H, eps, lane);
         ln_store_row<VPL>(v[j], ring + ((tail + k) % dst.cap) * row_elems + (size_t)t * H, H, lane);
       }
     }
@@ -251,9 +251,15 @@ e3_status ln_compact_run(const void *y, const int64_t *id, const uint8_t *alive,
   auto *gp = reinterpret_cast<const __nv_bfloat16 *>(g);
   auto *bp = reinterpret_cast<const __nv_bfloat16 *>(b);
   const int vpl = (H / 8 + 31) / 32;
-#define E3_LNC(V) \
-  E3_CUDA_TRY(launch_k(ln_compact_kernel<V>, dim3((unsigned)grid), dim3(kThreads), 0, st, yp, id, alive, B, S, H, \
-                       gp, bp, eps, dst, n_surv_dev))
+#define E3_LNC(V)                                                                                          \
+  do {                                                                                                     \
+    if (gp)                                                                                                \
+      E3_CUDA_TRY(launch_k(ln_compact_kernel<V, true>, dim3((unsigned)grid), dim3(kThreads), 0, st, yp, id, \
+                           alive, B, S, H, gp, bp, eps, dst, n_surv_dev));                                 \
+    else                                                                                                   \
+      E3_CUDA_TRY(launch_k(ln_compact_kernel<V, false>, dim3((unsigned)grid), dim3(kThreads), 0, st, yp,   \
+                           id, alive, B, S, H, gp, bp, eps, dst, n_surv_dev));                             \
+  } while (0)
   if (vpl <= 1) E3_LNC(1);
   else if (vpl <= 3) E3_LNC(3);
   else if (vpl <= 4) E3_LNC(4);

@@ -76,7 +76,8 @@ e3_status compact_run(const void *x, const int64_t *id, const uint8_t *alive, in
                       const RingDst &dst, int32_t *n_surv_dev, unsigned *done_ctr, int sms, cudaStream_t st);
 
 // fused LN2 + compaction: survivors of the PRE-LN rows y [B,S,H] are
-// LayerNorm-ed (g, b, eps) and written to dst
+// LayerNorm-ed (g, b, eps) and written to dst; g == NULL: copied unchanged
+// (pre-LN ViT, whose layer output needs no normalisation)
 e3_status ln_compact_run(const void *y, const int64_t *id, const uint8_t *alive, int B, int S, int H, const void *g,
                          const void *b, float eps, const RingDst &dst, int32_t *n_surv_dev, int sms,
                          cudaStream_t st);

@@ -28,6 +28,8 @@
 //            argmax (lowest index on ties), threshold test, exit record by
 //            input id and the alive flag.
 // All ramp math is fp32, never rounded to bf16 (rounding contract).
+// The ViT ramp (LayerNorm + linear over C <= 2048 classes) is ramp_vit_kernel
+// below.
 #include "common.cuh"
 #include "kernels.h"
 #include "ln_row.cuh"
@@ -283,11 +285,272 @@ __global__ void ramp_bert_kernel(RampArgs a, int CS) {
   }
 }
 
+// ============================================================== ViT ramp
+// ViT exit ramp (R1): n = LN_r(x[b, 0, :]) (the ramp's own
+// LayerNorm), z = W_c n + b_c over C classes (C = 1000 for EE-ViT-B/16).  All
+// fp32: the normalised row is never rounded (rounding contract), so the
+// classifier runs on the FMA pipe (B x H x C = 197 MFMA per call at VT; a few
+// microseconds spread over the grid).
+//
+// grid (CS, ceil(B / 16)), clusters of CS = ceil(C / CB) CTAs: CTA rank r owns
+// classes [r*CB, (r+1)*CB) of one group of 16 rows.  Thread t owns the class
+// pair 2j, 2j+1 (j = t mod CB/2) for the 4 rows of row group t / (CB/2); every
+// lane of a warp reads the same normalised row values (smem broadcast) and its
+// own two classifier rows (16-byte loads).  Per row and CTA the softmax
+// statistics are reduced to (max m, argmax, s = sum e^(z-m), u = sum
+// e^(z-m)(z-m)) and sent to rank 0 through DSMEM; rank 0 merges the CS
+// partials in rank order (exact merge of log-sum-exp partials), tests the
+// threshold, writes the record and the alive flag, and publishes the decision;
+// each CTA then writes its slice of the logits of the exiting rows.
+constexpr int kVitRows = 16;
+
+__device__ __forceinline__ int ld_cluster_s32(uint32_t addr) {
+  int v;
+  asm volatile("ld.shared::cluster.s32 %0, [%1];" : "=r"(v) : "r"(addr) : "memory");
+  return v;
+}
+
+struct SoftStat {
+  float m, s, u;
+  int idx;
+};
+
+// merge b into a (a covers lower class indices on ties when merged in order)
+__device__ __forceinline__ SoftStat soft_merge(SoftStat a, SoftStat b) {
+  if (b.idx < 0) return a;
+  if (a.idx < 0) return b;
+  const float M = fmaxf(a.m, b.m);
+  const float ea = expf(a.m - M), eb = expf(b.m - M);
+  SoftStat r;
+  r.m = M;
+  r.s = a.s * ea + b.s * eb;
+  r.u = ea * (a.u + a.s * (a.m - M)) + eb * (b.u + b.s * (b.m - M));
+  r.idx = (b.m > a.m || (b.m == a.m && b.idx < a.idx)) ? b.idx : a.idx;
+  return r;
+}
+
+template <int CB>
+__global__ void __launch_bounds__(2 * CB) ramp_vit_kernel(RampArgs a, int CS) {
+  constexpr int kThreads = 2 * CB, kWarps = kThreads / 32, kWarpsPerRg = CB / 64;
+  extern __shared__ float sN[];                       // [16][H + 4] normalised CLS rows (fp32)
+  __shared__ SoftStat sRed[kWarps][4];
+  __shared__ SoftStat sQ[16][kVitRows];               // rank 0: [rank][row]
+  __shared__ int sDec[kVitRows];                      // rank 0: 1 = row exits here
+  __shared__ bool row_ok[kVitRows];
+  const int H = a.H, P = H + 4, C = a.C;
+  const int t = threadIdx.x, warp = t >> 5, lane = t & 31;
+  const uint32_t rank = cluster_ctarank();
+  const int b0 = blockIdx.y * kVitRows;
+  const int j = t % (CB / 2), rg = t / (CB / 2);
+  const int c0 = (int)rank * CB + 2 * j, c1 = c0 + 1;
+  const __nv_bfloat16 *W = reinterpret_cast<const __nv_bfloat16 *>(a.w.w_c);
+  const __nv_bfloat16 *bc = reinterpret_cast<const __nv_bfloat16 *>(a.w.b_c);
+  const float bias0 = c0 < C ? bf2f(bc[c0]) : 0.f, bias1 = c1 < C ? bf2f(bc[c1]) : 0.f;
+
+  pdl_wait();
+  pdl_trigger();
+  const int n_valid = a.n_valid_dev ? *a.n_valid_dev : a.n_valid_host;
+  if (t < kVitRows) row_ok[t] = row_alive(a, b0 + t, n_valid);
+  __syncthreads();
+
+  // ---- LayerNorm of the CLS rows (two passes, fp32), one warp per row
+  const __nv_bfloat16 *x = reinterpret_cast<const __nv_bfloat16 *>(a.x);
+  const __nv_bfloat16 *lg = reinterpret_cast<const __nv_bfloat16 *>(a.w.ln_g);
+  const __nv_bfloat16 *lb = reinterpret_cast<const __nv_bfloat16 *>(a.w.ln_b);
+  for (int r = warp; r < kVitRows; r += kWarps) {
+    float *row = sN + r * P;
+    if (!row_ok[r]) {
+      for (int k = lane; k < H; k += 32) row[k] = 0.f;
+      continue;
+    }
+    const __nv_bfloat16 *xr = x + (size_t)(b0 + r) * a.S * H;
+    float s = 0.f;
+    for (int k = lane; k < H; k += 32) {
+      const float v = bf2f(xr[k]);
+      row[k] = v;
+      s += v;
+    }
+#pragma unroll
+    for (int o = 16; o; o >>= 1) s += __shfl_xor_sync(0xffffffffu, s, o);
+    const float mean = s / (float)H;
+    float q = 0.f;
+    for (int k = lane; k < H; k += 32) {
+      const float d = row[k] - mean;
+      q += d * d;
+    }
+#pragma unroll
+    for (int o = 16; o; o >>= 1) q += __shfl_xor_sync(0xffffffffu, q, o);
+    const float rstd = 1.0f / sqrtf(q / (float)H + a.eps);
+    for (int k = lane; k < H; k += 32) row[k] = (row[k] - mean) * rstd * bf2f(lg[k]) + bf2f(lb[k]);
+  }
+  __syncthreads();
+
+  // ---- classifier: 4 rows x 2 classes per thread, fp32 FMA over K = H
+  float acc[4][2] = {};
+  {
+    const uint4 *w0 = reinterpret_cast<const uint4 *>(W + (size_t)(c0 < C ? c0 : 0) * H);
+    const uint4 *w1 = reinterpret_cast<const uint4 *>(W + (size_t)(c1 < C ? c1 : 0) * H);
+    const bool v0 = c0 < C, v1 = c1 < C;
+    const float *rows = sN + rg * 4 * P;
+#pragma unroll 2
+    for (int k = 0; k < H; k += 8) {
+      const uint4 wa = v0 ? __ldg(w0 + k / 8) : make_uint4(0, 0, 0, 0);
+      const uint4 wb = v1 ? __ldg(w1 + k / 8) : make_uint4(0, 0, 0, 0);
+      const float fa[8] = {bf_lo(wa.x), bf_hi(wa.x), bf_lo(wa.y), bf_hi(wa.y),
+                           bf_lo(wa.z), bf_hi(wa.z), bf_lo(wa.w), bf_hi(wa.w)};
+      const float fb[8] = {bf_lo(wb.x), bf_hi(wb.x), bf_lo(wb.y), bf_hi(wb.y),
+                           bf_lo(wb.z), bf_hi(wb.z), bf_lo(wb.w), bf_hi(wb.w)};
+#pragma unroll
+      for (int rr = 0; rr < 4; ++rr) {
+        const float4 n0 = *reinterpret_cast<const float4 *>(rows + rr * P + k);
+        const float4 n1 = *reinterpret_cast<const float4 *>(rows + rr * P + k + 4);
+        const float nv[8] = {n0.x, n0.y, n0.z, n0.w, n1.x, n1.y, n1.z, n1.w};
+#pragma unroll
+        for (int e = 0; e < 8; ++e) {
+          acc[rr][0] = fmaf(nv[e], fa[e], acc[rr][0]);
+          acc[rr][1] = fmaf(nv[e], fb[e], acc[rr][1]);
+        }
+      }
+    }
+  }
+  float z[4][2];
+#pragma unroll
+  for (int rr = 0; rr < 4; ++rr) {
+    z[rr][0] = acc[rr][0] + bias0;
+    z[rr][1] = acc[rr][1] + bias1;
+  }
+
+  // ---- per-row softmax statistics of this CTA's classes
+#pragma unroll
+  for (int rr = 0; rr < 4; ++rr) {
+    SoftStat st{-INFINITY, 0.f, 0.f, -1};
+    if (c0 < C) st = SoftStat{z[rr][0], 1.f, 0.f, c0};
+    if (c1 < C) st = soft_merge(st, SoftStat{z[rr][1], 1.f, 0.f, c1});
+#pragma unroll
+    for (int o = 16; o; o >>= 1) {
+      SoftStat ot;
+      ot.m = __shfl_xor_sync(0xffffffffu, st.m, o);
+      ot.s = __shfl_xor_sync(0xffffffffu, st.s, o);
+      ot.u = __shfl_xor_sync(0xffffffffu, st.u, o);
+      ot.idx = __shfl_xor_sync(0xffffffffu, st.idx, o);
+      st = soft_merge(st, ot);
+    }
+    if (lane == 0) sRed[warp][rr] = st;
+  }
+  __syncthreads();
+  if (t < kVitRows) {                        // row t: merge this CTA's warps, send to rank 0
+    const int g = t / 4, rr = t % 4;
+    SoftStat st = sRed[g * kWarpsPerRg][rr];
+    for (int w = 1; w < kWarpsPerRg; ++w) st = soft_merge(st, sRed[g * kWarpsPerRg + w][rr]);
+    const uint32_t dst = mapa_shared(smem_u32(&sQ[rank][t]), 0);
+    st_cluster_f32(dst, st.m);
+    st_cluster_f32(dst + 4, st.s);
+    st_cluster_f32(dst + 8, st.u);
+    asm volatile("st.shared::cluster.s32 [%0], %1;" ::"r"(dst + 12), "r"(st.idx) : "memory");
+  }
+  cluster_sync();
+
+  // ---- rank 0 decides (rows t < 16 of warp 0)
+  if (rank == 0 && warp == 0) {
+    const int r = lane, b = b0 + r;
+    bool exit_now = false;
+    if (r < kVitRows && b < a.B) {
+      if (!row_ok[r]) {
+        if (a.init_alive) a.alive[b] = 0;
+      } else {
+        SoftStat st = sQ[0][r];
+        for (int q = 1; q < CS; ++q) st = soft_merge(st, sQ[q][r]);
+        float metric;
+        bool pass;
+        if (a.test == E3_TEST_MAXPROB) {
+          metric = 1.0f / st.s;
+          pass = metric > a.tau;
+        } else {
+          metric = logf(st.s) - st.u / st.s;
+          pass = metric < a.tau;
+        }
+        exit_now = pass || a.final_ramp;
+        const int64_t id = a.id[b];
+        if (exit_now && id >= 0 && id < a.ex.capacity) {
+          if (a.ex.exit_layer) a.ex.exit_layer[id] = a.layer;
+          if (a.ex.label) a.ex.label[id] = st.idx;
+          if (a.ex.conf) a.ex.conf[id] = metric;
+        }
+        a.alive[b] = exit_now ? 0 : 1;
+      }
+    }
+    if (r < kVitRows) sDec[r] = exit_now ? 1 : 0;
+    const int n_ex = __popc(__ballot_sync(0xffffffffu, exit_now));
+    if (lane == 0 && n_ex) {
+      if (a.ex.n_exit) atomicAdd(a.ex.n_exit, n_ex);
+      if (a.ex.ramp_count) atomicAdd(a.ex.ramp_count + a.ramp_index, n_ex);
+    }
+  }
+  cluster_sync();
+  // ---- logits of the exiting rows: each CTA writes its class slice
+  if (a.ex.logits) {
+#pragma unroll
+    for (int rr = 0; rr < 4; ++rr) {
+      const int r = rg * 4 + rr, b = b0 + r;
+      if (b >= a.B) continue;
+      if (!ld_cluster_s32(mapa_shared(smem_u32(&sDec[r]), 0))) continue;
+      const int64_t id = a.id[b];
+      if (id < 0 || id >= a.ex.capacity) continue;
+      if (c0 < C) a.ex.logits[id * C + c0] = z[rr][0];
+      if (c1 < C) a.ex.logits[id * C + c1] = z[rr][1];
+    }
+  }
+  cluster_sync();                            // rank 0's smem stays valid until every CTA has read it
+}
+
+e3_status ramp_vit_run(const RampArgs &a, cudaStream_t st) {
+  if (a.C < 1 || a.C > 16 * 128 || a.H % 8 || a.H > 3072 || !a.w.ln_g || !a.w.ln_b) {
+    set_error("ViT ramp: need 1 <= C <= 2048, H % 8 == 0, H <= 3072 and ramp LayerNorm weights");
+    return E3_EUNSUPPORTED;
+  }
+  const int CB = (a.C <= 16 * 64) ? 64 : 128;
+  const int CS = (a.C + CB - 1) / CB;
+  const int smem = kVitRows * (a.H + 4) * 4;
+  cudaLaunchConfig_t cfg = {};
+  cfg.gridDim = dim3(CS, (a.B + kVitRows - 1) / kVitRows);
+  cfg.blockDim = dim3(2 * CB);
+  cfg.dynamicSmemBytes = smem;
+  cfg.stream = st;
+  cudaLaunchAttribute attr[2];
+  attr[0].id = cudaLaunchAttributeClusterDimension;
+  attr[0].val.clusterDim.x = CS;
+  attr[0].val.clusterDim.y = 1;
+  attr[0].val.clusterDim.z = 1;
+  attr[1].id = cudaLaunchAttributeProgrammaticStreamSerialization;
+  attr[1].val.programmaticStreamSerializationAllowed = 1;
+  cfg.attrs = attr;
+  cfg.numAttrs = pdl_enabled() ? 2 : 1;
+#define E3_VRAMP(V)                                                                                        \
+  do {                                                                                                     \
+    static bool attr_done = false;                                                                         \
+    if (!attr_done) {                                                                                      \
+      E3_CUDA_TRY(cudaFuncSetAttribute(ramp_vit_kernel<V>, cudaFuncAttributeMaxDynamicSharedMemorySize,   \
+                                       kVitRows * (3072 + 4) * 4));                                        \
+      E3_CUDA_TRY(cudaFuncSetAttribute(ramp_vit_kernel<V>, cudaFuncAttributeNonPortableClusterSizeAllowed, \
+                                       1));                                                                \
+      attr_done = true;                                                                                    \
+    }                                                                                                      \
+    E3_CUDA_TRY(cudaLaunchKernelEx(&cfg, ramp_vit_kernel<V>, a, CS));                                      \
+  } while (0)
+  if (CB == 64) E3_VRAMP(64);
+  else E3_VRAMP(128);
+#undef E3_VRAMP
+  E3_CUDA_TRY(cudaGetLastError());
+  count_launch();
+  return E3_OK;
+}
+
 }  // namespace
 
 e3_status ramp_run(const RampArgs &a, cudaStream_t st) {
+  if (a.arch == E3_ARCH_VIT) return ramp_vit_run(a, st);
   if (a.arch != E3_ARCH_BERT) {
-    set_error("ramp: only the BERT (pooler) ramp is implemented");
+    set_error("ramp: arch not implemented");
     return E3_EUNSUPPORTED;
   }
   int CS = 8;

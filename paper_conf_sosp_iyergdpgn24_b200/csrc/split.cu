@@ -62,19 +62,20 @@ static bool aligned16(const void *p) { return (reinterpret_cast<uintptr_t>(p) & 
 
 e3_status split_validate(const e3_split_desc *d, const e3_weights *w) {
   E3_CHECK_ARG(d && w, "null descriptor or weights");
-  if (d->arch != E3_ARCH_BERT) {
-    set_error("e3_split_create: only arch BERT is implemented on the GPU path");
+  if (d->arch != E3_ARCH_BERT && d->arch != E3_ARCH_VIT) {
+    set_error("e3_split_create: arch not implemented on the GPU path (BERT, VIT)");
     return E3_EUNSUPPORTED;
   }
+  const bool vit = d->arch == E3_ARCH_VIT;
   if (d->dtype != E3_DTYPE_BF16) {
     set_error("e3_split_create: only dtype BF16 is implemented");
     return E3_EUNSUPPORTED;
   }
   E3_CHECK_ARG(d->hidden > 0 && d->heads > 0 && d->ffn > 0 && d->seq_len > 0 && d->batch > 0, "non-positive dims");
   if (d->hidden % 128 || d->hidden / d->heads != 64 || d->hidden % d->heads || d->ffn % 128 || d->seq_len > 256 ||
-      d->batch > 4096 || d->num_labels < 1 || d->num_labels > 16 || d->hidden > 4096) {
+      d->batch > 4096 || d->num_labels < 1 || d->num_labels > (vit ? 2048 : 16) || d->hidden > 4096) {
     set_error("e3_split_create: unsupported shape (need H % 128 == 0, head_dim 64, F % 128 == 0, S <= 256, "
-              "B <= 4096, 1 <= C <= 16, H <= 4096)");
+              "B <= 4096, 1 <= C <= 16 (BERT) or 2048 (VIT), H <= 4096)");
     return E3_EUNSUPPORTED;
   }
   E3_CHECK_ARG(d->layer_begin >= 0 && d->layer_end > d->layer_begin && d->layer_end <= w->n_layers,
@@ -95,7 +96,10 @@ e3_status split_validate(const e3_split_desc *d, const e3_weights *w) {
   }
   for (int r = 0; r < d->n_ramps; ++r) {
     const e3_ramp_weights &R = w->ramp[d->ramp_index[r]];
-    E3_CHECK_ARG(R.w_p && R.b_p && R.w_c && R.b_c && aligned16(R.w_p), "ramp weight pointer null / misaligned");
+    if (vit)
+      E3_CHECK_ARG(R.ln_g && R.ln_b && R.w_c && R.b_c && aligned16(R.w_c), "ViT ramp weight pointer null / misaligned");
+    else
+      E3_CHECK_ARG(R.w_p && R.b_p && R.w_c && R.b_c && aligned16(R.w_p), "ramp weight pointer null / misaligned");
   }
   return E3_OK;
 }
@@ -148,13 +152,21 @@ e3_status split_create_shared(const e3_split_desc *d, const e3_weights *w, int d
   s->bn_f2 = gemm_pick_bn(M, H, s->sms);
   const int nl = d->layer_end - d->layer_begin;
   s->maps.resize(nl);
+  const bool vit = d->arch == E3_ARCH_VIT;
   for (int i = 0; i < nl && st == E3_OK; ++i) {
     auto &m = s->maps[i];
     const void *prev = (i % 2 == 1) ? ws->xa : ws->xb;   // output of layer i-1
-    if (i > 0) st = gemm_tmaps(&m.qkv, prev, H, s->L[i].w_qkv, ws->qkv, M, 3 * H, H, s->bn_qkv);
+    void *out = (i % 2 == 0) ? ws->xa : ws->xb;          // output of layer i
+    if (vit) {
+      // pre-LN: QKV and FFN1 read the LayerNorm output in x1; FFN2 writes the
+      // layer output (x1 + MLP) to the ping-pong buffer
+      st = gemm_tmaps(&m.qkv, ws->x1, H, s->L[i].w_qkv, ws->qkv, M, 3 * H, H, s->bn_qkv);
+    } else if (i > 0) {
+      st = gemm_tmaps(&m.qkv, prev, H, s->L[i].w_qkv, ws->qkv, M, 3 * H, H, s->bn_qkv);
+    }
     if (st == E3_OK) st = gemm_tmaps(&m.o, ws->ctx, H, s->L[i].w_o, ws->y, M, H, H, s->bn_o);
     if (st == E3_OK) st = gemm_tmaps(&m.f1, ws->x1, H, s->L[i].w_1, ws->h, M, F, H, s->bn_f1);
-    if (st == E3_OK) st = gemm_tmaps(&m.f2, ws->h, F, s->L[i].w_2, ws->y, M, H, F, s->bn_f2);
+    if (st == E3_OK) st = gemm_tmaps(&m.f2, ws->h, F, s->L[i].w_2, vit ? out : ws->y, M, H, F, s->bn_f2);
   }
   if (st == E3_OK) st = attn_tmaps(&s->attn, ws->qkv, ws->ctx, B, S, H);
   if (st != E3_OK) {
@@ -187,11 +199,46 @@ e3_status split_run_to(e3_split *s, cudaStream_t st, const void *x_in, const int
   const double nvS = (double)n_valid_host * S;
   const double f_qkv = 2.0 * nvS * 3 * H * H, f_o = 2.0 * nvS * H * H, f_1 = 2.0 * nvS * F * H;
   const double f_att = 4.0 * n_valid_host * (double)S * S * H, b_ln = 2.0 * nvS * H * 2;
+  const bool vit = d.arch == E3_ARCH_VIT;
   for (int i = 0; i < nl; ++i) {
     const int l = d.layer_begin + i;
     const e3_layer_weights &L = s->L[i];
     auto &m = s->maps[i];
     void *out = (i % 2 == 0) ? ws.xa : ws.xb;
+    const bool last_layer = (i == nl - 1);
+    if (vit) {
+      // ViT pre-LN (R11): n1 = LN1(x); x1 = x + attn(n1 W_qkv) W_o;
+      // n2 = LN2(x1); x2 = x1 + GELU(n2 W_1) W_2
+      {
+        ProfScope ps(PK_LN, st, 0, b_ln);
+        E3_RUN(layernorm_run(cur, L.ln1_g, L.ln1_b, ws.x1, M, H, d.norm_eps, st));
+      }
+      {
+        ProfScope ps(PK_GEMM_QKV, st, f_qkv, 0);
+        E3_RUN(gemm_run(m.qkv, L.b_qkv, nullptr, M, 3 * H, H, E3_EPI_BIAS, s->sms, st));
+      }
+      {
+        ProfScope ps(PK_ATTN, st, f_att, 0);
+        E3_RUN(attn_run(s->attn, B, S, H, d.heads, st));
+      }
+      {
+        ProfScope ps(PK_GEMM_O, st, f_o, 0);
+        E3_RUN(gemm_run(m.o, L.b_o, cur, M, H, H, E3_EPI_BIAS_RESID, s->sms, st));
+      }
+      {
+        ProfScope ps(PK_LN, st, 0, b_ln);
+        E3_RUN(layernorm_run(ws.y, L.ln2_g, L.ln2_b, ws.x1, M, H, d.norm_eps, st));
+      }
+      {
+        ProfScope ps(PK_GEMM_FFN1, st, f_1, 0);
+        E3_RUN(gemm_run(m.f1, L.b_1, nullptr, M, F, H, E3_EPI_BIAS_GELU, s->sms, st));
+      }
+      {
+        ProfScope ps(PK_GEMM_FFN2, st, f_1, 0);
+        E3_RUN(gemm_run(m.f2, L.b_2, ws.y, M, H, F, E3_EPI_BIAS_RESID, s->sms, st));
+      }
+      cur = out;
+    } else {
     {
       ProfScope ps(PK_GEMM_QKV, st, f_qkv, 0);
       if (i == 0) {
@@ -225,20 +272,21 @@ e3_status split_run_to(e3_split *s, cudaStream_t st, const void *x_in, const int
     // The split's last layer never materialises LN2: its ramp normalises the
     // CLS rows itself and the fused LN2 + compaction normalises only the
     // survivors, writing them straight to the destination.
-    const bool last_layer = (i == nl - 1);
     if (!last_layer) {
       ProfScope ps(PK_LN, st, 0, b_ln);
       E3_RUN(layernorm_run(ws.y, L.ln2_g, L.ln2_b, out, M, H, d.norm_eps, st));
       cur = out;
+    }
     }
     while (ri < d.n_ramps && d.ramp_layer[ri] == l) {
       const bool last = (ri == d.n_ramps - 1);
       if (last || d.inner == E3_INNER_EXACT) {
         RampArgs a{};
         a.arch = d.arch;
-        a.x = last_layer ? ws.y : cur;
-        a.ln_g = last_layer ? L.ln2_g : nullptr;
-        a.ln_b = last_layer ? L.ln2_b : nullptr;
+        const bool pre_ln_rows = last_layer && !vit;   // BERT: the ramp applies LN2 itself
+        a.x = pre_ln_rows ? ws.y : cur;
+        a.ln_g = pre_ln_rows ? L.ln2_g : nullptr;
+        a.ln_b = pre_ln_rows ? L.ln2_b : nullptr;
         a.id = id_in;
         a.B = B;
         a.S = S;
@@ -260,8 +308,9 @@ e3_status split_run_to(e3_split *s, cudaStream_t st, const void *x_in, const int
         a.done_ctr = ws.ctr + 1;   // per-row-group tickets
         {
           // pooler weights + CLS rows + classifier weights (bytes); 2H^2 + 2HC per row (flops)
-          ProfScope ps(PK_RAMP, st, (double)n_valid_host * (2.0 * H * H + 2.0 * H * d.num_labels),
-                       2.0 * H * H + 2.0 * n_valid_host * H + 2.0 * d.num_labels * H);
+          const double hh = vit ? 0.0 : 2.0 * H * H;
+          ProfScope ps(PK_RAMP, st, (double)n_valid_host * (hh + 2.0 * H * d.num_labels),
+                       hh + 2.0 * n_valid_host * H + 2.0 * d.num_labels * H);
           E3_RUN(ramp_run(a, st));
         }
         first_ramp = false;
@@ -274,8 +323,12 @@ e3_status split_run_to(e3_split *s, cudaStream_t st, const void *x_in, const int
     // (bytes added once n_surv is known, in the pipeline)
     const e3_layer_weights &L = s->L[nl - 1];
     ProfScope ps(PK_COMPACT, st, 0, 0);
-    E3_RUN(ln_compact_run(ws.y, id_in, ws.alive, B, S, H, L.ln2_g, L.ln2_b, d.norm_eps, dst, n_surv_dev, s->sms,
-                          st));
+    if (vit)   // pre-LN: the layer output is final, survivors are copied
+      E3_RUN(ln_compact_run(cur, id_in, ws.alive, B, S, H, nullptr, nullptr, d.norm_eps, dst, n_surv_dev, s->sms,
+                            st));
+    else
+      E3_RUN(ln_compact_run(ws.y, id_in, ws.alive, B, S, H, L.ln2_g, L.ln2_b, d.norm_eps, dst, n_surv_dev, s->sms,
+                            st));
   }
 #undef E3_RUN
   return E3_OK;
@@ -370,7 +423,7 @@ e3_status e3_op_ramp(void *stream, int32_t arch, const void *x, const int64_t *i
                      const int32_t *n_valid_dev, const e3_exits *ex) {
   E3_CHECK_ARG(x && id && rw && alive && B > 0 && S > 0 && H > 0 && C > 0, "bad arguments");
   E3_CHECK_ARG(B <= 4096, "B > 4096");
-  E3_CHECK_ARG(aligned16(x) && aligned16(rw->w_p), "misaligned");
+  E3_CHECK_ARG(aligned16(x) && aligned16(arch == E3_ARCH_VIT ? rw->w_c : rw->w_p), "misaligned");
   int dev = 0;
   E3_CUDA_TRY(cudaGetDevice(&dev));
   // per-call scratch: pooled activations + ticket (freed asynchronously)

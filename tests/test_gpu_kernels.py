@@ -192,3 +192,63 @@ def test_ramp_matches_oracle(api, test, C):
                  n_valid=n_valid)
     torch.cuda.synchronize()
     assert int(ex2.n_exit.item()) == 45 and int(alive2.sum()) == 0
+
+
+@pytest.mark.parametrize("base,test,C", [("tiny", "maxprob", 10), ("tiny", "entropy", 1000),
+                                         ("tiny", "maxprob", 1500), ("vt", "maxprob", 1000)])
+def test_vit_ramp_matches_oracle(api, base, test, C):
+    """ViT ramp (LN + linear over C classes, cluster-merged softmax statistics)
+    vs oracle.ramp on the same bf16 rows: decisions exact where the margin
+    exceeds 1e-3, label = argmax, logits / metric within fp32 accumulation."""
+    import dataclasses
+    import e3data
+    from oracle import ramp as oramp
+    cfg = dataclasses.replace(e3data.get(base), arch="vit", test=test, classes=C, norm_eps=1e-6)
+    W = {"layers": [], "ramps": [e3data.make_ramp(cfg, 0, seed=13), e3data.make_ramp(cfg, 1, seed=13)]}
+    model = api.DeviceModel(cfg, W, DEV)
+    B, nv = 45, 40
+    rng = np.random.default_rng(C)
+    x = rand_bf16(rng, (B, cfg.seq if base == "tiny" else 4, cfg.hidden))
+    xt = bf16_tensor(x)
+    ids = torch.arange(B, device=DEV, dtype=torch.int64) * 2 + 1
+    n_valid = torch.tensor([nv], dtype=torch.int32, device=DEV)
+    R = {k: v.astype(np.float64) for k, v in W["ramps"][0].items()}
+    z = oramp.ramp_logits(cfg, x.astype(np.float64), R)
+    m = oramp.metric(test, z)
+    tau = float(np.float32(np.median(m[:nv])))
+    alive = torch.zeros(B, dtype=torch.uint8, device=DEV)
+    ex = api.ExitBuffers(2 * B + 2, C, 2, DEV)
+    api.ops.ramp(cfg, model, 0, xt, ids, tau, alive, ex, final=False, layer=5, n_valid=n_valid)
+    torch.cuda.synchronize()
+    passed = oramp.passes(test, m, tau)
+    margin = np.abs(m - np.float64(np.float32(tau)))
+    al = alive.cpu().numpy().astype(bool)
+    el, lab = ex.exit_layer.cpu().numpy(), ex.label.cpu().numpy()
+    conf, lg = ex.conf.cpu().numpy(), ex.logits.cpu().numpy()
+    n_dec = 0
+    for b in range(B):
+        i = 2 * b + 1
+        if b >= nv:
+            assert not al[b] and el[i] == -1
+            continue
+        if margin[b] > 1e-3:
+            assert al[b] == (not passed[b])
+            n_dec += 1
+        if not al[b]:
+            assert el[i] == 5
+            top2 = np.sort(z[b])[-2:]
+            if top2[1] - top2[0] > 1e-4:
+                assert lab[i] == int(np.argmax(z[b]))
+            assert abs(conf[i] - m[b]) < 1e-4
+            assert np.max(np.abs(lg[i] - z[b])) < 1e-3
+        else:
+            assert el[i] == -1
+    assert n_dec >= nv - 3
+    assert int(ex.n_exit.item()) == int((~al[:nv]).sum())
+    # final ramp exits every alive valid row
+    alive2 = torch.zeros(B, dtype=torch.uint8, device=DEV)
+    ex2 = api.ExitBuffers(2 * B + 2, C, 2, DEV)
+    api.ops.ramp(cfg, model, 1, xt, ids, 2.0 if test == "maxprob" else -1.0, alive2, ex2, final=True,
+                 n_valid=n_valid)
+    torch.cuda.synchronize()
+    assert int(ex2.n_exit.item()) == nv and int(alive2.sum()) == 0

@@ -39,6 +39,14 @@ def tiny(api):
     return cfg, W, model
 
 
+@pytest.fixture(scope="module")
+def tiny_vit(api):
+    cfg = e3data.get("tiny-vit")
+    W = e3data.make_weights(cfg)
+    model = api.DeviceModel(cfg, W, DEV)
+    return cfg, W, model
+
+
 def _compare_records(recs, ex, ids, cfg, margin=MARGIN, logit_tol=LOGIT_TOL):
     el = ex.exit_layer.cpu().numpy()
     lab = ex.label.cpu().numpy()
@@ -54,8 +62,11 @@ def _compare_records(recs, ex, ids, cfg, margin=MARGIN, logit_tol=LOGIT_TOL):
         if el[i] == r.exit_layer and top2[1] - top2[0] > 2 * logit_tol:   # argmax unique (R12)
             assert lab[i] == r.label
         if el[i] == r.exit_layer:
-            assert np.max(np.abs(lg[i] - r.logits)) < logit_tol, (i, lg[i], r.logits)
-            assert abs(conf[i] - r.metric) < logit_tol
+            # R13: absolute for logits up to 4 in magnitude, relative beyond
+            # (an un-squashed LN + linear head scales the bf16 error with |z|)
+            tol = logit_tol * max(1.0, float(np.max(np.abs(r.logits))) / 4.0)
+            assert np.max(np.abs(lg[i] - r.logits)) < tol, (i, lg[i], r.logits)
+            assert abs(conf[i] - r.metric) < tol
     return n_checked
 
 
@@ -132,6 +143,36 @@ def test_pipeline_tiny_matches_oracle_and_simulator(api, tiny):
             assert st.batches[s] == sim.per_split[s]["batches"]
             assert st.valid_rows[s] == sim.per_split[s]["valid"]
             assert st.rows_out[s] == sim.per_split[s]["rows_out"]
+
+
+def test_vit_split_run_per_split_parity_chain(api, tiny_vit):
+    """Pre-LN ViT layers + LN/linear ramp over 10 classes, S = 37 (ragged
+    128-row tiles): split [0,2) then [2,4) on the GPU's survivors."""
+    cfg, W, model = tiny_vit
+    X = e3data.make_inputs(cfg, range(cfg.batch))
+    rows, ids = _split_parity(api, cfg, W, model, X[:29], list(range(29)), 0, 2, cfg.tau)
+    _split_parity(api, cfg, W, model, rows, ids, 2, 4, cfg.tau)
+
+
+def test_vit_pipeline_matches_oracle_and_simulator(api, tiny_vit):
+    cfg, W, model = tiny_vit
+    N = 200
+    X = e3data.make_inputs(cfg, range(N), seed=3)
+    recs = oracle.run(cfg, W, X, mode="bf16")
+    ex = api.ExitBuffers(N, cfg.classes, cfg.n_ramps, DEV)
+    bounds = Plan.per_ramp(cfg.ramp_layers).bounds
+    pipe = api.Pipeline(model, api.make_plan(cfg, bounds, cfg.tau, lag=1, trace=True))
+    pipe.run(bf16_tensor(X), torch.arange(N, dtype=torch.int64, device=DEV), ex)
+    n_checked = _compare_records(recs, ex, range(N), cfg, E2E_MARGIN, E2E_LOGIT_TOL)
+    assert n_checked >= 0.8 * N and int(ex.n_exit.item()) == N
+    exit_layer = {i: int(v) for i, v in enumerate(ex.exit_layer.cpu().numpy())}
+    sim = simulate_pipeline(exit_layer, list(range(N)), Plan(bounds), cfg.batch, lag=1)
+    assert [(r.split, r.n_valid, r.ids) for r in sim.runs] == pipe.trace()
+    # plan invariance (inner EXACT): one split holding both ramps, bitwise
+    ex1 = api.ExitBuffers(N, cfg.classes, cfg.n_ramps, DEV)
+    api.Pipeline(model, api.make_plan(cfg, (0, 4), cfg.tau)).run(
+        bf16_tensor(X), torch.arange(N, dtype=torch.int64, device=DEV), ex1)
+    assert torch.equal(ex1.exit_layer, ex.exit_layer) and torch.equal(ex1.logits, ex.logits)
 
 
 def test_pipeline_plan_invariance_inner_exact(api, tiny):

@@ -51,3 +51,23 @@ def test_bert_ramp_is_pooler_then_fc():
          "b_c": np.array([0.0, 0.25])}
     z = ramp.ramp_logits(cfg, h, R)
     assert np.allclose(z, [np.tanh(1.0), np.tanh(-1.0) + 0.25])
+
+
+def test_vit_ramp_matches_torch_layernorm_linear():
+    """ViT ramp = LayerNorm(CLS) then Linear (R1), pinned to torch.nn in fp64."""
+    import torch
+    from e3data.configs import ModelConfig
+    H, C = 16, 1000
+    cfg = ModelConfig(name="t", arch="vit", layers=1, hidden=H, heads=1, ffn=H, seq=5,
+                      classes=C, norm_eps=1e-6, ramp_layers=(0,), batch=1, test="maxprob")
+    rng = np.random.default_rng(4)
+    h = rng.standard_normal((3, 5, H)) * 2 + 0.3
+    R = {"ln_g": 1 + 0.1 * rng.standard_normal(H), "ln_b": 0.1 * rng.standard_normal(H),
+         "w_c": rng.standard_normal((C, H)), "b_c": rng.standard_normal(C)}
+    ln = torch.nn.LayerNorm(H, eps=1e-6).double()
+    lin = torch.nn.Linear(H, C).double()
+    with torch.no_grad():
+        ln.weight.copy_(torch.from_numpy(R["ln_g"])); ln.bias.copy_(torch.from_numpy(R["ln_b"]))
+        lin.weight.copy_(torch.from_numpy(R["w_c"])); lin.bias.copy_(torch.from_numpy(R["b_c"]))
+        ref = lin(ln(torch.from_numpy(h[:, 0, :]))).numpy()
+    assert np.allclose(ramp.ramp_logits(cfg, h, R), ref, rtol=1e-12, atol=1e-12)
