@@ -312,3 +312,99 @@ def test_bert_base_pipeline_full_size_sampled(api, bert_base):
     sample = [int(i) for i in np.random.default_rng(0).choice(N, 6, replace=False)]
     recs = oracle.run(cfg, W, X[sample], ids=sample, tau=tau, mode="bf16")
     _compare_records(recs, ex, sample, cfg, E2E_MARGIN, E2E_LOGIT_TOL)
+
+
+def _split_parity_sampled(api, cfg, W, model, X, begin, end, tau, sample):
+    """Full-size split run on the batch X (n_valid = B); the oracle checks the
+    rows in `sample` only (rows are independent: R8 batch invariance)."""
+    from oracle.model import run_split
+    B = cfg.batch
+    split = api.Split(model, api.split_desc(cfg, begin, end, tau))
+    x = bf16_tensor(X)
+    id_t = torch.arange(B, dtype=torch.int64, device=DEV)
+    x_out = torch.zeros_like(x)
+    id_out = torch.full((B,), -9, dtype=torch.int64, device=DEV)
+    n_surv = torch.zeros(1, dtype=torch.int32, device=DEV)
+    ex = api.ExitBuffers(B, cfg.classes, cfg.n_ramps, DEV)
+    split.run(x, id_t, x_out, id_out, n_surv, ex)
+    torch.cuda.synchronize()
+    ns = int(n_surv.item())
+    assert ns + int(ex.n_exit.item()) == B
+    got = id_out[:ns].cpu().tolist()
+    assert got == sorted(got)                                   # stable compaction
+    assert set(got).isdisjoint(set(np.nonzero(ex.exit_layer.cpu().numpy() >= 0)[0].tolist()))
+    recs, surv_ids, h, margins = run_split(cfg, W, X[sample], begin, end, ids=list(sample), tau=tau, mode="bf16")
+    _compare_records(recs, ex, [r.id for r in recs], cfg, MARGIN, LOGIT_TOL * (end - begin))
+    for i in sample:
+        if margins[i] > MARGIN:
+            assert (i in got) == (i in surv_ids)
+    for i in surv_ids:
+        if i in got:
+            g = to64(x_out[got.index(i)])
+            o = h[surv_ids.index(i)]
+            assert np.mean(np.abs(g - o)) < 5e-3 and np.max(np.abs(g - o)) < 0.25
+
+
+@pytest.fixture(scope="module")
+def bert_large(api):
+    cfg = e3data.get("bl")
+    tau = e3data.tau_for(cfg)
+    W = e3data.make_weights(cfg)
+    model = api.DeviceModel(cfg, W, DEV)
+    return cfg, tau, W, model
+
+
+def test_bert_large_split_parity_full_size_sampled(api, bert_large):
+    """EE-BERT-large split [0,4) (one ramp at layer 4) on a full B=128 batch."""
+    cfg, tau, W, model = bert_large
+    X = e3data.make_inputs(cfg, range(cfg.batch))
+    _split_parity_sampled(api, cfg, W, model, X, 0, 4, tau, [0, 1, 17, 64, 100, 127])
+
+
+def test_bert_large_pipeline_full_size_sampled(api, bert_large):
+    cfg, tau, W, model = bert_large
+    N = 768
+    X = e3data.make_inputs(cfg, range(N))
+    ex = api.ExitBuffers(N, cfg.classes, cfg.n_ramps, DEV)
+    pipe = api.Pipeline(model, api.make_plan(cfg, Plan.per_ramp(cfg.ramp_layers).bounds, tau))
+    pipe.run(bf16_tensor(X), torch.arange(N, dtype=torch.int64, device=DEV), ex)
+    el = ex.exit_layer.cpu().numpy()
+    assert int(ex.n_exit.item()) == N and np.all(el >= 0)
+    hist = np.array([(el == l).mean() for l in cfg.ramp_layers])
+    assert np.all(np.abs(hist - np.array(cfg.exit_profile)) < 0.08), hist
+    sample = [int(i) for i in np.random.default_rng(1).choice(N, 3, replace=False)]
+    recs = oracle.run(cfg, W, X[sample], ids=sample, tau=tau, mode="bf16")
+    _compare_records(recs, ex, sample, cfg, E2E_MARGIN, E2E_LOGIT_TOL)
+
+
+@pytest.fixture(scope="module")
+def vit_base(api):
+    cfg = e3data.get("vt")
+    tau = e3data.tau_for(cfg)
+    W = e3data.make_weights(cfg)
+    model = api.DeviceModel(cfg, W, DEV)
+    return cfg, tau, W, model
+
+
+def test_vit_base_split_parity_full_size_sampled(api, vit_base):
+    """EE-ViT-B/16 split [0,2) (ramp after layer 2, C = 1000) on a full
+    B=256 x S=197 batch."""
+    cfg, tau, W, model = vit_base
+    X = e3data.make_inputs(cfg, range(cfg.batch))
+    _split_parity_sampled(api, cfg, W, model, X, 0, 2, tau, [0, 5, 128, 200, 255])
+
+
+def test_vit_base_pipeline_full_size_sampled(api, vit_base):
+    cfg, tau, W, model = vit_base
+    N = 1024
+    X = e3data.make_inputs(cfg, range(N))
+    ex = api.ExitBuffers(N, cfg.classes, cfg.n_ramps, DEV)
+    pipe = api.Pipeline(model, api.make_plan(cfg, Plan.per_ramp(cfg.ramp_layers).bounds, tau))
+    pipe.run(bf16_tensor(X), torch.arange(N, dtype=torch.int64, device=DEV), ex)
+    el = ex.exit_layer.cpu().numpy()
+    assert int(ex.n_exit.item()) == N and np.all(el >= 0)
+    hist = np.array([(el == l).mean() for l in cfg.ramp_layers])
+    assert np.all(np.abs(hist - np.array(cfg.exit_profile)) < 0.08), hist
+    sample = [int(i) for i in np.random.default_rng(2).choice(N, 3, replace=False)]
+    recs = oracle.run(cfg, W, X[sample], ids=sample, tau=tau, mode="bf16")
+    _compare_records(recs, ex, sample, cfg, E2E_MARGIN, E2E_LOGIT_TOL)
