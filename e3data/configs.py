@@ -95,15 +95,23 @@ VIT_BASE = ModelConfig(
     exit_profile=survival_profile((1, 3, 5, 7, 9, 11), 6.0),
 )
 
+# LLaMA-shaped tiny decode case: head_dim 128 as Llama-2, 2 heads, V = 1000,
+# 40 cached positions
+TINY_LLAMA = ModelConfig(
+    name="tiny-llama", arch="llama", layers=4, hidden=256, heads=2, ffn=512, seq=1,
+    classes=1000, norm_eps=1e-5, ramp_layers=(1, 3), batch=16, test="maxprob",
+    tau=(0.74, 0.74), cls_gain=8.0, kv_heads=2, ctx=40,
+)
+
 LLAMA_7B = ModelConfig(
     name="ee-llama-7b-decode", arch="llama", layers=32, hidden=4096, heads=32,
     ffn=11008, seq=1, classes=32000, norm_eps=1e-5, ramp_layers=(7, 15, 23, 31),
     batch=64, test="maxprob", exit_profile=(0.05, 0.10, 0.35, 0.50),
-    kv_heads=32, ctx=512,
+    kv_heads=32, ctx=512, cls_gain=8.0,
 )
 
-CONFIGS = {c.name: c for c in (TINY, TINY_VIT, BERT_BASE, BERT_LARGE, VIT_BASE, LLAMA_7B)}
-ALIASES = {"t": "tiny", "tv": "tiny-vit", "bb": "ee-bert-base", "bl": "ee-bert-large",
+CONFIGS = {c.name: c for c in (TINY, TINY_VIT, BERT_BASE, BERT_LARGE, VIT_BASE, TINY_LLAMA, LLAMA_7B)}
+ALIASES = {"t": "tiny", "tv": "tiny-vit", "tl": "tiny-llama", "bb": "ee-bert-base", "bl": "ee-bert-large",
            "vt": "ee-vit-b16", "lm": "ee-llama-7b-decode"}
 
 

@@ -13,6 +13,7 @@ Modules
   encoder       BERT post-LN / ViT pre-LN encoder layer (fp64 | bf16-emulate)
   ramp          exit ramps, max-prob / entropy metrics, exit test
   model         per-input early-exit forward + brute-force variant
+  llama         early-exit LLM decode step (RMSNorm/RoPE/KV cache/SwiGLU, LM-head ramp)
   pipeline_sim  split/queue bookkeeping of the constant-batch pipeline
   calibrate     per-ramp thresholds from a target exit profile
 
