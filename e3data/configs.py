@@ -99,7 +99,7 @@ VIT_BASE = ModelConfig(
 # 40 cached positions
 TINY_LLAMA = ModelConfig(
     name="tiny-llama", arch="llama", layers=4, hidden=256, heads=2, ffn=512, seq=1,
-    classes=1000, norm_eps=1e-5, ramp_layers=(1, 3), batch=16, test="maxprob",
+    classes=1000, norm_eps=1e-5, ramp_layers=(1, 3), batch=32, test="maxprob",
     tau=(0.74, 0.74), cls_gain=8.0, kv_heads=2, ctx=40,
 )
 

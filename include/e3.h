@@ -104,17 +104,38 @@ typedef struct e3_split_desc {
 typedef struct e3_layer_weights {
   const void *w_qkv, *b_qkv;   /* [3H,H], [3H]  rows: q | k | v, head-major   */
   const void *w_o, *b_o;       /* [H,H], [H]                                  */
-  const void *ln1_g, *ln1_b;   /* [H]                                         */
-  const void *w_1, *b_1;       /* [F,H], [F]                                  */
-  const void *w_2, *b_2;       /* [H,F], [H]                                  */
+  const void *ln1_g, *ln1_b;   /* [H]  (LLAMA: RMSNorm gain, ln1_b NULL)      */
+  const void *w_1, *b_1;       /* [F,H], [F]   (LLAMA: W_gate, no bias)       */
+  const void *w_2, *b_2;       /* [H,F], [H]   (LLAMA: W_down, no bias)       */
   const void *ln2_g, *ln2_b;   /* [H]                                         */
+  const void *w_3;             /* LLAMA: W_up [F,H] (NULL otherwise)          */
 } e3_layer_weights;
 
 typedef struct e3_ramp_weights {
   const void *w_p, *b_p;       /* BERT pooler [H,H], [H]   */
-  const void *w_c, *b_c;       /* classifier [C,H], [C]                       */
-  const void *ln_g, *ln_b;     /* VIT ramp LayerNorm [H] (NULL for BERT)      */
+  const void *w_c, *b_c;       /* classifier [C,H], [C] (LLAMA: LM head [V,H], */
+                               /* b_c NULL)               */
+  const void *ln_g, *ln_b;     /* VIT ramp LayerNorm [H] / LLAMA final RMSNorm */
+                               /* gain [H] (ln_b NULL); NULL for BERT          */
 } e3_ramp_weights;
+
+/* LLAMA decode: the caller-owned KV cache (R22-R24).
+ * Per layer l, k[l] and v[l] point to [n_slots][kv_heads][max_ctx][head_dim]
+ * bf16 device arrays.  Token id i belongs to the sequence in slot
+ * slot_of_id[i] (device int32, indexed by id < id_capacity) whose cached
+ * length is pos_of_slot[slot] (device int32): the decode step writes the
+ * token's k, v at that position of every layer it runs and attends over
+ * positions 0..pos.  Nothing is written for layers a token skips (R24).
+ * The library never advances pos_of_slot (the caller does, between steps). */
+typedef struct e3_kv_cache {
+  int32_t n_layers;
+  void *const *k;              /* host array of n_layers device pointers       */
+  void *const *v;
+  int32_t n_slots, max_ctx;
+  const int32_t *slot_of_id;
+  int64_t id_capacity;
+  const int32_t *pos_of_slot;
+} e3_kv_cache;
 
 /* Model weights indexed by model-wide layer / ramp number. */
 typedef struct e3_weights {
@@ -122,6 +143,7 @@ typedef struct e3_weights {
   const e3_layer_weights *layer;
   int32_t n_ramps;
   const e3_ramp_weights *ramp;
+  const e3_kv_cache *kv;       /* LLAMA only (NULL otherwise); borrowed        */
 } e3_weights;
 
 /* Exit records, written by the ramp kernel for every exiting valid row into

@@ -65,6 +65,31 @@ def calibrate(cfg, weights, X, mode="bf16"):
     return calibrate_from_metrics(cfg.test, M, cfg.exit_profile), M
 
 
+def calibrate_llama(cfg, n, seed_w=0, seed_x=2, seed_kv=4, mode="bf16"):
+    """llama decode: every calibration token through all layers (weights and
+    its KV cache generated layer by layer, so fp64 memory stays ~ one layer),
+    the shared LM-head ramp evaluated at every ramp layer; then the same
+    quantile rule.  Token i sits in its own slot at position cfg.ctx."""
+    import e3data
+    from .llama import decode_layer, ramp_logits
+    from .ramp import metric
+    X = e3data.make_inputs(cfg, range(n), seed=seed_x)[:, 0, :].astype(np.float64)
+    R = {k: np.asarray(v, dtype=np.float64) for k, v in e3data.make_ramp(cfg, 0, seed_w).items()}
+    M = np.zeros((n, cfg.n_ramps))
+    pos = np.full(n, cfg.ctx, dtype=np.int64)
+    h = X
+    for l in range(cfg.layers):
+        W = {k: np.asarray(v, dtype=np.float64) for k, v in e3data.make_layer(cfg, l, seed_w).items()}
+        kv = e3data.make_kv(cfg, l, range(n), cfg.ctx + 1, seed=seed_kv)
+        K, V = kv[0].astype(np.float64), kv[1].astype(np.float64)
+        del kv
+        h = decode_layer(cfg, h, W, K, V, pos, mode)
+        del W, K, V
+        if l in cfg.ramp_layers:
+            M[:, cfg.ramp_layers.index(l)] = metric(cfg.test, ramp_logits(cfg, h, R, mode))
+    return calibrate_from_metrics(cfg.test, M, cfg.exit_profile), M
+
+
 def golden_path(cfg_name):
     here = os.path.dirname(os.path.abspath(__file__))
     return os.path.join(os.path.dirname(here), "tests", "golden", f"tau_{cfg_name}.json")
@@ -80,10 +105,13 @@ def main(argv):
     cfg = e3data.get(argv[0])
     n = int(argv[1]) if len(argv) > 1 else 256
     seed_w, seed_x = 0, 2                     # calibration inputs: seed 2 (§8(d))
-    W = e3data.make_weights(cfg, seed_w)
-    X = e3data.make_inputs(cfg, range(n), seed=seed_x)
     t0 = time.time()
-    tau, M = calibrate(cfg, W, X)
+    if cfg.arch == "llama":
+        tau, M = calibrate_llama(cfg, n, seed_w, seed_x)
+    else:
+        W = e3data.make_weights(cfg, seed_w)
+        X = e3data.make_inputs(cfg, range(n), seed=seed_x)
+        tau, M = calibrate(cfg, W, X)
     rec = {"config": cfg.name, "tau": list(tau), "n_calib": n, "weight_seed": seed_w,
            "input_seed": seed_x, "mode": "bf16", "exit_profile": list(cfg.exit_profile),
            "script": "python -m oracle.calibrate " + " ".join(argv),

@@ -46,16 +46,21 @@ class SplitDesc(C.Structure):
 
 class LayerWeights(C.Structure):
     _fields_ = [(n, P) for n in ("w_qkv", "b_qkv", "w_o", "b_o", "ln1_g", "ln1_b", "w_1", "b_1",
-                                 "w_2", "b_2", "ln2_g", "ln2_b")]
+                                 "w_2", "b_2", "ln2_g", "ln2_b", "w_3")]
 
 
 class RampWeights(C.Structure):
     _fields_ = [(n, P) for n in ("w_p", "b_p", "w_c", "b_c", "ln_g", "ln_b")]
 
 
+class KVCache(C.Structure):
+    _fields_ = [("n_layers", I32), ("k", C.POINTER(P)), ("v", C.POINTER(P)), ("n_slots", I32),
+                ("max_ctx", I32), ("slot_of_id", P), ("id_capacity", I64), ("pos_of_slot", P)]
+
+
 class Weights(C.Structure):
     _fields_ = [("n_layers", I32), ("layer", C.POINTER(LayerWeights)), ("n_ramps", I32),
-                ("ramp", C.POINTER(RampWeights))]
+                ("ramp", C.POINTER(RampWeights)), ("kv", C.POINTER(KVCache))]
 
 
 class Exits(C.Structure):

@@ -22,7 +22,7 @@ import torch
 from . import _lib
 from ._lib import check, lib
 
-_LAYER_KEYS = ("w_qkv", "b_qkv", "w_o", "b_o", "ln1_g", "ln1_b", "w_1", "b_1", "w_2", "b_2",
+_LAYER_KEYS = ("w_qkv", "b_qkv", "w_o", "b_o", "ln1_g", "ln1_b", "w_1", "b_1", "w_2", "b_2", "w_3",
                "ln2_g", "ln2_b")
 _RAMP_KEYS = ("w_p", "b_p", "w_c", "b_c", "ln_g", "ln_b")
 
@@ -44,13 +44,25 @@ def to_bf16(a, device) -> torch.Tensor:
 
 
 class DeviceModel:
-    """EE-model weights uploaded once to HBM; builds the e3_weights struct."""
+    """EE-model weights uploaded once to HBM; builds the e3_weights struct.
 
-    def __init__(self, cfg, weights, device="cuda:0"):
+    llama: layer tensors w_gate / w_up / w_down travel as w_1 / w_3 / w_2; the
+    ramps share one LM head (uploaded once); `kv` is the KVCache the decode
+    step reads and appends to."""
+
+    _LLAMA_NAMES = {"w_gate": "w_1", "w_up": "w_3", "w_down": "w_2"}
+
+    def __init__(self, cfg, weights, device="cuda:0", kv=None):
         self.cfg = cfg
         self.device = torch.device(device)
-        self.layers = [{k: to_bf16(v, self.device) for k, v in w.items()} for w in weights["layers"]]
-        self.ramps = [{k: to_bf16(v, self.device) for k, v in w.items()} for w in weights["ramps"]]
+        ren = self._LLAMA_NAMES if cfg.arch == "llama" else {}
+        self.layers = [{ren.get(k, k): to_bf16(v, self.device) for k, v in w.items()} for w in weights["layers"]]
+        uploaded = {}
+        self.ramps = []
+        for w in weights["ramps"]:
+            if id(w) not in uploaded:
+                uploaded[id(w)] = {k: to_bf16(v, self.device) for k, v in w.items()}
+            self.ramps.append(uploaded[id(w)])
         n_l, n_r = len(self.layers), len(self.ramps)
         self._lw = (_lib.LayerWeights * max(n_l, 1))()
         for i, w in enumerate(self.layers):
@@ -60,10 +72,30 @@ class DeviceModel:
         for i, w in enumerate(self.ramps):
             for k in _RAMP_KEYS:
                 setattr(self._rw[i], k, w[k].data_ptr() if k in w else None)
-        self.c_weights = _lib.Weights(n_l, self._lw, n_r, self._rw)
+        self.kv = kv
+        self.c_weights = _lib.Weights(n_l, self._lw, n_r, self._rw, C.pointer(kv.c) if kv is not None else None)
 
     def ramp_struct(self, r):
         return self._rw[r]
+
+
+class KVCache:
+    """Caller-owned KV cache of the llama decode step (e3_kv_cache): per layer
+    K and V [n_slots, kv_heads, max_ctx, head_dim] bf16, the slot of every
+    token id and the cached length of every slot."""
+
+    def __init__(self, cfg, n_slots, max_ctx, id_capacity, device="cuda:0", fill=None):
+        dev = torch.device(device)
+        kvh, d = cfg.kv_heads or cfg.heads, cfg.head_dim
+        shape = (n_slots, kvh, max_ctx, d)
+        self.k = [torch.zeros(shape, dtype=torch.bfloat16, device=dev) for _ in range(cfg.layers)]
+        self.v = [torch.zeros(shape, dtype=torch.bfloat16, device=dev) for _ in range(cfg.layers)]
+        self.slot_of_id = torch.zeros(id_capacity, dtype=torch.int32, device=dev)
+        self.pos_of_slot = torch.full((n_slots,), cfg.ctx, dtype=torch.int32, device=dev)
+        self._kp = (C.c_void_p * cfg.layers)(*[t.data_ptr() for t in self.k])
+        self._vp = (C.c_void_p * cfg.layers)(*[t.data_ptr() for t in self.v])
+        self.c = _lib.KVCache(cfg.layers, self._kp, self._vp, n_slots, max_ctx, self.slot_of_id.data_ptr(),
+                              id_capacity, self.pos_of_slot.data_ptr())
 
 
 def split_desc(cfg, begin: int, end: int, tau, batch: Optional[int] = None,
@@ -132,7 +164,7 @@ class Split:
               "e3_split_run")
 
     def __del__(self):
-        if getattr(self, "h", None) and _lib.lib is not None:
+        if getattr(self, "h", None) and _lib is not None and _lib.lib is not None:
             _lib.lib.e3_split_destroy(self.h)
             self.h = None
 
@@ -162,7 +194,7 @@ class Queue:
         return bool(e.value)
 
     def __del__(self):
-        if getattr(self, "h", None) and _lib.lib is not None:
+        if getattr(self, "h", None) and _lib is not None and _lib.lib is not None:
             _lib.lib.e3_queue_destroy(self.h)
             self.h = None
 
@@ -224,7 +256,7 @@ class Pipeline:
         return [(split[i], nv[i], tuple(int(v) for v in ids[i, :nv[i]])) for i in range(k)]
 
     def __del__(self):
-        if getattr(self, "h", None) and _lib.lib is not None:
+        if getattr(self, "h", None) and _lib is not None and _lib.lib is not None:
             _lib.lib.e3_pipeline_destroy(self.h)
             self.h = None
 

@@ -58,8 +58,55 @@ struct RampArgs {
   e3_exits ex;
   float *pool_ws;           // [B,H] fp32 workspace
   unsigned *done_ctr;       // device tickets [ceil(B/kRampRowsPerCta)] (zero between launches)
+  // LLAMA: logits [B, C] fp32 and per-128-class-tile softmax statistics from
+  // the LM-head GEMM (gemm_dec.cu, E3_DEC_LOGITS); the decide kernel merges them
+  const float *lm_z;
+  const float4 *lm_stats;   // [tiles][B] (max, sum e, sum e*(z-max), argmax bits)
+  int lm_tiles;
 };
 e3_status ramp_run(const RampArgs &a, cudaStream_t st);
+
+// ---- K7 decode GEMM (gemm_dec.cu): Y[T,N] = epi(X[T,K] W[N,K]^T), swap-AB tcgen05
+enum { E3_DEC_STORE = 0, E3_DEC_RESID = 1, E3_DEC_SWIGLU = 2, E3_DEC_QKV_ROPE = 3, E3_DEC_LOGITS = 4 };
+struct DecMaps {
+  CUtensorMap w;    // W [N,K], box 128 (SWIGLU: 64) x 64, 128-B swizzle
+  CUtensorMap w2;   // SWIGLU: W_up, same box
+  CUtensorMap x;    // X [T,K], box T x 64
+};
+struct DecArgs {
+  int T, N, K, ks, epi;
+  const __nv_bfloat16 *R;   // RESID: residual [T, ldo]
+  __nv_bfloat16 *Y;         // STORE / RESID / SWIGLU / QKV (q): [T, ldo]
+  int ldo;
+  float *Z;                 // LOGITS: [T, N]
+  float4 *stats;            // LOGITS: [tiles][T]
+  float *part;              // split-K partials [tiles * ks][T][128]
+  unsigned *tickets;        // split-K tickets [tiles], zero between launches
+  // QKV_ROPE: this layer's cache and the tokens' slots / positions
+  int nh, kvh, max_ctx;
+  __nv_bfloat16 *kc, *vc;
+  const float2 *rope;       // [max_ctx][64] (cos, sin) of exact angles
+  const int64_t *ids;
+  const int32_t *n_valid_dev;
+  int n_valid_host;
+  const int32_t *slot_of_id;
+  int64_t id_cap;
+  const int32_t *pos_of_slot;
+};
+int dec_tiles(int N, int epi);
+int dec_pick_ks(int N, int K, int epi, int sms);
+e3_status dec_tmaps(DecMaps *m, const void *X, int T, int K, const void *W, const void *W2, int N, int epi);
+e3_status dec_run(const DecMaps &m, const DecArgs &a, int sms, cudaStream_t st);
+e3_status rope_table(int max_ctx, int head_dim, double theta, float2 **out);
+
+// ---- K8 LLaMA decode helpers (llama.cu)
+e3_status rmsnorm_run(const void *x, const void *g, void *y, int rows, int H, float eps, cudaStream_t st);
+// ctx[t, h*128 + :] = softmax(q_t,h . K[slot, g(h), 0..pos]^T / sqrt 128) V[...]
+e3_status attn_dec_run(const void *q, void *ctx, const void *kc, const void *vc, const int64_t *ids,
+                       const int32_t *n_valid_dev, int n_valid_host, const int32_t *slot_of_id, int64_t id_cap,
+                       const int32_t *pos_of_slot, int T, int nh, int kvh, int max_ctx, cudaStream_t st);
+// merge the LM-head statistics, threshold test, exit records (RampArgs with lm_*)
+e3_status lm_decide_run(const RampArgs &a, cudaStream_t st);
 
 // ---- K5 compaction (compact.cu)
 struct RingDst {

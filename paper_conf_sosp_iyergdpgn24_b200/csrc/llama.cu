@@ -1,0 +1,276 @@
+// LLaMA decode helpers of the split path (DESIGN.md §6
+// K8): RMSNorm, single-query attention over the KV cache, and the LM-head
+// ramp's decision.  The GEMMs of the decode layer are gemm_dec.cu.
+//
+//   rmsnorm_kernel   warp per token row: y = bf16(x / sqrt(mean x^2 + eps) * g)
+//   attn_dec_kernel  one CTA per (head, token): q from the QKV epilogue (RoPE
+//                    applied), keys/values of the token's slot at positions
+//                    0..pos (the new one written by the same epilogue);
+//                    scores fp32, p = exp(s - max) unrounded, out = bf16(p V / l)
+//                    -- HBM-bound on the cache stream (537 MB per Llama-7B
+//                    layer at 64 tokens x 513 positions)
+//   lm_decide_kernel warp per row: merges the LM-head tiles' softmax
+//                    statistics in tile order (softstat.cuh), max-prob /
+//                    entropy, strict threshold, exit record + logits copy,
+//                    alive flag -- the same semantics as the encoder ramps.
+#include "common.cuh"
+#include "kernels.h"
+#include "prof.h"
+#include "softstat.cuh"
+
+namespace e3 {
+
+namespace {
+
+template <int VPL>
+__global__ void __launch_bounds__(256) rmsnorm_kernel(const __nv_bfloat16 *__restrict__ x,
+                                                      const __nv_bfloat16 *__restrict__ g,
+                                                      __nv_bfloat16 *__restrict__ y, int rows, int H, float eps) {
+  const int warp = warp_id(), lane = lane_id();
+  const int row = blockIdx.x * 8 + warp;
+  const int nvec = H / 8;
+  uint4 gv[VPL];
+#pragma unroll
+  for (int i = 0; i < VPL; ++i) {
+    const int k = lane + 32 * i;
+    gv[i] = (k < nvec) ? __ldg(reinterpret_cast<const uint4 *>(g) + k) : make_uint4(0, 0, 0, 0);
+  }
+  pdl_wait();
+  pdl_trigger();
+  if (row >= rows) return;
+  const uint4 *xr = reinterpret_cast<const uint4 *>(x + (size_t)row * H);
+  uint4 v[VPL];
+  float ss = 0.f;
+#pragma unroll
+  for (int i = 0; i < VPL; ++i) {
+    const int k = lane + 32 * i;
+    v[i] = (k < nvec) ? xr[k] : make_uint4(0, 0, 0, 0);
+    const uint32_t w[4] = {v[i].x, v[i].y, v[i].z, v[i].w};
+#pragma unroll
+    for (int e = 0; e < 4; ++e) ss += bf_lo(w[e]) * bf_lo(w[e]) + bf_hi(w[e]) * bf_hi(w[e]);
+  }
+#pragma unroll
+  for (int o = 16; o; o >>= 1) ss += __shfl_xor_sync(0xffffffffu, ss, o);
+  const float rinv = 1.0f / sqrtf(ss / (float)H + eps);
+  uint4 *yr = reinterpret_cast<uint4 *>(y + (size_t)row * H);
+#pragma unroll
+  for (int i = 0; i < VPL; ++i) {
+    const int k = lane + 32 * i;
+    if (k >= nvec) continue;
+    const uint32_t w[4] = {v[i].x, v[i].y, v[i].z, v[i].w};
+    const uint32_t gw[4] = {gv[i].x, gv[i].y, gv[i].z, gv[i].w};
+    uint32_t o[4];
+#pragma unroll
+    for (int e = 0; e < 4; ++e)
+      o[e] = pack_bf16(bf_lo(w[e]) * rinv * bf_lo(gw[e]), bf_hi(w[e]) * rinv * bf_hi(gw[e]));
+    yr[k] = make_uint4(o[0], o[1], o[2], o[3]);
+  }
+}
+
+constexpr int kAttnThreads = 128;
+constexpr int kHd = 128;   // head_dim
+
+__device__ __forceinline__ float block_reduce(float v, float *red, bool is_max) {
+  const int warp = warp_id(), lane = lane_id();
+#pragma unroll
+  for (int o = 16; o; o >>= 1) {
+    const float w = __shfl_xor_sync(0xffffffffu, v, o);
+    v = is_max ? fmaxf(v, w) : v + w;
+  }
+  __syncthreads();   // red[] free
+  if (lane == 0) red[warp] = v;
+  __syncthreads();
+  float r = red[0];
+#pragma unroll
+  for (int w = 1; w < kAttnThreads / 32; ++w) r = is_max ? fmaxf(r, red[w]) : r + red[w];
+  return r;
+}
+
+__global__ void __launch_bounds__(kAttnThreads)
+    attn_dec_kernel(const __nv_bfloat16 *__restrict__ q, __nv_bfloat16 *__restrict__ ctx,
+                    const __nv_bfloat16 *__restrict__ kc, const __nv_bfloat16 *__restrict__ vc,
+                    const int64_t *__restrict__ ids, const int32_t *n_valid_dev, int n_valid_host,
+                    const int32_t *__restrict__ slot_of_id, int64_t id_cap, const int32_t *__restrict__ pos_of_slot,
+                    int nh, int kvh, int max_ctx, float scale) {
+  extern __shared__ float sp[];                 // [max_ctx] scores / probabilities
+  __shared__ float sq[kHd];
+  __shared__ float red[kAttnThreads / 32];
+  __shared__ float4 sacc[kAttnThreads / 32][32];
+  const int h = blockIdx.x, t = blockIdx.y;
+  const int tid = threadIdx.x, warp = warp_id(), lane = lane_id();
+  const int H = nh * kHd;
+  pdl_wait();
+  pdl_trigger();
+  const int nv = n_valid_dev ? *n_valid_dev : n_valid_host;
+  const int64_t id = ids[t];
+  __nv_bfloat16 *out = ctx + (size_t)t * H + h * kHd;
+  if (t >= nv || id < 0 || id >= id_cap) {     // padding row: finite zeros
+    if (tid < kHd / 2) reinterpret_cast<uint32_t *>(out)[tid] = 0u;
+    return;
+  }
+  const int slot = slot_of_id[id];
+  const int pos = pos_of_slot[slot];
+  const int L = pos + 1;
+  const int g = h / (nh / kvh);
+  sq[tid] = bf2f(q[(size_t)t * H + h * kHd + tid]);
+  __syncthreads();
+  const size_t base = ((size_t)slot * kvh + g) * max_ctx * kHd;
+  const uint4 *K = reinterpret_cast<const uint4 *>(kc + base);
+  // ---- scores: one key per thread (16 x 16-byte loads of its row)
+  float lmax = -INFINITY;
+  for (int j = tid; j < L; j += kAttnThreads) {
+    const uint4 *kr = K + (size_t)j * (kHd / 8);
+    float s = 0.f;
+#pragma unroll 4
+    for (int c = 0; c < kHd / 8; ++c) {
+      const uint4 kv = kr[c];
+      const uint32_t w[4] = {kv.x, kv.y, kv.z, kv.w};
+#pragma unroll
+      for (int e = 0; e < 4; ++e) {
+        s = fmaf(sq[c * 8 + 2 * e], bf_lo(w[e]), s);
+        s = fmaf(sq[c * 8 + 2 * e + 1], bf_hi(w[e]), s);
+      }
+    }
+    s *= scale;
+    sp[j] = s;
+    lmax = fmaxf(lmax, s);
+  }
+  const float m = block_reduce(lmax, red, true);
+  float lsum = 0.f;
+  for (int j = tid; j < L; j += kAttnThreads) {
+    const float e = expf(sp[j] - m);
+    sp[j] = e;
+    lsum += e;
+  }
+  const float l = block_reduce(lsum, red, false);   // also orders the sp[] writes
+  // ---- P V: warp w takes positions j = w mod 4, lane owns dims 4*lane .. +3
+  const uint2 *V = reinterpret_cast<const uint2 *>(vc + base);
+  float4 acc = make_float4(0.f, 0.f, 0.f, 0.f);
+#pragma unroll 4
+  for (int j = warp; j < L; j += kAttnThreads / 32) {
+    const uint2 vv = V[(size_t)j * (kHd / 4) + lane];
+    const float p = sp[j];
+    acc.x = fmaf(p, bf_lo(vv.x), acc.x);
+    acc.y = fmaf(p, bf_hi(vv.x), acc.y);
+    acc.z = fmaf(p, bf_lo(vv.y), acc.z);
+    acc.w = fmaf(p, bf_hi(vv.y), acc.w);
+  }
+  sacc[warp][lane] = acc;
+  __syncthreads();
+  if (warp == 0) {
+    float4 s = sacc[0][lane];
+#pragma unroll
+    for (int w = 1; w < kAttnThreads / 32; ++w) {
+      s.x += sacc[w][lane].x;
+      s.y += sacc[w][lane].y;
+      s.z += sacc[w][lane].z;
+      s.w += sacc[w][lane].w;
+    }
+    const float il = 1.0f / l;
+    uint2 o;
+    o.x = pack_bf16(s.x * il, s.y * il);
+    o.y = pack_bf16(s.z * il, s.w * il);
+    reinterpret_cast<uint2 *>(out)[lane] = o;
+  }
+}
+
+__global__ void __launch_bounds__(128) lm_decide_kernel(RampArgs a) {
+  const int warp = warp_id(), lane = lane_id();
+  const int b = blockIdx.x * 4 + warp;
+  pdl_wait();
+  pdl_trigger();
+  if (b >= a.B) return;
+  const int nv = a.n_valid_dev ? *a.n_valid_dev : a.n_valid_host;
+  const bool ok = b < nv && (a.init_alive || a.alive[b] != 0);
+  if (!ok) {
+    if (lane == 0 && a.init_alive) a.alive[b] = 0;
+    return;
+  }
+  SoftStat st{-INFINITY, 0.f, 0.f, -1};
+  for (int i = lane; i < a.lm_tiles; i += 32) {    // tile order within the lane
+    const float4 v = a.lm_stats[(size_t)i * a.B + b];
+    st = soft_merge(st, SoftStat{v.x, v.y, v.z, __float_as_int(v.w)});
+  }
+#pragma unroll
+  for (int o = 16; o; o >>= 1) st = soft_merge(st, soft_shfl_xor(st, o));
+  float metric;
+  bool pass;
+  if (a.test == E3_TEST_MAXPROB) {
+    metric = 1.0f / st.s;
+    pass = metric > a.tau;
+  } else {
+    metric = logf(st.s) - st.u / st.s;
+    pass = metric < a.tau;
+  }
+  const bool exit_now = pass || a.final_ramp;
+  const int64_t id = a.id[b];
+  if (exit_now && id >= 0 && id < a.ex.capacity) {
+    if (lane == 0) {
+      if (a.ex.exit_layer) a.ex.exit_layer[id] = a.layer;
+      if (a.ex.label) a.ex.label[id] = st.idx;
+      if (a.ex.conf) a.ex.conf[id] = metric;
+    }
+    if (a.ex.logits)
+      for (int c = lane; c < a.C; c += 32) a.ex.logits[id * a.C + c] = a.lm_z[(size_t)b * a.C + c];
+  }
+  if (lane == 0) {
+    a.alive[b] = exit_now ? 0 : 1;
+    if (exit_now) {
+      if (a.ex.n_exit) atomicAdd(a.ex.n_exit, 1);
+      if (a.ex.ramp_count) atomicAdd(a.ex.ramp_count + a.ramp_index, 1);
+    }
+  }
+}
+
+}  // namespace
+
+e3_status rmsnorm_run(const void *x, const void *g, void *y, int rows, int H, float eps, cudaStream_t st) {
+  if (H % 8 || H > 8192) {
+    set_error("rmsnorm: need H % 8 == 0, H <= 8192");
+    return E3_EUNSUPPORTED;
+  }
+  auto *xp = reinterpret_cast<const __nv_bfloat16 *>(x);
+  auto *gp = reinterpret_cast<const __nv_bfloat16 *>(g);
+  auto *yp = reinterpret_cast<__nv_bfloat16 *>(y);
+  const dim3 grid((rows + 7) / 8);
+  const int vpl = (H / 8 + 31) / 32;
+  if (vpl <= 1) E3_CUDA_TRY(launch_k(rmsnorm_kernel<1>, grid, dim3(256), 0, st, xp, gp, yp, rows, H, eps));
+  else if (vpl <= 4) E3_CUDA_TRY(launch_k(rmsnorm_kernel<4>, grid, dim3(256), 0, st, xp, gp, yp, rows, H, eps));
+  else if (vpl <= 16) E3_CUDA_TRY(launch_k(rmsnorm_kernel<16>, grid, dim3(256), 0, st, xp, gp, yp, rows, H, eps));
+  else E3_CUDA_TRY(launch_k(rmsnorm_kernel<32>, grid, dim3(256), 0, st, xp, gp, yp, rows, H, eps));
+  E3_CUDA_TRY(cudaGetLastError());
+  count_launch();
+  return E3_OK;
+}
+
+e3_status attn_dec_run(const void *q, void *ctx, const void *kc, const void *vc, const int64_t *ids,
+                       const int32_t *n_valid_dev, int n_valid_host, const int32_t *slot_of_id, int64_t id_cap,
+                       const int32_t *pos_of_slot, int T, int nh, int kvh, int max_ctx, cudaStream_t st) {
+  if (max_ctx > 16384 || nh % kvh) {
+    set_error("decode attention: need max_ctx <= 16384 and heads % kv_heads == 0");
+    return E3_EUNSUPPORTED;
+  }
+  const size_t smem = (size_t)max_ctx * 4;
+  static size_t attr_done = 0;
+  if (smem > 48 * 1024 && smem > attr_done) {
+    E3_CUDA_TRY(cudaFuncSetAttribute(attn_dec_kernel, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem));
+    attr_done = smem;
+  }
+  E3_CUDA_TRY(launch_k(attn_dec_kernel, dim3(nh, T), dim3(kAttnThreads), smem, st,
+                       reinterpret_cast<const __nv_bfloat16 *>(q), reinterpret_cast<__nv_bfloat16 *>(ctx),
+                       reinterpret_cast<const __nv_bfloat16 *>(kc), reinterpret_cast<const __nv_bfloat16 *>(vc),
+                       ids, n_valid_dev, n_valid_host, slot_of_id, id_cap, pos_of_slot, nh, kvh, max_ctx,
+                       1.0f / sqrtf((float)kHd)));
+  E3_CUDA_TRY(cudaGetLastError());
+  count_launch();
+  return E3_OK;
+}
+
+e3_status lm_decide_run(const RampArgs &a, cudaStream_t st) {
+  E3_CUDA_TRY(launch_k(lm_decide_kernel, dim3((a.B + 3) / 4), dim3(128), 0, st, a));
+  E3_CUDA_TRY(cudaGetLastError());
+  count_launch();
+  return E3_OK;
+}
+
+}  // namespace e3

@@ -33,6 +33,7 @@
 #include "common.cuh"
 #include "kernels.h"
 #include "ln_row.cuh"
+#include "softstat.cuh"
 #include "prof.h"
 
 namespace e3 {
@@ -310,25 +311,6 @@ __device__ __forceinline__ int ld_cluster_s32(uint32_t addr) {
   return v;
 }
 
-struct SoftStat {
-  float m, s, u;
-  int idx;
-};
-
-// merge b into a (a covers lower class indices on ties when merged in order)
-__device__ __forceinline__ SoftStat soft_merge(SoftStat a, SoftStat b) {
-  if (b.idx < 0) return a;
-  if (a.idx < 0) return b;
-  const float M = fmaxf(a.m, b.m);
-  const float ea = expf(a.m - M), eb = expf(b.m - M);
-  SoftStat r;
-  r.m = M;
-  r.s = a.s * ea + b.s * eb;
-  r.u = ea * (a.u + a.s * (a.m - M)) + eb * (b.u + b.s * (b.m - M));
-  r.idx = (b.m > a.m || (b.m == a.m && b.idx < a.idx)) ? b.idx : a.idx;
-  return r;
-}
-
 template <int CB>
 __global__ void __launch_bounds__(2 * CB) ramp_vit_kernel(RampArgs a, int CS) {
   constexpr int kThreads = 2 * CB, kWarps = kThreads / 32, kWarpsPerRg = CB / 64;
@@ -427,14 +409,7 @@ __global__ void __launch_bounds__(2 * CB) ramp_vit_kernel(RampArgs a, int CS) {
     if (c0 < C) st = SoftStat{z[rr][0], 1.f, 0.f, c0};
     if (c1 < C) st = soft_merge(st, SoftStat{z[rr][1], 1.f, 0.f, c1});
 #pragma unroll
-    for (int o = 16; o; o >>= 1) {
-      SoftStat ot;
-      ot.m = __shfl_xor_sync(0xffffffffu, st.m, o);
-      ot.s = __shfl_xor_sync(0xffffffffu, st.s, o);
-      ot.u = __shfl_xor_sync(0xffffffffu, st.u, o);
-      ot.idx = __shfl_xor_sync(0xffffffffu, st.idx, o);
-      st = soft_merge(st, ot);
-    }
+    for (int o = 16; o; o >>= 1) st = soft_merge(st, soft_shfl_xor(st, o));
     if (lane == 0) sRed[warp][rr] = st;
   }
   __syncthreads();

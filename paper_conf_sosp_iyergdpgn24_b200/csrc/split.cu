@@ -28,10 +28,49 @@ Workspace::~Workspace() {
   int prev = 0;
   cudaGetDevice(&prev);
   cudaSetDevice(device);
-  void *bufs[] = {qkv, ctx, y, x1, h, xa, xb, pool, alive, ctr};
+  void *bufs[] = {qkv, ctx, y, x1, h, xa, xb, pool, alive, ctr, lm_z, lm_stats, dec_part, dec_tickets, rope};
   for (void *p : bufs)
     if (p) cudaFree(p);
   cudaSetDevice(prev);
+}
+
+e3_status Workspace::ensure_llama(int V, size_t part, size_t tickets, int max_ctx, int head_dim, double theta) {
+  const size_t z = (size_t)B * V, st = (size_t)((V + 127) / 128) * B;
+  if (z > lm_z_elems) {
+    if (lm_z) cudaFree(lm_z);
+    lm_z = nullptr;
+    E3_CUDA_TRY(cudaMalloc(&lm_z, z * sizeof(float)));
+    lm_z_elems = z;
+  }
+  if (st > lm_stats_elems) {
+    if (lm_stats) cudaFree(lm_stats);
+    lm_stats = nullptr;
+    E3_CUDA_TRY(cudaMalloc(&lm_stats, st * sizeof(float4)));
+    lm_stats_elems = st;
+  }
+  if (part > part_elems) {
+    if (dec_part) cudaFree(dec_part);
+    dec_part = nullptr;
+    E3_CUDA_TRY(cudaMalloc(&dec_part, part * sizeof(float)));
+    part_elems = part;
+  }
+  if (tickets > ticket_elems) {
+    if (dec_tickets) cudaFree(dec_tickets);
+    dec_tickets = nullptr;
+    E3_CUDA_TRY(cudaMalloc(&dec_tickets, tickets * sizeof(unsigned)));
+    E3_CUDA_TRY(cudaMemset(dec_tickets, 0, tickets * sizeof(unsigned)));
+    ticket_elems = tickets;
+  }
+  if (!rope || rope_ctx != max_ctx || rope_hd != head_dim || rope_theta != theta) {
+    if (rope) cudaFree(rope);
+    rope = nullptr;
+    e3_status r = rope_table(max_ctx, head_dim, theta, &rope);
+    if (r != E3_OK) return r;
+    rope_ctx = max_ctx;
+    rope_hd = head_dim;
+    rope_theta = theta;
+  }
+  return E3_OK;
 }
 
 e3_status Workspace::create(int device, int B, int S, int H, int F, std::shared_ptr<Workspace> *out) {
@@ -60,12 +99,59 @@ e3_status Workspace::create(int device, int B, int S, int H, int F, std::shared_
 
 static bool aligned16(const void *p) { return (reinterpret_cast<uintptr_t>(p) & 15) == 0; }
 
-e3_status split_validate(const e3_split_desc *d, const e3_weights *w) {
-  E3_CHECK_ARG(d && w, "null descriptor or weights");
-  if (d->arch != E3_ARCH_BERT && d->arch != E3_ARCH_VIT) {
-    set_error("e3_split_create: arch not implemented on the GPU path (BERT, VIT)");
+// LLAMA decode: head_dim 128, one token per row (S = 1),
+// B in {32, 64, 128}, the caller's KV cache covering the split's layers.
+static e3_status llama_validate(const e3_split_desc *d, const e3_weights *w) {
+  if (d->dtype != E3_DTYPE_BF16) {
+    set_error("e3_split_create: only dtype BF16 is implemented");
     return E3_EUNSUPPORTED;
   }
+  const int kvh = d->kv_heads > 0 ? d->kv_heads : d->heads;
+  if (d->heads <= 0 || d->hidden != d->heads * 128 || d->heads % kvh || d->seq_len != 1 || d->ffn % 64 ||
+      d->ffn <= 0 || (d->batch != 32 && d->batch != 64 && d->batch != 128) || d->num_labels < 1 ||
+      d->hidden > 8192) {
+    set_error("e3_split_create (LLAMA): need head_dim 128 (H = 128 * heads), heads % kv_heads == 0, S == 1, "
+              "F % 64 == 0, B in {32, 64, 128}, H <= 8192");
+    return E3_EUNSUPPORTED;
+  }
+  E3_CHECK_ARG(d->layer_begin >= 0 && d->layer_end > d->layer_begin && d->layer_end <= w->n_layers,
+               "layer range outside the model");
+  E3_CHECK_ARG(d->n_ramps >= 1 && d->n_ramps <= E3_MAX_RAMPS, "a split needs 1..64 ramps");
+  for (int r = 0; r < d->n_ramps; ++r) {
+    E3_CHECK_ARG(d->ramp_layer[r] >= d->layer_begin && d->ramp_layer[r] < d->layer_end, "ramp outside split");
+    E3_CHECK_ARG(r == 0 || d->ramp_layer[r] > d->ramp_layer[r - 1], "ramp layers not ascending");
+    E3_CHECK_ARG(d->ramp_index[r] >= 0 && d->ramp_index[r] < w->n_ramps, "ramp index outside the model");
+    const e3_ramp_weights &R = w->ramp[d->ramp_index[r]];
+    E3_CHECK_ARG(R.ln_g && R.w_c && aligned16(R.w_c), "LLAMA ramp needs ln_g (final norm) and w_c (LM head)");
+  }
+  E3_CHECK_ARG(d->ramp_layer[d->n_ramps - 1] == d->layer_end - 1, "a split must end in a ramp");
+  E3_CHECK_ARG(d->test == E3_TEST_MAXPROB || d->test == E3_TEST_ENTROPY, "bad test");
+  E3_CHECK_ARG(d->inner == E3_INNER_EXACT || d->inner == E3_INNER_DISABLED, "bad inner mode");
+  for (int l = d->layer_begin; l < d->layer_end; ++l) {
+    const e3_layer_weights &L = w->layer[l];
+    const void *ps[] = {L.w_qkv, L.w_o, L.ln1_g, L.w_1, L.w_2, L.w_3, L.ln2_g};
+    for (const void *p : ps) E3_CHECK_ARG(p && aligned16(p), "LLAMA layer weight pointer null or misaligned");
+  }
+  const e3_kv_cache *kv = w->kv;
+  E3_CHECK_ARG(kv && kv->k && kv->v && kv->slot_of_id && kv->pos_of_slot, "LLAMA needs e3_weights.kv");
+  E3_CHECK_ARG(kv->n_layers >= d->layer_end && kv->n_slots > 0 && kv->max_ctx > 0 && kv->id_capacity > 0,
+               "KV cache does not cover the split");
+  if (kv->max_ctx > 16384) {
+    set_error("e3_split_create (LLAMA): max_ctx > 16384");
+    return E3_EUNSUPPORTED;
+  }
+  for (int l = d->layer_begin; l < d->layer_end; ++l)
+    E3_CHECK_ARG(kv->k[l] && kv->v[l] && aligned16(kv->k[l]) && aligned16(kv->v[l]), "KV layer pointer");
+  return E3_OK;
+}
+
+e3_status split_validate(const e3_split_desc *d, const e3_weights *w) {
+  E3_CHECK_ARG(d && w, "null descriptor or weights");
+  if (d->arch != E3_ARCH_BERT && d->arch != E3_ARCH_VIT && d->arch != E3_ARCH_LLAMA_DECODE) {
+    set_error("e3_split_create: unknown arch");
+    return E3_EUNSUPPORTED;
+  }
+  if (d->arch == E3_ARCH_LLAMA_DECODE) return llama_validate(d, w);
   const bool vit = d->arch == E3_ARCH_VIT;
   if (d->dtype != E3_DTYPE_BF16) {
     set_error("e3_split_create: only dtype BF16 is implemented");
@@ -114,6 +200,52 @@ static e3_status check_device(int device) {
   return E3_OK;
 }
 
+// LLAMA: tensor maps of the decode GEMMs (activations in the workspace, so
+// the maps are fixed for the handle's life), split-K choices, shared buffers
+static e3_status llama_create(e3_split *s, const e3_weights *w) {
+  const e3_split_desc &d = s->d;
+  Workspace &ws = *s->ws;
+  const int B = d.batch, H = d.hidden, F = d.ffn, V = d.num_labels;
+  const int kvh = d.kv_heads > 0 ? d.kv_heads : d.heads;
+  const int nqkv = (d.heads + 2 * kvh) * 128;
+  s->kv = *w->kv;
+  for (int l = 0; l < w->kv->n_layers; ++l) {
+    s->kv_k.push_back(w->kv->k[l]);
+    s->kv_v.push_back(w->kv->v[l]);
+  }
+  s->ks_qkv = dec_pick_ks(nqkv, H, E3_DEC_QKV_ROPE, s->sms);
+  s->ks_o = dec_pick_ks(H, H, E3_DEC_RESID, s->sms);
+  s->ks_gu = dec_pick_ks(F, H, E3_DEC_SWIGLU, s->sms);
+  s->ks_down = dec_pick_ks(H, F, E3_DEC_RESID, s->sms);
+  s->ks_lm = 1;
+  size_t part = 0, tickets = 0;
+  auto need = [&](int N, int ks, int epi) {
+    const size_t t = (size_t)dec_tiles(N, epi);
+    if (ks > 1 && t * ks * B * 128 > part) part = t * ks * B * 128;
+    if (t > tickets) tickets = t;
+  };
+  need(nqkv, s->ks_qkv, E3_DEC_QKV_ROPE);
+  need(H, s->ks_o, E3_DEC_RESID);
+  need(F, s->ks_gu, E3_DEC_SWIGLU);
+  need(H, s->ks_down, E3_DEC_RESID);
+  e3_status st = ws.ensure_llama(V, part, tickets, w->kv->max_ctx, 128, 10000.0);
+  if (st != E3_OK) return st;
+  const int nl = d.layer_end - d.layer_begin;
+  s->dmaps.resize(nl);
+  for (int i = 0; i < nl && st == E3_OK; ++i) {
+    const e3_layer_weights &L = s->L[i];
+    auto &m = s->dmaps[i];
+    st = dec_tmaps(&m.qkv, ws.x1, B, H, L.w_qkv, nullptr, nqkv, E3_DEC_QKV_ROPE);
+    if (st == E3_OK) st = dec_tmaps(&m.o, ws.ctx, B, H, L.w_o, nullptr, H, E3_DEC_RESID);
+    if (st == E3_OK) st = dec_tmaps(&m.gu, ws.x1, B, H, L.w_1, L.w_3, F, E3_DEC_SWIGLU);
+    if (st == E3_OK) st = dec_tmaps(&m.down, ws.h, B, F, L.w_2, nullptr, H, E3_DEC_RESID);
+  }
+  s->lm_maps.resize(d.n_ramps);
+  for (int r = 0; r < d.n_ramps && st == E3_OK; ++r)
+    st = dec_tmaps(&s->lm_maps[r], ws.x1, B, H, s->R[r].w_c, nullptr, V, E3_DEC_LOGITS);
+  return st;
+}
+
 e3_status split_create_shared(const e3_split_desc *d, const e3_weights *w, int device, std::shared_ptr<Workspace> ws,
                               e3_split **out) {
   E3_CHECK_ARG(out, "null out");
@@ -145,6 +277,15 @@ e3_status split_create_shared(const e3_split_desc *d, const e3_weights *w, int d
     return E3_EINVAL;
   }
   s->ws = ws;
+  if (d->arch == E3_ARCH_LLAMA_DECODE) {
+    st = llama_create(s, w);
+    if (st != E3_OK) {
+      delete s;
+      return st;
+    }
+    *out = s;
+    return E3_OK;
+  }
   const int M = B * S;
   s->bn_qkv = gemm_pick_bn(M, 3 * H, s->sms);
   s->bn_o = gemm_pick_bn(M, H, s->sms);
@@ -177,9 +318,175 @@ e3_status split_create_shared(const e3_split_desc *d, const e3_weights *w, int d
   return E3_OK;
 }
 
+// LLAMA decode split (R22-R24): per layer
+//   n1 = RMSNorm1(x)                          rmsnorm_kernel
+//   q | cache[k, v] = RoPE(n1 W_qkv^T)         decode GEMM, QKV_ROPE epilogue
+//   ctx = attention(q, cache[0..pos])          attn_dec_kernel
+//   h = x + ctx W_o^T                          decode GEMM (split-K), RESID
+//   n2 = RMSNorm2(h)
+//   a = SiLU(n2 W_gate^T) * (n2 W_up^T)        decode GEMM, SWIGLU
+//   x' = h + a W_down^T                        decode GEMM (split-K), RESID
+// ramp after layer l: nf = RMSNorm_f(x'), z = nf W_lm^T (LOGITS epilogue with
+// per-tile softmax statistics), lm_decide; then the survivors are compacted.
+static e3_status llama_run(e3_split *s, cudaStream_t st, const void *x_in, const int64_t *id_in,
+                           const int32_t *n_valid_dev, int n_valid_host, const RingDst &dst, int32_t *n_surv_dev,
+                           const e3_exits *ex) {
+  const e3_split_desc &d = s->d;
+  Workspace &ws = *s->ws;
+  const int B = d.batch, H = d.hidden, F = d.ffn, V = d.num_labels;
+  const int kvh = d.kv_heads > 0 ? d.kv_heads : d.heads;
+  const int nqkv = (d.heads + 2 * kvh) * 128;
+  const int nl = d.layer_end - d.layer_begin;
+  e3_exits exits{};
+  if (ex) exits = *ex;
+  const void *cur = x_in;
+  bool first_ramp = true;
+  int ri = 0;
+  e3_status r = E3_OK;
+#define E3_RUN(expr)              \
+  do {                            \
+    r = (expr);                   \
+    if (r != E3_OK) return r;     \
+  } while (0)
+  // algorithmic bytes (the path is HBM-bound): weights once per launch, the
+  // valid tokens' activations, the KV positions 0..ctx of every valid token
+  const double nv = n_valid_host, b2 = 2.0;
+  const double kv_bytes = nv * d.heads * (double)(d.ctx_len + 1) * 128 * 2 * b2 / (d.heads / kvh);
+  DecArgs base{};
+  base.T = B;
+  base.part = ws.dec_part;
+  base.tickets = ws.dec_tickets;
+  for (int i = 0; i < nl; ++i) {
+    const int l = d.layer_begin + i;
+    const e3_layer_weights &L = s->L[i];
+    auto &m = s->dmaps[i];
+    void *out = (i % 2 == 0) ? ws.xa : ws.xb;
+    {
+      ProfScope ps(PK_LN, st, 0, nv * H * 2 * b2);
+      E3_RUN(rmsnorm_run(cur, L.ln1_g, ws.x1, B, H, d.norm_eps, st));
+    }
+    {
+      DecArgs a = base;
+      a.N = nqkv;
+      a.K = H;
+      a.ks = s->ks_qkv;
+      a.epi = E3_DEC_QKV_ROPE;
+      a.Y = reinterpret_cast<__nv_bfloat16 *>(ws.qkv);
+      a.ldo = d.heads * 128;
+      a.nh = d.heads;
+      a.kvh = kvh;
+      a.max_ctx = s->kv.max_ctx;
+      a.kc = reinterpret_cast<__nv_bfloat16 *>(s->kv_k[l]);
+      a.vc = reinterpret_cast<__nv_bfloat16 *>(s->kv_v[l]);
+      a.rope = ws.rope;
+      a.ids = id_in;
+      a.n_valid_dev = n_valid_dev;
+      a.n_valid_host = n_valid_host;
+      a.slot_of_id = s->kv.slot_of_id;
+      a.id_cap = s->kv.id_capacity;
+      a.pos_of_slot = s->kv.pos_of_slot;
+      ProfScope ps(PK_GEMM_QKV, st, 0, (double)nqkv * H * b2 + nv * (H + nqkv) * b2);
+      E3_RUN(dec_run(m.qkv, a, s->sms, st));
+    }
+    {
+      ProfScope ps(PK_ATTN, st, 0, kv_bytes);
+      E3_RUN(attn_dec_run(ws.qkv, ws.ctx, s->kv_k[l], s->kv_v[l], id_in, n_valid_dev, n_valid_host,
+                          s->kv.slot_of_id, s->kv.id_capacity, s->kv.pos_of_slot, B, d.heads, kvh, s->kv.max_ctx,
+                          st));
+    }
+    {
+      DecArgs a = base;
+      a.N = H;
+      a.K = H;
+      a.ks = s->ks_o;
+      a.epi = E3_DEC_RESID;
+      a.R = reinterpret_cast<const __nv_bfloat16 *>(cur);
+      a.Y = reinterpret_cast<__nv_bfloat16 *>(ws.y);
+      a.ldo = H;
+      ProfScope ps(PK_GEMM_O, st, 0, (double)H * H * b2 + nv * 3 * H * b2);
+      E3_RUN(dec_run(m.o, a, s->sms, st));
+    }
+    {
+      ProfScope ps(PK_LN, st, 0, nv * H * 2 * b2);
+      E3_RUN(rmsnorm_run(ws.y, L.ln2_g, ws.x1, B, H, d.norm_eps, st));
+    }
+    {
+      DecArgs a = base;
+      a.N = F;
+      a.K = H;
+      a.ks = s->ks_gu;
+      a.epi = E3_DEC_SWIGLU;
+      a.Y = reinterpret_cast<__nv_bfloat16 *>(ws.h);
+      a.ldo = F;
+      ProfScope ps(PK_GEMM_FFN1, st, 0, 2.0 * F * H * b2 + nv * (H + F) * b2);
+      E3_RUN(dec_run(m.gu, a, s->sms, st));
+    }
+    {
+      DecArgs a = base;
+      a.N = H;
+      a.K = F;
+      a.ks = s->ks_down;
+      a.epi = E3_DEC_RESID;
+      a.R = reinterpret_cast<const __nv_bfloat16 *>(ws.y);
+      a.Y = reinterpret_cast<__nv_bfloat16 *>(out);
+      a.ldo = H;
+      ProfScope ps(PK_GEMM_FFN2, st, 0, (double)F * H * b2 + nv * (F + 2 * H) * b2);
+      E3_RUN(dec_run(m.down, a, s->sms, st));
+    }
+    cur = out;
+    while (ri < d.n_ramps && d.ramp_layer[ri] == l) {
+      const bool last = (ri == d.n_ramps - 1);
+      if (last || d.inner == E3_INNER_EXACT) {
+        ProfScope ps(PK_RAMP, st, 0, (double)V * H * b2 + nv * (H * b2 + V * 4.0));
+        E3_RUN(rmsnorm_run(cur, s->R[ri].ln_g, ws.x1, B, H, d.norm_eps, st));
+        DecArgs a = base;
+        a.N = V;
+        a.K = H;
+        a.ks = 1;
+        a.epi = E3_DEC_LOGITS;
+        a.Z = ws.lm_z;
+        a.stats = ws.lm_stats;
+        E3_RUN(dec_run(s->lm_maps[ri], a, s->sms, st));
+        RampArgs ra{};
+        ra.arch = d.arch;
+        ra.id = id_in;
+        ra.B = B;
+        ra.S = 1;
+        ra.H = H;
+        ra.C = V;
+        ra.test = d.test;
+        ra.tau = d.tau[ri];
+        ra.final_ramp = last && d.final_ramp;
+        ra.layer = l;
+        ra.ramp_index = d.ramp_index[ri];
+        ra.alive = ws.alive;
+        ra.init_alive = first_ramp;
+        ra.n_valid_dev = n_valid_dev;
+        ra.n_valid_host = n_valid_host;
+        ra.ex = exits;
+        ra.lm_z = ws.lm_z;
+        ra.lm_stats = ws.lm_stats;
+        ra.lm_tiles = dec_tiles(V, E3_DEC_LOGITS);
+        E3_RUN(lm_decide_run(ra, st));
+        first_ramp = false;
+      }
+      ++ri;
+    }
+  }
+  {
+    ProfScope ps(PK_COMPACT, st, 0, 0);
+    E3_RUN(ln_compact_run(cur, id_in, ws.alive, B, 1, H, nullptr, nullptr, d.norm_eps, dst, n_surv_dev, s->sms,
+                          st));
+  }
+#undef E3_RUN
+  return E3_OK;
+}
+
 e3_status split_run_to(e3_split *s, cudaStream_t st, const void *x_in, const int64_t *id_in,
                        const int32_t *n_valid_dev, int n_valid_host, const RingDst &dst, int32_t *n_surv_dev,
                        const e3_exits *ex) {
+  if (s->d.arch == E3_ARCH_LLAMA_DECODE)
+    return llama_run(s, st, x_in, id_in, n_valid_dev, n_valid_host, dst, n_surv_dev, ex);
   const e3_split_desc &d = s->d;
   Workspace &ws = *s->ws;
   const int B = d.batch, S = d.seq_len, H = d.hidden, F = d.ffn, M = B * S;

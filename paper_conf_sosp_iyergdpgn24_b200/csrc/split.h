@@ -20,6 +20,17 @@ struct Workspace {
   float *pool = nullptr;
   uint8_t *alive = nullptr;
   unsigned *ctr = nullptr;        // [kCtrWords]: compaction ticket, ramp row-group tickets
+  // LLAMA decode (allocated by ensure_llama): LM-head logits / tile statistics,
+  // split-K partials and tickets of the decode GEMMs, RoPE cos/sin table
+  float *lm_z = nullptr;
+  float4 *lm_stats = nullptr;
+  float *dec_part = nullptr;
+  unsigned *dec_tickets = nullptr;
+  float2 *rope = nullptr;
+  size_t lm_z_elems = 0, lm_stats_elems = 0, part_elems = 0, ticket_elems = 0;
+  int rope_ctx = 0, rope_hd = 0;
+  double rope_theta = 0;
+  e3_status ensure_llama(int V, size_t part_elems, size_t tickets, int max_ctx, int head_dim, double theta);
   ~Workspace();
   static e3_status create(int device, int B, int S, int H, int F, std::shared_ptr<Workspace> *out);
 };
@@ -38,6 +49,15 @@ struct e3_split {
     e3::GemmMaps qkv, o, f1, f2;
   };
   std::vector<LayerMaps> maps;
+  // LLAMA decode: per layer the four decode GEMMs, per ramp the LM head
+  struct DecLayer {
+    e3::DecMaps qkv, o, gu, down;
+  };
+  std::vector<DecLayer> dmaps;
+  std::vector<e3::DecMaps> lm_maps;
+  int ks_qkv = 1, ks_o = 1, ks_gu = 1, ks_down = 1, ks_lm = 1;
+  e3_kv_cache kv{};
+  std::vector<void *> kv_k, kv_v;       // this split's layers' cache pointers
   e3::AttnMaps attn;
   int bn_qkv = 0, bn_o = 0, bn_f1 = 0, bn_f2 = 0;
 };
