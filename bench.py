@@ -51,7 +51,8 @@ def parse():
     ap.add_argument("--warmup", type=int, default=3)
     ap.add_argument("--impl", default="ours", choices=["ours", "reference"])
     ap.add_argument("--config", default="bb")
-    ap.add_argument("--inputs-per-gpu", type=int, default=8192)
+    ap.add_argument("--inputs-per-gpu", type=int, default=None,
+                    help="default 8192 (encoders: > L2 of activations), 256 (llama: 256 sequences' KV caches)")
     ap.add_argument("--plan", default="per-ramp", choices=["per-ramp", "cut6"])
     ap.add_argument("--no-e2e", action="store_true")
     ap.add_argument("--no-cpu", action="store_true")
@@ -137,11 +138,41 @@ def cpu_oracle_rate(cfg, tau, n_inputs, seed_offset=0):
     """The oracle as it stands (fp64 NumPy, all host cores) on a bounded sample."""
     import e3data
     import oracle
+    if cfg.arch == "llama":
+        return cpu_oracle_rate_llama(cfg, tau, n_inputs, seed_offset)
     W = e3data.make_weights(cfg)
     X = e3data.make_inputs(cfg, range(seed_offset, seed_offset + n_inputs))
     t0 = time.perf_counter()
     oracle.run(cfg, W, X, tau=tau, mode="fp64")
     dt = time.perf_counter() - t0
+    return n_inputs / dt, dt
+
+
+def cpu_oracle_rate_llama(cfg, tau, n_inputs, seed_offset=0):
+    """oracle.llama on n tokens, layer by layer (weights and caches generated
+    per layer outside the timed part so fp64 memory stays ~ one layer)."""
+    import e3data
+    from oracle import llama as olm
+    from oracle.ramp import metric, passes
+    X = e3data.make_inputs(cfg, range(seed_offset, seed_offset + n_inputs))[:, 0, :].astype(np.float64)
+    R = {k: np.asarray(v, dtype=np.float64) for k, v in e3data.make_ramp(cfg, 0).items()}
+    alive = np.arange(n_inputs)
+    pos = np.full(n_inputs, cfg.ctx, dtype=np.int64)
+    h, dt = X, 0.0
+    for l in range(cfg.layers):
+        if alive.size == 0:
+            break
+        W = {k: np.asarray(v, dtype=np.float64) for k, v in e3data.make_layer(cfg, l).items()}
+        kv = e3data.make_kv(cfg, l, range(seed_offset, seed_offset + n_inputs), cfg.ctx + 1)
+        K, V = kv[0][alive].astype(np.float64), kv[1][alive].astype(np.float64)
+        t0 = time.perf_counter()
+        h = olm.decode_layer(cfg, h, W, K, V, pos[alive], "fp64")
+        if l in cfg.ramp_layers:
+            r = cfg.ramp_layers.index(l)
+            m = metric(cfg.test, olm.ramp_logits(cfg, h, R))
+            ok = np.ones(alive.size, bool) if r == cfg.n_ramps - 1 else passes(cfg.test, m, tau[r])
+            alive, h = alive[~ok], h[~ok]
+        dt += time.perf_counter() - t0
     return n_inputs / dt, dt
 
 
@@ -191,11 +222,30 @@ def main():
 
     cfg, tau = load_workload(args.config)
     bounds, plan_name = plan_bounds(cfg, args.plan)
-    W = e3data.make_weights(cfg)
-    model = api.DeviceModel(cfg, W, dev)
-    n = args.inputs_per_gpu
+    llama = cfg.arch == "llama"
+    n = args.inputs_per_gpu or (256 if llama else 8192)
+    if llama:
+        # weights generated layer by layer straight into HBM (13.5 GB bf16);
+        # one KV cache slot per sequence (token), ctx positions pre-filled with
+        # N(0, 1) on the device (same recipe as e3data.make_kv, device stream)
+        layers = (e3data.make_layer(cfg, l) for l in range(cfg.layers))
+        ramp = e3data.make_ramp(cfg, 0)
+        kv = api.KVCache(cfg, n, cfg.ctx + 1, n * world, dev)
+        g = torch.Generator(device=dev)
+        g.manual_seed(1234 + rank)
+        for t in kv.k + kv.v:
+            t[:, :, :cfg.ctx].normal_(generator=g)
+        kv.slot_of_id.copy_(torch.arange(n * world, device=dev, dtype=torch.int32) % n)
+        model = api.DeviceModel(cfg, {"layers": layers, "ramps": [ramp] * cfg.n_ramps}, dev, kv=kv)
+    else:
+        W = e3data.make_weights(cfg)
+        model = api.DeviceModel(cfg, W, dev)
     stream = torch.cuda.Stream(dev)
+    model_bytes = sum(t.numel() * 2 for w in model.layers for t in w.values())
+    kv_bytes = sum(t.numel() * 2 for t in (model.kv.k + model.kv.v)) if llama else 0
     stage_mode = args.mode == "stage" and world > 1
+    if stage_mode and llama:
+        raise SystemExit("--mode stage: encoder configs only (the llama KV cache is per GPU)")
     if stage_mode:
         # stages on different GPUs: chunk c of the job enters at the stage-0
         # replica owning it; ids are global so exits land at their input's slot
@@ -363,7 +413,9 @@ def main():
                        "seq_len": cfg.seq, "ramps": cfg.n_ramps, "test": cfg.test, "plan": plan_name,
                        "inputs_per_step_per_gpu": n,
                        "parallelism": (f"stage x{world}" if stage_mode else f"replica x{world}") if world > 1 else "1 GPU",
-                       "l2": "inputs larger than L2 (%.2f GB per step per GPU)" % (n * cfg.seq * cfg.hidden * 2 / 1e9)},
+                       "l2": ("weights %.1f GB + KV cache %.1f GB streamed per step, >> L2" % (
+                           model_bytes / 1e9, kv_bytes / 1e9) if llama else
+                           "inputs larger than L2 (%.2f GB per step per GPU)" % (n * cfg.seq * cfg.hidden * 2 / 1e9))},
             "roofline": roof,
             "whole_path_roofline_frac": round(whole, 4),
             "per_kernel": per_kernel,

@@ -32,15 +32,19 @@ constexpr int D = 64;          // head dim
 constexpr int QT = 128;        // query rows per item
 constexpr int kThreads = 256;  // 8 warps: two threads per query row
 
+// SKV = keys per tile: S rounded up to 128 or, above 128, to a multiple of 32
+// (S = 197 -> 224: 12 % fewer masked exponentials than 256 and small enough
+// K/V tiles to double-buffer the next item's loads)
 template <int SKV>
 struct ACfg {
   static constexpr int kQ = QT * D * 2;                  // 16 KB
-  static constexpr int kKV = SKV * D * 2;                // 16 / 32 KB
-  static constexpr int kP = QT * SKV * 2;                // 32 / 64 KB
+  static constexpr int kKV = SKV * D * 2;                // 16 .. 32 KB
+  static constexpr int kP = ((SKV + 63) / 64) * QT * 128;   // bf16 P in 64-key SW128 blocks
   static constexpr int kBuf = kQ + 2 * kKV;              // Q | K | V
-  static constexpr int kNBuf = (SKV == 128) ? 2 : 1;     // double buffer when it fits
   static constexpr bool kPInQK = (kP <= kQ + kKV);       // P overwrites the dead Q|K tiles
-  static constexpr int kSmem = kNBuf * kBuf + (kPInQK ? 0 : kP) + 1024 + 64 + 2 * 2 * QT * 4;
+  static constexpr int kExtra = 1024 + 64 + 2 * 2 * QT * 4;
+  static constexpr int kNBuf = (2 * kBuf + (kPInQK ? 0 : kP) + kExtra <= 232448) ? 2 : 1;   // double buffer if it fits
+  static constexpr int kSmem = kNBuf * kBuf + (kPInQK ? 0 : kP) + kExtra;
   static constexpr int kTmemCols = SKV <= 128 ? 128 : 256;   // S, later O (64 columns)
 };
 
@@ -49,7 +53,7 @@ __global__ void __launch_bounds__(kThreads)
     attn_tc_kernel(const __grid_constant__ CUtensorMap tq, const __grid_constant__ CUtensorMap tkv,
                    const __grid_constant__ CUtensorMap tctx, int S, int H, int heads, int n_items) {
   using CF = ACfg<SKV>;
-  constexpr int HALF = SKV / 2;     // keys per thread
+  constexpr int NCH = SKV / 32;     // 32-key chunks; thread half 0 takes the first ceil(NCH/2)
   extern __shared__ uint8_t smem_raw[];
   uint8_t *smem = reinterpret_cast<uint8_t *>((reinterpret_cast<uintptr_t>(smem_raw) + 1023) & ~uintptr_t(1023));
   uint8_t *pbuf_sep = smem + CF::kNBuf * CF::kBuf;      // only when !kPInQK
@@ -136,10 +140,11 @@ __global__ void __launch_bounds__(kThreads)
     mbar_wait(bar_s, sphase);
     sphase ^= 1;
     tc_fence_after();
-    const int c_begin = khalf * HALF;
+    const int c_begin = khalf ? ((NCH + 1) / 2) * 32 : 0;
+    const int c_end = khalf ? SKV : ((NCH + 1) / 2) * 32;
     float mx = -INFINITY;
 #pragma unroll 1
-    for (int c = c_begin; c < c_begin + HALF; c += 32) {
+    for (int c = c_begin; c < c_end; c += 32) {
       uint32_t r[32];
       tmem_ld32(tbase + lane_off + c, r);
       tmem_wait_ld();
@@ -160,7 +165,7 @@ __global__ void __launch_bounds__(kThreads)
     float l4[4] = {0.f, 0.f, 0.f, 0.f};
     uint8_t *prow = sP + row * 128;
 #pragma unroll 1
-    for (int c = c_begin; c < c_begin + HALF; c += 32) {
+    for (int c = c_begin; c < c_end; c += 32) {
       uint32_t r[32];
       tmem_ld32(tbase + lane_off + c, r);
       tmem_wait_ld();
@@ -253,7 +258,7 @@ e3_status launch_attn(const AttnMaps &m, int B, int S, int H, int heads, cudaStr
     attr_done = true;
   }
   const int n_items = B * heads * ((S + QT - 1) / QT);
-  const int per_sm = (SKV == 128) ? 2 : 1;
+  const int per_sm = (2 * ACfg<SKV>::kSmem <= 232448) ? 2 : 1;
   const int grid = n_items < per_sm * sms ? n_items : per_sm * sms;
   E3_CUDA_TRY(launch_k(kern, dim3(grid), dim3(kThreads), ACfg<SKV>::kSmem, st, m.q, m.kv, m.ctx, S, H, heads,
                        n_items));
@@ -265,7 +270,7 @@ e3_status launch_attn(const AttnMaps &m, int B, int S, int H, int heads, cudaStr
 }  // namespace
 
 e3_status attn_tmaps(AttnMaps *m, const void *qkv, const void *ctx, int B, int S, int H) {
-  m->skv = S <= 128 ? 128 : 256;
+  m->skv = S <= 128 ? 128 : ((S + 31) / 32) * 32;
   const uint64_t W3 = 3ull * H;
   e3_status s = make_tmap_3d(&m->q, qkv, W3, (uint64_t)S, (uint64_t)B, W3, W3 * S, D, QT, 1);
   if (s == E3_OK) s = make_tmap_3d(&m->kv, qkv, W3, (uint64_t)S, (uint64_t)B, W3, W3 * S, D, (uint32_t)m->skv, 1);
@@ -275,8 +280,15 @@ e3_status attn_tmaps(AttnMaps *m, const void *qkv, const void *ctx, int B, int S
 }
 
 e3_status attn_run(const AttnMaps &m, int B, int S, int H, int heads, cudaStream_t st) {
-  if (m.skv == 128) return launch_attn<128>(m, B, S, H, heads, st);
-  return launch_attn<256>(m, B, S, H, heads, st);
+  switch (m.skv) {
+    case 128: return launch_attn<128>(m, B, S, H, heads, st);
+    case 160: return launch_attn<160>(m, B, S, H, heads, st);
+    case 192: return launch_attn<192>(m, B, S, H, heads, st);
+    case 224: return launch_attn<224>(m, B, S, H, heads, st);
+    case 256: return launch_attn<256>(m, B, S, H, heads, st);
+  }
+  set_error("attention: S > 256");
+  return E3_EUNSUPPORTED;
 }
 
 }  // namespace e3

@@ -73,7 +73,8 @@ def test_gemm_full_bert_base_shapes_sampled(api, N, K, epi):
 
 
 @pytest.mark.parametrize("B,S,H,heads", [(2, 32, 128, 2), (3, 128, 768, 12), (2, 197, 128, 2),
-                                         (1, 256, 64, 1), (2, 77, 192, 3)])
+                                         (1, 256, 64, 1), (2, 77, 192, 3), (3, 150, 128, 2), (2, 170, 64, 1),
+                                         (80, 197, 128, 2), (90, 128, 128, 2)])
 def test_attention_matches_oracle(api, B, S, H, heads):
     from oracle.encoder import attention
     rng = np.random.default_rng(S * H)
