@@ -29,6 +29,14 @@ typedef enum {
 e3_status e3_op_gemm(void *stream, const void *A, int64_t lda, const void *W, const void *bias,
                      const void *resid, void *C, int32_t M, int32_t N, int32_t K, int32_t epilogue);
 
+/* Decode-shaped GEMM of the LLaMA split (a8; gemm_dec.cu): Y[T,N] =
+ * epi(X[T,K] W[N,K]^T), bf16 in, fp32 accumulate, bf16 out, T in {32, 64,
+ * 128} tokens, K % 64 == 0.  epilogue: 0 plain, 1 + R[T,N] (residual),
+ * 2 SwiGLU: Y[T,N] = SiLU(X W^T) * (X W2^T) with W = W_gate, W2 = W_up [N,K]
+ * (N % 64 == 0).  Stream-K scratch is allocated on the stream per call. */
+e3_status e3_op_dec_gemm(void *stream, const void *X, int32_t T, const void *W, const void *W2, int32_t N,
+                         int32_t K, int32_t epilogue, const void *R, void *Y);
+
 /* Self-attention (a2) on tcgen05: qkv [B*S, 3H] (q | k | v, head h owning
  * columns h*64..h*64+63 of each third) -> ctx [B*S, H].  head_dim 64,
  * S <= 256, no mask.  softmax(q k^T / sqrt(64)) v with the rounding contract

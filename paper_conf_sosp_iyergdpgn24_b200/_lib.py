@@ -10,7 +10,7 @@ import ctypes as C
 import os
 
 HERE = os.path.dirname(os.path.abspath(__file__))
-LIB_PATH = os.path.join(HERE, "libe3.so")
+LIB_PATH = os.environ.get("E3_LIB_PATH") or os.path.join(HERE, "libe3.so")   # override: diagnostics only
 
 E3_MAX_RAMPS = 64
 E3_MAX_SPLITS = 64
@@ -98,6 +98,7 @@ SIGNATURES = {
                                   C.POINTER(I64)]),
     "e3_pipeline_trace": (I32, [P, P, P, P, I64, C.POINTER(I64)]),
     "e3_op_gemm": (I32, [P, P, I64, P, P, P, P, I32, I32, I32, I32]),
+    "e3_op_dec_gemm": (I32, [P, P, I32, P, P, I32, I32, I32, P, P]),
     "e3_op_attention": (I32, [P, P, P, I32, I32, I32, I32]),
     "e3_op_layernorm": (I32, [P, P, P, P, P, I32, I32, C.c_float]),
     "e3_op_ramp": (I32, [P, I32, P, P, I32, I32, I32, I32, C.POINTER(RampWeights), I32, C.c_float, I32,

@@ -265,6 +265,17 @@ class ops:
     """Kernel-level entry points (include/e3_ops.h)."""
 
     @staticmethod
+    def dec_gemm(X, W, epilogue="store", W2=None, resid=None, out=None, stream=None):
+        """Decode GEMM (swap-AB tcgen05, stream-K): X [T,K] bf16, W [N,K]."""
+        T, K = X.shape
+        N = W.shape[0]
+        out = torch.empty((T, N), dtype=torch.bfloat16, device=X.device) if out is None else out
+        epi = {"store": 0, "resid": 1, "swiglu": 2}[epilogue]
+        check(lib.e3_op_dec_gemm(_stream(stream), _ptr(X), T, _ptr(W), _ptr(W2), N, K, epi, _ptr(resid), _ptr(out)),
+              "e3_op_dec_gemm")
+        return out
+
+    @staticmethod
     def gemm(A, W, bias, epilogue="bias", resid=None, out=None, stream=None):
         M, K = A.shape
         N = W.shape[0]

@@ -243,22 +243,25 @@ e3_status ln_compact_run(const void *y, const int64_t *id, const uint8_t *alive,
     set_error("ln_compact: need B <= 4096, H % 8 == 0, H <= 4096");
     return E3_EUNSUPPORTED;
   }
-  // kRowsInFlight token rows per warp on a full batch
+  // kRowsInFlight token rows per warp on a full batch, but never more CTAs
+  // than are resident at once: a second wave would repeat the whole latency
+  // chain (scan, loads, stores) -- 4 waves cost 12.8 us at BB (r01 ncu)
   int64_t grid = ((int64_t)B * S + 8 * kRowsInFlight - 1) / (8 * kRowsInFlight);
-  if (grid > 4 * sms) grid = 4 * sms;
-  if (grid < 1) grid = 1;
   auto *yp = reinterpret_cast<const __nv_bfloat16 *>(y);
   auto *gp = reinterpret_cast<const __nv_bfloat16 *>(g);
   auto *bp = reinterpret_cast<const __nv_bfloat16 *>(b);
   const int vpl = (H / 8 + 31) / 32;
 #define E3_LNC(V)                                                                                          \
   do {                                                                                                     \
-    if (gp)                                                                                                \
-      E3_CUDA_TRY(launch_k(ln_compact_kernel<V, true>, dim3((unsigned)grid), dim3(kThreads), 0, st, yp, id, \
-                           alive, B, S, H, gp, bp, eps, dst, n_surv_dev));                                 \
-    else                                                                                                   \
-      E3_CUDA_TRY(launch_k(ln_compact_kernel<V, false>, dim3((unsigned)grid), dim3(kThreads), 0, st, yp,   \
-                           id, alive, B, S, H, gp, bp, eps, dst, n_surv_dev));                             \
+    auto kern = gp ? ln_compact_kernel<V, true> : ln_compact_kernel<V, false>;                             \
+    static int occ_[2] = {0, 0};                                                                           \
+    int &occ = occ_[gp ? 1 : 0];                                                                           \
+    if (!occ) E3_CUDA_TRY(cudaOccupancyMaxActiveBlocksPerMultiprocessor(&occ, kern, kThreads, 0));        \
+    if (occ < 1) occ = 1;                                                                                  \
+    if (grid > (int64_t)occ * sms) grid = (int64_t)occ * sms;                                              \
+    if (grid < 1) grid = 1;                                                                                \
+    E3_CUDA_TRY(launch_k(kern, dim3((unsigned)grid), dim3(kThreads), 0, st, yp, id, alive, B, S, H, gp, bp, \
+                         eps, dst, n_surv_dev));                                                           \
   } while (0)
   if (vpl <= 1) E3_LNC(1);
   else if (vpl <= 3) E3_LNC(3);

@@ -9,11 +9,12 @@
 //     tokens are its N side: D[128, T] = W_tile . X^T with both operands
 //     K-major in 128-byte-swizzled smem, tcgen05.mma.cta_group::1 M=128 N=T.
 //     No padding of T up to a 128-row tile, no wasted tensor work.
-//   * persistent CTAs (one per SM) walk UNITS = (128-row tile, K slice);
-//     split-K (ks slices) keeps >= 148 units in flight for the narrow
-//     matrices (W_o, W_down: 32 tiles).  A slice's fp32 partial goes to a
-//     workspace; the last CTA of a tile (atomic ticket) sums the ks partials
-//     in slice order (deterministic) and runs the epilogue.
+//   * stream-K: one CTA per SM, each taking an equal contiguous range of the
+//     (tile, 64-wide k-block) iterations, so every SM streams the same weight
+//     bytes (a tile-granular split left SMs idle: W_o / W_down have only 32
+//     tiles).  Tiles split between CTAs are finished by their last
+//     contributor (atomic ticket), summing the contributors' fp32 partials in
+//     contributor order (deterministic).
 //   * warp 0 = TMA producer: the first stages' W boxes are issued BEFORE
 //     griddepcontrol.wait (weights never depend on the previous kernel), so
 //     the weight stream starts while the previous kernel drains; warp 1 = one
@@ -54,6 +55,25 @@ struct DCfg {
 
 __device__ __forceinline__ void epi_bar() { asm volatile("bar.sync 1, 128;" ::: "memory"); }
 
+// Stream-K work split: the tiles x (K / 64) k-block iterations are cut into
+// gridDim.x equal contiguous ranges, one per CTA, so every SM streams the same
+// number of weight bytes (with 96..250 tiles per launch a tile-granular split
+// leaves up to half the SMs idle for the last wave).  A CTA's range crosses at
+// most a few tiles; a tile computed by one CTA is finished in place, a tile
+// shared by several CTAs is reduced by its last contributor (atomic ticket)
+// from the contributors' fp32 partials in contributor order (deterministic).
+struct SK {
+  long total;   // tiles * nkb
+  int nkb, G;
+  __device__ long start(int c) const { return (long)c * total / G; }
+  __device__ int owner(long i) const {   // CTA whose range holds iteration i
+    int c = (int)((i * G) / total);
+    while (c + 1 < G && start(c + 1) <= i) ++c;
+    while (c > 0 && start(c) > i) --c;
+    return c;
+  }
+};
+
 template <int T, int EPI>
 __global__ void __launch_bounds__(kDThreads, 1)
     gemm_dec_kernel(const __grid_constant__ CUtensorMap tmW, const __grid_constant__ CUtensorMap tmW2,
@@ -77,8 +97,11 @@ __global__ void __launch_bounds__(kDThreads, 1)
 
   const int warp = warp_id(), lane = lane_id();
   const int tiles = (EPI == E3_DEC_SWIGLU) ? a.N / 64 : (a.N + DM - 1) / DM;
-  const int units = tiles * a.ks;
-  const int nkb = a.K / DK / a.ks;
+  SK sk;
+  sk.nkb = a.K / DK;
+  sk.total = (long)tiles * sk.nkb;
+  sk.G = gridDim.x;
+  const long my0 = sk.start(blockIdx.x), my1 = sk.start(blockIdx.x + 1);
 
   if (warp == 0 && lane == 0) {
     tma_prefetch(&tmW);
@@ -105,51 +128,34 @@ __global__ void __launch_bounds__(kDThreads, 1)
   if (warp == 0) {
     // ------------------------------------------------------- TMA producer
     if (lane == 0) {
-      auto coords = [&](int it, int &n0, int &k0) {   // it-th (unit, kb) of this CTA
-        const int u = blockIdx.x + (it / nkb) * gridDim.x;
-        const int kb = it % nkb;
-        const int tile = u / a.ks, ksl = u % a.ks;
-        n0 = (EPI == E3_DEC_SWIGLU) ? tile * 64 : tile * DM;
-        k0 = (ksl * nkb + kb) * DK;
-        return u < units;
+      const int total = (int)(my1 - my0);
+      auto load_w = [&](int it, int st) {
+        const long i = my0 + it;
+        const int tile = (int)(i / sk.nkb), k0 = (int)(i % sk.nkb) * DK;
+        if (EPI == E3_DEC_SWIGLU) {
+          tma_load_2d(sW + st * CF::kWBytes, &tmW, &full[st], k0, tile * 64);
+          tma_load_2d(sW + st * CF::kWBytes + CF::kWBytes / 2, &tmW2, &full[st], k0, tile * 64);
+        } else {
+          tma_load_2d(sW + st * CF::kWBytes, &tmW, &full[st], k0, tile * DM);
+        }
       };
-      int my_units = 0;
-      for (int u = blockIdx.x; u < units; u += gridDim.x) ++my_units;
-      const int total = my_units * nkb;
       const int pre = total < S ? total : S;
       // weights first: they do not depend on the previous kernel
       for (int it = 0; it < pre; ++it) {
-        int n0, k0;
-        coords(it, n0, k0);
         mbar_expect_tx(&full[it], CF::kStageBytes);
-        if (EPI == E3_DEC_SWIGLU) {
-          tma_load_2d(sW + it * CF::kWBytes, &tmW, &full[it], k0, n0);
-          tma_load_2d(sW + it * CF::kWBytes + CF::kWBytes / 2, &tmW2, &full[it], k0, n0);
-        } else {
-          tma_load_2d(sW + it * CF::kWBytes, &tmW, &full[it], k0, n0);
-        }
+        load_w(it, it);
       }
       pdl_wait();
       pdl_trigger();
-      for (int it = 0; it < pre; ++it) {
-        int n0, k0;
-        coords(it, n0, k0);
-        tma_load_2d(sX + it * CF::kXBytes, &tmX, &full[it], k0, 0);
-      }
+      for (int it = 0; it < pre; ++it)
+        tma_load_2d(sX + it * CF::kXBytes, &tmX, &full[it], (int)((my0 + it) % sk.nkb) * DK, 0);
       int stage = pre % S;
       uint32_t phase = (pre == S) ? 1 : 0;
       for (int it = pre; it < total; ++it) {
-        int n0, k0;
-        coords(it, n0, k0);
         mbar_wait(&empty[stage], phase ^ 1);
         mbar_expect_tx(&full[stage], CF::kStageBytes);
-        if (EPI == E3_DEC_SWIGLU) {
-          tma_load_2d(sW + stage * CF::kWBytes, &tmW, &full[stage], k0, n0);
-          tma_load_2d(sW + stage * CF::kWBytes + CF::kWBytes / 2, &tmW2, &full[stage], k0, n0);
-        } else {
-          tma_load_2d(sW + stage * CF::kWBytes, &tmW, &full[stage], k0, n0);
-        }
-        tma_load_2d(sX + stage * CF::kXBytes, &tmX, &full[stage], k0, 0);
+        load_w(it, stage);
+        tma_load_2d(sX + stage * CF::kXBytes, &tmX, &full[stage], (int)((my0 + it) % sk.nkb) * DK, 0);
         if (++stage == S) { stage = 0; phase ^= 1; }
       }
     }
@@ -163,23 +169,26 @@ __global__ void __launch_bounds__(kDThreads, 1)
       uint32_t phase = 0;
       int acc = 0;
       uint32_t acc_phase = 0;
-      for (int u = blockIdx.x; u < units; u += gridDim.x) {
+      for (long i = my0; i < my1;) {                 // one segment = this CTA's part of one tile
+        const int tile = (int)(i / sk.nkb);
+        const long seg_end = min(my1, (long)(tile + 1) * sk.nkb);
         mbar_wait(&tempty[acc], acc_phase ^ 1);
         tc_fence_after();
         const uint32_t d_tmem = tmem_base + acc * T;
-        for (int kb = 0; kb < nkb; ++kb) {
+        for (long j = i; j < seg_end; ++j) {
           mbar_wait(&full[stage], phase);
           tc_fence_after();
           const uint64_t da = smem_desc_sw128(smem_u32(sW + stage * CF::kWBytes), 16, 1024);
           const uint64_t db = smem_desc_sw128(smem_u32(sX + stage * CF::kXBytes), 16, 1024);
 #pragma unroll
           for (int k = 0; k < DK / 16; ++k)
-            tc_mma_f16(d_tmem, da + (uint64_t)(2 * k), db + (uint64_t)(2 * k), idesc, (kb | k) != 0);
+            tc_mma_f16(d_tmem, da + (uint64_t)(2 * k), db + (uint64_t)(2 * k), idesc, (j != i) || k != 0);
           tc_commit(&empty[stage]);
           if (++stage == S) { stage = 0; phase ^= 1; }
         }
         tc_commit(&tfull[acc]);
         if (++acc == 2) { acc = 0; acc_phase ^= 1; }
+        i = seg_end;
       }
     }
   } else {
@@ -205,8 +214,12 @@ __global__ void __launch_bounds__(kDThreads, 1)
     }
     int acc = 0;
     uint32_t acc_phase = 0;
-    for (int u = blockIdx.x; u < units; u += gridDim.x) {
-      const int tile = u / a.ks;
+    for (long i = my0; i < my1;) {
+      const int tile = (int)(i / sk.nkb);
+      const long t0i = (long)tile * sk.nkb, t1i = t0i + sk.nkb;
+      const long seg_end = min(my1, t1i);
+      const bool whole = (i == t0i) && (seg_end == t1i);
+      i = seg_end;
       mbar_wait(&tfull[acc], acc_phase);
       tc_fence_after();
       const uint32_t taddr = tmem_base + ((uint32_t)(q * 32) << 16) + acc * T;
@@ -224,37 +237,85 @@ __global__ void __launch_bounds__(kDThreads, 1)
       if (++acc == 2) { acc = 0; acc_phase ^= 1; }
       epi_bar();
 
-      if (a.ks > 1) {
-        // split-K: publish this slice, the tile's last arrival reduces in slice order
-        float *part = a.part + (size_t)u * T * DM;
-        for (int t = 0; t < T; ++t) part[t * DM + r] = sE[r * P + t];
+      if (!whole) {
+        // shared tile: publish this contributor's partial; the tile's last
+        // arrival sums the contributors' partials in contributor order
+        const int c_first = sk.owner(t0i), c_last = sk.owner(t1i - 1);
+        const int slot = (int)blockIdx.x - c_first, ncon = c_last - c_first + 1;
+        // partial layout [tile][slot][T/4][row] of float4 (4 tokens): each
+        // thread moves its row's T values as 16-byte vectors and a warp's
+        // access is 512 contiguous bytes
+        float4 *part = reinterpret_cast<float4 *>(a.part) + ((size_t)tile * a.max_contrib + slot) * (T / 4) * DM + r;
+#pragma unroll
+        for (int i = 0; i < T / 4; ++i)
+          part[(size_t)i * DM] =
+              make_float4(sE[r * P + 4 * i], sE[r * P + 4 * i + 1], sE[r * P + 4 * i + 2], sE[r * P + 4 * i + 3]);
         __threadfence();
         epi_bar();
         if (et == 0) {
           const unsigned prev = atomicAdd(&a.tickets[tile], 1u);
-          *s_last = (prev == (unsigned)(a.ks - 1));
+          *s_last = (prev == (unsigned)(ncon - 1));
           if (*s_last) a.tickets[tile] = 0;   // ready for the next launch
         }
         epi_bar();
         if (!*s_last) continue;
         __threadfence();
-        const float *base = a.part + (size_t)tile * a.ks * T * DM;
-        for (int t = 0; t < T; ++t) {
-          float s = 0.f;
-          for (int j = 0; j < a.ks; ++j) s += __ldcg(base + ((size_t)j * T + t) * DM + r);
-          sE[r * P + t] = s;
+        // sum the contributors' partials in contributor order; contributor
+        // j+1's loads are in flight while j is accumulated (one round trip
+        // per contributor; a serial load -> add chain cost ~10 us, r01)
+        const float4 *base = reinterpret_cast<const float4 *>(a.part) + (size_t)tile * a.max_contrib * (T / 4) * DM + r;
+        const size_t cstride = (size_t)DM * T / 4;   // float4s between contributors
+#pragma unroll 1
+        for (int h = 0; h < T / 64 + (T % 64 ? 1 : 0); ++h) {
+          constexpr int NV = (T < 64 ? T : 64) / 4;
+          float4 acc4[NV], cur[NV], nxt[NV];
+#pragma unroll
+          for (int i = 0; i < NV; ++i) {
+            acc4[i] = make_float4(0.f, 0.f, 0.f, 0.f);
+            cur[i] = __ldcg(base + (size_t)(h * NV + i) * DM);
+          }
+#pragma unroll 1
+          for (int j = 0; j < ncon; ++j) {
+            if (j + 1 < ncon) {
+#pragma unroll
+              for (int i = 0; i < NV; ++i) nxt[i] = __ldcg(base + (j + 1) * cstride + (size_t)(h * NV + i) * DM);
+            }
+#pragma unroll
+            for (int i = 0; i < NV; ++i) {
+              acc4[i].x += cur[i].x;
+              acc4[i].y += cur[i].y;
+              acc4[i].z += cur[i].z;
+              acc4[i].w += cur[i].w;
+              cur[i] = nxt[i];
+            }
+          }
+#pragma unroll
+          for (int i = 0; i < NV; ++i) {
+            const int t = h * 64 + 4 * i;
+            sE[r * P + t] = acc4[i].x;
+            sE[r * P + t + 1] = acc4[i].y;
+            sE[r * P + t + 2] = acc4[i].z;
+            sE[r * P + t + 3] = acc4[i].w;
+          }
         }
         epi_bar();
       }
 
       // ---------------------------------------------------- final epilogue
+      // global loads of a token batch are issued together before its stores
+      // (a load -> store chain per token cost ~1 us x T per launch)
       if (EPI == E3_DEC_STORE || EPI == E3_DEC_RESID) {
         const int n = tile * DM + r;
         if (n < a.N) {
-          for (int t = 0; t < T; ++t) {
-            float v = sE[r * P + t];
-            if (EPI == E3_DEC_RESID) v += bf2f(a.R[(size_t)t * a.ldo + n]);
-            a.Y[(size_t)t * a.ldo + n] = __float2bfloat16_rn(v);
+#pragma unroll 1
+          for (int tb = 0; tb < T; tb += 32) {
+            float rv[32];
+#pragma unroll
+            for (int ii = 0; ii < 32; ++ii)
+              rv[ii] = (EPI == E3_DEC_RESID) ? bf2f(a.R[(size_t)(tb + ii) * a.ldo + n]) : 0.f;
+#pragma unroll
+            for (int ii = 0; ii < 32; ++ii)
+              a.Y[(size_t)(tb + ii) * a.ldo + n] = __float2bfloat16_rn(sE[r * P + tb + ii] + rv[ii]);
           }
         }
       } else if (EPI == E3_DEC_SWIGLU) {
@@ -270,20 +331,28 @@ __global__ void __launch_bounds__(kDThreads, 1)
         const int hq = tile;
         const bool is_q = hq < a.nh, is_k = !is_q && hq < a.nh + a.kvh;
         const int j = r & 63;
-        for (int t = 0; t < T; ++t) {
-          float v = sE[r * P + t];
-          if (is_q || is_k) {
-            const float pr = sE[(r ^ 64) * P + t];
-            const float2 cs = a.rope[(size_t)sPos[t] * 64 + j];
-            v = (r < 64) ? fmaf(v, cs.x, -pr * cs.y) : fmaf(v, cs.x, pr * cs.y);
-          }
-          const __nv_bfloat16 o = __float2bfloat16_rn(v);
-          if (is_q) {
-            a.Y[(size_t)t * a.ldo + hq * 128 + r] = o;
-          } else if (sSlot[t] >= 0) {
-            const int kh = is_k ? hq - a.nh : hq - a.nh - a.kvh;
-            __nv_bfloat16 *cache = is_k ? a.kc : a.vc;
-            cache[(((size_t)sSlot[t] * a.kvh + kh) * a.max_ctx + sPos[t]) * 128 + r] = o;
+#pragma unroll 1
+        for (int tb = 0; tb < T; tb += 16) {
+          float2 cs[16];
+#pragma unroll
+          for (int ii = 0; ii < 16; ++ii)
+            cs[ii] = (is_q || is_k) ? a.rope[(size_t)sPos[tb + ii] * 64 + j] : make_float2(1.f, 0.f);
+#pragma unroll
+          for (int ii = 0; ii < 16; ++ii) {
+            const int t = tb + ii;
+            float v = sE[r * P + t];
+            if (is_q || is_k) {
+              const float pr = sE[(r ^ 64) * P + t];
+              v = (r < 64) ? fmaf(v, cs[ii].x, -pr * cs[ii].y) : fmaf(v, cs[ii].x, pr * cs[ii].y);
+            }
+            const __nv_bfloat16 o = __float2bfloat16_rn(v);
+            if (is_q) {
+              a.Y[(size_t)t * a.ldo + hq * 128 + r] = o;
+            } else if (sSlot[t] >= 0) {
+              const int kh = is_k ? hq - a.nh : hq - a.nh - a.kvh;
+              __nv_bfloat16 *cache = is_k ? a.kc : a.vc;
+              cache[(((size_t)sSlot[t] * a.kvh + kh) * a.max_ctx + sPos[t]) * 128 + r] = o;
+            }
           }
         }
       } else if (EPI == E3_DEC_LOGITS) {
@@ -348,20 +417,18 @@ e3_status dec_launch_epi(const DecMaps &m, const DecArgs &a, int grid, cudaStrea
 
 int dec_tiles(int N, int epi) { return epi == E3_DEC_SWIGLU ? N / 64 : (N + DM - 1) / DM; }
 
-int dec_pick_ks(int N, int K, int epi, int sms) {
-  // minimise (units per CTA) x (K per unit + split-K traffic in K columns);
-  // a partial [T x 128] fp32 written and read back ~ 256 columns of W
-  const int tiles = dec_tiles(N, epi);
-  int best = 1;
-  long best_cost = -1;
-  for (int ks = 1; ks <= 16; ++ks) {
-    if (K % (ks * DK)) continue;
-    const long units = (long)tiles * ks;
-    const long per = (units + sms - 1) / sms;
-    const long cost = per * (K / ks + (ks > 1 ? 256 : 0));
-    if (best_cost < 0 || cost < best_cost) { best = ks; best_cost = cost; }
-  }
-  return best;
+static int dec_grid(int N, int K, int epi, int sms) {
+  const long total = (long)dec_tiles(N, epi) * (K / DK);
+  return (int)(total < sms ? total : sms);
+}
+
+int dec_max_contrib(int N, int K, int epi, int sms) {
+  // every CTA's range holds >= floor(total / G) iterations, so a tile of nkb
+  // iterations meets at most ceil(nkb / that) + 1 ranges
+  const long nkb = K / DK, total = (long)dec_tiles(N, epi) * nkb;
+  const long G = dec_grid(N, K, epi, sms);
+  const long per = total / G;
+  return (int)((nkb + per - 1) / per + 1);
 }
 
 e3_status dec_tmaps(DecMaps *m, const void *X, int T, int K, const void *W, const void *W2, int N, int epi) {
@@ -373,8 +440,7 @@ e3_status dec_tmaps(DecMaps *m, const void *X, int T, int K, const void *W, cons
 }
 
 e3_status dec_run(const DecMaps &m, const DecArgs &a, int sms, cudaStream_t st) {
-  const int units = dec_tiles(a.N, a.epi) * a.ks;
-  const int grid = units < sms ? units : sms;
+  const int grid = dec_grid(a.N, a.K, a.epi, sms);
   switch (a.T) {
     case 32: return dec_launch_epi<32>(m, a, grid, st);
     case 64: return dec_launch_epi<64>(m, a, grid, st);

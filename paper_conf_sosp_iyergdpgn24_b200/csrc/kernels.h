@@ -74,14 +74,15 @@ struct DecMaps {
   CUtensorMap x;    // X [T,K], box T x 64
 };
 struct DecArgs {
-  int T, N, K, ks, epi;
+  int T, N, K, epi;
+  int max_contrib;          // partial slots per tile (dec_max_contrib)
   const __nv_bfloat16 *R;   // RESID: residual [T, ldo]
   __nv_bfloat16 *Y;         // STORE / RESID / SWIGLU / QKV (q): [T, ldo]
   int ldo;
   float *Z;                 // LOGITS: [T, N]
   float4 *stats;            // LOGITS: [tiles][T]
-  float *part;              // split-K partials [tiles * ks][T][128]
-  unsigned *tickets;        // split-K tickets [tiles], zero between launches
+  float *part;              // stream-K partials [tiles][max_contrib][T/4][128 rows] of float4
+  unsigned *tickets;        // stream-K tickets [tiles], zero between launches
   // QKV_ROPE: this layer's cache and the tokens' slots / positions
   int nh, kvh, max_ctx;
   __nv_bfloat16 *kc, *vc;
@@ -94,7 +95,7 @@ struct DecArgs {
   const int32_t *pos_of_slot;
 };
 int dec_tiles(int N, int epi);
-int dec_pick_ks(int N, int K, int epi, int sms);
+int dec_max_contrib(int N, int K, int epi, int sms);
 e3_status dec_tmaps(DecMaps *m, const void *X, int T, int K, const void *W, const void *W2, int N, int epi);
 e3_status dec_run(const DecMaps &m, const DecArgs &a, int sms, cudaStream_t st);
 e3_status rope_table(int max_ctx, int head_dim, double theta, float2 **out);

@@ -6,27 +6,29 @@
 // exit test (R3/R4/R12): max softmax(z) > tau, or
 // entropy(softmax(z)) < tau; the model's last ramp exits every row (R6).
 //
-// One launch; grid (CS, ceil(B / 16)) in clusters of CS = 8 (16 for H > 768)
-// CTAs -- one cluster per group of 16 rows, CTA rank r owning H/CS pooler
-// outputs, one warp per 8 of them:
-//   stage    the H/CS W_p rows of the tile by cp.async into padded smem (row
-//            pitch H + 8 bf16: conflict-free fragments) and the 16 CLS rows:
-//            either copied (cp.async) or, at a split's last layer, read
-//            PRE-LayerNorm and normalised here by the shared warp-per-row LN
-//            (ln_row.cuh) -- bit-identical to what the fused LN + compaction
-//            writes for the survivors, and no full LN2 pass is needed;
-//   pooler   warp w owns outputs 8w..8w+7 of the tile: mma.sync m16n8k16
-//            bf16 -> fp32 over K = H (a 16 x H/CS x H GEMM per CTA is far too
-//            small for a tcgen05 tile; the tensor pipe is still the one used);
-//   partial  p = tanh(acc + b_p) stays in registers and is immediately folded
-//            into partial logits sum_{o in tile} p[b,o] W_c[c,o], reduced over
-//            the quad with __shfl_xor_sync and over the warps in smem, then
-//            stored into rank 0's shared memory (DSMEM) -- no global
-//            partials, no float atomics, no grid-wide ticket;
-//   decide   after one cluster barrier rank 0 sums the CS partials per (row,
-//            class) in fixed rank order, then softmax / max-prob / entropy,
-//            argmax (lowest index on ties), threshold test, exit record by
-//            input id and the alive flag.
+// One launch; grid (16, ceil(B / 16)): one cluster of 16 CTAs per group of
+// 16 rows (the mma M), CTA rank r owning pooler outputs [r*TN, (r+1)*TN),
+// TN = H/16.  The work is spread over B/16 x 16 SMs (BB: 64) -- measured on
+// B200 the ramp is instruction-issue-bound per SM, so fewer, fatter CTAs
+// (one cluster for the whole batch) were 1.6x slower:
+//   stage    the CTA's TN W_p rows by cp.async into padded smem (row pitch
+//            H + 8 bf16: conflict-free fragments) BEFORE the PDL wait;
+//   CLS      distributed LayerNorm: CTA rank r normalises CLS row r of the
+//            group alone (one warp; at a split's last layer the rows arrive
+//            PRE-LayerNorm and the shared warp-per-row LN of ln_row.cuh makes
+//            them bit-identical to what the fused LN + compaction writes) and
+//            stores it into all 16 CTAs' shared memory through DSMEM;
+//   pooler   one warp per n8 tile of the CTA's outputs: mma.sync m16n8k16
+//            bf16 -> fp32 over K = H in two accumulator chains (a 16 x 48 x
+//            768 GEMM per CTA is far too small for a tcgen05 tile);
+//   partial  p = tanh(acc + b_p) stays in registers and is folded into
+//            partial logits sum_{o in tile} p[b,o] W_c[c,o], reduced over the
+//            quad with __shfl_xor_sync, then over the CTA's tiles in fixed
+//            order, and stored into rank 0's shared memory (DSMEM);
+//   decide   after a cluster barrier rank 0 sums the 16 partials per (row,
+//            class) in rank order, then softmax / max-prob / entropy, argmax
+//            (lowest index on ties), threshold test, exit record by input id
+//            and the alive flag.  Deterministic: no float atomics anywhere.
 // All ramp math is fp32, never rounded to bf16 (rounding contract).
 // The ViT ramp (LayerNorm + linear over C <= 2048 classes) is ramp_vit_kernel
 // below.
@@ -41,7 +43,9 @@ namespace e3 {
 namespace {
 
 constexpr int kMaxC = 16;
-constexpr int kRows = kRampRowsPerCta;   // 16 = mma M
+constexpr int kCS = 16;          // cluster size (non-portable)
+constexpr int kRows = 16;        // rows per cluster (mma M)
+constexpr int kRThreads = 256;
 
 __device__ __forceinline__ void cp_async16(void *smem, const void *gmem) {
   asm volatile("cp.async.cg.shared.global [%0], [%1], 16;" ::"r"(smem_u32(smem)), "l"(gmem) : "memory");
@@ -59,110 +63,109 @@ __device__ __forceinline__ void mma_bf16_16816(float (&d)[4], const uint32_t (&a
 __device__ __forceinline__ void st_cluster_f32(uint32_t addr, float v) {
   asm volatile("st.shared::cluster.f32 [%0], %1;" ::"r"(addr), "f"(v) : "memory");
 }
+__device__ __forceinline__ void st_cluster_v4(uint32_t addr, uint4 v) {
+  asm volatile("st.shared::cluster.v4.u32 [%0], {%1, %2, %3, %4};" ::"r"(addr), "r"(v.x), "r"(v.y), "r"(v.z),
+               "r"(v.w)
+               : "memory");
+}
+
+// split cluster barrier: arrive at kernel start, wait before the first DSMEM
+// access, so every CTA of the cluster is known to be running
+__device__ __forceinline__ void cluster_arrive_relaxed() {
+  asm volatile("barrier.cluster.arrive.relaxed.aligned;" ::: "memory");
+}
+__device__ __forceinline__ void cluster_wait() { asm volatile("barrier.cluster.wait.aligned;" ::: "memory"); }
 
 __device__ __forceinline__ bool row_alive(const RampArgs &a, int b, int n_valid) {
   return b < a.B && (a.init_alive ? (b < n_valid) : (a.alive[b] != 0));
 }
 
-// smem: CLS [16][P] | W tile [TN][P] | per-warp partials [nw][16][kMaxC] |
-//       cluster partials (rank 0) [CS][16][kMaxC]
-__host__ __device__ inline int ramp_smem_bytes(int H, int CS) {
-  const int TN = H / CS, nw = TN / 8, P = H + 8;
-  return (kRows + TN) * P * 2 + nw * kRows * kMaxC * 4 + CS * kRows * kMaxC * 4;
+// smem: W tile [TN][P] | CLS [16][P] | per-tile partials [NT][16][C] | cluster partials (rank 0) [kCS][16][C]
+__host__ __device__ inline int ramp_smem_bytes(int H, int C) {
+  const int TN = H / kCS, NT = TN / 8, P = H + 8;
+  return (TN + kRows) * P * 2 + NT * kRows * C * 4 + kCS * kRows * C * 4;
 }
 
-// Cluster of CS CTAs per group of 16 rows; CTA rank r computes pooler outputs
-// [r*TN, (r+1)*TN), TN = H / CS, one n8 column tile per warp.
 template <int VPL>
-__global__ void ramp_bert_kernel(RampArgs a, int CS) {
+__global__ void __launch_bounds__(kRThreads, 1) ramp_bert_kernel(RampArgs a) {
   extern __shared__ uint8_t smem_raw[];
-  const int H = a.H;
-  const int TN = H / CS;
-  const int nw = TN / 8;
+  const int H = a.H, C = a.C;
+  const int TN = H / kCS, NT = TN / 8;
   const int P = H + 8;                                   // padded pitch (bf16)
-  __nv_bfloat16 *sC = reinterpret_cast<__nv_bfloat16 *>(smem_raw);   // [16][P]
-  __nv_bfloat16 *sW = sC + kRows * P;                                 // [TN][P]
-  float *sZ = reinterpret_cast<float *>(sW + TN * P);                 // [nw][16][kMaxC]
-  float *sQ = sZ + nw * kRows * kMaxC;                                // [CS][16][kMaxC] (rank 0)
+  __nv_bfloat16 *sW = reinterpret_cast<__nv_bfloat16 *>(smem_raw);   // [TN][P]
+  __nv_bfloat16 *sC = sW + TN * P;                                    // [16][P]
+  float *sZ = reinterpret_cast<float *>(sC + kRows * P);              // [NT][16][C]
+  float *sQ = sZ + NT * kRows * C;                                    // [kCS][16][C] (rank 0)
   __shared__ bool row_ok[kRows];
 
   const int warp = warp_id(), lane = lane_id();
-  const int g = lane >> 2, t = lane & 3;
+  constexpr int nw = kRThreads / 32;
+  const int gq = lane >> 2, tq = lane & 3;
   const uint32_t rank = cluster_ctarank();
   const int b0 = blockIdx.y * kRows;
   const int o0 = (int)rank * TN;
-  const int C = a.C;
   const int nvec = H / 8;
   const __nv_bfloat16 *x = reinterpret_cast<const __nv_bfloat16 *>(a.x);
   const size_t row_stride = (size_t)a.S * H;
 
-  // ---------------------------------------------------------- stage
+  cluster_arrive_relaxed();
+  // ---------------------------------------------------------- stage W_p
   const uint4 *wp = reinterpret_cast<const uint4 *>(a.w.w_p);
-  for (int i = threadIdx.x; i < TN * nvec; i += blockDim.x) {   // weights first: no dependency
+  for (int i = threadIdx.x; i < TN * nvec; i += kRThreads) {   // weights first: no dependency
     const int r = i / nvec, k = i - r * nvec;
     cp_async16(reinterpret_cast<uint4 *>(sW + r * P) + k, wp + (size_t)(o0 + r) * nvec + k);
   }
-  pdl_wait();                      // CLS rows / alive flags of the previous kernels now visible
-  pdl_trigger();
-  const int n_valid = a.n_valid_dev ? *a.n_valid_dev : a.n_valid_host;
-  if (threadIdx.x < kRows) row_ok[threadIdx.x] = row_alive(a, b0 + threadIdx.x, n_valid);
-  __syncthreads();
-  if (a.ln_g) {
-    LnParams<VPL> lp;
+  LnParams<VPL> lp;
+  if (warp == 0 && a.ln_g)
     ln_load_params<VPL>(lp, reinterpret_cast<const __nv_bfloat16 *>(a.ln_g),
                         reinterpret_cast<const __nv_bfloat16 *>(a.ln_b), H, lane);
-    constexpr int kMaxPerWarp = (VPL >= 3) ? 2 : 8;     // >= 16 rows / nw (nw >= 8 when H >= 768)
-    uint4 v[kMaxPerWarp][VPL];
+  pdl_wait();                      // CLS rows / alive flags of the previous kernels now visible
+  const int n_valid = a.n_valid_dev ? *a.n_valid_dev : a.n_valid_host;
+  if (threadIdx.x < kRows) row_ok[threadIdx.x] = row_alive(a, b0 + threadIdx.x, n_valid);
+
+  // ---------------------------------------------------------- CLS row `rank`: LN here, broadcast by DSMEM
+  cluster_wait();                  // every CTA of the cluster is running
+  if (warp == 0) {
+    const int r = (int)rank;
+    const bool ok = row_alive(a, b0 + r, n_valid);
+    uint4 v[VPL];
+    if (ok) {
+      ln_load_row<VPL>(v, x + (size_t)(b0 + r) * row_stride, H, lane);
+      if (a.ln_g) ln_apply<VPL>(v, lp, H, a.eps, lane);
+    } else {
 #pragma unroll
-    for (int u = 0; u < kMaxPerWarp; ++u) {            // all this warp's rows in flight together
-      const int r = warp + u * nw;
-      if (r < kRows && row_ok[r]) ln_load_row<VPL>(v[u], x + (size_t)(b0 + r) * row_stride, H, lane);
+      for (int i = 0; i < VPL; ++i) v[i] = make_uint4(0, 0, 0, 0);
     }
+    const uint32_t row_addr = smem_u32(sC + r * P);
+#pragma unroll 1
+    for (int q = 0; q < kCS; ++q) {
+      const uint32_t dst = mapa_shared(row_addr, (uint32_t)q);
 #pragma unroll
-    for (int u = 0; u < kMaxPerWarp; ++u) {
-      const int r = warp + u * nw;
-      if (r < kRows) {
-        if (row_ok[r]) {
-          ln_apply<VPL>(v[u], lp, H, a.eps, lane);
-        } else {
-#pragma unroll
-          for (int i = 0; i < VPL; ++i) v[u][i] = make_uint4(0, 0, 0, 0);
-        }
-        ln_store_row<VPL>(v[u], sC + r * P, H, lane);
+      for (int i = 0; i < VPL; ++i) {
+        const int k = lane + 32 * i;
+        if (k < nvec) st_cluster_v4(dst + k * 16, v[i]);
       }
-    }
-  } else {
-    for (int i = threadIdx.x; i < kRows * nvec; i += blockDim.x) {
-      const int r = i / nvec, k = i - r * nvec;
-      uint4 *dst = reinterpret_cast<uint4 *>(sC + r * P) + k;
-      if (row_ok[r])
-        cp_async16(dst, reinterpret_cast<const uint4 *>(x + (size_t)(b0 + r) * row_stride) + k);
-      else
-        *dst = make_uint4(0, 0, 0, 0);
     }
   }
   cp_async_wait_all();
-  __syncthreads();
+  cluster_sync();                  // all 16 CLS rows in every CTA; W tile landed
 
-  // ---------------------------------------------------------- pooler (mma.sync)
-  // classifier weights / biases / ids this thread needs later: loaded now so
-  // their latency hides under the MMA loop
+  // ---------------------------------------------------------- pooler + partial logits
   const __nv_bfloat16 *wc = reinterpret_cast<const __nv_bfloat16 *>(a.w.w_c);
-  const int col = o0 + warp * 8 + 2 * t;                    // this lane's two pooler outputs
-  const float bb0 = bf2f(reinterpret_cast<const __nv_bfloat16 *>(a.w.b_p)[col]);
-  const float bb1 = bf2f(reinterpret_cast<const __nv_bfloat16 *>(a.w.b_p)[col + 1]);
-  float wc0[kMaxC], wc1[kMaxC];
+  const __nv_bfloat16 *bp = reinterpret_cast<const __nv_bfloat16 *>(a.w.b_p);
+  for (int t = warp; t < NT; t += nw) {
+    const int col = o0 + t * 8 + 2 * tq;                  // this lane's two pooler outputs
+    const float bb0 = bf2f(bp[col]), bb1 = bf2f(bp[col + 1]);
+    float wc0[kMaxC], wc1[kMaxC];
 #pragma unroll
-  for (int c = 0; c < kMaxC; ++c) {
-    wc0[c] = (c < C) ? bf2f(wc[(size_t)c * H + col]) : 0.f;
-    wc1[c] = (c < C) ? bf2f(wc[(size_t)c * H + col + 1]) : 0.f;
-  }
-  float acc[4] = {0.f, 0.f, 0.f, 0.f};
-  {
-    float acc2[4] = {0.f, 0.f, 0.f, 0.f};                   // second chain: halves the MMA latency chain
-    const __nv_bfloat16 *a_lo = sC + g * P + 2 * t;           // row g
-    const __nv_bfloat16 *a_hi = sC + (g + 8) * P + 2 * t;     // row g + 8
-    const __nv_bfloat16 *bp = sW + (warp * 8 + g) * P + 2 * t;
+    for (int c = 0; c < kMaxC; ++c) {
+      wc0[c] = (c < C) ? bf2f(wc[(size_t)c * H + col]) : 0.f;
+      wc1[c] = (c < C) ? bf2f(wc[(size_t)c * H + col + 1]) : 0.f;
+    }
+    float acc[4] = {0.f, 0.f, 0.f, 0.f}, acc2[4] = {0.f, 0.f, 0.f, 0.f};
+    const __nv_bfloat16 *a_lo = sC + gq * P + 2 * tq;
+    const __nv_bfloat16 *a_hi = sC + (gq + 8) * P + 2 * tq;
+    const __nv_bfloat16 *bw = sW + (t * 8 + gq) * P + 2 * tq;
 #pragma unroll 2
     for (int kk = 0; kk < H; kk += 32) {
 #pragma unroll
@@ -173,20 +176,14 @@ __global__ void ramp_bert_kernel(RampArgs a, int CS) {
         af[1] = *reinterpret_cast<const uint32_t *>(a_hi + k);
         af[2] = *reinterpret_cast<const uint32_t *>(a_lo + k + 8);
         af[3] = *reinterpret_cast<const uint32_t *>(a_hi + k + 8);
-        const uint32_t bf0 = *reinterpret_cast<const uint32_t *>(bp + k);
-        const uint32_t bf1 = *reinterpret_cast<const uint32_t *>(bp + k + 8);
+        const uint32_t bf0 = *reinterpret_cast<const uint32_t *>(bw + k);
+        const uint32_t bf1 = *reinterpret_cast<const uint32_t *>(bw + k + 8);
         if (h2 == 0) mma_bf16_16816(acc, af, bf0, bf1);
         else mma_bf16_16816(acc2, af, bf0, bf1);
       }
     }
-#pragma unroll
-    for (int i = 0; i < 4; ++i) acc[i] += acc2[i];
-  }
-
-  // ---------------------------------------------------------- partial logits
-  {
-    const float p00 = tanhf(acc[0] + bb0), p01 = tanhf(acc[1] + bb1);   // row g
-    const float p10 = tanhf(acc[2] + bb0), p11 = tanhf(acc[3] + bb1);   // row g + 8
+    const float p00 = tanhf(acc[0] + acc2[0] + bb0), p01 = tanhf(acc[1] + acc2[1] + bb1);   // row gq
+    const float p10 = tanhf(acc[2] + acc2[2] + bb0), p11 = tanhf(acc[3] + acc2[3] + bb1);   // row gq + 8
 #pragma unroll
     for (int c = 0; c < kMaxC; ++c) {
       if (c < C) {
@@ -196,23 +193,22 @@ __global__ void ramp_bert_kernel(RampArgs a, int CS) {
         z0 += __shfl_xor_sync(0xffffffffu, z0, 2);
         z1 += __shfl_xor_sync(0xffffffffu, z1, 1);
         z1 += __shfl_xor_sync(0xffffffffu, z1, 2);
-        if (t == 0) {
-          sZ[(warp * kRows + g) * kMaxC + c] = z0;
-          sZ[(warp * kRows + g + 8) * kMaxC + c] = z1;
+        if (tq == 0) {
+          sZ[(t * kRows + gq) * C + c] = z0;
+          sZ[(t * kRows + gq + 8) * C + c] = z1;
         }
       }
     }
   }
   __syncthreads();
-  // this CTA's partial logits -> rank 0's smem slot [rank] (DSMEM)
-  for (int i = threadIdx.x; i < kRows * C; i += blockDim.x) {
-    const int r = i / C, c = i - r * C;
-    float s = sZ[(0 * kRows + r) * kMaxC + c];
-    for (int w = 1; w < nw; ++w) s += sZ[(w * kRows + r) * kMaxC + c];
-    st_cluster_f32(mapa_shared(smem_u32(sQ + ((int)rank * kRows + r) * kMaxC + c), 0), s);
+  // this CTA's partial logits (tiles summed in order) -> rank 0's slot [rank] (DSMEM)
+  for (int i = threadIdx.x; i < kRows * C; i += kRThreads) {
+    float s = sZ[i];
+    for (int t = 1; t < NT; ++t) s += sZ[t * kRows * C + i];
+    st_cluster_f32(mapa_shared(smem_u32(sQ + (int)rank * kRows * C + i), 0), s);
   }
-  // rank 0, warp 0 decides row r = lane (< 16): its id and the class biases
-  // are fetched before the cluster barrier
+  // rank 0 decides row r = threadIdx.x < 16: its id and the class biases are
+  // fetched before the cluster barrier
   const int r = threadIdx.x;
   const int b = b0 + r;
   const bool decider = rank == 0 && r < kRows && b < a.B;
@@ -223,6 +219,9 @@ __global__ void ramp_bert_kernel(RampArgs a, int CS) {
     bcv[c] = (decider && c < C) ? bf2f(reinterpret_cast<const __nv_bfloat16 *>(a.w.b_c)[c]) : 0.f;
   if (decider) row_id = a.id[b];
   cluster_sync();                  // every CTA's partials are in rank 0's smem
+  // late trigger: the dependent kernel's CTAs, once resident, would compete
+  // for issue slots with this issue-bound kernel (measured: +6 us per launch)
+  pdl_trigger();
   if (rank != 0 || warp != 0) return;
 
   // ---------------------------------------------------------- decide (rank 0)
@@ -230,53 +229,53 @@ __global__ void ramp_bert_kernel(RampArgs a, int CS) {
   if (decider && !row_ok[r]) {
     if (a.init_alive) a.alive[b] = 0;
   } else if (decider) {
-  float z[kMaxC];
+    float z[kMaxC];
 #pragma unroll
-  for (int c = 0; c < kMaxC; ++c) {
-    z[c] = 0.f;
-    if (c < C) {
-      float s = 0.f;
-      for (int q = 0; q < CS; ++q) s += sQ[(q * kRows + r) * kMaxC + c];   // fixed order
-      z[c] = s + bcv[c];
-    }
-  }
-  float m = z[0];
-  int label = 0;
-#pragma unroll
-  for (int c = 1; c < kMaxC; ++c)
-    if (c < C && z[c] > m) { m = z[c]; label = c; }   // lowest index on ties
-  float sum = 0.f, qz = 0.f;
-#pragma unroll
-  for (int c = 0; c < kMaxC; ++c)
-    if (c < C) {
-      const float e = expf(z[c] - m);
-      sum += e;
-      qz += e * (z[c] - m);
-    }
-  float metric;
-  bool pass;
-  if (a.test == E3_TEST_MAXPROB) {
-    metric = 1.0f / sum;                       // max_c softmax(z)_c
-    pass = metric > a.tau;
-  } else {
-    metric = logf(sum) - qz / sum;             // H = lse - sum_c q_c z_c
-    pass = metric < a.tau;
-  }
-  exit_now = pass || a.final_ramp;
-  if (exit_now) {
-    const int64_t id = row_id;
-    if (id >= 0 && id < a.ex.capacity) {
-      if (a.ex.exit_layer) a.ex.exit_layer[id] = a.layer;
-      if (a.ex.label) a.ex.label[id] = label;
-      if (a.ex.conf) a.ex.conf[id] = metric;
-      if (a.ex.logits) {
-#pragma unroll
-        for (int c = 0; c < kMaxC; ++c)
-          if (c < C) a.ex.logits[id * C + c] = z[c];
+    for (int c = 0; c < kMaxC; ++c) {
+      z[c] = 0.f;
+      if (c < C) {
+        float s = 0.f;
+        for (int q = 0; q < kCS; ++q) s += sQ[(q * kRows + r) * C + c];   // fixed order
+        z[c] = s + bcv[c];
       }
     }
-  }
-  a.alive[b] = exit_now ? 0 : 1;
+    float m = z[0];
+    int label = 0;
+#pragma unroll
+    for (int c = 1; c < kMaxC; ++c)
+      if (c < C && z[c] > m) { m = z[c]; label = c; }   // lowest index on ties
+    float sum = 0.f, qz = 0.f;
+#pragma unroll
+    for (int c = 0; c < kMaxC; ++c)
+      if (c < C) {
+        const float e = expf(z[c] - m);
+        sum += e;
+        qz += e * (z[c] - m);
+      }
+    float metric;
+    bool pass;
+    if (a.test == E3_TEST_MAXPROB) {
+      metric = 1.0f / sum;                       // max_c softmax(z)_c
+      pass = metric > a.tau;
+    } else {
+      metric = logf(sum) - qz / sum;             // H = lse - sum_c q_c z_c
+      pass = metric < a.tau;
+    }
+    exit_now = pass || a.final_ramp;
+    if (exit_now) {
+      const int64_t id = row_id;
+      if (id >= 0 && id < a.ex.capacity) {
+        if (a.ex.exit_layer) a.ex.exit_layer[id] = a.layer;
+        if (a.ex.label) a.ex.label[id] = label;
+        if (a.ex.conf) a.ex.conf[id] = metric;
+        if (a.ex.logits) {
+#pragma unroll
+          for (int c = 0; c < kMaxC; ++c)
+            if (c < C) a.ex.logits[id * C + c] = z[c];
+        }
+      }
+    }
+    a.alive[b] = exit_now ? 0 : 1;
   }
   // one counter update per warp (exit counts are order-independent)
   const int n_ex = __popc(__ballot_sync(0xffffffffu, exit_now));
@@ -328,6 +327,7 @@ __global__ void __launch_bounds__(2 * CB) ramp_vit_kernel(RampArgs a, int CS) {
   const __nv_bfloat16 *W = reinterpret_cast<const __nv_bfloat16 *>(a.w.w_c);
   const __nv_bfloat16 *bc = reinterpret_cast<const __nv_bfloat16 *>(a.w.b_c);
   const float bias0 = c0 < C ? bf2f(bc[c0]) : 0.f, bias1 = c1 < C ? bf2f(bc[c1]) : 0.f;
+  cluster_arrive_relaxed();
 
   pdl_wait();
   pdl_trigger();
@@ -413,6 +413,7 @@ __global__ void __launch_bounds__(2 * CB) ramp_vit_kernel(RampArgs a, int CS) {
     if (lane == 0) sRed[warp][rr] = st;
   }
   __syncthreads();
+  cluster_wait();                            // every CTA of the cluster is running
   if (t < kVitRows) {                        // row t: merge this CTA's warps, send to rank 0
     const int g = t / 4, rr = t % 4;
     SoftStat st = sRed[g * kWarpsPerRg][rr];
@@ -528,23 +529,19 @@ e3_status ramp_run(const RampArgs &a, cudaStream_t st) {
     set_error("ramp: arch not implemented");
     return E3_EUNSUPPORTED;
   }
-  int CS = 8;
-  if (ramp_smem_bytes(a.H, 8) > 200 * 1024) CS = 16;
-  if (a.C < 1 || a.C > kMaxC || a.H % (8 * CS) || a.H > 4096 || ramp_smem_bytes(a.H, CS) > 220 * 1024 ||
-      (a.H / CS) / 8 > 32) {
-    set_error("ramp: need 1 <= C <= 16, H % 64 == 0 and H <= 1024");
+  if (a.C < 1 || a.C > kMaxC || a.H % (8 * kCS) || a.H > 2048 || ramp_smem_bytes(a.H, a.C) > 220 * 1024) {
+    set_error("ramp: need 1 <= C <= 16, H % 128 == 0 and H <= 2048");
     return E3_EUNSUPPORTED;
   }
-  const int smem = ramp_smem_bytes(a.H, CS);
-  const int threads = (a.H / CS) / 8 * 32;
+  const int smem = ramp_smem_bytes(a.H, a.C);
   cudaLaunchConfig_t cfg = {};
-  cfg.gridDim = dim3(CS, (a.B + kRows - 1) / kRows);
-  cfg.blockDim = dim3(threads);
+  cfg.gridDim = dim3(kCS, (a.B + kRows - 1) / kRows);
+  cfg.blockDim = dim3(kRThreads);
   cfg.dynamicSmemBytes = smem;
   cfg.stream = st;
   cudaLaunchAttribute attr[2];
   attr[0].id = cudaLaunchAttributeClusterDimension;
-  attr[0].val.clusterDim.x = CS;
+  attr[0].val.clusterDim.x = kCS;
   attr[0].val.clusterDim.y = 1;
   attr[0].val.clusterDim.z = 1;
   attr[1].id = cudaLaunchAttributeProgrammaticStreamSerialization;
@@ -562,11 +559,12 @@ e3_status ramp_run(const RampArgs &a, cudaStream_t st) {
                                        1));                                                                 \
       attr_done = true;                                                                                     \
     }                                                                                                       \
-    E3_CUDA_TRY(cudaLaunchKernelEx(&cfg, ramp_bert_kernel<V>, a, CS));                                      \
+    E3_CUDA_TRY(cudaLaunchKernelEx(&cfg, ramp_bert_kernel<V>, a));                                          \
   } while (0)
   if (vpl <= 1) E3_RAMP(1);
   else if (vpl <= 3) E3_RAMP(3);
-  else E3_RAMP(4);
+  else if (vpl <= 4) E3_RAMP(4);
+  else E3_RAMP(8);
 #undef E3_RAMP
   E3_CUDA_TRY(cudaGetLastError());
   count_launch();

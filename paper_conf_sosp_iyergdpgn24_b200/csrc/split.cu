@@ -213,21 +213,22 @@ static e3_status llama_create(e3_split *s, const e3_weights *w) {
     s->kv_k.push_back(w->kv->k[l]);
     s->kv_v.push_back(w->kv->v[l]);
   }
-  s->ks_qkv = dec_pick_ks(nqkv, H, E3_DEC_QKV_ROPE, s->sms);
-  s->ks_o = dec_pick_ks(H, H, E3_DEC_RESID, s->sms);
-  s->ks_gu = dec_pick_ks(F, H, E3_DEC_SWIGLU, s->sms);
-  s->ks_down = dec_pick_ks(H, F, E3_DEC_RESID, s->sms);
-  s->ks_lm = 1;
+  s->mc_qkv = dec_max_contrib(nqkv, H, E3_DEC_QKV_ROPE, s->sms);
+  s->mc_o = dec_max_contrib(H, H, E3_DEC_RESID, s->sms);
+  s->mc_gu = dec_max_contrib(F, H, E3_DEC_SWIGLU, s->sms);
+  s->mc_down = dec_max_contrib(H, F, E3_DEC_RESID, s->sms);
+  s->mc_lm = dec_max_contrib(V, H, E3_DEC_LOGITS, s->sms);
   size_t part = 0, tickets = 0;
-  auto need = [&](int N, int ks, int epi) {
+  auto need = [&](int N, int mc, int epi) {
     const size_t t = (size_t)dec_tiles(N, epi);
-    if (ks > 1 && t * ks * B * 128 > part) part = t * ks * B * 128;
+    if (t * mc * B * 128 > part) part = t * mc * B * 128;
     if (t > tickets) tickets = t;
   };
-  need(nqkv, s->ks_qkv, E3_DEC_QKV_ROPE);
-  need(H, s->ks_o, E3_DEC_RESID);
-  need(F, s->ks_gu, E3_DEC_SWIGLU);
-  need(H, s->ks_down, E3_DEC_RESID);
+  need(nqkv, s->mc_qkv, E3_DEC_QKV_ROPE);
+  need(H, s->mc_o, E3_DEC_RESID);
+  need(F, s->mc_gu, E3_DEC_SWIGLU);
+  need(H, s->mc_down, E3_DEC_RESID);
+  need(V, s->mc_lm, E3_DEC_LOGITS);
   e3_status st = ws.ensure_llama(V, part, tickets, w->kv->max_ctx, 128, 10000.0);
   if (st != E3_OK) return st;
   const int nl = d.layer_end - d.layer_begin;
@@ -369,7 +370,7 @@ static e3_status llama_run(e3_split *s, cudaStream_t st, const void *x_in, const
       DecArgs a = base;
       a.N = nqkv;
       a.K = H;
-      a.ks = s->ks_qkv;
+      a.max_contrib = s->mc_qkv;
       a.epi = E3_DEC_QKV_ROPE;
       a.Y = reinterpret_cast<__nv_bfloat16 *>(ws.qkv);
       a.ldo = d.heads * 128;
@@ -398,7 +399,7 @@ static e3_status llama_run(e3_split *s, cudaStream_t st, const void *x_in, const
       DecArgs a = base;
       a.N = H;
       a.K = H;
-      a.ks = s->ks_o;
+      a.max_contrib = s->mc_o;
       a.epi = E3_DEC_RESID;
       a.R = reinterpret_cast<const __nv_bfloat16 *>(cur);
       a.Y = reinterpret_cast<__nv_bfloat16 *>(ws.y);
@@ -414,7 +415,7 @@ static e3_status llama_run(e3_split *s, cudaStream_t st, const void *x_in, const
       DecArgs a = base;
       a.N = F;
       a.K = H;
-      a.ks = s->ks_gu;
+      a.max_contrib = s->mc_gu;
       a.epi = E3_DEC_SWIGLU;
       a.Y = reinterpret_cast<__nv_bfloat16 *>(ws.h);
       a.ldo = F;
@@ -425,7 +426,7 @@ static e3_status llama_run(e3_split *s, cudaStream_t st, const void *x_in, const
       DecArgs a = base;
       a.N = H;
       a.K = F;
-      a.ks = s->ks_down;
+      a.max_contrib = s->mc_down;
       a.epi = E3_DEC_RESID;
       a.R = reinterpret_cast<const __nv_bfloat16 *>(ws.y);
       a.Y = reinterpret_cast<__nv_bfloat16 *>(out);
@@ -442,7 +443,7 @@ static e3_status llama_run(e3_split *s, cudaStream_t st, const void *x_in, const
         DecArgs a = base;
         a.N = V;
         a.K = H;
-        a.ks = 1;
+        a.max_contrib = s->mc_lm;
         a.epi = E3_DEC_LOGITS;
         a.Z = ws.lm_z;
         a.stats = ws.lm_stats;
@@ -700,6 +701,48 @@ e3_status e3_op_gemm(void *stream, const void *A, int64_t lda, const void *W, co
   e3_status r = gemm_tmaps(&g, A, lda, W, C, M, N, K, gemm_pick_bn(M, N, sms));
   if (r != E3_OK) return r;
   return gemm_run(g, bias, resid, M, N, K, epilogue, sms, reinterpret_cast<cudaStream_t>(stream));
+}
+
+e3_status e3_op_dec_gemm(void *stream, const void *X, int32_t T, const void *W, const void *W2, int32_t N, int32_t K,
+                         int32_t epilogue, const void *R, void *Y) {
+  E3_CHECK_ARG(X && W && Y && N > 0 && K > 0, "bad arguments");
+  E3_CHECK_ARG(epilogue >= 0 && epilogue <= 2, "bad epilogue");
+  E3_CHECK_ARG(epilogue != 1 || R, "residual epilogue needs R");
+  E3_CHECK_ARG(epilogue != 2 || W2, "SwiGLU epilogue needs W2");
+  if ((T != 32 && T != 64 && T != 128) || K % 64 || (epilogue == 2 && N % 64) || !aligned16(X) || !aligned16(W) ||
+      (W2 && !aligned16(W2))) {
+    set_error("e3_op_dec_gemm: need T in {32,64,128}, K % 64 == 0, SwiGLU N % 64 == 0, aligned operands");
+    return E3_EUNSUPPORTED;
+  }
+  int dev = 0;
+  E3_CUDA_TRY(cudaGetDevice(&dev));
+  const int sms = num_sms(dev);
+  const int epi = epilogue == 0 ? E3_DEC_STORE : epilogue == 1 ? E3_DEC_RESID : E3_DEC_SWIGLU;
+  cudaStream_t st = reinterpret_cast<cudaStream_t>(stream);
+  DecMaps m;
+  e3_status r = dec_tmaps(&m, X, T, K, W, W2, N, epi);
+  if (r != E3_OK) return r;
+  const int tiles = dec_tiles(N, epi), mc = dec_max_contrib(N, K, epi, sms);
+  float *part = nullptr;
+  unsigned *tick = nullptr;
+  E3_CUDA_TRY(cudaMallocAsync(reinterpret_cast<void **>(&part), (size_t)tiles * mc * T * 128 * 4, st));
+  E3_CUDA_TRY(cudaMallocAsync(reinterpret_cast<void **>(&tick), (size_t)tiles * 4, st));
+  E3_CUDA_TRY(cudaMemsetAsync(tick, 0, (size_t)tiles * 4, st));
+  DecArgs a{};
+  a.T = T;
+  a.N = N;
+  a.K = K;
+  a.epi = epi;
+  a.max_contrib = mc;
+  a.R = reinterpret_cast<const __nv_bfloat16 *>(R);
+  a.Y = reinterpret_cast<__nv_bfloat16 *>(Y);
+  a.ldo = N;
+  a.part = part;
+  a.tickets = tick;
+  r = dec_run(m, a, sms, st);
+  cudaFreeAsync(part, st);
+  cudaFreeAsync(tick, st);
+  return r;
 }
 
 e3_status e3_op_attention(void *stream, const void *qkv, void *ctx, int32_t B, int32_t S, int32_t H, int32_t heads) {

@@ -55,7 +55,7 @@ struct e3_split {
   };
   std::vector<DecLayer> dmaps;
   std::vector<e3::DecMaps> lm_maps;
-  int ks_qkv = 1, ks_o = 1, ks_gu = 1, ks_down = 1, ks_lm = 1;
+  int mc_qkv = 1, mc_o = 1, mc_gu = 1, mc_down = 1, mc_lm = 1;   // stream-K partial slots per tile
   e3_kv_cache kv{};
   std::vector<void *> kv_k, kv_v;       // this split's layers' cache pointers
   e3::AttnMaps attn;

@@ -253,3 +253,26 @@ def test_vit_ramp_matches_oracle(api, base, test, C):
                  n_valid=n_valid)
     torch.cuda.synchronize()
     assert int(ex2.n_exit.item()) == nv and int(alive2.sum()) == 0
+
+
+@pytest.mark.parametrize("T,N,K", [(32, 256, 128), (64, 1280, 4096), (128, 384, 640), (64, 4096, 11008)])
+@pytest.mark.parametrize("epi", ["store", "resid", "swiglu"])
+def test_dec_gemm_matches_definition(api, T, N, K, epi):
+    """Decode GEMM (swap-AB tcgen05, stream-K with tiles shared between CTAs):
+    Y = X W^T (+ R) or SiLU(X Wg^T) * (X Wu^T), one bf16 rounding."""
+    from oracle.llama import silu
+    rng = np.random.default_rng(T + N + K)
+    X = rand_bf16(rng, (T, K))
+    W = rand_bf16(rng, (N, K), K ** -0.5)
+    W2 = rand_bf16(rng, (N, K), K ** -0.5) if epi == "swiglu" else None
+    R = rand_bf16(rng, (T, N)) if epi == "resid" else None
+    out = api.ops.dec_gemm(bf16_tensor(X), bf16_tensor(W), epi, W2=None if W2 is None else bf16_tensor(W2),
+                           resid=None if R is None else bf16_tensor(R))
+    torch.cuda.synchronize()
+    y = X.astype(np.float64) @ W.astype(np.float64).T
+    if epi == "resid":
+        y = y + R
+    if epi == "swiglu":
+        y = silu(y) * (X.astype(np.float64) @ W2.astype(np.float64).T)
+    # fp32 accumulation over up to 11008 terms + SiLU in fp32: 1 ulp + small atol
+    _assert_bf16_close(to64(out), y, ulps=1.0, atol=2e-3 if K > 4096 else 5e-4, min_exact=0.9)
