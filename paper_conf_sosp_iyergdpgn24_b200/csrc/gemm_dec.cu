@@ -48,9 +48,9 @@ struct DCfg {
   static constexpr int kXBytes = T * DK * 2;
   static constexpr int kStageBytes = kWBytes + kXBytes;
   static constexpr int kEBytes = DM * (T + 1) * 4;          // fp32 epilogue tile
-  static constexpr int kStages = (kSmemMax - kEBytes - 1024 - 2048) / kStageBytes;
+  static constexpr int kStages = (kSmemMax - kEBytes - 1024 - 3072) / kStageBytes;
   static constexpr int kTmemCols = (2 * T <= 32) ? 32 : (2 * T <= 64) ? 64 : (2 * T <= 128) ? 128 : 256;
-  static constexpr int kSmem = kStages * kStageBytes + kEBytes + 1024 + 2048;   // + barriers, token tables
+  static constexpr int kSmem = kStages * kStageBytes + kEBytes + 1024 + 3072;   // + barriers, token tables
 };
 
 __device__ __forceinline__ void epi_bar() { asm volatile("bar.sync 1, 128;" ::: "memory"); }
@@ -94,6 +94,7 @@ __global__ void __launch_bounds__(kDThreads, 1)
   int *s_last = reinterpret_cast<int *>(tmem_slot + 1);
   int *sPos = s_last + 1;          // [T]
   int *sSlot = sPos + T;           // [T]
+  int64_t *sTok = reinterpret_cast<int64_t *>(sSlot + T + (T & 1));   // [T] LOGITS: exit-record row of token t
 
   const int warp = warp_id(), lane = lane_id();
   const int tiles = (EPI == E3_DEC_SWIGLU) ? a.N / 64 : (a.N + DM - 1) / DM;
@@ -198,6 +199,17 @@ __global__ void __launch_bounds__(kDThreads, 1)
     const int q = warp & 3;
     const int r = q * 32 + lane;       // weight row of the tile == TMEM lane
     const int et = threadIdx.x - 64;   // 0..127
+    if (EPI == E3_DEC_LOGITS) {
+      const int nv = a.n_valid_dev ? *a.n_valid_dev : a.n_valid_host;
+      for (int t = et; t < T; t += 128) {
+        const int64_t id = a.ids ? a.ids[t] : -1;
+        // only rows still alive at this ramp (a row that exited at an inner
+        // ramp of the split keeps that ramp's logits)
+        const bool live = t < nv && (a.init_alive || a.alive[t] != 0);
+        sTok[t] = (live && id >= 0 && id < a.id_cap) ? id : -1;
+      }
+      epi_bar();
+    }
     if (EPI == E3_DEC_QKV_ROPE) {
       const int nv = a.n_valid_dev ? *a.n_valid_dev : a.n_valid_host;
       for (int t = et; t < T; t += 128) {
@@ -358,8 +370,13 @@ __global__ void __launch_bounds__(kDThreads, 1)
       } else if (EPI == E3_DEC_LOGITS) {
         const int n0 = tile * DM;
         const int rows = (a.N - n0) < DM ? (a.N - n0) : DM;
-        if (r < rows)
-          for (int t = 0; t < T; ++t) a.Z[(size_t)t * a.N + n0 + r] = sE[r * P + t];
+        // logits go straight to the exit records, row id_t of [capacity, V]
+        // (a row that does not exit here is rewritten by the ramp it exits
+        // at -- the last ramp exits every row), so no second pass copies
+        // 128 KB per exiting token; sTok[t] = id_t or -1 (padding / no logits)
+        if (a.Z && r < rows)
+          for (int t = 0; t < T; ++t)
+            if (sTok[t] >= 0) a.Z[(size_t)sTok[t] * a.N + n0 + r] = sE[r * P + t];
         for (int t = et; t < T; t += 128) {
           float m = sE[t];
           int idx = 0;

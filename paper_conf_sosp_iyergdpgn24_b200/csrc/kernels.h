@@ -58,9 +58,9 @@ struct RampArgs {
   e3_exits ex;
   float *pool_ws;           // [B,H] fp32 workspace
   unsigned *done_ctr;       // device tickets [ceil(B/kRampRowsPerCta)] (zero between launches)
-  // LLAMA: logits [B, C] fp32 and per-128-class-tile softmax statistics from
-  // the LM-head GEMM (gemm_dec.cu, E3_DEC_LOGITS); the decide kernel merges them
-  const float *lm_z;
+  // LLAMA: per-128-class-tile softmax statistics from the LM-head GEMM
+  // (gemm_dec.cu, E3_DEC_LOGITS, which also wrote the logits to the exit
+  // records); the decide kernel merges them
   const float4 *lm_stats;   // [tiles][B] (max, sum e, sum e*(z-max), argmax bits)
   int lm_tiles;
 };
@@ -79,7 +79,9 @@ struct DecArgs {
   const __nv_bfloat16 *R;   // RESID: residual [T, ldo]
   __nv_bfloat16 *Y;         // STORE / RESID / SWIGLU / QKV (q): [T, ldo]
   int ldo;
-  float *Z;                 // LOGITS: [T, N]
+  float *Z;                 // LOGITS: exit-record logits [id_cap, N] (NULL: not recorded)
+  const uint8_t *alive;     // LOGITS: rows alive at this ramp (unless init_alive)
+  int init_alive;
   float4 *stats;            // LOGITS: [tiles][T]
   float *part;              // stream-K partials [tiles][max_contrib][T/4][128 rows] of float4
   unsigned *tickets;        // stream-K tickets [tiles], zero between launches

@@ -3,16 +3,20 @@
 // ramp's decision.  The GEMMs of the decode layer are gemm_dec.cu.
 //
 //   rmsnorm_kernel   warp per token row: y = bf16(x / sqrt(mean x^2 + eps) * g)
-//   attn_dec_kernel  one CTA per (head, token): q from the QKV epilogue (RoPE
-//                    applied), keys/values of the token's slot at positions
-//                    0..pos (the new one written by the same epilogue);
+//   attn_dec_kernel  one CTA per (head, token), 8 warps: q from the QKV
+//                    epilogue (RoPE applied), keys/values of the token's slot
+//                    at positions 0..pos (the new one written by the same
+//                    epilogue); every key / value row is one coalesced
+//                    256-byte warp load, 8 keys per warp step reduced with 9
+//                    shuffles;
 //                    scores fp32, p = exp(s - max) unrounded, out = bf16(p V / l)
 //                    -- HBM-bound on the cache stream (537 MB per Llama-7B
 //                    layer at 64 tokens x 513 positions)
 //   lm_decide_kernel warp per row: merges the LM-head tiles' softmax
 //                    statistics in tile order (softstat.cuh), max-prob /
-//                    entropy, strict threshold, exit record + logits copy,
-//                    alive flag -- the same semantics as the encoder ramps.
+//                    entropy, strict threshold, exit record, alive flag --
+//                    the same semantics as the encoder ramps (the logits
+//                    were written to the records by the LM-head epilogue).
 #include "common.cuh"
 #include "kernels.h"
 #include "prof.h"
@@ -67,8 +71,10 @@ __global__ void __launch_bounds__(256) rmsnorm_kernel(const __nv_bfloat16 *__res
   }
 }
 
-constexpr int kAttnThreads = 128;
-constexpr int kHd = 128;   // head_dim
+constexpr int kAttnThreads = 256;
+constexpr int kAW = kAttnThreads / 32;   // warps
+constexpr int kHd = 128;                 // head_dim
+constexpr int kKeysPerStep = 8;          // keys per warp per step (one 256-B row each)
 
 __device__ __forceinline__ float block_reduce(float v, float *red, bool is_max) {
   const int warp = warp_id(), lane = lane_id();
@@ -82,8 +88,31 @@ __device__ __forceinline__ float block_reduce(float v, float *red, bool is_max) 
   __syncthreads();
   float r = red[0];
 #pragma unroll
-  for (int w = 1; w < kAttnThreads / 32; ++w) r = is_max ? fmaxf(r, red[w]) : r + red[w];
+  for (int w = 1; w < kAW; ++w) r = is_max ? fmaxf(r, red[w]) : r + red[w];
   return r;
+}
+
+// 8 per-lane partial dot products -> lane L holds the full sum of key
+// ((L>>4)&1)*4 + ((L>>3)&1)*2 + ((L>>2)&1)  (9 shuffles for 8 keys)
+__device__ __forceinline__ float reduce8(float (&v)[8], int lane) {
+  const bool b16 = lane & 16, b8 = lane & 8, b4 = lane & 4;
+#pragma unroll
+  for (int i = 0; i < 4; ++i) {
+    const float send = b16 ? v[i] : v[i + 4], keep = b16 ? v[i + 4] : v[i];
+    v[i] = keep + __shfl_xor_sync(0xffffffffu, send, 16);
+  }
+#pragma unroll
+  for (int i = 0; i < 2; ++i) {
+    const float send = b8 ? v[i] : v[i + 2], keep = b8 ? v[i + 2] : v[i];
+    v[i] = keep + __shfl_xor_sync(0xffffffffu, send, 8);
+  }
+  {
+    const float send = b4 ? v[0] : v[1], keep = b4 ? v[1] : v[0];
+    v[0] = keep + __shfl_xor_sync(0xffffffffu, send, 4);
+  }
+  v[0] += __shfl_xor_sync(0xffffffffu, v[0], 2);
+  v[0] += __shfl_xor_sync(0xffffffffu, v[0], 1);
+  return v[0];
 }
 
 __global__ void __launch_bounds__(kAttnThreads)
@@ -93,9 +122,8 @@ __global__ void __launch_bounds__(kAttnThreads)
                     const int32_t *__restrict__ slot_of_id, int64_t id_cap, const int32_t *__restrict__ pos_of_slot,
                     int nh, int kvh, int max_ctx, float scale) {
   extern __shared__ float sp[];                 // [max_ctx] scores / probabilities
-  __shared__ float sq[kHd];
-  __shared__ float red[kAttnThreads / 32];
-  __shared__ float4 sacc[kAttnThreads / 32][32];
+  __shared__ float red[kAW];
+  __shared__ float4 sacc[kAW][32];
   const int h = blockIdx.x, t = blockIdx.y;
   const int tid = threadIdx.x, warp = warp_id(), lane = lane_id();
   const int H = nh * kHd;
@@ -105,35 +133,37 @@ __global__ void __launch_bounds__(kAttnThreads)
   const int64_t id = ids[t];
   __nv_bfloat16 *out = ctx + (size_t)t * H + h * kHd;
   if (t >= nv || id < 0 || id >= id_cap) {     // padding row: finite zeros
-    if (tid < kHd / 2) reinterpret_cast<uint32_t *>(out)[tid] = 0u;
+    if (tid < kHd / 4) reinterpret_cast<uint2 *>(out)[tid] = make_uint2(0u, 0u);
     return;
   }
   const int slot = slot_of_id[id];
   const int pos = pos_of_slot[slot];
   const int L = pos + 1;
   const int g = h / (nh / kvh);
-  sq[tid] = bf2f(q[(size_t)t * H + h * kHd + tid]);
-  __syncthreads();
+  // lane owns dims 4*lane .. 4*lane+3 of q, of every key and every value row
+  const uint2 qv = reinterpret_cast<const uint2 *>(q + (size_t)t * H + h * kHd)[lane];
+  const float q0 = bf_lo(qv.x) * scale, q1 = bf_hi(qv.x) * scale, q2 = bf_lo(qv.y) * scale,
+              q3 = bf_hi(qv.y) * scale;
   const size_t base = ((size_t)slot * kvh + g) * max_ctx * kHd;
-  const uint4 *K = reinterpret_cast<const uint4 *>(kc + base);
-  // ---- scores: one key per thread (16 x 16-byte loads of its row)
+  const uint2 *K = reinterpret_cast<const uint2 *>(kc + base) + lane;   // + j * 32 for key j
+  // ---- scores: warp w takes keys [8s, 8s+8) for s = w, w + 8, ...; each key
+  // row is one coalesced 256-byte warp load
   float lmax = -INFINITY;
-  for (int j = tid; j < L; j += kAttnThreads) {
-    const uint4 *kr = K + (size_t)j * (kHd / 8);
-    float s = 0.f;
-#pragma unroll 4
-    for (int c = 0; c < kHd / 8; ++c) {
-      const uint4 kv = kr[c];
-      const uint32_t w[4] = {kv.x, kv.y, kv.z, kv.w};
+  for (int j0 = warp * kKeysPerStep; j0 < L; j0 += kAW * kKeysPerStep) {
+    uint2 kv[kKeysPerStep];
 #pragma unroll
-      for (int e = 0; e < 4; ++e) {
-        s = fmaf(sq[c * 8 + 2 * e], bf_lo(w[e]), s);
-        s = fmaf(sq[c * 8 + 2 * e + 1], bf_hi(w[e]), s);
-      }
+    for (int i = 0; i < kKeysPerStep; ++i)
+      kv[i] = (j0 + i < L) ? K[(size_t)(j0 + i) * (kHd / 4)] : make_uint2(0u, 0u);
+    float d[kKeysPerStep];
+#pragma unroll
+    for (int i = 0; i < kKeysPerStep; ++i)
+      d[i] = fmaf(q0, bf_lo(kv[i].x), fmaf(q1, bf_hi(kv[i].x), fmaf(q2, bf_lo(kv[i].y), q3 * bf_hi(kv[i].y))));
+    const float sc = reduce8(d, lane);
+    const int k = ((lane >> 4) & 1) * 4 + ((lane >> 3) & 1) * 2 + ((lane >> 2) & 1);
+    if ((lane & 3) == 0 && j0 + k < L) {
+      sp[j0 + k] = sc;
+      lmax = fmaxf(lmax, sc);
     }
-    s *= scale;
-    sp[j] = s;
-    lmax = fmaxf(lmax, s);
   }
   const float m = block_reduce(lmax, red, true);
   float lsum = 0.f;
@@ -143,12 +173,12 @@ __global__ void __launch_bounds__(kAttnThreads)
     lsum += e;
   }
   const float l = block_reduce(lsum, red, false);   // also orders the sp[] writes
-  // ---- P V: warp w takes positions j = w mod 4, lane owns dims 4*lane .. +3
-  const uint2 *V = reinterpret_cast<const uint2 *>(vc + base);
+  // ---- P V: warp w takes positions j = w mod 8, lane owns dims 4*lane .. +3
+  const uint2 *V = reinterpret_cast<const uint2 *>(vc + base) + lane;
   float4 acc = make_float4(0.f, 0.f, 0.f, 0.f);
-#pragma unroll 4
-  for (int j = warp; j < L; j += kAttnThreads / 32) {
-    const uint2 vv = V[(size_t)j * (kHd / 4) + lane];
+#pragma unroll 8
+  for (int j = warp; j < L; j += kAW) {
+    const uint2 vv = V[(size_t)j * (kHd / 4)];
     const float p = sp[j];
     acc.x = fmaf(p, bf_lo(vv.x), acc.x);
     acc.y = fmaf(p, bf_hi(vv.x), acc.y);
@@ -158,18 +188,18 @@ __global__ void __launch_bounds__(kAttnThreads)
   sacc[warp][lane] = acc;
   __syncthreads();
   if (warp == 0) {
-    float4 s = sacc[0][lane];
+    float4 s4 = sacc[0][lane];
 #pragma unroll
-    for (int w = 1; w < kAttnThreads / 32; ++w) {
-      s.x += sacc[w][lane].x;
-      s.y += sacc[w][lane].y;
-      s.z += sacc[w][lane].z;
-      s.w += sacc[w][lane].w;
+    for (int w = 1; w < kAW; ++w) {
+      s4.x += sacc[w][lane].x;
+      s4.y += sacc[w][lane].y;
+      s4.z += sacc[w][lane].z;
+      s4.w += sacc[w][lane].w;
     }
     const float il = 1.0f / l;
     uint2 o;
-    o.x = pack_bf16(s.x * il, s.y * il);
-    o.y = pack_bf16(s.z * il, s.w * il);
+    o.x = pack_bf16(s4.x * il, s4.y * il);
+    o.y = pack_bf16(s4.z * il, s4.w * il);
     reinterpret_cast<uint2 *>(out)[lane] = o;
   }
 }
@@ -210,8 +240,6 @@ __global__ void __launch_bounds__(128) lm_decide_kernel(RampArgs a) {
       if (a.ex.label) a.ex.label[id] = st.idx;
       if (a.ex.conf) a.ex.conf[id] = metric;
     }
-    if (a.ex.logits)
-      for (int c = lane; c < a.C; c += 32) a.ex.logits[id * a.C + c] = a.lm_z[(size_t)b * a.C + c];
   }
   if (lane == 0) {
     a.alive[b] = exit_now ? 0 : 1;

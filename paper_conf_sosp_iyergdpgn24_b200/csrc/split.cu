@@ -28,20 +28,14 @@ Workspace::~Workspace() {
   int prev = 0;
   cudaGetDevice(&prev);
   cudaSetDevice(device);
-  void *bufs[] = {qkv, ctx, y, x1, h, xa, xb, pool, alive, ctr, lm_z, lm_stats, dec_part, dec_tickets, rope};
+  void *bufs[] = {qkv, ctx, y, x1, h, xa, xb, pool, alive, ctr, lm_stats, dec_part, dec_tickets, rope};
   for (void *p : bufs)
     if (p) cudaFree(p);
   cudaSetDevice(prev);
 }
 
 e3_status Workspace::ensure_llama(int V, size_t part, size_t tickets, int max_ctx, int head_dim, double theta) {
-  const size_t z = (size_t)B * V, st = (size_t)((V + 127) / 128) * B;
-  if (z > lm_z_elems) {
-    if (lm_z) cudaFree(lm_z);
-    lm_z = nullptr;
-    E3_CUDA_TRY(cudaMalloc(&lm_z, z * sizeof(float)));
-    lm_z_elems = z;
-  }
+  const size_t st = (size_t)((V + 127) / 128) * B;
   if (st > lm_stats_elems) {
     if (lm_stats) cudaFree(lm_stats);
     lm_stats = nullptr;
@@ -445,7 +439,13 @@ static e3_status llama_run(e3_split *s, cudaStream_t st, const void *x_in, const
         a.K = H;
         a.max_contrib = s->mc_lm;
         a.epi = E3_DEC_LOGITS;
-        a.Z = ws.lm_z;
+        a.Z = exits.logits;
+        a.ids = id_in;
+        a.n_valid_dev = n_valid_dev;
+        a.n_valid_host = n_valid_host;
+        a.id_cap = exits.capacity;
+        a.alive = ws.alive;
+        a.init_alive = first_ramp;
         a.stats = ws.lm_stats;
         E3_RUN(dec_run(s->lm_maps[ri], a, s->sms, st));
         RampArgs ra{};
@@ -465,7 +465,6 @@ static e3_status llama_run(e3_split *s, cudaStream_t st, const void *x_in, const
         ra.n_valid_dev = n_valid_dev;
         ra.n_valid_host = n_valid_host;
         ra.ex = exits;
-        ra.lm_z = ws.lm_z;
         ra.lm_stats = ws.lm_stats;
         ra.lm_tiles = dec_tiles(V, E3_DEC_LOGITS);
         E3_RUN(lm_decide_run(ra, st));

@@ -20,14 +20,13 @@ struct Workspace {
   float *pool = nullptr;
   uint8_t *alive = nullptr;
   unsigned *ctr = nullptr;        // [kCtrWords]: compaction ticket, ramp row-group tickets
-  // LLAMA decode (allocated by ensure_llama): LM-head logits / tile statistics,
-  // split-K partials and tickets of the decode GEMMs, RoPE cos/sin table
-  float *lm_z = nullptr;
+  // LLAMA decode (allocated by ensure_llama): LM-head tile statistics,
+  // stream-K partials and tickets of the decode GEMMs, RoPE cos/sin table
   float4 *lm_stats = nullptr;
   float *dec_part = nullptr;
   unsigned *dec_tickets = nullptr;
   float2 *rope = nullptr;
-  size_t lm_z_elems = 0, lm_stats_elems = 0, part_elems = 0, ticket_elems = 0;
+  size_t lm_stats_elems = 0, part_elems = 0, ticket_elems = 0;
   int rope_ctx = 0, rope_hd = 0;
   double rope_theta = 0;
   e3_status ensure_llama(int V, size_t part_elems, size_t tickets, int max_ctx, int head_dim, double theta);
