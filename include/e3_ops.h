@@ -37,6 +37,14 @@ e3_status e3_op_gemm(void *stream, const void *A, int64_t lda, const void *W, co
 e3_status e3_op_dec_gemm(void *stream, const void *X, int32_t T, const void *W, const void *W2, int32_t N,
                          int32_t K, int32_t epilogue, const void *R, void *Y);
 
+/* Attention output projection with the LayerNorm fused (a2; gemm_ln.cu):
+ *   y   = bf16(A[M,K] W[N,K]^T + bias + R[M,N])     (written to pre if non-NULL)
+ *   out = bf16(LN(y) * g + b), fp32 statistics of the rounded y, eps.
+ * N in {128, 256, 384, 512, 640, 768, 1024} (a cluster of 2 CTAs holds a
+ * whole row), K % 64 == 0, any M. */
+e3_status e3_op_gemm_ln(void *stream, const void *A, const void *W, const void *bias, const void *R, const void *g,
+                        const void *b, float eps, void *pre, void *out, int32_t M, int32_t N, int32_t K);
+
 /* Self-attention (a2) on tcgen05: qkv [B*S, 3H] (q | k | v, head h owning
  * columns h*64..h*64+63 of each third) -> ctx [B*S, H].  head_dim 64,
  * S <= 256, no mask.  softmax(q k^T / sqrt(64)) v with the rounding contract

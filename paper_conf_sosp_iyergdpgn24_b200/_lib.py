@@ -99,6 +99,7 @@ SIGNATURES = {
     "e3_pipeline_trace": (I32, [P, P, P, P, I64, C.POINTER(I64)]),
     "e3_op_gemm": (I32, [P, P, I64, P, P, P, P, I32, I32, I32, I32]),
     "e3_op_dec_gemm": (I32, [P, P, I32, P, P, I32, I32, I32, P, P]),
+    "e3_op_gemm_ln": (I32, [P, P, P, P, P, P, P, C.c_float, P, P, I32, I32, I32]),
     "e3_op_attention": (I32, [P, P, P, I32, I32, I32, I32]),
     "e3_op_layernorm": (I32, [P, P, P, P, P, I32, I32, C.c_float]),
     "e3_op_ramp": (I32, [P, I32, P, P, I32, I32, I32, I32, C.POINTER(RampWeights), I32, C.c_float, I32,

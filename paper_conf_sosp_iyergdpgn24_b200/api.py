@@ -276,6 +276,17 @@ class ops:
         return out
 
     @staticmethod
+    def gemm_ln(A, W, bias, resid, g, b, eps, pre=None, out=None, stream=None):
+        """out = LN(A W^T + bias + resid) (fused O projection + LayerNorm); pre
+        receives the pre-LN rows when given."""
+        M, K = A.shape
+        N = W.shape[0]
+        out = torch.empty((M, N), dtype=torch.bfloat16, device=A.device) if out is None else out
+        check(lib.e3_op_gemm_ln(_stream(stream), _ptr(A), _ptr(W), _ptr(bias), _ptr(resid), _ptr(g), _ptr(b),
+                                float(eps), _ptr(pre), _ptr(out), M, N, K), "e3_op_gemm_ln")
+        return out
+
+    @staticmethod
     def gemm(A, W, bias, epilogue="bias", resid=None, out=None, stream=None):
         M, K = A.shape
         N = W.shape[0]

@@ -43,13 +43,17 @@ struct ACfg {
   static constexpr int kBuf = kQ + 2 * kKV;              // Q | K | V
   static constexpr bool kPInQK = (kP <= kQ + kKV);       // P overwrites the dead Q|K tiles
   static constexpr int kExtra = 1024 + 64 + 2 * 2 * QT * 4;
+#ifdef E3_ATTN_SINGLE_BUF   // diagnostics: occupancy instead of double buffering
+  static constexpr int kNBuf = 1;
+#else
   static constexpr int kNBuf = (2 * kBuf + (kPInQK ? 0 : kP) + kExtra <= 232448) ? 2 : 1;   // double buffer if it fits
+#endif
   static constexpr int kSmem = kNBuf * kBuf + (kPInQK ? 0 : kP) + kExtra;
   static constexpr int kTmemCols = SKV <= 128 ? 128 : 256;   // S, later O (64 columns)
 };
 
 template <int SKV>
-__global__ void __launch_bounds__(kThreads)
+__global__ void __launch_bounds__(kThreads, SKV == 128 ? 2 : 1)
     attn_tc_kernel(const __grid_constant__ CUtensorMap tq, const __grid_constant__ CUtensorMap tkv,
                    const __grid_constant__ CUtensorMap tctx, int S, int H, int heads, int n_items) {
   using CF = ACfg<SKV>;
@@ -140,19 +144,31 @@ __global__ void __launch_bounds__(kThreads)
     mbar_wait(bar_s, sphase);
     sphase ^= 1;
     tc_fence_after();
-    const int c_begin = khalf ? ((NCH + 1) / 2) * 32 : 0;
-    const int c_end = khalf ? SKV : ((NCH + 1) / 2) * 32;
+    // S = 128: S is read from TMEM once, this thread's 64 keys stay in
+    // registers between the max pass and the exponentiation pass (-6 %);
+    // longer rows would spill, so they are read twice
+    constexpr int NCH0 = (NCH + 1) / 2;                   // chunks of thread half 0 (half 1: NCH / 2)
+    constexpr bool kKeep = NCH0 <= 2;                     // S = 128: 64 registers; longer rows reload
+    const int c_begin = khalf ? NCH0 * 32 : 0;
+    const int nch = khalf ? NCH / 2 : NCH0;
+    float sv[kKeep ? NCH0 * 32 : 32];
     float mx = -INFINITY;
-#pragma unroll 1
-    for (int c = c_begin; c < c_end; c += 32) {
-      uint32_t r[32];
-      tmem_ld32(tbase + lane_off + c, r);
-      tmem_wait_ld();
-      float m4[4] = {-INFINITY, -INFINITY, -INFINITY, -INFINITY};
 #pragma unroll
-      for (int jj = 0; jj < 32; ++jj)
-        if (c + jj < S) m4[jj & 3] = fmaxf(m4[jj & 3], __uint_as_float(r[jj]));
-      mx = fmaxf(mx, fmaxf(fmaxf(m4[0], m4[1]), fmaxf(m4[2], m4[3])));
+    for (int ci = 0; ci < NCH0; ++ci) {
+      if (ci < nch) {
+        const int c = c_begin + ci * 32;
+        uint32_t r[32];
+        tmem_ld32(tbase + lane_off + c, r);
+        tmem_wait_ld();
+        float m4[4] = {-INFINITY, -INFINITY, -INFINITY, -INFINITY};
+#pragma unroll
+        for (int jj = 0; jj < 32; ++jj) {
+          const float v = __uint_as_float(r[jj]);
+          if (kKeep) sv[ci * 32 + jj] = v;
+          if (c + jj < S) m4[jj & 3] = fmaxf(m4[jj & 3], v);
+        }
+        mx = fmaxf(mx, fmaxf(fmaxf(m4[0], m4[1]), fmaxf(m4[2], m4[3])));
+      }
     }
     float *xmax = xch + (j & 1) * 2 * QT;                  // double-buffered exchange slots
     float *xsum = xmax + QT;
@@ -164,28 +180,35 @@ __global__ void __launch_bounds__(kThreads)
     const float mb = mx * sl2;
     float l4[4] = {0.f, 0.f, 0.f, 0.f};
     uint8_t *prow = sP + row * 128;
-#pragma unroll 1
-    for (int c = c_begin; c < c_end; c += 32) {
-      uint32_t r[32];
-      tmem_ld32(tbase + lane_off + c, r);
-      tmem_wait_ld();
-      float p[32];
 #pragma unroll
-      for (int jj = 0; jj < 32; ++jj) {
-        p[jj] = (c + jj < S) ? ex2_approx(fmaf(__uint_as_float(r[jj]), sl2, -mb)) : 0.f;
-        l4[jj & 3] += p[jj];
-      }
-      // columns c..c+31 -> block c/64, 16-byte chunks (c%64)/8 .. +3, XOR-swizzled by row%8
-      uint8_t *blk = prow + (c / 64) * (QT * 128);
-      const int ch0 = (c % 64) / 8;
+    for (int ci = 0; ci < NCH0; ++ci) {
+      if (ci < nch) {
+        const int c = c_begin + ci * 32;
+        if (!kKeep) {
+          uint32_t r[32];
+          tmem_ld32(tbase + lane_off + c, r);
+          tmem_wait_ld();
 #pragma unroll
-      for (int jj = 0; jj < 4; ++jj) {
-        uint4 o;
-        o.x = pack_bf16(p[8 * jj + 0], p[8 * jj + 1]);
-        o.y = pack_bf16(p[8 * jj + 2], p[8 * jj + 3]);
-        o.z = pack_bf16(p[8 * jj + 4], p[8 * jj + 5]);
-        o.w = pack_bf16(p[8 * jj + 6], p[8 * jj + 7]);
-        *reinterpret_cast<uint4 *>(blk + (((ch0 + jj) ^ (row & 7)) << 4)) = o;
+          for (int jj = 0; jj < 32; ++jj) sv[jj] = __uint_as_float(r[jj]);
+        }
+        float p[32];
+#pragma unroll
+        for (int jj = 0; jj < 32; ++jj) {
+          p[jj] = (c + jj < S) ? ex2_approx(fmaf(sv[(kKeep ? ci * 32 : 0) + jj], sl2, -mb)) : 0.f;
+          l4[jj & 3] += p[jj];
+        }
+        // columns c..c+31 -> block c/64, 16-byte chunks (c%64)/8 .. +3, XOR-swizzled by row%8
+        uint8_t *blk = prow + (c / 64) * (QT * 128);
+        const int ch0 = (c % 64) / 8;
+#pragma unroll
+        for (int jj = 0; jj < 4; ++jj) {
+          uint4 o;
+          o.x = pack_bf16(p[8 * jj + 0], p[8 * jj + 1]);
+          o.y = pack_bf16(p[8 * jj + 2], p[8 * jj + 3]);
+          o.z = pack_bf16(p[8 * jj + 4], p[8 * jj + 5]);
+          o.w = pack_bf16(p[8 * jj + 6], p[8 * jj + 7]);
+          *reinterpret_cast<uint4 *>(blk + (((ch0 + jj) ^ (row & 7)) << 4)) = o;
+        }
       }
     }
     const float lpart = (l4[0] + l4[1]) + (l4[2] + l4[3]);
@@ -258,7 +281,9 @@ e3_status launch_attn(const AttnMaps &m, int B, int S, int H, int heads, cudaStr
     attr_done = true;
   }
   const int n_items = B * heads * ((S + QT - 1) / QT);
-  const int per_sm = (2 * ACfg<SKV>::kSmem <= 232448) ? 2 : 1;
+  int per_sm = 0;
+  E3_CUDA_TRY(cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per_sm, kern, kThreads, ACfg<SKV>::kSmem));
+  if (per_sm < 1) per_sm = 1;
   const int grid = n_items < per_sm * sms ? n_items : per_sm * sms;
   E3_CUDA_TRY(launch_k(kern, dim3(grid), dim3(kThreads), ACfg<SKV>::kSmem, st, m.q, m.kv, m.ctx, S, H, heads,
                        n_items));

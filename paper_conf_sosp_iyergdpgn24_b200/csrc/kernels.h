@@ -23,6 +23,23 @@ e3_status gemm_tmaps(GemmMaps *g, const void *A, int64_t lda, const void *W, con
 e3_status gemm_run(const GemmMaps &g, const void *bias, const void *R, int M, int N, int K, int epi, int sms,
                    cudaStream_t st);
 
+// ---- K1b projection + bias + residual + LayerNorm (gemm_ln.cu): cluster of
+// 2 CTAs per 128 rows, each owning N/2 columns; pre (optional) receives
+// y = bf16(A W^T + bias + R), out = bf16(LN(y) * g + b)
+struct LnGemmMaps {
+  CUtensorMap a, w, r, pre, out;
+};
+struct LnGemmArgs {
+  const __nv_bfloat16 *bias, *R, *g, *b;
+  float eps;
+  int M, N, K;
+  int store_pre;
+};
+bool ln_gemm_supported(int N, int K);
+e3_status ln_gemm_tmaps(LnGemmMaps *m, const void *A, const void *W, const void *R, const void *pre, const void *out,
+                        int M, int N, int K);
+e3_status ln_gemm_run(const LnGemmMaps &m, const LnGemmArgs &a, cudaStream_t st);
+
 // ---- K2 attention (attn_tc.cu)
 struct AttnMaps {
   CUtensorMap q;    // qkv [B][S][3H], box 64 x 128 x 1

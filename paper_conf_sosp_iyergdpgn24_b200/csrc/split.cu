@@ -15,6 +15,7 @@
 // of the split ("mark and carry"; R7), which yields plan-independent
 // results.  Activations ping-pong between two workspace buffers so the caller's
 // x_in is never written.
+#include <cstdlib>
 #include <cstring>
 #include <new>
 
@@ -289,6 +290,11 @@ e3_status split_create_shared(const e3_split_desc *d, const e3_weights *w, int d
   const int nl = d->layer_end - d->layer_begin;
   s->maps.resize(nl);
   const bool vit = d->arch == E3_ARCH_VIT;
+  // Fused O projection + LayerNorm (gemm_ln.cu) is opt-in: measured on B200
+  // at BB it is 16.3 us alone vs 18.6 us for the two kernels, but the split
+  // run is 2 % slower with it (128 one-CTA-per-SM clusters lose the PDL
+  // overlap the two shorter kernels get); DESIGN.md §6.
+  s->use_oln = ln_gemm_supported(H, H) && getenv("E3_FUSED_LN") != nullptr;
   for (int i = 0; i < nl && st == E3_OK; ++i) {
     auto &m = s->maps[i];
     const void *prev = (i % 2 == 1) ? ws->xa : ws->xb;   // output of layer i-1
@@ -301,6 +307,9 @@ e3_status split_create_shared(const e3_split_desc *d, const e3_weights *w, int d
       st = gemm_tmaps(&m.qkv, prev, H, s->L[i].w_qkv, ws->qkv, M, 3 * H, H, s->bn_qkv);
     }
     if (st == E3_OK) st = gemm_tmaps(&m.o, ws->ctx, H, s->L[i].w_o, ws->y, M, H, H, s->bn_o);
+    if (st == E3_OK && s->use_oln)   // BERT: x1 = LN1(y1); ViT: y1 kept (residual), n2 = LN2(y1)
+      st = ln_gemm_tmaps(&m.oln, ws->ctx, s->L[i].w_o, prev /* layer 0: the run's input, re-encoded per run */,
+                         vit ? ws->y : nullptr, ws->x1, M, H, H);
     if (st == E3_OK) st = gemm_tmaps(&m.f1, ws->x1, H, s->L[i].w_1, ws->h, M, F, H, s->bn_f1);
     if (st == E3_OK) st = gemm_tmaps(&m.f2, ws->h, F, s->L[i].w_2, vit ? out : ws->y, M, H, F, s->bn_f2);
   }
@@ -482,6 +491,21 @@ static e3_status llama_run(e3_split *s, cudaStream_t st, const void *x_in, const
   return E3_OK;
 }
 
+static LnGemmArgs oln_args(const void *bias, const void *R, const void *g, const void *b, float eps, int M, int H,
+                           int store_pre) {
+  LnGemmArgs a{};
+  a.bias = reinterpret_cast<const __nv_bfloat16 *>(bias);
+  a.R = reinterpret_cast<const __nv_bfloat16 *>(R);
+  a.g = reinterpret_cast<const __nv_bfloat16 *>(g);
+  a.b = reinterpret_cast<const __nv_bfloat16 *>(b);
+  a.eps = eps;
+  a.M = M;
+  a.N = H;
+  a.K = H;
+  a.store_pre = store_pre;
+  return a;
+}
+
 e3_status split_run_to(e3_split *s, cudaStream_t st, const void *x_in, const int64_t *id_in,
                        const int32_t *n_valid_dev, int n_valid_host, const RingDst &dst, int32_t *n_surv_dev,
                        const e3_exits *ex) {
@@ -528,11 +552,16 @@ e3_status split_run_to(e3_split *s, cudaStream_t st, const void *x_in, const int
         ProfScope ps(PK_ATTN, st, f_att, 0);
         E3_RUN(attn_run(s->attn, B, S, H, d.heads, st));
       }
-      {
+      if (s->use_oln) {
+        LnGemmMaps lm = m.oln;
+        if (i == 0) E3_RUN(make_tmap_2d(&lm.r, cur, (uint64_t)M, (uint64_t)H, (uint64_t)H, 128, 64));
         ProfScope ps(PK_GEMM_O, st, f_o, 0);
-        E3_RUN(gemm_run(m.o, L.b_o, cur, M, H, H, E3_EPI_BIAS_RESID, s->sms, st));
-      }
-      {
+        E3_RUN(ln_gemm_run(lm, oln_args(L.b_o, cur, L.ln2_g, L.ln2_b, d.norm_eps, M, H, 1), st));
+      } else {
+        {
+          ProfScope ps(PK_GEMM_O, st, f_o, 0);
+          E3_RUN(gemm_run(m.o, L.b_o, cur, M, H, H, E3_EPI_BIAS_RESID, s->sms, st));
+        }
         ProfScope ps(PK_LN, st, 0, b_ln);
         E3_RUN(layernorm_run(ws.y, L.ln2_g, L.ln2_b, ws.x1, M, H, d.norm_eps, st));
       }
@@ -560,11 +589,16 @@ e3_status split_run_to(e3_split *s, cudaStream_t st, const void *x_in, const int
       ProfScope ps(PK_ATTN, st, f_att, 0);
       E3_RUN(attn_run(s->attn, B, S, H, d.heads, st));
     }
-    {
+    if (s->use_oln) {
+      LnGemmMaps lm = m.oln;
+      if (i == 0) E3_RUN(make_tmap_2d(&lm.r, cur, (uint64_t)M, (uint64_t)H, (uint64_t)H, 128, 64));
       ProfScope ps(PK_GEMM_O, st, f_o, 0);
-      E3_RUN(gemm_run(m.o, L.b_o, cur, M, H, H, E3_EPI_BIAS_RESID, s->sms, st));
-    }
-    {
+      E3_RUN(ln_gemm_run(lm, oln_args(L.b_o, cur, L.ln1_g, L.ln1_b, d.norm_eps, M, H, 0), st));
+    } else {
+      {
+        ProfScope ps(PK_GEMM_O, st, f_o, 0);
+        E3_RUN(gemm_run(m.o, L.b_o, cur, M, H, H, E3_EPI_BIAS_RESID, s->sms, st));
+      }
       ProfScope ps(PK_LN, st, 0, b_ln);
       E3_RUN(layernorm_run(ws.y, L.ln1_g, L.ln1_b, ws.x1, M, H, d.norm_eps, st));
     }
@@ -742,6 +776,22 @@ e3_status e3_op_dec_gemm(void *stream, const void *X, int32_t T, const void *W, 
   cudaFreeAsync(part, st);
   cudaFreeAsync(tick, st);
   return r;
+}
+
+e3_status e3_op_gemm_ln(void *stream, const void *A, const void *W, const void *bias, const void *R, const void *g,
+                        const void *b, float eps, void *pre, void *out, int32_t M, int32_t N, int32_t K) {
+  E3_CHECK_ARG(A && W && bias && R && g && b && out && M > 0, "bad arguments");
+  if (!ln_gemm_supported(N, K) || !aligned16(A) || !aligned16(W) || !aligned16(R) || !aligned16(out) ||
+      (pre && !aligned16(pre))) {
+    set_error("e3_op_gemm_ln: need N in {128,256,384,512,640,768,1024}, K % 64 == 0, aligned buffers");
+    return E3_EUNSUPPORTED;
+  }
+  LnGemmMaps m;
+  e3_status r = ln_gemm_tmaps(&m, A, W, R, pre, out, M, N, K);
+  if (r != E3_OK) return r;
+  LnGemmArgs a = oln_args(bias, R, g, b, eps, M, N, pre != nullptr);
+  a.K = K;
+  return ln_gemm_run(m, a, reinterpret_cast<cudaStream_t>(stream));
 }
 
 e3_status e3_op_attention(void *stream, const void *qkv, void *ctx, int32_t B, int32_t S, int32_t H, int32_t heads) {

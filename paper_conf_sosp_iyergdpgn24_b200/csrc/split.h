@@ -46,7 +46,9 @@ struct e3_split {
   std::shared_ptr<e3::Workspace> ws;
   struct LayerMaps {
     e3::GemmMaps qkv, o, f1, f2;
+    e3::LnGemmMaps oln;   // fused O projection + residual + LayerNorm (when use_oln)
   };
+  bool use_oln = false;
   std::vector<LayerMaps> maps;
   // LLAMA decode: per layer the four decode GEMMs, per ramp the LM head
   struct DecLayer {

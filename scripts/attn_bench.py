@@ -14,11 +14,16 @@ out = torch.empty(B * S, H, device="cuda", dtype=torch.bfloat16)
 for _ in range(5):
     api.ops.attention(qkv, B, S, H, nh, out=out)
 torch.cuda.synchronize()
-a, b = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
 n = 50
+g = torch.cuda.CUDAGraph()            # device time only (the op API encodes tensor maps per call)
+with torch.cuda.graph(g):
+    for _ in range(n):
+        api.ops.attention(qkv, B, S, H, nh, out=out)
+g.replay()
+torch.cuda.synchronize()
+a, b = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
 a.record()
-for _ in range(n):
-    api.ops.attention(qkv, B, S, H, nh, out=out)
+g.replay()
 b.record()
 torch.cuda.synchronize()
 t = a.elapsed_time(b) / n * 1000

@@ -276,3 +276,37 @@ def test_dec_gemm_matches_definition(api, T, N, K, epi):
         y = silu(y) * (X.astype(np.float64) @ W2.astype(np.float64).T)
     # fp32 accumulation over up to 11008 terms + SiLU in fp32: 1 ulp + small atol
     _assert_bf16_close(to64(out), y, ulps=1.0, atol=2e-3 if K > 4096 else 5e-4, min_exact=0.9)
+
+
+@pytest.mark.parametrize("M,N,K", [(300, 128, 128), (1000, 768, 768), (520, 1024, 1024), (256, 384, 3072)])
+@pytest.mark.parametrize("with_pre", [False, True])
+def test_gemm_ln_matches_definition(api, M, N, K, with_pre):
+    """Fused O projection + residual + LayerNorm (cluster of 2 CTAs per row
+    block, row statistics exchanged through DSMEM) vs the oracle's
+    definition: y = bf16(A W^T + b + R), out = bf16(LN(y))."""
+    from oracle.encoder import layer_norm, linear
+    from oracle.numerics import bf16_rne
+    rng = np.random.default_rng(M + N + K)
+    A = rand_bf16(rng, (M, K))
+    W = rand_bf16(rng, (N, K), K ** -0.5)
+    b = rand_bf16(rng, (N,), 0.1)
+    R = rand_bf16(rng, (M, N))
+    g = rand_bf16(rng, (N,), 0.1) + 1.0
+    beta = rand_bf16(rng, (N,), 0.1)
+    pre = torch.zeros((M, N), dtype=torch.bfloat16, device=DEV) if with_pre else None
+    out = api.ops.gemm_ln(bf16_tensor(A), bf16_tensor(W), bf16_tensor(b), bf16_tensor(R), bf16_tensor(g),
+                          bf16_tensor(beta), 1e-12, pre=pre)
+    torch.cuda.synchronize()
+    y = bf16_rne(linear(A.astype(np.float64), W.astype(np.float64), b.astype(np.float64)) + R)
+    if with_pre:
+        _assert_bf16_close(to64(pre), linear(A.astype(np.float64), W.astype(np.float64), b.astype(np.float64)) + R,
+                           atol=1e-4)
+    # on the GPU's own rounded y: one rounding of the LN output (1 ulp); on
+    # the oracle's y, a 1-ulp difference of a y element (fp32 vs fp64
+    # accumulation) moves that output element by about one more ulp
+    yg = to64(pre) if with_pre else y
+    ref = layer_norm(yg, g.astype(np.float64), beta.astype(np.float64), 1e-12)
+    # (single-pass statistics E[y^2] - mean^2 in fp32: ~1e-7 relative on var)
+    # (a y element one ulp (<= 2^-7 |y|) off moves its output by <= 2^-7 |y| rstd g)
+    _assert_bf16_close(to64(out), ref, ulps=1.0 if with_pre else 3.0, atol=2e-3 if with_pre else 1e-2,
+                       min_exact=0.9 if with_pre else 0.5)
