@@ -291,7 +291,8 @@ def test_gemm_ln_matches_definition(api, M, N, K, with_pre):
     W = rand_bf16(rng, (N, K), K ** -0.5)
     b = rand_bf16(rng, (N,), 0.1)
     R = rand_bf16(rng, (M, N))
-    g = rand_bf16(rng, (N,), 0.1) + 1.0
+    from e3data import bf16_round
+    g = bf16_round(rand_bf16(rng, (N,), 0.1) + 1.0)     # gamma must be bf16-representable
     beta = rand_bf16(rng, (N,), 0.1)
     pre = torch.zeros((M, N), dtype=torch.bfloat16, device=DEV) if with_pre else None
     out = api.ops.gemm_ln(bf16_tensor(A), bf16_tensor(W), bf16_tensor(b), bf16_tensor(R), bf16_tensor(g),
@@ -308,5 +309,5 @@ def test_gemm_ln_matches_definition(api, M, N, K, with_pre):
     ref = layer_norm(yg, g.astype(np.float64), beta.astype(np.float64), 1e-12)
     # (single-pass statistics E[y^2] - mean^2 in fp32: ~1e-7 relative on var)
     # (a y element one ulp (<= 2^-7 |y|) off moves its output by <= 2^-7 |y| rstd g)
-    _assert_bf16_close(to64(out), ref, ulps=1.0 if with_pre else 3.0, atol=2e-3 if with_pre else 1e-2,
+    _assert_bf16_close(to64(out), ref, ulps=1.0 if with_pre else 2.0, atol=1e-3 if with_pre else 1e-2,
                        min_exact=0.9 if with_pre else 0.5)
