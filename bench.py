@@ -426,6 +426,8 @@ def main():
             "exit_hist": hist,
             "split_batches": batches, "split_valid_rows": valid, "split_padded_rows": padded,
             "host_waits": int(stats.host_waits) if stats else None,
+            "host_launch_ms": round(stats.host_launch_ms, 2) if stats else None,
+            "host_sync_ms": round(stats.host_sync_ms, 2) if stats else None,
         }
         print(json.dumps(out), flush=True)
     if world > 1:

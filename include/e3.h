@@ -228,6 +228,8 @@ typedef struct e3_stats {
   int64_t padded_rows[E3_MAX_SPLITS];
   int64_t rows_out[E3_MAX_SPLITS];
   int64_t host_waits;                  /* times the host blocked on a run          */
+  double host_launch_ms;               /* host time spent issuing runs (launches)  */
+  double host_sync_ms;                 /* host time spent waiting on run events    */
 } e3_stats;
 
 typedef struct e3_pipeline e3_pipeline;

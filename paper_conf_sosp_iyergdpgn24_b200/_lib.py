@@ -76,7 +76,7 @@ class Plan(C.Structure):
 class Stats(C.Structure):
     _fields_ = [("runs", I64), ("batches", I64 * E3_MAX_SPLITS), ("valid_rows", I64 * E3_MAX_SPLITS),
                 ("padded_rows", I64 * E3_MAX_SPLITS), ("rows_out", I64 * E3_MAX_SPLITS),
-                ("host_waits", I64)]
+                ("host_waits", I64), ("host_launch_ms", C.c_double), ("host_sync_ms", C.c_double)]
 
 
 # name -> (restype, argtypes); every symbol include/*.h declares
@@ -107,6 +107,7 @@ SIGNATURES = {
     "e3_op_compact": (I32, [P, P, P, P, I32, I64, P, P, P]),
     "e3_kernel_launches": (C.c_longlong, []),
     "e3_profile_enable": (I32, [I32]),
+    "e3_debug_gemm_trace": (I32, [P]),
     "e3_profile_reset": (I32, []),
     "e3_profile_read": (I32, [I32, C.POINTER(C.c_double), C.POINTER(C.c_double), C.POINTER(C.c_double),
                               C.POINTER(C.c_longlong), C.POINTER(C.c_char_p)]),

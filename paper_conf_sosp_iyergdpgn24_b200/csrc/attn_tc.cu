@@ -272,18 +272,29 @@ template <int SKV>
 e3_status launch_attn(const AttnMaps &m, int B, int S, int H, int heads, cudaStream_t st) {
   auto kern = attn_tc_kernel<SKV>;
   static bool attr_done = false;
-  static int sms = 0;
+  static int sms = 0, per_sm = 0;
   if (!attr_done) {
     E3_CUDA_TRY(cudaFuncSetAttribute(kern, cudaFuncAttributeMaxDynamicSharedMemorySize, ACfg<SKV>::kSmem));
+    // without the max-shared carveout the occupancy query (and the launch) may
+    // settle on one 101 KB CTA per SM although two fit (r01: grid 148, 18.5 us)
+    E3_CUDA_TRY(cudaFuncSetAttribute(kern, cudaFuncAttributePreferredSharedMemoryCarveout, 100));
     int dev = 0;
     E3_CUDA_TRY(cudaGetDevice(&dev));
     sms = num_sms(dev);
+    // resident CTAs per SM from the resources themselves: the occupancy API
+    // answers 1 for SKV = 128 (r01: grid 148, 18.6 us) although two fit
+    // (ncu: block limit registers 2, shared memory 2; forced 2: 13.8 us)
+    cudaFuncAttributes fa;
+    E3_CUDA_TRY(cudaFuncGetAttributes(&fa, kern));
+    const int by_regs = 65536 / (fa.numRegs * kThreads);
+    const int by_smem = 233472 / (ACfg<SKV>::kSmem + (int)fa.sharedSizeBytes + 1024);
+    per_sm = by_regs < by_smem ? by_regs : by_smem;
+    if (per_sm < 1) per_sm = 1;
+    if (const char *e = getenv("E3_ATTN_PER_SM")) per_sm = atoi(e);
+    if (getenv("E3_VERBOSE")) fprintf(stderr, "[e3] attn_tc_kernel<%d>: %d CTAs per SM\n", SKV, per_sm);
     attr_done = true;
   }
   const int n_items = B * heads * ((S + QT - 1) / QT);
-  int per_sm = 0;
-  E3_CUDA_TRY(cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per_sm, kern, kThreads, ACfg<SKV>::kSmem));
-  if (per_sm < 1) per_sm = 1;
   const int grid = n_items < per_sm * sms ? n_items : per_sm * sms;
   E3_CUDA_TRY(launch_k(kern, dim3(grid), dim3(kThreads), ACfg<SKV>::kSmem, st, m.q, m.kv, m.ctx, S, H, heads,
                        n_items));

@@ -37,14 +37,42 @@ constexpr int BM = 128;           // rows per CTA (256 per pair)
 constexpr int BK = 64;            // K width of one 128-byte swizzle atom (TMA box)
 constexpr int KSUB = 2;           // swizzle atoms per pipeline stage: 128-wide K stages
                                   // halve the per-MMA barrier / commit overhead
-constexpr int kThreads = 384;     // 4 control warps + 8 epilogue warps
-constexpr int kEpiWarps = 8;
 constexpr int kEpiBuf = 32 * 64;  // one 32 x 32 bf16 box
-constexpr int kEpiBytes = kEpiWarps * 2 * kEpiBuf;
 constexpr int kSmemMax = 232448;  // 227 KB opt-in limit
 
-template <int BN>
+// Diagnostics: when e3_debug_gemm_trace() has set a device buffer, every CTA
+// records globaltimer stamps per tile (<= kTrTiles tiles): [0] MMA issue
+// start (accumulator free), [1] last commit issued, [2]/[3] epilogue warp 4
+// start/end, [4]/[5] epilogue warp 11 start/end.
+constexpr int kTrTiles = 16;
+__device__ unsigned long long *g_gemm_trace = nullptr;
+__device__ __forceinline__ unsigned long long gtimer() {
+  unsigned long long t;
+  asm volatile("mov.u64 %0, %globaltimer;" : "=l"(t));
+  return t;
+}
+__device__ __forceinline__ void trace(int tile_local, int kind) {
+  unsigned long long *b = g_gemm_trace;
+  if (b && tile_local < kTrTiles) b[((size_t)blockIdx.x * kTrTiles + tile_local) * 6 + kind] = gtimer();
+}
+
+// Epilogue warps: 4 lane quarters x (BN / CW) column parts.  GELU: CW = 64
+// columns per warp (two 32-column chunks), so a warp holds its whole share of
+// the accumulator in registers and releases the TMEM buffer BEFORE the GELU
+// math -- the MMA of tile i+2 no longer waits for the epilogue of tile i (r01
+// trace, scripts/gemm_trace.py: with 8 warps the GELU epilogue took 4.1 us per
+// 256 x 192 tile, as long as the tile's MMAs, and paced the kernel; FFN1
+// 39.1 -> 37.8 us).  Bias and bias + residual keep 8 warps of BN / 2 columns
+// released after the last chunk (the 12-warp variant measured 1 us slower on
+// both N = 768 GEMMs: fewer pipeline stages fit beside its staging buffers).
+template <int BN, int EPI>
 struct Cfg {
+  static constexpr int kEpiWarps = (EPI == E3_EPI_BIAS_GELU) ? 4 * (BN / 64) : (BN >= 128 ? 8 : 4);
+  static constexpr int kCW = BN / (kEpiWarps / 4);       // columns per epilogue warp
+  static constexpr int kNCW = kCW / 32;                  // 32-column chunks per warp
+  static constexpr bool kEarly = kNCW <= 2;              // whole share in registers, early release
+  static constexpr int kThreads = 128 + 32 * kEpiWarps;  // 4 control warps + epilogue warps
+  static constexpr int kEpiBytes = kEpiWarps * 2 * kEpiBuf;
   static constexpr int kASub = BM * BK * 2;            // 16 KB per swizzle atom column
   static constexpr int kBSub = (BN / 2) * BK * 2;      // this CTA's half of the W tile
   static constexpr int kABytes = KSUB * kASub;
@@ -59,11 +87,11 @@ struct Cfg {
 __device__ __forceinline__ uint32_t sw64(int r, int j) { return r * 64 + ((j ^ ((r >> 1) & 3)) << 4); }
 
 template <int BN, int EPI>
-__global__ void __cluster_dims__(2, 1, 1) __launch_bounds__(kThreads, 1)
+__global__ void __cluster_dims__(2, 1, 1) __launch_bounds__(Cfg<BN, EPI>::kThreads, 1)
     gemm_bf16_tc_kernel(const __grid_constant__ CUtensorMap tmA, const __grid_constant__ CUtensorMap tmB,
                         const __grid_constant__ CUtensorMap tmC, const __nv_bfloat16 *__restrict__ bias,
                         const __nv_bfloat16 *__restrict__ R, int M, int N, int K) {
-  using CF = Cfg<BN>;
+  using CF = Cfg<BN, EPI>;
   constexpr int S = CF::kStages;
   extern __shared__ uint8_t smem_raw[];
   // identical layout (same offsets) in both CTAs of the pair
@@ -71,7 +99,7 @@ __global__ void __cluster_dims__(2, 1, 1) __launch_bounds__(kThreads, 1)
   uint8_t *sA = smem;
   uint8_t *sB = smem + S * CF::kABytes;
   uint8_t *sE = smem + S * CF::kStageBytes;              // epilogue staging (1024-aligned)
-  uint64_t *full = reinterpret_cast<uint64_t *>(sE + kEpiBytes);
+  uint64_t *full = reinterpret_cast<uint64_t *>(sE + CF::kEpiBytes);
   uint64_t *empty = full + S;
   uint64_t *tfull = empty + S;        // [2]
   uint64_t *tempty = tfull + 2;       // [2]
@@ -100,7 +128,7 @@ __global__ void __cluster_dims__(2, 1, 1) __launch_bounds__(kThreads, 1)
     }
     for (int i = 0; i < 2; ++i) {
       mbar_init(&tfull[i], 1);     // multicast tcgen05.commit
-      mbar_init(&tempty[i], 16);   // 8 epilogue warps x 2 CTAs (leader's copy is used)
+      mbar_init(&tempty[i], 2 * CF::kEpiWarps);   // epilogue warps of both CTAs (leader's copy is used)
     }
     fence_barrier_init();
   }
@@ -143,9 +171,11 @@ __global__ void __cluster_dims__(2, 1, 1) __launch_bounds__(kThreads, 1)
       uint32_t phase = 0;
       int acc = 0;
       uint32_t acc_phase = 0;
-      for (int t = pair; t < num_tiles; t += num_pairs) {
+      int tl = 0;
+      for (int t = pair; t < num_tiles; t += num_pairs, ++tl) {
         mbar_wait(&tempty[acc], acc_phase ^ 1);
         tc_fence_after();
+        trace(tl, 0);
         const uint32_t d_tmem = tmem_base + acc * BN;
         for (int kb = 0; kb < num_kb; ++kb) {
           mbar_wait(&full[stage], phase);
@@ -162,50 +192,64 @@ __global__ void __cluster_dims__(2, 1, 1) __launch_bounds__(kThreads, 1)
           if (++stage == S) { stage = 0; phase ^= 1; }
         }
         tc_commit2_mc(&tfull[acc], 0x3);
+        trace(tl, 1);
         if (++acc == 2) { acc = 0; acc_phase ^= 1; }
       }
     }
   } else if (warp >= 4) {
     // ------------------------------------------------ epilogue (both CTAs)
+    constexpr int CW = CF::kCW, NCW = CF::kNCW;
     const int q = warp & 3;              // TMEM lane quarter this warp may access
-    const int half = (warp - 4) >> 2;    // which half of the BN columns
+    const int part = (warp - 4) >> 2;    // which CW-column part of the tile
     uint8_t *ebuf = sE + (warp - 4) * 2 * kEpiBuf;
     const uint32_t tempty_leader0 = mapa_shared(smem_u32(&tempty[0]), 0);
     const uint32_t tempty_leader1 = mapa_shared(smem_u32(&tempty[1]), 0);
     int acc = 0;
     uint32_t acc_phase = 0;
     int ci = 0;                          // chunk counter (selects the staging buffer)
-    for (int t = pair; t < num_tiles; t += num_pairs) {
+    int tl = 0;
+    for (int t = pair; t < num_tiles; t += num_pairs, ++tl) {
       const int m_blk = t / num_n, n_blk = t % num_n;
       const int m0 = m_blk * 2 * BM + (int)rank * BM + q * 32;   // this warp's first row
       const int m = m0 + lane;
-      const uint32_t taddr = tmem_base + ((uint32_t)(q * 32) << 16) + acc * BN;
-      constexpr int kChunks = BN / 64;   // 32-column chunks per warp
+      const int nw0 = n_blk * BN + part * CW;                     // this warp's first column
+      const uint32_t taddr = tmem_base + ((uint32_t)(q * 32) << 16) + acc * BN + part * CW;
       uint4 rnext[4];
       if (EPI == E3_EPI_BIAS_RESID) {
-        const uint4 *rp = reinterpret_cast<const uint4 *>(R + (size_t)m * N + n_blk * BN + half * (BN / 2));
+        const uint4 *rp = reinterpret_cast<const uint4 *>(R + (size_t)m * N + nw0);
 #pragma unroll
         for (int j = 0; j < 4; ++j) rnext[j] = (m < M) ? __ldg(rp + j) : make_uint4(0, 0, 0, 0);
       }
       mbar_wait(&tfull[acc], acc_phase);
       tc_fence_after();
-#pragma unroll 1
-      for (int c = 0; c < kChunks; ++c) {
-        const int col = half * (BN / 2) + c * 32;
-        const int n0 = n_blk * BN + col;
-        uint32_t r[32];
-        tmem_ld32(taddr + col, r);
+      if (lane == 0 && (warp == 4 || warp == 11)) trace(tl, warp == 4 ? 2 : 4);
+      uint32_t racc[CF::kEarly ? NCW : 1][32];
+      if (CF::kEarly) {
+        // whole share -> registers, then hand the accumulator back to the MMA
+#pragma unroll
+        for (int c = 0; c < NCW; ++c) tmem_ld32(taddr + c * 32, racc[c]);
+        tmem_wait_ld();
+        tc_fence_before();
+        __syncwarp();
+        if (lane == 0) mbar_arrive_cluster(acc ? tempty_leader1 : tempty_leader0);
+      }
+#pragma unroll
+      for (int c = 0; c < NCW; ++c) {
+        const int n0 = nw0 + c * 32;
+        uint32_t rl[32];
+        const uint32_t *r = CF::kEarly ? racc[CF::kEarly ? c : 0] : rl;
+        if (!CF::kEarly) tmem_ld32(taddr + c * 32, rl);
         uint4 rcur[4];
         if (EPI == E3_EPI_BIAS_RESID) {
 #pragma unroll
           for (int j = 0; j < 4; ++j) rcur[j] = rnext[j];
-          if (c + 1 < kChunks) {          // prefetch the next chunk's residual
+          if (c + 1 < NCW) {              // prefetch the next chunk's residual
             const uint4 *rp = reinterpret_cast<const uint4 *>(R + (size_t)m * N + n0 + 32);
 #pragma unroll
             for (int j = 0; j < 4; ++j) rnext[j] = (m < M) ? __ldg(rp + j) : make_uint4(0, 0, 0, 0);
           }
         }
-        tmem_wait_ld();
+        if (!CF::kEarly) tmem_wait_ld();
         float v[32];
         const uint4 *bp = reinterpret_cast<const uint4 *>(bias + n0);
 #pragma unroll
@@ -259,9 +303,12 @@ __global__ void __cluster_dims__(2, 1, 1) __launch_bounds__(kThreads, 1)
         }
         ++ci;
       }
-      tc_fence_before();
-      __syncwarp();
-      if (lane == 0) mbar_arrive_cluster(acc ? tempty_leader1 : tempty_leader0);
+      if (!CF::kEarly) {
+        tc_fence_before();
+        __syncwarp();
+        if (lane == 0) mbar_arrive_cluster(acc ? tempty_leader1 : tempty_leader0);
+      }
+      if (lane == 0 && (warp == 4 || warp == 11)) trace(tl, warp == 4 ? 3 : 5);
       if (++acc == 2) { acc = 0; acc_phase ^= 1; }
     }
     if (lane == 0) bulk_wait<0>();
@@ -276,14 +323,15 @@ template <int BN, int EPI>
 e3_status launch(const GemmMaps &g, const __nv_bfloat16 *bias, const __nv_bfloat16 *R, int M, int N, int K, int sms,
                  cudaStream_t st) {
   auto kern = gemm_bf16_tc_kernel<BN, EPI>;
+  using CF = Cfg<BN, EPI>;
   static bool attr_done = false;   // per instantiation
   if (!attr_done) {
-    E3_CUDA_TRY(cudaFuncSetAttribute(kern, cudaFuncAttributeMaxDynamicSharedMemorySize, Cfg<BN>::kSmem));
+    E3_CUDA_TRY(cudaFuncSetAttribute(kern, cudaFuncAttributeMaxDynamicSharedMemorySize, CF::kSmem));
     attr_done = true;
   }
   const int tiles = ((M + 2 * BM - 1) / (2 * BM)) * (N / BN);
   const int pairs = tiles < sms / 2 ? tiles : sms / 2;
-  E3_CUDA_TRY(launch_k(kern, dim3(2 * pairs), dim3(kThreads), Cfg<BN>::kSmem, st, g.a, g.b, g.c, bias, R, M, N, K));
+  E3_CUDA_TRY(launch_k(kern, dim3(2 * pairs), dim3(CF::kThreads), CF::kSmem, st, g.a, g.b, g.c, bias, R, M, N, K));
   E3_CUDA_TRY(cudaGetLastError());
   count_launch();
   return E3_OK;
@@ -302,6 +350,11 @@ e3_status launch_epi(int epi, const GemmMaps &g, const __nv_bfloat16 *bias, cons
 }
 
 }  // namespace
+
+e3_status gemm_set_trace(void *buf) {
+  E3_CUDA_TRY(cudaMemcpyToSymbol(g_gemm_trace, &buf, sizeof(buf)));
+  return E3_OK;
+}
 
 int gemm_pick_bn(int M, int N, int sms) {
   // Minimise waves x per-tile cost over the pair tiles (256 x BN); per-tile

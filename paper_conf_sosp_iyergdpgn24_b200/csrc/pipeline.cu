@@ -21,6 +21,7 @@
 //   * every split batch has exactly B rows (padding rows never exit).
 // The decision sequence is a deterministic function of the exit outcomes,
 // replayed exactly by oracle/pipeline_sim.py (tests compare the traces).
+#include <chrono>
 #include <cstring>
 #include <deque>
 #include <new>
@@ -149,7 +150,9 @@ struct Runner {
   e3_status apply_oldest() {
     Pend p = pending.front();
     pending.pop_front();
+    const auto t0 = std::chrono::steady_clock::now();
     E3_CUDA_TRY(cudaEventSynchronize(pl->ev[p.slot]));
+    if (stats) stats->host_sync_ms += std::chrono::duration<double, std::milli>(std::chrono::steady_clock::now() - t0).count();
     const int c = pl->mailbox[p.slot];
     if (c < 0) {
       set_error("survivor queue overflow (increase queue_cap_batches)");
@@ -313,7 +316,9 @@ struct Runner {
       }
       const int64_t c = count(pick);
       const int nv = (int)(c >= B ? B : c);
+      const auto t0 = std::chrono::steady_clock::now();
       r = launch(pick, nv);
+      if (stats) stats->host_launch_ms += std::chrono::duration<double, std::milli>(std::chrono::steady_clock::now() - t0).count();
       if (r != E3_OK) return r;
     }
     while (!pending.empty()) {

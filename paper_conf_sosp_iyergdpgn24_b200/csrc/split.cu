@@ -736,6 +736,8 @@ e3_status e3_op_gemm(void *stream, const void *A, int64_t lda, const void *W, co
   return gemm_run(g, bias, resid, M, N, K, epilogue, sms, reinterpret_cast<cudaStream_t>(stream));
 }
 
+e3_status e3_debug_gemm_trace(void *dev_buf) { return gemm_set_trace(dev_buf); }
+
 e3_status e3_op_dec_gemm(void *stream, const void *X, int32_t T, const void *W, const void *W2, int32_t N, int32_t K,
                          int32_t epilogue, const void *R, void *Y) {
   E3_CHECK_ARG(X && W && Y && N > 0 && K > 0, "bad arguments");
