@@ -25,6 +25,20 @@
 
 namespace e3 {
 
+namespace {
+// Diagnostics only: E3_SKIP=<bitmask of profile kinds> leaves those kernels of
+// the BERT split path out (results are then meaningless; used to measure each
+// kernel's incremental cost inside the PDL-chained sequence,
+// scripts/layer_time.py).
+bool skip(int kind) {
+  static const int mask = [] {
+    const char *e = getenv("E3_SKIP");
+    return e ? atoi(e) : 0;
+  }();
+  return (mask >> kind) & 1;
+}
+}  // namespace
+
 Workspace::~Workspace() {
   int prev = 0;
   cudaGetDevice(&prev);
@@ -580,42 +594,42 @@ e3_status split_run_to(e3_split *s, cudaStream_t st, const void *x_in, const int
       if (i == 0) {
         GemmMaps g0;
         E3_RUN(gemm_tmaps(&g0, cur, H, L.w_qkv, ws.qkv, M, 3 * H, H, s->bn_qkv));
-        E3_RUN(gemm_run(g0, L.b_qkv, nullptr, M, 3 * H, H, E3_EPI_BIAS, s->sms, st));
+        if (!skip(PK_GEMM_QKV)) E3_RUN(gemm_run(g0, L.b_qkv, nullptr, M, 3 * H, H, E3_EPI_BIAS, s->sms, st));
       } else {
-        E3_RUN(gemm_run(m.qkv, L.b_qkv, nullptr, M, 3 * H, H, E3_EPI_BIAS, s->sms, st));
+        if (!skip(PK_GEMM_QKV)) E3_RUN(gemm_run(m.qkv, L.b_qkv, nullptr, M, 3 * H, H, E3_EPI_BIAS, s->sms, st));
       }
     }
     {
       ProfScope ps(PK_ATTN, st, f_att, 0);
-      E3_RUN(attn_run(s->attn, B, S, H, d.heads, st));
+      if (!skip(PK_ATTN)) E3_RUN(attn_run(s->attn, B, S, H, d.heads, st));
     }
     if (s->use_oln) {
       LnGemmMaps lm = m.oln;
       if (i == 0) E3_RUN(make_tmap_2d(&lm.r, cur, (uint64_t)M, (uint64_t)H, (uint64_t)H, 128, 64));
       ProfScope ps(PK_GEMM_O, st, f_o, 0);
-      E3_RUN(ln_gemm_run(lm, oln_args(L.b_o, cur, L.ln1_g, L.ln1_b, d.norm_eps, M, H, 0), st));
+      if (!skip(PK_GEMM_O)) E3_RUN(ln_gemm_run(lm, oln_args(L.b_o, cur, L.ln1_g, L.ln1_b, d.norm_eps, M, H, 0), st));
     } else {
       {
         ProfScope ps(PK_GEMM_O, st, f_o, 0);
-        E3_RUN(gemm_run(m.o, L.b_o, cur, M, H, H, E3_EPI_BIAS_RESID, s->sms, st));
+        if (!skip(PK_GEMM_O)) E3_RUN(gemm_run(m.o, L.b_o, cur, M, H, H, E3_EPI_BIAS_RESID, s->sms, st));
       }
       ProfScope ps(PK_LN, st, 0, b_ln);
-      E3_RUN(layernorm_run(ws.y, L.ln1_g, L.ln1_b, ws.x1, M, H, d.norm_eps, st));
+      if (!skip(PK_LN)) E3_RUN(layernorm_run(ws.y, L.ln1_g, L.ln1_b, ws.x1, M, H, d.norm_eps, st));
     }
     {
       ProfScope ps(PK_GEMM_FFN1, st, f_1, 0);
-      E3_RUN(gemm_run(m.f1, L.b_1, nullptr, M, F, H, E3_EPI_BIAS_GELU, s->sms, st));
+      if (!skip(PK_GEMM_FFN1)) E3_RUN(gemm_run(m.f1, L.b_1, nullptr, M, F, H, E3_EPI_BIAS_GELU, s->sms, st));
     }
     {
       ProfScope ps(PK_GEMM_FFN2, st, f_1, 0);
-      E3_RUN(gemm_run(m.f2, L.b_2, ws.x1, M, H, F, E3_EPI_BIAS_RESID, s->sms, st));
+      if (!skip(PK_GEMM_FFN2)) E3_RUN(gemm_run(m.f2, L.b_2, ws.x1, M, H, F, E3_EPI_BIAS_RESID, s->sms, st));
     }
     // The split's last layer never materialises LN2: its ramp normalises the
     // CLS rows itself and the fused LN2 + compaction normalises only the
     // survivors, writing them straight to the destination.
     if (!last_layer) {
       ProfScope ps(PK_LN, st, 0, b_ln);
-      E3_RUN(layernorm_run(ws.y, L.ln2_g, L.ln2_b, out, M, H, d.norm_eps, st));
+      if (!skip(PK_LN)) E3_RUN(layernorm_run(ws.y, L.ln2_g, L.ln2_b, out, M, H, d.norm_eps, st));
       cur = out;
     }
     }
@@ -652,7 +666,7 @@ e3_status split_run_to(e3_split *s, cudaStream_t st, const void *x_in, const int
           const double hh = vit ? 0.0 : 2.0 * H * H;
           ProfScope ps(PK_RAMP, st, (double)n_valid_host * (hh + 2.0 * H * d.num_labels),
                        hh + 2.0 * n_valid_host * H + 2.0 * d.num_labels * H);
-          E3_RUN(ramp_run(a, st));
+          if (!skip(PK_RAMP)) E3_RUN(ramp_run(a, st));
         }
         first_ramp = false;
       }
@@ -664,6 +678,7 @@ e3_status split_run_to(e3_split *s, cudaStream_t st, const void *x_in, const int
     // (bytes added once n_surv is known, in the pipeline)
     const e3_layer_weights &L = s->L[nl - 1];
     ProfScope ps(PK_COMPACT, st, 0, 0);
+    if (skip(PK_COMPACT)) return E3_OK;
     if (vit)   // pre-LN: the layer output is final, survivors are copied
       E3_RUN(ln_compact_run(cur, id_in, ws.alive, B, S, H, nullptr, nullptr, d.norm_eps, dst, n_surv_dev, s->sms,
                             st));
