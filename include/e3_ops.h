@@ -90,12 +90,14 @@ e3_status e3_profile_reset(void);
 e3_status e3_profile_read(int32_t kind, double *ms, double *flops, double *bytes, long long *launches,
                           const char **name);
 
-/* Layer-GEMM timeline (diagnostics).  dev_buf: NULL (off, the default) or a
- * caller-owned device buffer of grid x 16 x 6 uint64 that every later
- * e3_op_gemm / split GEMM launch fills with globaltimer stamps (ns) per CTA and
- * per tile (<= 16 tiles): MMA start, last MMA commit, epilogue warp 4
- * start / end, epilogue warp 11 start / end.  Not thread-safe; E3_ECUDA if
- * the symbol copy fails. */
+/* Kernel timelines (diagnostics).  dev_buf: NULL (off, the default) or a
+ * caller-owned device buffer of 148 x 16 x 6 + 296 x 8 x 6 uint64.  Every
+ * later layer-GEMM launch fills the first part with globaltimer stamps (ns)
+ * per CTA and per tile (<= 16 tiles): MMA start, last MMA commit, epilogue
+ * warp 4 start / end, epilogue warp 11 start / end; every attention launch
+ * fills the second part per CTA and item (<= 8): loads landed, S ready, P
+ * ready, O ready, output stored.  Not thread-safe; E3_ECUDA if the symbol
+ * copy fails. */
 e3_status e3_debug_gemm_trace(void *dev_buf);
 
 #ifdef __cplusplus

@@ -52,6 +52,19 @@ struct ACfg {
   static constexpr int kTmemCols = SKV <= 128 ? 128 : 256;   // S, later O (64 columns)
 };
 
+// Diagnostics (e3_debug_gemm_trace): per CTA and item (<= 8), globaltimer
+// stamps: [0] loads landed, [1] S in TMEM, [2] P in smem (MMA2 issued),
+// [3] O in TMEM, [4] output staged (store issued)
+__device__ unsigned long long *g_attn_trace = nullptr;
+__device__ __forceinline__ void atrace(int j, int kind) {
+  unsigned long long *b = g_attn_trace;
+  if (b && j < 8) {
+    unsigned long long t;
+    asm volatile("mov.u64 %0, %globaltimer;" : "=l"(t));
+    b[((size_t)blockIdx.x * 8 + j) * 6 + kind] = t;
+  }
+}
+
 template <int SKV>
 __global__ void __launch_bounds__(kThreads, SKV == 128 ? 2 : 1)
     attn_tc_kernel(const __grid_constant__ CUtensorMap tq, const __grid_constant__ CUtensorMap tkv,
@@ -124,6 +137,7 @@ __global__ void __launch_bounds__(kThreads, SKV == 128 ? 2 : 1)
     if (tid == 0) {
       mbar_wait(&bar_load[buf], (load_phases >> buf) & 1u);
       tc_fence_after();
+      atrace(j, 0);
       const uint32_t idesc = idesc_bf16_f32(QT, SKV, 0);
       const uint64_t dq = smem_desc_sw128(smem_u32(sQ), 16, 1024);
       const uint64_t dk = smem_desc_sw128(smem_u32(sK), 16, 1024);
@@ -144,6 +158,7 @@ __global__ void __launch_bounds__(kThreads, SKV == 128 ? 2 : 1)
     mbar_wait(bar_s, sphase);
     sphase ^= 1;
     tc_fence_after();
+    if (tid == 0) atrace(j, 1);
     // S = 128: S is read from TMEM once, this thread's 64 keys stay in
     // registers between the max pass and the exponentiation pass (-6 %);
     // longer rows would spill, so they are read twice
@@ -221,6 +236,7 @@ __global__ void __launch_bounds__(kThreads, SKV == 128 ? 2 : 1)
 
     if (tid == 0) {
       tc_fence_after();
+      atrace(j, 2);
       const uint32_t idesc = idesc_bf16_f32(QT, D, 1);   // B (= V) is MN-major
 #pragma unroll
       for (int kk = 0; kk < SKV / 16; ++kk) {
@@ -234,6 +250,7 @@ __global__ void __launch_bounds__(kThreads, SKV == 128 ? 2 : 1)
     mbar_wait(bar_o, ophase);     // MMA2 done: V tile is dead -> output staging
     ophase ^= 1;
     tc_fence_after();
+    if (tid == 0) atrace(j, 3);
     __syncthreads();              // xsum[row] written by the khalf-0 thread
     const float inv_l = 1.0f / xsum[row];
     {
@@ -255,6 +272,7 @@ __global__ void __launch_bounds__(kThreads, SKV == 128 ? 2 : 1)
     tc_fence_before();            // O read before the next MMA1 overwrites TMEM
     __syncthreads();
     if (tid == 0) {
+      atrace(j, 4);
       tma_store_3d(&tctx, sV, h * D, q0, b);
       bulk_commit();
       if (CF::kNBuf == 1 && next < n_items) {
@@ -304,6 +322,11 @@ e3_status launch_attn(const AttnMaps &m, int B, int S, int H, int heads, cudaStr
 }
 
 }  // namespace
+
+e3_status attn_set_trace(void *buf) {
+  E3_CUDA_TRY(cudaMemcpyToSymbol(g_attn_trace, &buf, sizeof(buf)));
+  return E3_OK;
+}
 
 e3_status attn_tmaps(AttnMaps *m, const void *qkv, const void *ctx, int B, int S, int H) {
   m->skv = S <= 128 ? 128 : ((S + 31) / 32) * 32;

@@ -751,7 +751,10 @@ e3_status e3_op_gemm(void *stream, const void *A, int64_t lda, const void *W, co
   return gemm_run(g, bias, resid, M, N, K, epilogue, sms, reinterpret_cast<cudaStream_t>(stream));
 }
 
-e3_status e3_debug_gemm_trace(void *dev_buf) { return gemm_set_trace(dev_buf); }
+e3_status e3_debug_gemm_trace(void *dev_buf) {
+  const e3_status r = gemm_set_trace(dev_buf);
+  return r != E3_OK ? r : attn_set_trace(dev_buf ? static_cast<uint64_t *>(dev_buf) + 148 * 16 * 6 : nullptr);
+}
 
 e3_status e3_op_dec_gemm(void *stream, const void *X, int32_t T, const void *W, const void *W2, int32_t N, int32_t K,
                          int32_t epilogue, const void *R, void *Y) {

@@ -18,7 +18,7 @@ W = (torch.randn(N, K, device=dev) * K ** -0.5).to(torch.bfloat16)
 bias = torch.randn(N, device=dev).to(torch.bfloat16)
 R = torch.randn(M, N, device=dev).to(torch.bfloat16)
 C = torch.empty(M, N, device=dev, dtype=torch.bfloat16)
-buf = torch.zeros(148 * 16 * 6, dtype=torch.int64, device=dev)
+buf = torch.zeros(148 * 16 * 6 + 296 * 8 * 6, dtype=torch.int64, device=dev)
 run = lambda: api.ops.gemm(A, W, bias, epi, resid=R if epi == "bias_resid" else None, out=C)  # noqa: E731
 for _ in range(3):
     run()
@@ -27,7 +27,7 @@ _lib.lib.e3_debug_gemm_trace(buf.data_ptr())
 run()
 torch.cuda.synchronize()
 _lib.lib.e3_debug_gemm_trace(None)
-t = buf.cpu().numpy().reshape(148, 16, 6).astype(np.float64)
+t = buf.cpu().numpy()[: 148 * 16 * 6].reshape(148, 16, 6).astype(np.float64)
 valid = t[:, :, 2] > 0
 has_mma = t[:, :, 1] > 0
 t0 = t[t > 0].min()
