@@ -100,6 +100,16 @@ e3_status e3_profile_read(int32_t kind, double *ms, double *flops, double *bytes
  * copy fails. */
 e3_status e3_debug_gemm_trace(void *dev_buf);
 
+/* Diagnostics: kernel timeline of the encoder split path.  dev_buf = NULL
+ * disables it; otherwise a zeroed device buffer of 1 + 4 * 32768 uint64:
+ * buf[0] counts records, and thread 0 of every CTA of the layer GEMMs,
+ * attention, LayerNorm, BERT ramp and fused LN + compaction kernels appends
+ * {kernel id | blockIdx.x << 16, entry, released from griddepcontrol.wait,
+ * end} globaltimer stamps (ns).  Kernel ids: 1000 + BN + epilogue (GEMM),
+ * 2000 + key tile (attention), 3 LayerNorm, 4 ramp CTA, 5 ramp decision
+ * CTA, 6 compaction.  Not thread-safe; E3_ECUDA if a symbol copy fails. */
+e3_status e3_debug_timeline(void *dev_buf);
+
 #ifdef __cplusplus
 }
 #endif

@@ -108,6 +108,7 @@ SIGNATURES = {
     "e3_kernel_launches": (C.c_longlong, []),
     "e3_profile_enable": (I32, [I32]),
     "e3_debug_gemm_trace": (I32, [P]),
+    "e3_debug_timeline": (I32, [P]),
     "e3_profile_reset": (I32, []),
     "e3_profile_read": (I32, [I32, C.POINTER(C.c_double), C.POINTER(C.c_double), C.POINTER(C.c_double),
                               C.POINTER(C.c_longlong), C.POINTER(C.c_char_p)]),

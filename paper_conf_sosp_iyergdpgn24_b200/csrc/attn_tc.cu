@@ -83,6 +83,7 @@ __global__ void __launch_bounds__(kThreads, SKV == 128 ? 2 : 1)
 
   const int warp = warp_id(), lane = lane_id();
   const int tid = threadIdx.x;
+  const unsigned long long tl0 = tl_now();
   const int qtiles = (S + QT - 1) / QT;
   const int quarter = warp & 3;
   const int khalf = warp >> 2;                            // which half of the keys / of D
@@ -107,6 +108,7 @@ __global__ void __launch_bounds__(kThreads, SKV == 128 ? 2 : 1)
   const uint32_t tbase = *tslot;
   pdl_wait();                       // qkv of the previous kernel now visible
   pdl_trigger();
+  const unsigned long long tl1 = tl_now();
 
   auto issue_load = [&](int item, int buf) {
     const int bh = item / qtiles, qt = item % qtiles;
@@ -284,6 +286,7 @@ __global__ void __launch_bounds__(kThreads, SKV == 128 ? 2 : 1)
   if (tid == 0) bulk_wait<0>();
   __syncthreads();
   if (warp == 0) tmem_dealloc(tbase, CF::kTmemCols);
+  if (tid == 0) tl_rec(2000 + SKV, tl0, tl1);
 }
 
 template <int SKV>
@@ -322,6 +325,8 @@ e3_status launch_attn(const AttnMaps &m, int B, int S, int H, int heads, cudaStr
 }
 
 }  // namespace
+
+E3_TL_SETTER(tl_set_attn)
 
 e3_status attn_set_trace(void *buf) {
   E3_CUDA_TRY(cudaMemcpyToSymbol(g_attn_trace, &buf, sizeof(buf)));

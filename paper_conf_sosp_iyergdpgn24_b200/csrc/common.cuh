@@ -7,6 +7,7 @@
 #include <cuda_bf16.h>
 #include <cuda_runtime.h>
 #include <stdint.h>
+#include <stdlib.h>
 
 #include <string>
 
@@ -344,6 +345,38 @@ __device__ __forceinline__ float2 gelu_fast2(float2 x) {
 
 __device__ __forceinline__ int warp_id() { return threadIdx.x >> 5; }
 __device__ __forceinline__ int lane_id() { return threadIdx.x & 31; }
+
+
+// ---- diagnostics: kernel timeline (e3_debug_timeline).  When a device buffer
+// is set (per translation unit: tl_set_<file>), thread 0 of every CTA of the
+// instrumented kernels appends {kernel id | blockIdx.x << 16, entry, released
+// (after griddepcontrol.wait), end} globaltimer stamps; buf[0] is the count.
+namespace {
+__device__ unsigned long long *g_tl = nullptr;
+}
+constexpr int kTlCap = 1 << 15;
+__device__ __forceinline__ unsigned long long tl_now() {
+  unsigned long long t;
+  asm volatile("mov.u64 %0, %globaltimer;" : "=l"(t));
+  return t;
+}
+__device__ __forceinline__ void tl_rec(int kid, unsigned long long t0, unsigned long long t1) {
+  unsigned long long *b = g_tl;
+  if (!b) return;
+  const unsigned long long t2 = tl_now();
+  const unsigned long long i = atomicAdd(b, 1ull);
+  if (i >= (unsigned long long)kTlCap) return;
+  b[1 + 4 * i] = (unsigned long long)kid | ((unsigned long long)blockIdx.x << 16);
+  b[2 + 4 * i] = t0;
+  b[3 + 4 * i] = t1;
+  b[4 + 4 * i] = t2;
+}
+#define E3_TL_SETTER(name)                                             \
+  e3_status name(void *buf) {                                         \
+    unsigned long long *p = static_cast<unsigned long long *>(buf);   \
+    E3_CUDA_TRY(cudaMemcpyToSymbol(g_tl, &p, sizeof(p)));             \
+    return E3_OK;                                                     \
+  }
 
 #endif  // __CUDACC__
 

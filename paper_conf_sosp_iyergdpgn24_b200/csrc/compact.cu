@@ -189,11 +189,13 @@ __global__ void __launch_bounds__(kThreads)
                       const __nv_bfloat16 *__restrict__ bb, float eps, RingDst dst, int32_t *n_surv_dev) {
   __shared__ int16_t src_of[kMaxB];
   __shared__ int word_cnt[kMaxB / 32 + 1];
+  const unsigned long long tl0 = tl_now();
   const int warp = warp_id(), lane = lane_id();
   LnParams<VPL> p;
   if (kLn) ln_load_params<VPL>(p, g, bb, H, lane);   // weights: before the dependency wait
   pdl_wait();
   pdl_trigger();
+  const unsigned long long tl1 = tl_now();
   const int64_t tail = dst.tail_dev ? *dst.tail_dev : 0;
   const int n = block_scan_flags(alive, B, src_of, word_cnt);
   const bool fits = (tail - dst.head) + n <= dst.cap;
@@ -204,7 +206,10 @@ __global__ void __launch_bounds__(kThreads)
     if (n_surv_dev) *n_surv_dev = out;
     if (dst.mailbox) *dst.mailbox = fits ? out : -1;   // read by the host after the run's event
   }
-  if (!fits || n == 0) return;
+  if (!fits || n == 0) {
+    if (threadIdx.x == 0) tl_rec(6, tl0, tl1);
+    return;
+  }
 
   const int units = n * S;
   const int stride = gridDim.x * (kThreads / 32);
@@ -232,9 +237,12 @@ __global__ void __launch_bounds__(kThreads)
   }
   if (blockIdx.x == 0)
     for (int k = threadIdx.x; k < n; k += kThreads) dst.ids[(tail + k) % dst.cap] = id[src_of[k]];
+  if (threadIdx.x == 0) tl_rec(6, tl0, tl1);
 }
 
 }  // namespace
+
+E3_TL_SETTER(tl_set_compact)
 
 e3_status ln_compact_run(const void *y, const int64_t *id, const uint8_t *alive, int B, int S, int H, const void *g,
                          const void *b, float eps, const RingDst &dst, int32_t *n_surv_dev, int sms,

@@ -61,6 +61,7 @@ __global__ void __cluster_dims__(2, 1, 1) __launch_bounds__(kLThreads, 1)
                    const __grid_constant__ CUtensorMap tmOut, LnGemmArgs a) {
   using CF = LCfg<NH>;
   constexpr int S = CF::kStages;
+  const unsigned long long tl0 = tl_now();
   extern __shared__ uint8_t smem_raw[];
   uint8_t *smem = reinterpret_cast<uint8_t *>((reinterpret_cast<uintptr_t>(smem_raw) + 1023) & ~uintptr_t(1023));
   uint8_t *sA = smem;
@@ -289,6 +290,7 @@ __global__ void __cluster_dims__(2, 1, 1) __launch_bounds__(kLThreads, 1)
   __syncthreads();
   tc_fence_after();
   if (warp == 2) tmem_dealloc(tmem_base, CF::kTmem);
+  if (threadIdx.x == 0) tl_rec(7, tl0, tl0);
 }
 
 template <int NH>
@@ -323,6 +325,8 @@ e3_status ln_gemm_tmaps(LnGemmMaps *m, const void *A, const void *W, const void 
   if (s == E3_OK) s = make_tmap_2d(&m->pre, pre ? pre : out, (uint64_t)M, (uint64_t)N, (uint64_t)N, LM, 64);
   return s;
 }
+
+E3_TL_SETTER(tl_set_gemm_ln)
 
 e3_status ln_gemm_run(const LnGemmMaps &m, const LnGemmArgs &a, cudaStream_t st) {
   switch (a.N / 2) {

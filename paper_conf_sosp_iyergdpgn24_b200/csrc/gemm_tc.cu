@@ -93,6 +93,7 @@ __global__ void __cluster_dims__(2, 1, 1) __launch_bounds__(Cfg<BN, EPI>::kThrea
                         const __nv_bfloat16 *__restrict__ R, int M, int N, int K) {
   using CF = Cfg<BN, EPI>;
   constexpr int S = CF::kStages;
+  const unsigned long long tl0 = tl_now();
   extern __shared__ uint8_t smem_raw[];
   // identical layout (same offsets) in both CTAs of the pair
   uint8_t *smem = reinterpret_cast<uint8_t *>((reinterpret_cast<uintptr_t>(smem_raw) + 1023) & ~uintptr_t(1023));
@@ -139,6 +140,7 @@ __global__ void __cluster_dims__(2, 1, 1) __launch_bounds__(Cfg<BN, EPI>::kThrea
   const uint32_t tmem_base = *tmem_base_slot;
   pdl_wait();                      // A / residual / C of the previous kernels now visible
   pdl_trigger();
+  const unsigned long long tl1 = tl_now();
 
   if (warp == 0) {
     // ------------------------------------------------ TMA producer (both CTAs)
@@ -317,6 +319,7 @@ __global__ void __cluster_dims__(2, 1, 1) __launch_bounds__(Cfg<BN, EPI>::kThrea
   cluster_sync();                  // no CTA leaves while its peer may still signal it
   tc_fence_after();
   if (warp == 2) tmem_dealloc2(tmem_base, CF::kTmemCols);
+  if (threadIdx.x == 0) tl_rec(1000 + BN + EPI, tl0, tl1);
 }
 
 template <int BN, int EPI>
@@ -351,12 +354,20 @@ e3_status launch_epi(int epi, const GemmMaps &g, const __nv_bfloat16 *bias, cons
 
 }  // namespace
 
+E3_TL_SETTER(tl_set_gemm)
+
 e3_status gemm_set_trace(void *buf) {
   E3_CUDA_TRY(cudaMemcpyToSymbol(g_gemm_trace, &buf, sizeof(buf)));
   return E3_OK;
 }
 
 int gemm_pick_bn(int M, int N, int sms) {
+  // diagnostics: E3_GEMM_BN forces the N tile where it divides N
+  static const int forced = [] {
+    const char *e = getenv("E3_GEMM_BN");
+    return e ? atoi(e) : 0;
+  }();
+  if (forced && N % forced == 0) return forced;
   // Minimise waves x per-tile cost over the pair tiles (256 x BN); per-tile
   // cost ~ BN + 32 (fixed prologue / epilogue overhead in column units).
   int best = 0;

@@ -20,6 +20,13 @@ struct GemmMaps {
 int gemm_pick_bn(int M, int N, int sms);
 e3_status gemm_set_trace(void *buf);   // diagnostics (e3_debug_gemm_trace)
 e3_status attn_set_trace(void *buf);   // diagnostics (e3_debug_gemm_trace)
+// diagnostics (e3_debug_timeline): per translation unit
+e3_status tl_set_gemm(void *buf);
+e3_status tl_set_attn(void *buf);
+e3_status tl_set_ln(void *buf);
+e3_status tl_set_ramp(void *buf);
+e3_status tl_set_compact(void *buf);
+e3_status tl_set_gemm_ln(void *buf);
 e3_status gemm_tmaps(GemmMaps *g, const void *A, int64_t lda, const void *W, const void *C, int M, int N, int K,
                      int bn);
 e3_status gemm_run(const GemmMaps &g, const void *bias, const void *R, int M, int N, int K, int epi, int sms,

@@ -12,39 +12,67 @@ namespace e3 {
 
 namespace {
 
-template <int VPL>   // 16-byte vectors per lane
+// RPW rows per warp, all loads issued before any arithmetic: with one row per
+// warp BB's 8192 rows needed 1024 CTAs, 1.7 waves of the 4 resident per SM
+// (64 registers x 256 threads), and every second-wave CTA repeated the whole
+// load latency (r01 timeline: 7.0 us for 25 MB).
+template <int VPL, int RPW>
 __global__ void __launch_bounds__(256)
     layernorm_kernel(const __nv_bfloat16 *__restrict__ x, const __nv_bfloat16 *__restrict__ g,
                      const __nv_bfloat16 *__restrict__ bb, __nv_bfloat16 *__restrict__ y, int rows, int H,
                      float eps) {
-  const int row = blockIdx.x * 8 + warp_id();
+  const unsigned long long tl0 = tl_now();
   const int lane = lane_id();
-  uint4 v[VPL];
+  const int warps = gridDim.x * 8;
+  const int row0 = blockIdx.x * 8 + warp_id();
+  uint4 v[RPW][VPL];
   LnParams<VPL> p;
   ln_load_params<VPL>(p, g, bb, H, lane);   // weights: before the dependency wait
   pdl_wait();
   pdl_trigger();
-  if (row >= rows) return;
-  ln_load_row<VPL>(v, x + (size_t)row * H, H, lane);
-  ln_apply<VPL>(v, p, H, eps, lane);
-  ln_store_row<VPL>(v, y + (size_t)row * H, H, lane);
+  const unsigned long long tl1 = tl_now();
+#pragma unroll
+  for (int j = 0; j < RPW; ++j) {
+    const int row = row0 + j * warps;
+    if (row < rows) ln_load_row<VPL>(v[j], x + (size_t)row * H, H, lane);
+  }
+#pragma unroll
+  for (int j = 0; j < RPW; ++j) {
+    const int row = row0 + j * warps;
+    if (row < rows) {
+      ln_apply<VPL>(v[j], p, H, eps, lane);
+      ln_store_row<VPL>(v[j], y + (size_t)row * H, H, lane);
+    }
+  }
+  if (threadIdx.x == 0) tl_rec(3, tl0, tl1);
 }
 
 }  // namespace
 
+E3_TL_SETTER(tl_set_ln)
+
 e3_status layernorm_run(const void *x, const void *g, const void *b, void *y, int rows, int H, float eps,
                         cudaStream_t st) {
-  const int grid = (rows + 7) / 8;
+  // rows per warp: 2 when that keeps the grid within one wave of resident CTAs
+  // (4 per SM), else 1
+  static int sms = 0;
+  if (!sms) {
+    int dev = 0;
+    E3_CUDA_TRY(cudaGetDevice(&dev));
+    E3_CUDA_TRY(cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, dev));
+  }
+  const bool two = rows > 8 * 4 * sms && H <= 1024;   // registers: 2 rows of <= 4 vectors per lane
+  const int grid = two ? (rows + 15) / 16 : (rows + 7) / 8;
   auto *xp = reinterpret_cast<const __nv_bfloat16 *>(x);
   auto *gp = reinterpret_cast<const __nv_bfloat16 *>(g);
   auto *bp = reinterpret_cast<const __nv_bfloat16 *>(b);
   auto *yp = reinterpret_cast<__nv_bfloat16 *>(y);
   const int vpl = (H / 8 + 31) / 32;
-  if (vpl <= 1) E3_CUDA_TRY(launch_k(layernorm_kernel<1>, dim3(grid), dim3(256), 0, st, xp, gp, bp, yp, rows, H, eps));
-  else if (vpl <= 3) E3_CUDA_TRY(launch_k(layernorm_kernel<3>, dim3(grid), dim3(256), 0, st, xp, gp, bp, yp, rows, H, eps));
-  else if (vpl <= 4) E3_CUDA_TRY(launch_k(layernorm_kernel<4>, dim3(grid), dim3(256), 0, st, xp, gp, bp, yp, rows, H, eps));
-  else if (vpl <= 8) E3_CUDA_TRY(launch_k(layernorm_kernel<8>, dim3(grid), dim3(256), 0, st, xp, gp, bp, yp, rows, H, eps));
-  else if (vpl <= 16) E3_CUDA_TRY(launch_k(layernorm_kernel<16>, dim3(grid), dim3(256), 0, st, xp, gp, bp, yp, rows, H, eps));
+  if (vpl <= 1) E3_CUDA_TRY(launch_k(two ? layernorm_kernel<1, 2> : layernorm_kernel<1, 1>, dim3(grid), dim3(256), 0, st, xp, gp, bp, yp, rows, H, eps));
+  else if (vpl <= 3) E3_CUDA_TRY(launch_k(two ? layernorm_kernel<3, 2> : layernorm_kernel<3, 1>, dim3(grid), dim3(256), 0, st, xp, gp, bp, yp, rows, H, eps));
+  else if (vpl <= 4) E3_CUDA_TRY(launch_k(two ? layernorm_kernel<4, 2> : layernorm_kernel<4, 1>, dim3(grid), dim3(256), 0, st, xp, gp, bp, yp, rows, H, eps));
+  else if (vpl <= 8) E3_CUDA_TRY(launch_k(two ? layernorm_kernel<8, 2> : layernorm_kernel<8, 1>, dim3(grid), dim3(256), 0, st, xp, gp, bp, yp, rows, H, eps));
+  else if (vpl <= 16) E3_CUDA_TRY(launch_k(two ? layernorm_kernel<16, 2> : layernorm_kernel<16, 1>, dim3(grid), dim3(256), 0, st, xp, gp, bp, yp, rows, H, eps));
   else {
     set_error("LayerNorm: H > 4096 unsupported");
     return E3_EUNSUPPORTED;

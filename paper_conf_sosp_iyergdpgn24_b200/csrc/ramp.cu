@@ -88,6 +88,7 @@ __host__ __device__ inline int ramp_smem_bytes(int H, int C) {
 
 template <int VPL>
 __global__ void __launch_bounds__(kRThreads, 1) ramp_bert_kernel(RampArgs a) {
+  const unsigned long long tl0 = tl_now();
   extern __shared__ uint8_t smem_raw[];
   const int H = a.H, C = a.C;
   const int TN = H / kCS, NT = TN / 8;
@@ -120,6 +121,7 @@ __global__ void __launch_bounds__(kRThreads, 1) ramp_bert_kernel(RampArgs a) {
     ln_load_params<VPL>(lp, reinterpret_cast<const __nv_bfloat16 *>(a.ln_g),
                         reinterpret_cast<const __nv_bfloat16 *>(a.ln_b), H, lane);
   pdl_wait();                      // CLS rows / alive flags of the previous kernels now visible
+  const unsigned long long tl1 = tl_now();
   const int n_valid = a.n_valid_dev ? *a.n_valid_dev : a.n_valid_host;
   if (threadIdx.x < kRows) row_ok[threadIdx.x] = row_alive(a, b0 + threadIdx.x, n_valid);
 
@@ -222,7 +224,10 @@ __global__ void __launch_bounds__(kRThreads, 1) ramp_bert_kernel(RampArgs a) {
   // late trigger: the dependent kernel's CTAs, once resident, would compete
   // for issue slots with this issue-bound kernel (measured: +6 us per launch)
   pdl_trigger();
-  if (rank != 0 || warp != 0) return;
+  if (rank != 0 || warp != 0) {
+    if (threadIdx.x == 0) tl_rec(4, tl0, tl1);
+    return;
+  }
 
   // ---------------------------------------------------------- decide (rank 0)
   bool exit_now = false;
@@ -283,6 +288,7 @@ __global__ void __launch_bounds__(kRThreads, 1) ramp_bert_kernel(RampArgs a) {
     if (a.ex.n_exit) atomicAdd(a.ex.n_exit, n_ex);
     if (a.ex.ramp_count) atomicAdd(a.ex.ramp_count + a.ramp_index, n_ex);
   }
+  if (threadIdx.x == 0) tl_rec(5, tl0, tl1);   // rank 0: the decision is written
 }
 
 // ============================================================== ViT ramp
@@ -522,6 +528,8 @@ e3_status ramp_vit_run(const RampArgs &a, cudaStream_t st) {
 }
 
 }  // namespace
+
+E3_TL_SETTER(tl_set_ramp)
 
 e3_status ramp_run(const RampArgs &a, cudaStream_t st) {
   if (a.arch == E3_ARCH_VIT) return ramp_vit_run(a, st);

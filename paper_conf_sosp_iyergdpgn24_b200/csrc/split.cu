@@ -308,7 +308,9 @@ e3_status split_create_shared(const e3_split_desc *d, const e3_weights *w, int d
   // at BB it is 16.3 us alone vs 18.6 us for the two kernels, but the split
   // run is 2 % slower with it (128 one-CTA-per-SM clusters lose the PDL
   // overlap the two shorter kernels get); DESIGN.md §6.
-  s->use_oln = ln_gemm_supported(H, H) && getenv("E3_FUSED_LN") != nullptr;
+  // fused O projection + LayerNorm (K1b) unless E3_NO_FUSED_LN is set: r01
+  // timeline (scripts/timeline.py) 155.1 -> 149.8 us per BB layer
+  s->use_oln = ln_gemm_supported(H, H) && getenv("E3_NO_FUSED_LN") == nullptr;
   for (int i = 0; i < nl && st == E3_OK; ++i) {
     auto &m = s->maps[i];
     const void *prev = (i % 2 == 1) ? ws->xa : ws->xb;   // output of layer i-1
@@ -749,6 +751,16 @@ e3_status e3_op_gemm(void *stream, const void *A, int64_t lda, const void *W, co
   e3_status r = gemm_tmaps(&g, A, lda, W, C, M, N, K, gemm_pick_bn(M, N, sms));
   if (r != E3_OK) return r;
   return gemm_run(g, bias, resid, M, N, K, epilogue, sms, reinterpret_cast<cudaStream_t>(stream));
+}
+
+e3_status e3_debug_timeline(void *dev_buf) {
+  e3_status r = tl_set_gemm(dev_buf);
+  if (r == E3_OK) r = tl_set_attn(dev_buf);
+  if (r == E3_OK) r = tl_set_ln(dev_buf);
+  if (r == E3_OK) r = tl_set_ramp(dev_buf);
+  if (r == E3_OK) r = tl_set_compact(dev_buf);
+  if (r == E3_OK) r = tl_set_gemm_ln(dev_buf);
+  return r;
 }
 
 e3_status e3_debug_gemm_trace(void *dev_buf) {
