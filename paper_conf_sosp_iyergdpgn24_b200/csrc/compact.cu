@@ -182,8 +182,11 @@ __global__ void fill_kernel(int32_t *dst, int v) { *dst = v; }
 // alternate per push, chosen by the host.
 constexpr int kRowsInFlight = 4;
 
+// two CTAs per SM where the row fits in <= 3 vectors per lane: with one
+// (160 registers) only 8 warps x 4 rows were in flight per SM and the gather
+// was latency-bound (r01 timeline: ~7 us for 22 MB of L2-resident rows)
 template <int VPL, bool kLn>
-__global__ void __launch_bounds__(kThreads)
+__global__ void __launch_bounds__(kThreads, VPL <= 3 ? 2 : 1)
     ln_compact_kernel(const __nv_bfloat16 *__restrict__ y, const int64_t *__restrict__ id,
                       const uint8_t *__restrict__ alive, int B, int S, int H, const __nv_bfloat16 *__restrict__ g,
                       const __nv_bfloat16 *__restrict__ bb, float eps, RingDst dst, int32_t *n_surv_dev) {
@@ -198,6 +201,7 @@ __global__ void __launch_bounds__(kThreads)
   const unsigned long long tl1 = tl_now();
   const int64_t tail = dst.tail_dev ? *dst.tail_dev : 0;
   const int n = block_scan_flags(alive, B, src_of, word_cnt);
+  if (threadIdx.x == 0) tl_rec(60, tl1, tl1);   // scan done
   const bool fits = (tail - dst.head) + n <= dst.cap;
   if (blockIdx.x == 0 && threadIdx.x == 0) {
     const int out = fits ? n : 0;

@@ -12,19 +12,21 @@
 // B200 the ramp is instruction-issue-bound per SM, so fewer, fatter CTAs
 // (one cluster for the whole batch) were 1.6x slower:
 //   stage    the CTA's TN W_p rows by cp.async into padded smem (row pitch
-//            H + 8 bf16: conflict-free fragments) BEFORE the PDL wait;
-//   CLS      distributed LayerNorm: CTA rank r normalises CLS row r of the
-//            group alone (one warp; at a split's last layer the rows arrive
+//            H + 8 bf16: conflict-free fragments), its W_c / b_p slices as
+//            fp32, all BEFORE the PDL wait;
+//   CLS      every CTA normalises the group's 16 CLS rows itself (warp w:
+//            rows w and w + 8; at a split's last layer the rows arrive
 //            PRE-LayerNorm and the shared warp-per-row LN of ln_row.cuh makes
-//            them bit-identical to what the fused LN + compaction writes) and
-//            stores it into all 16 CTAs' shared memory through DSMEM;
-//   pooler   one warp per n8 tile of the CTA's outputs: mma.sync m16n8k16
-//            bf16 -> fp32 over K = H in two accumulator chains (a 16 x 48 x
-//            768 GEMM per CTA is far too small for a tcgen05 tile);
-//   partial  p = tanh(acc + b_p) stays in registers and is folded into
-//            partial logits sum_{o in tile} p[b,o] W_c[c,o], reduced over the
-//            quad with __shfl_xor_sync, then over the CTA's tiles in fixed
-//            order, and stored into rank 0's shared memory (DSMEM);
+//            them bit-identical to what the fused LN + compaction writes) --
+//            redundant across the cluster but one L2 round trip, where a
+//            DSMEM broadcast from one warp per CTA cost a serial store chain
+//            and a cluster barrier (r01 timeline: 3 us);
+//   pooler   mma.sync m16n8k16 bf16 -> fp32 with K split over the 8 warps
+//            (warp w: k16 steps w, w + 8, ...; NT = TN / 8 independent chains
+//            per warp instead of one 48-step chain on 6 of 8 warps), per-warp
+//            partials summed in warp order through smem, p = tanh(. + b_p);
+//   partial  partial logits sum_{o in CTA} p[b,o] W_c[c,o] by warp shuffles,
+//            stored into rank 0's shared memory (DSMEM);
 //   decide   after a cluster barrier rank 0 sums the 16 partials per (row,
 //            class) in rank order, then softmax / max-prob / entropy, argmax
 //            (lowest index on ties), threshold test, exit record by input id
@@ -80,27 +82,34 @@ __device__ __forceinline__ bool row_alive(const RampArgs &a, int b, int n_valid)
   return b < a.B && (a.init_alive ? (b < n_valid) : (a.alive[b] != 0));
 }
 
-// smem: W tile [TN][P] | CLS [16][P] | per-tile partials [NT][16][C] | cluster partials (rank 0) [kCS][16][C]
+// smem: W tile [TN][P] bf16 | CLS [16][P] bf16 | per-warp pooler partials
+// [8][16][TN] f32 | pooled p [16][TN] f32 | W_c slice [C][TN] f32 | b_p slice
+// [TN] f32 | cluster partials (rank 0) [kCS][16][C] f32
 __host__ __device__ inline int ramp_smem_bytes(int H, int C) {
-  const int TN = H / kCS, NT = TN / 8, P = H + 8;
-  return (TN + kRows) * P * 2 + NT * kRows * C * 4 + kCS * kRows * C * 4;
+  const int TN = H / kCS, P = H + 8;
+  return (TN + kRows) * P * 2 + (kRThreads / 32) * kRows * TN * 4 + kRows * TN * 4 + C * TN * 4 + TN * 4 +
+         kCS * kRows * C * 4;
 }
 
 template <int VPL>
 __global__ void __launch_bounds__(kRThreads, 1) ramp_bert_kernel(RampArgs a) {
   const unsigned long long tl0 = tl_now();
   extern __shared__ uint8_t smem_raw[];
+  constexpr int nw = kRThreads / 32;
+  constexpr int kMaxNT = 2 * VPL;                        // TN / 8 <= H / 128
   const int H = a.H, C = a.C;
   const int TN = H / kCS, NT = TN / 8;
   const int P = H + 8;                                   // padded pitch (bf16)
   __nv_bfloat16 *sW = reinterpret_cast<__nv_bfloat16 *>(smem_raw);   // [TN][P]
   __nv_bfloat16 *sC = sW + TN * P;                                    // [16][P]
-  float *sZ = reinterpret_cast<float *>(sC + kRows * P);              // [NT][16][C]
-  float *sQ = sZ + NT * kRows * C;                                    // [kCS][16][C] (rank 0)
+  float *sRed = reinterpret_cast<float *>(sC + kRows * P);            // [nw][16][TN]
+  float *sP = sRed + nw * kRows * TN;                                 // [16][TN]
+  float *sWc = sP + kRows * TN;                                       // [C][TN]
+  float *sBp = sWc + C * TN;                                          // [TN]
+  float *sQ = sBp + TN;                                               // [kCS][16][C] (rank 0)
   __shared__ bool row_ok[kRows];
 
   const int warp = warp_id(), lane = lane_id();
-  constexpr int nw = kRThreads / 32;
   const int gq = lane >> 2, tq = lane & 3;
   const uint32_t rank = cluster_ctarank();
   const int b0 = blockIdx.y * kRows;
@@ -110,14 +119,23 @@ __global__ void __launch_bounds__(kRThreads, 1) ramp_bert_kernel(RampArgs a) {
   const size_t row_stride = (size_t)a.S * H;
 
   cluster_arrive_relaxed();
-  // ---------------------------------------------------------- stage W_p
+  // ---------------------------------------------------------- weights: no dependency
   const uint4 *wp = reinterpret_cast<const uint4 *>(a.w.w_p);
-  for (int i = threadIdx.x; i < TN * nvec; i += kRThreads) {   // weights first: no dependency
+  for (int i = threadIdx.x; i < TN * nvec; i += kRThreads) {
     const int r = i / nvec, k = i - r * nvec;
     cp_async16(reinterpret_cast<uint4 *>(sW + r * P) + k, wp + (size_t)(o0 + r) * nvec + k);
   }
+  {
+    const __nv_bfloat16 *wc = reinterpret_cast<const __nv_bfloat16 *>(a.w.w_c);
+    const __nv_bfloat16 *bp = reinterpret_cast<const __nv_bfloat16 *>(a.w.b_p);
+    for (int i = threadIdx.x; i < C * TN; i += kRThreads) {
+      const int c = i / TN, o = i - c * TN;
+      sWc[i] = bf2f(wc[(size_t)c * H + o0 + o]);
+    }
+    for (int i = threadIdx.x; i < TN; i += kRThreads) sBp[i] = bf2f(bp[o0 + i]);
+  }
   LnParams<VPL> lp;
-  if (warp == 0 && a.ln_g)
+  if (a.ln_g)
     ln_load_params<VPL>(lp, reinterpret_cast<const __nv_bfloat16 *>(a.ln_g),
                         reinterpret_cast<const __nv_bfloat16 *>(a.ln_b), H, lane);
   pdl_wait();                      // CLS rows / alive flags of the previous kernels now visible
@@ -125,89 +143,92 @@ __global__ void __launch_bounds__(kRThreads, 1) ramp_bert_kernel(RampArgs a) {
   const int n_valid = a.n_valid_dev ? *a.n_valid_dev : a.n_valid_host;
   if (threadIdx.x < kRows) row_ok[threadIdx.x] = row_alive(a, b0 + threadIdx.x, n_valid);
 
-  // ---------------------------------------------------------- CLS row `rank`: LN here, broadcast by DSMEM
-  cluster_wait();                  // every CTA of the cluster is running
-  if (warp == 0) {
-    const int r = (int)rank;
-    const bool ok = row_alive(a, b0 + r, n_valid);
-    uint4 v[VPL];
-    if (ok) {
-      ln_load_row<VPL>(v, x + (size_t)(b0 + r) * row_stride, H, lane);
-      if (a.ln_g) ln_apply<VPL>(v, lp, H, a.eps, lane);
-    } else {
+  // ---------------------------------------------------------- CLS rows: every CTA normalises all 16
+  // itself (warp w: rows w and w + 8; at a split's last layer the rows arrive
+  // PRE-LayerNorm, and the shared warp-per-row LN of ln_row.cuh makes them
+  // bit-identical to what the fused LN + compaction writes)
+  {
+    uint4 v[2][VPL];
+    bool ok[2];
 #pragma unroll
-      for (int i = 0; i < VPL; ++i) v[i] = make_uint4(0, 0, 0, 0);
+    for (int j = 0; j < 2; ++j) {
+      const int r = warp + j * nw;
+      ok[j] = row_alive(a, b0 + r, n_valid);
+      if (ok[j]) ln_load_row<VPL>(v[j], x + (size_t)(b0 + r) * row_stride, H, lane);
     }
-    const uint32_t row_addr = smem_u32(sC + r * P);
-#pragma unroll 1
-    for (int q = 0; q < kCS; ++q) {
-      const uint32_t dst = mapa_shared(row_addr, (uint32_t)q);
 #pragma unroll
-      for (int i = 0; i < VPL; ++i) {
-        const int k = lane + 32 * i;
-        if (k < nvec) st_cluster_v4(dst + k * 16, v[i]);
+    for (int j = 0; j < 2; ++j) {
+      const int r = warp + j * nw;
+      if (ok[j]) {
+        if (a.ln_g) ln_apply<VPL>(v[j], lp, H, a.eps, lane);
+      } else {
+#pragma unroll
+        for (int i = 0; i < VPL; ++i) v[j][i] = make_uint4(0, 0, 0, 0);
       }
+      uint4 *dst = reinterpret_cast<uint4 *>(sC + r * P);
+#pragma unroll
+      for (int i = 0; i < VPL; ++i)
+        if (lane + 32 * i < nvec) dst[lane + 32 * i] = v[j][i];
     }
   }
   cp_async_wait_all();
-  cluster_sync();                  // all 16 CLS rows in every CTA; W tile landed
+  __syncthreads();                 // CLS rows and the W tile in smem
+  const unsigned long long tl2 = tl_now();
 
-  // ---------------------------------------------------------- pooler + partial logits
-  const __nv_bfloat16 *wc = reinterpret_cast<const __nv_bfloat16 *>(a.w.w_c);
-  const __nv_bfloat16 *bp = reinterpret_cast<const __nv_bfloat16 *>(a.w.b_p);
-  for (int t = warp; t < NT; t += nw) {
-    const int col = o0 + t * 8 + 2 * tq;                  // this lane's two pooler outputs
-    const float bb0 = bf2f(bp[col]), bb1 = bf2f(bp[col + 1]);
-    float wc0[kMaxC], wc1[kMaxC];
+  // ---------------------------------------------------------- pooler: K split over the warps
+  // warp w accumulates the k16 steps w, w + 8, ... for all NT n8 tiles (NT
+  // independent mma chains), partials summed across warps in warp order
+  {
+    float acc[kMaxNT][4];
 #pragma unroll
-    for (int c = 0; c < kMaxC; ++c) {
-      wc0[c] = (c < C) ? bf2f(wc[(size_t)c * H + col]) : 0.f;
-      wc1[c] = (c < C) ? bf2f(wc[(size_t)c * H + col + 1]) : 0.f;
-    }
-    float acc[4] = {0.f, 0.f, 0.f, 0.f}, acc2[4] = {0.f, 0.f, 0.f, 0.f};
+    for (int t = 0; t < kMaxNT; ++t) acc[t][0] = acc[t][1] = acc[t][2] = acc[t][3] = 0.f;
     const __nv_bfloat16 *a_lo = sC + gq * P + 2 * tq;
     const __nv_bfloat16 *a_hi = sC + (gq + 8) * P + 2 * tq;
-    const __nv_bfloat16 *bw = sW + (t * 8 + gq) * P + 2 * tq;
-#pragma unroll 2
-    for (int kk = 0; kk < H; kk += 32) {
+    const __nv_bfloat16 *bw = sW + gq * P + 2 * tq;
+    for (int k = 16 * warp; k < H; k += 16 * nw) {
+      uint32_t af[4];
+      af[0] = *reinterpret_cast<const uint32_t *>(a_lo + k);
+      af[1] = *reinterpret_cast<const uint32_t *>(a_hi + k);
+      af[2] = *reinterpret_cast<const uint32_t *>(a_lo + k + 8);
+      af[3] = *reinterpret_cast<const uint32_t *>(a_hi + k + 8);
 #pragma unroll
-      for (int h2 = 0; h2 < 2; ++h2) {
-        const int k = kk + 16 * h2;
-        uint32_t af[4];
-        af[0] = *reinterpret_cast<const uint32_t *>(a_lo + k);
-        af[1] = *reinterpret_cast<const uint32_t *>(a_hi + k);
-        af[2] = *reinterpret_cast<const uint32_t *>(a_lo + k + 8);
-        af[3] = *reinterpret_cast<const uint32_t *>(a_hi + k + 8);
-        const uint32_t bf0 = *reinterpret_cast<const uint32_t *>(bw + k);
-        const uint32_t bf1 = *reinterpret_cast<const uint32_t *>(bw + k + 8);
-        if (h2 == 0) mma_bf16_16816(acc, af, bf0, bf1);
-        else mma_bf16_16816(acc2, af, bf0, bf1);
+      for (int t = 0; t < kMaxNT; ++t) {
+        if (t < NT) {
+          const uint32_t bf0 = *reinterpret_cast<const uint32_t *>(bw + t * 8 * P + k);
+          const uint32_t bf1 = *reinterpret_cast<const uint32_t *>(bw + t * 8 * P + k + 8);
+          mma_bf16_16816(acc[t], af, bf0, bf1);
+        }
       }
     }
-    const float p00 = tanhf(acc[0] + acc2[0] + bb0), p01 = tanhf(acc[1] + acc2[1] + bb1);   // row gq
-    const float p10 = tanhf(acc[2] + acc2[2] + bb0), p11 = tanhf(acc[3] + acc2[3] + bb1);   // row gq + 8
+    float *red = sRed + warp * kRows * TN;
 #pragma unroll
-    for (int c = 0; c < kMaxC; ++c) {
-      if (c < C) {
-        float z0 = fmaf(p00, wc0[c], p01 * wc1[c]);
-        float z1 = fmaf(p10, wc0[c], p11 * wc1[c]);
-        z0 += __shfl_xor_sync(0xffffffffu, z0, 1);
-        z0 += __shfl_xor_sync(0xffffffffu, z0, 2);
-        z1 += __shfl_xor_sync(0xffffffffu, z1, 1);
-        z1 += __shfl_xor_sync(0xffffffffu, z1, 2);
-        if (tq == 0) {
-          sZ[(t * kRows + gq) * C + c] = z0;
-          sZ[(t * kRows + gq + 8) * C + c] = z1;
-        }
+    for (int t = 0; t < kMaxNT; ++t) {
+      if (t < NT) {
+        const int col = t * 8 + 2 * tq;
+        *reinterpret_cast<float2 *>(red + gq * TN + col) = make_float2(acc[t][0], acc[t][1]);
+        *reinterpret_cast<float2 *>(red + (gq + 8) * TN + col) = make_float2(acc[t][2], acc[t][3]);
       }
     }
   }
   __syncthreads();
-  // this CTA's partial logits (tiles summed in order) -> rank 0's slot [rank] (DSMEM)
-  for (int i = threadIdx.x; i < kRows * C; i += kRThreads) {
-    float s = sZ[i];
-    for (int t = 1; t < NT; ++t) s += sZ[t * kRows * C + i];
-    st_cluster_f32(mapa_shared(smem_u32(sQ + (int)rank * kRows * C + i), 0), s);
+  for (int i = threadIdx.x; i < kRows * TN; i += kRThreads) {
+    float s = sRed[i];
+#pragma unroll
+    for (int w = 1; w < nw; ++w) s += sRed[w * kRows * TN + i];
+    sP[i] = tanhf(s + sBp[i % TN]);              // p = tanh(W_p c + b_p)
+  }
+  __syncthreads();
+  // partial logits over this CTA's TN pooler outputs: warp w, rows w and w + 8
+  cluster_wait();                  // every CTA of the cluster is running (DSMEM below)
+  for (int j = 0; j < 2; ++j) {
+    const int r = warp + j * nw;
+    for (int c = 0; c < C; ++c) {
+      float z = 0.f;
+      for (int o = lane; o < TN; o += 32) z = fmaf(sP[r * TN + o], sWc[c * TN + o], z);
+#pragma unroll
+      for (int off = 16; off; off >>= 1) z += __shfl_xor_sync(0xffffffffu, z, off);
+      if (lane == 0) st_cluster_f32(mapa_shared(smem_u32(sQ + ((int)rank * kRows + r) * C + c), 0), z);
+    }
   }
   // rank 0 decides row r = threadIdx.x < 16: its id and the class biases are
   // fetched before the cluster barrier
@@ -220,10 +241,16 @@ __global__ void __launch_bounds__(kRThreads, 1) ramp_bert_kernel(RampArgs a) {
   for (int c = 0; c < kMaxC; ++c)
     bcv[c] = (decider && c < C) ? bf2f(reinterpret_cast<const __nv_bfloat16 *>(a.w.b_c)[c]) : 0.f;
   if (decider) row_id = a.id[b];
+  const unsigned long long tl3 = tl_now();
   cluster_sync();                  // every CTA's partials are in rank 0's smem
-  // late trigger: the dependent kernel's CTAs, once resident, would compete
-  // for issue slots with this issue-bound kernel (measured: +6 us per launch)
-  pdl_trigger();
+  const unsigned long long tlA = tl_now();
+  if (threadIdx.x == 0 && rank != 0) tl_rec(40, tl2, tl3);   // phases: CLS + W ready, partials stored, synced
+  unsigned long long tlB = 0;
+  // PDL trigger only once the decision is written (non-deciding CTAs trigger
+  // by exiting): dependent CTAs made resident earlier sit in
+  // griddepcontrol.wait on the deciding CTA's SM and slowed its few hundred
+  // instructions from <1 to ~3 us (r01 timeline); before the pooler they cost
+  // +6 us
   if (rank != 0 || warp != 0) {
     if (threadIdx.x == 0) tl_rec(4, tl0, tl1);
     return;
@@ -267,6 +294,7 @@ __global__ void __launch_bounds__(kRThreads, 1) ramp_bert_kernel(RampArgs a) {
       pass = metric < a.tau;
     }
     exit_now = pass || a.final_ramp;
+    tlB = tl_now();
     if (exit_now) {
       const int64_t id = row_id;
       if (id >= 0 && id < a.ex.capacity) {
@@ -288,7 +316,10 @@ __global__ void __launch_bounds__(kRThreads, 1) ramp_bert_kernel(RampArgs a) {
     if (a.ex.n_exit) atomicAdd(a.ex.n_exit, n_ex);
     if (a.ex.ramp_count) atomicAdd(a.ex.ramp_count + a.ramp_index, n_ex);
   }
+  __syncwarp();
+  pdl_trigger();
   if (threadIdx.x == 0) tl_rec(5, tl0, tl1);   // rank 0: the decision is written
+  if (threadIdx.x == 0) tl_rec(41, tlA, tlB);
 }
 
 // ============================================================== ViT ramp
