@@ -65,7 +65,9 @@ __device__ __forceinline__ void atrace(int j, int kind) {
   }
 }
 
-template <int SKV>
+// kMask: S < SKV, keys >= S are masked; without it (S == SKV, BB) the
+// softmax loops carry no per-element compare / select
+template <int SKV, bool kMask>
 __global__ void __launch_bounds__(kThreads, SKV == 128 ? 2 : 1)
     attn_tc_kernel(const __grid_constant__ CUtensorMap tq, const __grid_constant__ CUtensorMap tkv,
                    const __grid_constant__ CUtensorMap tctx, int S, int H, int heads, int n_items) {
@@ -182,7 +184,7 @@ __global__ void __launch_bounds__(kThreads, SKV == 128 ? 2 : 1)
         for (int jj = 0; jj < 32; ++jj) {
           const float v = __uint_as_float(r[jj]);
           if (kKeep) sv[ci * 32 + jj] = v;
-          if (c + jj < S) m4[jj & 3] = fmaxf(m4[jj & 3], v);
+          if (!kMask || c + jj < S) m4[jj & 3] = fmaxf(m4[jj & 3], v);
         }
         mx = fmaxf(mx, fmaxf(fmaxf(m4[0], m4[1]), fmaxf(m4[2], m4[3])));
       }
@@ -208,11 +210,29 @@ __global__ void __launch_bounds__(kThreads, SKV == 128 ? 2 : 1)
 #pragma unroll
           for (int jj = 0; jj < 32; ++jj) sv[jj] = __uint_as_float(r[jj]);
         }
+        // p = 2^(s log2e / 8 - m log2e / 8): packed fp32x2 FMAs and sums (the
+        // same roundings and summation order as the scalar form)
         float p[32];
 #pragma unroll
-        for (int jj = 0; jj < 32; ++jj) {
-          p[jj] = (c + jj < S) ? ex2_approx(fmaf(sv[(kKeep ? ci * 32 : 0) + jj], sl2, -mb)) : 0.f;
-          l4[jj & 3] += p[jj];
+        for (int jj = 0; jj < 32; jj += 4) {
+          const float *sp = sv + (kKeep ? ci * 32 : 0) + jj;
+          const float2 t0 = __ffma2_rn(make_float2(sp[0], sp[1]), make_float2(sl2, sl2), make_float2(-mb, -mb));
+          const float2 t1 = __ffma2_rn(make_float2(sp[2], sp[3]), make_float2(sl2, sl2), make_float2(-mb, -mb));
+          p[jj] = ex2_approx(t0.x);
+          p[jj + 1] = ex2_approx(t0.y);
+          p[jj + 2] = ex2_approx(t1.x);
+          p[jj + 3] = ex2_approx(t1.y);
+          if (kMask) {
+#pragma unroll
+            for (int e = 0; e < 4; ++e)
+              if (c + jj + e >= S) p[jj + e] = 0.f;
+          }
+          const float2 a0 = __fadd2_rn(make_float2(l4[0], l4[1]), make_float2(p[jj], p[jj + 1]));
+          const float2 a1 = __fadd2_rn(make_float2(l4[2], l4[3]), make_float2(p[jj + 2], p[jj + 3]));
+          l4[0] = a0.x;
+          l4[1] = a0.y;
+          l4[2] = a1.x;
+          l4[3] = a1.y;
         }
         // columns c..c+31 -> block c/64, 16-byte chunks (c%64)/8 .. +3, XOR-swizzled by row%8
         uint8_t *blk = prow + (c / 64) * (QT * 128);
@@ -286,12 +306,12 @@ __global__ void __launch_bounds__(kThreads, SKV == 128 ? 2 : 1)
   if (tid == 0) bulk_wait<0>();
   __syncthreads();
   if (warp == 0) tmem_dealloc(tbase, CF::kTmemCols);
-  if (tid == 0) tl_rec(2000 + SKV, tl0, tl1);
+  if (tid == 0) tl_rec(2000 + SKV + (kMask ? 500 : 0), tl0, tl1);
 }
 
-template <int SKV>
+template <int SKV, bool kMask>
 e3_status launch_attn(const AttnMaps &m, int B, int S, int H, int heads, cudaStream_t st) {
-  auto kern = attn_tc_kernel<SKV>;
+  auto kern = attn_tc_kernel<SKV, kMask>;
   static bool attr_done = false;
   static int sms = 0, per_sm = 0;
   if (!attr_done) {
@@ -345,11 +365,11 @@ e3_status attn_tmaps(AttnMaps *m, const void *qkv, const void *ctx, int B, int S
 
 e3_status attn_run(const AttnMaps &m, int B, int S, int H, int heads, cudaStream_t st) {
   switch (m.skv) {
-    case 128: return launch_attn<128>(m, B, S, H, heads, st);
-    case 160: return launch_attn<160>(m, B, S, H, heads, st);
-    case 192: return launch_attn<192>(m, B, S, H, heads, st);
-    case 224: return launch_attn<224>(m, B, S, H, heads, st);
-    case 256: return launch_attn<256>(m, B, S, H, heads, st);
+    case 128: return S == 128 ? launch_attn<128, false>(m, B, S, H, heads, st) : launch_attn<128, true>(m, B, S, H, heads, st);
+    case 160: return S == 160 ? launch_attn<160, false>(m, B, S, H, heads, st) : launch_attn<160, true>(m, B, S, H, heads, st);
+    case 192: return S == 192 ? launch_attn<192, false>(m, B, S, H, heads, st) : launch_attn<192, true>(m, B, S, H, heads, st);
+    case 224: return S == 224 ? launch_attn<224, false>(m, B, S, H, heads, st) : launch_attn<224, true>(m, B, S, H, heads, st);
+    case 256: return S == 256 ? launch_attn<256, false>(m, B, S, H, heads, st) : launch_attn<256, true>(m, B, S, H, heads, st);
   }
   set_error("attention: S > 256");
   return E3_EUNSUPPORTED;
