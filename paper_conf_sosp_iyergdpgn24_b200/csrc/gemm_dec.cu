@@ -81,6 +81,7 @@ __global__ void __launch_bounds__(kDThreads, 1)
   using CF = DCfg<T>;
   constexpr int S = CF::kStages;
   constexpr int P = T + 1;
+  const unsigned long long tl0 = tl_now();
   extern __shared__ uint8_t smem_raw[];
   uint8_t *smem = reinterpret_cast<uint8_t *>((reinterpret_cast<uintptr_t>(smem_raw) + 1023) & ~uintptr_t(1023));
   uint8_t *sW = smem;
@@ -196,6 +197,8 @@ __global__ void __launch_bounds__(kDThreads, 1)
     // ------------------------------------------------------- epilogue (warps 2-5)
     pdl_wait();
     pdl_trigger();
+    const unsigned long long tl1 = tl_now();
+    unsigned long long tlf = 0, tlm = 0;   // first / last accumulator ready
     const int q = warp & 3;
     const int r = q * 32 + lane;       // weight row of the tile == TMEM lane
     const int et = threadIdx.x - 64;   // 0..127
@@ -234,6 +237,8 @@ __global__ void __launch_bounds__(kDThreads, 1)
       i = seg_end;
       mbar_wait(&tfull[acc], acc_phase);
       tc_fence_after();
+      tlm = tl_now();
+      if (!tlf) tlf = tlm;
       const uint32_t taddr = tmem_base + ((uint32_t)(q * 32) << 16) + acc * T;
 #pragma unroll
       for (int c = 0; c < T / 32; ++c) {
@@ -271,6 +276,7 @@ __global__ void __launch_bounds__(kDThreads, 1)
         }
         epi_bar();
         if (!*s_last) continue;
+        const unsigned long long tlr0 = tl_now();
         __threadfence();
         // sum the contributors' partials in contributor order; contributor
         // j+1's loads are in flight while j is accumulated (one round trip
@@ -311,12 +317,64 @@ __global__ void __launch_bounds__(kDThreads, 1)
           }
         }
         epi_bar();
+        if (threadIdx.x == 64) tl_rec(8200 + EPI, tlr0, tlr0);   // reduction: start, end
       }
 
       // ---------------------------------------------------- final epilogue
       // global loads of a token batch are issued together before its stores
       // (a load -> store chain per token cost ~1 us x T per launch)
-      if (EPI == E3_DEC_STORE || EPI == E3_DEC_RESID) {
+      // STORE / RESID / SWIGLU: transposed through sE so that 16 (8) lanes
+      // write one token's 128 (64) features as 16-byte vectors, 256 (128)
+      // contiguous bytes; the residual is read the same way.  The per-thread
+      // scalar form (one 2-byte load + store per token and feature) took
+      // 4-14 us per tile (r01 dec_timeline: gate_up epilogue 14 us)
+      const bool vec = (a.ldo % 8 == 0) && (a.N % 8 == 0) && ((reinterpret_cast<uintptr_t>(a.Y) & 15) == 0) &&
+                       (EPI != E3_DEC_RESID || (reinterpret_cast<uintptr_t>(a.R) & 15) == 0);
+      if ((EPI == E3_DEC_STORE || EPI == E3_DEC_RESID) && vec) {
+        const int g = et & 15, n = tile * DM + 8 * g;
+        if (n < a.N) {
+          // every residual vector of this thread is loaded before the first
+          // store (Y may alias R as far as the compiler knows, so a load
+          // after a store would cost one round trip per token pass: ~5 us)
+          uint4 rres[T / 8];
+          if (EPI == E3_DEC_RESID) {
+#pragma unroll
+            for (int k = 0; k < T / 8; ++k)
+              rres[k] = __ldg(reinterpret_cast<const uint4 *>(a.R + (size_t)((et >> 4) + 8 * k) * a.ldo + n));
+          }
+#pragma unroll
+          for (int k = 0; k < T / 8; ++k) {
+            const int t = (et >> 4) + 8 * k;
+            float v[8];
+#pragma unroll
+            for (int j = 0; j < 8; ++j) v[j] = sE[(8 * g + j) * P + t];
+            if (EPI == E3_DEC_RESID) {
+              const uint4 rr = rres[k];
+              const uint32_t rw[4] = {rr.x, rr.y, rr.z, rr.w};
+#pragma unroll
+              for (int e = 0; e < 4; ++e) {
+                v[2 * e] += bf_lo(rw[e]);
+                v[2 * e + 1] += bf_hi(rw[e]);
+              }
+            }
+            *reinterpret_cast<uint4 *>(a.Y + (size_t)t * a.ldo + n) =
+                make_uint4(pack_bf16(v[0], v[1]), pack_bf16(v[2], v[3]), pack_bf16(v[4], v[5]), pack_bf16(v[6], v[7]));
+          }
+        }
+      } else if (EPI == E3_DEC_SWIGLU && vec) {
+        const int g = et & 7, f = tile * 64 + 8 * g;
+#pragma unroll 4
+        for (int t = et >> 3; t < T; t += 16) {
+          float o[8];
+#pragma unroll
+          for (int j = 0; j < 8; ++j) {
+            const float gv = sE[(8 * g + j) * P + t], up = sE[(64 + 8 * g + j) * P + t];
+            o[j] = gv / (1.0f + expf(-gv)) * up;
+          }
+          *reinterpret_cast<uint4 *>(a.Y + (size_t)t * a.ldo + f) =
+              make_uint4(pack_bf16(o[0], o[1]), pack_bf16(o[2], o[3]), pack_bf16(o[4], o[5]), pack_bf16(o[6], o[7]));
+        }
+      } else if (EPI == E3_DEC_STORE || EPI == E3_DEC_RESID) {
         const int n = tile * DM + r;
         if (n < a.N) {
 #pragma unroll 1
@@ -336,6 +394,64 @@ __global__ void __launch_bounds__(kDThreads, 1)
           for (int t = 0; t < T; ++t) {
             const float g = sE[r * P + t], up = sE[(r + 64) * P + t];
             a.Y[(size_t)t * a.ldo + f] = __float2bfloat16_rn(g / (1.0f + expf(-g)) * up);
+          }
+        }
+      } else if (EPI == E3_DEC_QKV_ROPE && vec) {
+        // tile = one head (head_dim 128): q heads, then k heads, then v heads.
+        // Thread = (token t, dims 8g..8g+7 and their RoPE partners 64+8g..):
+        // the (cos, sin) of the 8 pairs come as four 16-byte loads, both
+        // halves leave as 16-byte stores (the scalar form's table loads
+        // were a round trip per 16 tokens: ~6 us per tile, r01)
+        const int hq = tile;
+        const bool is_q = hq < a.nh, is_k = !is_q && hq < a.nh + a.kvh;
+        const int g = et & 7;
+        // all (cos, sin) vectors of this thread's tokens before the first
+        // store (the stores may alias the table as far as the compiler knows)
+        float4 rc[T / 16][4];
+        if (is_q || is_k) {
+#pragma unroll
+          for (int k = 0; k < T / 16; ++k) {
+            const float4 *cp = reinterpret_cast<const float4 *>(a.rope + (size_t)sPos[(et >> 3) + 16 * k] * 64 + 8 * g);
+#pragma unroll
+            for (int i = 0; i < 4; ++i) rc[k][i] = __ldg(cp + i);
+          }
+        }
+#pragma unroll
+        for (int k = 0; k < T / 16; ++k) {
+          const int t = (et >> 3) + 16 * k;
+          float lo[8], hi[8];
+#pragma unroll
+          for (int j = 0; j < 8; ++j) {
+            lo[j] = sE[(8 * g + j) * P + t];
+            hi[j] = sE[(64 + 8 * g + j) * P + t];
+          }
+          if (is_q || is_k) {
+            const float cs[16] = {rc[k][0].x, rc[k][0].y, rc[k][0].z, rc[k][0].w, rc[k][1].x, rc[k][1].y,
+                                  rc[k][1].z, rc[k][1].w, rc[k][2].x, rc[k][2].y, rc[k][2].z, rc[k][2].w,
+                                  rc[k][3].x, rc[k][3].y, rc[k][3].z, rc[k][3].w};
+#pragma unroll
+            for (int j = 0; j < 8; ++j) {
+              const float c = cs[2 * j], sn = cs[2 * j + 1];
+              const float l = fmaf(lo[j], c, -hi[j] * sn), h = fmaf(hi[j], c, lo[j] * sn);
+              lo[j] = l;
+              hi[j] = h;
+            }
+          }
+          const uint4 olo = make_uint4(pack_bf16(lo[0], lo[1]), pack_bf16(lo[2], lo[3]), pack_bf16(lo[4], lo[5]),
+                                       pack_bf16(lo[6], lo[7]));
+          const uint4 ohi = make_uint4(pack_bf16(hi[0], hi[1]), pack_bf16(hi[2], hi[3]), pack_bf16(hi[4], hi[5]),
+                                       pack_bf16(hi[6], hi[7]));
+          __nv_bfloat16 *dst = nullptr;
+          if (is_q) {
+            dst = a.Y + (size_t)t * a.ldo + hq * 128;
+          } else if (sSlot[t] >= 0) {
+            const int kh = is_k ? hq - a.nh : hq - a.nh - a.kvh;
+            __nv_bfloat16 *cache = is_k ? a.kc : a.vc;
+            dst = cache + (((size_t)sSlot[t] * a.kvh + kh) * a.max_ctx + sPos[t]) * 128;
+          }
+          if (dst) {
+            *reinterpret_cast<uint4 *>(dst + 8 * g) = olo;
+            *reinterpret_cast<uint4 *>(dst + 64 + 8 * g) = ohi;
           }
         }
       } else if (EPI == E3_DEC_QKV_ROPE) {
@@ -396,12 +512,22 @@ __global__ void __launch_bounds__(kDThreads, 1)
       }
       epi_bar();                        // sE is reused by the next unit
     }
+    if (threadIdx.x == 64) {
+      tl_rec(8100 + EPI, tl0, tl1);
+      tl_rec(8000 + EPI, tlf, tlm);
+    }
   }
   tc_fence_before();
   __syncthreads();
   tc_fence_after();
   if (warp == 2) tmem_dealloc(tmem_base, CF::kTmemCols);
 }
+
+}  // namespace
+
+E3_TL_SETTER(tl_set_dec)
+
+namespace {
 
 template <int T, int EPI>
 e3_status dec_launch(const DecMaps &m, const DecArgs &a, int grid, cudaStream_t st) {

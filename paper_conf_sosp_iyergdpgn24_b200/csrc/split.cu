@@ -760,6 +760,7 @@ e3_status e3_debug_timeline(void *dev_buf) {
   if (r == E3_OK) r = tl_set_ramp(dev_buf);
   if (r == E3_OK) r = tl_set_compact(dev_buf);
   if (r == E3_OK) r = tl_set_gemm_ln(dev_buf);
+  if (r == E3_OK) r = tl_set_dec(dev_buf);
   return r;
 }
 
