@@ -340,6 +340,7 @@ __global__ void __launch_bounds__(kRThreads, 1) ramp_bert_kernel(RampArgs a) {
 // threshold, writes the record and the alive flag, and publishes the decision;
 // each CTA then writes its slice of the logits of the exiting rows.
 constexpr int kVitRows = 16;
+constexpr int kVitKQ = 4;                              // CTA = kVitKQ x 2 CB threads = 8 per class
 
 __device__ __forceinline__ int ld_cluster_s32(uint32_t addr) {
   int v;
@@ -347,16 +348,22 @@ __device__ __forceinline__ int ld_cluster_s32(uint32_t addr) {
   return v;
 }
 
-template <int CB>
-__global__ void __launch_bounds__(2 * CB) ramp_vit_kernel(RampArgs a, int CS) {
+template <int CB, bool kLate>
+__global__ void __launch_bounds__(kVitKQ * 2 * CB) ramp_vit_kernel(RampArgs a, int CS) {
+  const unsigned long long tl0 = tl_now();
+  // 8 threads per class for the classifier; the first 2 CB threads then own
+  // 2 classes x 4 rows each for the softmax statistics and the logits
   constexpr int kThreads = 2 * CB, kWarps = kThreads / 32, kWarpsPerRg = CB / 64;
+  constexpr int kAll = kVitKQ * kThreads, kAllWarps = kAll / 32;
+  constexpr int kVitCls = CB;
   extern __shared__ float sN[];                       // [16][H + 4] normalised CLS rows (fp32)
   __shared__ SoftStat sRed[kWarps][4];
   __shared__ SoftStat sQ[16][kVitRows];               // rank 0: [rank][row]
   __shared__ int sDec[kVitRows];                      // rank 0: 1 = row exits here
   __shared__ bool row_ok[kVitRows];
   const int H = a.H, P = H + 4, C = a.C;
-  const int t = threadIdx.x, warp = t >> 5, lane = t & 31;
+  const int tAll = threadIdx.x;
+  const int t = tAll % kThreads, warp = t >> 5, lane = t & 31, wAll = tAll >> 5;
   const uint32_t rank = cluster_ctarank();
   const int b0 = blockIdx.y * kVitRows;
   const int j = t % (CB / 2), rg = t / (CB / 2);
@@ -367,16 +374,17 @@ __global__ void __launch_bounds__(2 * CB) ramp_vit_kernel(RampArgs a, int CS) {
   cluster_arrive_relaxed();
 
   pdl_wait();
-  pdl_trigger();
+  if (!kLate) pdl_trigger();
+  const unsigned long long tl1 = tl_now();
   const int n_valid = a.n_valid_dev ? *a.n_valid_dev : a.n_valid_host;
-  if (t < kVitRows) row_ok[t] = row_alive(a, b0 + t, n_valid);
+  if (tAll < kVitRows) row_ok[tAll] = row_alive(a, b0 + tAll, n_valid);
   __syncthreads();
 
   // ---- LayerNorm of the CLS rows (two passes, fp32), one warp per row
   const __nv_bfloat16 *x = reinterpret_cast<const __nv_bfloat16 *>(a.x);
   const __nv_bfloat16 *lg = reinterpret_cast<const __nv_bfloat16 *>(a.w.ln_g);
   const __nv_bfloat16 *lb = reinterpret_cast<const __nv_bfloat16 *>(a.w.ln_b);
-  for (int r = warp; r < kVitRows; r += kWarps) {
+  for (int r = wAll; r < kVitRows; r += kAllWarps) {
     float *row = sN + r * P;
     if (!row_ok[r]) {
       for (int k = lane; k < H; k += 32) row[k] = 0.f;
@@ -404,39 +412,61 @@ __global__ void __launch_bounds__(2 * CB) ramp_vit_kernel(RampArgs a, int CS) {
   }
   __syncthreads();
 
-  // ---- classifier: 4 rows x 2 classes per thread, fp32 FMA over K = H
-  float acc[4][2] = {};
+  const unsigned long long tlLn = tl_now();
+  // ---- classifier, fp32 FMA over K = H: thread (class cl, k lane q) sums
+  // k = 8q + 64i for all 16 rows, so the 8 lanes of a class read 128
+  // contiguous bytes of its W_c row per step (one class row per lane was a
+  // 32-line scattered load per instruction: ~60 us per launch at VT, r01);
+  // partial sums are reduced over q by shuffles in a fixed order
+  __shared__ float sZ[kVitRows][kVitCls];
   {
-    const uint4 *w0 = reinterpret_cast<const uint4 *>(W + (size_t)(c0 < C ? c0 : 0) * H);
-    const uint4 *w1 = reinterpret_cast<const uint4 *>(W + (size_t)(c1 < C ? c1 : 0) * H);
-    const bool v0 = c0 < C, v1 = c1 < C;
-    const float *rows = sN + rg * 4 * P;
+    const int cl = tAll >> 3, q = tAll & 7;
+    const int cg = (int)rank * CB + cl;
+    float acc[kVitRows];
+#pragma unroll
+    for (int r = 0; r < kVitRows; ++r) acc[r] = 0.f;
+    if (cg < C) {
+      const uint4 *wr = reinterpret_cast<const uint4 *>(W + (size_t)cg * H);
 #pragma unroll 2
-    for (int k = 0; k < H; k += 8) {
-      const uint4 wa = v0 ? __ldg(w0 + k / 8) : make_uint4(0, 0, 0, 0);
-      const uint4 wb = v1 ? __ldg(w1 + k / 8) : make_uint4(0, 0, 0, 0);
-      const float fa[8] = {bf_lo(wa.x), bf_hi(wa.x), bf_lo(wa.y), bf_hi(wa.y),
-                           bf_lo(wa.z), bf_hi(wa.z), bf_lo(wa.w), bf_hi(wa.w)};
-      const float fb[8] = {bf_lo(wb.x), bf_hi(wb.x), bf_lo(wb.y), bf_hi(wb.y),
-                           bf_lo(wb.z), bf_hi(wb.z), bf_lo(wb.w), bf_hi(wb.w)};
+      for (int k = 8 * q; k < H; k += 64) {
+        const uint4 w = __ldg(wr + k / 8);
+        const float wf[8] = {bf_lo(w.x), bf_hi(w.x), bf_lo(w.y), bf_hi(w.y),
+                             bf_lo(w.z), bf_hi(w.z), bf_lo(w.w), bf_hi(w.w)};
 #pragma unroll
-      for (int rr = 0; rr < 4; ++rr) {
-        const float4 n0 = *reinterpret_cast<const float4 *>(rows + rr * P + k);
-        const float4 n1 = *reinterpret_cast<const float4 *>(rows + rr * P + k + 4);
-        const float nv[8] = {n0.x, n0.y, n0.z, n0.w, n1.x, n1.y, n1.z, n1.w};
-#pragma unroll
-        for (int e = 0; e < 8; ++e) {
-          acc[rr][0] = fmaf(nv[e], fa[e], acc[rr][0]);
-          acc[rr][1] = fmaf(nv[e], fb[e], acc[rr][1]);
+        for (int r = 0; r < kVitRows; ++r) {
+          const float4 n0 = *reinterpret_cast<const float4 *>(sN + r * P + k);
+          const float4 n1 = *reinterpret_cast<const float4 *>(sN + r * P + k + 4);
+          float v = acc[r];
+          v = fmaf(n0.x, wf[0], v);
+          v = fmaf(n0.y, wf[1], v);
+          v = fmaf(n0.z, wf[2], v);
+          v = fmaf(n0.w, wf[3], v);
+          v = fmaf(n1.x, wf[4], v);
+          v = fmaf(n1.y, wf[5], v);
+          v = fmaf(n1.z, wf[6], v);
+          v = fmaf(n1.w, wf[7], v);
+          acc[r] = v;
         }
       }
     }
+#pragma unroll
+    for (int r = 0; r < kVitRows; ++r) {
+      float v = acc[r];
+      v += __shfl_xor_sync(0xffffffffu, v, 1);
+      v += __shfl_xor_sync(0xffffffffu, v, 2);
+      v += __shfl_xor_sync(0xffffffffu, v, 4);
+      if (q == 0) sZ[r][cl] = v;
+    }
   }
+  __syncthreads();
+  const unsigned long long tlCls = tl_now();
+  // threads t < 2 CB continue with 2 classes x 4 rows each
+  const bool g0 = tAll < kThreads;
   float z[4][2];
 #pragma unroll
   for (int rr = 0; rr < 4; ++rr) {
-    z[rr][0] = acc[rr][0] + bias0;
-    z[rr][1] = acc[rr][1] + bias1;
+    z[rr][0] = (g0 ? sZ[rg * 4 + rr][2 * j] : 0.f) + bias0;
+    z[rr][1] = (g0 ? sZ[rg * 4 + rr][2 * j + 1] : 0.f) + bias1;
   }
 
   // ---- per-row softmax statistics of this CTA's classes
@@ -447,11 +477,11 @@ __global__ void __launch_bounds__(2 * CB) ramp_vit_kernel(RampArgs a, int CS) {
     if (c1 < C) st = soft_merge(st, SoftStat{z[rr][1], 1.f, 0.f, c1});
 #pragma unroll
     for (int o = 16; o; o >>= 1) st = soft_merge(st, soft_shfl_xor(st, o));
-    if (lane == 0) sRed[warp][rr] = st;
+    if (lane == 0 && g0) sRed[warp][rr] = st;
   }
   __syncthreads();
   cluster_wait();                            // every CTA of the cluster is running
-  if (t < kVitRows) {                        // row t: merge this CTA's warps, send to rank 0
+  if (g0 && t < kVitRows) {                  // row t: merge this CTA's warps, send to rank 0
     const int g = t / 4, rr = t % 4;
     SoftStat st = sRed[g * kWarpsPerRg][rr];
     for (int w = 1; w < kWarpsPerRg; ++w) st = soft_merge(st, sRed[g * kWarpsPerRg + w][rr]);
@@ -464,7 +494,7 @@ __global__ void __launch_bounds__(2 * CB) ramp_vit_kernel(RampArgs a, int CS) {
   cluster_sync();
 
   // ---- rank 0 decides (rows t < 16 of warp 0)
-  if (rank == 0 && warp == 0) {
+  if (rank == 0 && warp == 0 && g0) {
     const int r = lane, b = b0 + r;
     bool exit_now = false;
     if (r < kVitRows && b < a.B) {
@@ -501,7 +531,7 @@ __global__ void __launch_bounds__(2 * CB) ramp_vit_kernel(RampArgs a, int CS) {
   }
   cluster_sync();
   // ---- logits of the exiting rows: each CTA writes its class slice
-  if (a.ex.logits) {
+  if (a.ex.logits && g0) {
 #pragma unroll
     for (int rr = 0; rr < 4; ++rr) {
       const int r = rg * 4 + rr, b = b0 + r;
@@ -514,11 +544,269 @@ __global__ void __launch_bounds__(2 * CB) ramp_vit_kernel(RampArgs a, int CS) {
     }
   }
   cluster_sync();                            // rank 0's smem stays valid until every CTA has read it
+  if (kLate) pdl_trigger();
+  if (tAll == 0) tl_rec(9, tl0, tl1);
+  if (tAll == 0) tl_rec(91, tlLn, tlCls);   // phases: CLS LN done, classifier done, end
 }
 
+
+// ViT ramp on the tensor cores (C <= 1024, H % 64 == 0, H <= 1024): the
+// classifier z = W_c n over a cluster's 16 rows is a dense [16 x H] x [H x 64]
+// contraction per CTA.  The fp32 normalised rows n are split exactly into
+// three bf16 terms n = hi + mid + lo (|n - (hi + mid + lo)| <= 2^-24 |n|), so
+// the three mma.sync m16n8k16 products with the bf16 W_c accumulate in fp32
+// what the fp32 FMA loop computed (products of 8-bit mantissas are exact in
+// fp32; only the summation order differs).  Warp w owns classes [8w, 8w + 8)
+// of the CTA's 64; W_c's slice is staged by cp.async before the PDL wait.
+// The old FMA kernel (kept for C > 1024) was shared-memory-bound re-reading
+// the rows per class group: 100 us per VT launch (r01 timeline).
+constexpr int kVtcThreads = 256;
+
+__host__ __device__ inline int ramp_vit_tc_smem(int H) {
+  const int P = H + 8;
+  return 64 * P * 2 + 3 * kVitRows * P * 2;
+}
+
+template <bool kLate>
+__global__ void __launch_bounds__(kVtcThreads, 1) ramp_vit_tc_kernel(RampArgs a, int CS) {
+  constexpr int CB = 64, kThreads = 2 * CB, kWarps = kThreads / 32, kWarpsPerRg = CB / 64;
+  const unsigned long long tl0 = tl_now();
+  extern __shared__ uint8_t smem_raw[];
+  const int H = a.H, C = a.C, P = H + 8;
+  __nv_bfloat16 *sW = reinterpret_cast<__nv_bfloat16 *>(smem_raw);   // [64][P]
+  __nv_bfloat16 *sA = sW + 64 * P;                                    // [3][16][P]: hi, mid, lo
+  __shared__ float sZ[kVitRows][CB];
+  __shared__ SoftStat sRed[kWarps][4];
+  __shared__ SoftStat sQ[16][kVitRows];               // rank 0: [rank][row]
+  __shared__ int sDec[kVitRows];                      // rank 0: 1 = row exits here
+  __shared__ bool row_ok[kVitRows];
+  const int tAll = threadIdx.x, wAll = tAll >> 5;
+  const int t = tAll % kThreads, warp = t >> 5, lane = t & 31;
+  const int gq = lane >> 2, tq = lane & 3;
+  const uint32_t rank = cluster_ctarank();
+  const int b0 = blockIdx.y * kVitRows;
+  const int j = t % (CB / 2), rg = t / (CB / 2);
+  const int c0 = (int)rank * CB + 2 * j, c1 = c0 + 1;
+  const __nv_bfloat16 *W = reinterpret_cast<const __nv_bfloat16 *>(a.w.w_c);
+  const __nv_bfloat16 *bc = reinterpret_cast<const __nv_bfloat16 *>(a.w.b_c);
+  const float bias0 = c0 < C ? bf2f(bc[c0]) : 0.f, bias1 = c1 < C ? bf2f(bc[c1]) : 0.f;
+  const int nvec = H / 8;
+  cluster_arrive_relaxed();
+  // W_c rows [rank*64, +64) -> smem (zero rows past C): no dependency
+  for (int i = tAll; i < 64 * nvec; i += kVtcThreads) {
+    const int r = i / nvec, k = i - r * nvec;
+    const int c = (int)rank * CB + r;
+    uint4 *dst = reinterpret_cast<uint4 *>(sW + r * P) + k;
+    if (c < C) cp_async16(dst, reinterpret_cast<const uint4 *>(W + (size_t)c * H) + k);
+    else *dst = make_uint4(0, 0, 0, 0);
+  }
+  pdl_wait();
+  if (!kLate) pdl_trigger();
+  const unsigned long long tl1 = tl_now();
+  const int n_valid = a.n_valid_dev ? *a.n_valid_dev : a.n_valid_host;
+  if (tAll < kVitRows) row_ok[tAll] = row_alive(a, b0 + tAll, n_valid);
+
+  // ---- LayerNorm of the CLS rows (fp32, two passes), warp w: rows w, w + 8;
+  // lane l owns the 16-byte vectors l, l + 32, ... of the row
+  {
+    const __nv_bfloat16 *x = reinterpret_cast<const __nv_bfloat16 *>(a.x);
+    const uint4 *lg = reinterpret_cast<const uint4 *>(a.w.ln_g);
+    const uint4 *lb = reinterpret_cast<const uint4 *>(a.w.ln_b);
+    constexpr int VM = 4;                              // H <= 1024
+    for (int r = wAll; r < kVitRows; r += kVtcThreads / 32) {
+      const bool ok = row_alive(a, b0 + r, n_valid);
+      float v[VM][8];
+      uint4 gv[VM], bv[VM];
+      const uint4 *xr = reinterpret_cast<const uint4 *>(x + (size_t)(b0 + r) * a.S * H);
+#pragma unroll
+      for (int i = 0; i < VM; ++i) {
+        const int k = lane + 32 * i;
+        const uint4 u = (ok && k < nvec) ? xr[k] : make_uint4(0, 0, 0, 0);
+        gv[i] = k < nvec ? __ldg(lg + k) : make_uint4(0, 0, 0, 0);
+        bv[i] = k < nvec ? __ldg(lb + k) : make_uint4(0, 0, 0, 0);
+        const uint32_t w[4] = {u.x, u.y, u.z, u.w};
+#pragma unroll
+        for (int e = 0; e < 4; ++e) {
+          v[i][2 * e] = bf_lo(w[e]);
+          v[i][2 * e + 1] = bf_hi(w[e]);
+        }
+      }
+      float sum = 0.f;
+#pragma unroll
+      for (int i = 0; i < VM; ++i)
+#pragma unroll
+        for (int e = 0; e < 8; ++e) sum += v[i][e];
+#pragma unroll
+      for (int o = 16; o; o >>= 1) sum += __shfl_xor_sync(0xffffffffu, sum, o);
+      const float mean = sum / (float)H;
+      float qs = 0.f;
+#pragma unroll
+      for (int i = 0; i < VM; ++i)
+        if (lane + 32 * i < nvec)
+#pragma unroll
+          for (int e = 0; e < 8; ++e) {
+            const float d = v[i][e] - mean;
+            qs += d * d;
+          }
+#pragma unroll
+      for (int o = 16; o; o >>= 1) qs += __shfl_xor_sync(0xffffffffu, qs, o);
+      const float rstd = 1.0f / sqrtf(qs / (float)H + a.eps);
+#pragma unroll
+      for (int i = 0; i < VM; ++i) {
+        const int k = lane + 32 * i;
+        if (k >= nvec) continue;
+        const uint32_t gw[4] = {gv[i].x, gv[i].y, gv[i].z, gv[i].w};
+        const uint32_t bw[4] = {bv[i].x, bv[i].y, bv[i].z, bv[i].w};
+        uint32_t hi[4], mi[4], lo[4];
+#pragma unroll
+        for (int e = 0; e < 4; ++e) {
+          float y[2];
+          y[0] = ok ? (v[i][2 * e] - mean) * rstd * bf_lo(gw[e]) + bf_lo(bw[e]) : 0.f;
+          y[1] = ok ? (v[i][2 * e + 1] - mean) * rstd * bf_hi(gw[e]) + bf_hi(bw[e]) : 0.f;
+          float h2[2], m2[2], l2[2];
+#pragma unroll
+          for (int u = 0; u < 2; ++u) {   // exact three-term bf16 split
+            h2[u] = __bfloat162float(__float2bfloat16_rn(y[u]));
+            const float r1 = y[u] - h2[u];
+            m2[u] = __bfloat162float(__float2bfloat16_rn(r1));
+            l2[u] = r1 - m2[u];
+          }
+          hi[e] = pack_bf16(h2[0], h2[1]);
+          mi[e] = pack_bf16(m2[0], m2[1]);
+          lo[e] = pack_bf16(l2[0], l2[1]);
+        }
+        reinterpret_cast<uint4 *>(sA + (0 * kVitRows + r) * P)[k] = make_uint4(hi[0], hi[1], hi[2], hi[3]);
+        reinterpret_cast<uint4 *>(sA + (1 * kVitRows + r) * P)[k] = make_uint4(mi[0], mi[1], mi[2], mi[3]);
+        reinterpret_cast<uint4 *>(sA + (2 * kVitRows + r) * P)[k] = make_uint4(lo[0], lo[1], lo[2], lo[3]);
+      }
+    }
+  }
+  cp_async_wait_all();
+  __syncthreads();
+  const unsigned long long tlLn = tl_now();
+
+  // ---- classifier: warp w, classes 8w .. 8w + 7, three split products
+  {
+    float acc[4] = {0.f, 0.f, 0.f, 0.f};
+    const __nv_bfloat16 *bw = sW + (8 * wAll + gq) * P + 2 * tq;
+#pragma unroll 1
+    for (int sp = 0; sp < 3; ++sp) {
+      const __nv_bfloat16 *a_lo = sA + (sp * kVitRows + gq) * P + 2 * tq;
+      const __nv_bfloat16 *a_hi = sA + (sp * kVitRows + gq + 8) * P + 2 * tq;
+#pragma unroll 4
+      for (int k = 0; k < H; k += 16) {
+        uint32_t af[4];
+        af[0] = *reinterpret_cast<const uint32_t *>(a_lo + k);
+        af[1] = *reinterpret_cast<const uint32_t *>(a_hi + k);
+        af[2] = *reinterpret_cast<const uint32_t *>(a_lo + k + 8);
+        af[3] = *reinterpret_cast<const uint32_t *>(a_hi + k + 8);
+        const uint32_t bf0 = *reinterpret_cast<const uint32_t *>(bw + k);
+        const uint32_t bf1 = *reinterpret_cast<const uint32_t *>(bw + k + 8);
+        mma_bf16_16816(acc, af, bf0, bf1);
+      }
+    }
+    const int col = 8 * wAll + 2 * tq;
+    sZ[gq][col] = acc[0];
+    sZ[gq][col + 1] = acc[1];
+    sZ[gq + 8][col] = acc[2];
+    sZ[gq + 8][col + 1] = acc[3];
+  }
+  __syncthreads();
+  const unsigned long long tlCls = tl_now();
+  // threads t < 2 CB continue with 2 classes x 4 rows each
+  const bool g0 = tAll < kThreads;
+  float z[4][2];
+#pragma unroll
+  for (int rr = 0; rr < 4; ++rr) {
+    z[rr][0] = (g0 ? sZ[rg * 4 + rr][2 * j] : 0.f) + bias0;
+    z[rr][1] = (g0 ? sZ[rg * 4 + rr][2 * j + 1] : 0.f) + bias1;
+  }
+
+  // ---- per-row softmax statistics of this CTA's classes
+#pragma unroll
+  for (int rr = 0; rr < 4; ++rr) {
+    SoftStat st{-INFINITY, 0.f, 0.f, -1};
+    if (c0 < C) st = SoftStat{z[rr][0], 1.f, 0.f, c0};
+    if (c1 < C) st = soft_merge(st, SoftStat{z[rr][1], 1.f, 0.f, c1});
+#pragma unroll
+    for (int o = 16; o; o >>= 1) st = soft_merge(st, soft_shfl_xor(st, o));
+    if (lane == 0 && g0) sRed[warp][rr] = st;
+  }
+  __syncthreads();
+  cluster_wait();                            // every CTA of the cluster is running
+  if (g0 && t < kVitRows) {                  // row t: merge this CTA's warps, send to rank 0
+    const int g = t / 4, rr = t % 4;
+    SoftStat st = sRed[g * kWarpsPerRg][rr];
+    for (int w = 1; w < kWarpsPerRg; ++w) st = soft_merge(st, sRed[g * kWarpsPerRg + w][rr]);
+    const uint32_t dst = mapa_shared(smem_u32(&sQ[rank][t]), 0);
+    st_cluster_f32(dst, st.m);
+    st_cluster_f32(dst + 4, st.s);
+    st_cluster_f32(dst + 8, st.u);
+    asm volatile("st.shared::cluster.s32 [%0], %1;" ::"r"(dst + 12), "r"(st.idx) : "memory");
+  }
+  cluster_sync();
+
+  // ---- rank 0 decides (rows t < 16 of warp 0)
+  if (rank == 0 && warp == 0 && g0) {
+    const int r = lane, b = b0 + r;
+    bool exit_now = false;
+    if (r < kVitRows && b < a.B) {
+      if (!row_ok[r]) {
+        if (a.init_alive) a.alive[b] = 0;
+      } else {
+        SoftStat st = sQ[0][r];
+        for (int q = 1; q < CS; ++q) st = soft_merge(st, sQ[q][r]);
+        float metric;
+        bool pass;
+        if (a.test == E3_TEST_MAXPROB) {
+          metric = 1.0f / st.s;
+          pass = metric > a.tau;
+        } else {
+          metric = logf(st.s) - st.u / st.s;
+          pass = metric < a.tau;
+        }
+        exit_now = pass || a.final_ramp;
+        const int64_t id = a.id[b];
+        if (exit_now && id >= 0 && id < a.ex.capacity) {
+          if (a.ex.exit_layer) a.ex.exit_layer[id] = a.layer;
+          if (a.ex.label) a.ex.label[id] = st.idx;
+          if (a.ex.conf) a.ex.conf[id] = metric;
+        }
+        a.alive[b] = exit_now ? 0 : 1;
+      }
+    }
+    if (r < kVitRows) sDec[r] = exit_now ? 1 : 0;
+    const int n_ex = __popc(__ballot_sync(0xffffffffu, exit_now));
+    if (lane == 0 && n_ex) {
+      if (a.ex.n_exit) atomicAdd(a.ex.n_exit, n_ex);
+      if (a.ex.ramp_count) atomicAdd(a.ex.ramp_count + a.ramp_index, n_ex);
+    }
+  }
+  cluster_sync();
+  // ---- logits of the exiting rows: each CTA writes its class slice
+  if (a.ex.logits && g0) {
+#pragma unroll
+    for (int rr = 0; rr < 4; ++rr) {
+      const int r = rg * 4 + rr, b = b0 + r;
+      if (b >= a.B) continue;
+      if (!ld_cluster_s32(mapa_shared(smem_u32(&sDec[r]), 0))) continue;
+      const int64_t id = a.id[b];
+      if (id < 0 || id >= a.ex.capacity) continue;
+      if (c0 < C) a.ex.logits[id * C + c0] = z[rr][0];
+      if (c1 < C) a.ex.logits[id * C + c1] = z[rr][1];
+    }
+  }
+  cluster_sync();                            // rank 0's smem stays valid until every CTA has read it
+  if (kLate) pdl_trigger();
+  if (tAll == 0) tl_rec(9, tl0, tl1);
+  if (tAll == 0) tl_rec(91, tlLn, tlCls);   // phases: CLS LN done, classifier done, end
+}
+
+
+
 e3_status ramp_vit_run(const RampArgs &a, cudaStream_t st) {
-  if (a.C < 1 || a.C > 16 * 128 || a.H % 8 || a.H > 3072 || !a.w.ln_g || !a.w.ln_b) {
-    set_error("ViT ramp: need 1 <= C <= 2048, H % 8 == 0, H <= 3072 and ramp LayerNorm weights");
+  if (a.C < 1 || a.C > 16 * 128 || a.H % 64 || a.H > 3072 || !a.w.ln_g || !a.w.ln_b) {
+    set_error("ViT ramp: need 1 <= C <= 2048, H % 64 == 0, H <= 3072 and ramp LayerNorm weights");
     return E3_EUNSUPPORTED;
   }
   const int CB = (a.C <= 16 * 64) ? 64 : 128;
@@ -526,7 +814,7 @@ e3_status ramp_vit_run(const RampArgs &a, cudaStream_t st) {
   const int smem = kVitRows * (a.H + 4) * 4;
   cudaLaunchConfig_t cfg = {};
   cfg.gridDim = dim3(CS, (a.B + kVitRows - 1) / kVitRows);
-  cfg.blockDim = dim3(2 * CB);
+  cfg.blockDim = dim3(kVitKQ * 2 * CB);
   cfg.dynamicSmemBytes = smem;
   cfg.stream = st;
   cudaLaunchAttribute attr[2];
@@ -538,20 +826,39 @@ e3_status ramp_vit_run(const RampArgs &a, cudaStream_t st) {
   attr[1].val.programmaticStreamSerializationAllowed = 1;
   cfg.attrs = attr;
   cfg.numAttrs = pdl_enabled() ? 2 : 1;
-#define E3_VRAMP(V)                                                                                        \
-  do {                                                                                                     \
-    static bool attr_done = false;                                                                         \
-    if (!attr_done) {                                                                                      \
-      E3_CUDA_TRY(cudaFuncSetAttribute(ramp_vit_kernel<V>, cudaFuncAttributeMaxDynamicSharedMemorySize,   \
-                                       kVitRows * (3072 + 4) * 4));                                        \
-      E3_CUDA_TRY(cudaFuncSetAttribute(ramp_vit_kernel<V>, cudaFuncAttributeNonPortableClusterSizeAllowed, \
-                                       1));                                                                \
-      attr_done = true;                                                                                    \
-    }                                                                                                      \
-    E3_CUDA_TRY(cudaLaunchKernelEx(&cfg, ramp_vit_kernel<V>, a, CS));                                      \
+#define E3_VRAMP(V, L)                                                                                      \
+  do {                                                                                                      \
+    static bool attr_done = false;                                                                          \
+    if (!attr_done) {                                                                                       \
+      E3_CUDA_TRY(cudaFuncSetAttribute(ramp_vit_kernel<V, L>, cudaFuncAttributeMaxDynamicSharedMemorySize, \
+                                       kVitRows * (3072 + 4) * 4));                                         \
+      E3_CUDA_TRY(cudaFuncSetAttribute(ramp_vit_kernel<V, L>, cudaFuncAttributeNonPortableClusterSizeAllowed, \
+                                       1));                                                                 \
+      attr_done = true;                                                                                     \
+    }                                                                                                       \
+    E3_CUDA_TRY(cudaLaunchKernelEx(&cfg, ramp_vit_kernel<V, L>, a, CS));                                    \
   } while (0)
-  if (CB == 64) E3_VRAMP(64);
-  else E3_VRAMP(128);
+  static const bool early = getenv("E3_VIT_EARLY_TRIGGER") != nullptr;   // diagnostics
+  if (a.C <= 16 * 64 && a.H <= 1024 && ramp_vit_tc_smem(a.H) <= 200 * 1024 && getenv("E3_VIT_RAMP_FMA") == nullptr) {
+    cfg.blockDim = dim3(kVtcThreads);
+    cfg.dynamicSmemBytes = ramp_vit_tc_smem(a.H);
+    static bool tc_attr = false;
+    if (!tc_attr) {
+      for (auto k : {ramp_vit_tc_kernel<true>, ramp_vit_tc_kernel<false>}) {
+        E3_CUDA_TRY(cudaFuncSetAttribute(k, cudaFuncAttributeMaxDynamicSharedMemorySize, 200 * 1024));
+        E3_CUDA_TRY(cudaFuncSetAttribute(k, cudaFuncAttributeNonPortableClusterSizeAllowed, 1));
+      }
+      tc_attr = true;
+    }
+    if (early) E3_CUDA_TRY(cudaLaunchKernelEx(&cfg, ramp_vit_tc_kernel<false>, a, CS));
+    else E3_CUDA_TRY(cudaLaunchKernelEx(&cfg, ramp_vit_tc_kernel<true>, a, CS));
+  } else if (CB == 64) {
+    if (early) E3_VRAMP(64, false);
+    else E3_VRAMP(64, true);
+  } else {
+    if (early) E3_VRAMP(128, false);
+    else E3_VRAMP(128, true);
+  }
 #undef E3_VRAMP
   E3_CUDA_TRY(cudaGetLastError());
   count_launch();

@@ -304,13 +304,12 @@ e3_status split_create_shared(const e3_split_desc *d, const e3_weights *w, int d
   const int nl = d->layer_end - d->layer_begin;
   s->maps.resize(nl);
   const bool vit = d->arch == E3_ARCH_VIT;
-  // Fused O projection + LayerNorm (gemm_ln.cu) is opt-in: measured on B200
-  // at BB it is 16.3 us alone vs 18.6 us for the two kernels, but the split
-  // run is 2 % slower with it (128 one-CTA-per-SM clusters lose the PDL
-  // overlap the two shorter kernels get); DESIGN.md §6.
-  // fused O projection + LayerNorm (K1b) unless E3_NO_FUSED_LN is set: r01
-  // timeline (scripts/timeline.py) 155.1 -> 149.8 us per BB layer
-  s->use_oln = ln_gemm_supported(H, H) && getenv("E3_NO_FUSED_LN") == nullptr;
+  // Fused O projection + LayerNorm (K1b, gemm_ln.cu) unless E3_NO_FUSED_LN
+  // is set: r01 timeline (scripts/timeline.py) 155.1 -> 149.8 us per BB
+  // layer; E3_FUSED_LN forces it.  Only where its one-CTA-per-(128 rows, H/2 columns) grid is a
+  // single wave: VT (788 CTAs) ran it at ~450 TF/s, 131 us vs ~85 us split
+  s->use_oln = ln_gemm_supported(H, H) && getenv("E3_NO_FUSED_LN") == nullptr &&
+               (getenv("E3_FUSED_LN") != nullptr || 2 * ((d->batch * d->seq_len + 127) / 128) <= s->sms);
   for (int i = 0; i < nl && st == E3_OK; ++i) {
     auto &m = s->maps[i];
     const void *prev = (i % 2 == 1) ? ws->xa : ws->xb;   // output of layer i-1
