@@ -317,6 +317,33 @@ __device__ __forceinline__ float gelu_fast(float x) {
 // gelu_fast on a pair of values with Blackwell's packed fp32x2 FMA/MUL
 // (FFMA2): same arithmetic, same rounding per element, ~35 % fewer issued
 // instructions -- the FFN1 epilogue is issue-bound.
+#ifndef E3_GELU_NR
+// GELU(x) = x Phi(x) on packed fp32x2 with Abramowitz-Stegun 7.1.26:
+// erfc(z) = t (a1 + a2 t + ... + a5 t^4) e^{-z^2}, t = 1 / (1 + p z), |error|
+// <= 1.5e-7 absolute (GELU relative error <= 5e-5 for |x| < 3; the output is
+// rounded to bf16, 2^-9).  Half the polynomial of the Numerical Recipes erfc
+// (E3_GELU_NR): the GELU epilogue of FFN1 is issue-bound next to the MMAs.
+__device__ __forceinline__ float2 gelu_fast2(float2 x) {
+  const float2 z = __fmul2_rn(make_float2(fabsf(x.x), fabsf(x.y)), make_float2(0.70710678118654752f, 0.70710678118654752f));
+  const float2 d = __ffma2_rn(make_float2(0.3275911f, 0.3275911f), z, make_float2(1.0f, 1.0f));
+  float2 t;
+  asm("rcp.approx.ftz.f32 %0, %1;" : "=f"(t.x) : "f"(d.x));
+  asm("rcp.approx.ftz.f32 %0, %1;" : "=f"(t.y) : "f"(d.y));
+  // 0.5 * a_i folded in: he = Phi(-|x|) = 0.5 erfc(|x| / sqrt 2)
+  float2 p = make_float2(0.5307027145f, 0.5307027145f);
+  p = __ffma2_rn(p, t, make_float2(-0.7265760135f, -0.7265760135f));
+  p = __ffma2_rn(p, t, make_float2(0.7107068705f, 0.7107068705f));
+  p = __ffma2_rn(p, t, make_float2(-0.142248368f, -0.142248368f));
+  p = __ffma2_rn(p, t, make_float2(0.127414796f, 0.127414796f));
+  const float2 arg = __fmul2_rn(x, __fmul2_rn(x, make_float2(-0.7213475204444817f, -0.7213475204444817f)));
+  float2 e;
+  asm("ex2.approx.ftz.f32 %0, %1;" : "=f"(e.x) : "f"(arg.x));
+  asm("ex2.approx.ftz.f32 %0, %1;" : "=f"(e.y) : "f"(arg.y));
+  const float2 he = __fmul2_rn(__fmul2_rn(t, p), e);
+  const float2 phi = make_float2(x.x >= 0.f ? 1.0f - he.x : he.x, x.y >= 0.f ? 1.0f - he.y : he.y);
+  return __fmul2_rn(x, phi);
+}
+#else
 __device__ __forceinline__ float2 gelu_fast2(float2 x) {
   const float2 z = __fmul2_rn(make_float2(fabsf(x.x), fabsf(x.y)), make_float2(0.70710678118654752f, 0.70710678118654752f));
   const float2 d = __ffma2_rn(make_float2(0.5f, 0.5f), z, make_float2(1.0f, 1.0f));
@@ -342,6 +369,7 @@ __device__ __forceinline__ float2 gelu_fast2(float2 x) {
   const float2 phi = make_float2(x.x >= 0.f ? 1.0f - he.x : he.x, x.y >= 0.f ? 1.0f - he.y : he.y);
   return __fmul2_rn(x, phi);
 }
+#endif
 
 __device__ __forceinline__ int warp_id() { return threadIdx.x >> 5; }
 __device__ __forceinline__ int lane_id() { return threadIdx.x & 31; }

@@ -138,32 +138,56 @@ __global__ void __cluster_dims__(2, 1, 1) __launch_bounds__(Cfg<BN, EPI>::kThrea
   cluster_sync();                  // peer barriers initialised, TMEM allocated in both CTAs
   tc_fence_after();
   const uint32_t tmem_base = *tmem_base_slot;
-  pdl_wait();                      // A / residual / C of the previous kernels now visible
-  pdl_trigger();
+  if (warp != 0) {
+    pdl_wait();                    // A / residual / C of the previous kernels now visible
+    pdl_trigger();
+  }
   const unsigned long long tl1 = tl_now();
 
   if (warp == 0) {
     // ------------------------------------------------ TMA producer (both CTAs)
     if (lane == 0) {
-      int stage = 0;
+      // the W boxes of the first S stages do not depend on the previous
+      // kernel: issued before griddepcontrol.wait, so the weight fetch
+      // overlaps the hand-off; the A boxes of those stages follow the wait
+      int npre = 0;
+      for (int t = pair; t < num_tiles && npre < S; t += num_pairs) {
+        const int bn = (t % num_n) * BN + (int)rank * (BN / 2);
+        for (int kb = 0; kb < num_kb && npre < S; ++kb, ++npre) {
+          const uint32_t fb = mapa_shared(smem_u32(&full[npre]), 0);
+          if (leader) mbar_expect_tx(&full[npre], 2 * CF::kStageBytes);
+#pragma unroll
+          for (int ks = 0; ks < KSUB; ++ks)
+            tma_load_2d_2sm(sB + npre * CF::kBBytes + ks * CF::kBSub, &tmB, fb, (kb * KSUB + ks) * BK, bn);
+        }
+      }
+      pdl_wait();
+      pdl_trigger();
+      int stage = 0, it = 0;
       uint32_t phase = 0;
       for (int t = pair; t < num_tiles; t += num_pairs) {
         const int m_blk = t / num_n, n_blk = t % num_n;
         const int am = m_blk * 2 * BM + (int)rank * BM;
         const int bn = n_blk * BN + (int)rank * (BN / 2);
-        for (int kb = 0; kb < num_kb; ++kb) {
-          mbar_wait(&empty[stage], phase ^ 1);
+        for (int kb = 0; kb < num_kb; ++kb, ++it) {
           const uint32_t fb = mapa_shared(smem_u32(&full[stage]), 0);
-          if (leader) mbar_expect_tx(&full[stage], 2 * CF::kStageBytes);
+          const bool pre = it < npre;
+          if (!pre) {
+            mbar_wait(&empty[stage], phase ^ 1);
+            if (leader) mbar_expect_tx(&full[stage], 2 * CF::kStageBytes);
+          }
 #pragma unroll
           for (int ks = 0; ks < KSUB; ++ks) {
             const int k0 = (kb * KSUB + ks) * BK;
             tma_load_2d_2sm(sA + stage * CF::kABytes + ks * CF::kASub, &tmA, fb, k0, am);
-            tma_load_2d_2sm(sB + stage * CF::kBBytes + ks * CF::kBSub, &tmB, fb, k0, bn);
+            if (!pre) tma_load_2d_2sm(sB + stage * CF::kBBytes + ks * CF::kBSub, &tmB, fb, k0, bn);
           }
           if (++stage == S) { stage = 0; phase ^= 1; }
         }
       }
+    } else {
+      pdl_wait();
+      pdl_trigger();
     }
   } else if (warp == 1) {
     // ------------------------------------------------ MMA issuer (leader, one thread)
