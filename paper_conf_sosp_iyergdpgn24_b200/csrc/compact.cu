@@ -25,7 +25,8 @@ constexpr int kMaxB = 4096;
 constexpr int kThreads = 256;
 constexpr int kUnroll = 4;
 
-__device__ __forceinline__ int block_scan_flags(const uint8_t *alive, int B, int16_t *src_of, int *word_cnt) {
+__device__ __forceinline__ int block_scan_flags(const uint8_t *alive, int B, int16_t *src_of, int *word_cnt,
+                                                int16_t *pos_of = nullptr) {
   // word_cnt: [kMaxB/32 + 1] smem
   const int warp = warp_id(), lane = lane_id();
   const int nwords = (B + 31) / 32;
@@ -49,7 +50,9 @@ __device__ __forceinline__ int block_scan_flags(const uint8_t *alive, int B, int
     const int i = w * 32 + lane;
     const bool f = i < B && alive[i] != 0;
     const unsigned bal = __ballot_sync(0xffffffffu, f);
-    if (f) src_of[word_cnt[w] + __popc(bal & ((1u << lane) - 1u))] = (int16_t)i;
+    const int pos = word_cnt[w] + __popc(bal & ((1u << lane) - 1u));
+    if (f) src_of[pos] = (int16_t)i;
+    if (pos_of && i < B) pos_of[i] = f ? (int16_t)pos : (int16_t)-1;
   }
   __syncthreads();
   return word_cnt[nwords];
@@ -191,6 +194,7 @@ __global__ void __launch_bounds__(kThreads, VPL <= 3 ? 2 : 1)
                       const uint8_t *__restrict__ alive, int B, int S, int H, const __nv_bfloat16 *__restrict__ g,
                       const __nv_bfloat16 *__restrict__ bb, float eps, RingDst dst, int32_t *n_surv_dev) {
   __shared__ int16_t src_of[kMaxB];
+  __shared__ int16_t pos_of[kMaxB];
   __shared__ int word_cnt[kMaxB / 32 + 1];
   const unsigned long long tl0 = tl_now();
   const int warp = warp_id(), lane = lane_id();
@@ -199,8 +203,25 @@ __global__ void __launch_bounds__(kThreads, VPL <= 3 ? 2 : 1)
   pdl_wait();
   pdl_trigger();
   const unsigned long long tl1 = tl_now();
+  const int stride = gridDim.x * (kThreads / 32);
+  const int all_units = B * S;
+  // One pass over the SOURCE rows when every row has a slot (BB: 8192 rows,
+  // 2 x 148 CTAs x 8 warps x 4): the row loads are issued before the scan of
+  // the alive flags, LayerNorm runs on them, and only survivors are stored at
+  // their compacted position -- the load latency overlaps the scan instead of
+  // following it (exiting rows are read and normalised for nothing, <= B S H 2
+  // bytes of L2 traffic).  Otherwise survivors are gathered by destination.
+  const bool spec = all_units <= kRowsInFlight * stride;
+  uint4 v[kRowsInFlight][VPL];
+  if (spec) {
+#pragma unroll
+    for (int j = 0; j < kRowsInFlight; ++j) {
+      const int u = blockIdx.x * (kThreads / 32) + warp + j * stride;
+      if (u < all_units) ln_load_row<VPL>(v[j], y + (size_t)u * H, H, lane);
+    }
+  }
   const int64_t tail = dst.tail_dev ? *dst.tail_dev : 0;
-  const int n = block_scan_flags(alive, B, src_of, word_cnt);
+  const int n = block_scan_flags(alive, B, src_of, word_cnt, pos_of);
   if (threadIdx.x == 0) tl_rec(60, tl1, tl1);   // scan done
   const bool fits = (tail - dst.head) + n <= dst.cap;
   if (blockIdx.x == 0 && threadIdx.x == 0) {
@@ -216,11 +237,23 @@ __global__ void __launch_bounds__(kThreads, VPL <= 3 ? 2 : 1)
   }
 
   const int units = n * S;
-  const int stride = gridDim.x * (kThreads / 32);
   __nv_bfloat16 *ring = reinterpret_cast<__nv_bfloat16 *>(dst.rows);
   const size_t row_elems = (size_t)S * H;
-  for (int u0 = blockIdx.x * (kThreads / 32) + warp; u0 < units; u0 += kRowsInFlight * stride) {
-    uint4 v[kRowsInFlight][VPL];
+  if (spec) {
+#pragma unroll
+    for (int j = 0; j < kRowsInFlight; ++j) {
+      const int u = blockIdx.x * (kThreads / 32) + warp + j * stride;
+      if (u < all_units) {
+        const int b = u / S, t = u - b * S;
+        const int k = pos_of[b];
+        if (k >= 0) {
+          if (kLn) ln_apply<VPL>(v[j], p, H, eps, lane);
+          ln_store_row<VPL>(v[j], ring + ((tail + k) % dst.cap) * row_elems + (size_t)t * H, H, lane);
+        }
+      }
+    }
+  }
+  for (int u0 = blockIdx.x * (kThreads / 32) + warp; !spec && u0 < units; u0 += kRowsInFlight * stride) {
 #pragma unroll
     for (int j = 0; j < kRowsInFlight; ++j) {
       const int u = u0 + j * stride;
