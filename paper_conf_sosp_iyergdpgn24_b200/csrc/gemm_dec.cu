@@ -74,7 +74,21 @@ struct SK {
   }
 };
 
-template <int T, int EPI>
+__device__ __forceinline__ float ld_dsmem_f32(uint32_t addr) {
+  float v;
+  asm volatile("ld.shared::cluster.f32 %0, [%1];" : "=f"(v) : "r"(addr) : "memory");
+  return v;
+}
+
+// CSK > 1: cluster split-K instead of stream-K (the narrow W_o / W_down,
+// 32 tiles): a cluster of CSK CTAs per tile, CTA r summing k-blocks
+// [r nkb / CSK, (r + 1) nkb / CSK); the fp32 partial tiles stay in each CTA's
+// smem and CTA r reduces rows [r 128 / CSK, +128 / CSK) of the tile over the
+// cluster through DSMEM in rank order (deterministic; every tile has the same
+// split, so a row's rounding does not depend on its position), then runs the
+// epilogue on those rows.  No global partials, tickets or fences: the stream-K
+// fixup cost ~5 us after the mainloop on these shapes (r01 dec_timeline).
+template <int T, int EPI, int CSK>
 __global__ void __launch_bounds__(kDThreads, 1)
     gemm_dec_kernel(const __grid_constant__ CUtensorMap tmW, const __grid_constant__ CUtensorMap tmW2,
                     const __grid_constant__ CUtensorMap tmX, DecArgs a) {
@@ -103,7 +117,15 @@ __global__ void __launch_bounds__(kDThreads, 1)
   sk.nkb = a.K / DK;
   sk.total = (long)tiles * sk.nkb;
   sk.G = gridDim.x;
-  const long my0 = sk.start(blockIdx.x), my1 = sk.start(blockIdx.x + 1);
+  long my0, my1;
+  if (CSK > 1) {
+    const long tile = blockIdx.x / CSK, rr = blockIdx.x % CSK;   // rr == cluster rank (cluster dims CSK x 1 x 1)
+    my0 = tile * sk.nkb + rr * sk.nkb / CSK;
+    my1 = tile * sk.nkb + (rr + 1) * sk.nkb / CSK;
+  } else {
+    my0 = sk.start(blockIdx.x);
+    my1 = sk.start(blockIdx.x + 1);
+  }
 
   if (warp == 0 && lane == 0) {
     tma_prefetch(&tmW);
@@ -253,6 +275,7 @@ __global__ void __launch_bounds__(kDThreads, 1)
       if (lane == 0) mbar_arrive(&tempty[acc]);
       if (++acc == 2) { acc = 0; acc_phase ^= 1; }
       epi_bar();
+      if (CSK > 1) break;               // one segment; reduced across the cluster below
 
       if (!whole) {
         // shared tile: publish this contributor's partial; the tile's last
@@ -517,6 +540,54 @@ __global__ void __launch_bounds__(kDThreads, 1)
       tl_rec(8000 + EPI, tlf, tlm);
     }
   }
+  if (CSK > 1) {
+    constexpr int RPC = DM / CSK;       // rows reduced and stored by this CTA
+    const int cr = (int)cluster_ctarank();
+    const int tile = blockIdx.x / CSK;
+    cluster_sync();                     // every CTA's partial tile is in its smem
+    if (warp >= 2) {
+      const int et = threadIdx.x - 64;
+      for (int e = et; e < RPC * T; e += 128) {
+        const int row = cr * RPC + e / T, t = e % T;
+        const uint32_t off = smem_u32(&sE[row * P + t]);
+        float acc = 0.f;
+#pragma unroll
+        for (int q = 0; q < CSK; ++q) acc += (q == cr) ? sE[row * P + t] : ld_dsmem_f32(mapa_shared(off, (uint32_t)q));
+        sE[row * P + t] = acc;          // only this CTA reads its own rows from here on
+      }
+    }
+    cluster_sync();                     // no CTA leaves while a peer may still read its smem
+    if (warp >= 2 && (EPI == E3_DEC_STORE || EPI == E3_DEC_RESID)) {
+      const int et = threadIdx.x - 64;
+      constexpr int NG = RPC / 8, TP = 128 / NG;   // 8-row groups, tokens per pass
+      const int g = et % NG, n = tile * DM + cr * RPC + 8 * g;
+      if (n < a.N) {
+        uint4 rres[T / TP];
+        if (EPI == E3_DEC_RESID) {
+#pragma unroll
+          for (int k = 0; k < T / TP; ++k)
+            rres[k] = __ldg(reinterpret_cast<const uint4 *>(a.R + (size_t)(et / NG + TP * k) * a.ldo + n));
+        }
+#pragma unroll
+        for (int k = 0; k < T / TP; ++k) {
+          const int t = et / NG + TP * k;
+          float v[8];
+#pragma unroll
+          for (int j = 0; j < 8; ++j) v[j] = sE[(cr * RPC + 8 * g + j) * P + t];
+          if (EPI == E3_DEC_RESID) {
+            const uint32_t rw[4] = {rres[k].x, rres[k].y, rres[k].z, rres[k].w};
+#pragma unroll
+            for (int e = 0; e < 4; ++e) {
+              v[2 * e] += bf_lo(rw[e]);
+              v[2 * e + 1] += bf_hi(rw[e]);
+            }
+          }
+          *reinterpret_cast<uint4 *>(a.Y + (size_t)t * a.ldo + n) =
+              make_uint4(pack_bf16(v[0], v[1]), pack_bf16(v[2], v[3]), pack_bf16(v[4], v[5]), pack_bf16(v[6], v[7]));
+        }
+      }
+    }
+  }
   tc_fence_before();
   __syncthreads();
   tc_fence_after();
@@ -529,28 +600,48 @@ E3_TL_SETTER(tl_set_dec)
 
 namespace {
 
-template <int T, int EPI>
+template <int T, int EPI, int CSK>
 e3_status dec_launch(const DecMaps &m, const DecArgs &a, int grid, cudaStream_t st) {
-  auto kern = gemm_dec_kernel<T, EPI>;
+  auto kern = gemm_dec_kernel<T, EPI, CSK>;
   static bool attr_done = false;
   if (!attr_done) {
     E3_CUDA_TRY(cudaFuncSetAttribute(kern, cudaFuncAttributeMaxDynamicSharedMemorySize, DCfg<T>::kSmem));
     attr_done = true;
   }
-  E3_CUDA_TRY(launch_k(kern, dim3(grid), dim3(kDThreads), DCfg<T>::kSmem, st, m.w, m.w2, m.x, a));
+  if (CSK > 1) {
+    cudaLaunchConfig_t cfg = {};
+    cfg.gridDim = dim3(grid);
+    cfg.blockDim = dim3(kDThreads);
+    cfg.dynamicSmemBytes = DCfg<T>::kSmem;
+    cfg.stream = st;
+    cudaLaunchAttribute attr[2];
+    attr[0].id = cudaLaunchAttributeClusterDimension;
+    attr[0].val.clusterDim.x = CSK;
+    attr[0].val.clusterDim.y = 1;
+    attr[0].val.clusterDim.z = 1;
+    attr[1].id = cudaLaunchAttributeProgrammaticStreamSerialization;
+    attr[1].val.programmaticStreamSerializationAllowed = 1;
+    cfg.attrs = attr;
+    cfg.numAttrs = pdl_enabled() ? 2 : 1;
+    E3_CUDA_TRY(cudaLaunchKernelEx(&cfg, kern, m.w, m.w2, m.x, a));
+  } else {
+    E3_CUDA_TRY(launch_k(kern, dim3(grid), dim3(kDThreads), DCfg<T>::kSmem, st, m.w, m.w2, m.x, a));
+  }
   E3_CUDA_TRY(cudaGetLastError());
   count_launch();
   return E3_OK;
 }
 
 template <int T>
-e3_status dec_launch_epi(const DecMaps &m, const DecArgs &a, int grid, cudaStream_t st) {
+e3_status dec_launch_epi(const DecMaps &m, const DecArgs &a, int grid, int csk, cudaStream_t st) {
   switch (a.epi) {
-    case E3_DEC_STORE: return dec_launch<T, E3_DEC_STORE>(m, a, grid, st);
-    case E3_DEC_RESID: return dec_launch<T, E3_DEC_RESID>(m, a, grid, st);
-    case E3_DEC_SWIGLU: return dec_launch<T, E3_DEC_SWIGLU>(m, a, grid, st);
-    case E3_DEC_QKV_ROPE: return dec_launch<T, E3_DEC_QKV_ROPE>(m, a, grid, st);
-    case E3_DEC_LOGITS: return dec_launch<T, E3_DEC_LOGITS>(m, a, grid, st);
+    case E3_DEC_STORE:
+      return csk == 4 ? dec_launch<T, E3_DEC_STORE, 4>(m, a, grid, st) : dec_launch<T, E3_DEC_STORE, 1>(m, a, grid, st);
+    case E3_DEC_RESID:
+      return csk == 4 ? dec_launch<T, E3_DEC_RESID, 4>(m, a, grid, st) : dec_launch<T, E3_DEC_RESID, 1>(m, a, grid, st);
+    case E3_DEC_SWIGLU: return dec_launch<T, E3_DEC_SWIGLU, 1>(m, a, grid, st);
+    case E3_DEC_QKV_ROPE: return dec_launch<T, E3_DEC_QKV_ROPE, 1>(m, a, grid, st);
+    case E3_DEC_LOGITS: return dec_launch<T, E3_DEC_LOGITS, 1>(m, a, grid, st);
   }
   set_error("bad decode epilogue");
   return E3_EINVAL;
@@ -582,12 +673,26 @@ e3_status dec_tmaps(DecMaps *m, const void *X, int T, int K, const void *W, cons
   return s;
 }
 
+// Cluster split-K (4 CTAs per tile) where the tiles fill at most a quarter
+// of the SMs (W_o, W_down of Llama-7B: 32 tiles -> 128 CTAs) and the
+// epilogue is a plain / residual store with 16-byte vectors; E3_DEC_STREAMK
+// forces stream-K everywhere (diagnostics)
+static int dec_csk(const DecArgs &a, int sms) {
+  static const bool off = getenv("E3_DEC_STREAMK") != nullptr;
+  if (off || (a.epi != E3_DEC_STORE && a.epi != E3_DEC_RESID)) return 1;
+  const int tiles = dec_tiles(a.N, a.epi);
+  const bool vec = a.ldo % 8 == 0 && a.N % 8 == 0 && (reinterpret_cast<uintptr_t>(a.Y) & 15) == 0 &&
+                   (a.epi != E3_DEC_RESID || (reinterpret_cast<uintptr_t>(a.R) & 15) == 0);
+  return (vec && 4 * tiles <= sms && a.K / DK >= 4) ? 4 : 1;
+}
+
 e3_status dec_run(const DecMaps &m, const DecArgs &a, int sms, cudaStream_t st) {
-  const int grid = dec_grid(a.N, a.K, a.epi, sms);
+  const int csk = dec_csk(a, sms);
+  const int grid = csk > 1 ? csk * dec_tiles(a.N, a.epi) : dec_grid(a.N, a.K, a.epi, sms);
   switch (a.T) {
-    case 32: return dec_launch_epi<32>(m, a, grid, st);
-    case 64: return dec_launch_epi<64>(m, a, grid, st);
-    case 128: return dec_launch_epi<128>(m, a, grid, st);
+    case 32: return dec_launch_epi<32>(m, a, grid, csk, st);
+    case 64: return dec_launch_epi<64>(m, a, grid, csk, st);
+    case 128: return dec_launch_epi<128>(m, a, grid, csk, st);
   }
   set_error("decode GEMM: batch must be 32, 64 or 128 tokens");
   return E3_EUNSUPPORTED;
