@@ -122,6 +122,7 @@ struct DecArgs {
   const int32_t *slot_of_id;
   int64_t id_cap;
   const int32_t *pos_of_slot;
+  int late_trigger;         // PDL trigger at the end instead of after the dependency wait
 };
 int dec_tiles(int N, int epi);
 int dec_max_contrib(int N, int K, int epi, int sms);
