@@ -562,19 +562,25 @@ __global__ void __launch_bounds__(kVitKQ * 2 * CB) ramp_vit_kernel(RampArgs a, i
 // the rows per class group: 100 us per VT launch (r01 timeline).
 constexpr int kVtcThreads = 256;
 
+constexpr int kVtcKC = 128;                            // K chunk of the staged W_c slice
+constexpr int kVtcPW = kVtcKC + 8;                     // its padded pitch (bf16)
 __host__ __device__ inline int ramp_vit_tc_smem(int H) {
   const int P = H + 8;
-  return 64 * P * 2 + 3 * kVitRows * P * 2;
+  return 3 * kVitRows * P * 2 + 2 * 128 * kVtcPW * 2;
 }
 
 template <bool kLate>
 __global__ void __launch_bounds__(kVtcThreads, 1) ramp_vit_tc_kernel(RampArgs a, int CS) {
-  constexpr int CB = 64, kThreads = 2 * CB, kWarps = kThreads / 32, kWarpsPerRg = CB / 64;
+  // 128 classes per CTA (8 warps x two n8 tiles): clusters of <= 8 CTAs for
+  // C <= 1024, all resident at once (16-CTA clusters of 64-class slices fit
+  // one per GPC and ran in 2-3 waves)
+  constexpr int CB = 128, kThreads = 2 * CB, kWarps = kThreads / 32, kWarpsPerRg = CB / 64;
+  static_assert(kThreads == kVtcThreads, "all threads own 2 classes x 4 rows");
   const unsigned long long tl0 = tl_now();
   extern __shared__ uint8_t smem_raw[];
   const int H = a.H, C = a.C, P = H + 8;
-  __nv_bfloat16 *sW = reinterpret_cast<__nv_bfloat16 *>(smem_raw);   // [64][P]
-  __nv_bfloat16 *sA = sW + 64 * P;                                    // [3][16][P]: hi, mid, lo
+  __nv_bfloat16 *sA = reinterpret_cast<__nv_bfloat16 *>(smem_raw);   // [3][16][P]: hi, mid, lo
+  __nv_bfloat16 *sWc = sA + 3 * kVitRows * P;                         // [2][128][kVtcPW] W_c chunks
   __shared__ float sZ[kVitRows][CB];
   __shared__ SoftStat sRed[kWarps][4];
   __shared__ SoftStat sQ[16][kVitRows];               // rank 0: [rank][row]
@@ -592,14 +598,22 @@ __global__ void __launch_bounds__(kVtcThreads, 1) ramp_vit_tc_kernel(RampArgs a,
   const float bias0 = c0 < C ? bf2f(bc[c0]) : 0.f, bias1 = c1 < C ? bf2f(bc[c1]) : 0.f;
   const int nvec = H / 8;
   cluster_arrive_relaxed();
-  // W_c rows [rank*64, +64) -> smem (zero rows past C): no dependency
-  for (int i = tAll; i < 64 * nvec; i += kVtcThreads) {
-    const int r = i / nvec, k = i - r * nvec;
-    const int c = (int)rank * CB + r;
-    uint4 *dst = reinterpret_cast<uint4 *>(sW + r * P) + k;
-    if (c < C) cp_async16(dst, reinterpret_cast<const uint4 *>(W + (size_t)c * H) + k);
-    else *dst = make_uint4(0, 0, 0, 0);
-  }
+  // W_c slice [rank*128, +128) x H in K chunks of 128 through a double
+  // buffer (cp.async, zero rows past C); chunk 0 before the PDL wait
+  const int nch = (H + kVtcKC - 1) / kVtcKC;
+  auto stage_chunk = [&](int c) {
+    __nv_bfloat16 *dstb = sWc + (c & 1) * 128 * kVtcPW;
+    const int k0 = c * kVtcKC, kw = min(kVtcKC, H - k0) / 8;   // 16-byte vectors per row
+    for (int i = tAll; i < 128 * kw; i += kVtcThreads) {
+      const int r = i / kw, v = i - r * kw;
+      const int cls = (int)rank * CB + r;
+      uint4 *d = reinterpret_cast<uint4 *>(dstb + r * kVtcPW) + v;
+      if (cls < C) cp_async16(d, reinterpret_cast<const uint4 *>(W + (size_t)cls * H + k0) + v);
+      else *d = make_uint4(0, 0, 0, 0);
+    }
+    asm volatile("cp.async.commit_group;" ::: "memory");
+  };
+  stage_chunk(0);
   pdl_wait();
   if (!kLate) pdl_trigger();
   const unsigned long long tl1 = tl_now();
@@ -681,35 +695,62 @@ __global__ void __launch_bounds__(kVtcThreads, 1) ramp_vit_tc_kernel(RampArgs a,
       }
     }
   }
-  cp_async_wait_all();
   __syncthreads();
   const unsigned long long tlLn = tl_now();
 
-  // ---- classifier: warp w, classes 8w .. 8w + 7, three split products
+  // ---- classifier: warp w, classes 16w .. 16w + 15 (two n8 tiles), three
+  // split products per k16 step, W_c fragments from the staged chunk (the
+  // first version staged the whole 64-class slice, 99 KB, in 16-CTA clusters
+  // that ran in three waves: ~60 us per VT launch; fragments straight from L2
+  // were scattered 4-byte loads: 20-28 us)
   {
-    float acc[4] = {0.f, 0.f, 0.f, 0.f};
-    const __nv_bfloat16 *bw = sW + (8 * wAll + gq) * P + 2 * tq;
+    float acc[2][4] = {};
+    const __nv_bfloat16 *a0 = sA + gq * P + 2 * tq;
 #pragma unroll 1
-    for (int sp = 0; sp < 3; ++sp) {
-      const __nv_bfloat16 *a_lo = sA + (sp * kVitRows + gq) * P + 2 * tq;
-      const __nv_bfloat16 *a_hi = sA + (sp * kVitRows + gq + 8) * P + 2 * tq;
-#pragma unroll 4
-      for (int k = 0; k < H; k += 16) {
-        uint32_t af[4];
-        af[0] = *reinterpret_cast<const uint32_t *>(a_lo + k);
-        af[1] = *reinterpret_cast<const uint32_t *>(a_hi + k);
-        af[2] = *reinterpret_cast<const uint32_t *>(a_lo + k + 8);
-        af[3] = *reinterpret_cast<const uint32_t *>(a_hi + k + 8);
-        const uint32_t bf0 = *reinterpret_cast<const uint32_t *>(bw + k);
-        const uint32_t bf1 = *reinterpret_cast<const uint32_t *>(bw + k + 8);
-        mma_bf16_16816(acc, af, bf0, bf1);
+    for (int c = 0; c < nch; ++c) {
+      if (c + 1 < nch) {
+        stage_chunk(c + 1);
+        asm volatile("cp.async.wait_group 1;" ::: "memory");
+      } else {
+        asm volatile("cp.async.wait_group 0;" ::: "memory");
       }
+      __syncthreads();                              // chunk c landed for every thread
+      const int kb = c * kVtcKC;
+      const __nv_bfloat16 *bwc = sWc + (c & 1) * 128 * kVtcPW + (16 * wAll + gq) * kVtcPW + 2 * tq;
+#pragma unroll
+      for (int i = 0; i < kVtcKC / 16; ++i) {
+        const int k = kb + 16 * i;
+        if (k < H) {
+          uint32_t bf[2][2];
+#pragma unroll
+          for (int nt = 0; nt < 2; ++nt) {
+            bf[nt][0] = *reinterpret_cast<const uint32_t *>(bwc + nt * 8 * kVtcPW + 16 * i);
+            bf[nt][1] = *reinterpret_cast<const uint32_t *>(bwc + nt * 8 * kVtcPW + 16 * i + 8);
+          }
+#pragma unroll
+          for (int sp = 0; sp < 3; ++sp) {
+            const __nv_bfloat16 *a_lo = a0 + sp * kVitRows * P + k;
+            const __nv_bfloat16 *a_hi = a_lo + 8 * P;
+            uint32_t af[4];
+            af[0] = *reinterpret_cast<const uint32_t *>(a_lo);
+            af[1] = *reinterpret_cast<const uint32_t *>(a_hi);
+            af[2] = *reinterpret_cast<const uint32_t *>(a_lo + 8);
+            af[3] = *reinterpret_cast<const uint32_t *>(a_hi + 8);
+            mma_bf16_16816(acc[0], af, bf[0][0], bf[0][1]);
+            mma_bf16_16816(acc[1], af, bf[1][0], bf[1][1]);
+          }
+        }
+      }
+      __syncthreads();                              // buffer c & 1 is restaged for chunk c + 2
     }
-    const int col = 8 * wAll + 2 * tq;
-    sZ[gq][col] = acc[0];
-    sZ[gq][col + 1] = acc[1];
-    sZ[gq + 8][col] = acc[2];
-    sZ[gq + 8][col + 1] = acc[3];
+#pragma unroll
+    for (int nt = 0; nt < 2; ++nt) {
+      const int col = 16 * wAll + 8 * nt + 2 * tq;
+      sZ[gq][col] = acc[nt][0];
+      sZ[gq][col + 1] = acc[nt][1];
+      sZ[gq + 8][col] = acc[nt][2];
+      sZ[gq + 8][col + 1] = acc[nt][3];
+    }
   }
   __syncthreads();
   const unsigned long long tlCls = tl_now();
@@ -775,7 +816,11 @@ __global__ void __launch_bounds__(kVtcThreads, 1) ramp_vit_tc_kernel(RampArgs a,
         a.alive[b] = exit_now ? 0 : 1;
       }
     }
-    if (r < kVitRows) sDec[r] = exit_now ? 1 : 0;
+    if (r < kVitRows)                        // the decision to every CTA of the cluster (DSMEM)
+      for (int q = 0; q < CS; ++q)
+        asm volatile("st.shared::cluster.s32 [%0], %1;" ::"r"(mapa_shared(smem_u32(&sDec[r]), (uint32_t)q)),
+                     "r"(exit_now ? 1 : 0)
+                     : "memory");
     const int n_ex = __popc(__ballot_sync(0xffffffffu, exit_now));
     if (lane == 0 && n_ex) {
       if (a.ex.n_exit) atomicAdd(a.ex.n_exit, n_ex);
@@ -789,7 +834,7 @@ __global__ void __launch_bounds__(kVtcThreads, 1) ramp_vit_tc_kernel(RampArgs a,
     for (int rr = 0; rr < 4; ++rr) {
       const int r = rg * 4 + rr, b = b0 + r;
       if (b >= a.B) continue;
-      if (!ld_cluster_s32(mapa_shared(smem_u32(&sDec[r]), 0))) continue;
+      if (!sDec[r]) continue;
       const int64_t id = a.id[b];
       if (id < 0 || id >= a.ex.capacity) continue;
       if (c0 < C) a.ex.logits[id * C + c0] = z[rr][0];
@@ -810,7 +855,7 @@ e3_status ramp_vit_run(const RampArgs &a, cudaStream_t st) {
     return E3_EUNSUPPORTED;
   }
   const int CB = (a.C <= 16 * 64) ? 64 : 128;
-  const int CS = (a.C + CB - 1) / CB;
+  int CS = (a.C + CB - 1) / CB;
   const int smem = kVitRows * (a.H + 4) * 4;
   cudaLaunchConfig_t cfg = {};
   cfg.gridDim = dim3(CS, (a.B + kVitRows - 1) / kVitRows);
@@ -839,7 +884,10 @@ e3_status ramp_vit_run(const RampArgs &a, cudaStream_t st) {
     E3_CUDA_TRY(cudaLaunchKernelEx(&cfg, ramp_vit_kernel<V, L>, a, CS));                                    \
   } while (0)
   static const bool early = getenv("E3_VIT_EARLY_TRIGGER") != nullptr;   // diagnostics
-  if (a.C <= 16 * 64 && a.H <= 1024 && ramp_vit_tc_smem(a.H) <= 200 * 1024 && getenv("E3_VIT_RAMP_FMA") == nullptr) {
+  if (a.C <= 8 * 128 && a.H <= 1024 && ramp_vit_tc_smem(a.H) <= 200 * 1024 && getenv("E3_VIT_RAMP_FMA") == nullptr) {
+    CS = (a.C + 127) / 128;
+    cfg.gridDim = dim3(CS, (a.B + kVitRows - 1) / kVitRows);
+    attr[0].val.clusterDim.x = CS;
     cfg.blockDim = dim3(kVtcThreads);
     cfg.dynamicSmemBytes = ramp_vit_tc_smem(a.H);
     static bool tc_attr = false;
