@@ -31,17 +31,21 @@ __global__ void __launch_bounds__(256)
   pdl_wait();
   pdl_trigger();
   const unsigned long long tl1 = tl_now();
+  // persistent: the grid is at most one wave; each warp walks its rows RPW at
+  // a time (loads of a batch first)
+  for (int base = row0; base < rows; base += RPW * warps) {
 #pragma unroll
-  for (int j = 0; j < RPW; ++j) {
-    const int row = row0 + j * warps;
-    if (row < rows) ln_load_row<VPL>(v[j], x + (size_t)row * H, H, lane);
-  }
+    for (int j = 0; j < RPW; ++j) {
+      const int row = base + j * warps;
+      if (row < rows) ln_load_row<VPL>(v[j], x + (size_t)row * H, H, lane);
+    }
 #pragma unroll
-  for (int j = 0; j < RPW; ++j) {
-    const int row = row0 + j * warps;
-    if (row < rows) {
-      ln_apply<VPL>(v[j], p, H, eps, lane);
-      ln_store_row<VPL>(v[j], y + (size_t)row * H, H, lane);
+    for (int j = 0; j < RPW; ++j) {
+      const int row = base + j * warps;
+      if (row < rows) {
+        ln_apply<VPL>(v[j], p, H, eps, lane);
+        ln_store_row<VPL>(v[j], y + (size_t)row * H, H, lane);
+      }
     }
   }
   if (threadIdx.x == 0) tl_rec(3, tl0, tl1);
@@ -53,30 +57,38 @@ E3_TL_SETTER(tl_set_ln)
 
 e3_status layernorm_run(const void *x, const void *g, const void *b, void *y, int rows, int H, float eps,
                         cudaStream_t st) {
-  // rows per warp: 2 when that keeps the grid within one wave of resident CTAs
-  // (4 per SM), else 1
+  // rows per warp: 2 when one row per warp would exceed one wave of resident
+  // CTAs; the grid is capped at one wave and the warps walk the rest
   static int sms = 0;
   if (!sms) {
     int dev = 0;
     E3_CUDA_TRY(cudaGetDevice(&dev));
     E3_CUDA_TRY(cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, dev));
   }
-  const bool two = rows > 8 * 4 * sms && H <= 1024;   // registers: 2 rows of <= 4 vectors per lane
-  const int grid = two ? (rows + 15) / 16 : (rows + 7) / 8;
-  auto *xp = reinterpret_cast<const __nv_bfloat16 *>(x);
-  auto *gp = reinterpret_cast<const __nv_bfloat16 *>(g);
-  auto *bp = reinterpret_cast<const __nv_bfloat16 *>(b);
-  auto *yp = reinterpret_cast<__nv_bfloat16 *>(y);
   const int vpl = (H / 8 + 31) / 32;
-  if (vpl <= 1) E3_CUDA_TRY(launch_k(two ? layernorm_kernel<1, 2> : layernorm_kernel<1, 1>, dim3(grid), dim3(256), 0, st, xp, gp, bp, yp, rows, H, eps));
-  else if (vpl <= 3) E3_CUDA_TRY(launch_k(two ? layernorm_kernel<3, 2> : layernorm_kernel<3, 1>, dim3(grid), dim3(256), 0, st, xp, gp, bp, yp, rows, H, eps));
-  else if (vpl <= 4) E3_CUDA_TRY(launch_k(two ? layernorm_kernel<4, 2> : layernorm_kernel<4, 1>, dim3(grid), dim3(256), 0, st, xp, gp, bp, yp, rows, H, eps));
-  else if (vpl <= 8) E3_CUDA_TRY(launch_k(two ? layernorm_kernel<8, 2> : layernorm_kernel<8, 1>, dim3(grid), dim3(256), 0, st, xp, gp, bp, yp, rows, H, eps));
-  else if (vpl <= 16) E3_CUDA_TRY(launch_k(two ? layernorm_kernel<16, 2> : layernorm_kernel<16, 1>, dim3(grid), dim3(256), 0, st, xp, gp, bp, yp, rows, H, eps));
-  else {
+  if (vpl > 16) {
     set_error("LayerNorm: H > 4096 unsupported");
     return E3_EUNSUPPORTED;
   }
+  const bool two = rows > 8 * 4 * sms && H <= 1024;   // registers: 2 rows of <= 4 vectors per lane
+  using Kern = void (*)(const __nv_bfloat16 *, const __nv_bfloat16 *, const __nv_bfloat16 *, __nv_bfloat16 *, int,
+                        int, float);
+  const int vi = vpl <= 1 ? 0 : vpl <= 3 ? 1 : vpl <= 4 ? 2 : vpl <= 8 ? 3 : 4;
+  static const Kern kerns[5][2] = {{layernorm_kernel<1, 1>, layernorm_kernel<1, 2>},
+                                   {layernorm_kernel<3, 1>, layernorm_kernel<3, 2>},
+                                   {layernorm_kernel<4, 1>, layernorm_kernel<4, 2>},
+                                   {layernorm_kernel<8, 1>, layernorm_kernel<8, 2>},
+                                   {layernorm_kernel<16, 1>, layernorm_kernel<16, 2>}};
+  static int occ[5][2] = {};
+  const Kern kern = kerns[vi][two ? 1 : 0];
+  int &o = occ[vi][two ? 1 : 0];
+  if (!o) E3_CUDA_TRY(cudaOccupancyMaxActiveBlocksPerMultiprocessor(&o, kern, 256, 0));
+  if (o < 1) o = 1;
+  int grid = two ? (rows + 15) / 16 : (rows + 7) / 8;
+  if (grid > o * sms) grid = o * sms;
+  E3_CUDA_TRY(launch_k(kern, dim3(grid), dim3(256), 0, st, reinterpret_cast<const __nv_bfloat16 *>(x),
+                       reinterpret_cast<const __nv_bfloat16 *>(g), reinterpret_cast<const __nv_bfloat16 *>(b),
+                       reinterpret_cast<__nv_bfloat16 *>(y), rows, H, eps));
   E3_CUDA_TRY(cudaGetLastError());
   count_launch();
   return E3_OK;
