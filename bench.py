@@ -373,7 +373,9 @@ def main():
     traffic = None
     ncu_path = os.path.join(ROOT, "profiles", "ncu_traffic.json")
     if os.path.exists(ncu_path):
-        traffic = json.load(open(ncu_path)).get(top)
+        nt = json.load(open(ncu_path))
+        if nt.get("_workload") == cfg.name:   # the capture is of one workload's kernels
+            traffic = nt.get(top)
     if tk["flops"] > 0:
         ach = tk["flops"] / (tk["ms"] / 1e3) / 1e12
         roof = {"bound": "tensor", "achieved": round(ach, 1), "peak": tf_peak, "unit": "TFLOP/s",
