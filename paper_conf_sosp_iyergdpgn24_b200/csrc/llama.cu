@@ -149,20 +149,30 @@ __global__ void __launch_bounds__(kAttnThreads)
   // ---- scores: warp w takes keys [8s, 8s+8) for s = w, w + 8, ...; each key
   // row is one coalesced 256-byte warp load
   float lmax = -INFINITY;
-  for (int j0 = warp * kKeysPerStep; j0 < L; j0 += kAW * kKeysPerStep) {
-    uint2 kv[kKeysPerStep];
+  constexpr int kG = 2;                         // groups of kKeysPerStep keys in flight per warp step
+  for (int j0 = warp * kG * kKeysPerStep; j0 < L; j0 += kAW * kG * kKeysPerStep) {
+    uint2 kv[kG][kKeysPerStep];
 #pragma unroll
-    for (int i = 0; i < kKeysPerStep; ++i)
-      kv[i] = (j0 + i < L) ? K[(size_t)(j0 + i) * (kHd / 4)] : make_uint2(0u, 0u);
-    float d[kKeysPerStep];
+    for (int gi = 0; gi < kG; ++gi)
 #pragma unroll
-    for (int i = 0; i < kKeysPerStep; ++i)
-      d[i] = fmaf(q0, bf_lo(kv[i].x), fmaf(q1, bf_hi(kv[i].x), fmaf(q2, bf_lo(kv[i].y), q3 * bf_hi(kv[i].y))));
-    const float sc = reduce8(d, lane);
-    const int k = ((lane >> 4) & 1) * 4 + ((lane >> 3) & 1) * 2 + ((lane >> 2) & 1);
-    if ((lane & 3) == 0 && j0 + k < L) {
-      sp[j0 + k] = sc;
-      lmax = fmaxf(lmax, sc);
+      for (int i = 0; i < kKeysPerStep; ++i) {
+        const int j = j0 + gi * kKeysPerStep + i;
+        kv[gi][i] = (j < L) ? K[(size_t)j * (kHd / 4)] : make_uint2(0u, 0u);
+      }
+#pragma unroll
+    for (int gi = 0; gi < kG; ++gi) {
+      float d[kKeysPerStep];
+#pragma unroll
+      for (int i = 0; i < kKeysPerStep; ++i)
+        d[i] = fmaf(q0, bf_lo(kv[gi][i].x),
+                    fmaf(q1, bf_hi(kv[gi][i].x), fmaf(q2, bf_lo(kv[gi][i].y), q3 * bf_hi(kv[gi][i].y))));
+      const float sc = reduce8(d, lane);
+      const int k = ((lane >> 4) & 1) * 4 + ((lane >> 3) & 1) * 2 + ((lane >> 2) & 1);
+      const int jj = j0 + gi * kKeysPerStep + k;
+      if ((lane & 3) == 0 && jj < L) {
+        sp[jj] = sc;
+        lmax = fmaxf(lmax, sc);
+      }
     }
   }
   const float m = block_reduce(lmax, red, true);
@@ -176,7 +186,7 @@ __global__ void __launch_bounds__(kAttnThreads)
   // ---- P V: warp w takes positions j = w mod 8, lane owns dims 4*lane .. +3
   const uint2 *V = reinterpret_cast<const uint2 *>(vc + base) + lane;
   float4 acc = make_float4(0.f, 0.f, 0.f, 0.f);
-#pragma unroll 8
+#pragma unroll 16
   for (int j = warp; j < L; j += kAW) {
     const uint2 vv = V[(size_t)j * (kHd / 4)];
     const float p = sp[j];
