@@ -39,18 +39,22 @@ namespace {
 
 constexpr int DM = 128;            // weight rows per tile (MMA M)
 constexpr int DK = 64;             // K per 128-byte swizzle atom / TMA box
-constexpr int kDThreads = 192;     // warp 0 TMA, warp 1 MMA, warps 2-5 epilogue
+constexpr int kDThreads = 224;     // warp 0 W TMA, warp 1 MMA, warps 2-5 epilogue, warp 6 X TMA
 constexpr int kSmemMax = 232448;
 
 template <int T>
+// Separate rings for W (HBM: deep, 9 stages at T = 64) and X (L2-resident
+// tokens: 4 stages), each with its own producer warp: one shared ring of
+// W + X stages held 7 x 16 KB of weights in flight per SM
 struct DCfg {
   static constexpr int kWBytes = DM * DK * 2;               // 16 KB
   static constexpr int kXBytes = T * DK * 2;
-  static constexpr int kStageBytes = kWBytes + kXBytes;
+  static constexpr int kXStages = 4;
   static constexpr int kEBytes = DM * (T + 1) * 4;          // fp32 epilogue tile
-  static constexpr int kStages = (kSmemMax - kEBytes - 1024 - 3072) / kStageBytes;
+  static constexpr int kStages = (kSmemMax - kEBytes - 1024 - 3072 - kXStages * kXBytes) / kWBytes;
   static constexpr int kTmemCols = (2 * T <= 32) ? 32 : (2 * T <= 64) ? 64 : (2 * T <= 128) ? 128 : 256;
-  static constexpr int kSmem = kStages * kStageBytes + kEBytes + 1024 + 3072;   // + barriers, token tables
+  static constexpr int kSmem = kStages * kWBytes + kXStages * kXBytes + kEBytes + 1024 + 3072;   // + barriers, token tables
+  static_assert(kStages >= 4, "weight ring too shallow");
 };
 
 __device__ __forceinline__ void epi_bar() { asm volatile("bar.sync 1, 128;" ::: "memory"); }
@@ -98,12 +102,15 @@ __global__ void __launch_bounds__(kDThreads, 1)
   const unsigned long long tl0 = tl_now();
   extern __shared__ uint8_t smem_raw[];
   uint8_t *smem = reinterpret_cast<uint8_t *>((reinterpret_cast<uintptr_t>(smem_raw) + 1023) & ~uintptr_t(1023));
+  constexpr int XS = CF::kXStages;
   uint8_t *sW = smem;
   uint8_t *sX = smem + S * CF::kWBytes;
-  float *sE = reinterpret_cast<float *>(smem + S * CF::kStageBytes);
+  float *sE = reinterpret_cast<float *>(sX + XS * CF::kXBytes);
   uint64_t *full = reinterpret_cast<uint64_t *>(reinterpret_cast<uint8_t *>(sE) + CF::kEBytes);
   uint64_t *empty = full + S;
-  uint64_t *tfull = empty + S;     // [2]
+  uint64_t *xfull = empty + S;     // [XS]
+  uint64_t *xempty = xfull + XS;   // [XS]
+  uint64_t *tfull = xempty + XS;   // [2]
   uint64_t *tempty = tfull + 2;    // [2]
   uint32_t *tmem_slot = reinterpret_cast<uint32_t *>(tempty + 2);
   int *s_last = reinterpret_cast<int *>(tmem_slot + 1);
@@ -137,6 +144,10 @@ __global__ void __launch_bounds__(kDThreads, 1)
       mbar_init(&full[i], 1);
       mbar_init(&empty[i], 1);
     }
+    for (int i = 0; i < XS; ++i) {
+      mbar_init(&xfull[i], 1);
+      mbar_init(&xempty[i], 1);
+    }
     for (int i = 0; i < 2; ++i) {
       mbar_init(&tfull[i], 1);
       mbar_init(&tempty[i], 4);    // 4 epilogue warps
@@ -166,21 +177,33 @@ __global__ void __launch_bounds__(kDThreads, 1)
       const int pre = total < S ? total : S;
       // weights first: they do not depend on the previous kernel
       for (int it = 0; it < pre; ++it) {
-        mbar_expect_tx(&full[it], CF::kStageBytes);
+        mbar_expect_tx(&full[it], CF::kWBytes);
         load_w(it, it);
       }
       pdl_wait();
       if (!a.late_trigger) pdl_trigger();
-      for (int it = 0; it < pre; ++it)
-        tma_load_2d(sX + it * CF::kXBytes, &tmX, &full[it], (int)((my0 + it) % sk.nkb) * DK, 0);
       int stage = pre % S;
       uint32_t phase = (pre == S) ? 1 : 0;
       for (int it = pre; it < total; ++it) {
         mbar_wait(&empty[stage], phase ^ 1);
-        mbar_expect_tx(&full[stage], CF::kStageBytes);
+        mbar_expect_tx(&full[stage], CF::kWBytes);
         load_w(it, stage);
-        tma_load_2d(sX + stage * CF::kXBytes, &tmX, &full[stage], (int)((my0 + it) % sk.nkb) * DK, 0);
         if (++stage == S) { stage = 0; phase ^= 1; }
+      }
+    }
+  } else if (warp == 6) {
+    // ------------------------------------------------------- X (tokens) producer
+    pdl_wait();
+    if (!a.late_trigger) pdl_trigger();
+    if (lane == 0) {
+      const int total = (int)(my1 - my0);
+      int xs = 0;
+      uint32_t xphase = 0;
+      for (int it = 0; it < total; ++it) {
+        mbar_wait(&xempty[xs], xphase ^ 1);
+        mbar_expect_tx(&xfull[xs], CF::kXBytes);
+        tma_load_2d(sX + xs * CF::kXBytes, &tmX, &xfull[xs], (int)((my0 + it) % sk.nkb) * DK, 0);
+        if (++xs == XS) { xs = 0; xphase ^= 1; }
       }
     }
   } else if (warp == 1) {
@@ -189,8 +212,8 @@ __global__ void __launch_bounds__(kDThreads, 1)
     if (!a.late_trigger) pdl_trigger();
     if (lane == 0) {
       constexpr uint32_t idesc = idesc_bf16_f32(DM, T, 0);
-      int stage = 0;
-      uint32_t phase = 0;
+      int stage = 0, xs = 0;
+      uint32_t phase = 0, xphase = 0;
       int acc = 0;
       uint32_t acc_phase = 0;
       for (long i = my0; i < my1;) {                 // one segment = this CTA's part of one tile
@@ -201,14 +224,17 @@ __global__ void __launch_bounds__(kDThreads, 1)
         const uint32_t d_tmem = tmem_base + acc * T;
         for (long j = i; j < seg_end; ++j) {
           mbar_wait(&full[stage], phase);
+          mbar_wait(&xfull[xs], xphase);
           tc_fence_after();
           const uint64_t da = smem_desc_sw128(smem_u32(sW + stage * CF::kWBytes), 16, 1024);
-          const uint64_t db = smem_desc_sw128(smem_u32(sX + stage * CF::kXBytes), 16, 1024);
+          const uint64_t db = smem_desc_sw128(smem_u32(sX + xs * CF::kXBytes), 16, 1024);
 #pragma unroll
           for (int k = 0; k < DK / 16; ++k)
             tc_mma_f16(d_tmem, da + (uint64_t)(2 * k), db + (uint64_t)(2 * k), idesc, (j != i) || k != 0);
           tc_commit(&empty[stage]);
+          tc_commit(&xempty[xs]);
           if (++stage == S) { stage = 0; phase ^= 1; }
+          if (++xs == XS) { xs = 0; xphase ^= 1; }
         }
         tc_commit(&tfull[acc]);
         if (++acc == 2) { acc = 0; acc_phase ^= 1; }
@@ -545,7 +571,7 @@ __global__ void __launch_bounds__(kDThreads, 1)
     const int cr = (int)cluster_ctarank();
     const int tile = blockIdx.x / CSK;
     cluster_sync();                     // every CTA's partial tile is in its smem
-    if (warp >= 2) {
+    if (warp >= 2 && warp <= 5) {
       const int et = threadIdx.x - 64;
       for (int e = et; e < RPC * T; e += 128) {
         const int row = cr * RPC + e / T, t = e % T;
@@ -557,7 +583,7 @@ __global__ void __launch_bounds__(kDThreads, 1)
       }
     }
     cluster_sync();                     // no CTA leaves while a peer may still read its smem
-    if (warp >= 2 && (EPI == E3_DEC_STORE || EPI == E3_DEC_RESID)) {
+    if (warp >= 2 && warp <= 5 && (EPI == E3_DEC_STORE || EPI == E3_DEC_RESID)) {
       const int et = threadIdx.x - 64;
       constexpr int NG = RPC / 8, TP = 128 / NG;   // 8-row groups, tokens per pass
       const int g = et % NG, n = tile * DM + cr * RPC + 8 * g;
