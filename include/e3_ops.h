@@ -31,7 +31,7 @@ e3_status e3_op_gemm(void *stream, const void *A, int64_t lda, const void *W, co
 
 /* Decode-shaped GEMM of the LLaMA split (a8; gemm_dec.cu): Y[T,N] =
  * epi(X[T,K] W[N,K]^T), bf16 in, fp32 accumulate, bf16 out, T in {32, 64,
- * 128} tokens, K % 64 == 0.  epilogue: 0 plain, 1 + R[T,N] (residual),
+ * 128} tokens, K % 128 == 0.  epilogue: 0 plain, 1 + R[T,N] (residual),
  * 2 SwiGLU: Y[T,N] = SiLU(X W^T) * (X W2^T) with W = W_gate, W2 = W_up [N,K]
  * (N % 64 == 0).  Stream-K scratch is allocated on the stream per call. */
 e3_status e3_op_dec_gemm(void *stream, const void *X, int32_t T, const void *W, const void *W2, int32_t N,

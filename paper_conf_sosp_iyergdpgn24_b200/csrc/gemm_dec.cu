@@ -39,6 +39,8 @@ namespace {
 
 constexpr int DM = 128;            // weight rows per tile (MMA M)
 constexpr int DK = 64;             // K per 128-byte swizzle atom / TMA box
+constexpr int DKS = 2 * DK;        // K per pipeline stage: two atoms, so the two 128-byte
+                                   // pieces of a weight row are requested back to back
 constexpr int kDThreads = 224;     // warp 0 W TMA, warp 1 MMA, warps 2-5 epilogue, warp 6 X TMA
 constexpr int kSmemMax = 232448;
 
@@ -47,14 +49,16 @@ template <int T>
 // tokens: 4 stages), each with its own producer warp: one shared ring of
 // W + X stages held 7 x 16 KB of weights in flight per SM
 struct DCfg {
-  static constexpr int kWBytes = DM * DK * 2;               // 16 KB
-  static constexpr int kXBytes = T * DK * 2;
-  static constexpr int kXStages = 4;
+  static constexpr int kWAtom = DM * DK * 2;                // 16 KB
+  static constexpr int kXAtom = T * DK * 2;
+  static constexpr int kWBytes = 2 * kWAtom;
+  static constexpr int kXBytes = 2 * kXAtom;
+  static constexpr int kXStages = 2;
   static constexpr int kEBytes = DM * (T + 1) * 4;          // fp32 epilogue tile
   static constexpr int kStages = (kSmemMax - kEBytes - 1024 - 3072 - kXStages * kXBytes) / kWBytes;
   static constexpr int kTmemCols = (2 * T <= 32) ? 32 : (2 * T <= 64) ? 64 : (2 * T <= 128) ? 128 : 256;
   static constexpr int kSmem = kStages * kWBytes + kXStages * kXBytes + kEBytes + 1024 + 3072;   // + barriers, token tables
-  static_assert(kStages >= 4, "weight ring too shallow");
+  static_assert(kStages >= 2, "weight ring too shallow");
 };
 
 __device__ __forceinline__ void epi_bar() { asm volatile("bar.sync 1, 128;" ::: "memory"); }
@@ -121,7 +125,7 @@ __global__ void __launch_bounds__(kDThreads, 1)
   const int warp = warp_id(), lane = lane_id();
   const int tiles = (EPI == E3_DEC_SWIGLU) ? a.N / 64 : (a.N + DM - 1) / DM;
   SK sk;
-  sk.nkb = a.K / DK;
+  sk.nkb = a.K / DKS;
   sk.total = (long)tiles * sk.nkb;
   sk.G = gridDim.x;
   long my0, my1;
@@ -166,12 +170,16 @@ __global__ void __launch_bounds__(kDThreads, 1)
       const int total = (int)(my1 - my0);
       auto load_w = [&](int it, int st) {
         const long i = my0 + it;
-        const int tile = (int)(i / sk.nkb), k0 = (int)(i % sk.nkb) * DK;
-        if (EPI == E3_DEC_SWIGLU) {
-          tma_load_2d(sW + st * CF::kWBytes, &tmW, &full[st], k0, tile * 64);
-          tma_load_2d(sW + st * CF::kWBytes + CF::kWBytes / 2, &tmW2, &full[st], k0, tile * 64);
-        } else {
-          tma_load_2d(sW + st * CF::kWBytes, &tmW, &full[st], k0, tile * DM);
+        const int tile = (int)(i / sk.nkb), k0 = (int)(i % sk.nkb) * DKS;
+#pragma unroll
+        for (int sub = 0; sub < 2; ++sub) {
+          uint8_t *dst = sW + st * CF::kWBytes + sub * CF::kWAtom;
+          if (EPI == E3_DEC_SWIGLU) {
+            tma_load_2d(dst, &tmW, &full[st], k0 + sub * DK, tile * 64);
+            tma_load_2d(dst + CF::kWAtom / 2, &tmW2, &full[st], k0 + sub * DK, tile * 64);
+          } else {
+            tma_load_2d(dst, &tmW, &full[st], k0 + sub * DK, tile * DM);
+          }
         }
       };
       const int pre = total < S ? total : S;
@@ -202,7 +210,10 @@ __global__ void __launch_bounds__(kDThreads, 1)
       for (int it = 0; it < total; ++it) {
         mbar_wait(&xempty[xs], xphase ^ 1);
         mbar_expect_tx(&xfull[xs], CF::kXBytes);
-        tma_load_2d(sX + xs * CF::kXBytes, &tmX, &xfull[xs], (int)((my0 + it) % sk.nkb) * DK, 0);
+#pragma unroll
+        for (int sub = 0; sub < 2; ++sub)
+          tma_load_2d(sX + xs * CF::kXBytes + sub * CF::kXAtom, &tmX, &xfull[xs],
+                      (int)((my0 + it) % sk.nkb) * DKS + sub * DK, 0);
         if (++xs == XS) { xs = 0; xphase ^= 1; }
       }
     }
@@ -226,11 +237,14 @@ __global__ void __launch_bounds__(kDThreads, 1)
           mbar_wait(&full[stage], phase);
           mbar_wait(&xfull[xs], xphase);
           tc_fence_after();
-          const uint64_t da = smem_desc_sw128(smem_u32(sW + stage * CF::kWBytes), 16, 1024);
-          const uint64_t db = smem_desc_sw128(smem_u32(sX + xs * CF::kXBytes), 16, 1024);
 #pragma unroll
-          for (int k = 0; k < DK / 16; ++k)
-            tc_mma_f16(d_tmem, da + (uint64_t)(2 * k), db + (uint64_t)(2 * k), idesc, (j != i) || k != 0);
+          for (int sub = 0; sub < 2; ++sub) {
+            const uint64_t da = smem_desc_sw128(smem_u32(sW + stage * CF::kWBytes + sub * CF::kWAtom), 16, 1024);
+            const uint64_t db = smem_desc_sw128(smem_u32(sX + xs * CF::kXBytes + sub * CF::kXAtom), 16, 1024);
+#pragma unroll
+            for (int k = 0; k < DK / 16; ++k)
+              tc_mma_f16(d_tmem, da + (uint64_t)(2 * k), db + (uint64_t)(2 * k), idesc, (j != i) || sub != 0 || k != 0);
+          }
           tc_commit(&empty[stage]);
           tc_commit(&xempty[xs]);
           if (++stage == S) { stage = 0; phase ^= 1; }
@@ -679,14 +693,14 @@ e3_status dec_launch_epi(const DecMaps &m, const DecArgs &a, int grid, int csk, 
 int dec_tiles(int N, int epi) { return epi == E3_DEC_SWIGLU ? N / 64 : (N + DM - 1) / DM; }
 
 static int dec_grid(int N, int K, int epi, int sms) {
-  const long total = (long)dec_tiles(N, epi) * (K / DK);
+  const long total = (long)dec_tiles(N, epi) * (K / DKS);
   return (int)(total < sms ? total : sms);
 }
 
 int dec_max_contrib(int N, int K, int epi, int sms) {
   // every CTA's range holds >= floor(total / G) iterations, so a tile of nkb
   // iterations meets at most ceil(nkb / that) + 1 ranges
-  const long nkb = K / DK, total = (long)dec_tiles(N, epi) * nkb;
+  const long nkb = K / DKS, total = (long)dec_tiles(N, epi) * nkb;
   const long G = dec_grid(N, K, epi, sms);
   const long per = total / G;
   return (int)((nkb + per - 1) / per + 1);
@@ -710,7 +724,7 @@ static int dec_csk(const DecArgs &a, int sms) {
   const int tiles = dec_tiles(a.N, a.epi);
   const bool vec = a.ldo % 8 == 0 && a.N % 8 == 0 && (reinterpret_cast<uintptr_t>(a.Y) & 15) == 0 &&
                    (a.epi != E3_DEC_RESID || (reinterpret_cast<uintptr_t>(a.R) & 15) == 0);
-  return (vec && 4 * tiles <= sms && a.K / DK >= 4) ? 4 : 1;
+  return (vec && 4 * tiles <= sms && a.K / DKS >= 4) ? 4 : 1;
 }
 
 e3_status dec_run(const DecMaps &m, const DecArgs &a_in, int sms, cudaStream_t st) {

@@ -116,11 +116,11 @@ static e3_status llama_validate(const e3_split_desc *d, const e3_weights *w) {
     return E3_EUNSUPPORTED;
   }
   const int kvh = d->kv_heads > 0 ? d->kv_heads : d->heads;
-  if (d->heads <= 0 || d->hidden != d->heads * 128 || d->heads % kvh || d->seq_len != 1 || d->ffn % 64 ||
+  if (d->heads <= 0 || d->hidden != d->heads * 128 || d->heads % kvh || d->seq_len != 1 || d->ffn % 128 ||
       d->ffn <= 0 || (d->batch != 32 && d->batch != 64 && d->batch != 128) || d->num_labels < 1 ||
       d->hidden > 8192) {
     set_error("e3_split_create (LLAMA): need head_dim 128 (H = 128 * heads), heads % kv_heads == 0, S == 1, "
-              "F % 64 == 0, B in {32, 64, 128}, H <= 8192");
+              "F % 128 == 0, B in {32, 64, 128}, H <= 8192");
     return E3_EUNSUPPORTED;
   }
   E3_CHECK_ARG(d->layer_begin >= 0 && d->layer_end > d->layer_begin && d->layer_end <= w->n_layers,
@@ -774,9 +774,9 @@ e3_status e3_op_dec_gemm(void *stream, const void *X, int32_t T, const void *W, 
   E3_CHECK_ARG(epilogue >= 0 && epilogue <= 2, "bad epilogue");
   E3_CHECK_ARG(epilogue != 1 || R, "residual epilogue needs R");
   E3_CHECK_ARG(epilogue != 2 || W2, "SwiGLU epilogue needs W2");
-  if ((T != 32 && T != 64 && T != 128) || K % 64 || (epilogue == 2 && N % 64) || !aligned16(X) || !aligned16(W) ||
+  if ((T != 32 && T != 64 && T != 128) || K % 128 || (epilogue == 2 && N % 64) || !aligned16(X) || !aligned16(W) ||
       (W2 && !aligned16(W2))) {
-    set_error("e3_op_dec_gemm: need T in {32,64,128}, K % 64 == 0, SwiGLU N % 64 == 0, aligned operands");
+    set_error("e3_op_dec_gemm: need T in {32,64,128}, K % 128 == 0, SwiGLU N % 64 == 0, aligned operands");
     return E3_EUNSUPPORTED;
   }
   int dev = 0;
