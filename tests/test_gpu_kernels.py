@@ -255,11 +255,15 @@ def test_vit_ramp_matches_oracle(api, base, test, C):
     assert int(ex2.n_exit.item()) == nv and int(alive2.sum()) == 0
 
 
-@pytest.mark.parametrize("T,N,K", [(32, 256, 128), (64, 1280, 4096), (128, 384, 640), (64, 4096, 11008)])
+@pytest.mark.parametrize("T,N,K", [(32, 256, 128), (64, 1280, 4096), (128, 384, 640), (64, 4096, 11008),
+                                   (64, 6144, 1024)])
 @pytest.mark.parametrize("epi", ["store", "resid", "swiglu"])
 def test_dec_gemm_matches_definition(api, T, N, K, epi):
-    """Decode GEMM (swap-AB tcgen05, stream-K with tiles shared between CTAs):
-    Y = X W^T (+ R) or SiLU(X Wg^T) * (X Wu^T), one bf16 rounding."""
+    """Decode GEMM (swap-AB tcgen05): Y = X W^T (+ R) or SiLU(X Wg^T) *
+    (X Wu^T), one bf16 rounding.  Store / residual GEMMs of <= 37 tiles take
+    the cluster split-K path (4 CTAs per tile, DSMEM reduction); N = 6144
+    (48 tiles) and every SwiGLU case take stream-K (tiles shared between CTAs,
+    global partials and tickets)."""
     from oracle.llama import silu
     rng = np.random.default_rng(T + N + K)
     X = rand_bf16(rng, (T, K))
