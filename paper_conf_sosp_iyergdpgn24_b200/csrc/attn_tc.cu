@@ -30,7 +30,16 @@ namespace {
 
 constexpr int D = 64;          // head dim
 constexpr int QT = 128;        // query rows per item
-constexpr int kThreads = 256;  // 8 warps: two threads per query row
+// KP threads per query row (warps w, w+4, ... own TMEM lane quarter w % 4 and
+// one of KP key ranges): 2 for S <= 128 (256 threads, 2 CTAs per SM), 4 above
+// (512 threads, one CTA per SM: each thread keeps its <= 64 scores in
+// registers instead of re-reading TMEM, and twice the warps hide the MUFU
+// and TMEM latencies)
+template <int SKV>
+struct AThr {
+  static constexpr int KP = SKV <= 128 ? 2 : 4;
+  static constexpr int kThreads = 128 * KP;
+};
 
 // SKV = keys per tile: S rounded up to 128 or, above 128, to a multiple of 32
 // (S = 197 -> 224: 12 % fewer masked exponentials than 256 and small enough
@@ -42,7 +51,7 @@ struct ACfg {
   static constexpr int kP = ((SKV + 63) / 64) * QT * 128;   // bf16 P in 64-key SW128 blocks
   static constexpr int kBuf = kQ + 2 * kKV;              // Q | K | V
   static constexpr bool kPInQK = (kP <= kQ + kKV);       // P overwrites the dead Q|K tiles
-  static constexpr int kExtra = 1024 + 64 + 2 * 2 * QT * 4;
+  static constexpr int kExtra = 1024 + 64 + 2 * 2 * AThr<SKV>::KP * QT * 4;
 #ifdef E3_ATTN_SINGLE_BUF   // diagnostics: occupancy instead of double buffering
   static constexpr int kNBuf = 1;
 #else
@@ -68,16 +77,18 @@ __device__ __forceinline__ void atrace(int j, int kind) {
 // kMask: S < SKV, keys >= S are masked; without it (S == SKV, BB) the
 // softmax loops carry no per-element compare / select
 template <int SKV, bool kMask>
-__global__ void __launch_bounds__(kThreads, SKV == 128 ? 2 : 1)
+__global__ void __launch_bounds__(AThr<SKV>::kThreads, SKV == 128 ? 2 : 1)
     attn_tc_kernel(const __grid_constant__ CUtensorMap tq, const __grid_constant__ CUtensorMap tkv,
                    const __grid_constant__ CUtensorMap tctx, int S, int H, int heads, int n_items) {
   using CF = ACfg<SKV>;
-  constexpr int NCH = SKV / 32;     // 32-key chunks; thread half 0 takes the first ceil(NCH/2)
+  constexpr int KP = AThr<SKV>::KP;
+  constexpr int NCH = SKV / 32;     // 32-key chunks; key part p takes chunks [p NCHP, (p + 1) NCHP)
+  constexpr int NCHP = (NCH + KP - 1) / KP;
   extern __shared__ uint8_t smem_raw[];
   uint8_t *smem = reinterpret_cast<uint8_t *>((reinterpret_cast<uintptr_t>(smem_raw) + 1023) & ~uintptr_t(1023));
   uint8_t *pbuf_sep = smem + CF::kNBuf * CF::kBuf;      // only when !kPInQK
-  float *xch = reinterpret_cast<float *>(smem + CF::kNBuf * CF::kBuf + (CF::kPInQK ? 0 : CF::kP));  // [2][2][QT]
-  uint64_t *bars = reinterpret_cast<uint64_t *>(xch + 2 * 2 * QT);
+  float *xch = reinterpret_cast<float *>(smem + CF::kNBuf * CF::kBuf + (CF::kPInQK ? 0 : CF::kP));  // [2][2][KP][QT]
+  uint64_t *bars = reinterpret_cast<uint64_t *>(xch + 2 * 2 * KP * QT);
   uint64_t *bar_load = bars;        // [2]
   uint64_t *bar_s = bars + 2;
   uint64_t *bar_o = bars + 3;
@@ -88,7 +99,7 @@ __global__ void __launch_bounds__(kThreads, SKV == 128 ? 2 : 1)
   const unsigned long long tl0 = tl_now();
   const int qtiles = (S + QT - 1) / QT;
   const int quarter = warp & 3;
-  const int khalf = warp >> 2;                            // which half of the keys / of D
+  const int khalf = warp >> 2;                            // which key part (and, for parts 0-1, half of D)
   const int row = quarter * 32 + lane;                    // query row within tile == TMEM lane
   const uint32_t lane_off = (uint32_t)(quarter * 32) << 16;
   const float sl2 = 1.4426950408889634f * 0.125f;         // log2(e) / sqrt(64)
@@ -166,10 +177,10 @@ __global__ void __launch_bounds__(kThreads, SKV == 128 ? 2 : 1)
     // S = 128: S is read from TMEM once, this thread's 64 keys stay in
     // registers between the max pass and the exponentiation pass (-6 %);
     // longer rows would spill, so they are read twice
-    constexpr int NCH0 = (NCH + 1) / 2;                   // chunks of thread half 0 (half 1: NCH / 2)
-    constexpr bool kKeep = NCH0 <= 2;                     // S = 128: 64 registers; longer rows reload
-    const int c_begin = khalf ? NCH0 * 32 : 0;
-    const int nch = khalf ? NCH / 2 : NCH0;
+    constexpr int NCH0 = NCHP;                            // chunks per key part (the last may have fewer)
+    constexpr bool kKeep = NCH0 <= 2;                     // <= 64 registers; longer rows reload
+    const int c_begin = khalf * NCH0 * 32;
+    const int nch = min(NCH0, NCH - khalf * NCH0);
     float sv[kKeep ? NCH0 * 32 : 32];
     float mx = -INFINITY;
 #pragma unroll
@@ -189,13 +200,13 @@ __global__ void __launch_bounds__(kThreads, SKV == 128 ? 2 : 1)
         mx = fmaxf(mx, fmaxf(fmaxf(m4[0], m4[1]), fmaxf(m4[2], m4[3])));
       }
     }
-    float *xmax = xch + (j & 1) * 2 * QT;                  // double-buffered exchange slots
-    float *xsum = xmax + QT;
-    if (khalf == 1) xmax[row] = mx;
+    float *xmax = xch + (j & 1) * 2 * KP * QT;             // double-buffered exchange slots [KP][QT]
+    float *xsum = xmax + KP * QT;
+    xmax[khalf * QT + row] = mx;
     __syncthreads();
-    if (khalf == 0) xmax[row] = mx = fmaxf(mx, xmax[row]);
-    __syncthreads();
-    if (khalf == 1) mx = xmax[row];
+    mx = xmax[row];
+#pragma unroll
+    for (int q = 1; q < KP; ++q) mx = fmaxf(mx, xmax[q * QT + row]);
     const float mb = mx * sl2;
     float l4[4] = {0.f, 0.f, 0.f, 0.f};
     uint8_t *prow = sP + row * 128;
@@ -249,12 +260,10 @@ __global__ void __launch_bounds__(kThreads, SKV == 128 ? 2 : 1)
       }
     }
     const float lpart = (l4[0] + l4[1]) + (l4[2] + l4[3]);
-    if (khalf == 1) xsum[row] = lpart;
+    xsum[khalf * QT + row] = lpart;
     fence_proxy_async_smem();     // generic-proxy smem writes -> visible to the tensor core
     tc_fence_before();            // S fully read before MMA2 overwrites it with O
     __syncthreads();
-    const float l = (khalf == 0) ? lpart + xsum[row] : 0.f;
-    if (khalf == 0) xsum[row] = l;
 
     if (tid == 0) {
       tc_fence_after();
@@ -273,9 +282,11 @@ __global__ void __launch_bounds__(kThreads, SKV == 128 ? 2 : 1)
     ophase ^= 1;
     tc_fence_after();
     if (tid == 0) atrace(j, 3);
-    __syncthreads();              // xsum[row] written by the khalf-0 thread
-    const float inv_l = 1.0f / xsum[row];
-    {
+    float l = xsum[row];          // key parts summed in order (written before the last barrier)
+#pragma unroll
+    for (int q = 1; q < KP; ++q) l += xsum[q * QT + row];
+    const float inv_l = 1.0f / l;
+    if (khalf < 2) {              // parts 0 and 1 write the 2 x 32 output columns
       uint32_t r[32];
       tmem_ld32(tbase + lane_off + khalf * 32, r);        // this thread's 32 of the 64 d columns
       tmem_wait_ld();
@@ -327,7 +338,7 @@ e3_status launch_attn(const AttnMaps &m, int B, int S, int H, int heads, cudaStr
     // (ncu: block limit registers 2, shared memory 2; forced 2: 13.8 us)
     cudaFuncAttributes fa;
     E3_CUDA_TRY(cudaFuncGetAttributes(&fa, kern));
-    const int by_regs = 65536 / (fa.numRegs * kThreads);
+    const int by_regs = 65536 / (fa.numRegs * AThr<SKV>::kThreads);
     const int by_smem = 233472 / (ACfg<SKV>::kSmem + (int)fa.sharedSizeBytes + 1024);
     per_sm = by_regs < by_smem ? by_regs : by_smem;
     if (per_sm < 1) per_sm = 1;
@@ -337,7 +348,7 @@ e3_status launch_attn(const AttnMaps &m, int B, int S, int H, int heads, cudaStr
   }
   const int n_items = B * heads * ((S + QT - 1) / QT);
   const int grid = n_items < per_sm * sms ? n_items : per_sm * sms;
-  E3_CUDA_TRY(launch_k(kern, dim3(grid), dim3(kThreads), ACfg<SKV>::kSmem, st, m.q, m.kv, m.ctx, S, H, heads,
+  E3_CUDA_TRY(launch_k(kern, dim3(grid), dim3(AThr<SKV>::kThreads), ACfg<SKV>::kSmem, st, m.q, m.kv, m.ctx, S, H, heads,
                        n_items));
   E3_CUDA_TRY(cudaGetLastError());
   count_launch();
