@@ -180,7 +180,11 @@ __global__ void __launch_bounds__(AThr<SKV>::kThreads, SKV == 128 ? 2 : 1)
     constexpr int NCH0 = NCHP;                            // chunks per key part (the last may have fewer)
     constexpr bool kKeep = NCH0 <= 2;                     // <= 64 registers; longer rows reload
     const int c_begin = khalf * NCH0 * 32;
-    const int nch = min(NCH0, NCH - khalf * NCH0);
+    // a lane quarter whose 32 query rows all lie past S (the second query
+    // tile of S = 197) skips its softmax and output: those rows are never
+    // stored, and P / O rows are independent in both MMAs
+    const bool qvalid = !kMask || q0 + quarter * 32 < S;
+    const int nch = qvalid ? min(NCH0, NCH - khalf * NCH0) : 0;
     float sv[kKeep ? NCH0 * 32 : 32];
     float mx = -INFINITY;
 #pragma unroll
@@ -286,7 +290,7 @@ __global__ void __launch_bounds__(AThr<SKV>::kThreads, SKV == 128 ? 2 : 1)
 #pragma unroll
     for (int q = 1; q < KP; ++q) l += xsum[q * QT + row];
     const float inv_l = 1.0f / l;
-    if (khalf < 2) {              // parts 0 and 1 write the 2 x 32 output columns
+    if (khalf < 2 && qvalid) {    // parts 0 and 1 write the 2 x 32 output columns
       uint32_t r[32];
       tmem_ld32(tbase + lane_off + khalf * 32, r);        // this thread's 32 of the 64 d columns
       tmem_wait_ld();
