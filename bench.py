@@ -61,6 +61,8 @@ def parse():
                     help="N>1: replicas of the whole chain, or stages on different GPUs (parallel.py)")
     ap.add_argument("--chunk", type=int, default=1024, help="stage mode: inputs per chunk")
     ap.add_argument("--stages", type=int, default=2, help="stage mode: number of stages")
+    ap.add_argument("--planner", default="balance", choices=["balance", "dp"],
+                    help="stage mode: survival-balanced cuts, or the profile-driven DP (planner.py)")
     return ap.parse_args()
 
 
@@ -250,8 +252,16 @@ def main():
         # stages on different GPUs: chunk c of the job enters at the stage-0
         # replica owning it; ids are global so exits land at their input's slot
         from paper_conf_sosp_iyergdpgn24_b200 import parallel as par
-        layout = par.plan_stages(cfg.ramp_layers, lambda l: survival(cfg, l), world,
-                                 n_stages=min(args.stages, world))
+        prof_path = os.path.join(ROOT, "profiles", f"r01_planner_profile_{args.config}.json")
+        if args.planner == "dp" and os.path.exists(prof_path):
+            # profile-driven DP (planner.py, NEXT-1) restricted to --stages stages
+            from paper_conf_sosp_iyergdpgn24_b200 import planner as pl
+            prof = pl.Profile.load(prof_path)
+            layout, _ = pl.plan_dp(cfg.ramp_layers, lambda l: survival(cfg, l), prof, world,
+                                   n_stages=min(args.stages, world))
+        else:
+            layout = par.plan_stages(cfg.ramp_layers, lambda l: survival(cfg, l), world,
+                                     n_stages=min(args.stages, world))
         g_stage, _ = layout.stage_of(rank)
         total = n * world
         n_chunks = (total + args.chunk - 1) // args.chunk
