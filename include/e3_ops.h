@@ -106,8 +106,14 @@ e3_status e3_debug_gemm_trace(void *dev_buf);
  * attention, LayerNorm, BERT ramp and fused LN + compaction kernels appends
  * {kernel id | blockIdx.x << 16, entry, released from griddepcontrol.wait,
  * end} globaltimer stamps (ns).  Kernel ids: 1000 + BN + epilogue (GEMM),
- * 2000 + key tile (attention), 3 LayerNorm, 4 ramp CTA, 5 ramp decision
- * CTA, 6 compaction.  Not thread-safe; E3_ECUDA if a symbol copy fails. */
+ * 2000 + key tile (+500 with the key mask; attention), 3 LayerNorm, 4 ramp
+ * CTA, 5 ramp decision CTA, 6 compaction, 7 fused O + LayerNorm, 9 ViT ramp,
+ * 8100 + epilogue decode GEMM; sub-phase records reuse the three stamps:
+ * 40 ramp (CLS ready, partials stored, synced), 41 ramp decision (synced,
+ * decided, recorded), 60 compaction scan done, 91 ViT ramp (LN done,
+ * classifier done, end), 8000 + epilogue decode GEMM (first / last
+ * accumulator ready, end), 8200 + epilogue stream-K tile reduction.  Not
+ * thread-safe; E3_ECUDA if a symbol copy fails. */
 e3_status e3_debug_timeline(void *dev_buf);
 
 #ifdef __cplusplus
