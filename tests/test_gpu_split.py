@@ -408,3 +408,36 @@ def test_vit_base_pipeline_full_size_sampled(api, vit_base):
     sample = [int(i) for i in np.random.default_rng(2).choice(N, 3, replace=False)]
     recs = oracle.run(cfg, W, X[sample], ids=sample, tau=tau, mode="bf16")
     _compare_records(recs, ex, sample, cfg, E2E_MARGIN, E2E_LOGIT_TOL)
+
+
+def test_bert_base_batch_position_invariance_bitwise(api, bert_base):
+    """R8 batch invariance at the bench shape: a row's result does not depend
+    on its batch partners or its position in the batch.  The same 64 inputs
+    run as a 4-layer split (inner ramps exact) in two different orders give
+    bitwise-equal exit layers, labels, confidences, logits and survivor rows."""
+    cfg, tau, W, model = bert_base
+    B = cfg.batch
+    X = e3data.make_inputs(cfg, range(B))
+    perm = np.random.default_rng(5).permutation(B)
+    outs = []
+    for order in (np.arange(B), perm):
+        split = api.Split(model, api.split_desc(cfg, 0, 4, tau))
+        x = bf16_tensor(X[order])
+        ids = torch.from_numpy(order.astype(np.int64)).to(DEV)
+        x_out = torch.zeros_like(x)
+        id_out = torch.full((B,), -9, dtype=torch.int64, device=DEV)
+        n_surv = torch.zeros(1, dtype=torch.int32, device=DEV)
+        ex = api.ExitBuffers(B, cfg.classes, cfg.n_ramps, DEV)
+        split.run(x, ids, x_out, id_out, n_surv, ex)
+        torch.cuda.synchronize()
+        n = int(n_surv.item())
+        surv = {int(i): x_out[k].clone() for k, i in enumerate(id_out[:n].tolist())}
+        outs.append((ex.exit_layer.clone(), ex.label.clone(), ex.conf.clone(), ex.logits.clone(), surv))
+    a, b = outs
+    for t0, t1 in zip(a[:4], b[:4]):           # bit patterns (unset records hold NaN)
+        if t0.dtype == torch.float32:
+            t0, t1 = t0.view(torch.int32), t1.view(torch.int32)
+        assert torch.equal(t0, t1)
+    assert a[4].keys() == b[4].keys() and len(a[4]) > 0
+    for i in a[4]:
+        assert torch.equal(a[4][i].view(torch.int16), b[4][i].view(torch.int16))
