@@ -58,7 +58,11 @@ struct ACfg {
   static constexpr int kNBuf = (2 * kBuf + (kPInQK ? 0 : kP) + kExtra <= 232448) ? 2 : 1;   // double buffer if it fits
 #endif
   static constexpr int kSmem = kNBuf * kBuf + (kPInQK ? 0 : kP) + kExtra;
-  static constexpr int kTmemCols = SKV <= 128 ? 128 : 256;   // S, later O (64 columns)
+  static constexpr int kSCols = SKV <= 128 ? 128 : 256;      // one S (later O, 64 columns) accumulator
+  // above 128 keys (one CTA per SM) two accumulators: MMA1 of item j+1 runs
+  // while item j's output is written
+  static constexpr bool kPipe = SKV > 128 && kNBuf == 2;
+  static constexpr int kTmemCols = kPipe ? 2 * kSCols : kSCols;
 };
 
 // Diagnostics (e3_debug_gemm_trace): per CTA and item (<= 8), globaltimer
@@ -133,9 +137,26 @@ __global__ void __launch_bounds__(AThr<SKV>::kThreads, SKV == 128 ? 2 : 1)
     tma_load_3d(base + CF::kQ + CF::kKV, &tkv, &bar_load[buf], 2 * H + h * D, 0, b);
   };
 
+  uint32_t load_phases = 0;                               // bit i: parity of bar_load[i] (thread 0)
+  // S = Q K^T of the item in buffer `bf` into S accumulator `acc`
+  auto issue_mma1 = [&](int bf, int acc) {
+    mbar_wait(&bar_load[bf], (load_phases >> bf) & 1u);
+    load_phases ^= 1u << bf;
+    tc_fence_after();
+    uint8_t *q = smem + bf * CF::kBuf;
+    const uint32_t idesc = idesc_bf16_f32(QT, SKV, 0);
+    const uint64_t dq = smem_desc_sw128(smem_u32(q), 16, 1024);
+    const uint64_t dk = smem_desc_sw128(smem_u32(q + CF::kQ), 16, 1024);
+#pragma unroll
+    for (int k = 0; k < D / 16; ++k) tc_mma_f16(tbase + acc * CF::kSCols, dq + 2 * k, dk + 2 * k, idesc, k != 0);
+    tc_commit(bar_s);
+  };
+
   int item = blockIdx.x;
-  if (tid == 0 && item < n_items) issue_load(item, 0);
-  uint32_t load_phases = 0;                               // bit i: parity of bar_load[i]
+  if (tid == 0 && item < n_items) {
+    issue_load(item, 0);
+    if (CF::kPipe) issue_mma1(0, 0);
+  }
   uint32_t sphase = 0, ophase = 0;
 
   for (int j = 0; item < n_items; ++j, item += gridDim.x) {
@@ -149,16 +170,11 @@ __global__ void __launch_bounds__(AThr<SKV>::kThreads, SKV == 128 ? 2 : 1)
     const int q0 = qt * QT;
     const int next = item + gridDim.x;
 
+    const uint32_t tS = tbase + (CF::kPipe ? (j & 1) * CF::kSCols : 0);   // this item's S, later O
+    (void)sK;
     if (tid == 0) {
-      mbar_wait(&bar_load[buf], (load_phases >> buf) & 1u);
-      tc_fence_after();
+      if (!CF::kPipe) issue_mma1(buf, 0);               // kPipe: issued during the previous item
       atrace(j, 0);
-      const uint32_t idesc = idesc_bf16_f32(QT, SKV, 0);
-      const uint64_t dq = smem_desc_sw128(smem_u32(sQ), 16, 1024);
-      const uint64_t dk = smem_desc_sw128(smem_u32(sK), 16, 1024);
-#pragma unroll
-      for (int k = 0; k < D / 16; ++k) tc_mma_f16(tbase, dq + 2 * k, dk + 2 * k, idesc, k != 0);
-      tc_commit(bar_s);
       if (CF::kNBuf == 2 && next < n_items) {
         // the other buffer's last readers: MMA2 of item j-1 (done: waited before
         // its epilogue) and the TMA store of its output from the V tile
@@ -166,7 +182,6 @@ __global__ void __launch_bounds__(AThr<SKV>::kThreads, SKV == 128 ? 2 : 1)
         issue_load(next, buf ^ 1);
       }
     }
-    load_phases ^= 1u << buf;
     __syncwarp();
 
     // ------------------------------------------------------------ softmax
@@ -192,7 +207,7 @@ __global__ void __launch_bounds__(AThr<SKV>::kThreads, SKV == 128 ? 2 : 1)
       if (ci < nch) {
         const int c = c_begin + ci * 32;
         uint32_t r[32];
-        tmem_ld32(tbase + lane_off + c, r);
+        tmem_ld32(tS + lane_off + c, r);
         tmem_wait_ld();
         float m4[4] = {-INFINITY, -INFINITY, -INFINITY, -INFINITY};
 #pragma unroll
@@ -220,7 +235,7 @@ __global__ void __launch_bounds__(AThr<SKV>::kThreads, SKV == 128 ? 2 : 1)
         const int c = c_begin + ci * 32;
         if (!kKeep) {
           uint32_t r[32];
-          tmem_ld32(tbase + lane_off + c, r);
+          tmem_ld32(tS + lane_off + c, r);
           tmem_wait_ld();
 #pragma unroll
           for (int jj = 0; jj < 32; ++jj) sv[jj] = __uint_as_float(r[jj]);
@@ -277,9 +292,10 @@ __global__ void __launch_bounds__(AThr<SKV>::kThreads, SKV == 128 ? 2 : 1)
       for (int kk = 0; kk < SKV / 16; ++kk) {
         const uint64_t dp = smem_desc_sw128(smem_u32(sP + (kk / 4) * (QT * 128) + (kk % 4) * 32), 16, 1024);
         const uint64_t dv = smem_desc_sw128(smem_u32(sV + kk * 16 * 128), SKV * 128, 1024);
-        tc_mma_f16(tbase, dp, dv, idesc, kk != 0);
+        tc_mma_f16(tS, dp, dv, idesc, kk != 0);
       }
       tc_commit(bar_o);
+      if (CF::kPipe && next < n_items) issue_mma1(buf ^ 1, (j + 1) & 1);   // overlaps this item's output
     }
     __syncwarp();
     mbar_wait(bar_o, ophase);     // MMA2 done: V tile is dead -> output staging
@@ -292,7 +308,7 @@ __global__ void __launch_bounds__(AThr<SKV>::kThreads, SKV == 128 ? 2 : 1)
     const float inv_l = 1.0f / l;
     if (khalf < 2 && qvalid) {    // parts 0 and 1 write the 2 x 32 output columns
       uint32_t r[32];
-      tmem_ld32(tbase + lane_off + khalf * 32, r);        // this thread's 32 of the 64 d columns
+      tmem_ld32(tS + lane_off + khalf * 32, r);           // this thread's 32 of the 64 d columns
       tmem_wait_ld();
       uint8_t *orow = sV + row * 128;                     // [128 q x 128 B], 128B swizzle
 #pragma unroll
