@@ -210,11 +210,20 @@ __global__ void __launch_bounds__(AThr<SKV>::kThreads, SKV == 128 ? 2 : 1)
         tmem_ld32(tS + lane_off + c, r);
         tmem_wait_ld();
         float m4[4] = {-INFINITY, -INFINITY, -INFINITY, -INFINITY};
+        if (kMask && c + 32 > S) {        // the chunk holding key S: masked keys become -inf (p = 0)
 #pragma unroll
-        for (int jj = 0; jj < 32; ++jj) {
-          const float v = __uint_as_float(r[jj]);
-          if (kKeep) sv[ci * 32 + jj] = v;
-          if (!kMask || c + jj < S) m4[jj & 3] = fmaxf(m4[jj & 3], v);
+          for (int jj = 0; jj < 32; ++jj) {
+            const float v = (c + jj < S) ? __uint_as_float(r[jj]) : -INFINITY;
+            if (kKeep) sv[ci * 32 + jj] = v;
+            m4[jj & 3] = fmaxf(m4[jj & 3], v);
+          }
+        } else {                           // full chunks: no per-key test
+#pragma unroll
+          for (int jj = 0; jj < 32; ++jj) {
+            const float v = __uint_as_float(r[jj]);
+            if (kKeep) sv[ci * 32 + jj] = v;
+            m4[jj & 3] = fmaxf(m4[jj & 3], v);
+          }
         }
         mx = fmaxf(mx, fmaxf(fmaxf(m4[0], m4[1]), fmaxf(m4[2], m4[3])));
       }
@@ -252,7 +261,7 @@ __global__ void __launch_bounds__(AThr<SKV>::kThreads, SKV == 128 ? 2 : 1)
           p[jj + 1] = ex2_approx(t0.y);
           p[jj + 2] = ex2_approx(t1.x);
           p[jj + 3] = ex2_approx(t1.y);
-          if (kMask) {
+          if (kMask && !kKeep) {           // kept scores are already -inf past S
 #pragma unroll
             for (int e = 0; e < 4; ++e)
               if (c + jj + e >= S) p[jj + e] = 0.f;
