@@ -262,6 +262,61 @@ __global__ void __launch_bounds__(128) lm_decide_kernel(RampArgs a) {
 
 }  // namespace
 
+// One CTA (8 warps) per row for the decode batch's few long rows (T <= 128
+// rows of H = 4096): a warp per row left 64 rows on 8 SMs, each lane summing
+// and scaling 128 values in sequence.  Thread t owns the 16-byte vectors t,
+// t + 256, ...; the sum of squares is reduced per warp by shuffles, then over
+// the 8 warps in warp order (deterministic).
+template <int VPT>
+__global__ void __launch_bounds__(256) rmsnorm_cta_kernel(const __nv_bfloat16 *__restrict__ x,
+                                                          const __nv_bfloat16 *__restrict__ g,
+                                                          __nv_bfloat16 *__restrict__ y, int rows, int H, float eps) {
+  __shared__ float red[8];
+  const int row = blockIdx.x, t = threadIdx.x, warp = warp_id(), lane = lane_id();
+  const int nvec = H / 8;
+  uint4 gv[VPT];
+#pragma unroll
+  for (int i = 0; i < VPT; ++i) {
+    const int k = t + 256 * i;
+    gv[i] = (k < nvec) ? __ldg(reinterpret_cast<const uint4 *>(g) + k) : make_uint4(0, 0, 0, 0);
+  }
+  pdl_wait();
+  pdl_trigger();
+  if (row >= rows) return;
+  const uint4 *xr = reinterpret_cast<const uint4 *>(x + (size_t)row * H);
+  uint4 v[VPT];
+  float ss = 0.f;
+#pragma unroll
+  for (int i = 0; i < VPT; ++i) {
+    const int k = t + 256 * i;
+    v[i] = (k < nvec) ? xr[k] : make_uint4(0, 0, 0, 0);
+    const uint32_t w[4] = {v[i].x, v[i].y, v[i].z, v[i].w};
+#pragma unroll
+    for (int e = 0; e < 4; ++e) ss += bf_lo(w[e]) * bf_lo(w[e]) + bf_hi(w[e]) * bf_hi(w[e]);
+  }
+#pragma unroll
+  for (int o = 16; o; o >>= 1) ss += __shfl_xor_sync(0xffffffffu, ss, o);
+  if (lane == 0) red[warp] = ss;
+  __syncthreads();
+  float tot = red[0];
+#pragma unroll
+  for (int w = 1; w < 8; ++w) tot += red[w];
+  const float rinv = 1.0f / sqrtf(tot / (float)H + eps);
+  uint4 *yr = reinterpret_cast<uint4 *>(y + (size_t)row * H);
+#pragma unroll
+  for (int i = 0; i < VPT; ++i) {
+    const int k = t + 256 * i;
+    if (k >= nvec) continue;
+    const uint32_t w[4] = {v[i].x, v[i].y, v[i].z, v[i].w};
+    const uint32_t gw[4] = {gv[i].x, gv[i].y, gv[i].z, gv[i].w};
+    uint32_t o[4];
+#pragma unroll
+    for (int e = 0; e < 4; ++e)
+      o[e] = pack_bf16(bf_lo(w[e]) * rinv * bf_lo(gw[e]), bf_hi(w[e]) * rinv * bf_hi(gw[e]));
+    yr[k] = make_uint4(o[0], o[1], o[2], o[3]);
+  }
+}
+
 e3_status rmsnorm_run(const void *x, const void *g, void *y, int rows, int H, float eps, cudaStream_t st) {
   if (H % 8 || H > 8192) {
     set_error("rmsnorm: need H % 8 == 0, H <= 8192");
@@ -270,6 +325,14 @@ e3_status rmsnorm_run(const void *x, const void *g, void *y, int rows, int H, fl
   auto *xp = reinterpret_cast<const __nv_bfloat16 *>(x);
   auto *gp = reinterpret_cast<const __nv_bfloat16 *>(g);
   auto *yp = reinterpret_cast<__nv_bfloat16 *>(y);
+  if (H >= 2048 && rows <= 256) {      // few long rows: one CTA per row
+    const int vpt = (H / 8 + 255) / 256;
+    if (vpt <= 2) E3_CUDA_TRY(launch_k(rmsnorm_cta_kernel<2>, dim3(rows), dim3(256), 0, st, xp, gp, yp, rows, H, eps));
+    else E3_CUDA_TRY(launch_k(rmsnorm_cta_kernel<4>, dim3(rows), dim3(256), 0, st, xp, gp, yp, rows, H, eps));
+    E3_CUDA_TRY(cudaGetLastError());
+    count_launch();
+    return E3_OK;
+  }
   const dim3 grid((rows + 7) / 8);
   const int vpl = (H / 8 + 31) / 32;
   if (vpl <= 1) E3_CUDA_TRY(launch_k(rmsnorm_kernel<1>, grid, dim3(256), 0, st, xp, gp, yp, rows, H, eps));
