@@ -385,15 +385,19 @@ e3_status gemm_set_trace(void *buf) {
   return E3_OK;
 }
 
-int gemm_pick_bn(int M, int N, int sms) {
+int gemm_pick_bn(int M, int N, int sms, int epi) {
   // diagnostics: E3_GEMM_BN forces the N tile where it divides N
   static const int forced = [] {
     const char *e = getenv("E3_GEMM_BN");
     return e ? atoi(e) : 0;
   }();
   if (forced && N % forced == 0) return forced;
-  // Minimise waves x per-tile cost over the pair tiles (256 x BN); per-tile
-  // cost ~ BN + 32 (fixed prologue / epilogue overhead in column units).
+  // Minimise waves x per-tile cost over the pair tiles (256 x BN).  The
+  // mainloop is bound by the TMA fill of 256 A rows + BN W rows per K step,
+  // so a tile costs ~ 256 + BN; the GELU epilogue adds ~ BN / 2 (it is
+  // issue-bound beside the MMAs).  Measured (scripts/gemm_bn_sweep*.sh):
+  // BL N = 1024 FFN2 102 us at BN 256 vs 120 at the old BN + 32 model's 128;
+  // BB FFN1 + GELU 37.8 us at 192 vs 38.9 at 256.
   int best = 0;
   long best_cost = 0;
   const int cands[4] = {256, 192, 128, 64};
@@ -403,7 +407,7 @@ int gemm_pick_bn(int M, int N, int sms) {
     if (N % bn) continue;
     const long tiles = (long)((M + 2 * BM - 1) / (2 * BM)) * (N / bn);
     const long waves = (tiles + pairs - 1) / pairs;
-    const long cost = waves * (bn + 32);
+    const long cost = waves * (2 * (2 * BM + bn) + (epi == E3_EPI_BIAS_GELU ? bn : 0));
     if (best == 0 || cost < best_cost) { best = bn; best_cost = cost; }
   }
   return best;
