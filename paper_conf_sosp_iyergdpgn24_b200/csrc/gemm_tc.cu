@@ -73,13 +73,20 @@ struct Cfg {
   static constexpr bool kEarly = kNCW <= 2;              // whole share in registers, early release
   static constexpr int kThreads = 128 + 32 * kEpiWarps;  // 4 control warps + epilogue warps
   static constexpr int kEpiBytes = kEpiWarps * 2 * kEpiBuf;
+  // BN = 384 (a whole N = 768 GEMM in one wave of pair tiles): two N = 192
+  // MMAs per K step, one TMEM accumulator (no epilogue overlap: one tile per
+  // pair), 64-wide K stages so that four stages fit
+  static constexpr int kNMma = BN > 256 ? 2 : 1;       // MMAs per k16 step (N <= 256 each)
+  static constexpr int kNAcc = 2 * BN <= 512 ? 2 : 1;  // TMEM accumulators
+  static constexpr int kKsub = BN > 256 ? 1 : KSUB;    // swizzle atoms per stage
+  static constexpr int kBox = BN / (2 * kNMma);        // W rows per TMA box (one box per MMA per CTA)
   static constexpr int kASub = BM * BK * 2;            // 16 KB per swizzle atom column
   static constexpr int kBSub = (BN / 2) * BK * 2;      // this CTA's half of the W tile
-  static constexpr int kABytes = KSUB * kASub;
-  static constexpr int kBBytes = KSUB * kBSub;
+  static constexpr int kABytes = kKsub * kASub;
+  static constexpr int kBBytes = kKsub * kBSub;
   static constexpr int kStageBytes = kABytes + kBBytes;
   static constexpr int kStages = (kSmemMax - kEpiBytes - 1024 - 256) / kStageBytes;
-  static constexpr int kTmemCols = (2 * BN <= 128) ? 128 : (2 * BN <= 256) ? 256 : 512;
+  static constexpr int kTmemCols = (kNAcc * BN <= 128) ? 128 : (kNAcc * BN <= 256) ? 256 : 512;
   static constexpr int kSmem = kStages * kStageBytes + kEpiBytes + 1024 /*align*/ + 256 /*barriers*/;
 };
 
@@ -115,7 +122,7 @@ __global__ void __cluster_dims__(2, 1, 1) __launch_bounds__(Cfg<BN, EPI>::kThrea
   const int num_m = (M + 2 * BM - 1) / (2 * BM);
   const int num_n = N / BN;
   const int num_tiles = num_m * num_n;
-  const int num_kb = K / (BK * KSUB);
+  const int num_kb = K / (BK * CF::kKsub);
 
   if (warp == 0 && lane == 0) {
     tma_prefetch(&tmA);
@@ -149,16 +156,24 @@ __global__ void __cluster_dims__(2, 1, 1) __launch_bounds__(Cfg<BN, EPI>::kThrea
     if (lane == 0) {
       // the W boxes of the first S stages do not depend on the previous
       // kernel: issued before griddepcontrol.wait, so the weight fetch
-      // overlaps the hand-off; the A boxes of those stages follow the wait
+      // overlaps the hand-off; the A boxes of those stages follow the wait.
+      // W rows of CTA r for MMA m: [n0 + m * BN / kNMma + r * kBox, + kBox),
+      // so that D's columns map linearly onto the tile's N range
+      auto load_w = [&](int st, int t, int kb) {
+        const uint32_t fb = mapa_shared(smem_u32(&full[st]), 0);
+#pragma unroll
+        for (int ks = 0; ks < CF::kKsub; ++ks)
+#pragma unroll
+          for (int m = 0; m < CF::kNMma; ++m)
+            tma_load_2d_2sm(sB + st * CF::kBBytes + ks * CF::kBSub + m * CF::kBox * 128, &tmB, fb,
+                            (kb * CF::kKsub + ks) * BK,
+                            (t % num_n) * BN + m * (BN / CF::kNMma) + (int)rank * CF::kBox);
+      };
       int npre = 0;
       for (int t = pair; t < num_tiles && npre < S; t += num_pairs) {
-        const int bn = (t % num_n) * BN + (int)rank * (BN / 2);
         for (int kb = 0; kb < num_kb && npre < S; ++kb, ++npre) {
-          const uint32_t fb = mapa_shared(smem_u32(&full[npre]), 0);
           if (leader) mbar_expect_tx(&full[npre], 2 * CF::kStageBytes);
-#pragma unroll
-          for (int ks = 0; ks < KSUB; ++ks)
-            tma_load_2d_2sm(sB + npre * CF::kBBytes + ks * CF::kBSub, &tmB, fb, (kb * KSUB + ks) * BK, bn);
+          load_w(npre, t, kb);
         }
       }
       pdl_wait();
@@ -166,9 +181,8 @@ __global__ void __cluster_dims__(2, 1, 1) __launch_bounds__(Cfg<BN, EPI>::kThrea
       int stage = 0, it = 0;
       uint32_t phase = 0;
       for (int t = pair; t < num_tiles; t += num_pairs) {
-        const int m_blk = t / num_n, n_blk = t % num_n;
+        const int m_blk = t / num_n;
         const int am = m_blk * 2 * BM + (int)rank * BM;
-        const int bn = n_blk * BN + (int)rank * (BN / 2);
         for (int kb = 0; kb < num_kb; ++kb, ++it) {
           const uint32_t fb = mapa_shared(smem_u32(&full[stage]), 0);
           const bool pre = it < npre;
@@ -177,11 +191,9 @@ __global__ void __cluster_dims__(2, 1, 1) __launch_bounds__(Cfg<BN, EPI>::kThrea
             if (leader) mbar_expect_tx(&full[stage], 2 * CF::kStageBytes);
           }
 #pragma unroll
-          for (int ks = 0; ks < KSUB; ++ks) {
-            const int k0 = (kb * KSUB + ks) * BK;
-            tma_load_2d_2sm(sA + stage * CF::kABytes + ks * CF::kASub, &tmA, fb, k0, am);
-            if (!pre) tma_load_2d_2sm(sB + stage * CF::kBBytes + ks * CF::kBSub, &tmB, fb, k0, bn);
-          }
+          for (int ks = 0; ks < CF::kKsub; ++ks)
+            tma_load_2d_2sm(sA + stage * CF::kABytes + ks * CF::kASub, &tmA, fb, (kb * CF::kKsub + ks) * BK, am);
+          if (!pre) load_w(stage, t, kb);
           if (++stage == S) { stage = 0; phase ^= 1; }
         }
       }
@@ -192,7 +204,7 @@ __global__ void __cluster_dims__(2, 1, 1) __launch_bounds__(Cfg<BN, EPI>::kThrea
   } else if (warp == 1) {
     // ------------------------------------------------ MMA issuer (leader, one thread)
     if (leader && lane == 0) {
-      constexpr uint32_t idesc = idesc_bf16_f32(2 * BM, BN, 0);
+      constexpr uint32_t idesc = idesc_bf16_f32(2 * BM, BN / CF::kNMma, 0);
       int stage = 0;
       uint32_t phase = 0;
       int acc = 0;
@@ -207,19 +219,24 @@ __global__ void __cluster_dims__(2, 1, 1) __launch_bounds__(Cfg<BN, EPI>::kThrea
           mbar_wait(&full[stage], phase);
           tc_fence_after();
 #pragma unroll
-          for (int ks = 0; ks < KSUB; ++ks) {
+          for (int ks = 0; ks < CF::kKsub; ++ks) {
             const uint64_t da = smem_desc_sw128(smem_u32(sA + stage * CF::kABytes + ks * CF::kASub), 16, 1024);
-            const uint64_t db = smem_desc_sw128(smem_u32(sB + stage * CF::kBBytes + ks * CF::kBSub), 16, 1024);
 #pragma unroll
-            for (int k = 0; k < BK / 16; ++k)   // +32 bytes per 16-element K step inside the swizzle atom
-              tc_mma2_f16(d_tmem, da + (uint64_t)(2 * k), db + (uint64_t)(2 * k), idesc, (kb | ks | k) != 0);
+            for (int m = 0; m < CF::kNMma; ++m) {
+              const uint64_t db =
+                  smem_desc_sw128(smem_u32(sB + stage * CF::kBBytes + ks * CF::kBSub + m * CF::kBox * 128), 16, 1024);
+#pragma unroll
+              for (int k = 0; k < BK / 16; ++k)   // +32 bytes per 16-element K step inside the swizzle atom
+                tc_mma2_f16(d_tmem + m * (BN / CF::kNMma), da + (uint64_t)(2 * k), db + (uint64_t)(2 * k), idesc,
+                            (kb | ks | k) != 0);
+            }
           }
           tc_commit2_mc(&empty[stage], 0x3);
           if (++stage == S) { stage = 0; phase ^= 1; }
         }
         tc_commit2_mc(&tfull[acc], 0x3);
         trace(tl, 1);
-        if (++acc == 2) { acc = 0; acc_phase ^= 1; }
+        if (++acc == CF::kNAcc) { acc = 0; acc_phase ^= 1; }
       }
     }
   } else if (warp >= 4) {
@@ -335,7 +352,7 @@ __global__ void __cluster_dims__(2, 1, 1) __launch_bounds__(Cfg<BN, EPI>::kThrea
         if (lane == 0) mbar_arrive_cluster(acc ? tempty_leader1 : tempty_leader0);
       }
       if (lane == 0 && (warp == 4 || warp == 11)) trace(tl, warp == 4 ? 3 : 5);
-      if (++acc == 2) { acc = 0; acc_phase ^= 1; }
+      if (++acc == CF::kNAcc) { acc = 0; acc_phase ^= 1; }
     }
     if (lane == 0) bulk_wait<0>();
   }
@@ -367,6 +384,12 @@ e3_status launch(const GemmMaps &g, const __nv_bfloat16 *bias, const __nv_bfloat
 template <int BN>
 e3_status launch_epi(int epi, const GemmMaps &g, const __nv_bfloat16 *bias, const __nv_bfloat16 *R, int M, int N,
                      int K, int sms, cudaStream_t st) {
+  if (BN > 256) {   // 384: bias / residual epilogues only
+    if (epi == E3_EPI_BIAS) return launch<(BN > 256 ? BN : 384), E3_EPI_BIAS>(g, bias, R, M, N, K, sms, st);
+    if (epi == E3_EPI_BIAS_RESID) return launch<(BN > 256 ? BN : 384), E3_EPI_BIAS_RESID>(g, bias, R, M, N, K, sms, st);
+    set_error("GEMM: N tile 384 has no GELU epilogue");
+    return E3_EUNSUPPORTED;
+  }
   switch (epi) {
     case E3_EPI_BIAS: return launch<BN, E3_EPI_BIAS>(g, bias, R, M, N, K, sms, st);
     case E3_EPI_BIAS_GELU: return launch<BN, E3_EPI_BIAS_GELU>(g, bias, R, M, N, K, sms, st);
@@ -385,29 +408,33 @@ e3_status gemm_set_trace(void *buf) {
   return E3_OK;
 }
 
-int gemm_pick_bn(int M, int N, int sms, int epi) {
+int gemm_pick_bn(int M, int N, int K, int sms, int epi) {
   // diagnostics: E3_GEMM_BN forces the N tile where it divides N
   static const int forced = [] {
     const char *e = getenv("E3_GEMM_BN");
     return e ? atoi(e) : 0;
   }();
   if (forced && N % forced == 0) return forced;
-  // Minimise waves x per-tile cost over the pair tiles (256 x BN).  The
-  // mainloop is bound by the TMA fill of 256 A rows + BN W rows per K step,
-  // so a tile costs ~ 256 + BN; the GELU epilogue adds ~ BN / 2 (it is
-  // issue-bound beside the MMAs).  Measured (scripts/gemm_bn_sweep*.sh):
-  // BL N = 1024 FFN2 102 us at BN 256 vs 120 at the old BN + 32 model's 128;
-  // BB FFN1 + GELU 37.8 us at 192 vs 38.9 at 256.
+  // Minimise waves x per-tile cost over the pair tiles (256 x BN), in units
+  // of one row of TMA fill per K element: the mainloop moves 256 + BN rows per
+  // K step (it is fill-bound), the issue-bound GELU epilogue adds ~ BN / 2 per
+  // K step, and BN = 384 (one TMEM accumulator: nothing to overlap its
+  // epilogue with) pays ~ 1720 x BN for the exposed epilogue.  Calibrated on
+  // scripts/gemm_bn_sweep*.sh: BL N = 1024 FFN2 102 us at BN 256 (120 at 128);
+  // BB FFN1 + GELU 37.8 us at 192 (38.9 at 256); BB FFN2 (K = 3072) 31.6 us
+  // at 384 (33.0 at 192) but BB O (K = 768) 14.1 us at 192 (14.8 at 384).
   int best = 0;
-  long best_cost = 0;
-  const int cands[4] = {256, 192, 128, 64};
+  long long best_cost = 0;
+  const int cands[5] = {384, 256, 192, 128, 64};
   const int pairs = sms / 2;
-  for (int i = 0; i < 4; ++i) {
+  for (int i = 0; i < 5; ++i) {
     const int bn = cands[i];
-    if (N % bn) continue;
-    const long tiles = (long)((M + 2 * BM - 1) / (2 * BM)) * (N / bn);
-    const long waves = (tiles + pairs - 1) / pairs;
-    const long cost = waves * (2 * (2 * BM + bn) + (epi == E3_EPI_BIAS_GELU ? bn : 0));
+    if (N % bn || (bn == 384 && epi == E3_EPI_BIAS_GELU)) continue;
+    const long long tiles = (long long)((M + 2 * BM - 1) / (2 * BM)) * (N / bn);
+    const long long waves = (tiles + pairs - 1) / pairs;
+    const long long tile = (long long)K * (2 * BM + bn) + (epi == E3_EPI_BIAS_GELU ? (long long)K * bn / 2 : 0) +
+                           (bn > 256 ? 1720LL * bn : 0);
+    const long long cost = waves * tile;
     if (best == 0 || cost < best_cost) { best = bn; best_cost = cost; }
   }
   return best;
@@ -416,7 +443,7 @@ int gemm_pick_bn(int M, int N, int sms, int epi) {
 e3_status gemm_tmaps(GemmMaps *g, const void *A, int64_t lda, const void *W, const void *C, int M, int N, int K,
                      int bn) {
   e3_status s = make_tmap_2d(&g->a, A, (uint64_t)M, (uint64_t)K, (uint64_t)lda, BM, BK);
-  if (s == E3_OK) s = make_tmap_2d(&g->b, W, (uint64_t)N, (uint64_t)K, (uint64_t)K, (uint32_t)(bn / 2), BK);
+  if (s == E3_OK) s = make_tmap_2d(&g->b, W, (uint64_t)N, (uint64_t)K, (uint64_t)K, (uint32_t)(bn > 256 ? bn / 4 : bn / 2), BK);
   if (s == E3_OK) s = make_tmap_2d_sw64(&g->c, C, (uint64_t)M, (uint64_t)N, (uint64_t)N, 32, 32);
   g->bn = bn;
   return s;
@@ -427,6 +454,7 @@ e3_status gemm_run(const GemmMaps &g, const void *bias, const void *R, int M, in
   auto *b = reinterpret_cast<const __nv_bfloat16 *>(bias);
   auto *r = reinterpret_cast<const __nv_bfloat16 *>(R);
   switch (g.bn) {
+    case 384: return launch_epi<384>(epi, g, b, r, M, N, K, sms, st);
     case 256: return launch_epi<256>(epi, g, b, r, M, N, K, sms, st);
     case 192: return launch_epi<192>(epi, g, b, r, M, N, K, sms, st);
     case 128: return launch_epi<128>(epi, g, b, r, M, N, K, sms, st);

@@ -17,7 +17,7 @@ struct GemmMaps {
   CUtensorMap c;   // C [M,N], box 32 x 32, 64-B swizzle (epilogue TMA store)
   int bn;
 };
-int gemm_pick_bn(int M, int N, int sms, int epi);
+int gemm_pick_bn(int M, int N, int K, int sms, int epi);
 e3_status gemm_set_trace(void *buf);   // diagnostics (e3_debug_gemm_trace)
 e3_status attn_set_trace(void *buf);   // diagnostics (e3_debug_gemm_trace)
 // diagnostics (e3_debug_timeline): per translation unit

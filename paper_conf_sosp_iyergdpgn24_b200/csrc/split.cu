@@ -297,10 +297,10 @@ e3_status split_create_shared(const e3_split_desc *d, const e3_weights *w, int d
     return E3_OK;
   }
   const int M = B * S;
-  s->bn_qkv = gemm_pick_bn(M, 3 * H, s->sms, E3_EPI_BIAS);
-  s->bn_o = gemm_pick_bn(M, H, s->sms, E3_EPI_BIAS_RESID);
-  s->bn_f1 = gemm_pick_bn(M, F, s->sms, E3_EPI_BIAS_GELU);
-  s->bn_f2 = gemm_pick_bn(M, H, s->sms, E3_EPI_BIAS_RESID);
+  s->bn_qkv = gemm_pick_bn(M, 3 * H, H, s->sms, E3_EPI_BIAS);
+  s->bn_o = gemm_pick_bn(M, H, H, s->sms, E3_EPI_BIAS_RESID);
+  s->bn_f1 = gemm_pick_bn(M, F, H, s->sms, E3_EPI_BIAS_GELU);
+  s->bn_f2 = gemm_pick_bn(M, H, F, s->sms, E3_EPI_BIAS_RESID);
   const int nl = d->layer_end - d->layer_begin;
   s->maps.resize(nl);
   const bool vit = d->arch == E3_ARCH_VIT;
@@ -747,7 +747,7 @@ e3_status e3_op_gemm(void *stream, const void *A, int64_t lda, const void *W, co
   E3_CUDA_TRY(cudaGetDevice(&dev));
   const int sms = num_sms(dev);
   GemmMaps g;
-  e3_status r = gemm_tmaps(&g, A, lda, W, C, M, N, K, gemm_pick_bn(M, N, sms, epilogue));
+  e3_status r = gemm_tmaps(&g, A, lda, W, C, M, N, K, gemm_pick_bn(M, N, K, sms, epilogue));
   if (r != E3_OK) return r;
   return gemm_run(g, bias, resid, M, N, K, epilogue, sms, reinterpret_cast<cudaStream_t>(stream));
 }
