@@ -101,6 +101,7 @@ __global__ void __launch_bounds__(AThr<SKV>::kThreads, SKV == 128 ? 2 : 1)
   const int warp = warp_id(), lane = lane_id();
   const int tid = threadIdx.x;
   const unsigned long long tl0 = tl_now();
+  unsigned long long *const tlb = g_tl;
   const int qtiles = (S + QT - 1) / QT;
   const int quarter = warp & 3;
   const int khalf = warp >> 2;                            // which key part (and, for parts 0-1, half of D)
@@ -346,7 +347,7 @@ __global__ void __launch_bounds__(AThr<SKV>::kThreads, SKV == 128 ? 2 : 1)
   if (tid == 0) bulk_wait<0>();
   __syncthreads();
   if (warp == 0) tmem_dealloc(tbase, CF::kTmemCols);
-  if (tid == 0) tl_rec(2000 + SKV + (kMask ? 500 : 0), tl0, tl1);
+  if (tid == 0) tl_rec(tlb, 2000 + SKV + (kMask ? 500 : 0), tl0, tl1);
 }
 
 template <int SKV, bool kMask>

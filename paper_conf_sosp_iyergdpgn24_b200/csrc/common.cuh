@@ -388,8 +388,9 @@ __device__ __forceinline__ unsigned long long tl_now() {
   asm volatile("mov.u64 %0, %globaltimer;" : "=l"(t));
   return t;
 }
-__device__ __forceinline__ void tl_rec(int kid, unsigned long long t0, unsigned long long t1) {
-  unsigned long long *b = g_tl;
+// b: g_tl read at kernel entry (a load at the CTA's last instruction would
+// hold its exit for an L2 round trip)
+__device__ __forceinline__ void tl_rec(unsigned long long *b, int kid, unsigned long long t0, unsigned long long t1) {
   if (!b) return;
   const unsigned long long t2 = tl_now();
   const unsigned long long i = atomicAdd(b, 1ull);

@@ -197,6 +197,7 @@ __global__ void __launch_bounds__(kThreads, VPL <= 3 ? 2 : 1)
   __shared__ int16_t pos_of[kMaxB];
   __shared__ int word_cnt[kMaxB / 32 + 1];
   const unsigned long long tl0 = tl_now();
+  unsigned long long *const tlb = g_tl;
   const int warp = warp_id(), lane = lane_id();
   LnParams<VPL> p;
   if (kLn) ln_load_params<VPL>(p, g, bb, H, lane);   // weights: before the dependency wait
@@ -222,7 +223,7 @@ __global__ void __launch_bounds__(kThreads, VPL <= 3 ? 2 : 1)
   }
   const int64_t tail = dst.tail_dev ? *dst.tail_dev : 0;
   const int n = block_scan_flags(alive, B, src_of, word_cnt, pos_of);
-  if (threadIdx.x == 0) tl_rec(60, tl1, tl1);   // scan done
+  if (threadIdx.x == 0) tl_rec(tlb, 60, tl1, tl1);   // scan done
   const bool fits = (tail - dst.head) + n <= dst.cap;
   if (blockIdx.x == 0 && threadIdx.x == 0) {
     const int out = fits ? n : 0;
@@ -232,7 +233,7 @@ __global__ void __launch_bounds__(kThreads, VPL <= 3 ? 2 : 1)
     if (dst.mailbox) *dst.mailbox = fits ? out : -1;   // read by the host after the run's event
   }
   if (!fits || n == 0) {
-    if (threadIdx.x == 0) tl_rec(6, tl0, tl1);
+    if (threadIdx.x == 0) tl_rec(tlb, 6, tl0, tl1);
     return;
   }
 
@@ -274,7 +275,7 @@ __global__ void __launch_bounds__(kThreads, VPL <= 3 ? 2 : 1)
   }
   if (blockIdx.x == 0)
     for (int k = threadIdx.x; k < n; k += kThreads) dst.ids[(tail + k) % dst.cap] = id[src_of[k]];
-  if (threadIdx.x == 0) tl_rec(6, tl0, tl1);
+  if (threadIdx.x == 0) tl_rec(tlb, 6, tl0, tl1);
 }
 
 }  // namespace

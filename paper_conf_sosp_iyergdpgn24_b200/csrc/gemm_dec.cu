@@ -104,6 +104,7 @@ __global__ void __launch_bounds__(kDThreads, 1)
   constexpr int S = CF::kStages;
   constexpr int P = T + 1;
   const unsigned long long tl0 = tl_now();
+  unsigned long long *const tlb = g_tl;
   extern __shared__ uint8_t smem_raw[];
   uint8_t *smem = reinterpret_cast<uint8_t *>((reinterpret_cast<uintptr_t>(smem_raw) + 1023) & ~uintptr_t(1023));
   constexpr int XS = CF::kXStages;
@@ -380,7 +381,7 @@ __global__ void __launch_bounds__(kDThreads, 1)
           }
         }
         epi_bar();
-        if (threadIdx.x == 64) tl_rec(8200 + EPI, tlr0, tlr0);   // reduction: start, end
+        if (threadIdx.x == 64) tl_rec(tlb, 8200 + EPI, tlr0, tlr0);   // reduction: start, end
       }
 
       // ---------------------------------------------------- final epilogue
@@ -576,8 +577,8 @@ __global__ void __launch_bounds__(kDThreads, 1)
       epi_bar();                        // sE is reused by the next unit
     }
     if (threadIdx.x == 64) {
-      tl_rec(8100 + EPI, tl0, tl1);
-      tl_rec(8000 + EPI, tlf, tlm);
+      tl_rec(tlb, 8100 + EPI, tl0, tl1);
+      tl_rec(tlb, 8000 + EPI, tlf, tlm);
     }
   }
   if (CSK > 1) {

@@ -62,6 +62,7 @@ __global__ void __cluster_dims__(2, 1, 1) __launch_bounds__(kLThreads, 1)
   using CF = LCfg<NH>;
   constexpr int S = CF::kStages;
   const unsigned long long tl0 = tl_now();
+  unsigned long long *const tlb = g_tl;
   extern __shared__ uint8_t smem_raw[];
   uint8_t *smem = reinterpret_cast<uint8_t *>((reinterpret_cast<uintptr_t>(smem_raw) + 1023) & ~uintptr_t(1023));
   uint8_t *sA = smem;
@@ -290,7 +291,7 @@ __global__ void __cluster_dims__(2, 1, 1) __launch_bounds__(kLThreads, 1)
   __syncthreads();
   tc_fence_after();
   if (warp == 2) tmem_dealloc(tmem_base, CF::kTmem);
-  if (threadIdx.x == 0) tl_rec(7, tl0, tl0);
+  if (threadIdx.x == 0) tl_rec(tlb, 7, tl0, tl0);
 }
 
 template <int NH>

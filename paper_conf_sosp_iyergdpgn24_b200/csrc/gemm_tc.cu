@@ -101,6 +101,7 @@ __global__ void __cluster_dims__(2, 1, 1) __launch_bounds__(Cfg<BN, EPI>::kThrea
   using CF = Cfg<BN, EPI>;
   constexpr int S = CF::kStages;
   const unsigned long long tl0 = tl_now();
+  unsigned long long *const tlb = g_tl;
   extern __shared__ uint8_t smem_raw[];
   // identical layout (same offsets) in both CTAs of the pair
   uint8_t *smem = reinterpret_cast<uint8_t *>((reinterpret_cast<uintptr_t>(smem_raw) + 1023) & ~uintptr_t(1023));
@@ -360,7 +361,7 @@ __global__ void __cluster_dims__(2, 1, 1) __launch_bounds__(Cfg<BN, EPI>::kThrea
   cluster_sync();                  // no CTA leaves while its peer may still signal it
   tc_fence_after();
   if (warp == 2) tmem_dealloc2(tmem_base, CF::kTmemCols);
-  if (threadIdx.x == 0) tl_rec(1000 + BN + EPI, tl0, tl1);
+  if (threadIdx.x == 0) tl_rec(tlb, 1000 + BN + EPI, tl0, tl1);
 }
 
 template <int BN, int EPI>

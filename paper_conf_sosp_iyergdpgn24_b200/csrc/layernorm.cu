@@ -22,6 +22,7 @@ __global__ void __launch_bounds__(256)
                      const __nv_bfloat16 *__restrict__ bb, __nv_bfloat16 *__restrict__ y, int rows, int H,
                      float eps) {
   const unsigned long long tl0 = tl_now();
+  unsigned long long *const tlb = g_tl;
   const int lane = lane_id();
   const int warps = gridDim.x * 8;
   const int row0 = blockIdx.x * 8 + warp_id();
@@ -48,7 +49,7 @@ __global__ void __launch_bounds__(256)
       }
     }
   }
-  if (threadIdx.x == 0) tl_rec(3, tl0, tl1);
+  if (threadIdx.x == 0) tl_rec(tlb, 3, tl0, tl1);
 }
 
 }  // namespace

@@ -94,6 +94,7 @@ __host__ __device__ inline int ramp_smem_bytes(int H, int C) {
 template <int VPL>
 __global__ void __launch_bounds__(kRThreads, 1) ramp_bert_kernel(RampArgs a) {
   const unsigned long long tl0 = tl_now();
+  unsigned long long *const tlb = g_tl;
   extern __shared__ uint8_t smem_raw[];
   constexpr int nw = kRThreads / 32;
   constexpr int kMaxNT = 2 * VPL;                        // TN / 8 <= H / 128
@@ -244,7 +245,7 @@ __global__ void __launch_bounds__(kRThreads, 1) ramp_bert_kernel(RampArgs a) {
   const unsigned long long tl3 = tl_now();
   cluster_sync();                  // every CTA's partials are in rank 0's smem
   const unsigned long long tlA = tl_now();
-  if (threadIdx.x == 0 && rank != 0) tl_rec(40, tl2, tl3);   // phases: CLS + W ready, partials stored, synced
+  if (threadIdx.x == 0 && rank != 0) tl_rec(tlb, 40, tl2, tl3);   // phases: CLS + W ready, partials stored, synced
   unsigned long long tlB = 0;
   // PDL trigger only once the decision is written (non-deciding CTAs trigger
   // by exiting): dependent CTAs made resident earlier sit in
@@ -252,7 +253,7 @@ __global__ void __launch_bounds__(kRThreads, 1) ramp_bert_kernel(RampArgs a) {
   // instructions from <1 to ~3 us (r01 timeline); before the pooler they cost
   // +6 us
   if (rank != 0 || warp != 0) {
-    if (threadIdx.x == 0) tl_rec(4, tl0, tl1);
+    if (threadIdx.x == 0) tl_rec(tlb, 4, tl0, tl1);
     return;
   }
 
@@ -318,8 +319,8 @@ __global__ void __launch_bounds__(kRThreads, 1) ramp_bert_kernel(RampArgs a) {
   }
   __syncwarp();
   pdl_trigger();
-  if (threadIdx.x == 0) tl_rec(5, tl0, tl1);   // rank 0: the decision is written
-  if (threadIdx.x == 0) tl_rec(41, tlA, tlB);
+  if (threadIdx.x == 0) tl_rec(tlb, 5, tl0, tl1);   // rank 0: the decision is written
+  if (threadIdx.x == 0) tl_rec(tlb, 41, tlA, tlB);
 }
 
 // ============================================================== ViT ramp
@@ -351,6 +352,7 @@ __device__ __forceinline__ int ld_cluster_s32(uint32_t addr) {
 template <int CB, bool kLate>
 __global__ void __launch_bounds__(kVitKQ * 2 * CB) ramp_vit_kernel(RampArgs a, int CS) {
   const unsigned long long tl0 = tl_now();
+  unsigned long long *const tlb = g_tl;
   // 8 threads per class for the classifier; the first 2 CB threads then own
   // 2 classes x 4 rows each for the softmax statistics and the logits
   constexpr int kThreads = 2 * CB, kWarps = kThreads / 32, kWarpsPerRg = CB / 64;
@@ -545,8 +547,8 @@ __global__ void __launch_bounds__(kVitKQ * 2 * CB) ramp_vit_kernel(RampArgs a, i
   }
   cluster_sync();                            // rank 0's smem stays valid until every CTA has read it
   if (kLate) pdl_trigger();
-  if (tAll == 0) tl_rec(9, tl0, tl1);
-  if (tAll == 0) tl_rec(91, tlLn, tlCls);   // phases: CLS LN done, classifier done, end
+  if (tAll == 0) tl_rec(tlb, 9, tl0, tl1);
+  if (tAll == 0) tl_rec(tlb, 91, tlLn, tlCls);   // phases: CLS LN done, classifier done, end
 }
 
 
@@ -577,6 +579,7 @@ __global__ void __launch_bounds__(kVtcThreads, 1) ramp_vit_tc_kernel(RampArgs a,
   constexpr int CB = 128, kThreads = 2 * CB, kWarps = kThreads / 32, kWarpsPerRg = CB / 64;
   static_assert(kThreads == kVtcThreads, "all threads own 2 classes x 4 rows");
   const unsigned long long tl0 = tl_now();
+  unsigned long long *const tlb = g_tl;
   extern __shared__ uint8_t smem_raw[];
   const int H = a.H, C = a.C, P = H + 8;
   __nv_bfloat16 *sA = reinterpret_cast<__nv_bfloat16 *>(smem_raw);   // [3][16][P]: hi, mid, lo
@@ -843,8 +846,8 @@ __global__ void __launch_bounds__(kVtcThreads, 1) ramp_vit_tc_kernel(RampArgs a,
   }
   cluster_sync();                            // rank 0's smem stays valid until every CTA has read it
   if (kLate) pdl_trigger();
-  if (tAll == 0) tl_rec(9, tl0, tl1);
-  if (tAll == 0) tl_rec(91, tlLn, tlCls);   // phases: CLS LN done, classifier done, end
+  if (tAll == 0) tl_rec(tlb, 9, tl0, tl1);
+  if (tAll == 0) tl_rec(tlb, 91, tlLn, tlCls);   // phases: CLS LN done, classifier done, end
 }
 
 
