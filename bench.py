@@ -258,10 +258,10 @@ def main():
             from paper_conf_sosp_iyergdpgn24_b200 import planner as pl
             prof = pl.Profile.load(prof_path)
             layout, _ = pl.plan_dp(cfg.ramp_layers, lambda l: survival(cfg, l), prof, world,
-                                   n_stages=min(args.stages, world))
+                                   n_stages=min(args.stages, world, cfg.n_ramps))
         else:
             layout = par.plan_stages(cfg.ramp_layers, lambda l: survival(cfg, l), world,
-                                     n_stages=min(args.stages, world))
+                                     n_stages=min(args.stages, world, cfg.n_ramps))
         g_stage, _ = layout.stage_of(rank)
         total = n * world
         n_chunks = (total + args.chunk - 1) // args.chunk

@@ -21,6 +21,7 @@ STATUS = {0: "E3_OK", 1: "E3_EINVAL", 2: "E3_EUNSUPPORTED", 3: "E3_ECUDA", 4: "E
 ARCH = {"bert": 0, "vit": 1, "llama": 2}
 TEST = {"maxprob": 0, "entropy": 1}
 INNER = {"exact": 0, "disabled": 1}
+DTYPE = {"bf16": 0, "fp32": 1}
 EPI = {"bias": 0, "bias_gelu": 1, "bias_resid": 2}
 
 P = C.c_void_p

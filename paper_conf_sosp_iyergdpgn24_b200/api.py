@@ -99,11 +99,12 @@ class KVCache:
 
 
 def split_desc(cfg, begin: int, end: int, tau, batch: Optional[int] = None,
-               inner: str = "exact") -> _lib.SplitDesc:
-    """e3_split_desc for layers [begin, end) of cfg (must end in a ramp)."""
+               inner: str = "exact", dtype: str = "bf16") -> _lib.SplitDesc:
+    """e3_split_desc for layers [begin, end) of cfg (must end in a ramp).
+    dtype: "bf16" (bf16 activations) or "fp32" (fp32 activations, E3_DTYPE_FP32)."""
     d = _lib.SplitDesc()
     d.arch = _lib.ARCH[cfg.arch]
-    d.dtype = 0
+    d.dtype = _lib.DTYPE[dtype]
     d.hidden, d.heads, d.kv_heads, d.ffn = cfg.hidden, cfg.heads, cfg.kv_heads, cfg.ffn
     d.seq_len, d.num_labels, d.ctx_len = cfg.seq, cfg.classes, cfg.ctx
     d.norm_eps = cfg.norm_eps
@@ -200,12 +201,12 @@ class Queue:
 
 
 def make_plan(cfg, bounds: Sequence[int], tau, batch=None, inner="exact", lag=1,
-              queue_cap_batches=4, trace=False) -> _lib.Plan:
+              queue_cap_batches=4, trace=False, dtype="bf16") -> _lib.Plan:
     """Plan with split s covering layers [bounds[s], bounds[s+1])."""
     p = _lib.Plan()
     p.n_splits = len(bounds) - 1
     for s in range(p.n_splits):
-        p.split[s] = split_desc(cfg, bounds[s], bounds[s + 1], tau, batch, inner)
+        p.split[s] = split_desc(cfg, bounds[s], bounds[s + 1], tau, batch, inner, dtype)
     p.lag = lag
     p.queue_cap_batches = queue_cap_batches
     p.trace = int(trace)

@@ -281,9 +281,22 @@ __global__ void __launch_bounds__(kDThreads, 1)
       for (int t = et; t < T; t += 128) {
         int pos = 0, slot = -1;
         const int64_t id = a.ids[t];
-        if (t < nv && id >= 0 && id < a.id_cap) {
+        // a row that exited at an earlier ramp of this split writes no K/V for
+        // the layers it skips (R15; oracle.llama.run_split)
+        const bool live = t < nv && (a.init_alive || a.alive == nullptr || a.alive[t] != 0);
+        if (live && id >= 0 && id < a.id_cap) {
           slot = a.slot_of_id[id];
-          pos = a.pos_of_slot[slot];
+          if (slot < 0 || slot >= a.n_slots) {
+            slot = -1;
+            if (a.err) *a.err = 1;
+          } else {
+            pos = a.pos_of_slot[slot];
+            if (pos < 0 || pos >= a.max_ctx) {
+              slot = -1;
+              pos = 0;
+              if (a.err) *a.err = 1;
+            }
+          }
         }
         sPos[t] = pos;
         sSlot[t] = slot;

@@ -122,6 +122,8 @@ struct DecArgs {
   const int32_t *slot_of_id;
   int64_t id_cap;
   const int32_t *pos_of_slot;
+  int n_slots;              // QKV_ROPE: slots of the cache; slot / pos outside it -> *err, row skipped
+  int *err;                 // device error flag (E3_EINVAL reported by the pipeline), may be NULL
   int late_trigger;         // PDL trigger at the end instead of after the dependency wait
 };
 int dec_tiles(int N, int epi);
@@ -135,7 +137,8 @@ e3_status rmsnorm_run(const void *x, const void *g, void *y, int rows, int H, fl
 // ctx[t, h*128 + :] = softmax(q_t,h . K[slot, g(h), 0..pos]^T / sqrt 128) V[...]
 e3_status attn_dec_run(const void *q, void *ctx, const void *kc, const void *vc, const int64_t *ids,
                        const int32_t *n_valid_dev, int n_valid_host, const int32_t *slot_of_id, int64_t id_cap,
-                       const int32_t *pos_of_slot, int T, int nh, int kvh, int max_ctx, cudaStream_t st);
+                       const int32_t *pos_of_slot, int n_slots, int T, int nh, int kvh, int max_ctx,
+                       cudaStream_t st);
 // merge the LM-head statistics, threshold test, exit records (RampArgs with lm_*)
 e3_status lm_decide_run(const RampArgs &a, cudaStream_t st);
 

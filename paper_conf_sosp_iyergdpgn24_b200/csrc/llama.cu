@@ -120,7 +120,7 @@ __global__ void __launch_bounds__(kAttnThreads)
                     const __nv_bfloat16 *__restrict__ kc, const __nv_bfloat16 *__restrict__ vc,
                     const int64_t *__restrict__ ids, const int32_t *n_valid_dev, int n_valid_host,
                     const int32_t *__restrict__ slot_of_id, int64_t id_cap, const int32_t *__restrict__ pos_of_slot,
-                    int nh, int kvh, int max_ctx, float scale) {
+                    int n_slots, int nh, int kvh, int max_ctx, float scale) {
   extern __shared__ float sp[];                 // [max_ctx] scores / probabilities
   __shared__ float red[kAW];
   __shared__ float4 sacc[kAW][32];
@@ -137,7 +137,11 @@ __global__ void __launch_bounds__(kAttnThreads)
     return;
   }
   const int slot = slot_of_id[id];
-  const int pos = pos_of_slot[slot];
+  const int pos = (slot >= 0 && slot < n_slots) ? pos_of_slot[slot] : -1;
+  if (pos < 0 || pos >= max_ctx) {             // outside the cache (flagged by the QKV epilogue)
+    if (tid < kHd / 4) reinterpret_cast<uint2 *>(out)[tid] = make_uint2(0u, 0u);
+    return;
+  }
   const int L = pos + 1;
   const int g = h / (nh / kvh);
   // lane owns dims 4*lane .. 4*lane+3 of q, of every key and every value row
@@ -346,7 +350,8 @@ e3_status rmsnorm_run(const void *x, const void *g, void *y, int rows, int H, fl
 
 e3_status attn_dec_run(const void *q, void *ctx, const void *kc, const void *vc, const int64_t *ids,
                        const int32_t *n_valid_dev, int n_valid_host, const int32_t *slot_of_id, int64_t id_cap,
-                       const int32_t *pos_of_slot, int T, int nh, int kvh, int max_ctx, cudaStream_t st) {
+                       const int32_t *pos_of_slot, int n_slots, int T, int nh, int kvh, int max_ctx,
+                       cudaStream_t st) {
   if (max_ctx > 16384 || nh % kvh) {
     set_error("decode attention: need max_ctx <= 16384 and heads % kv_heads == 0");
     return E3_EUNSUPPORTED;
@@ -360,7 +365,7 @@ e3_status attn_dec_run(const void *q, void *ctx, const void *kc, const void *vc,
   E3_CUDA_TRY(launch_k(attn_dec_kernel, dim3(nh, T), dim3(kAttnThreads), smem, st,
                        reinterpret_cast<const __nv_bfloat16 *>(q), reinterpret_cast<__nv_bfloat16 *>(ctx),
                        reinterpret_cast<const __nv_bfloat16 *>(kc), reinterpret_cast<const __nv_bfloat16 *>(vc),
-                       ids, n_valid_dev, n_valid_host, slot_of_id, id_cap, pos_of_slot, nh, kvh, max_ctx,
+                       ids, n_valid_dev, n_valid_host, slot_of_id, id_cap, pos_of_slot, n_slots, nh, kvh, max_ctx,
                        1.0f / sqrtf((float)kHd)));
   E3_CUDA_TRY(cudaGetLastError());
   count_launch();

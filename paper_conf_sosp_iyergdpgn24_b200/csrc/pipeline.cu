@@ -354,7 +354,10 @@ e3_status e3_pipeline_create(const e3_plan *p, const e3_weights *w, int device, 
   e3_pipeline *pl = new (std::nothrow) e3_pipeline();
   if (!pl) return E3_ECUDA;
   pl->plan = *p;
-  if (pl->plan.queue_cap_batches < 4) pl->plan.queue_cap_batches = 4;
+  // split s is launched while queue s+1 holds < B known rows; up to `lag`
+  // pending runs plus this one may each still push up to B rows
+  const int min_cap = p->lag + 2 > 4 ? p->lag + 2 : 4;
+  if (pl->plan.queue_cap_batches < min_cap) pl->plan.queue_cap_batches = min_cap;
   pl->device = device;
   pl->sms = num_sms(device);
   pl->B = d0.batch;
@@ -472,12 +475,18 @@ static e3_status pipeline_run_impl(e3_pipeline *pl, void *stream, const void *x,
   }
   e3_status r = R.run();
   if (r == E3_OK) {
-    int ovf = 0;
+    int ovf = 0, derr = 0;
     E3_CUDA_TRY(cudaMemcpyAsync(&ovf, pl->overflow, sizeof(int), cudaMemcpyDeviceToHost, R.st));
+    E3_CUDA_TRY(cudaMemcpyAsync(&derr, pl->ws->err, sizeof(int), cudaMemcpyDeviceToHost, R.st));
     E3_CUDA_TRY(cudaStreamSynchronize(R.st));
     if (ovf) {
       set_error("survivor queue overflow");
       r = E3_ECAPACITY;
+    } else if (derr) {
+      // rows whose KV slot / position lies outside the cache were skipped
+      E3_CUDA_TRY(cudaMemsetAsync(pl->ws->err, 0, sizeof(int), R.st));
+      set_error("a token's KV slot or position lies outside the cache (rows skipped)");
+      r = E3_EINVAL;
     }
   }
   if (r == E3_ECUDA || r == E3_ECAPACITY) pl->poisoned = true;

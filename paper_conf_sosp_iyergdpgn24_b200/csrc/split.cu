@@ -43,7 +43,7 @@ Workspace::~Workspace() {
   int prev = 0;
   cudaGetDevice(&prev);
   cudaSetDevice(device);
-  void *bufs[] = {qkv, ctx, y, x1, h, xa, xb, pool, alive, ctr, lm_stats, dec_part, dec_tickets, rope};
+  void *bufs[] = {qkv, ctx, y, x1, h, xa, xb, pool, alive, ctr, err, lm_stats, dec_part, dec_tickets, rope};
   for (void *p : bufs)
     if (p) cudaFree(p);
   cudaSetDevice(prev);
@@ -102,6 +102,8 @@ e3_status Workspace::create(int device, int B, int S, int H, int F, std::shared_
   E3_CUDA_TRY(cudaMalloc(&ws->ctr, kCtrWords * sizeof(unsigned)));
   E3_CUDA_TRY(cudaMemset(ws->ctr, 0, kCtrWords * sizeof(unsigned)));
   E3_CUDA_TRY(cudaMemset(ws->alive, 0, (size_t)B));
+  E3_CUDA_TRY(cudaMalloc(&ws->err, sizeof(int)));
+  E3_CUDA_TRY(cudaMemset(ws->err, 0, sizeof(int)));
   *out = ws;
   return E3_OK;
 }
@@ -404,13 +406,18 @@ static e3_status llama_run(e3_split *s, cudaStream_t st, const void *x_in, const
       a.slot_of_id = s->kv.slot_of_id;
       a.id_cap = s->kv.id_capacity;
       a.pos_of_slot = s->kv.pos_of_slot;
+      a.n_slots = s->kv.n_slots;
+      a.err = ws.err;
+      a.alive = first_ramp ? nullptr : ws.alive;   // after the split's first ramp: live rows only
+      a.init_alive = first_ramp;
       ProfScope ps(PK_GEMM_QKV, st, 0, (double)nqkv * H * b2 + nv * (H + nqkv) * b2);
       E3_RUN(dec_run(m.qkv, a, s->sms, st));
     }
     {
       ProfScope ps(PK_ATTN, st, 0, kv_bytes);
       E3_RUN(attn_dec_run(ws.qkv, ws.ctx, s->kv_k[l], s->kv_v[l], id_in, n_valid_dev, n_valid_host,
-                          s->kv.slot_of_id, s->kv.id_capacity, s->kv.pos_of_slot, B, d.heads, kvh, s->kv.max_ctx,
+                          s->kv.slot_of_id, s->kv.id_capacity, s->kv.pos_of_slot, s->kv.n_slots, B, d.heads, kvh,
+                          s->kv.max_ctx,
                           st));
     }
     {

@@ -20,6 +20,7 @@ struct Workspace {
   float *pool = nullptr;
   uint8_t *alive = nullptr;
   unsigned *ctr = nullptr;        // [kCtrWords]: compaction ticket, ramp row-group tickets
+  int *err = nullptr;             // device error flag: a kernel saw an argument outside its range
   // LLAMA decode (allocated by ensure_llama): LM-head tile statistics,
   // stream-K partials and tickets of the decode GEMMs, RoPE cos/sin table
   float4 *lm_stats = nullptr;

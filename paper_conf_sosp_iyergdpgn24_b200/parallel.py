@@ -91,6 +91,9 @@ def plan_stages(ramp_layers: Sequence[int], survival: Callable[[int], float], wo
     GPUs with free inter-GPU transfer pure replication is optimal (one stage);
     `n_stages` forces the number of stages (the paper's setting of models
     that do not fit one GPU, or to exercise the transport)."""
+    if n_stages is not None and not 1 <= n_stages <= min(world, len(ramp_layers)):
+        raise ValueError(f"n_stages={n_stages} needs 1 <= n_stages <= min(world={world}, "
+                         f"ramps={len(ramp_layers)})")
     cut_points = [l + 1 for l in ramp_layers[:-1]]
     L = ramp_layers[-1] + 1
     best = None
@@ -172,8 +175,10 @@ def run_stage_pipeline(executor, layout: StageLayout, rank: int, n_chunks: int,
         hdr = torch.tensor([n_s], dtype=torch.int64, device=dev if transport.device else "cpu")
         pending.append(transport.isend(hdr, dst))
         if n_s > 0:
-            pending.append(transport.isend(xs[:n_s], dst))
-            pending.append(transport.isend(ids_s[:n_s], dst))
+            # private copies: the executor reuses its output buffers for the
+            # next chunk while an NCCL isend of this one may still be queued
+            pending.append(transport.isend(xs[:n_s].clone(), dst))
+            pending.append(transport.isend(ids_s[:n_s].clone(), dst))
         stats["rows_out"] += n_s
         while len(pending) > 12:               # bound the in-flight buffers
             pending.pop(0)[0].wait()

@@ -189,3 +189,64 @@ def test_llama7b_shape_split_parity_sampled(api):
     kg = to64(cache.k[0])
     for k, i in enumerate(sample):
         assert np.max(np.abs(kg[i, :, cfg.ctx] - kv_or[0][0][k, :, cfg.ctx])) < 0.05
+
+
+def test_llama_multi_ramp_split_skips_kv_of_exited_tokens(api):
+    """One split holding both ramps (layers [0,4), inner EXACT): a token that
+    exits at the inner ramp (layer 1) writes no K/V at layers 2 and 3 (R15,
+    ADVICE r01), while the tokens that run on append theirs; results equal
+    the per-ramp plan bitwise."""
+    cfg = e3data.get("tiny-llama")
+    N = 32
+    slot_of = {i: i for i in range(N)}
+    pos_of = {s: cfg.ctx - (s % 4) for s in range(N)}
+    W, kv_np, cache, model = _setup(api, cfg, N, slot_of, pos_of, N)
+    X = e3data.make_inputs(cfg, range(N), seed=8)
+    ex = api.ExitBuffers(N, cfg.classes, cfg.n_ramps, DEV)
+    split = api.Split(model, api.split_desc(cfg, 0, 4, cfg.tau))
+    x_out = torch.zeros_like(bf16_tensor(X))
+    id_out = torch.full((N,), -9, dtype=torch.int64, device=DEV)
+    n_surv = torch.zeros(1, dtype=torch.int32, device=DEV)
+    split.run(bf16_tensor(X), torch.arange(N, dtype=torch.int64, device=DEV), x_out, id_out, n_surv, ex)
+    torch.cuda.synchronize()
+    el = ex.exit_layer.cpu().numpy()
+    assert int(n_surv.item()) == 0 and (el >= 0).all()
+    early = [i for i in range(N) if el[i] == 1]
+    late = [i for i in range(N) if el[i] == 3]
+    assert early and late, el
+    for l in (2, 3):
+        kg, vg = to64(cache.k[l]), to64(cache.v[l])
+        for i in early:
+            p = pos_of[i]
+            assert np.array_equal(kg[i, :, p], kv_np[l][0][i, :, p])
+            assert np.array_equal(vg[i, :, p], kv_np[l][1][i, :, p])
+        for i in late:
+            p = pos_of[i]
+            assert not np.array_equal(kg[i, :, p], kv_np[l][0][i, :, p])
+    # per-ramp plan on a fresh cache: identical exits and logits
+    W2, _, cache2, model2 = _setup(api, cfg, N, slot_of, pos_of, N, W=W)
+    ex2 = api.ExitBuffers(N, cfg.classes, cfg.n_ramps, DEV)
+    api.Pipeline(model2, api.make_plan(cfg, (0, 2, 4), cfg.tau)).run(
+        bf16_tensor(X), torch.arange(N, dtype=torch.int64, device=DEV), ex2)
+    assert torch.equal(ex2.exit_layer, ex.exit_layer) and torch.equal(ex2.logits, ex.logits)
+    for l in range(cfg.layers):
+        assert torch.equal(cache2.k[l], cache.k[l]) and torch.equal(cache2.v[l], cache.v[l])
+
+
+def test_llama_slot_outside_cache_is_an_error(api):
+    """A token whose KV slot lies outside the cache is skipped and reported
+    (E3_EINVAL at the pipeline's end), never a silent out-of-bounds write."""
+    cfg = e3data.get("tiny-llama")
+    N = 8
+    slot_of = {i: i for i in range(N)}
+    pos_of = {s: cfg.ctx for s in range(N)}
+    W, kv_np, cache, model = _setup(api, cfg, N, slot_of, pos_of, N)
+    cache.slot_of_id[3] = 1000
+    X = e3data.make_inputs(cfg, range(N), seed=9)
+    ex = api.ExitBuffers(N, cfg.classes, cfg.n_ramps, DEV)
+    from paper_conf_sosp_iyergdpgn24_b200._lib import E3Error
+    with pytest.raises(E3Error, match="EINVAL"):
+        api.Pipeline(model, api.make_plan(cfg, (0, 2, 4), cfg.tau)).run(
+            bf16_tensor(X), torch.arange(N, dtype=torch.int64, device=DEV), ex)
+    # no other slot was written on token 3's behalf: slot 3 is nobody's
+    assert np.array_equal(to64(cache.k[0][3]), kv_np[0][0][3])
