@@ -1,0 +1,362 @@
+// FP32 mode of the encoder split (E3_DTYPE_FP32; SURVEY §8(b) dtype, §8(c)
+// C13; R14): the same split semantics as the bf16 path -- layers,
+// fused ramp + threshold test, stable compaction into the next split's queue
+// -- with fp32 activations everywhere, so a whole job can be held to the
+// north_star's "1e-4 at fp32" against the fp64 oracle.  Weights stay the bf16
+// values the model was generated with (exactly representable in fp32, so the
+// oracle sees the same numbers).  Paper precision is unstated.
+//
+// This mode exists to prove the chained pipeline at tight bounds; its kernels
+// are plain SIMT (fp32 FMA, fixed summation order, no atomics in any value
+// path, so rows are batch-position invariant like the bf16 path):
+//   f32_gemm_kernel    Y = epi(A W^T + b): 128 x 128 CTA tile, 8 x 8 per
+//                      thread, K in steps of 16 staged in shared memory
+//   f32_attn_kernel    one CTA per (input, head): K, V of the head in shared
+//                      memory, a warp per query row, exact softmax
+//   f32_ln_kernel      warp per row, two-pass statistics
+//   f32_ramp_kernel    CTA per row: (LN) / pooler -> classifier -> softmax
+//                      metric -> strict threshold -> exit record, alive flag
+// Survivors are compacted by the byte-exact ln_compact kernel in copy mode.
+#include "common.cuh"
+#include "fp32_path.h"
+#include "prof.h"
+
+namespace e3 {
+
+namespace {
+
+constexpr int kGT = 256;   // GEMM threads
+constexpr int kBM = 128, kBN = 128, kBK = 16;
+
+template <int EPI>
+__global__ void __launch_bounds__(kGT)
+    f32_gemm_kernel(const float *__restrict__ A, int lda, const __nv_bfloat16 *__restrict__ W,
+                    const __nv_bfloat16 *__restrict__ bias, const float *__restrict__ R, float *__restrict__ Y, int M,
+                    int N, int K) {
+  __shared__ __align__(16) float As[kBK][kBM + 4];
+  __shared__ __align__(16) float Ws[kBK][kBN + 4];
+  const int tid = threadIdx.x;
+  const int m0 = blockIdx.y * kBM, n0 = blockIdx.x * kBN;
+  const int ty = tid / 16, tx = tid % 16;
+  float acc[8][8];
+#pragma unroll
+  for (int i = 0; i < 8; ++i)
+#pragma unroll
+    for (int j = 0; j < 8; ++j) acc[i][j] = 0.f;
+  for (int k0 = 0; k0 < K; k0 += kBK) {
+#pragma unroll
+    for (int u = 0; u < 2; ++u) {   // A tile: 128 rows x 16 k as float4
+      const int idx = tid + u * kGT;
+      const int row = idx >> 2, kq = idx & 3;
+      float4 v = make_float4(0.f, 0.f, 0.f, 0.f);
+      if (m0 + row < M) v = *reinterpret_cast<const float4 *>(A + (size_t)(m0 + row) * lda + k0 + kq * 4);
+      As[kq * 4 + 0][row] = v.x;
+      As[kq * 4 + 1][row] = v.y;
+      As[kq * 4 + 2][row] = v.z;
+      As[kq * 4 + 3][row] = v.w;
+    }
+    {   // W tile: 128 output rows x 16 k (bf16, 8 per 16-byte load)
+      const int n = tid >> 1, kh = tid & 1;
+      uint4 w = make_uint4(0u, 0u, 0u, 0u);
+      if (n0 + n < N) w = *reinterpret_cast<const uint4 *>(W + (size_t)(n0 + n) * K + k0 + kh * 8);
+      const uint32_t ws[4] = {w.x, w.y, w.z, w.w};
+#pragma unroll
+      for (int e = 0; e < 4; ++e) {
+        Ws[kh * 8 + 2 * e][n] = bf_lo(ws[e]);
+        Ws[kh * 8 + 2 * e + 1][n] = bf_hi(ws[e]);
+      }
+    }
+    __syncthreads();
+#pragma unroll
+    for (int k = 0; k < kBK; ++k) {
+      float a[8], b[8];
+      *reinterpret_cast<float4 *>(a) = *reinterpret_cast<const float4 *>(&As[k][ty * 8]);
+      *reinterpret_cast<float4 *>(a + 4) = *reinterpret_cast<const float4 *>(&As[k][ty * 8 + 4]);
+      *reinterpret_cast<float4 *>(b) = *reinterpret_cast<const float4 *>(&Ws[k][tx * 8]);
+      *reinterpret_cast<float4 *>(b + 4) = *reinterpret_cast<const float4 *>(&Ws[k][tx * 8 + 4]);
+#pragma unroll
+      for (int i = 0; i < 8; ++i)
+#pragma unroll
+        for (int j = 0; j < 8; ++j) acc[i][j] = fmaf(a[i], b[j], acc[i][j]);
+    }
+    __syncthreads();
+  }
+#pragma unroll
+  for (int i = 0; i < 8; ++i) {
+    const int r = m0 + ty * 8 + i;
+    if (r >= M) continue;
+#pragma unroll
+    for (int j = 0; j < 8; ++j) {
+      const int c = n0 + tx * 8 + j;
+      if (c >= N) continue;
+      float v = acc[i][j] + bf2f(bias[c]);
+      if (EPI == E3_EPI_BIAS_GELU) v = gelu_erf(v);
+      if (EPI == E3_EPI_BIAS_RESID) v += R[(size_t)r * N + c];
+      Y[(size_t)r * N + c] = v;
+    }
+  }
+}
+
+constexpr int kAT = 256;   // attention threads (8 warps)
+constexpr int kAW = kAT / 32;
+
+// ctx[b, i, h*64 + d] = sum_j softmax_j(q_i . k_j / 8) v_j[d] for the head h
+__global__ void __launch_bounds__(kAT) f32_attn_kernel(const float *__restrict__ qkv, float *__restrict__ ctx, int S,
+                                                       int H) {
+  extern __shared__ float sm[];
+  float *Ks = sm;                       // [S][65] (padded: lane j reads key row j)
+  float *Vs = Ks + (size_t)S * 65;      // [S][64]
+  float *Qs = Vs + (size_t)S * 64;      // [warps][64]
+  float *Ps = Qs + kAW * 64;            // [warps][S]
+  const int b = blockIdx.x / (H / 64), h = blockIdx.x % (H / 64);
+  const float *base = qkv + (size_t)b * S * 3 * H;
+  for (int idx = threadIdx.x; idx < S * 64; idx += kAT) {
+    const int j = idx >> 6, d = idx & 63;
+    Ks[j * 65 + d] = base[(size_t)j * 3 * H + H + h * 64 + d];
+    Vs[j * 64 + d] = base[(size_t)j * 3 * H + 2 * H + h * 64 + d];
+  }
+  __syncthreads();
+  const int warp = warp_id(), lane = lane_id();
+  float *q = Qs + warp * 64, *p = Ps + (size_t)warp * S;
+  for (int i = warp; i < S; i += kAW) {
+    q[lane] = base[(size_t)i * 3 * H + h * 64 + lane];
+    q[lane + 32] = base[(size_t)i * 3 * H + h * 64 + lane + 32];
+    __syncwarp();
+    float mx = -INFINITY;
+    for (int j = lane; j < S; j += 32) {
+      float s = 0.f;
+#pragma unroll 16
+      for (int d = 0; d < 64; ++d) s = fmaf(q[d], Ks[j * 65 + d], s);
+      s *= 0.125f;   // 1 / sqrt(64), exact
+      p[j] = s;
+      mx = fmaxf(mx, s);
+    }
+#pragma unroll
+    for (int o = 16; o; o >>= 1) mx = fmaxf(mx, __shfl_xor_sync(0xffffffffu, mx, o));
+    float l = 0.f;
+    for (int j = lane; j < S; j += 32) {
+      const float e = expf(p[j] - mx);
+      p[j] = e;
+      l += e;
+    }
+#pragma unroll
+    for (int o = 16; o; o >>= 1) l += __shfl_xor_sync(0xffffffffu, l, o);
+    __syncwarp();
+    float o0 = 0.f, o1 = 0.f;
+    for (int j = 0; j < S; ++j) {
+      const float pj = p[j];
+      o0 = fmaf(pj, Vs[j * 64 + lane], o0);
+      o1 = fmaf(pj, Vs[j * 64 + lane + 32], o1);
+    }
+    float *out = ctx + ((size_t)b * S + i) * H + h * 64;
+    out[lane] = o0 / l;
+    out[lane + 32] = o1 / l;
+    __syncwarp();
+  }
+}
+
+__device__ __forceinline__ float warp_sum(float v) {
+#pragma unroll
+  for (int o = 16; o; o >>= 1) v += __shfl_xor_sync(0xffffffffu, v, o);
+  return v;
+}
+
+// y = (x - mean) / sqrt(var + eps) * g + b per row, biased variance
+__global__ void __launch_bounds__(256) f32_ln_kernel(const float *__restrict__ x, const __nv_bfloat16 *__restrict__ g,
+                                                     const __nv_bfloat16 *__restrict__ bb, float *__restrict__ y,
+                                                     int rows, int H, float eps) {
+  const int row = blockIdx.x * 8 + warp_id(), lane = lane_id();
+  if (row >= rows) return;
+  const float *xr = x + (size_t)row * H;
+  float s = 0.f;
+  for (int k = lane; k < H; k += 32) s += xr[k];
+  const float mean = warp_sum(s) / (float)H;
+  float q = 0.f;
+  for (int k = lane; k < H; k += 32) {
+    const float d = xr[k] - mean;
+    q = fmaf(d, d, q);
+  }
+  const float rstd = 1.0f / sqrtf(warp_sum(q) / (float)H + eps);
+  float *yr = y + (size_t)row * H;
+  for (int k = lane; k < H; k += 32) yr[k] = (xr[k] - mean) * rstd * bf2f(g[k]) + bf2f(bb[k]);
+}
+
+constexpr int kRT = 256;
+
+// One CTA per batch row: the ramp of DESIGN.md R1 in fp32 and the exit test
+// (R3/R4/R6/R12), with the bf16 ramp's row semantics (padding never exits,
+// rows that exited at an earlier ramp of the split are skipped).
+__global__ void __launch_bounds__(kRT) f32_ramp_kernel(RampArgs a) {
+  extern __shared__ float rs[];
+  const int H = a.H, C = a.C;
+  float *c = rs;          // [H] CLS row (ViT: normalised)
+  float *p = c + H;       // [H] pooler output (BERT)
+  float *z = p + H;       // [C] logits
+  __shared__ float red[kRT / 32][3];
+  __shared__ int redi[kRT / 32];
+  const int b = blockIdx.x, tid = threadIdx.x, warp = warp_id(), lane = lane_id();
+  const int n_valid = a.n_valid_dev ? *a.n_valid_dev : a.n_valid_host;
+  const bool ok = a.init_alive ? (b < n_valid) : (a.alive[b] != 0);
+  if (!ok) {
+    if (a.init_alive && tid == 0) a.alive[b] = 0;
+    return;
+  }
+  const float *x = reinterpret_cast<const float *>(a.x) + (size_t)b * a.S * H;   // token 0
+  for (int k = tid; k < H; k += kRT) c[k] = x[k];
+  __syncthreads();
+  const bool vit = a.arch == E3_ARCH_VIT;
+  if (vit) {   // n = LN_r(c)
+    if (warp == 0) {
+      float s = 0.f;
+      for (int k = lane; k < H; k += 32) s += c[k];
+      const float mean = warp_sum(s) / (float)H;
+      float q = 0.f;
+      for (int k = lane; k < H; k += 32) q = fmaf(c[k] - mean, c[k] - mean, q);
+      const float rstd = 1.0f / sqrtf(warp_sum(q) / (float)H + a.eps);
+      const __nv_bfloat16 *g = reinterpret_cast<const __nv_bfloat16 *>(a.w.ln_g);
+      const __nv_bfloat16 *bb = reinterpret_cast<const __nv_bfloat16 *>(a.w.ln_b);
+      for (int k = lane; k < H; k += 32) p[k] = (c[k] - mean) * rstd * bf2f(g[k]) + bf2f(bb[k]);
+    }
+  } else {     // p = tanh(W_p c + b_p): a warp per output, lanes over k
+    const __nv_bfloat16 *wp = reinterpret_cast<const __nv_bfloat16 *>(a.w.w_p);
+    const __nv_bfloat16 *bp = reinterpret_cast<const __nv_bfloat16 *>(a.w.b_p);
+    for (int o = warp; o < H; o += kRT / 32) {
+      float s = 0.f;
+      for (int k = lane; k < H; k += 32) s = fmaf(bf2f(wp[(size_t)o * H + k]), c[k], s);
+      s = warp_sum(s);
+      if (lane == 0) p[o] = tanhf(s + bf2f(bp[o]));
+    }
+  }
+  __syncthreads();
+  {   // z = W_c p + b_c: a warp per class
+    const __nv_bfloat16 *wc = reinterpret_cast<const __nv_bfloat16 *>(a.w.w_c);
+    const __nv_bfloat16 *bc = reinterpret_cast<const __nv_bfloat16 *>(a.w.b_c);
+    for (int o = warp; o < C; o += kRT / 32) {
+      float s = 0.f;
+      for (int k = lane; k < H; k += 32) s = fmaf(bf2f(wc[(size_t)o * H + k]), p[k], s);
+      s = warp_sum(s);
+      if (lane == 0) z[o] = s + bf2f(bc[o]);
+    }
+  }
+  __syncthreads();
+  // max and argmax (lowest index on ties, R12)
+  float m = -INFINITY;
+  int arg = 0x7fffffff;
+  for (int k = tid; k < C; k += kRT)
+    if (z[k] > m) { m = z[k]; arg = k; }   // k ascending per thread: first max kept
+#pragma unroll
+  for (int o = 16; o; o >>= 1) {
+    const float m2 = __shfl_xor_sync(0xffffffffu, m, o);
+    const int a2 = __shfl_xor_sync(0xffffffffu, arg, o);
+    if (m2 > m || (m2 == m && a2 < arg)) { m = m2; arg = a2; }
+  }
+  if (lane == 0) { red[warp][0] = m; redi[warp] = arg; }
+  __syncthreads();
+  if (tid == 0) {
+    for (int w = 1; w < kRT / 32; ++w)
+      if (red[w][0] > red[0][0] || (red[w][0] == red[0][0] && redi[w] < redi[0])) {
+        red[0][0] = red[w][0];
+        redi[0] = redi[w];
+      }
+  }
+  __syncthreads();
+  m = red[0][0];
+  const int label = redi[0];
+  float se = 0.f, sq = 0.f;
+  for (int k = tid; k < C; k += kRT) {
+    const float e = expf(z[k] - m);
+    se += e;
+    sq = fmaf(e, z[k] - m, sq);
+  }
+  se = warp_sum(se);
+  sq = warp_sum(sq);
+  __syncthreads();
+  if (lane == 0) { red[warp][1] = se; red[warp][2] = sq; }
+  __syncthreads();
+  if (tid != 0) return;
+  float sum = 0.f, qz = 0.f;
+  for (int w = 0; w < kRT / 32; ++w) { sum += red[w][1]; qz += red[w][2]; }
+  float metric;
+  bool pass;
+  if (a.test == E3_TEST_MAXPROB) {
+    metric = 1.0f / sum;
+    pass = metric > a.tau;
+  } else {
+    metric = logf(sum) - qz / sum;
+    pass = metric < a.tau;
+  }
+  const bool exit_now = pass || a.final_ramp;
+  if (exit_now) {
+    const int64_t id = a.id[b];
+    if (id >= 0 && id < a.ex.capacity) {
+      if (a.ex.exit_layer) a.ex.exit_layer[id] = a.layer;
+      if (a.ex.label) a.ex.label[id] = label;
+      if (a.ex.conf) a.ex.conf[id] = metric;
+      if (a.ex.logits)
+        for (int k = 0; k < C; ++k) a.ex.logits[id * C + k] = z[k];
+    }
+    if (a.ex.n_exit) atomicAdd(a.ex.n_exit, 1);
+    if (a.ex.ramp_count) atomicAdd(a.ex.ramp_count + a.ramp_index, 1);
+  }
+  a.alive[b] = exit_now ? 0 : 1;
+}
+
+}  // namespace
+
+e3_status f32_gemm_run(const float *A, int lda, const void *W, const void *bias, const float *R, float *Y, int M,
+                       int N, int K, int epi, cudaStream_t st) {
+  if (K % kBK || lda % 4) {
+    set_error("fp32 GEMM: need K % 16 == 0 and lda % 4 == 0");
+    return E3_EUNSUPPORTED;
+  }
+  const dim3 grid((N + kBN - 1) / kBN, (M + kBM - 1) / kBM);
+  auto *w = reinterpret_cast<const __nv_bfloat16 *>(W);
+  auto *b = reinterpret_cast<const __nv_bfloat16 *>(bias);
+  if (epi == E3_EPI_BIAS) f32_gemm_kernel<E3_EPI_BIAS><<<grid, kGT, 0, st>>>(A, lda, w, b, R, Y, M, N, K);
+  else if (epi == E3_EPI_BIAS_GELU) f32_gemm_kernel<E3_EPI_BIAS_GELU><<<grid, kGT, 0, st>>>(A, lda, w, b, R, Y, M, N, K);
+  else f32_gemm_kernel<E3_EPI_BIAS_RESID><<<grid, kGT, 0, st>>>(A, lda, w, b, R, Y, M, N, K);
+  E3_CUDA_TRY(cudaGetLastError());
+  count_launch();
+  return E3_OK;
+}
+
+e3_status f32_attn_run(const float *qkv, float *ctx, int B, int S, int H, cudaStream_t st) {
+  if (H % 64 || S > 256) {
+    set_error("fp32 attention: need head_dim 64 and S <= 256");
+    return E3_EUNSUPPORTED;
+  }
+  const size_t smem = ((size_t)S * (65 + 64) + kAW * 64 + (size_t)kAW * S) * sizeof(float);
+  static size_t attr = 0;
+  if (smem > 48 * 1024 && smem > attr) {
+    E3_CUDA_TRY(cudaFuncSetAttribute(f32_attn_kernel, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem));
+    attr = smem;
+  }
+  f32_attn_kernel<<<B * (H / 64), kAT, smem, st>>>(qkv, ctx, S, H);
+  E3_CUDA_TRY(cudaGetLastError());
+  count_launch();
+  return E3_OK;
+}
+
+e3_status f32_ln_run(const float *x, const void *g, const void *b, float *y, int rows, int H, float eps,
+                     cudaStream_t st) {
+  f32_ln_kernel<<<(rows + 7) / 8, 256, 0, st>>>(x, reinterpret_cast<const __nv_bfloat16 *>(g),
+                                                reinterpret_cast<const __nv_bfloat16 *>(b), y, rows, H, eps);
+  E3_CUDA_TRY(cudaGetLastError());
+  count_launch();
+  return E3_OK;
+}
+
+e3_status f32_ramp_run(const RampArgs &a, cudaStream_t st) {
+  const size_t smem = (2 * (size_t)a.H + a.C) * sizeof(float);
+  static size_t attr = 0;
+  if (smem > 48 * 1024 && smem > attr) {
+    E3_CUDA_TRY(cudaFuncSetAttribute(f32_ramp_kernel, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem));
+    attr = smem;
+  }
+  f32_ramp_kernel<<<a.B, kRT, smem, st>>>(a);
+  E3_CUDA_TRY(cudaGetLastError());
+  count_launch();
+  return E3_OK;
+}
+
+}  // namespace e3

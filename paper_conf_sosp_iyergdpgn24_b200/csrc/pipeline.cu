@@ -341,7 +341,7 @@ e3_status e3_pipeline_create(const e3_plan *p, const e3_weights *w, int device, 
   for (int s = 0; s < p->n_splits; ++s) {
     const e3_split_desc &d = p->split[s];
     E3_CHECK_ARG(d.hidden == d0.hidden && d.seq_len == d0.seq_len && d.ffn == d0.ffn && d.batch == d0.batch &&
-                     d.heads == d0.heads && d.arch == d0.arch,
+                     d.heads == d0.heads && d.arch == d0.arch && d.dtype == d0.dtype,
                  "splits differ in model dims or batch");
     E3_CHECK_ARG(s == 0 || d.layer_begin == p->split[s - 1].layer_end, "splits not contiguous");
     E3_CHECK_ARG(s == p->n_splits - 1 || d.final_ramp == 0, "only the last split may hold the final ramp");
@@ -361,8 +361,9 @@ e3_status e3_pipeline_create(const e3_plan *p, const e3_weights *w, int device, 
   pl->device = device;
   pl->sms = num_sms(device);
   pl->B = d0.batch;
-  pl->row_bytes = (int64_t)d0.seq_len * d0.hidden * 2;
-  e3_status r = Workspace::create(device, d0.batch, d0.seq_len, d0.hidden, d0.ffn, &pl->ws);
+  const int elem = d0.dtype == E3_DTYPE_FP32 ? 4 : 2;
+  pl->row_bytes = (int64_t)d0.seq_len * d0.hidden * elem;
+  e3_status r = Workspace::create(device, d0.batch, d0.seq_len, d0.hidden, d0.ffn, elem, &pl->ws);
   for (int s = 0; s < p->n_splits && r == E3_OK; ++s) {
     e3_split *sp = nullptr;
     r = split_create_shared(&p->split[s], w, device, pl->ws, &sp);

@@ -22,6 +22,7 @@
 #include "common.cuh"
 #include "prof.h"
 #include "split.h"
+#include "fp32_path.h"
 
 namespace e3 {
 
@@ -82,21 +83,22 @@ e3_status Workspace::ensure_llama(int V, size_t part, size_t tickets, int max_ct
   return E3_OK;
 }
 
-e3_status Workspace::create(int device, int B, int S, int H, int F, std::shared_ptr<Workspace> *out) {
+e3_status Workspace::create(int device, int B, int S, int H, int F, int elem, std::shared_ptr<Workspace> *out) {
   auto ws = std::make_shared<Workspace>();
   ws->device = device;
   ws->B = B;
   ws->S = S;
   ws->H = H;
   ws->F = F;
-  const size_t M = (size_t)B * S;
-  E3_CUDA_TRY(cudaMalloc(&ws->qkv, M * 3 * H * 2));
-  E3_CUDA_TRY(cudaMalloc(&ws->ctx, M * H * 2));
-  E3_CUDA_TRY(cudaMalloc(&ws->y, M * H * 2));
-  E3_CUDA_TRY(cudaMalloc(&ws->x1, M * H * 2));
-  E3_CUDA_TRY(cudaMalloc(&ws->h, M * F * 2));
-  E3_CUDA_TRY(cudaMalloc(&ws->xa, M * H * 2));
-  E3_CUDA_TRY(cudaMalloc(&ws->xb, M * H * 2));
+  ws->elem = elem;
+  const size_t M = (size_t)B * S, e = (size_t)elem;
+  E3_CUDA_TRY(cudaMalloc(&ws->qkv, M * 3 * H * e));
+  E3_CUDA_TRY(cudaMalloc(&ws->ctx, M * H * e));
+  E3_CUDA_TRY(cudaMalloc(&ws->y, M * H * e));
+  E3_CUDA_TRY(cudaMalloc(&ws->x1, M * H * e));
+  E3_CUDA_TRY(cudaMalloc(&ws->h, M * F * e));
+  E3_CUDA_TRY(cudaMalloc(&ws->xa, M * H * e));
+  E3_CUDA_TRY(cudaMalloc(&ws->xb, M * H * e));
   E3_CUDA_TRY(cudaMalloc(&ws->pool, (size_t)B * H * 4));
   E3_CUDA_TRY(cudaMalloc(&ws->alive, (size_t)B));
   E3_CUDA_TRY(cudaMalloc(&ws->ctr, kCtrWords * sizeof(unsigned)));
@@ -114,7 +116,7 @@ static bool aligned16(const void *p) { return (reinterpret_cast<uintptr_t>(p) & 
 // B in {32, 64, 128}, the caller's KV cache covering the split's layers.
 static e3_status llama_validate(const e3_split_desc *d, const e3_weights *w) {
   if (d->dtype != E3_DTYPE_BF16) {
-    set_error("e3_split_create: only dtype BF16 is implemented");
+    set_error("e3_split_create (LLAMA): only dtype BF16 is implemented");
     return E3_EUNSUPPORTED;
   }
   const int kvh = d->kv_heads > 0 ? d->kv_heads : d->heads;
@@ -164,8 +166,12 @@ e3_status split_validate(const e3_split_desc *d, const e3_weights *w) {
   }
   if (d->arch == E3_ARCH_LLAMA_DECODE) return llama_validate(d, w);
   const bool vit = d->arch == E3_ARCH_VIT;
-  if (d->dtype != E3_DTYPE_BF16) {
-    set_error("e3_split_create: only dtype BF16 is implemented");
+  if (d->dtype != E3_DTYPE_BF16 && d->dtype != E3_DTYPE_FP32) {
+    set_error("e3_split_create: dtype must be BF16 or FP32");
+    return E3_EUNSUPPORTED;
+  }
+  if (d->dtype == E3_DTYPE_FP32 && d->hidden > 2048) {
+    set_error("e3_split_create: FP32 mode needs H <= 2048");
     return E3_EUNSUPPORTED;
   }
   E3_CHECK_ARG(d->hidden > 0 && d->heads > 0 && d->ffn > 0 && d->seq_len > 0 && d->batch > 0, "non-positive dims");
@@ -277,13 +283,14 @@ e3_status split_create_shared(const e3_split_desc *d, const e3_weights *w, int d
   const int B = d->batch, S = d->seq_len, H = d->hidden, F = d->ffn;
   for (int l = d->layer_begin; l < d->layer_end; ++l) s->L.push_back(w->layer[l]);
   for (int r = 0; r < d->n_ramps; ++r) s->R.push_back(w->ramp[d->ramp_index[r]]);
+  const int elem = d->dtype == E3_DTYPE_FP32 ? 4 : 2;
   if (!ws) {
-    st = Workspace::create(device, B, S, H, F, &ws);
+    st = Workspace::create(device, B, S, H, F, elem, &ws);
     if (st != E3_OK) {
       delete s;
       return st;
     }
-  } else if (ws->B != B || ws->S != S || ws->H != H || ws->F != F) {
+  } else if (ws->B != B || ws->S != S || ws->H != H || ws->F != F || ws->elem != elem) {
     delete s;
     set_error("shared workspace shape mismatch");
     return E3_EINVAL;
@@ -295,6 +302,10 @@ e3_status split_create_shared(const e3_split_desc *d, const e3_weights *w, int d
       delete s;
       return st;
     }
+    *out = s;
+    return E3_OK;
+  }
+  if (d->dtype == E3_DTYPE_FP32) {   // SIMT fp32 kernels: no tensor maps
     *out = s;
     return E3_OK;
   }
@@ -513,6 +524,88 @@ static e3_status llama_run(e3_split *s, cudaStream_t st, const void *x_in, const
   return E3_OK;
 }
 
+// FP32 mode (fp32_path.cu): the layer recipes of DESIGN.md R11 with fp32
+// activations, LN2 materialised for every layer, the ramp on the post-LN
+// rows, survivors copied (4-byte elements as pairs of 2-byte ones).
+static e3_status f32_run(e3_split *s, cudaStream_t st, const void *x_in, const int64_t *id_in,
+                         const int32_t *n_valid_dev, int n_valid_host, const RingDst &dst, int32_t *n_surv_dev,
+                         const e3_exits *ex) {
+  const e3_split_desc &d = s->d;
+  Workspace &ws = *s->ws;
+  const int B = d.batch, S = d.seq_len, H = d.hidden, F = d.ffn, M = B * S;
+  const int nl = d.layer_end - d.layer_begin;
+  const bool vit = d.arch == E3_ARCH_VIT;
+  e3_exits exits{};
+  if (ex) exits = *ex;
+  auto *qkv = static_cast<float *>(ws.qkv), *ctx = static_cast<float *>(ws.ctx), *y = static_cast<float *>(ws.y);
+  auto *x1 = static_cast<float *>(ws.x1), *hb = static_cast<float *>(ws.h);
+  const float *cur = static_cast<const float *>(x_in);
+  bool first_ramp = true;
+  int ri = 0;
+  e3_status r = E3_OK;
+#define E3_RUN(expr)              \
+  do {                            \
+    r = (expr);                   \
+    if (r != E3_OK) return r;     \
+  } while (0)
+  for (int i = 0; i < nl; ++i) {
+    const int l = d.layer_begin + i;
+    const e3_layer_weights &L = s->L[i];
+    float *out = static_cast<float *>((i % 2 == 0) ? ws.xa : ws.xb);
+    if (vit) {   // n1 = LN1(x); y1 = x + attn(n1) W_o; n2 = LN2(y1); x2 = y1 + MLP(n2)
+      E3_RUN(f32_ln_run(cur, L.ln1_g, L.ln1_b, x1, M, H, d.norm_eps, st));
+      E3_RUN(f32_gemm_run(x1, H, L.w_qkv, L.b_qkv, nullptr, qkv, M, 3 * H, H, E3_EPI_BIAS, st));
+      E3_RUN(f32_attn_run(qkv, ctx, B, S, H, st));
+      E3_RUN(f32_gemm_run(ctx, H, L.w_o, L.b_o, cur, y, M, H, H, E3_EPI_BIAS_RESID, st));
+      E3_RUN(f32_ln_run(y, L.ln2_g, L.ln2_b, x1, M, H, d.norm_eps, st));
+      E3_RUN(f32_gemm_run(x1, H, L.w_1, L.b_1, nullptr, hb, M, F, H, E3_EPI_BIAS_GELU, st));
+      E3_RUN(f32_gemm_run(hb, F, L.w_2, L.b_2, y, out, M, H, F, E3_EPI_BIAS_RESID, st));
+    } else {     // x1 = LN1(x + attn(x) W_o); x2 = LN2(x1 + MLP(x1))
+      E3_RUN(f32_gemm_run(cur, H, L.w_qkv, L.b_qkv, nullptr, qkv, M, 3 * H, H, E3_EPI_BIAS, st));
+      E3_RUN(f32_attn_run(qkv, ctx, B, S, H, st));
+      E3_RUN(f32_gemm_run(ctx, H, L.w_o, L.b_o, cur, y, M, H, H, E3_EPI_BIAS_RESID, st));
+      E3_RUN(f32_ln_run(y, L.ln1_g, L.ln1_b, x1, M, H, d.norm_eps, st));
+      E3_RUN(f32_gemm_run(x1, H, L.w_1, L.b_1, nullptr, hb, M, F, H, E3_EPI_BIAS_GELU, st));
+      E3_RUN(f32_gemm_run(hb, F, L.w_2, L.b_2, x1, y, M, H, F, E3_EPI_BIAS_RESID, st));
+      E3_RUN(f32_ln_run(y, L.ln2_g, L.ln2_b, out, M, H, d.norm_eps, st));
+    }
+    cur = out;
+    while (ri < d.n_ramps && d.ramp_layer[ri] == l) {
+      const bool last = (ri == d.n_ramps - 1);
+      if (last || d.inner == E3_INNER_EXACT) {
+        RampArgs a{};
+        a.arch = d.arch;
+        a.x = cur;
+        a.id = id_in;
+        a.B = B;
+        a.S = S;
+        a.H = H;
+        a.C = d.num_labels;
+        a.w = s->R[ri];
+        a.test = d.test;
+        a.tau = d.tau[ri];
+        a.final_ramp = last && d.final_ramp;
+        a.layer = l;
+        a.ramp_index = d.ramp_index[ri];
+        a.eps = d.norm_eps;
+        a.alive = ws.alive;
+        a.init_alive = first_ramp;
+        a.n_valid_dev = n_valid_dev;
+        a.n_valid_host = n_valid_host;
+        a.ex = exits;
+        E3_RUN(f32_ramp_run(a, st));
+        first_ramp = false;
+      }
+      ++ri;
+    }
+  }
+  // survivors: fp32 rows copied as 2H two-byte elements (no normalisation)
+  E3_RUN(ln_compact_run(cur, id_in, ws.alive, B, S, 2 * H, nullptr, nullptr, d.norm_eps, dst, n_surv_dev, s->sms,
+                        st));
+#undef E3_RUN
+  return E3_OK;
+}
+
 static LnGemmArgs oln_args(const void *bias, const void *R, const void *g, const void *b, float eps, int M, int H,
                            int store_pre) {
   LnGemmArgs a{};
@@ -533,6 +626,7 @@ e3_status split_run_to(e3_split *s, cudaStream_t st, const void *x_in, const int
                        const e3_exits *ex) {
   if (s->d.arch == E3_ARCH_LLAMA_DECODE)
     return llama_run(s, st, x_in, id_in, n_valid_dev, n_valid_host, dst, n_surv_dev, ex);
+  if (s->d.dtype == E3_DTYPE_FP32) return f32_run(s, st, x_in, id_in, n_valid_dev, n_valid_host, dst, n_surv_dev, ex);
   const e3_split_desc &d = s->d;
   Workspace &ws = *s->ws;
   const int B = d.batch, S = d.seq_len, H = d.hidden, F = d.ffn, M = B * S;

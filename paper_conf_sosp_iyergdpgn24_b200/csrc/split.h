@@ -16,6 +16,7 @@ constexpr int kCtrWords = 1 + 4096 / kRampRowsPerCta;
 struct Workspace {
   int device = 0;
   int B = 0, S = 0, H = 0, F = 0;
+  int elem = 2;                   // bytes per activation element: 2 (BF16) or 4 (FP32)
   void *qkv = nullptr, *ctx = nullptr, *y = nullptr, *x1 = nullptr, *h = nullptr, *xa = nullptr, *xb = nullptr;
   float *pool = nullptr;
   uint8_t *alive = nullptr;
@@ -32,7 +33,7 @@ struct Workspace {
   double rope_theta = 0;
   e3_status ensure_llama(int V, size_t part_elems, size_t tickets, int max_ctx, int head_dim, double theta);
   ~Workspace();
-  static e3_status create(int device, int B, int S, int H, int F, std::shared_ptr<Workspace> *out);
+  static e3_status create(int device, int B, int S, int H, int F, int elem, std::shared_ptr<Workspace> *out);
 };
 
 }  // namespace e3
