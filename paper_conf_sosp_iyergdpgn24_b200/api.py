@@ -84,12 +84,15 @@ class KVCache:
     K and V [n_slots, kv_heads, max_ctx, head_dim] bf16, the slot of every
     token id and the cached length of every slot."""
 
-    def __init__(self, cfg, n_slots, max_ctx, id_capacity, device="cuda:0", fill=None):
+    def __init__(self, cfg, n_slots, max_ctx, id_capacity, device="cuda:0", dtype="bf16"):
+        """dtype: element type of the cache, that of the splits reading it
+        ("bf16" for E3_DTYPE_BF16 splits, "fp32" for E3_DTYPE_FP32)."""
         dev = torch.device(device)
         kvh, d = cfg.kv_heads or cfg.heads, cfg.head_dim
         shape = (n_slots, kvh, max_ctx, d)
-        self.k = [torch.zeros(shape, dtype=torch.bfloat16, device=dev) for _ in range(cfg.layers)]
-        self.v = [torch.zeros(shape, dtype=torch.bfloat16, device=dev) for _ in range(cfg.layers)]
+        tdt = {"bf16": torch.bfloat16, "fp32": torch.float32}[dtype]
+        self.k = [torch.zeros(shape, dtype=tdt, device=dev) for _ in range(cfg.layers)]
+        self.v = [torch.zeros(shape, dtype=tdt, device=dev) for _ in range(cfg.layers)]
         self.slot_of_id = torch.zeros(id_capacity, dtype=torch.int32, device=dev)
         self.pos_of_slot = torch.full((n_slots,), cfg.ctx, dtype=torch.int32, device=dev)
         self._kp = (C.c_void_p * cfg.layers)(*[t.data_ptr() for t in self.k])

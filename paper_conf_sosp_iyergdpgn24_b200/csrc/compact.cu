@@ -114,7 +114,10 @@ __global__ void __launch_bounds__(kThreads)
     *done_ctr = 0;
     const int out = fits ? n : 0;
     if (!fits && dst.overflow_dev) *dst.overflow_dev = 1;
-    if (fits && dst.tail_dev) *(volatile int64_t *)dst.tail_dev = tail + n;
+    if (dst.tail_dev) {   // next tail into the queue's other slot when given (as ln_compact)
+      if (dst.tail_out) *(volatile int64_t *)dst.tail_out = fits ? tail + n : tail;
+      else if (fits) *(volatile int64_t *)dst.tail_dev = tail + n;
+    }
     if (n_surv_dev) *n_surv_dev = out;
     if (dst.mailbox) {
       *dst.mailbox = fits ? out : -1;

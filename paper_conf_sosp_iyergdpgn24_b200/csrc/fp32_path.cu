@@ -89,7 +89,7 @@ __global__ void __launch_bounds__(kGT)
     for (int j = 0; j < 8; ++j) {
       const int c = n0 + tx * 8 + j;
       if (c >= N) continue;
-      float v = acc[i][j] + bf2f(bias[c]);
+      float v = acc[i][j] + (bias ? bf2f(bias[c]) : 0.f);
       if (EPI == E3_EPI_BIAS_GELU) v = gelu_erf(v);
       if (EPI == E3_EPI_BIAS_RESID) v += R[(size_t)r * N + c];
       Y[(size_t)r * N + c] = v;
@@ -205,7 +205,15 @@ __global__ void __launch_bounds__(kRT) f32_ramp_kernel(RampArgs a) {
   for (int k = tid; k < H; k += kRT) c[k] = x[k];
   __syncthreads();
   const bool vit = a.arch == E3_ARCH_VIT;
-  if (vit) {   // n = LN_r(c)
+  if (a.arch == E3_ARCH_LLAMA_DECODE) {   // nf = RMSNorm_f(c) (R22)
+    if (warp == 0) {
+      float q = 0.f;
+      for (int k = lane; k < H; k += 32) q = fmaf(c[k], c[k], q);
+      const float r = 1.0f / sqrtf(warp_sum(q) / (float)H + a.eps);
+      const __nv_bfloat16 *g = reinterpret_cast<const __nv_bfloat16 *>(a.w.ln_g);
+      for (int k = lane; k < H; k += 32) p[k] = c[k] * r * bf2f(g[k]);
+    }
+  } else if (vit) {   // n = LN_r(c)
     if (warp == 0) {
       float s = 0.f;
       for (int k = lane; k < H; k += 32) s += c[k];
@@ -235,7 +243,7 @@ __global__ void __launch_bounds__(kRT) f32_ramp_kernel(RampArgs a) {
       float s = 0.f;
       for (int k = lane; k < H; k += 32) s = fmaf(bf2f(wc[(size_t)o * H + k]), p[k], s);
       s = warp_sum(s);
-      if (lane == 0) z[o] = s + bf2f(bc[o]);
+      if (lane == 0) z[o] = s + (bc ? bf2f(bc[o]) : 0.f);
     }
   }
   __syncthreads();
@@ -273,35 +281,201 @@ __global__ void __launch_bounds__(kRT) f32_ramp_kernel(RampArgs a) {
   __syncthreads();
   if (lane == 0) { red[warp][1] = se; red[warp][2] = sq; }
   __syncthreads();
-  if (tid != 0) return;
-  float sum = 0.f, qz = 0.f;
-  for (int w = 0; w < kRT / 32; ++w) { sum += red[w][1]; qz += red[w][2]; }
-  float metric;
-  bool pass;
-  if (a.test == E3_TEST_MAXPROB) {
-    metric = 1.0f / sum;
-    pass = metric > a.tau;
-  } else {
-    metric = logf(sum) - qz / sum;
-    pass = metric < a.tau;
-  }
-  const bool exit_now = pass || a.final_ramp;
-  if (exit_now) {
+  __shared__ int s_exit;
+  __shared__ int64_t s_id;
+  if (tid == 0) {
+    float sum = 0.f, qz = 0.f;
+    for (int w = 0; w < kRT / 32; ++w) { sum += red[w][1]; qz += red[w][2]; }
+    float metric;
+    bool pass;
+    if (a.test == E3_TEST_MAXPROB) {
+      metric = 1.0f / sum;
+      pass = metric > a.tau;
+    } else {
+      metric = logf(sum) - qz / sum;
+      pass = metric < a.tau;
+    }
+    const bool exit_now = pass || a.final_ramp;
     const int64_t id = a.id[b];
-    if (id >= 0 && id < a.ex.capacity) {
+    const bool rec = exit_now && id >= 0 && id < a.ex.capacity;
+    if (rec) {
       if (a.ex.exit_layer) a.ex.exit_layer[id] = a.layer;
       if (a.ex.label) a.ex.label[id] = label;
       if (a.ex.conf) a.ex.conf[id] = metric;
-      if (a.ex.logits)
-        for (int k = 0; k < C; ++k) a.ex.logits[id * C + k] = z[k];
     }
-    if (a.ex.n_exit) atomicAdd(a.ex.n_exit, 1);
-    if (a.ex.ramp_count) atomicAdd(a.ex.ramp_count + a.ramp_index, 1);
+    if (exit_now) {
+      if (a.ex.n_exit) atomicAdd(a.ex.n_exit, 1);
+      if (a.ex.ramp_count) atomicAdd(a.ex.ramp_count + a.ramp_index, 1);
+    }
+    a.alive[b] = exit_now ? 0 : 1;
+    s_exit = rec;
+    s_id = id;
   }
-  a.alive[b] = exit_now ? 0 : 1;
+  __syncthreads();
+  if (s_exit && a.ex.logits)
+    for (int k = tid; k < C; k += kRT) a.ex.logits[s_id * C + k] = z[k];
+}
+
+// ---- LLaMA decode (R22) in fp32 --------------------------------------
+
+// y = x / sqrt(mean(x^2) + eps) * g per row
+__global__ void __launch_bounds__(256) f32_rms_kernel(const float *__restrict__ x, const __nv_bfloat16 *__restrict__ g,
+                                                      float *__restrict__ y, int rows, int H, float eps) {
+  const int row = blockIdx.x * 8 + warp_id(), lane = lane_id();
+  if (row >= rows) return;
+  const float *xr = x + (size_t)row * H;
+  float q = 0.f;
+  for (int k = lane; k < H; k += 32) q = fmaf(xr[k], xr[k], q);
+  const float r = 1.0f / sqrtf(warp_sum(q) / (float)H + eps);
+  float *yr = y + (size_t)row * H;
+  for (int k = lane; k < H; k += 32) yr[k] = xr[k] * r * bf2f(g[k]);
+}
+
+// a = SiLU(g) * u elementwise
+__global__ void f32_swiglu_kernel(const float *__restrict__ g, const float *__restrict__ u, float *__restrict__ a,
+                                  size_t n) {
+  for (size_t i = blockIdx.x * (size_t)blockDim.x + threadIdx.x; i < n; i += (size_t)gridDim.x * blockDim.x) {
+    const float x = g[i];
+    a[i] = x / (1.0f + expf(-x)) * u[i];
+  }
+}
+
+// token t: q <- RoPE(q) into qo [T, nh*128]; k <- RoPE(k), v appended to the
+// fp32 cache at (slot, pos) -- only for valid rows still alive in the split
+// (R15); slot / pos outside the cache -> *err, row skipped
+__global__ void f32_rope_kv_kernel(const float *__restrict__ qkv, float *__restrict__ qo, float *__restrict__ kc,
+                                   float *__restrict__ vc, const float2 *__restrict__ rope, DecArgs a) {
+  const int t = blockIdx.x, j = threadIdx.x;   // 64 threads: rotation pairs (j, j + 64)
+  const int nv = a.n_valid_dev ? *a.n_valid_dev : a.n_valid_host;
+  const int64_t id = a.ids[t];
+  const bool live = t < nv && (a.init_alive || a.alive == nullptr || a.alive[t] != 0) && id >= 0 && id < a.id_cap;
+  int slot = -1, pos = 0;
+  if (live) {
+    slot = a.slot_of_id[id];
+    if (slot < 0 || slot >= a.n_slots) {
+      slot = -1;
+      if (j == 0 && a.err) *a.err = 1;
+    } else {
+      pos = a.pos_of_slot[slot];
+      if (pos < 0 || pos >= a.max_ctx) {
+        slot = -1;
+        pos = 0;
+        if (j == 0 && a.err) *a.err = 1;
+      }
+    }
+  }
+  const int ld = (a.nh + 2 * a.kvh) * 128;
+  const float *row = qkv + (size_t)t * ld;
+  const float2 cs = rope[(size_t)pos * 64 + j];
+  for (int h = 0; h < a.nh; ++h) {
+    const float lo = row[h * 128 + j], hi = row[h * 128 + j + 64];
+    qo[(size_t)t * a.nh * 128 + h * 128 + j] = lo * cs.x - hi * cs.y;
+    qo[(size_t)t * a.nh * 128 + h * 128 + j + 64] = hi * cs.x + lo * cs.y;
+  }
+  if (slot < 0) return;
+  for (int h = 0; h < a.kvh; ++h) {
+    const float lo = row[(a.nh + h) * 128 + j], hi = row[(a.nh + h) * 128 + j + 64];
+    float *kd = kc + (((size_t)slot * a.kvh + h) * a.max_ctx + pos) * 128;
+    float *vd = vc + (((size_t)slot * a.kvh + h) * a.max_ctx + pos) * 128;
+    kd[j] = lo * cs.x - hi * cs.y;
+    kd[j + 64] = hi * cs.x + lo * cs.y;
+    vd[j] = row[(a.nh + a.kvh + h) * 128 + j];
+    vd[j + 64] = row[(a.nh + a.kvh + h) * 128 + j + 64];
+  }
+}
+
+// ctx[t, h*128 + d] = sum_p softmax_p(q . K[p] / sqrt 128) V[p][d], p = 0..pos
+__global__ void __launch_bounds__(128) f32_attn_dec_kernel(const float *__restrict__ q, float *__restrict__ ctx,
+                                                           const float *__restrict__ kc, const float *__restrict__ vc,
+                                                           DecArgs a) {
+  extern __shared__ float sp[];   // [max_ctx]
+  __shared__ float qs[128];
+  __shared__ float red[4];
+  const int h = blockIdx.x, t = blockIdx.y, tid = threadIdx.x, warp = warp_id(), lane = lane_id();
+  const int nv = a.n_valid_dev ? *a.n_valid_dev : a.n_valid_host;
+  const int64_t id = a.ids[t];
+  float *out = ctx + (size_t)t * a.nh * 128 + h * 128;
+  int pos = -1, slot = -1;
+  if (t < nv && id >= 0 && id < a.id_cap) {
+    slot = a.slot_of_id[id];
+    if (slot >= 0 && slot < a.n_slots) pos = a.pos_of_slot[slot];
+  }
+  if (pos < 0 || pos >= a.max_ctx) {   // padding / outside the cache: finite zeros
+    out[tid] = 0.f;
+    return;
+  }
+  const int g = h / (a.nh / a.kvh);
+  qs[tid] = q[(size_t)t * a.nh * 128 + h * 128 + tid];
+  __syncthreads();
+  const float *K = kc + ((size_t)slot * a.kvh + g) * a.max_ctx * 128;
+  const float *V = vc + ((size_t)slot * a.kvh + g) * a.max_ctx * 128;
+  const float scale = 1.0f / sqrtf(128.0f);
+  float mx = -INFINITY;
+  for (int p = tid; p <= pos; p += 128) {
+    float s = 0.f;
+    for (int d = 0; d < 128; ++d) s = fmaf(qs[d], K[(size_t)p * 128 + d], s);
+    s *= scale;
+    sp[p] = s;
+    mx = fmaxf(mx, s);
+  }
+#pragma unroll
+  for (int o = 16; o; o >>= 1) mx = fmaxf(mx, __shfl_xor_sync(0xffffffffu, mx, o));
+  if (lane == 0) red[warp] = mx;
+  __syncthreads();
+  mx = fmaxf(fmaxf(red[0], red[1]), fmaxf(red[2], red[3]));
+  __syncthreads();
+  float l = 0.f;
+  for (int p = tid; p <= pos; p += 128) {
+    const float e = expf(sp[p] - mx);
+    sp[p] = e;
+    l += e;
+  }
+  l = warp_sum(l);
+  if (lane == 0) red[warp] = l;
+  __syncthreads();
+  l = red[0] + red[1] + red[2] + red[3];
+  float o = 0.f;
+  for (int p = 0; p <= pos; ++p) o = fmaf(sp[p], V[(size_t)p * 128 + tid], o);
+  out[tid] = o / l;
 }
 
 }  // namespace
+
+e3_status f32_rms_run(const float *x, const void *g, float *y, int rows, int H, float eps, cudaStream_t st) {
+  f32_rms_kernel<<<(rows + 7) / 8, 256, 0, st>>>(x, reinterpret_cast<const __nv_bfloat16 *>(g), y, rows, H, eps);
+  E3_CUDA_TRY(cudaGetLastError());
+  count_launch();
+  return E3_OK;
+}
+
+e3_status f32_swiglu_run(const float *g, const float *u, float *a, size_t n, cudaStream_t st) {
+  f32_swiglu_kernel<<<(unsigned)((n + 255) / 256 < 4096 ? (n + 255) / 256 : 4096), 256, 0, st>>>(g, u, a, n);
+  E3_CUDA_TRY(cudaGetLastError());
+  count_launch();
+  return E3_OK;
+}
+
+e3_status f32_rope_kv_run(const float *qkv, float *qo, float *kc, float *vc, const float2 *rope, const DecArgs &a,
+                          cudaStream_t st) {
+  f32_rope_kv_kernel<<<a.T, 64, 0, st>>>(qkv, qo, kc, vc, rope, a);
+  E3_CUDA_TRY(cudaGetLastError());
+  count_launch();
+  return E3_OK;
+}
+
+e3_status f32_attn_dec_run(const float *q, float *ctx, const float *kc, const float *vc, const DecArgs &a,
+                           cudaStream_t st) {
+  const size_t smem = (size_t)a.max_ctx * sizeof(float);
+  static size_t attr = 0;
+  if (smem > 48 * 1024 && smem > attr) {
+    E3_CUDA_TRY(cudaFuncSetAttribute(f32_attn_dec_kernel, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem));
+    attr = smem;
+  }
+  f32_attn_dec_kernel<<<dim3(a.nh, a.T), 128, smem, st>>>(q, ctx, kc, vc, a);
+  E3_CUDA_TRY(cudaGetLastError());
+  count_launch();
+  return E3_OK;
+}
 
 e3_status f32_gemm_run(const float *A, int lda, const void *W, const void *bias, const float *R, float *Y, int M,
                        int N, int K, int epi, cudaStream_t st) {

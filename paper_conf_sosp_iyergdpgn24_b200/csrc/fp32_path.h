@@ -13,6 +13,13 @@ e3_status f32_gemm_run(const float *A, int lda, const void *W, const void *bias,
 e3_status f32_attn_run(const float *qkv, float *ctx, int B, int S, int H, cudaStream_t st);
 e3_status f32_ln_run(const float *x, const void *g, const void *b, float *y, int rows, int H, float eps,
                      cudaStream_t st);
+// LLaMA decode pieces (DecArgs carries ids, n_valid, slots, positions, alive)
+e3_status f32_rms_run(const float *x, const void *g, float *y, int rows, int H, float eps, cudaStream_t st);
+e3_status f32_swiglu_run(const float *g, const float *u, float *a, size_t n, cudaStream_t st);
+e3_status f32_rope_kv_run(const float *qkv, float *qo, float *kc, float *vc, const float2 *rope, const DecArgs &a,
+                          cudaStream_t st);
+e3_status f32_attn_dec_run(const float *q, float *ctx, const float *kc, const float *vc, const DecArgs &a,
+                           cudaStream_t st);
 // RampArgs with x = fp32 rows [B,S,H] (post-LN for BERT; the ViT ramp applies its own LN)
 e3_status f32_ramp_run(const RampArgs &a, cudaStream_t st);
 

@@ -115,8 +115,12 @@ static bool aligned16(const void *p) { return (reinterpret_cast<uintptr_t>(p) & 
 // LLAMA decode: head_dim 128, one token per row (S = 1),
 // B in {32, 64, 128}, the caller's KV cache covering the split's layers.
 static e3_status llama_validate(const e3_split_desc *d, const e3_weights *w) {
-  if (d->dtype != E3_DTYPE_BF16) {
-    set_error("e3_split_create (LLAMA): only dtype BF16 is implemented");
+  if (d->dtype != E3_DTYPE_BF16 && d->dtype != E3_DTYPE_FP32) {
+    set_error("e3_split_create (LLAMA): dtype must be BF16 or FP32");
+    return E3_EUNSUPPORTED;
+  }
+  if (d->dtype == E3_DTYPE_FP32 && d->ffn > 3 * d->hidden) {
+    set_error("e3_split_create (LLAMA FP32): need F <= 3 H");
     return E3_EUNSUPPORTED;
   }
   const int kvh = d->kv_heads > 0 ? d->kv_heads : d->heads;
@@ -230,6 +234,8 @@ static e3_status llama_create(e3_split *s, const e3_weights *w) {
     s->kv_k.push_back(w->kv->k[l]);
     s->kv_v.push_back(w->kv->v[l]);
   }
+  if (d.dtype == E3_DTYPE_FP32)   // SIMT fp32 kernels: only the RoPE table
+    return ws.ensure_llama(V, 0, 0, w->kv->max_ctx, 128, 10000.0);
   s->mc_qkv = dec_max_contrib(nqkv, H, E3_DEC_QKV_ROPE, s->sms);
   s->mc_o = dec_max_contrib(H, H, E3_DEC_RESID, s->sms);
   s->mc_gu = dec_max_contrib(F, H, E3_DEC_SWIGLU, s->sms);
@@ -548,11 +554,43 @@ static e3_status f32_run(e3_split *s, cudaStream_t st, const void *x_in, const i
     r = (expr);                   \
     if (r != E3_OK) return r;     \
   } while (0)
+  const bool llama = d.arch == E3_ARCH_LLAMA_DECODE;
+  DecArgs da{};   // LLAMA: tokens, slots, positions (as the bf16 path's DecArgs)
+  if (llama) {
+    da.T = B;
+    da.nh = d.heads;
+    da.kvh = d.kv_heads > 0 ? d.kv_heads : d.heads;
+    da.max_ctx = s->kv.max_ctx;
+    da.ids = id_in;
+    da.n_valid_dev = n_valid_dev;
+    da.n_valid_host = n_valid_host;
+    da.slot_of_id = s->kv.slot_of_id;
+    da.id_cap = s->kv.id_capacity;
+    da.pos_of_slot = s->kv.pos_of_slot;
+    da.n_slots = s->kv.n_slots;
+    da.err = ws.err;
+  }
+  const int nqkv = llama ? (da.nh + 2 * da.kvh) * 128 : 3 * H;
   for (int i = 0; i < nl; ++i) {
     const int l = d.layer_begin + i;
     const e3_layer_weights &L = s->L[i];
     float *out = static_cast<float *>((i % 2 == 0) ? ws.xa : ws.xb);
-    if (vit) {   // n1 = LN1(x); y1 = x + attn(n1) W_o; n2 = LN2(y1); x2 = y1 + MLP(n2)
+    if (llama) {   // R22: n1 = RMSNorm1(x); q, k = RoPE; h = x + attn W_o; x' = h + SwiGLU(RMSNorm2(h)) W_down
+      DecArgs a = da;
+      a.alive = first_ramp ? nullptr : ws.alive;   // exited rows append no K/V (R15)
+      a.init_alive = first_ramp;
+      E3_RUN(f32_rms_run(cur, L.ln1_g, x1, B, H, d.norm_eps, st));
+      E3_RUN(f32_gemm_run(x1, H, L.w_qkv, nullptr, nullptr, qkv, B, nqkv, H, E3_EPI_BIAS, st));
+      float *kc = static_cast<float *>(s->kv_k[l]), *vc = static_cast<float *>(s->kv_v[l]);
+      E3_RUN(f32_rope_kv_run(qkv, ws.pool, kc, vc, ws.rope, a, st));
+      E3_RUN(f32_attn_dec_run(ws.pool, ctx, kc, vc, a, st));
+      E3_RUN(f32_gemm_run(ctx, H, L.w_o, nullptr, cur, y, B, H, H, E3_EPI_BIAS_RESID, st));
+      E3_RUN(f32_rms_run(y, L.ln2_g, x1, B, H, d.norm_eps, st));
+      E3_RUN(f32_gemm_run(x1, H, L.w_1, nullptr, nullptr, qkv, B, F, H, E3_EPI_BIAS, st));   // gate
+      E3_RUN(f32_gemm_run(x1, H, L.w_3, nullptr, nullptr, hb, B, F, H, E3_EPI_BIAS, st));    // up
+      E3_RUN(f32_swiglu_run(qkv, hb, hb, (size_t)B * F, st));
+      E3_RUN(f32_gemm_run(hb, F, L.w_2, nullptr, y, out, B, H, F, E3_EPI_BIAS_RESID, st));
+    } else if (vit) {   // n1 = LN1(x); y1 = x + attn(n1) W_o; n2 = LN2(y1); x2 = y1 + MLP(n2)
       E3_RUN(f32_ln_run(cur, L.ln1_g, L.ln1_b, x1, M, H, d.norm_eps, st));
       E3_RUN(f32_gemm_run(x1, H, L.w_qkv, L.b_qkv, nullptr, qkv, M, 3 * H, H, E3_EPI_BIAS, st));
       E3_RUN(f32_attn_run(qkv, ctx, B, S, H, st));
@@ -599,9 +637,8 @@ static e3_status f32_run(e3_split *s, cudaStream_t st, const void *x_in, const i
       ++ri;
     }
   }
-  // survivors: fp32 rows copied as 2H two-byte elements (no normalisation)
-  E3_RUN(ln_compact_run(cur, id_in, ws.alive, B, S, 2 * H, nullptr, nullptr, d.norm_eps, dst, n_surv_dev, s->sms,
-                        st));
+  // survivors: fp32 rows copied byte for byte (stable order)
+  E3_RUN(compact_run(cur, id_in, ws.alive, B, (int64_t)S * H * 4, dst, n_surv_dev, ws.ctr, s->sms, st));
 #undef E3_RUN
   return E3_OK;
 }
@@ -624,9 +661,9 @@ static LnGemmArgs oln_args(const void *bias, const void *R, const void *g, const
 e3_status split_run_to(e3_split *s, cudaStream_t st, const void *x_in, const int64_t *id_in,
                        const int32_t *n_valid_dev, int n_valid_host, const RingDst &dst, int32_t *n_surv_dev,
                        const e3_exits *ex) {
+  if (s->d.dtype == E3_DTYPE_FP32) return f32_run(s, st, x_in, id_in, n_valid_dev, n_valid_host, dst, n_surv_dev, ex);
   if (s->d.arch == E3_ARCH_LLAMA_DECODE)
     return llama_run(s, st, x_in, id_in, n_valid_dev, n_valid_host, dst, n_surv_dev, ex);
-  if (s->d.dtype == E3_DTYPE_FP32) return f32_run(s, st, x_in, id_in, n_valid_dev, n_valid_host, dst, n_surv_dev, ex);
   const e3_split_desc &d = s->d;
   Workspace &ws = *s->ws;
   const int B = d.batch, S = d.seq_len, H = d.hidden, F = d.ffn, M = B * S;

@@ -48,37 +48,11 @@ def encoder_case(api, cfg, n, dtype, modes):
 
 
 def llama_case(api, cfg, n, dtype, modes):
-    import torch
-    from oracle import llama as olm
-    tau = e3data.tau_for(cfg)
-    max_ctx = cfg.ctx + 1
-    slot_of = {i: i for i in range(n)}
-    pos_of = {s: cfg.ctx - (s % 5) for s in range(n)}
-    cache = api.KVCache(cfg, n, max_ctx, n, "cuda:0")
-    for l in range(cfg.layers):
-        k, v = e3data.make_kv(cfg, l, range(n), max_ctx)
-        cache.k[l].copy_(torch.from_numpy(k).to(torch.bfloat16))
-        cache.v[l].copy_(torch.from_numpy(v).to(torch.bfloat16))
-    cache.slot_of_id.copy_(torch.arange(n, dtype=torch.int32))
-    cache.pos_of_slot.copy_(torch.tensor([pos_of[s] for s in range(n)], dtype=torch.int32))
-    ramp = e3data.make_ramp(cfg, 0)
-    lazy = cfg.layers > 8
-    layers = pu.LazyLayers(cfg) if lazy else [e3data.make_layer(cfg, l) for l in range(cfg.layers)]
-    W = {"layers": layers, "ramps": [ramp] * cfg.n_ramps}
-    model = api.DeviceModel(cfg, {"layers": (layers[l] for l in range(cfg.layers)) if lazy else layers,
-                                  "ramps": W["ramps"]}, "cuda:0", kv=cache)
-    X = e3data.make_inputs(cfg, range(n), seed=5)
     t0 = time.time()
-    gpu = pu.run_gpu_pipeline(api, cfg, model, X, tau, dtype=dtype)
-    out = {"gpu_s": round(time.time() - t0, 1), "n_tokens": n, "positions": "ctx - (slot % 5)"}
-    del model, cache
-    torch.cuda.empty_cache()
+    gpu, recs = pu.llama_job(api, cfg, n, dtype, modes)
+    out = {"job_s": round(time.time() - t0, 1), "n_tokens": n, "positions": "ctx - (slot % 5)"}
     for mode in modes:
-        t0 = time.time()
-        kv = pu.LazyKV(cfg, range(n), max_ctx)
-        recs = olm.run(cfg, W, X[:, 0, :], list(range(n)), kv, slot_of, pos_of, tau=tau, mode=mode)
-        out[mode] = pu.compare(gpu, recs)
-        out[mode]["oracle_s"] = round(time.time() - t0, 1)
+        out[mode] = pu.compare(gpu, recs[mode])
     return out
 
 

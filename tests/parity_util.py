@@ -91,3 +91,39 @@ class LazyKV:
 
     def __getitem__(self, l):
         return e3data.make_kv(self.cfg, l, self.slots, self.max_ctx).astype(np.float64)
+
+
+def llama_job(api, cfg, n, dtype, modes=("bf16",), dev="cuda:0"):
+    """The decode step of n tokens through the whole calibrated per-ramp chain
+    (Llama-7B shape: 4 splits of 8 layers): GPU records and, per oracle mode,
+    oracle records.  Token i sits in KV slot i at position ctx - (i % 5); the
+    pre-filled caches come from e3data.make_kv (the same values on both sides,
+    fp32 caches for FP32 mode)."""
+    import torch
+    from oracle import llama as olm
+    tau = e3data.tau_for(cfg)
+    max_ctx = cfg.ctx + 1
+    slot_of = {i: i for i in range(n)}
+    pos_of = {s: cfg.ctx - (s % 5) for s in range(n)}
+    cache = api.KVCache(cfg, n, max_ctx, n, dev, dtype=dtype)
+    for l in range(cfg.layers):
+        k, v = e3data.make_kv(cfg, l, range(n), max_ctx)
+        cache.k[l].copy_(torch.from_numpy(k).to(cache.k[l].dtype))
+        cache.v[l].copy_(torch.from_numpy(v).to(cache.v[l].dtype))
+    cache.slot_of_id.copy_(torch.arange(n, dtype=torch.int32))
+    cache.pos_of_slot.copy_(torch.tensor([pos_of[s] for s in range(n)], dtype=torch.int32))
+    ramp = e3data.make_ramp(cfg, 0)
+    lazy = cfg.layers > 8
+    layers = LazyLayers(cfg) if lazy else [e3data.make_layer(cfg, l) for l in range(cfg.layers)]
+    W = {"layers": layers, "ramps": [ramp] * cfg.n_ramps}
+    model = api.DeviceModel(cfg, {"layers": (layers[l] for l in range(cfg.layers)) if lazy else layers,
+                                  "ramps": W["ramps"]}, dev, kv=cache)
+    X = e3data.make_inputs(cfg, range(n), seed=5)
+    gpu = run_gpu_pipeline(api, cfg, model, X, tau, dtype=dtype, dev=dev)
+    del model, cache
+    torch.cuda.empty_cache()
+    recs = {}
+    for mode in modes:
+        kv = LazyKV(cfg, range(n), max_ctx)
+        recs[mode] = olm.run(cfg, W, X[:, 0, :], list(range(n)), kv, slot_of, pos_of, tau=tau, mode=mode)
+    return gpu, recs

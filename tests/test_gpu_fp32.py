@@ -122,3 +122,23 @@ def test_fp32_plan_invariance_bitwise(api):
         api.Pipeline(model, api.make_plan(cfg, bounds, cfg.tau, dtype="fp32")).run(X, ids, ex)
         outs.append((ex.exit_layer.cpu(), ex.logits.cpu()))
     assert torch.equal(outs[0][0], outs[1][0]) and torch.equal(outs[0][1], outs[1][1])
+
+
+def test_fp32_tiny_llama_pipeline(api):
+    """LLaMA decode in FP32 (fp32 KV cache): 90 tokens at positions
+    ctx - (slot % 5) through the per-ramp plan vs the fp64 oracle."""
+    cfg = e3data.get("tiny-llama")
+    gpu, recs = pu.llama_job(api, cfg, 90, "fp32", ("fp64",))
+    _assert_job(gpu, recs["fp64"])
+
+
+def test_fp32_llama7b_calibrated_32_layer_chain(api):
+    """Llama-7B shape: 16 tokens through the calibrated 4-split, 32-layer
+    chain (ramps after layers 8/16/24/32, V = 32000) in FP32 vs the fp64
+    oracle: decisions exact at margin > 1e-3, logits within 1e-4."""
+    cfg = e3data.get("lm")
+    gpu, recs = pu.llama_job(api, cfg, 16, "fp32", ("fp64",))
+    st = pu.compare(gpu, recs["fp64"], MARGIN)
+    assert st["flips"] == 0, st
+    assert st["logit_err"]["max"] < LOGIT_TOL, st["logit_err"]
+    assert st["label_mismatch"] == 0
