@@ -208,17 +208,64 @@ e3_status e3_queue_count(e3_queue *q, int32_t *host_count);
 e3_status e3_rebatch(e3_queue *q, void *stream, int32_t B, int32_t flush, void *x_out, int64_t *id_out,
                      int32_t *n_valid_dev, int32_t *emitted);
 
+/* --------------------------------------------------------------- comm --- */
+
+/* Inter-split transfer: "Tx is the communication
+ * time for sending data from the end of a split to the next" (§3.2.1,
+ * PAPER.md:887-903); split outputs "are then directed to the machines hosting
+ * the next split" into "a queue that holds the partial results" (§3.3,
+ * PAPER.md:962-972).  One process per GPU; the communicator is owned by the
+ * library.
+ *   NCCL      ncclSend / ncclRecv over NVLink, one 2-rank communicator per
+ *             (sender, receiver) link split off the world communicator at
+ *             e3_pipeline_create (NCCL is resolved at run time from the
+ *             process's libnccl.so.2; E3_ENCCL if absent).
+ *   LOOPBACK  every rank of the plan lives in THIS process on one device
+ *             (tests and single-GPU runs of a multi-rank plan): a message is a
+ *             device-to-device copy matched by a host-side hub, with the same
+ *             ordering / EOS protocol as NCCL.
+ *   P2P       reserved (fused compaction -> peer-ring stores); E3_EUNSUPPORTED. */
+typedef enum { E3_TRANSPORT_NCCL = 0, E3_TRANSPORT_P2P = 1, E3_TRANSPORT_LOOPBACK = 2 } e3_transport;
+
+typedef struct e3_comm e3_comm;
+/* NCCL unique id, created on one rank and broadcast by the caller (e.g. over
+ * a torch process group) to every rank before e3_comm_init. */
+e3_status e3_comm_unique_id(uint8_t id[E3_COMM_ID_BYTES]);
+/* Collective over `world` ranks: the NCCL world communicator of this rank on
+ * `device`.  E3_ENCCL on any NCCL failure. */
+e3_status e3_comm_init(const uint8_t id[E3_COMM_ID_BYTES], int rank, int world, int device, e3_comm **out);
+/* LOOPBACK: `world` rank handles out[0..world-1] sharing one in-process hub on
+ * `device`.  Each handle is used by one thread at a time. */
+e3_status e3_comm_init_loopback(int world, int device, e3_comm **out);
+e3_status e3_comm_rank(const e3_comm *c, int32_t *rank, int32_t *world);
+/* Destroy every pipeline using the handle first. */
+e3_status e3_comm_destroy(e3_comm *c);
+
 /* ----------------------------------------------------------- pipeline --- */
+
+#define E3_MAX_REPLICA_SLOTS 256
 
 /* Split plan ("the apt number of splits ..., the number of resources to place
  * them, and the batch sizes to run the splits with"). */
 typedef struct e3_plan {
   int32_t n_splits;
   e3_split_desc split[E3_MAX_SPLITS];  /* contiguous: split[s+1].layer_begin == split[s].layer_end;
-                                          same model dims and batch in every split */
+                                          same model dims, batch and dtype in every split */
   int32_t lag;                         /* host look-behind: 0 serial, 1 (default)   */
   int32_t queue_cap_batches;           /* ring capacity per split in batches (>= 4) */
   int32_t trace;                       /* record dispatch order (e3_pipeline_trace) */
+  /* Placement (multi-GPU; all zero = every split on the calling rank):
+   * replicas[s] copies of split s; replica j of split s runs on comm rank
+   * device_of[off(s) + j], off(s) = sum_{t<s} replicas[t].  The splits a rank
+   * hosts must be contiguous and share one replica set (a STAGE); adjacent
+   * stages use disjoint ranks.  Stage g's replica i sends its k-th output
+   * batch to replica (i + k) mod r of stage g+1. */
+  int32_t replicas[E3_MAX_SPLITS];
+  int32_t device_of[E3_MAX_REPLICA_SLOTS];
+  int32_t transport;                   /* e3_transport (ignored on one rank)        */
+  int32_t deterministic;               /* 1: a receiver appends its senders' batches in
+                                          round-robin sender order (exact batch
+                                          composition); 0: in arrival order        */
 } e3_plan;
 
 typedef struct e3_stats {
@@ -230,35 +277,44 @@ typedef struct e3_stats {
   int64_t host_waits;                  /* times the host blocked on a run          */
   double host_launch_ms;               /* host time spent issuing runs (launches)  */
   double host_sync_ms;                 /* host time spent waiting on run events    */
+  int64_t msgs_sent, msgs_recv;        /* inter-stage data messages of this rank   */
+  int64_t flushes[E3_MAX_SPLITS];      /* padded (flush) batches per split          */
 } e3_stats;
 
 typedef struct e3_pipeline e3_pipeline;
-/* All splits of the plan on one GPU with local queues (the paper's base
- * formulation: "each GPU executes the splits sequentially").
- * Multi-GPU plans (replicas, or splits on different GPUs with survivors sent
- * over NVLink) are driven one rank per GPU from Python over torch.distributed
- * (paper_conf_sosp_iyergdpgn24_b200/parallel.py), each rank calling this API. */
-e3_status e3_pipeline_create(const e3_plan *p, const e3_weights *w, int device, e3_pipeline **out);
+/* SPMD: every rank of the plan calls it with the same plan (c == NULL: one
+ * rank, every split on `device` -- the paper's base formulation, "each GPU
+ * executes the splits sequentially").  With a communicator
+ * the rank creates only the splits it hosts (weights of other layers may be
+ * NULL) and, for NCCL, one link communicator per (sender, receiver) pair of
+ * adjacent stages (collective: all ranks must call).  `device` must equal the
+ * communicator's device. */
+e3_status e3_pipeline_create(const e3_plan *p, const e3_weights *w, int device, e3_comm *c, e3_pipeline **out);
 e3_status e3_pipeline_destroy(e3_pipeline *pl);
 /* Runs every input through the split chain until it exits.
- *   x    [n,S,H] bf16, ids [n] int64 (ids in [0, ex->capacity)).  Both may be
- *        DEVICE or HOST memory; host inputs are staged batch by batch on a
- *        copy stream (H2D copies overlap compute).
- *   ex   exit records (device arrays).
+ *   x    [n,S,H] activations (bf16, or fp32 for an FP32 plan), ids [n] int64
+ *        (ids in [0, ex->capacity)).  Both may be DEVICE or HOST memory; host
+ *        inputs are staged batch by batch on a copy stream (H2D copies
+ *        overlap compute).  Multi-rank: ranks hosting split 0 pass their own
+ *        share of the inputs, the others n = 0.
+ *   ex   exit records (device arrays) of the inputs exiting on THIS rank.
  * Blocks until all of this rank's work is done (returns with the stream idle).
  * Split 0 takes inputs in order, B at a time; every split runs exactly B rows
- * per batch; the deepest split holding >= B queued rows runs first; when no
- * queue is full and nothing upstream is pending, the shallowest non-empty
- * queue is flushed padded to B. */
+ * per batch; the deepest split holding >= B queued rows runs first; a queue
+ * is flushed (padded to B) only when nothing upstream of it can still
+ * deliver rows -- for the first split of a stage, after every sender's
+ * end-of-stream message.  Survivors of a stage's
+ * last split travel to the next stage as fixed-size messages [n, flag | B ids
+ * | B rows] (a rank's link buffers are reused only after the transfer
+ * completed); the host loop never blocks on a transfer while it has a run to
+ * issue. */
 e3_status e3_pipeline_run(e3_pipeline *pl, void *stream, const void *x, const int64_t *ids, int64_t n,
                           const e3_exits *ex, e3_stats *st);
-/* One STAGE of a multi-GPU stage pipeline: like e3_pipeline_run, for a plan
- * whose last split does not hold the model's final ramp.  The survivors of
- * that last split are appended in dispatch order (stable within each run) to
- * x_out / id_out (device, capacity out_cap rows; E3_ECAPACITY beyond it) and
- * *n_out (host) receives their number -- the rows the next stage's GPU must
- * receive ("outputs are then directed to the machines
- * hosting the next split"). */
+/* A plan truncated before the model's final ramp (single rank): like
+ * e3_pipeline_run, the survivors of the plan's last split are appended in
+ * dispatch order (stable within each run) to x_out / id_out (device,
+ * capacity out_cap rows; E3_ECAPACITY beyond it) and *n_out (host) receives
+ * their number. */
 e3_status e3_pipeline_run_out(e3_pipeline *pl, void *stream, const void *x, const int64_t *ids, int64_t n,
                               const e3_exits *ex, e3_stats *st, void *x_out, int64_t *id_out, int64_t out_cap,
                               int64_t *n_out);

@@ -14,6 +14,8 @@ LIB_PATH = os.environ.get("E3_LIB_PATH") or os.path.join(HERE, "libe3.so")   # o
 
 E3_MAX_RAMPS = 64
 E3_MAX_SPLITS = 64
+E3_MAX_REPLICA_SLOTS = 256
+E3_COMM_ID_BYTES = 128
 
 STATUS = {0: "E3_OK", 1: "E3_EINVAL", 2: "E3_EUNSUPPORTED", 3: "E3_ECUDA", 4: "E3_ENCCL",
           5: "E3_ECAPACITY", 6: "E3_ESTATE"}
@@ -23,6 +25,7 @@ TEST = {"maxprob": 0, "entropy": 1}
 INNER = {"exact": 0, "disabled": 1}
 DTYPE = {"bf16": 0, "fp32": 1}
 EPI = {"bias": 0, "bias_gelu": 1, "bias_resid": 2}
+TRANSPORT = {"nccl": 0, "p2p": 1, "loopback": 2}
 
 P = C.c_void_p
 I32 = C.c_int32
@@ -71,13 +74,15 @@ class Exits(C.Structure):
 
 class Plan(C.Structure):
     _fields_ = [("n_splits", I32), ("split", SplitDesc * E3_MAX_SPLITS), ("lag", I32),
-                ("queue_cap_batches", I32), ("trace", I32)]
+                ("queue_cap_batches", I32), ("trace", I32), ("replicas", I32 * E3_MAX_SPLITS),
+                ("device_of", I32 * E3_MAX_REPLICA_SLOTS), ("transport", I32), ("deterministic", I32)]
 
 
 class Stats(C.Structure):
     _fields_ = [("runs", I64), ("batches", I64 * E3_MAX_SPLITS), ("valid_rows", I64 * E3_MAX_SPLITS),
                 ("padded_rows", I64 * E3_MAX_SPLITS), ("rows_out", I64 * E3_MAX_SPLITS),
-                ("host_waits", I64), ("host_launch_ms", C.c_double), ("host_sync_ms", C.c_double)]
+                ("host_waits", I64), ("host_launch_ms", C.c_double), ("host_sync_ms", C.c_double),
+                ("msgs_sent", I64), ("msgs_recv", I64), ("flushes", I64 * E3_MAX_SPLITS)]
 
 
 # name -> (restype, argtypes); every symbol include/*.h declares
@@ -92,7 +97,12 @@ SIGNATURES = {
     "e3_queue_push": (I32, [P, P, P, P, P, I32]),
     "e3_queue_count": (I32, [P, C.POINTER(I32)]),
     "e3_rebatch": (I32, [P, P, I32, I32, P, P, P, C.POINTER(I32)]),
-    "e3_pipeline_create": (I32, [C.POINTER(Plan), C.POINTER(Weights), C.c_int, C.POINTER(P)]),
+    "e3_comm_unique_id": (I32, [C.c_char_p]),
+    "e3_comm_init": (I32, [C.c_char_p, C.c_int, C.c_int, C.c_int, C.POINTER(P)]),
+    "e3_comm_init_loopback": (I32, [C.c_int, C.c_int, C.POINTER(P)]),
+    "e3_comm_rank": (I32, [P, C.POINTER(I32), C.POINTER(I32)]),
+    "e3_comm_destroy": (I32, [P]),
+    "e3_pipeline_create": (I32, [C.POINTER(Plan), C.POINTER(Weights), C.c_int, P, C.POINTER(P)]),
     "e3_pipeline_destroy": (I32, [P]),
     "e3_pipeline_run": (I32, [P, P, P, P, I64, C.POINTER(Exits), C.POINTER(Stats)]),
     "e3_pipeline_run_out": (I32, [P, P, P, P, I64, C.POINTER(Exits), C.POINTER(Stats), P, P, I64,

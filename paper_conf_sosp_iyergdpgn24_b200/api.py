@@ -7,6 +7,7 @@ runs in libe3.so.  Names follow the C ABI (include/e3.h):
     split_desc       e3_split_desc for layers [begin, end) of a model
     Split            e3_split_create / e3_split_run
     Queue            e3_queue_* and e3_rebatch
+    Comm             e3_comm_* (NCCL world communicator, or an in-process loopback set)
     Pipeline         e3_pipeline_create / e3_pipeline_run / e3_pipeline_trace
     ExitBuffers      device arrays of exit records indexed by input id
     ops              kernel-level entry points (e3_ops.h)
@@ -204,8 +205,12 @@ class Queue:
 
 
 def make_plan(cfg, bounds: Sequence[int], tau, batch=None, inner="exact", lag=1,
-              queue_cap_batches=4, trace=False, dtype="bf16") -> _lib.Plan:
-    """Plan with split s covering layers [bounds[s], bounds[s+1])."""
+              queue_cap_batches=4, trace=False, dtype="bf16", placement=None, transport="nccl",
+              deterministic=False) -> _lib.Plan:
+    """Plan with split s covering layers [bounds[s], bounds[s+1]).
+
+    placement: None (every split on the calling rank) or, per split, the list
+    of communicator ranks hosting its replicas (e3_plan.replicas/device_of)."""
     p = _lib.Plan()
     p.n_splits = len(bounds) - 1
     for s in range(p.n_splits):
@@ -213,24 +218,76 @@ def make_plan(cfg, bounds: Sequence[int], tau, batch=None, inner="exact", lag=1,
     p.lag = lag
     p.queue_cap_batches = queue_cap_batches
     p.trace = int(trace)
+    if placement is not None:
+        assert len(placement) == p.n_splits
+        off = 0
+        for s, ranks in enumerate(placement):
+            p.replicas[s] = len(ranks)
+            for j, r in enumerate(ranks):
+                p.device_of[off + j] = int(r)
+            off += len(ranks)
+    p.transport = _lib.TRANSPORT[transport]
+    p.deterministic = int(deterministic)
     return p
 
 
-class Pipeline:
-    """All splits of a plan on one GPU (e3_pipeline_*)."""
+class Comm:
+    """e3_comm: the library-owned communicator of one rank.
 
-    def __init__(self, model: DeviceModel, plan: _lib.Plan):
-        self.model, self.plan = model, plan
+    Comm.unique_id() on one rank, broadcast the bytes (torch.distributed), then
+    Comm.nccl(uid, rank, world, device) on every rank; or Comm.loopback(world,
+    device) for every rank of a plan inside this process (one device)."""
+
+    def __init__(self, handle):
+        self.h = handle
+
+    @staticmethod
+    def unique_id() -> bytes:
+        buf = C.create_string_buffer(_lib.E3_COMM_ID_BYTES)
+        check(lib.e3_comm_unique_id(buf), "e3_comm_unique_id")
+        return buf.raw
+
+    @classmethod
+    def nccl(cls, uid: bytes, rank: int, world: int, device: int) -> "Comm":
+        h = C.c_void_p()
+        check(lib.e3_comm_init(C.create_string_buffer(uid, _lib.E3_COMM_ID_BYTES), rank, world, device,
+                               C.byref(h)), "e3_comm_init")
+        return cls(h)
+
+    @classmethod
+    def loopback(cls, world: int, device: int = 0) -> List["Comm"]:
+        hs = (C.c_void_p * world)()
+        check(lib.e3_comm_init_loopback(world, device, hs), "e3_comm_init_loopback")
+        return [cls(C.c_void_p(hs[i])) for i in range(world)]
+
+    def rank_world(self):
+        r, w = C.c_int32(), C.c_int32()
+        check(lib.e3_comm_rank(self.h, C.byref(r), C.byref(w)), "e3_comm_rank")
+        return r.value, w.value
+
+    def close(self):
+        if getattr(self, "h", None) and _lib is not None and _lib.lib is not None:
+            _lib.lib.e3_comm_destroy(self.h)
+            self.h = None
+
+
+class Pipeline:
+    """The splits of a plan this rank hosts (e3_pipeline_*): all of them on one
+    GPU, or this rank's stage of a multi-rank plan (comm given)."""
+
+    def __init__(self, model: DeviceModel, plan: _lib.Plan, comm: Optional[Comm] = None):
+        self.model, self.plan, self.comm = model, plan, comm
         h = C.c_void_p()
         check(lib.e3_pipeline_create(C.byref(plan), C.byref(model.c_weights), model.device.index or 0,
-                                     C.byref(h)), "e3_pipeline_create")
+                                     comm.h if comm is not None else None, C.byref(h)), "e3_pipeline_create")
         self.h = h
         self.B = plan.split[0].batch
 
     def run(self, x, ids, exits: ExitBuffers, stream=None) -> _lib.Stats:
-        """x [n,S,H] bf16 and ids [n] int64, both on the device or both on the host."""
+        """x [n,S,H] and ids [n] int64, both on the device or both on the host
+        (x None / ids None: no inputs on this rank)."""
         st = _lib.Stats()
-        n = int(ids.shape[0])
+        n = int(ids.shape[0]) if ids is not None else 0
         check(lib.e3_pipeline_run(self.h, _stream(stream), _ptr(x) if n else None,
                                   _ptr(ids) if n else None, n, C.byref(exits.c), C.byref(st)),
               "e3_pipeline_run")

@@ -7,8 +7,11 @@
 // oracle sees the same numbers).  Paper precision is unstated.
 //
 // This mode exists to prove the chained pipeline at tight bounds; its kernels
-// are plain SIMT (fp32 FMA, fixed summation order, no atomics in any value
-// path, so rows are batch-position invariant like the bf16 path):
+// are plain SIMT with fp32 STORAGE of every activation and fp64 accumulation
+// of every dot product / reduction (an fp32 x bf16 product is exact in fp64;
+// over 32 LLaMA layers fp32 accumulation alone drifted 3e-4 in the logits),
+// fixed summation order, no atomics in any value path, so rows are
+// batch-position invariant like the bf16 path:
 //   f32_gemm_kernel    Y = epi(A W^T + b): 128 x 128 CTA tile, 8 x 8 per
 //                      thread, K in steps of 16 staged in shared memory
 //   f32_attn_kernel    one CTA per (input, head): K, V of the head in shared
@@ -38,11 +41,11 @@ __global__ void __launch_bounds__(kGT)
   const int tid = threadIdx.x;
   const int m0 = blockIdx.y * kBM, n0 = blockIdx.x * kBN;
   const int ty = tid / 16, tx = tid % 16;
-  float acc[8][8];
+  double acc[8][8];   // fp64 accumulation: fp32 x bf16 products are exact in fp64
 #pragma unroll
   for (int i = 0; i < 8; ++i)
 #pragma unroll
-    for (int j = 0; j < 8; ++j) acc[i][j] = 0.f;
+    for (int j = 0; j < 8; ++j) acc[i][j] = 0.0;
   for (int k0 = 0; k0 < K; k0 += kBK) {
 #pragma unroll
     for (int u = 0; u < 2; ++u) {   // A tile: 128 rows x 16 k as float4
@@ -77,7 +80,7 @@ __global__ void __launch_bounds__(kGT)
 #pragma unroll
       for (int i = 0; i < 8; ++i)
 #pragma unroll
-        for (int j = 0; j < 8; ++j) acc[i][j] = fmaf(a[i], b[j], acc[i][j]);
+        for (int j = 0; j < 8; ++j) acc[i][j] = fma((double)a[i], (double)b[j], acc[i][j]);
     }
     __syncthreads();
   }
@@ -89,10 +92,10 @@ __global__ void __launch_bounds__(kGT)
     for (int j = 0; j < 8; ++j) {
       const int c = n0 + tx * 8 + j;
       if (c >= N) continue;
-      float v = acc[i][j] + (bias ? bf2f(bias[c]) : 0.f);
-      if (EPI == E3_EPI_BIAS_GELU) v = gelu_erf(v);
-      if (EPI == E3_EPI_BIAS_RESID) v += R[(size_t)r * N + c];
-      Y[(size_t)r * N + c] = v;
+      double v = acc[i][j] + (bias ? (double)bf2f(bias[c]) : 0.0);
+      if (EPI == E3_EPI_BIAS_GELU) v = 0.5 * v * (1.0 + erf(v * 0.70710678118654752440));
+      if (EPI == E3_EPI_BIAS_RESID) v += (double)R[(size_t)r * N + c];
+      Y[(size_t)r * N + c] = (float)v;
     }
   }
 }
@@ -103,11 +106,11 @@ constexpr int kAW = kAT / 32;
 // ctx[b, i, h*64 + d] = sum_j softmax_j(q_i . k_j / 8) v_j[d] for the head h
 __global__ void __launch_bounds__(kAT) f32_attn_kernel(const float *__restrict__ qkv, float *__restrict__ ctx, int S,
                                                        int H) {
-  extern __shared__ float sm[];
-  float *Ks = sm;                       // [S][65] (padded: lane j reads key row j)
+  extern __shared__ double smd[];
+  double *Ps = smd;                     // [warps][S] scores / probabilities (fp64)
+  float *Ks = reinterpret_cast<float *>(Ps + (size_t)kAW * S);   // [S][65] (padded: lane j reads key row j)
   float *Vs = Ks + (size_t)S * 65;      // [S][64]
   float *Qs = Vs + (size_t)S * 64;      // [warps][64]
-  float *Ps = Qs + kAW * 64;            // [warps][S]
   const int b = blockIdx.x / (H / 64), h = blockIdx.x % (H / 64);
   const float *base = qkv + (size_t)b * S * 3 * H;
   for (int idx = threadIdx.x; idx < S * 64; idx += kAT) {
@@ -117,40 +120,41 @@ __global__ void __launch_bounds__(kAT) f32_attn_kernel(const float *__restrict__
   }
   __syncthreads();
   const int warp = warp_id(), lane = lane_id();
-  float *q = Qs + warp * 64, *p = Ps + (size_t)warp * S;
+  float *q = Qs + warp * 64;
+  double *p = Ps + (size_t)warp * S;
   for (int i = warp; i < S; i += kAW) {
     q[lane] = base[(size_t)i * 3 * H + h * 64 + lane];
     q[lane + 32] = base[(size_t)i * 3 * H + h * 64 + lane + 32];
     __syncwarp();
-    float mx = -INFINITY;
+    double mx = -INFINITY;
     for (int j = lane; j < S; j += 32) {
-      float s = 0.f;
+      double s = 0.0;
 #pragma unroll 16
-      for (int d = 0; d < 64; ++d) s = fmaf(q[d], Ks[j * 65 + d], s);
-      s *= 0.125f;   // 1 / sqrt(64), exact
+      for (int d = 0; d < 64; ++d) s = fma((double)q[d], (double)Ks[j * 65 + d], s);
+      s *= 0.125;   // 1 / sqrt(64), exact
       p[j] = s;
-      mx = fmaxf(mx, s);
+      mx = fmax(mx, s);
     }
 #pragma unroll
-    for (int o = 16; o; o >>= 1) mx = fmaxf(mx, __shfl_xor_sync(0xffffffffu, mx, o));
-    float l = 0.f;
+    for (int o = 16; o; o >>= 1) mx = fmax(mx, __shfl_xor_sync(0xffffffffu, mx, o));
+    double l = 0.0;
     for (int j = lane; j < S; j += 32) {
-      const float e = expf(p[j] - mx);
+      const double e = exp(p[j] - mx);
       p[j] = e;
       l += e;
     }
 #pragma unroll
     for (int o = 16; o; o >>= 1) l += __shfl_xor_sync(0xffffffffu, l, o);
     __syncwarp();
-    float o0 = 0.f, o1 = 0.f;
+    double o0 = 0.0, o1 = 0.0;
     for (int j = 0; j < S; ++j) {
-      const float pj = p[j];
-      o0 = fmaf(pj, Vs[j * 64 + lane], o0);
-      o1 = fmaf(pj, Vs[j * 64 + lane + 32], o1);
+      const double pj = p[j];
+      o0 = fma(pj, (double)Vs[j * 64 + lane], o0);
+      o1 = fma(pj, (double)Vs[j * 64 + lane + 32], o1);
     }
     float *out = ctx + ((size_t)b * S + i) * H + h * 64;
-    out[lane] = o0 / l;
-    out[lane + 32] = o1 / l;
+    out[lane] = (float)(o0 / l);
+    out[lane + 32] = (float)(o1 / l);
     __syncwarp();
   }
 }
@@ -161,24 +165,30 @@ __device__ __forceinline__ float warp_sum(float v) {
   return v;
 }
 
-// y = (x - mean) / sqrt(var + eps) * g + b per row, biased variance
+__device__ __forceinline__ double warp_sumd(double v) {
+#pragma unroll
+  for (int o = 16; o; o >>= 1) v += __shfl_xor_sync(0xffffffffu, v, o);
+  return v;
+}
+
+// y = (x - mean) / sqrt(var + eps) * g + b per row, biased variance (fp64 sums)
 __global__ void __launch_bounds__(256) f32_ln_kernel(const float *__restrict__ x, const __nv_bfloat16 *__restrict__ g,
                                                      const __nv_bfloat16 *__restrict__ bb, float *__restrict__ y,
                                                      int rows, int H, float eps) {
   const int row = blockIdx.x * 8 + warp_id(), lane = lane_id();
   if (row >= rows) return;
   const float *xr = x + (size_t)row * H;
-  float s = 0.f;
+  double s = 0.0;
   for (int k = lane; k < H; k += 32) s += xr[k];
-  const float mean = warp_sum(s) / (float)H;
-  float q = 0.f;
+  const double mean = warp_sumd(s) / H;
+  double q = 0.0;
   for (int k = lane; k < H; k += 32) {
-    const float d = xr[k] - mean;
-    q = fmaf(d, d, q);
+    const double d = xr[k] - mean;
+    q = fma(d, d, q);
   }
-  const float rstd = 1.0f / sqrtf(warp_sum(q) / (float)H + eps);
+  const double rstd = 1.0 / sqrt(warp_sumd(q) / H + (double)eps);
   float *yr = y + (size_t)row * H;
-  for (int k = lane; k < H; k += 32) yr[k] = (xr[k] - mean) * rstd * bf2f(g[k]) + bf2f(bb[k]);
+  for (int k = lane; k < H; k += 32) yr[k] = (float)((xr[k] - mean) * rstd * bf2f(g[k]) + bf2f(bb[k]));
 }
 
 constexpr int kRT = 256;
@@ -192,7 +202,7 @@ __global__ void __launch_bounds__(kRT) f32_ramp_kernel(RampArgs a) {
   float *c = rs;          // [H] CLS row (ViT: normalised)
   float *p = c + H;       // [H] pooler output (BERT)
   float *z = p + H;       // [C] logits
-  __shared__ float red[kRT / 32][3];
+  __shared__ double red[kRT / 32][3];
   __shared__ int redi[kRT / 32];
   const int b = blockIdx.x, tid = threadIdx.x, warp = warp_id(), lane = lane_id();
   const int n_valid = a.n_valid_dev ? *a.n_valid_dev : a.n_valid_host;
@@ -207,32 +217,32 @@ __global__ void __launch_bounds__(kRT) f32_ramp_kernel(RampArgs a) {
   const bool vit = a.arch == E3_ARCH_VIT;
   if (a.arch == E3_ARCH_LLAMA_DECODE) {   // nf = RMSNorm_f(c) (R22)
     if (warp == 0) {
-      float q = 0.f;
-      for (int k = lane; k < H; k += 32) q = fmaf(c[k], c[k], q);
-      const float r = 1.0f / sqrtf(warp_sum(q) / (float)H + a.eps);
+      double q = 0.0;
+      for (int k = lane; k < H; k += 32) q = fma((double)c[k], (double)c[k], q);
+      const double r = 1.0 / sqrt(warp_sumd(q) / H + (double)a.eps);
       const __nv_bfloat16 *g = reinterpret_cast<const __nv_bfloat16 *>(a.w.ln_g);
-      for (int k = lane; k < H; k += 32) p[k] = c[k] * r * bf2f(g[k]);
+      for (int k = lane; k < H; k += 32) p[k] = (float)(c[k] * r * bf2f(g[k]));
     }
   } else if (vit) {   // n = LN_r(c)
     if (warp == 0) {
-      float s = 0.f;
+      double s = 0.0;
       for (int k = lane; k < H; k += 32) s += c[k];
-      const float mean = warp_sum(s) / (float)H;
-      float q = 0.f;
-      for (int k = lane; k < H; k += 32) q = fmaf(c[k] - mean, c[k] - mean, q);
-      const float rstd = 1.0f / sqrtf(warp_sum(q) / (float)H + a.eps);
+      const double mean = warp_sumd(s) / H;
+      double q = 0.0;
+      for (int k = lane; k < H; k += 32) q = fma(c[k] - mean, c[k] - mean, q);
+      const double rstd = 1.0 / sqrt(warp_sumd(q) / H + (double)a.eps);
       const __nv_bfloat16 *g = reinterpret_cast<const __nv_bfloat16 *>(a.w.ln_g);
       const __nv_bfloat16 *bb = reinterpret_cast<const __nv_bfloat16 *>(a.w.ln_b);
-      for (int k = lane; k < H; k += 32) p[k] = (c[k] - mean) * rstd * bf2f(g[k]) + bf2f(bb[k]);
+      for (int k = lane; k < H; k += 32) p[k] = (float)((c[k] - mean) * rstd * bf2f(g[k]) + bf2f(bb[k]));
     }
   } else {     // p = tanh(W_p c + b_p): a warp per output, lanes over k
     const __nv_bfloat16 *wp = reinterpret_cast<const __nv_bfloat16 *>(a.w.w_p);
     const __nv_bfloat16 *bp = reinterpret_cast<const __nv_bfloat16 *>(a.w.b_p);
     for (int o = warp; o < H; o += kRT / 32) {
-      float s = 0.f;
-      for (int k = lane; k < H; k += 32) s = fmaf(bf2f(wp[(size_t)o * H + k]), c[k], s);
-      s = warp_sum(s);
-      if (lane == 0) p[o] = tanhf(s + bf2f(bp[o]));
+      double s = 0.0;
+      for (int k = lane; k < H; k += 32) s = fma((double)bf2f(wp[(size_t)o * H + k]), (double)c[k], s);
+      s = warp_sumd(s);
+      if (lane == 0) p[o] = (float)tanh(s + bf2f(bp[o]));
     }
   }
   __syncthreads();
@@ -240,21 +250,21 @@ __global__ void __launch_bounds__(kRT) f32_ramp_kernel(RampArgs a) {
     const __nv_bfloat16 *wc = reinterpret_cast<const __nv_bfloat16 *>(a.w.w_c);
     const __nv_bfloat16 *bc = reinterpret_cast<const __nv_bfloat16 *>(a.w.b_c);
     for (int o = warp; o < C; o += kRT / 32) {
-      float s = 0.f;
-      for (int k = lane; k < H; k += 32) s = fmaf(bf2f(wc[(size_t)o * H + k]), p[k], s);
-      s = warp_sum(s);
-      if (lane == 0) z[o] = s + (bc ? bf2f(bc[o]) : 0.f);
+      double s = 0.0;
+      for (int k = lane; k < H; k += 32) s = fma((double)bf2f(wc[(size_t)o * H + k]), (double)p[k], s);
+      s = warp_sumd(s);
+      if (lane == 0) z[o] = (float)(s + (bc ? bf2f(bc[o]) : 0.f));
     }
   }
   __syncthreads();
   // max and argmax (lowest index on ties, R12)
-  float m = -INFINITY;
+  double m = -INFINITY;
   int arg = 0x7fffffff;
   for (int k = tid; k < C; k += kRT)
     if (z[k] > m) { m = z[k]; arg = k; }   // k ascending per thread: first max kept
 #pragma unroll
   for (int o = 16; o; o >>= 1) {
-    const float m2 = __shfl_xor_sync(0xffffffffu, m, o);
+    const double m2 = __shfl_xor_sync(0xffffffffu, m, o);
     const int a2 = __shfl_xor_sync(0xffffffffu, arg, o);
     if (m2 > m || (m2 == m && a2 < arg)) { m = m2; arg = a2; }
   }
@@ -270,29 +280,29 @@ __global__ void __launch_bounds__(kRT) f32_ramp_kernel(RampArgs a) {
   __syncthreads();
   m = red[0][0];
   const int label = redi[0];
-  float se = 0.f, sq = 0.f;
+  double se = 0.0, sq = 0.0;
   for (int k = tid; k < C; k += kRT) {
-    const float e = expf(z[k] - m);
+    const double e = exp((double)z[k] - m);
     se += e;
-    sq = fmaf(e, z[k] - m, sq);
+    sq = fma(e, (double)z[k] - m, sq);
   }
-  se = warp_sum(se);
-  sq = warp_sum(sq);
+  se = warp_sumd(se);
+  sq = warp_sumd(sq);
   __syncthreads();
   if (lane == 0) { red[warp][1] = se; red[warp][2] = sq; }
   __syncthreads();
   __shared__ int s_exit;
   __shared__ int64_t s_id;
   if (tid == 0) {
-    float sum = 0.f, qz = 0.f;
+    double sum = 0.0, qz = 0.0;
     for (int w = 0; w < kRT / 32; ++w) { sum += red[w][1]; qz += red[w][2]; }
     float metric;
     bool pass;
-    if (a.test == E3_TEST_MAXPROB) {
-      metric = 1.0f / sum;
+    if (a.test == E3_TEST_MAXPROB) {   // the metric is reported (and tested) as fp32
+      metric = (float)(1.0 / sum);
       pass = metric > a.tau;
     } else {
-      metric = logf(sum) - qz / sum;
+      metric = (float)(log(sum) - qz / sum);
       pass = metric < a.tau;
     }
     const bool exit_now = pass || a.final_ramp;
@@ -324,19 +334,19 @@ __global__ void __launch_bounds__(256) f32_rms_kernel(const float *__restrict__ 
   const int row = blockIdx.x * 8 + warp_id(), lane = lane_id();
   if (row >= rows) return;
   const float *xr = x + (size_t)row * H;
-  float q = 0.f;
-  for (int k = lane; k < H; k += 32) q = fmaf(xr[k], xr[k], q);
-  const float r = 1.0f / sqrtf(warp_sum(q) / (float)H + eps);
+  double q = 0.0;
+  for (int k = lane; k < H; k += 32) q = fma((double)xr[k], (double)xr[k], q);
+  const double r = 1.0 / sqrt(warp_sumd(q) / H + (double)eps);
   float *yr = y + (size_t)row * H;
-  for (int k = lane; k < H; k += 32) yr[k] = xr[k] * r * bf2f(g[k]);
+  for (int k = lane; k < H; k += 32) yr[k] = (float)(xr[k] * r * bf2f(g[k]));
 }
 
 // a = SiLU(g) * u elementwise
 __global__ void f32_swiglu_kernel(const float *__restrict__ g, const float *__restrict__ u, float *__restrict__ a,
                                   size_t n) {
   for (size_t i = blockIdx.x * (size_t)blockDim.x + threadIdx.x; i < n; i += (size_t)gridDim.x * blockDim.x) {
-    const float x = g[i];
-    a[i] = x / (1.0f + expf(-x)) * u[i];
+    const double x = g[i];
+    a[i] = (float)(x / (1.0 + exp(-x)) * u[i]);
   }
 }
 
@@ -366,19 +376,20 @@ __global__ void f32_rope_kv_kernel(const float *__restrict__ qkv, float *__restr
   }
   const int ld = (a.nh + 2 * a.kvh) * 128;
   const float *row = qkv + (size_t)t * ld;
-  const float2 cs = rope[(size_t)pos * 64 + j];
+  const float2 csf = rope[(size_t)pos * 64 + j];
+  const double2 cs = make_double2(csf.x, csf.y);
   for (int h = 0; h < a.nh; ++h) {
     const float lo = row[h * 128 + j], hi = row[h * 128 + j + 64];
-    qo[(size_t)t * a.nh * 128 + h * 128 + j] = lo * cs.x - hi * cs.y;
-    qo[(size_t)t * a.nh * 128 + h * 128 + j + 64] = hi * cs.x + lo * cs.y;
+    qo[(size_t)t * a.nh * 128 + h * 128 + j] = (float)(lo * cs.x - hi * cs.y);
+    qo[(size_t)t * a.nh * 128 + h * 128 + j + 64] = (float)(hi * cs.x + lo * cs.y);
   }
   if (slot < 0) return;
   for (int h = 0; h < a.kvh; ++h) {
     const float lo = row[(a.nh + h) * 128 + j], hi = row[(a.nh + h) * 128 + j + 64];
     float *kd = kc + (((size_t)slot * a.kvh + h) * a.max_ctx + pos) * 128;
     float *vd = vc + (((size_t)slot * a.kvh + h) * a.max_ctx + pos) * 128;
-    kd[j] = lo * cs.x - hi * cs.y;
-    kd[j + 64] = hi * cs.x + lo * cs.y;
+    kd[j] = (float)(lo * cs.x - hi * cs.y);
+    kd[j + 64] = (float)(hi * cs.x + lo * cs.y);
     vd[j] = row[(a.nh + a.kvh + h) * 128 + j];
     vd[j + 64] = row[(a.nh + a.kvh + h) * 128 + j + 64];
   }
@@ -388,9 +399,9 @@ __global__ void f32_rope_kv_kernel(const float *__restrict__ qkv, float *__restr
 __global__ void __launch_bounds__(128) f32_attn_dec_kernel(const float *__restrict__ q, float *__restrict__ ctx,
                                                            const float *__restrict__ kc, const float *__restrict__ vc,
                                                            DecArgs a) {
-  extern __shared__ float sp[];   // [max_ctx]
+  extern __shared__ double sp[];   // [max_ctx]
   __shared__ float qs[128];
-  __shared__ float red[4];
+  __shared__ double red[4];
   const int h = blockIdx.x, t = blockIdx.y, tid = threadIdx.x, warp = warp_id(), lane = lane_id();
   const int nv = a.n_valid_dev ? *a.n_valid_dev : a.n_valid_host;
   const int64_t id = a.ids[t];
@@ -409,34 +420,34 @@ __global__ void __launch_bounds__(128) f32_attn_dec_kernel(const float *__restri
   __syncthreads();
   const float *K = kc + ((size_t)slot * a.kvh + g) * a.max_ctx * 128;
   const float *V = vc + ((size_t)slot * a.kvh + g) * a.max_ctx * 128;
-  const float scale = 1.0f / sqrtf(128.0f);
-  float mx = -INFINITY;
+  const double scale = 1.0 / sqrt(128.0);
+  double mx = -INFINITY;
   for (int p = tid; p <= pos; p += 128) {
-    float s = 0.f;
-    for (int d = 0; d < 128; ++d) s = fmaf(qs[d], K[(size_t)p * 128 + d], s);
+    double s = 0.0;
+    for (int d = 0; d < 128; ++d) s = fma((double)qs[d], (double)K[(size_t)p * 128 + d], s);
     s *= scale;
     sp[p] = s;
-    mx = fmaxf(mx, s);
+    mx = fmax(mx, s);
   }
 #pragma unroll
-  for (int o = 16; o; o >>= 1) mx = fmaxf(mx, __shfl_xor_sync(0xffffffffu, mx, o));
+  for (int o = 16; o; o >>= 1) mx = fmax(mx, __shfl_xor_sync(0xffffffffu, mx, o));
   if (lane == 0) red[warp] = mx;
   __syncthreads();
-  mx = fmaxf(fmaxf(red[0], red[1]), fmaxf(red[2], red[3]));
+  mx = fmax(fmax(red[0], red[1]), fmax(red[2], red[3]));
   __syncthreads();
-  float l = 0.f;
+  double l = 0.0;
   for (int p = tid; p <= pos; p += 128) {
-    const float e = expf(sp[p] - mx);
+    const double e = exp(sp[p] - mx);
     sp[p] = e;
     l += e;
   }
-  l = warp_sum(l);
+  l = warp_sumd(l);
   if (lane == 0) red[warp] = l;
   __syncthreads();
   l = red[0] + red[1] + red[2] + red[3];
-  float o = 0.f;
-  for (int p = 0; p <= pos; ++p) o = fmaf(sp[p], V[(size_t)p * 128 + tid], o);
-  out[tid] = o / l;
+  double o = 0.0;
+  for (int p = 0; p <= pos; ++p) o = fma(sp[p], (double)V[(size_t)p * 128 + tid], o);
+  out[tid] = (float)(o / l);
 }
 
 }  // namespace
@@ -465,7 +476,7 @@ e3_status f32_rope_kv_run(const float *qkv, float *qo, float *kc, float *vc, con
 
 e3_status f32_attn_dec_run(const float *q, float *ctx, const float *kc, const float *vc, const DecArgs &a,
                            cudaStream_t st) {
-  const size_t smem = (size_t)a.max_ctx * sizeof(float);
+  const size_t smem = (size_t)a.max_ctx * sizeof(double);
   static size_t attr = 0;
   if (smem > 48 * 1024 && smem > attr) {
     E3_CUDA_TRY(cudaFuncSetAttribute(f32_attn_dec_kernel, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem));
@@ -499,7 +510,7 @@ e3_status f32_attn_run(const float *qkv, float *ctx, int B, int S, int H, cudaSt
     set_error("fp32 attention: need head_dim 64 and S <= 256");
     return E3_EUNSUPPORTED;
   }
-  const size_t smem = ((size_t)S * (65 + 64) + kAW * 64 + (size_t)kAW * S) * sizeof(float);
+  const size_t smem = ((size_t)S * (65 + 64) + kAW * 64) * sizeof(float) + (size_t)kAW * S * sizeof(double);
   static size_t attr = 0;
   if (smem > 48 * 1024 && smem > attr) {
     E3_CUDA_TRY(cudaFuncSetAttribute(f32_attn_kernel, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem));
