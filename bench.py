@@ -14,12 +14,16 @@ starts; `e2e` repeats the measurement through the same C-ABI call with HOST
 (pinned) inputs, the H2D copies and the D2H read of the exit records inside
 the timed region.
 
-N > 1 (torchrun): replica mode -- every rank runs the whole split chain on
-its own shard (weak scaling, no data-path collective).
---mode stage: the chain is cut into stages on different GPUs (parallel.py,
-plan_stages balanced on the calibrated survival profile); survivors travel
-GPU to GPU over NCCL send/recv, chunk by chunk.
-Time = max over ranks of CUDA-event time, barrier + synchronize around it.
+N > 1 (torchrun): stage mode (default) -- the per-ramp split chain is cut
+into stages on different GPUs (parallel.plan_stages, balanced on the
+calibrated survival profile; --stages, default min(N, 4)) and run by the
+library's multi-rank pipeline: every rank calls e3_pipeline_run on the same
+plan, survivors travel GPU to GPU as NCCL messages issued by libe3.so
+(e3_comm_*, e3_plan.replicas / device_of).  The replica mode (every rank runs
+the whole chain on its own shard, no data-path collective) is timed right
+after and printed as "replica_comparison".  --mode replica times only that.
+Per-GPU load is fixed (weak scaling).  Time = max over ranks of CUDA-event
+time, barrier + synchronize around it.
 
 --impl reference: the CPU oracle (oracle/, NumPy float64) timed on the host
 cores on a bounded sample of the same workload (this tier has no reference
@@ -57,10 +61,9 @@ def parse():
     ap.add_argument("--no-e2e", action="store_true")
     ap.add_argument("--no-cpu", action="store_true")
     ap.add_argument("--cpu-inputs", type=int, default=32)
-    ap.add_argument("--mode", default="replica", choices=["replica", "stage"],
-                    help="N>1: replicas of the whole chain, or stages on different GPUs (parallel.py)")
-    ap.add_argument("--chunk", type=int, default=1024, help="stage mode: inputs per chunk")
-    ap.add_argument("--stages", type=int, default=2, help="stage mode: number of stages")
+    ap.add_argument("--mode", default="stage", choices=["replica", "stage"],
+                    help="N>1: stages on different GPUs (library NCCL transfers), or replicas of the whole chain")
+    ap.add_argument("--stages", type=int, default=0, help="stage mode: number of stages (0: min(N, 4))")
     ap.add_argument("--planner", default="balance", choices=["balance", "dp"],
                     help="stage mode: survival-balanced cuts, or the profile-driven DP (planner.py)")
     return ap.parse_args()
@@ -245,43 +248,42 @@ def main():
     stream = torch.cuda.Stream(dev)
     model_bytes = sum(t.numel() * 2 for w in model.layers for t in w.values())
     kv_bytes = sum(t.numel() * 2 for t in (model.kv.k + model.kv.v)) if llama else 0
-    stage_mode = args.mode == "stage" and world > 1
-    if stage_mode and llama:
-        raise SystemExit("--mode stage: encoder configs only (the llama KV cache is per GPU)")
+    stage_mode = args.mode == "stage" and world > 1 and not llama
+    first_id = rank * n
+    ids_all = None
     if stage_mode:
-        # stages on different GPUs: chunk c of the job enters at the stage-0
-        # replica owning it; ids are global so exits land at their input's slot
+        # stages on different GPUs; the job is n inputs per GPU, fed into
+        # split 0 by the stage-0 replicas; ids are global so every exit record
+        # lands at its input's slot on the rank where the input exits
         from paper_conf_sosp_iyergdpgn24_b200 import parallel as par
+        k = args.stages or min(world, 4)
         prof_path = os.path.join(ROOT, "profiles", f"r01_planner_profile_{args.config}.json")
         if args.planner == "dp" and os.path.exists(prof_path):
-            # profile-driven DP (planner.py, NEXT-1) restricted to --stages stages
-            from paper_conf_sosp_iyergdpgn24_b200 import planner as pl
-            prof = pl.Profile.load(prof_path)
-            layout, _ = pl.plan_dp(cfg.ramp_layers, lambda l: survival(cfg, l), prof, world,
-                                   n_stages=min(args.stages, world, cfg.n_ramps))
+            # profile-driven DP (planner.py, NEXT-1) restricted to k stages
+            from paper_conf_sosp_iyergdpgn24_b200 import planner as pln
+            layout, _ = pln.plan_dp(cfg.ramp_layers, lambda l: survival(cfg, l), pln.Profile.load(prof_path),
+                                    world, n_stages=min(k, world, cfg.n_ramps))
         else:
             layout = par.plan_stages(cfg.ramp_layers, lambda l: survival(cfg, l), world,
-                                     n_stages=min(args.stages, world, cfg.n_ramps))
-        g_stage, _ = layout.stage_of(rank)
+                                     n_stages=min(k, world, cfg.n_ramps))
         total = n * world
-        n_chunks = (total + args.chunk - 1) // args.chunk
-        mine = [c for c in range(n_chunks) if layout.owner(0, c) == rank] if g_stage == 0 else []
-        chunk_ids = {c: range(c * args.chunk, min(total, (c + 1) * args.chunk)) for c in mine}
-        chunk_x = {c: torch.from_numpy(e3data.make_inputs(cfg, r)).to(torch.bfloat16).to(dev)
-                   for c, r in chunk_ids.items()}
-        chunk_id_t = {c: torch.tensor(list(r), dtype=torch.int64, device=dev) for c, r in chunk_ids.items()}
+        lo, hi = par.input_share(layout, rank, total)
+        comm = par.make_comm(rank, world, local)
+        plan = api.make_plan(cfg, bounds, tau, lag=1, placement=par.placement(layout, bounds), transport="nccl")
+        pipe = api.Pipeline(model, plan, comm)
         ex = api.ExitBuffers(total, cfg.classes, cfg.n_ramps, dev)
-        executor = par.GpuStageExecutor(model, cfg, layout.bounds[g_stage], layout.bounds[g_stage + 1], tau, ex,
-                                        args.chunk)
-        transport = par.Transport(device=True)
         plan_name = f"stages {list(layout.bounds)} replicas {list(layout.replicas)} (per-ramp splits inside)"
+        first_id, n_mine = lo, hi - lo
     else:
-        first_id = rank * n
-        # synthetic inputs of the paper-shaped workload (seeded; one stream per id)
-        X = e3data.make_inputs(cfg, range(first_id, first_id + n))
-        x_host = torch.from_numpy(X).to(torch.bfloat16).pin_memory()
-        del X
-        x_dev = x_host.to(dev)
+        n_mine = n
+    X = e3data.make_inputs(cfg, range(first_id, first_id + n_mine))
+    x_host = torch.from_numpy(X).to(torch.bfloat16).pin_memory() if n_mine else None
+    del X
+    x_dev = x_host.to(dev) if n_mine else None
+    if stage_mode:
+        ids_dev = torch.arange(first_id, first_id + n_mine, dtype=torch.int64, device=dev) if n_mine else None
+        ids_host = ids_dev.cpu().pin_memory() if n_mine else None
+    else:
         ids_dev = torch.arange(0, n, dtype=torch.int64, device=dev)   # local ids index the exit arrays
         ids_host = torch.arange(0, n, dtype=torch.int64).pin_memory()
         ex = api.ExitBuffers(n, cfg.classes, cfg.n_ramps, dev)
@@ -291,14 +293,10 @@ def main():
         if world > 1:
             dist.barrier()
 
-    def step(host=False, res=None):
-        if stage_mode:
-            with torch.cuda.stream(stream):
-                par.run_stage_pipeline(executor, layout, rank, n_chunks, lambda c: (chunk_x[c], chunk_id_t[c]),
-                                       (cfg.seq, cfg.hidden), torch.bfloat16, dev, transport)
-            return None
+    def step(host=False, res=None, p=None):
+        p = p or pipe
         with torch.cuda.stream(stream):
-            st = pipe.run(x_host if host else x_dev, ids_host if host else ids_dev, ex, stream=stream)
+            st = p.run(x_host if host else x_dev, ids_host if host else ids_dev, ex, stream=stream)
             if res is not None:   # D2H read of the step's result (exit records)
                 res[0].copy_(ex.exit_layer, non_blocking=True)
                 res[1].copy_(ex.label, non_blocking=True)
@@ -312,7 +310,7 @@ def main():
         dist.all_reduce(t, op=dist.ReduceOp.MAX)
         return float(t.item())
 
-    def timed(K, host=False, res=None):
+    def timed(K, host=False, res=None, p=None):
         barrier()
         torch.cuda.synchronize()
         e0 = torch.cuda.Event(enable_timing=True)
@@ -320,7 +318,7 @@ def main():
         e0.record(stream)
         stats = None
         for _ in range(K):
-            stats = step(host, res)
+            stats = step(host, res, p)
         e1.record(stream)
         torch.cuda.synchronize()
         barrier()
@@ -350,15 +348,48 @@ def main():
 
     # e2e: host-pinned inputs through the same C-ABI call, results read back
     e2e = None
-    if not args.no_e2e and not stage_mode:
-        res = (torch.empty(n, dtype=torch.int32).pin_memory(), torch.empty(n, dtype=torch.int32).pin_memory(),
-               torch.empty(n, dtype=torch.float32).pin_memory())
+    if not args.no_e2e:
+        cap = ex.capacity
+        res = (torch.empty(cap, dtype=torch.int32).pin_memory(), torch.empty(cap, dtype=torch.int32).pin_memory(),
+               torch.empty(cap, dtype=torch.float32).pin_memory())
         step(host=True, res=res)
         torch.cuda.synchronize()
         ms_e2e, _ = timed(args.steps, host=True, res=res)
+        row = cfg.seq * cfg.hidden * 2
         e2e = {"value": round(total_inputs / (ms_e2e / 1000.0), 1), "unit": "inputs/s",
-               "h2d_bytes_per_step": int(x_host.numel() * 2 + ids_host.numel() * 8),
-               "d2h_bytes_per_step": int(n * 12)}
+               "h2d_bytes_per_step": int(n * world * (row + 8)),        # the whole job's inputs + ids
+               "d2h_bytes_per_step": int(cap * 12 * world)}             # every rank reads its exit records
+
+    # stage mode: the replica mode on the same per-GPU load, as the comparison
+    replica_cmp = None
+    if stage_mode:
+        Xr = e3data.make_inputs(cfg, range(rank * n, rank * n + n))
+        xr = torch.from_numpy(Xr).to(torch.bfloat16).to(dev)
+        del Xr
+        idr = torch.arange(0, n, dtype=torch.int64, device=dev)
+        exr = api.ExitBuffers(n, cfg.classes, cfg.n_ramps, dev)
+        rpipe = api.Pipeline(model, api.make_plan(cfg, bounds, tau, lag=1))
+
+        def rstep():
+            with torch.cuda.stream(stream):
+                rpipe.run(xr, idr, exr, stream=stream)
+
+        for _ in range(max(args.warmup, 3)):
+            rstep()
+        barrier()
+        torch.cuda.synchronize()
+        e0 = torch.cuda.Event(enable_timing=True)
+        e1 = torch.cuda.Event(enable_timing=True)
+        e0.record(stream)
+        for _ in range(args.steps):
+            rstep()
+        e1.record(stream)
+        torch.cuda.synchronize()
+        barrier()
+        ms_r = max_over_ranks(e0.elapsed_time(e1))
+        replica_cmp = {"value": round(total_inputs / (ms_r / 1000.0), 1), "unit": "inputs/s",
+                       "ms_per_step": round(ms_r / args.steps, 3), "mode": "replica (whole chain per GPU)"}
+        del rpipe, xr, exr
 
     # per-kernel CUDA-event profile of one extra step (same stream, same launches)
     _lib.lib.e3_profile_reset()
@@ -433,6 +464,7 @@ def main():
             "per_kernel": per_kernel,
             "cpu_baseline": cpu,
             "e2e": e2e,
+            "replica_comparison": replica_cmp,
             "gpu_launches": int(launches),
             "clocks": clocks,
             "exit_hist": hist,

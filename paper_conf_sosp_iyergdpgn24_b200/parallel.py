@@ -1,35 +1,24 @@
-"""Multi-GPU drivers of the split path: one process per GPU, torch.distributed
-for the plumbing.
+"""Multi-GPU plumbing of the split path: one process per GPU, torch.distributed
+for rendezvous only.  The data path -- the
+stage loop, survivor messages over NCCL, re-batching -- runs in libe3.so
+(e3_comm_* / e3_pipeline_* with e3_plan placement); this module only
 
-Two modes:
+* plans the stages (``plan_stages``: the paper's pipelined balance,
+  PAPER.md:907-930, restricted to one GPU type): contiguous cuts at ramps and
+  replica counts minimising the bottleneck max_g W_g / r_g, W_g = expected
+  survivor-layers of stage g;
+* turns a stage layout into the per-split placement of e3_plan
+  (``placement``) and each stage-0 replica's share of the inputs
+  (``input_share``);
+* creates the library's NCCL communicator from a torch process group
+  (``make_comm``: the unique id travels over the group);
+* merges the per-rank exit records (``reduce_exits``).
 
-* replica  -- every rank runs the whole split chain on its own shard of the
-  inputs (inputs are independent, so the path shards with no data-path
-  collective).  ``shard`` gives the contiguous shard of a rank.
-
-* stage    -- E3's model-parallel execution (Fig. 5): the
-  split chain is cut into contiguous STAGES placed on different GPUs, each
-  stage optionally replicated.  Inputs flow in chunks; stage g runs its
-  splits on a chunk (constant batch inside, e3_pipeline_run_out) and ships
-  the survivors -- a count, then the [n, S, H] rows and their ids -- to the
-  replica of stage g+1 that owns the chunk ("outputs are then directed to the
-  machines hosting the next split").  With the NCCL backend
-  the rows go GPU-to-GPU over NVLink (ncclSend/ncclRecv); the count header
-  lets the receiver post a receive of exactly the right size (NCCL needs
-  matching counts).  Chunk c of stage g is handled by replica c mod r_g, so
-  every rank knows, without any coordination, whom to receive from and send
-  to.  Sends are asynchronous (isend): stage g computes chunk c+1 while chunk
-  c travels and stage g+1 computes it -- the steady-state pipeline of §3.2.2
-  (PAPER.md:907-913).
-
-``plan_stages`` balances the stages (the paper's pipelined DP, PAPER.md:
-907-930, restricted to one GPU type): minimise max_g W_g / r_g over contiguous
-cuts at ramps and replica counts r_g (sum r_g = G), W_g = expected
-survivor-layers of stage g.
-
-The executor is duck-typed so the host-side logic runs under the gloo backend
-on CPU with a stand-in executor (tests/test_parallel.py); on GPUs
-``GpuStageExecutor`` wraps the C-ABI pipeline.
+Two modes of bench.py --gpus N:
+  stage    E3's model-parallel execution (Fig. 5): stages
+           on different GPUs, survivors shipped by the library over NVLink;
+  replica  every rank runs the whole chain on its own shard (no data-path
+           collective) -- printed as the comparison.
 """
 from __future__ import annotations
 
@@ -75,10 +64,6 @@ class StageLayout:
                 return g, rs.index(rank)
         raise ValueError(rank)
 
-    def owner(self, g: int, chunk: int) -> int:
-        """Rank of stage g that processes chunk `chunk`."""
-        return self.ranks_of(g)[chunk % self.replicas[g]]
-
 
 def plan_stages(ramp_layers: Sequence[int], survival: Callable[[int], float], world: int,
                 max_stages: Optional[int] = None, n_stages: Optional[int] = None) -> StageLayout:
@@ -115,100 +100,36 @@ def plan_stages(ramp_layers: Sequence[int], survival: Callable[[int], float], wo
     return best[1]
 
 
-# ---------------------------------------------------------------- transport
-
-class Transport:
-    """Point-to-point rows between ranks.  device=True: tensors stay on the GPU
-    (NCCL over NVLink); device=False: staged through host memory (gloo)."""
-
-    def __init__(self, device: bool):
-        self.device = device
-
-    def isend(self, t: torch.Tensor, dst: int):
-        if not self.device and t.is_cuda:
-            t = t.cpu()
-        return dist.isend(t.contiguous(), dst), t
-
-    def recv(self, shape, dtype, src: int, dev) -> torch.Tensor:
-        if self.device:
-            t = torch.empty(shape, dtype=dtype, device=dev)
-        else:
-            t = torch.empty(shape, dtype=dtype)
-        dist.recv(t, src)
-        return t.to(dev) if (not self.device and dev is not None and torch.device(dev).type == "cuda") else t
+def placement(layout: StageLayout, split_bounds: Sequence[int]) -> List[List[int]]:
+    """Per split (split s = layers [split_bounds[s], split_bounds[s+1])) the
+    ranks of its replicas: those of the stage containing it.  Every stage
+    boundary must be a split boundary."""
+    for b in layout.bounds:
+        if b not in split_bounds:
+            raise ValueError(f"stage boundary {b} is not a split boundary {tuple(split_bounds)}")
+    out = []
+    for s in range(len(split_bounds) - 1):
+        g = max(i for i in range(layout.n_stages) if layout.bounds[i] <= split_bounds[s])
+        out.append(layout.ranks_of(g))
+    return out
 
 
-def run_stage_pipeline(executor, layout: StageLayout, rank: int, n_chunks: int,
-                       chunk_inputs: Callable[[int], Tuple[torch.Tensor, torch.Tensor]],
-                       row_shape: Tuple[int, ...], row_dtype, dev, transport: Transport) -> dict:
-    """Run this rank's stage over every chunk it owns (SPMD: call on all ranks).
-
-    executor.run(x, ids) -> (x_surv, ids_surv, n_surv)   (stage not last)
-    executor.run(x, ids) -> (None, None, 0)               (last stage)
-    chunk_inputs(c) -> (x, ids) for the stage-0 owner of chunk c.
-    Returns counters {chunks, rows_in, rows_out}."""
-    g, _ = layout.stage_of(rank)
-    last = g == layout.n_stages - 1
-    stats = {"chunks": 0, "rows_in": 0, "rows_out": 0}
-    pending = []                               # in-flight sends (keep tensors alive)
-    for c in range(n_chunks):
-        if layout.owner(g, c) != rank:
-            continue
-        if g == 0:
-            x, ids = chunk_inputs(c)
-        else:
-            src = layout.owner(g - 1, c)
-            hdr = transport.recv((1,), torch.int64, src, dev)
-            n = int(hdr.item())
-            if n > 0:
-                x = transport.recv((n,) + tuple(row_shape), row_dtype, src, dev)
-                ids = transport.recv((n,), torch.int64, src, dev)
-            else:
-                x = torch.empty((0,) + tuple(row_shape), dtype=row_dtype, device=dev)
-                ids = torch.empty((0,), dtype=torch.int64, device=dev)
-        stats["chunks"] += 1
-        stats["rows_in"] += int(ids.shape[0])
-        xs, ids_s, n_s = executor.run(x, ids)
-        if last:
-            continue
-        dst = layout.owner(g + 1, c)
-        hdr = torch.tensor([n_s], dtype=torch.int64, device=dev if transport.device else "cpu")
-        pending.append(transport.isend(hdr, dst))
-        if n_s > 0:
-            # private copies: the executor reuses its output buffers for the
-            # next chunk while an NCCL isend of this one may still be queued
-            pending.append(transport.isend(xs[:n_s].clone(), dst))
-            pending.append(transport.isend(ids_s[:n_s].clone(), dst))
-        stats["rows_out"] += n_s
-        while len(pending) > 12:               # bound the in-flight buffers
-            pending.pop(0)[0].wait()
-    for work, _ in pending:
-        work.wait()
-    return stats
+def input_share(layout: StageLayout, rank: int, n: int) -> Tuple[int, int]:
+    """Inputs [lo, hi) of a job of n that `rank` feeds into split 0 (stage-0
+    replicas split the job contiguously; other ranks get an empty range)."""
+    g, i = layout.stage_of(rank)
+    if g != 0:
+        return 0, 0
+    return shard(n, layout.replicas[0], i)
 
 
-class GpuStageExecutor:
-    """One stage on this GPU: the split chain of layers [begin, end) through the
-    C ABI (e3_pipeline_run / e3_pipeline_run_out), survivors into a buffer."""
-
-    def __init__(self, model, cfg, begin: int, end: int, tau, exits, max_rows: int, lag: int = 1):
-        from . import api
-        bounds = [begin] + [l + 1 for l in cfg.ramp_layers if begin <= l < end]
-        self.pipe = api.Pipeline(model, api.make_plan(cfg, bounds, tau, lag=lag))
-        self.final = end == cfg.layers
-        self.exits = exits
-        dev = model.device
-        if not self.final:
-            self.x_out = torch.empty((max_rows, cfg.seq, cfg.hidden), dtype=torch.bfloat16, device=dev)
-            self.id_out = torch.empty((max_rows,), dtype=torch.int64, device=dev)
-
-    def run(self, x, ids):
-        if self.final:
-            self.pipe.run(x, ids, self.exits)
-            return None, None, 0
-        n = int(ids.shape[0])
-        _, n_out = self.pipe.run_out(x, ids, self.exits, self.x_out[:max(n, 1)], self.id_out[:max(n, 1)])
-        return self.x_out, self.id_out, n_out
+def make_comm(rank: int, world: int, device: int, group=None):
+    """The library's NCCL communicator for this rank: rank 0 creates the
+    unique id, the torch process group carries it to every rank."""
+    from . import api
+    obj = [api.Comm.unique_id() if rank == 0 else None]
+    dist.broadcast_object_list(obj, src=0, group=group)
+    return api.Comm.nccl(obj[0], rank, world, device)
 
 
 def reduce_exits(exits, group=None):

@@ -1,8 +1,8 @@
-"""Multi-process (gloo, CPU) tests of the multi-GPU drivers in parallel.py:
-replica sharding, the stage-pipeline transport (count header + rows + ids,
-chunk ownership), stage planning and the exit-record reduction.  The GPU
-executor is replaced by a stand-in that applies a fixed exit-layer table, so
-what is tested is exactly the host-side routing."""
+"""Multi-process (gloo, CPU) tests of the multi-GPU plumbing in parallel.py:
+stage planning, per-split placement, input shares, the communicator-id
+broadcast and the exit-record reduction.  The data path
+itself (stage loop, messages, re-batching) is in libe3.so and is tested on
+the GPU (tests/test_gpu_stage.py, LOOPBACK transport, and NCCL on >= 2 GPUs)."""
 import os
 import socket
 
@@ -16,44 +16,6 @@ from paper_conf_sosp_iyergdpgn24_b200 import parallel as par
 L = 12
 RAMPS = list(range(L))
 N_IDS = 300
-CHUNK = 40
-ROW = (2, 3)
-
-
-def _exit_table(seed=5):
-    g = torch.Generator().manual_seed(seed)
-    return torch.randint(0, L, (N_IDS,), generator=g)
-
-
-class StandIn:
-    """Stage [a, b): inputs whose exit layer < b exit here, the rest survive.
-    Checks the payload arrived intact (row of input i == i)."""
-
-    def __init__(self, a, b, table):
-        self.a, self.b, self.table = a, b, table
-        self.exit_at = torch.full((N_IDS,), -1, dtype=torch.int64)
-        self.seen = torch.zeros((N_IDS,), dtype=torch.int64)
-        self.bad = 0
-
-    def run(self, x, ids):
-        for r in range(ids.shape[0]):
-            i = int(ids[r])
-            self.seen[i] += 1
-            if not torch.all(x[r] == float(i)):
-                self.bad += 1
-            if int(self.table[i]) < self.a:
-                self.bad += 1              # should have exited upstream
-        e = self.table[ids] < self.b
-        self.exit_at[ids[e]] = self.table[ids[e]]
-        keep = ~e
-        if self.b == L:
-            return None, None, 0
-        xs, ids_s = x[keep].clone(), ids[keep].clone()
-        # pad the survivor buffer the way the GPU executor does (capacity >= n)
-        pad = 3
-        xs = torch.cat([xs, torch.zeros((pad,) + ROW)])
-        ids_s = torch.cat([ids_s, torch.full((pad,), -7, dtype=torch.int64)])
-        return xs, ids_s, int(keep.sum())
 
 
 def _free_port():
@@ -64,34 +26,53 @@ def _free_port():
     return p
 
 
+class _FakeExits:
+    """The fields of api.ExitBuffers that reduce_exits combines (CPU tensors)."""
+
+    def __init__(self, n, c, r):
+        self.exit_layer = torch.full((n,), -1, dtype=torch.int32)
+        self.label = torch.full((n,), -1, dtype=torch.int32)
+        self.conf = torch.full((n,), float("nan"))
+        self.logits = torch.zeros((n, c))
+        self.n_exit = torch.zeros((1,), dtype=torch.int32)
+        self.ramp_count = torch.zeros((r,), dtype=torch.int32)
+
+
 def _worker(rank, world, port, bounds, replicas, q):
+    """One rank of a stage layout over gloo: every rank derives the same
+    placement, the stage-0 replicas' input shares partition the job, the
+    communicator id broadcast reaches every rank, and the exit records of
+    inputs exiting on different ranks merge into one record per input."""
     os.environ["MASTER_ADDR"] = "127.0.0.1"
     os.environ["MASTER_PORT"] = str(port)
     dist.init_process_group("gloo", rank=rank, world_size=world)
     try:
         layout = par.StageLayout(tuple(bounds), tuple(replicas))
+        split_bounds = tuple(range(L + 1))          # per-ramp splits
+        pl = par.placement(layout, split_bounds)
+        allp = [None] * world
+        dist.all_gather_object(allp, pl)
+        lo, hi = par.input_share(layout, rank, N_IDS)
+        shares = [None] * world
+        dist.all_gather_object(shares, (lo, hi))
+        uid = [bytes(range(128)) if rank == 0 else None]   # stands in for e3_comm_unique_id
+        dist.broadcast_object_list(uid, src=0)
+        # exit records: input i exits on the rank of the stage holding layer table[i]
+        table = torch.arange(N_IDS) % L
         g, _ = layout.stage_of(rank)
-        table = _exit_table()
-        ex = StandIn(bounds[g], bounds[g + 1], table)
-        n_chunks = (N_IDS + CHUNK - 1) // CHUNK
-
-        def chunk_inputs(c):
-            ids = torch.arange(c * CHUNK, min(N_IDS, (c + 1) * CHUNK), dtype=torch.int64)
-            x = ids.to(torch.float32)[:, None, None].expand((ids.shape[0],) + ROW).contiguous()
-            return x, ids
-
-        st = par.run_stage_pipeline(ex, layout, rank, n_chunks, chunk_inputs, ROW, torch.float32, "cpu",
-                                    par.Transport(device=False))
-        exit_at = ex.exit_at.clone()
-        dist.all_reduce(exit_at, op=dist.ReduceOp.MAX)
-        exited_here = (ex.exit_at >= 0).to(torch.int64)
-        dist.all_reduce(exited_here, op=dist.ReduceOp.SUM)
-        seen = ex.seen.clone()
-        dist.all_reduce(seen, op=dist.ReduceOp.SUM)
-        bad = torch.tensor([ex.bad])
-        dist.all_reduce(bad, op=dist.ReduceOp.SUM)
+        ex = _FakeExits(N_IDS, 2, L)
+        mine = [i for i in range(N_IDS) if layout.bounds[g] <= int(table[i]) < layout.bounds[g + 1]
+                and i % layout.replicas[g] == layout.stage_of(rank)[1]]
+        for i in mine:
+            ex.exit_layer[i] = int(table[i])
+            ex.label[i] = i % 2
+            ex.conf[i] = 0.5
+            ex.logits[i] = torch.tensor([float(i), -float(i)])
+        ex.n_exit[0] = len(mine)
+        par.reduce_exits(ex)
         if rank == 0:
-            q.put({"exit_at": exit_at, "count": exited_here, "seen": seen, "bad": int(bad), "stats": st})
+            q.put({"placements": allp, "shares": shares, "uid": uid[0], "exit_layer": ex.exit_layer,
+                   "logits": ex.logits, "n_exit": int(ex.n_exit[0]), "label": ex.label})
     finally:
         dist.destroy_process_group()
 
@@ -115,16 +96,30 @@ def _run(bounds, replicas):
                                              ((0, 4, 12), (1, 2)),
                                              ((0, 3, 12), (2, 1)),
                                              ((0, 2, 6, 12), (1, 1, 1))])
-def test_stage_pipeline_routes_every_input_once(bounds, replicas):
+def test_stage_plumbing_world_size_gt_1(bounds, replicas):
     res = _run(bounds, replicas)
-    table = _exit_table()
-    assert res["bad"] == 0
-    assert torch.equal(res["exit_at"], table)           # every input exits at its own layer
-    assert torch.equal(res["count"], torch.ones(N_IDS, dtype=torch.int64))   # exactly once
-    # input i is seen by every stage whose first layer is <= its exit layer
-    starts = torch.tensor(bounds[:-1])
-    expect_seen = (starts[None, :] <= table[:, None]).sum(1)
-    assert torch.equal(res["seen"], expect_seen)
+    world = sum(replicas)
+    assert all(p == res["placements"][0] for p in res["placements"])       # one plan on every rank
+    pl = res["placements"][0]
+    lay = par.StageLayout(tuple(bounds), tuple(replicas))
+    for s in range(L):
+        g = max(i for i in range(lay.n_stages) if bounds[i] <= s)
+        assert pl[s] == lay.ranks_of(g)
+    shares = [tuple(x) for x in res["shares"] if x[1] > x[0]]
+    assert sorted(shares)[0][0] == 0 and sorted(shares)[-1][1] == N_IDS
+    assert sum(h - l for l, h in shares) == N_IDS and len(shares) == replicas[0]
+    assert res["uid"] == bytes(range(128))
+    table = torch.arange(N_IDS) % L
+    assert torch.equal(res["exit_layer"].to(torch.int64), table)       # merged: one record per input
+    assert res["n_exit"] == N_IDS
+    assert torch.equal(res["logits"][:, 0], torch.arange(N_IDS, dtype=torch.float32))
+
+
+def test_placement_rejects_cuts_inside_a_split():
+    lay = par.StageLayout((0, 3, 12), (1, 1))
+    with pytest.raises(ValueError):
+        par.placement(lay, (0, 2, 4, 12))
+    assert par.placement(lay, (0, 3, 12)) == [[0], [1]]
 
 
 def test_shard_covers_all():
@@ -140,8 +135,8 @@ def test_layout_ownership():
     lay = par.StageLayout((0, 4, 12), (1, 3))
     assert lay.world == 4 and lay.n_stages == 2
     assert lay.ranks_of(1) == [1, 2, 3]
-    assert [lay.owner(1, c) for c in range(6)] == [1, 2, 3, 1, 2, 3]
     assert lay.stage_of(2) == (1, 1)
+    assert par.input_share(lay, 0, 10) == (0, 10) and par.input_share(lay, 2, 10) == (0, 0)
 
 
 def test_plan_stages_balances():
