@@ -37,7 +37,7 @@ e3_status gemm_run(const GemmMaps &g, const void *bias, const void *R, int M, in
 // 2 CTAs per 128 rows, each owning N/2 columns; pre (optional) receives
 // y = bf16(A W^T + bias + R), out = bf16(LN(y) * g + b)
 struct LnGemmMaps {
-  CUtensorMap a, w, r, pre, out;
+  CUtensorMap a, w, w2, r, pre, out;   // w2: W boxes of the CTA-pair variant (half the MMA N)
 };
 struct LnGemmArgs {
   const __nv_bfloat16 *bias, *R, *g, *b;
