@@ -445,6 +445,13 @@ def main():
                "kind": "oracle",
                "sample": f"{args.cpu_inputs} inputs of the {cfg.name} workload through the fp64 NumPy "
                          f"oracle ({dt:.1f} s)"}
+        # the same oracle on ONE host thread (core count stated)
+        from threadpoolctl import threadpool_limits
+        n1 = max(1, args.cpu_inputs // 4)
+        with threadpool_limits(limits=1):
+            rate1, dt1 = cpu_oracle_rate(cfg, tau, n1, seed_offset=10_000)
+        cpu["one_thread"] = {"value": round(rate1, 3), "unit": "inputs/s", "cores": 1,
+                             "sample": f"{n1} inputs ({dt1:.1f} s)"}
 
     if rank == 0:
         out = {

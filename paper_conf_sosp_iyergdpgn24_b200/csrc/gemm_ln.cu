@@ -617,12 +617,11 @@ e3_status ln_gemm_tmaps(LnGemmMaps *m, const void *A, const void *W, const void 
 E3_TL_SETTER(tl_set_gemm_ln)
 
 e3_status ln_gemm_run(const LnGemmMaps &m, const LnGemmArgs &a, cudaStream_t st) {
-  if (ln2_enabled()) {   // CTA-pair variant where the shapes allow it
-    switch (a.N / 2) {
-      case 384: return ln2_launch<384>(m, a, st);
-      case 512: return ln2_launch<512>(m, a, st);
-    }
-  }
+  // CTA-pair variant only where it measured faster (scripts/gemm_ln_bench.py,
+  // B200, graph-replayed): N = 2048 rows of 1024 (BL shape) 50.2 vs 53.0 us;
+  // at N = 768 (BB) the 1-SM kernel stays ahead, 16.4 vs 17.4 us -- the
+  // halved W fill does not shorten a tile whose epilogue cannot overlap
+  if (ln2_enabled() && a.N / 2 == 512) return ln2_launch<512>(m, a, st);
   switch (a.N / 2) {
     case 64: return ln_launch<64>(m, a, st);
     case 128: return ln_launch<128>(m, a, st);
