@@ -66,6 +66,11 @@ e3_status layernorm_run(const void *x, const void *g, const void *b, void *y, in
 
 // ---- K4 exit ramp (ramp.cu)
 constexpr int kRampRowsPerCta = 16;   // rows per ramp row group (one ticket each)
+// workspace counter words: [0] compaction ticket, [1 .. 256] ramp group
+// tickets, then the fused ramp + compaction's decision and exit counters
+constexpr int kRampCtrGroupsDone = 1 + 4096 / kRampRowsPerCta;
+constexpr int kRampCtrExit = kRampCtrGroupsDone + 1;
+constexpr int kCtrWordsAll = kRampCtrExit + 1;
 struct RampArgs {
   int arch;
   const void *x;            // [B,S,H] bf16 (pre-LN rows when ln_g != NULL)
@@ -83,8 +88,8 @@ struct RampArgs {
   const int32_t *n_valid_dev;   // NULL: n_valid_host
   int n_valid_host;
   e3_exits ex;
-  float *pool_ws;           // [B,H] fp32 workspace
-  unsigned *done_ctr;       // device tickets [ceil(B/kRampRowsPerCta)] (zero between launches)
+  float *pool_ws;           // [B,H] fp32 workspace (BERT: the slices' partial logits)
+  unsigned *done_ctr;       // device counters [kCtrWordsAll] (zero between launches)
   // LLAMA: per-128-class-tile softmax statistics from the LM-head GEMM
   // (gemm_dec.cu, E3_DEC_LOGITS, which also wrote the logits to the exit
   // records); the decide kernel merges them
@@ -92,6 +97,16 @@ struct RampArgs {
   int lm_tiles;
 };
 e3_status ramp_run(const RampArgs &a, cudaStream_t st);
+// BERT ramp on (group, slice) CTAs without clusters (rampc.cu); ctr_words =
+// the workspace counters (RampArgs.done_ctr)
+bool ramp_bert2_supported(int H, int C);
+e3_status ramp_bert2_run(const RampArgs &a, unsigned *ctr_words, cudaStream_t st);
+// the split's last BERT ramp (pre-LN rows, a.ln_g set) fused with the stable
+// LN + compaction of the survivors into dst; *done = false when the shape
+// does not fit one cooperative wave (the caller then runs ramp + ln_compact)
+e3_status ramp_compact_run(const RampArgs &a, unsigned *ctr_words, const struct RingDst &dst, int32_t *n_surv_dev,
+                           int sms, cudaStream_t st, bool *done);
+e3_status tl_set_rampc(void *buf);
 
 // ---- K7 decode GEMM (gemm_dec.cu): Y[T,N] = epi(X[T,K] W[N,K]^T), swap-AB tcgen05
 enum { E3_DEC_STORE = 0, E3_DEC_RESID = 1, E3_DEC_SWIGLU = 2, E3_DEC_QKV_ROPE = 3, E3_DEC_LOGITS = 4 };

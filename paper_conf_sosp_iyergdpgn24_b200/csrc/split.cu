@@ -684,6 +684,7 @@ e3_status split_run_to(e3_split *s, cudaStream_t st, const void *x_in, const int
   const double f_qkv = 2.0 * nvS * 3 * H * H, f_o = 2.0 * nvS * H * H, f_1 = 2.0 * nvS * F * H;
   const double f_att = 4.0 * n_valid_host * (double)S * S * H, b_ln = 2.0 * nvS * H * 2;
   const bool vit = d.arch == E3_ARCH_VIT;
+  bool compacted = false;   // the last ramp's fused kernel also compacted the survivors
   for (int i = 0; i < nl; ++i) {
     const int l = d.layer_begin + i;
     const e3_layer_weights &L = s->L[i];
@@ -799,20 +800,26 @@ e3_status split_run_to(e3_split *s, cudaStream_t st, const void *x_in, const int
         a.n_valid_host = n_valid_host;
         a.ex = exits;
         a.pool_ws = ws.pool;
-        a.done_ctr = ws.ctr + 1;   // per-row-group tickets
+        a.done_ctr = ws.ctr;       // workspace counters (tickets, fused ramp + compaction)
         {
           // pooler weights + CLS rows + classifier weights (bytes); 2H^2 + 2HC per row (flops)
           const double hh = vit ? 0.0 : 2.0 * H * H;
           ProfScope ps(PK_RAMP, st, (double)n_valid_host * (hh + 2.0 * H * d.num_labels),
                        hh + 2.0 * n_valid_host * H + 2.0 * d.num_labels * H);
-          if (!skip(PK_RAMP)) E3_RUN(ramp_run(a, st));
+          if (last && pre_ln_rows && !skip(PK_RAMP)) {
+            // the split's last ramp and the LN2 + compaction of its survivors in one launch
+            bool fused = false;
+            E3_RUN(ramp_compact_run(a, ws.ctr, dst, n_surv_dev, s->sms, st, &fused));
+            compacted = fused;
+          }
+          if (!compacted && !skip(PK_RAMP)) E3_RUN(ramp_run(a, st));
         }
         first_ramp = false;
       }
       ++ri;
     }
   }
-  {
+  if (!compacted) {
     // survivors: LN2 of the last layer fused with the stable compaction
     // (bytes added once n_surv is known, in the pipeline)
     const e3_layer_weights &L = s->L[nl - 1];
@@ -898,6 +905,7 @@ e3_status e3_debug_timeline(void *dev_buf) {
   if (r == E3_OK) r = tl_set_compact(dev_buf);
   if (r == E3_OK) r = tl_set_gemm_ln(dev_buf);
   if (r == E3_OK) r = tl_set_dec(dev_buf);
+  if (r == E3_OK) r = tl_set_rampc(dev_buf);
   return r;
 }
 
@@ -1000,7 +1008,7 @@ e3_status e3_op_ramp(void *stream, int32_t arch, const void *x, const int64_t *i
   float *pool = nullptr;
   unsigned *ctr = nullptr;
   E3_CUDA_TRY(cudaMallocAsync(reinterpret_cast<void **>(&pool), (size_t)B * H * 4, st));
-  const size_t nctr = (size_t)(B + kRampRowsPerCta - 1) / kRampRowsPerCta * sizeof(unsigned);
+  const size_t nctr = (size_t)kCtrWords * sizeof(unsigned);
   E3_CUDA_TRY(cudaMallocAsync(reinterpret_cast<void **>(&ctr), nctr, st));
   E3_CUDA_TRY(cudaMemsetAsync(ctr, 0, nctr, st));
   RampArgs a{};

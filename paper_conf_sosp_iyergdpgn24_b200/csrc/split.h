@@ -8,8 +8,9 @@
 
 namespace e3 {
 
-// 1 compaction ticket + one ramp ticket per group of kRampRowsPerCta rows (B <= 4096)
-constexpr int kCtrWords = 1 + 4096 / kRampRowsPerCta;
+// compaction ticket, one ramp ticket per group of kRampRowsPerCta rows (B <=
+// 4096), the fused ramp + compaction's counters (kernels.h)
+constexpr int kCtrWords = kCtrWordsAll;
 
 // Activation workspace for one batch of B rows.  Splits that run serially on
 // one stream may share a workspace (the pipeline does).
