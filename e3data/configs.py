@@ -110,9 +110,25 @@ LLAMA_7B = ModelConfig(
     kv_heads=32, ctx=512, cls_gain=8.0,
 )
 
-CONFIGS = {c.name: c for c in (TINY, TINY_VIT, BERT_BASE, BERT_LARGE, VIT_BASE, TINY_LLAMA, LLAMA_7B)}
+# Dependent exits (NEXT-4; PABEE): the counter-based criterion
+# with patience t (DESIGN R26).  TINY_PABEE: tiny dims, a ramp after every
+# layer; BERT_BASE_PABEE: EE-BERT-base's shape and weights, patience 2.
+TINY_PABEE = ModelConfig(
+    name="tiny-pabee", arch="bert", layers=4, hidden=128, heads=2, ffn=512, seq=32,
+    classes=2, norm_eps=1e-12, ramp_layers=(0, 1, 2, 3), batch=32, test="patience",
+    tau=(1.0, 1.0, 1.0, 1.0),
+)
+
+BERT_BASE_PABEE = ModelConfig(
+    name="ee-bert-base-pabee", arch="bert", layers=12, hidden=768, heads=12, ffn=3072,
+    seq=128, classes=2, norm_eps=1e-12, ramp_layers=tuple(range(12)), batch=64,
+    test="patience", tau=(2.0,) * 12,
+)
+
+CONFIGS = {c.name: c for c in (TINY, TINY_VIT, BERT_BASE, BERT_LARGE, VIT_BASE, TINY_LLAMA, LLAMA_7B,
+                               TINY_PABEE, BERT_BASE_PABEE)}
 ALIASES = {"t": "tiny", "tv": "tiny-vit", "tl": "tiny-llama", "bb": "ee-bert-base", "bl": "ee-bert-large",
-           "vt": "ee-vit-b16", "lm": "ee-llama-7b-decode"}
+           "vt": "ee-vit-b16", "lm": "ee-llama-7b-decode", "tp": "tiny-pabee", "bbp": "ee-bert-base-pabee"}
 
 
 def get(name: str) -> ModelConfig:

@@ -61,7 +61,14 @@ typedef enum { E3_DTYPE_BF16 = 0, E3_DTYPE_FP32 = 1 } e3_dtype;
  * than a pre-defined threshold") -> exit iff max softmax > tau; entropy
  * ("entropy ... smaller than pre-defined threshold") -> exit iff H < tau
  * (natural log).  Comparisons are strict. */
-typedef enum { E3_TEST_MAXPROB = 0, E3_TEST_ENTROPY = 1 } e3_test;
+typedef enum { E3_TEST_MAXPROB = 0, E3_TEST_ENTROPY = 1, E3_TEST_PATIENCE = 2 } e3_test;
+/* E3_TEST_PATIENCE -- dependent exits, the counter-based criterion ("require
+ * off-ramps classifiers to continuously generate identical predictions for
+ * pre-defined times"; PABEE, §5.6; R26): at
+ * every evaluated ramp the counter of an input becomes prev + 1 if its argmax
+ * equals the previous ramp's, else 0; exit iff counter >= tau (the patience).
+ * The per-input state lives in e3_exits.state (caller-zeroed per job) and
+ * travels with the input across splits; single-rank plans only. */
 /* Ramps inside a split (§3.4 exit-wrapper; §5.8.6):
  * EXACT evaluates every ramp (plan-independent results; rows that exit at an
  * inner ramp are recorded there and carried, masked, to the split end);
@@ -159,6 +166,8 @@ typedef struct e3_exits {
   int64_t capacity;
   int32_t *n_exit;
   int32_t *ramp_count;
+  int32_t *state;      /* E3_TEST_PATIENCE: [capacity] per-input (label + 1) << 16 | counter,
+                          zero before an input's first ramp; NULL otherwise            */
 } e3_exits;
 
 typedef struct e3_split e3_split;

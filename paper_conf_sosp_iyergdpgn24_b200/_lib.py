@@ -21,7 +21,7 @@ STATUS = {0: "E3_OK", 1: "E3_EINVAL", 2: "E3_EUNSUPPORTED", 3: "E3_ECUDA", 4: "E
           5: "E3_ECAPACITY", 6: "E3_ESTATE"}
 
 ARCH = {"bert": 0, "vit": 1, "llama": 2}
-TEST = {"maxprob": 0, "entropy": 1}
+TEST = {"maxprob": 0, "entropy": 1, "patience": 2}
 INNER = {"exact": 0, "disabled": 1}
 DTYPE = {"bf16": 0, "fp32": 1}
 EPI = {"bias": 0, "bias_gelu": 1, "bias_resid": 2}
@@ -69,7 +69,7 @@ class Weights(C.Structure):
 
 class Exits(C.Structure):
     _fields_ = [("exit_layer", P), ("label", P), ("conf", P), ("logits", P), ("capacity", I64),
-                ("n_exit", P), ("ramp_count", P)]
+                ("n_exit", P), ("ramp_count", P), ("state", P)]
 
 
 class Plan(C.Structure):

@@ -138,9 +138,11 @@ class ExitBuffers:
         self.logits = torch.zeros((capacity, classes), dtype=torch.float32, device=dev) if logits else None
         self.n_exit = torch.zeros((1,), dtype=torch.int32, device=dev)
         self.ramp_count = torch.zeros((max(n_ramps, 1),), dtype=torch.int32, device=dev)
+        # dependent exits (E3_TEST_PATIENCE): per-input counter state, zero per job
+        self.state = torch.zeros((capacity,), dtype=torch.int32, device=dev)
         self.c = _lib.Exits(self.exit_layer.data_ptr(), self.label.data_ptr(), self.conf.data_ptr(),
                             None if self.logits is None else self.logits.data_ptr(), capacity,
-                            self.n_exit.data_ptr(), self.ramp_count.data_ptr())
+                            self.n_exit.data_ptr(), self.ramp_count.data_ptr(), self.state.data_ptr())
 
     def reset(self):
         self.exit_layer.fill_(-1)
@@ -150,6 +152,7 @@ class ExitBuffers:
             self.logits.zero_()
         self.n_exit.zero_()
         self.ramp_count.zero_()
+        self.state.zero_()
 
 
 class Split:

@@ -21,6 +21,7 @@
 //                      metric -> strict threshold -> exit record, alive flag
 // Survivors are compacted by the byte-exact ln_compact kernel in copy mode.
 #include "common.cuh"
+#include "exitrule.cuh"
 #include "fp32_path.h"
 #include "prof.h"
 
@@ -298,7 +299,9 @@ __global__ void __launch_bounds__(kRT) f32_ramp_kernel(RampArgs a) {
     for (int w = 0; w < kRT / 32; ++w) { sum += red[w][1]; qz += red[w][2]; }
     float metric;
     bool pass;
-    if (a.test == E3_TEST_MAXPROB) {   // the metric is reported (and tested) as fp32
+    if (a.test == E3_TEST_PATIENCE) {
+      pass = patience_step(a.ex.state, a.id[b], a.ex.capacity, label, a.tau, &metric);
+    } else if (a.test == E3_TEST_MAXPROB) {   // the metric is reported (and tested) as fp32
       metric = (float)(1.0 / sum);
       pass = metric > a.tau;
     } else {

@@ -18,6 +18,7 @@
 //                    the same semantics as the encoder ramps (the logits
 //                    were written to the records by the LM-head epilogue).
 #include "common.cuh"
+#include "exitrule.cuh"
 #include "kernels.h"
 #include "prof.h"
 #include "softstat.cuh"
@@ -239,7 +240,11 @@ __global__ void __launch_bounds__(128) lm_decide_kernel(RampArgs a) {
   for (int o = 16; o; o >>= 1) st = soft_merge(st, soft_shfl_xor(st, o));
   float metric;
   bool pass;
-  if (a.test == E3_TEST_MAXPROB) {
+  if (a.test == E3_TEST_PATIENCE) {   // one state update per row (lane 0), then broadcast
+    if (lane == 0) pass = patience_step(a.ex.state, a.id[b], a.ex.capacity, st.idx, a.tau, &metric);
+    pass = __shfl_sync(0xffffffffu, pass, 0);
+    metric = __shfl_sync(0xffffffffu, metric, 0);
+  } else if (a.test == E3_TEST_MAXPROB) {
     metric = 1.0f / st.s;
     pass = metric > a.tau;
   } else {

@@ -756,6 +756,12 @@ e3_status e3_pipeline_create(const e3_plan *p, const e3_weights *w, int device, 
       return E3_EUNSUPPORTED;
     }
     E3_CHECK_ARG(p->transport == comm_transport(comm), "plan transport differs from the communicator's");
+    for (int s = 0; s < p->n_splits; ++s)
+      if (p->split[s].test == E3_TEST_PATIENCE) {
+        set_error("e3_pipeline_create: dependent exits (E3_TEST_PATIENCE) keep per-input state in the caller's "
+                  "e3_exits.state: single-rank plans only");
+        return E3_EUNSUPPORTED;
+      }
     e3_status r = plan_stages(p, world, &stages);
     if (r != E3_OK) return r;
     my_stage = -1;

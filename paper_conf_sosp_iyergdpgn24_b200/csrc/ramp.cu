@@ -35,6 +35,7 @@
 // The ViT ramp (LayerNorm + linear over C <= 2048 classes) is ramp_vit_kernel
 // below.
 #include "common.cuh"
+#include "exitrule.cuh"
 #include "kernels.h"
 #include "ln_row.cuh"
 #include "softstat.cuh"
@@ -287,7 +288,9 @@ __global__ void __launch_bounds__(kRThreads, 1) ramp_bert_kernel(RampArgs a) {
       }
     float metric;
     bool pass;
-    if (a.test == E3_TEST_MAXPROB) {
+    if (a.test == E3_TEST_PATIENCE) {
+      pass = patience_step(a.ex.state, row_id, a.ex.capacity, label, a.tau, &metric);
+    } else if (a.test == E3_TEST_MAXPROB) {
       metric = 1.0f / sum;                       // max_c softmax(z)_c
       pass = metric > a.tau;
     } else {
@@ -507,7 +510,9 @@ __global__ void __launch_bounds__(kVitKQ * 2 * CB) ramp_vit_kernel(RampArgs a, i
         for (int q = 1; q < CS; ++q) st = soft_merge(st, sQ[q][r]);
         float metric;
         bool pass;
-        if (a.test == E3_TEST_MAXPROB) {
+        if (a.test == E3_TEST_PATIENCE) {
+          pass = patience_step(a.ex.state, a.id[b], a.ex.capacity, st.idx, a.tau, &metric);
+        } else if (a.test == E3_TEST_MAXPROB) {
           metric = 1.0f / st.s;
           pass = metric > a.tau;
         } else {
@@ -802,7 +807,9 @@ __global__ void __launch_bounds__(kVtcThreads, 1) ramp_vit_tc_kernel(RampArgs a,
         for (int q = 1; q < CS; ++q) st = soft_merge(st, sQ[q][r]);
         float metric;
         bool pass;
-        if (a.test == E3_TEST_MAXPROB) {
+        if (a.test == E3_TEST_PATIENCE) {
+          pass = patience_step(a.ex.state, a.id[b], a.ex.capacity, st.idx, a.tau, &metric);
+        } else if (a.test == E3_TEST_MAXPROB) {
           metric = 1.0f / st.s;
           pass = metric > a.tau;
         } else {

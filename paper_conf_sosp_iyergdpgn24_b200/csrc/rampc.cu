@@ -25,6 +25,7 @@
 // into the next split's queue ring.  The row loads and the LayerNorm overlap
 // the ramp; one kernel boundary less than ramp -> compaction.
 #include "common.cuh"
+#include "exitrule.cuh"
 #include "kernels.h"
 #include "ln_row.cuh"
 #include "prof.h"
@@ -257,7 +258,9 @@ struct RampSlice {
           }
         float metric;
         bool pass;
-        if (a.test == E3_TEST_MAXPROB) {
+        if (a.test == E3_TEST_PATIENCE) {
+          pass = patience_step(a.ex.state, a.id[b], a.ex.capacity, label, a.tau, &metric);
+        } else if (a.test == E3_TEST_MAXPROB) {
           metric = 1.0f / sum;
           pass = metric > a.tau;
         } else {

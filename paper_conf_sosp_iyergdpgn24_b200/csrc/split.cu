@@ -142,7 +142,7 @@ static e3_status llama_validate(const e3_split_desc *d, const e3_weights *w) {
     E3_CHECK_ARG(R.ln_g && R.w_c && aligned16(R.w_c), "LLAMA ramp needs ln_g (final norm) and w_c (LM head)");
   }
   E3_CHECK_ARG(d->ramp_layer[d->n_ramps - 1] == d->layer_end - 1, "a split must end in a ramp");
-  E3_CHECK_ARG(d->test == E3_TEST_MAXPROB || d->test == E3_TEST_ENTROPY, "bad test");
+  E3_CHECK_ARG(d->test == E3_TEST_MAXPROB || d->test == E3_TEST_ENTROPY || d->test == E3_TEST_PATIENCE, "bad test");
   E3_CHECK_ARG(d->inner == E3_INNER_EXACT || d->inner == E3_INNER_DISABLED, "bad inner mode");
   for (int l = d->layer_begin; l < d->layer_end; ++l) {
     const e3_layer_weights &L = w->layer[l];
@@ -194,7 +194,7 @@ e3_status split_validate(const e3_split_desc *d, const e3_weights *w) {
     E3_CHECK_ARG(d->ramp_index[r] >= 0 && d->ramp_index[r] < w->n_ramps, "ramp index outside the model");
   }
   E3_CHECK_ARG(d->ramp_layer[d->n_ramps - 1] == d->layer_end - 1, "a split must end in a ramp");
-  E3_CHECK_ARG(d->test == E3_TEST_MAXPROB || d->test == E3_TEST_ENTROPY, "bad test");
+  E3_CHECK_ARG(d->test == E3_TEST_MAXPROB || d->test == E3_TEST_ENTROPY || d->test == E3_TEST_PATIENCE, "bad test");
   E3_CHECK_ARG(d->inner == E3_INNER_EXACT || d->inner == E3_INNER_DISABLED, "bad inner mode");
   for (int l = d->layer_begin; l < d->layer_end; ++l) {
     const e3_layer_weights &L = w->layer[l];

@@ -73,5 +73,10 @@ def test_plan_placement_validation_before_any_launch(L):
     assert st == 1 and "final" in msg
     # device differs from the communicator's
     assert _create(_lib, ok, cs[0], device=1)[0] == 1
+    # dependent exits keep per-input state in the caller's records: one rank only
+    pcfg = e3data.get("tp")
+    bad = api.make_plan(pcfg, (0, 2, 4), pcfg.tau, placement=[[0], [1]], transport="loopback")
+    st, msg = _create(_lib, bad, cs[0])
+    assert st == 2 and "single-rank" in msg
     for c in cs:
         c.close()
