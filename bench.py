@@ -296,6 +296,8 @@ def main():
     def step(host=False, res=None, p=None):
         p = p or pipe
         with torch.cuda.stream(stream):
+            if cfg.test == "patience":   # dependent exits: per-input counters start at zero every job
+                ex.state.zero_()
             st = p.run(x_host if host else x_dev, ids_host if host else ids_dev, ex, stream=stream)
             if res is not None:   # D2H read of the step's result (exit records)
                 res[0].copy_(ex.exit_layer, non_blocking=True)

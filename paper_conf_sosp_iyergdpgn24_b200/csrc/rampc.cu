@@ -226,6 +226,15 @@ struct RampSlice {
   __device__ void decide(int n_valid, const float *part) {
     const int C = a.C;
     const int warp = warp_id(), lane = lane_id();
+    // the group's kSl x 16 x C partials -> smem with every thread's loads in
+    // flight at once (a lane summing them straight from L2 serialised kSl x C
+    // round trips: r02 timeline, ~23 us to the decision), then summed per row
+    // in slice order below (deterministic)
+    float *sPart = sRed;   // [kSl][16][C] <= 8 x 16 x TN floats (kSl C <= H)
+    const int np = kSl * kGRows * C;
+    const float *gp = part + (size_t)g * kSl * kGRows * C;
+    for (int i = threadIdx.x; i < np; i += kT) sPart[i] = __ldcg(gp + i);
+    __syncthreads();
     if (warp != 0) return;
     const int r = lane, b = g * kGRows + r;
     bool exit_now = false;
@@ -239,7 +248,7 @@ struct RampSlice {
           z[c] = 0.f;
           if (c < C) {
             float s = 0.f;
-            for (int q = 0; q < kSl; ++q) s += __ldcg(part + ((size_t)(g * kSl + q) * kGRows + r) * C + c);
+            for (int q = 0; q < kSl; ++q) s += sPart[(q * kGRows + r) * C + c];
             z[c] = s + bf2f(reinterpret_cast<const __nv_bfloat16 *>(a.w.b_c)[c]);
           }
         }
@@ -302,12 +311,20 @@ __global__ void __launch_bounds__(kT, 2) ramp_bert2_kernel(RampArgs a, float *pa
   if (a.ln_g)
     ln_load_params<VPL>(lp, reinterpret_cast<const __nv_bfloat16 *>(a.ln_g),
                         reinterpret_cast<const __nv_bfloat16 *>(a.ln_b), a.H, lane_id());
+  const unsigned long long tl0 = tl_now();
   pdl_wait();
+  const unsigned long long tl1 = tl_now();
   const int n_valid = a.n_valid_dev ? *a.n_valid_dev : a.n_valid_host;
   rs.compute(lp, n_valid, part);
-  if (rs.arrive(ctr, &s_flag)) rs.decide(n_valid, part);
+  const unsigned long long tl2 = tl_now();
+  const bool dec = rs.arrive(ctr, &s_flag);
+  if (dec) rs.decide(n_valid, part);
   __syncthreads();
   pdl_trigger();
+  if (threadIdx.x == 0) {
+    tl_rec(g_tl, 74, tl0, tl1);                          // ramp2: entry | release | end
+    tl_rec(g_tl, dec ? 76 : 75, tl1, tl2);               // slice computed (75) / decider (76): release | partials | end
+  }
 }
 
 // block scan of the alive flags (ballot / popc per 32, serial over words)
@@ -377,9 +394,12 @@ __global__ void __launch_bounds__(kT, 2)
     const int u = blockIdx.x * kNW + warp + jj * stride;
     if (u < all_units) ln_load_row<VPL>(v[jj], y + (size_t)u * H, H, lane);
   }
+  const unsigned long long tlr0 = tl_now();
   if (ramp_cta) {
     rs.compute(lp, n_valid, part);
+    if (threadIdx.x == 0) tl_rec(tlb, 72, tl1, tlr0);     // ramp slice: release | rows issued | computed
     if (rs.arrive(ctr, &s_flag)) {
+      if (threadIdx.x == 0) tl_rec(tlb, 73, tl1, tl1);    // decider start
       rs.decide(n_valid, part);
       __syncthreads();
       if (threadIdx.x == 0) {
@@ -456,7 +476,9 @@ E3_TL_SETTER(tl_set_rampc)
 bool ramp_bert2_supported(int H, int C) {
   const int kSl = ramp_slices(H);
   // partials [groups][kSl][16][C] f32 live in the [B, H] f32 pool workspace
-  return C >= 1 && C <= kMaxCl && H % (8 * kSl) == 0 && H <= 1024 && H / kSl <= 32 && kSl * C <= H;
+  // (and their smem copy in the decider, [kSl][16][C] in the [8][16][TN] partial-sum buffer)
+  return C >= 1 && C <= kMaxCl && H % (8 * kSl) == 0 && H <= 1024 && H / kSl <= 32 && kSl * C <= H &&
+         kSl * kSl * C <= 8 * H;
 }
 
 static RCtr make_ctr(unsigned *ctr_words) {
