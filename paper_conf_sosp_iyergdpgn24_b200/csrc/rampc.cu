@@ -520,7 +520,13 @@ e3_status ramp_bert2_run(const RampArgs &a, unsigned *ctr_words, cudaStream_t st
 e3_status ramp_compact_run(const RampArgs &a, unsigned *ctr_words, const RingDst &dst, int32_t *n_surv_dev, int sms,
                            cudaStream_t st, bool *done) {
   *done = false;
-  if (!ramp_bert2_supported(a.H, a.C) || a.B > kMaxBc || !a.ln_g || getenv("E3_NO_FUSED_RC")) return E3_OK;
+  // Off by default (E3_FUSED_RC=1 enables it): measured on B200 (scripts/timeline.py bb, r02) the fused
+  // launch took 21.8 us per BB split run from FFN2's end to the next QKV GEMM against 20.5 us for the
+  // ticketed ramp + ln_compact pair (154.1 vs 148.8 us per run): its decision chain (slice partials,
+  // ticket, partial reload, decision) slows while 296 CTAs stream the 12.6 MB of token rows beside it,
+  // which outweighs the saved kernel boundary.
+  static const bool on = getenv("E3_FUSED_RC") != nullptr;
+  if (!on || !ramp_bert2_supported(a.H, a.C) || a.B > kMaxBc || !a.ln_g) return E3_OK;
   const int kSl = ramp_slices(a.H);
   const int groups = (a.B + kGRows - 1) / kGRows;
   const int n_ramp = groups * kSl;
