@@ -441,3 +441,46 @@ def test_bert_base_batch_position_invariance_bitwise(api, bert_base):
     assert a[4].keys() == b[4].keys() and len(a[4]) > 0
     for i in a[4]:
         assert torch.equal(a[4][i].view(torch.int16), b[4][i].view(torch.int16))
+
+
+_FUSED_SCRIPT = r'''
+import sys, numpy as np, torch
+sys.path.insert(0, ".")
+import e3data
+from paper_conf_sosp_iyergdpgn24_b200 import api
+from oracle.pipeline_sim import Plan
+cfg = e3data.get(sys.argv[1]); tau = e3data.tau_for(cfg)
+model = api.DeviceModel(cfg, e3data.make_weights(cfg), "cuda:0")
+N = int(sys.argv[2])
+X = api.to_bf16(e3data.make_inputs(cfg, range(N)), "cuda:0")
+ex = api.ExitBuffers(N, cfg.classes, cfg.n_ramps, "cuda:0")
+api.Pipeline(model, api.make_plan(cfg, Plan.per_ramp(cfg.ramp_layers).bounds, tau)).run(
+    X, torch.arange(N, dtype=torch.int64, device="cuda:0"), ex)
+torch.cuda.synchronize()
+np.save(sys.argv[3], np.concatenate([ex.exit_layer.cpu().numpy()[:, None].astype(np.float32),
+                                     ex.logits.cpu().numpy()], axis=1))
+'''
+
+
+@pytest.mark.parametrize("name,n", [("tiny", 200), ("bb", 256)])
+def test_fused_ramp_compaction_equals_two_kernel_path(name, n, tmp_path):
+    """E3_FUSED_RC=1 (the cooperative ramp + LN2 + compaction launch, off by
+    default) gives bitwise the records of the default ticketed ramp +
+    ln_compact path: both share the ramp arithmetic (rampc.cu)."""
+    import os
+    import subprocess
+    import sys
+    root = os.path.dirname(os.path.dirname(os.path.abspath(__file__)))
+    script = tmp_path / "run.py"
+    script.write_text(_FUSED_SCRIPT)
+    outs = []
+    for fused in (False, True):
+        env = dict(os.environ)
+        env.pop("E3_FUSED_RC", None)
+        if fused:
+            env["E3_FUSED_RC"] = "1"
+        f = tmp_path / f"o{int(fused)}.npy"
+        subprocess.run([sys.executable, str(script), name, str(n), str(f)], cwd=root, env=env, check=True,
+                       timeout=600)
+        outs.append(np.load(f))
+    assert np.array_equal(outs[0], outs[1])
