@@ -115,7 +115,8 @@ def _as64(W):
 
 
 def run_split(cfg, weights, X, begin: int, end: int, ids: Sequence[int], kv, slot_of_id, pos_of_slot,
-              tau=None, mode: str = "fp64", inner: str = "exact", record_all: bool = False):
+              tau=None, mode: str = "fp64", inner: str = "exact", record_all: bool = False,
+              exit_hidden: Optional[dict] = None):
     """Decode layers [begin, end) (ending in a ramp) for the tokens X [n, H].
 
     weights["layers"][l] / weights["ramps"][r]: dicts (may be lazy sequences);
@@ -124,7 +125,8 @@ def run_split(cfg, weights, X, begin: int, end: int, ids: Sequence[int], kv, slo
     token.  Same return values as oracle.model.run_split:
     (records of the tokens exiting here, survivor ids in order, survivors'
     hidden rows [k, H], {id: min margin}).  record_all: also return every
-    ramp's metric per token (brute-force pin)."""
+    ramp's metric per token (brute-force pin).  exit_hidden: if a dict, it
+    receives {id: the token's hidden row at its exit} (multi-step decode)."""
     X = np.asarray(X, dtype=np.float64).reshape(len(ids), cfg.hidden)
     n = X.shape[0]
     ids = [int(i) for i in ids]
@@ -163,6 +165,8 @@ def run_split(cfg, weights, X, begin: int, end: int, ids: Sequence[int], kv, slo
             i = alive[j]
             exited[i] = ExitRecord(ids[i], l, r, int(np.argmax(z[j])), float(m[j]), z[j].copy(),
                                    float(margin[i]))
+            if exit_hidden is not None:
+                exit_hidden[ids[i]] = h[j].copy()
         alive, h = alive[~ok], h[~ok]
     recs = [exited[i] for i in sorted(exited)]
     return recs, [ids[i] for i in alive], h, {ids[i]: float(margin[i]) for i in range(n)}
@@ -209,3 +213,83 @@ def brute_force(cfg, weights, X, ids, kv, slot_of_id, pos_of_slot, tau=None, mod
                 break
         exit_layer[i] = cfg.ramp_layers[first]
     return exit_layer, Z, M
+
+
+# --------------------------------------------------------------------------
+# Multi-step autoregressive early-exit decode.
+#
+# PAPER.md leaves the KV cache of exited tokens open ("the problem of managing
+# the KV cache still needs to be resolved ... an open problem: while CALM
+# proposes a solution to this problem, it is focused on encoder-decoder
+# architecture") and restricts its Llama runs to one output
+# token; its multi-token gains come from CALM.
+# Reading (R27), CALM-style state propagation for a decoder-only
+# model: a token that exits after layer e is treated by every skipped layer
+# l > e as if its input there were h_e, the hidden state it exited with; the
+# skipped layer's only lasting effect -- its K/V cache entry at the token's
+# position -- is computed from that input:
+#     n1 = RMSNorm1_l(h_e);  k = RoPE(n1 W_k^l, pos);  v = n1 W_v^l
+# with the decode layer's storage points (bf16 mode).  Greedy multi-step
+# decode: the next input of a token is E[y] (E the token embedding table, y
+# its argmax label at its exit) at position pos + 1.
+
+def fill_kv(cfg, W, h, K, V, pos, mode="fp64"):
+    """Write the K/V entries of one skipped layer (weights W) for tokens with
+    exit hidden rows h [n, H] into K, V [n, kvh, max_ctx, d] at pos[i]."""
+    n = h.shape[0]
+    nh, d = cfg.heads, cfg.head_dim
+    kvh = cfg.kv_heads or nh
+    n1 = store(rms_norm(h, W["ln1_g"], cfg.norm_eps), mode)
+    kv_rows = n1 @ W["w_qkv"][nh * d:].T
+    k = kv_rows[:, :kvh * d].reshape(n, kvh, d)
+    v = kv_rows[:, kvh * d:].reshape(n, kvh, d)
+    pos = np.asarray(pos, dtype=np.int64)
+    k = store(rope(k, pos[:, None], cfg.rope_theta), mode)
+    v = store(v, mode)
+    for i in range(n):
+        K[i, :, int(pos[i]), :] = k[i]
+        V[i, :, int(pos[i]), :] = v[i]
+
+
+def run_steps(cfg, weights, X0, ids, kv, slot_of_id, pos_of_slot, embed, steps, tau=None, mode="fp64"):
+    """Greedy early-exit decode of `steps` tokens per sequence.
+
+    X0 [n, H]: the first inputs; kv[l]: [2, n_slots, kvh, max_ctx, d] arrays,
+    updated in place (the layers each token runs, then the filled skipped
+    layers); pos_of_slot: dict slot -> position, advanced by one per step;
+    embed [V, H].  Returns (records per step (lists in input order), tokens
+    [steps, n], filled {(step, id): list of filled layers})."""
+    ids = [int(i) for i in ids]
+    n = len(ids)
+    X = np.asarray(X0, dtype=np.float64).reshape(n, cfg.hidden)
+    E = np.asarray(embed, dtype=np.float64)
+    all_recs, tokens, filled = [], np.zeros((steps, n), dtype=np.int64), {}
+    slots = [int(slot_of_id[i]) for i in ids]
+    for s in range(steps):
+        hx = {}
+        recs, surv, _, _ = run_split(cfg, weights, X, 0, cfg.layers, ids, kv, slot_of_id, pos_of_slot, tau, mode,
+                                     exit_hidden=hx)
+        assert not surv, "a token did not exit"
+        by_id = {r.id: r for r in recs}
+        recs = [by_id[i] for i in ids]
+        for l in range(1, cfg.layers):
+            need = [k for k, i in enumerate(ids) if by_id[i].exit_layer < l]
+            if not need:
+                continue
+            W = {k2: np.asarray(v2, dtype=np.float64) for k2, v2 in weights["layers"][l].items()}
+            sl = [slots[k] for k in need]
+            K = kv[l][0][sl].astype(np.float64)
+            V = kv[l][1][sl].astype(np.float64)
+            pos = [int(pos_of_slot[q]) for q in sl]
+            fill_kv(cfg, W, np.stack([hx[ids[k]] for k in need]), K, V, pos, mode)
+            kv[l][0][sl] = K
+            kv[l][1][sl] = V
+            for k in need:
+                filled.setdefault((s, ids[k]), []).append(l)
+        for k, i in enumerate(ids):
+            tokens[s, k] = by_id[i].label
+        X = E[tokens[s]]
+        for q in slots:
+            pos_of_slot[q] = int(pos_of_slot[q]) + 1
+        all_recs.append(recs)
+    return all_recs, tokens, filled
