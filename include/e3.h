@@ -133,7 +133,8 @@ typedef struct e3_ramp_weights {
  * length is pos_of_slot[slot] (device int32): the decode step writes the
  * token's k, v at that position of every layer it runs and attends over
  * positions 0..pos.  Nothing is written for layers a token skips (R24).
- * The library never advances pos_of_slot (the caller does, between steps). */
+ * e3_pipeline_run never advances pos_of_slot (the caller does, between
+ * steps); e3_decode_run advances it by one per step. */
 typedef struct e3_kv_cache {
   int32_t n_layers;
   void *const *k;              /* host array of n_layers device pointers       */
@@ -168,6 +169,9 @@ typedef struct e3_exits {
   int32_t *ramp_count;
   int32_t *state;      /* E3_TEST_PATIENCE: [capacity] per-input (label + 1) << 16 | counter,
                           zero before an input's first ramp; NULL otherwise            */
+  void *hidden;        /* LLAMA: [capacity, H] (activation dtype) -- the hidden row each
+                          token exited with (e3_decode_run fills the skipped layers'
+                          K/V from it); NULL: not recorded                             */
 } e3_exits;
 
 typedef struct e3_split e3_split;
@@ -327,6 +331,23 @@ e3_status e3_pipeline_run(e3_pipeline *pl, void *stream, const void *x, const in
 e3_status e3_pipeline_run_out(e3_pipeline *pl, void *stream, const void *x, const int64_t *ids, int64_t n,
                               const e3_exits *ex, e3_stats *st, void *x_out, int64_t *id_out, int64_t out_cap,
                               int64_t *n_out);
+/* Multi-step greedy early-exit decode (LLAMA_DECODE plans, every split on
+ * this rank; R27).  PAPER.md leaves the KV of
+ * exited tokens open; here, CALM-style state propagation: for
+ * step = 0 .. steps-1
+ *   1. the n tokens run through the plan as in e3_pipeline_run (x [n, H],
+ *      ids [n] device; each token its own sequence: slot_of_id[id] distinct);
+ *   2. for every layer l after a token's exit layer, its K/V at its position
+ *      are filled from the hidden row it exited with (ex->hidden, required):
+ *      k = RoPE(RMSNorm1_l(h) W_k^l), v = RMSNorm1_l(h) W_v^l (the decode
+ *      layer's own K/V arithmetic and storage points);
+ *   3. tokens_out[step * n + i] = its label (argmax); x[i] <- embed[label]
+ *      (embed [V, H] device, activation dtype); pos_of_slot[slot] += 1.
+ * Blocks until done.  E3_EINVAL if a position would pass the cache
+ * (max_ctx); st (optional) accumulates over the steps. */
+e3_status e3_decode_run(e3_pipeline *pl, void *stream, void *x, const int64_t *ids, int64_t n, int32_t steps,
+                        const void *embed, int32_t *tokens_out, const e3_exits *ex, e3_stats *st);
+
 /* Dispatch order of the last run (plan.trace = 1): per run its split, valid
  * count and the B ids (padding = -1) into ids_out[run * B ...]. */
 e3_status e3_pipeline_trace(e3_pipeline *pl, int32_t *split, int32_t *n_valid, int64_t *ids_out,

@@ -69,7 +69,7 @@ class Weights(C.Structure):
 
 class Exits(C.Structure):
     _fields_ = [("exit_layer", P), ("label", P), ("conf", P), ("logits", P), ("capacity", I64),
-                ("n_exit", P), ("ramp_count", P), ("state", P)]
+                ("n_exit", P), ("ramp_count", P), ("state", P), ("hidden", P)]
 
 
 class Plan(C.Structure):
@@ -108,6 +108,7 @@ SIGNATURES = {
     "e3_pipeline_run_out": (I32, [P, P, P, P, I64, C.POINTER(Exits), C.POINTER(Stats), P, P, I64,
                                   C.POINTER(I64)]),
     "e3_pipeline_trace": (I32, [P, P, P, P, I64, C.POINTER(I64)]),
+    "e3_decode_run": (I32, [P, P, P, P, I64, I32, P, P, C.POINTER(Exits), C.POINTER(Stats)]),
     "e3_op_gemm": (I32, [P, P, I64, P, P, P, P, I32, I32, I32, I32]),
     "e3_op_dec_gemm": (I32, [P, P, I32, P, P, I32, I32, I32, P, P]),
     "e3_op_gemm_ln": (I32, [P, P, P, P, P, P, P, C.c_float, P, P, I32, I32, I32]),

@@ -129,7 +129,10 @@ def split_desc(cfg, begin: int, end: int, tau, batch: Optional[int] = None,
 class ExitBuffers:
     """Exit records indexed by input id (e3_exits)."""
 
-    def __init__(self, capacity: int, classes: int, n_ramps: int, device, logits=True):
+    def __init__(self, capacity: int, classes: int, n_ramps: int, device, logits=True, hidden=0,
+                 hidden_dtype=torch.bfloat16):
+        """hidden > 0: also record each token's exit hidden row ([capacity,
+        hidden], the activation dtype) -- needed by Pipeline.decode."""
         dev = torch.device(device)
         self.capacity = capacity
         self.exit_layer = torch.full((capacity,), -1, dtype=torch.int32, device=dev)
@@ -140,9 +143,11 @@ class ExitBuffers:
         self.ramp_count = torch.zeros((max(n_ramps, 1),), dtype=torch.int32, device=dev)
         # dependent exits (E3_TEST_PATIENCE): per-input counter state, zero per job
         self.state = torch.zeros((capacity,), dtype=torch.int32, device=dev)
+        self.hidden = torch.zeros((capacity, hidden), dtype=hidden_dtype, device=dev) if hidden else None
         self.c = _lib.Exits(self.exit_layer.data_ptr(), self.label.data_ptr(), self.conf.data_ptr(),
                             None if self.logits is None else self.logits.data_ptr(), capacity,
-                            self.n_exit.data_ptr(), self.ramp_count.data_ptr(), self.state.data_ptr())
+                            self.n_exit.data_ptr(), self.ramp_count.data_ptr(), self.state.data_ptr(),
+                            None if self.hidden is None else self.hidden.data_ptr())
 
     def reset(self):
         self.exit_layer.fill_(-1)
@@ -306,6 +311,17 @@ class Pipeline:
                                       n, C.byref(exits.c), C.byref(st), _ptr(x_out), _ptr(id_out),
                                       int(id_out.shape[0]), C.byref(n_out)), "e3_pipeline_run_out")
         return st, n_out.value
+
+    def decode(self, x, ids, steps: int, embed, exits: ExitBuffers, stream=None):
+        """Multi-step greedy early-exit decode (e3_decode_run): x [n, H] the
+        first inputs (overwritten with the next inputs), ids [n], embed [V, H]
+        on the device; returns (tokens [steps, n] int32, stats)."""
+        n = int(ids.shape[0])
+        tokens = torch.empty((steps, n), dtype=torch.int32, device=ids.device)
+        st = _lib.Stats()
+        check(lib.e3_decode_run(self.h, _stream(stream), _ptr(x), _ptr(ids), n, steps, _ptr(embed), _ptr(tokens),
+                                C.byref(exits.c), C.byref(st)), "e3_decode_run")
+        return tokens, st
 
     def trace(self):
         n = C.c_int64()

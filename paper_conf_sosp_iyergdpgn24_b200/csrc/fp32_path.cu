@@ -327,6 +327,8 @@ __global__ void __launch_bounds__(kRT) f32_ramp_kernel(RampArgs a) {
   __syncthreads();
   if (s_exit && a.ex.logits)
     for (int k = tid; k < C; k += kRT) a.ex.logits[s_id * C + k] = z[k];
+  if (s_exit && a.ex.hidden && a.arch == E3_ARCH_LLAMA_DECODE)   // the exit row (multi-step decode)
+    for (int k = tid; k < H; k += kRT) reinterpret_cast<float *>(a.ex.hidden)[s_id * H + k] = c[k];
 }
 
 // ---- LLaMA decode (R22) in fp32 --------------------------------------

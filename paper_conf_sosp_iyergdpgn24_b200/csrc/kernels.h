@@ -154,8 +154,15 @@ e3_status attn_dec_run(const void *q, void *ctx, const void *kc, const void *vc,
                        const int32_t *n_valid_dev, int n_valid_host, const int32_t *slot_of_id, int64_t id_cap,
                        const int32_t *pos_of_slot, int n_slots, int T, int nh, int kvh, int max_ctx,
                        cudaStream_t st);
-// merge the LM-head statistics, threshold test, exit records (RampArgs with lm_*)
+// merge the LM-head statistics, threshold test, exit records (RampArgs with lm_*);
+// a.x (the rows) is copied into ex.hidden for the exiting tokens when both are set
 e3_status lm_decide_run(const RampArgs &a, cudaStream_t st);
+// multi-step decode helpers (llama.cu; e3_decode_run)
+e3_status fill_prep_run(const int64_t *ids, int nv, int B, const void *hidden, int64_t cap, const int32_t *exit_layer,
+                        int layer, int64_t row_bytes, void *x, int64_t *ids_out, uint8_t *mask, cudaStream_t st);
+e3_status decode_advance_run(const int64_t *ids, int64_t n, const int32_t *label, int64_t cap, int32_t *tokens_out,
+                             const void *embed, int32_t vocab, int64_t row_bytes, void *x, const int32_t *slot_of_id,
+                             int32_t *pos_of_slot, int n_slots, int *err, cudaStream_t st);
 
 // ---- K5 compaction (compact.cu)
 struct RingDst {

@@ -259,6 +259,11 @@ __global__ void __launch_bounds__(128) lm_decide_kernel(RampArgs a) {
       if (a.ex.label) a.ex.label[id] = st.idx;
       if (a.ex.conf) a.ex.conf[id] = metric;
     }
+    if (a.ex.hidden && a.x) {   // the row it exits with (multi-step decode fills skipped layers' K/V from it)
+      const uint4 *src = reinterpret_cast<const uint4 *>(a.x) + (size_t)b * (a.H / 8);
+      uint4 *dst = reinterpret_cast<uint4 *>(a.ex.hidden) + (size_t)id * (a.H / 8);
+      for (int k = lane; k < a.H / 8; k += 32) dst[k] = src[k];
+    }
   }
   if (lane == 0) {
     a.alive[b] = exit_now ? 0 : 1;
@@ -269,7 +274,74 @@ __global__ void __launch_bounds__(128) lm_decide_kernel(RampArgs a) {
   }
 }
 
+// multi-step decode, fill of layer l (R27): token slot t of the
+// chunk gets its exit hidden row (elem bytes per value) and the mask "its
+// exit layer lies before l"; rows >= nv are zero with id -1
+__global__ void fill_prep_kernel(const int64_t *__restrict__ ids, int nv, int B, const uint8_t *__restrict__ hidden,
+                                 int64_t cap, const int32_t *__restrict__ exit_layer, int layer, int64_t row_bytes,
+                                 uint8_t *__restrict__ x, int64_t *__restrict__ ids_out, uint8_t *__restrict__ mask) {
+  const int t = blockIdx.x;
+  const int64_t id = t < nv ? ids[t] : -1;
+  const bool ok = id >= 0 && id < cap;
+  const int el = ok ? exit_layer[id] : -1;
+  const uint4 *src = reinterpret_cast<const uint4 *>(hidden + (ok ? id : 0) * row_bytes);
+  uint4 *dst = reinterpret_cast<uint4 *>(x + (int64_t)t * row_bytes);
+  for (int64_t k = threadIdx.x; k < row_bytes / 16; k += blockDim.x) dst[k] = ok ? src[k] : make_uint4(0, 0, 0, 0);
+  if (threadIdx.x == 0) {
+    ids_out[t] = ok ? id : -1;
+    mask[t] = (ok && el >= 0 && el < layer) ? 1 : 0;
+  }
+}
+
+// token i: tokens_out[i] = label; x[i] = embed[label]; its slot's position + 1
+__global__ void decode_advance_kernel(const int64_t *__restrict__ ids, int64_t n, const int32_t *__restrict__ label,
+                                      int64_t cap, int32_t *__restrict__ tokens_out, const uint8_t *__restrict__ embed,
+                                      int32_t vocab, int64_t row_bytes, uint8_t *__restrict__ x,
+                                      const int32_t *__restrict__ slot_of_id, int32_t *pos_of_slot, int n_slots,
+                                      int *err) {
+  const int64_t i = blockIdx.x;
+  if (i >= n) return;
+  const int64_t id = ids[i];
+  const bool ok = id >= 0 && id < cap;
+  const int y = ok ? label[id] : -1;
+  const bool yok = y >= 0 && y < vocab;
+  const uint4 *src = reinterpret_cast<const uint4 *>(embed + (yok ? (int64_t)y : 0) * row_bytes);
+  uint4 *dst = reinterpret_cast<uint4 *>(x + i * row_bytes);
+  for (int64_t k = threadIdx.x; k < row_bytes / 16; k += blockDim.x) dst[k] = yok ? src[k] : make_uint4(0, 0, 0, 0);
+  if (threadIdx.x == 0) {
+    if (tokens_out) tokens_out[i] = y;
+    if (!yok && err) *err = 1;
+    if (ok) {
+      const int slot = slot_of_id[id];
+      if (slot >= 0 && slot < n_slots) pos_of_slot[slot] += 1;
+      else if (err) *err = 1;
+    }
+  }
+}
+
 }  // namespace
+
+e3_status fill_prep_run(const int64_t *ids, int nv, int B, const void *hidden, int64_t cap, const int32_t *exit_layer,
+                        int layer, int64_t row_bytes, void *x, int64_t *ids_out, uint8_t *mask, cudaStream_t st) {
+  fill_prep_kernel<<<B, 128, 0, st>>>(ids, nv, B, reinterpret_cast<const uint8_t *>(hidden), cap, exit_layer, layer,
+                                      row_bytes, reinterpret_cast<uint8_t *>(x), ids_out, mask);
+  E3_CUDA_TRY(cudaGetLastError());
+  count_launch();
+  return E3_OK;
+}
+
+e3_status decode_advance_run(const int64_t *ids, int64_t n, const int32_t *label, int64_t cap, int32_t *tokens_out,
+                             const void *embed, int32_t vocab, int64_t row_bytes, void *x, const int32_t *slot_of_id,
+                             int32_t *pos_of_slot, int n_slots, int *err, cudaStream_t st) {
+  if (n <= 0) return E3_OK;
+  decode_advance_kernel<<<(unsigned)n, 128, 0, st>>>(ids, n, label, cap, tokens_out,
+                                                     reinterpret_cast<const uint8_t *>(embed), vocab, row_bytes,
+                                                     reinterpret_cast<uint8_t *>(x), slot_of_id, pos_of_slot, n_slots,
+                                                     err);
+  E3_CUDA_TRY(cudaGetLastError());
+  count_launch();
+  return E3_OK;
+}
 
 // One CTA (8 warps) per row for the decode batch's few long rows (T <= 128
 // rows of H = 4096): a warp per row left 64 rows on 8 SMs, each lane summing

@@ -1012,6 +1012,72 @@ e3_status e3_pipeline_run_out(e3_pipeline *pl, void *stream, const void *x, cons
   return pipeline_run_impl(pl, stream, x, ids, n, ex, st, x_out, id_out, out_cap, n_out);
 }
 
+e3_status e3_decode_run(e3_pipeline *pl, void *stream, void *x, const int64_t *ids, int64_t n, int32_t steps,
+                        const void *embed, int32_t *tokens_out, const e3_exits *ex, e3_stats *st) {
+  E3_CHECK_ARG(pl && ex && x && ids && embed && n > 0 && steps >= 0, "bad arguments");
+  if (pl->poisoned) {
+    set_error("pipeline poisoned by an earlier failure");
+    return E3_ESTATE;
+  }
+  const e3_split_desc &d0 = pl->plan.split[0];
+  E3_CHECK_ARG(d0.arch == E3_ARCH_LLAMA_DECODE, "e3_decode_run needs a LLAMA_DECODE plan");
+  E3_CHECK_ARG(pl->s_lo == 0 && pl->s_hi == pl->plan.n_splits && pl->in.empty() && pl->out.empty(),
+               "e3_decode_run: every split on this rank (the fill needs every layer)");
+  E3_CHECK_ARG(pl->plan.split[pl->plan.n_splits - 1].final_ramp, "the plan must end in the model's final ramp");
+  E3_CHECK_ARG(ex->hidden && ex->exit_layer && ex->label, "e3_decode_run needs ex->hidden, exit_layer and label");
+  E3_CHECK_ARG(is_device_ptr(x) && is_device_ptr(ids) && is_device_ptr(embed), "x, ids, embed must be device memory");
+  cudaStream_t cs = reinterpret_cast<cudaStream_t>(stream);
+  const e3_split *s0 = pl->splits[0];
+  if (st) std::memset(st, 0, sizeof(*st));
+  const int elem = d0.dtype == E3_DTYPE_FP32 ? 4 : 2;
+  for (int step = 0; step < steps; ++step) {
+    e3_stats sst;
+    e3_status r = e3_pipeline_run(pl, stream, x, ids, n, ex, &sst);
+    if (r != E3_OK) return r;
+    if (st) {
+      st->runs += sst.runs;
+      for (int s = 0; s < pl->plan.n_splits; ++s) {
+        st->batches[s] += sst.batches[s];
+        st->valid_rows[s] += sst.valid_rows[s];
+        st->padded_rows[s] += sst.padded_rows[s];
+        st->rows_out[s] += sst.rows_out[s];
+        st->flushes[s] += sst.flushes[s];
+      }
+      st->host_waits += sst.host_waits;
+      st->host_launch_ms += sst.host_launch_ms;
+      st->host_sync_ms += sst.host_sync_ms;
+    }
+    E3_CUDA_TRY(cudaSetDevice(pl->device));
+    // K/V of the skipped layers, chunk by chunk of B tokens (layer 0 is never skipped)
+    for (int64_t c0 = 0; c0 < n; c0 += pl->B) {
+      const int nv = (int)std::min<int64_t>(pl->B, n - c0);
+      for (int s = 0; s < pl->plan.n_splits; ++s) {
+        const e3_split_desc &d = pl->plan.split[s];
+        for (int l = std::max(1, d.layer_begin); l < d.layer_end; ++l) {
+          r = llama_fill_layer(pl->splits[s], l, cs, ids + c0, nv, *ex, pl->staging_ids);
+          if (r != E3_OK) {
+            if (r == E3_ECUDA) pl->poisoned = true;
+            return r;
+          }
+        }
+      }
+    }
+    r = decode_advance_run(ids, n, ex->label, ex->capacity, tokens_out ? tokens_out + (int64_t)step * n : nullptr,
+                           embed, d0.num_labels, (int64_t)d0.hidden * elem, x, s0->kv.slot_of_id,
+                           const_cast<int32_t *>(s0->kv.pos_of_slot), s0->kv.n_slots, pl->ws->err, cs);
+    if (r != E3_OK) return r;
+    int derr = 0;
+    E3_CUDA_TRY(cudaMemcpyAsync(&derr, pl->ws->err, sizeof(int), cudaMemcpyDeviceToHost, cs));
+    E3_CUDA_TRY(cudaStreamSynchronize(cs));
+    if (derr) {
+      E3_CUDA_TRY(cudaMemsetAsync(pl->ws->err, 0, sizeof(int), cs));
+      set_error("e3_decode_run: a token's slot, position or label lies outside the cache / vocabulary");
+      return E3_EINVAL;
+    }
+  }
+  return E3_OK;
+}
+
 e3_status e3_pipeline_trace(e3_pipeline *pl, int32_t *split, int32_t *n_valid, int64_t *ids_out, int64_t max_runs,
                             int64_t *n_runs) {
   E3_CHECK_ARG(pl && n_runs, "null argument");

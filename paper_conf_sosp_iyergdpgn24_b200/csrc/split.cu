@@ -515,6 +515,7 @@ static e3_status llama_run(e3_split *s, cudaStream_t st, const void *x_in, const
         ra.ex = exits;
         ra.lm_stats = ws.lm_stats;
         ra.lm_tiles = dec_tiles(V, E3_DEC_LOGITS);
+        ra.x = cur;   // the exiting rows -> ex.hidden (multi-step decode)
         E3_RUN(lm_decide_run(ra, st));
         first_ramp = false;
       }
@@ -641,6 +642,63 @@ static e3_status f32_run(e3_split *s, cudaStream_t st, const void *x_in, const i
   E3_RUN(compact_run(cur, id_in, ws.alive, B, (int64_t)S * H * 4, dst, n_surv_dev, ws.ctr, s->sms, st));
 #undef E3_RUN
   return E3_OK;
+}
+
+// Multi-step decode (e3_decode_run; R27): layer l of this split's
+// K/V entries for the tokens of one chunk (<= B, ids_in [nv]) whose exit
+// layer lies before l, computed from their exit hidden rows (ex->hidden):
+// RMSNorm1_l -> the layer's QKV projection with the RoPE + KV-append epilogue
+// (rows outside the mask write nothing; q goes to scratch).
+e3_status llama_fill_layer(e3_split *s, int l, cudaStream_t st, const int64_t *ids_in, int nv, const e3_exits &ex,
+                           int64_t *ids_buf) {
+  const e3_split_desc &d = s->d;
+  Workspace &ws = *s->ws;
+  const int B = d.batch, H = d.hidden;
+  const int i = l - d.layer_begin;
+  const int kvh = d.kv_heads > 0 ? d.kv_heads : d.heads;
+  const int nqkv = (d.heads + 2 * kvh) * 128;
+  const int elem = d.dtype == E3_DTYPE_FP32 ? 4 : 2;
+  const e3_layer_weights &L = s->L[i];
+  e3_status r = fill_prep_run(ids_in, nv, B, ex.hidden, ex.capacity, ex.exit_layer, l, (int64_t)H * elem, ws.xa,
+                              ids_buf, ws.alive, st);
+  if (r != E3_OK) return r;
+  DecArgs a{};
+  a.T = B;
+  a.nh = d.heads;
+  a.kvh = kvh;
+  a.max_ctx = s->kv.max_ctx;
+  a.ids = ids_buf;
+  a.n_valid_host = B;
+  a.slot_of_id = s->kv.slot_of_id;
+  a.id_cap = s->kv.id_capacity;
+  a.pos_of_slot = s->kv.pos_of_slot;
+  a.n_slots = s->kv.n_slots;
+  a.err = ws.err;
+  a.alive = ws.alive;
+  a.init_alive = 0;
+  if (d.dtype == E3_DTYPE_FP32) {
+    auto *x1 = static_cast<float *>(ws.x1), *qkv = static_cast<float *>(ws.qkv);
+    r = f32_rms_run(static_cast<const float *>(ws.xa), L.ln1_g, x1, B, H, d.norm_eps, st);
+    if (r == E3_OK) r = f32_gemm_run(x1, H, L.w_qkv, nullptr, nullptr, qkv, B, nqkv, H, E3_EPI_BIAS, st);
+    if (r == E3_OK)
+      r = f32_rope_kv_run(qkv, ws.pool, static_cast<float *>(s->kv_k[l]), static_cast<float *>(s->kv_v[l]), ws.rope,
+                          a, st);
+    return r;
+  }
+  r = rmsnorm_run(ws.xa, L.ln1_g, ws.x1, B, H, d.norm_eps, st);
+  if (r != E3_OK) return r;
+  a.N = nqkv;
+  a.K = H;
+  a.max_contrib = s->mc_qkv;
+  a.epi = E3_DEC_QKV_ROPE;
+  a.Y = reinterpret_cast<__nv_bfloat16 *>(ws.qkv);
+  a.ldo = d.heads * 128;
+  a.kc = reinterpret_cast<__nv_bfloat16 *>(s->kv_k[l]);
+  a.vc = reinterpret_cast<__nv_bfloat16 *>(s->kv_v[l]);
+  a.rope = ws.rope;
+  a.part = ws.dec_part;
+  a.tickets = ws.dec_tickets;
+  return dec_run(s->dmaps[i].qkv, a, s->sms, st);
 }
 
 static LnGemmArgs oln_args(const void *bias, const void *R, const void *g, const void *b, float eps, int M, int H,

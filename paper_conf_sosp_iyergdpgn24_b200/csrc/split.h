@@ -75,5 +75,8 @@ e3_status split_create_shared(const e3_split_desc *d, const e3_weights *w, int d
 e3_status split_run_to(e3_split *s, cudaStream_t st, const void *x_in, const int64_t *id_in,
                        const int32_t *n_valid_dev, int n_valid_host, const RingDst &dst, int32_t *n_surv_dev,
                        const e3_exits *ex);
+// multi-step decode: K/V of layer l (in this split) for the chunk's tokens exited before l
+e3_status llama_fill_layer(e3_split *s, int l, cudaStream_t st, const int64_t *ids_in, int nv, const e3_exits &ex,
+                           int64_t *ids_buf);
 
 }  // namespace e3
