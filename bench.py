@@ -46,6 +46,7 @@ if ROOT not in sys.path:
     sys.path.insert(0, ROOT)
 
 METRIC = "inputs/sec at constant batch (EE-BERT-base) at 1/2/4/8 B200; % roofline"
+METRIC_LM = "tokens/sec of the early-exit decode step (EE decoder LLM, Llama-7B shape) at constant batch"
 
 
 def parse():
@@ -56,7 +57,11 @@ def parse():
     ap.add_argument("--impl", default="ours", choices=["ours", "reference"])
     ap.add_argument("--config", default="bb")
     ap.add_argument("--inputs-per-gpu", type=int, default=None,
-                    help="default 8192 (encoders: > L2 of activations), 256 (llama: 256 sequences' KV caches)")
+                    help="default 8192 (encoders: > L2 of activations), 512 (llama: 512 sequences' KV caches, "
+                         "~138 GB, so that padding stays near 5 %% at every split)")
+    ap.add_argument("--decode-steps", type=int, default=0,
+                    help="llama: one step = e3_decode_run of this many greedy tokens per sequence (NEXT-2: "
+                         "skipped layers' K/V filled from the exit state); 0 = one token (e3_pipeline_run)")
     ap.add_argument("--plan", default="per-ramp", choices=["per-ramp", "cut6"])
     ap.add_argument("--no-e2e", action="store_true")
     ap.add_argument("--no-cpu", action="store_true")
@@ -196,15 +201,17 @@ def run_reference(args):
         total += n
         t_all += dt
     v = total / t_all
+    unit = "tokens/s" if cfg.arch == "llama" else "inputs/s"
     print(json.dumps({
-        "impl": "reference", "metric": METRIC, "value": round(v, 3), "unit": "inputs/s",
+        "impl": "reference", "metric": METRIC_LM if cfg.arch == "llama" else METRIC, "value": round(v, 3),
+        "unit": unit,
         "n_gpus": args.gpus, "steps": args.steps, "warmup": args.warmup,
         "ms_per_step": round(1000 * t_all / args.steps, 1), "higher_is_better": True, "scaling": "weak",
         "vs_baseline": None, "dtype": "f64", "data": "synthetic",
         "config": {"workload": cfg.name, "batch": cfg.batch, "seq_len": cfg.seq, "plan": "per-input (oracle)"},
-        "cpu_baseline": {"value": round(v, 3), "unit": "inputs/s", "cores": cores, "kind": "oracle",
+        "cpu_baseline": {"value": round(v, 3), "unit": unit, "cores": cores, "kind": "oracle",
                          "sample": f"{n} inputs per step of the {cfg.name} workload, fp64 NumPy oracle"},
-        "e2e": {"value": round(v, 3), "unit": "inputs/s", "h2d_bytes_per_step": 0, "d2h_bytes_per_step": 0},
+        "e2e": {"value": round(v, 3), "unit": unit, "h2d_bytes_per_step": 0, "d2h_bytes_per_step": 0},
     }), flush=True)
 
 
@@ -228,20 +235,23 @@ def main():
     cfg, tau = load_workload(args.config)
     bounds, plan_name = plan_bounds(cfg, args.plan)
     llama = cfg.arch == "llama"
-    n = args.inputs_per_gpu or (256 if llama else 8192)
+    n = args.inputs_per_gpu or (512 if llama else 8192)
+    dsteps = args.decode_steps if llama else 0
     if llama:
         # weights generated layer by layer straight into HBM (13.5 GB bf16);
         # one KV cache slot per sequence (token), ctx positions pre-filled with
         # N(0, 1) on the device (same recipe as e3data.make_kv, device stream)
         layers = (e3data.make_layer(cfg, l) for l in range(cfg.layers))
         ramp = e3data.make_ramp(cfg, 0)
-        kv = api.KVCache(cfg, n, cfg.ctx + 1, n * world, dev)
+        kv = api.KVCache(cfg, n, cfg.ctx + max(1, dsteps), n * world, dev)
         g = torch.Generator(device=dev)
         g.manual_seed(1234 + rank)
         for t in kv.k + kv.v:
             t[:, :, :cfg.ctx].normal_(generator=g)
         kv.slot_of_id.copy_(torch.arange(n * world, device=dev, dtype=torch.int32) % n)
         model = api.DeviceModel(cfg, {"layers": layers, "ramps": [ramp] * cfg.n_ramps}, dev, kv=kv)
+        if dsteps:
+            embed = torch.from_numpy(e3data.make_embed(cfg)).to(torch.bfloat16).to(dev)
     else:
         W = e3data.make_weights(cfg)
         model = api.DeviceModel(cfg, W, dev)
@@ -286,8 +296,10 @@ def main():
     else:
         ids_dev = torch.arange(0, n, dtype=torch.int64, device=dev)   # local ids index the exit arrays
         ids_host = torch.arange(0, n, dtype=torch.int64).pin_memory()
-        ex = api.ExitBuffers(n, cfg.classes, cfg.n_ramps, dev)
+        ex = api.ExitBuffers(n, cfg.classes, cfg.n_ramps, dev, hidden=cfg.hidden if dsteps else 0)
         pipe = api.Pipeline(model, api.make_plan(cfg, bounds, tau, lag=1))
+        if dsteps:
+            x_dec = torch.empty_like(x_dev[:, 0, :])
 
     def barrier():
         if world > 1:
@@ -298,6 +310,10 @@ def main():
         with torch.cuda.stream(stream):
             if cfg.test == "patience":   # dependent exits: per-input counters start at zero every job
                 ex.state.zero_()
+            if dsteps:                   # multi-step decode: every sequence restarts at position ctx
+                model.kv.pos_of_slot.fill_(cfg.ctx)
+                x_dec.copy_(x_dev[:, 0, :])
+                return p.decode(x_dec, ids_dev, dsteps, embed, ex, stream=stream)[1]
             st = p.run(x_host if host else x_dev, ids_host if host else ids_dev, ex, stream=stream)
             if res is not None:   # D2H read of the step's result (exit records)
                 res[0].copy_(ex.exit_layer, non_blocking=True)
@@ -334,8 +350,9 @@ def main():
         ms, stats = timed(args.steps)
     launches = (_lib.lib.e3_kernel_launches() - launches0) // args.steps * args.steps
     clocks = clk.summary()
-    total_inputs = n * world * args.steps
+    total_inputs = n * world * args.steps * max(1, dsteps)    # llama: tokens
     value = total_inputs / (ms / 1000.0)
+    unit = "tokens/s" if llama else "inputs/s"
 
     # exit histogram + invariants of the last step
     if stage_mode:
@@ -350,7 +367,7 @@ def main():
 
     # e2e: host-pinned inputs through the same C-ABI call, results read back
     e2e = None
-    if not args.no_e2e:
+    if not args.no_e2e and not dsteps:
         cap = ex.capacity
         res = (torch.empty(cap, dtype=torch.int32).pin_memory(), torch.empty(cap, dtype=torch.int32).pin_memory(),
                torch.empty(cap, dtype=torch.float32).pin_memory())
@@ -358,7 +375,7 @@ def main():
         torch.cuda.synchronize()
         ms_e2e, _ = timed(args.steps, host=True, res=res)
         row = cfg.seq * cfg.hidden * 2
-        e2e = {"value": round(total_inputs / (ms_e2e / 1000.0), 1), "unit": "inputs/s",
+        e2e = {"value": round(total_inputs / (ms_e2e / 1000.0), 1), "unit": unit,
                "h2d_bytes_per_step": int(n * world * (row + 8)),        # the whole job's inputs + ids
                "d2h_bytes_per_step": int(cap * 12 * world)}             # every rank reads its exit records
 
@@ -443,7 +460,7 @@ def main():
     cpu = None
     if rank == 0 and world == 1 and not args.no_cpu:
         rate, dt = cpu_oracle_rate(cfg, tau, args.cpu_inputs)
-        cpu = {"value": round(rate, 3), "unit": "inputs/s", "cores": len(os.sched_getaffinity(0)),
+        cpu = {"value": round(rate, 3), "unit": unit, "cores": len(os.sched_getaffinity(0)),
                "kind": "oracle",
                "sample": f"{args.cpu_inputs} inputs of the {cfg.name} workload through the fp64 NumPy "
                          f"oracle ({dt:.1f} s)"}
@@ -452,12 +469,12 @@ def main():
         n1 = max(1, args.cpu_inputs // 4)
         with threadpool_limits(limits=1):
             rate1, dt1 = cpu_oracle_rate(cfg, tau, n1, seed_offset=10_000)
-        cpu["one_thread"] = {"value": round(rate1, 3), "unit": "inputs/s", "cores": 1,
+        cpu["one_thread"] = {"value": round(rate1, 3), "unit": unit, "cores": 1,
                              "sample": f"{n1} inputs ({dt1:.1f} s)"}
 
     if rank == 0:
         out = {
-            "metric": METRIC, "value": round(value, 1), "unit": "inputs/s", "n_gpus": world,
+            "metric": METRIC if not llama else METRIC_LM, "value": round(value, 1), "unit": unit, "n_gpus": world,
             "steps": args.steps, "warmup": max(args.warmup, 3), "ms_per_step": round(ms_step, 3),
             "higher_is_better": True, "scaling": "weak", "vs_baseline": None, "dtype": "bf16",
             "data": "synthetic (seeded random-init weights and N(0,1) embedded inputs, e3data)",
