@@ -267,7 +267,9 @@ def main():
         # lands at its input's slot on the rank where the input exits
         from paper_conf_sosp_iyergdpgn24_b200 import parallel as par
         k = args.stages or min(world, 4)
-        prof_path = os.path.join(ROOT, "profiles", f"r01_planner_profile_{args.config}.json")
+        prof_path = os.path.join(ROOT, "profiles", f"r02_planner_profile_{args.config}.json")
+        if not os.path.exists(prof_path):
+            prof_path = os.path.join(ROOT, "profiles", f"r01_planner_profile_{args.config}.json")
         if args.planner == "dp" and os.path.exists(prof_path):
             # profile-driven DP (planner.py, NEXT-1) restricted to k stages
             from paper_conf_sosp_iyergdpgn24_b200 import planner as pln
