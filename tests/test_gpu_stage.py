@@ -222,3 +222,35 @@ def test_two_stage_nccl_two_gpus(api):
     model = api.DeviceModel(cfg, e3data.make_weights(cfg), DEV)
     el1, _ = _single(api, model, cfg, (0, 2, 4), cfg.tau, bf16_tensor(e3data.make_inputs(cfg, range(N))))
     assert np.array_equal(el, el1)
+
+
+def test_dp_planned_layout_runs_through_the_library(api):
+    """NEXT-1 end to end: planner.plan_dp on the measured r02 profile chooses
+    cuts and replicas for 4 GPUs (forced to 3 stages so that transfers
+    happen); the layout runs through the library's stage pipeline (LOOPBACK,
+    4 ranks on this GPU) and matches the single-rank pipeline bitwise."""
+    import os
+    from paper_conf_sosp_iyergdpgn24_b200 import parallel as par, planner
+    cfg = e3data.get("bb")
+    tau = e3data.tau_for(cfg)
+    root = os.path.dirname(os.path.dirname(os.path.abspath(__file__)))
+    prof = planner.Profile.load(os.path.join(root, "profiles", "r02_planner_profile_bb.json"))
+    surv = lambda l: 1.0 - sum(e for r, e in zip(cfg.ramp_layers, cfg.exit_profile) if r < l)
+    layout, _ = planner.plan_dp(cfg.ramp_layers, surv, prof, 4, n_stages=3)
+    assert layout.world == 4 and layout.n_stages == 3
+    bounds = tuple(range(13))
+    W = e3data.make_weights(cfg)
+    model = api.DeviceModel(cfg, W, DEV)
+    N = 384
+    X = bf16_tensor(e3data.make_inputs(cfg, range(N)))
+    ids = torch.arange(N, dtype=torch.int64, device=DEV)
+    lo, hi = par.input_share(layout, 0, N)
+    inputs = {}
+    for r in range(layout.world):
+        a, b = par.input_share(layout, r, N)
+        if b > a:
+            inputs[r] = (X[a:b], ids[a:b])
+    res = _run_ranks(api, model, cfg, bounds, tau, par.placement(layout, bounds), inputs, layout.world)
+    el, lg = _merge(res, N, cfg.classes)
+    el1, lg1 = _single(api, model, cfg, bounds, tau, X)
+    assert (el >= 0).all() and np.array_equal(el, el1) and np.array_equal(lg, lg1)
