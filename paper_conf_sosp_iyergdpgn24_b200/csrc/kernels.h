@@ -100,6 +100,7 @@ e3_status ramp_run(const RampArgs &a, cudaStream_t st);
 // BERT ramp on (group, slice) CTAs without clusters (rampc.cu); ctr_words =
 // the workspace counters (RampArgs.done_ctr)
 bool ramp_bert2_supported(int H, int C);
+bool ramp_ticket_mode();   // E3_RAMP_TICKET / E3_FUSED_RC: the ticketed ramp for every BERT ramp
 e3_status ramp_bert2_run(const RampArgs &a, unsigned *ctr_words, cudaStream_t st);
 // the split's last BERT ramp (pre-LN rows, a.ln_g set) fused with the stable
 // LN + compaction of the survivors into dst; *done = false when the shape

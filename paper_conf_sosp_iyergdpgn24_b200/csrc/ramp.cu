@@ -933,10 +933,13 @@ e3_status ramp_run(const RampArgs &a, cudaStream_t st) {
     set_error("ramp: arch not implemented");
     return E3_EUNSUPPORTED;
   }
-  // r02: the cluster-free (group, slice) ramp of rampc.cu wherever it applies
-  // (it shares its arithmetic with the fused ramp + compaction, so a ramp
-  // evaluated inside a split and at a split's end gives identical bits)
-  if (ramp_bert2_supported(a.H, a.C) && a.done_ctr && a.pool_ws && getenv("E3_RAMP_CLUSTER") == nullptr)
+  // r02: the cluster-free (group, slice) ramp of rampc.cu on request
+  // (E3_RAMP_TICKET=1, or E3_FUSED_RC=1 whose fused last ramp shares its
+  // arithmetic, so a ramp inside a split and at a split's end give identical
+  // bits).  Not the default: in the BB pipeline it measured 2.2 % slower than
+  // this cluster kernel on the same box (bench: 58.4k vs 59.7k inputs/s; the
+  // graph-replayed single split of scripts/timeline.py had shown the reverse)
+  if (ramp_ticket_mode() && ramp_bert2_supported(a.H, a.C) && a.done_ctr && a.pool_ws)
     return ramp_bert2_run(a, a.done_ctr, st);
   if (a.C < 1 || a.C > kMaxC || a.H % (8 * kCS) || a.H > 2048 || ramp_smem_bytes(a.H, a.C) > 220 * 1024) {
     set_error("ramp: need 1 <= C <= 16, H % 128 == 0 and H <= 2048");

@@ -473,6 +473,11 @@ e3_status rc_occupancy(int smem, int *occ) {
 
 E3_TL_SETTER(tl_set_rampc)
 
+bool ramp_ticket_mode() {
+  static const bool on = getenv("E3_RAMP_TICKET") != nullptr || getenv("E3_FUSED_RC") != nullptr;
+  return on;
+}
+
 bool ramp_bert2_supported(int H, int C) {
   const int kSl = ramp_slices(H);
   // partials [groups][kSl][16][C] f32 live in the [B, H] f32 pool workspace

@@ -465,8 +465,8 @@ np.save(sys.argv[3], np.concatenate([ex.exit_layer.cpu().numpy()[:, None].astype
 @pytest.mark.parametrize("name,n", [("tiny", 200), ("bb", 256)])
 def test_fused_ramp_compaction_equals_two_kernel_path(name, n, tmp_path):
     """E3_FUSED_RC=1 (the cooperative ramp + LN2 + compaction launch, off by
-    default) gives bitwise the records of the default ticketed ramp +
-    ln_compact path: both share the ramp arithmetic (rampc.cu)."""
+    default) gives bitwise the records of the ticketed ramp + ln_compact path
+    (E3_RAMP_TICKET=1): both share the ramp arithmetic (rampc.cu)."""
     import os
     import subprocess
     import sys
@@ -477,6 +477,7 @@ def test_fused_ramp_compaction_equals_two_kernel_path(name, n, tmp_path):
     for fused in (False, True):
         env = dict(os.environ)
         env.pop("E3_FUSED_RC", None)
+        env["E3_RAMP_TICKET"] = "1"
         if fused:
             env["E3_FUSED_RC"] = "1"
         f = tmp_path / f"o{int(fused)}.npy"
