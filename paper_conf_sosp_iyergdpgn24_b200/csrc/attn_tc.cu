@@ -37,7 +37,9 @@ constexpr int QT = 128;        // query rows per item
 // and TMEM latencies)
 template <int SKV>
 struct AThr {
-  static constexpr int KP = SKV <= 128 ? 2 : 4;
+  // r02: 2 threads per query row at every SKV (above 128 keys the second CTA
+  // per SM, below, replaces the r01 layout of 4 threads per row in one CTA)
+  static constexpr int KP = 2;
   static constexpr int kThreads = 128 * KP;
 };
 
@@ -49,13 +51,21 @@ struct ACfg {
   static constexpr int kQ = QT * D * 2;                  // 16 KB
   static constexpr int kKV = SKV * D * 2;                // 16 .. 32 KB
   static constexpr int kP = ((SKV + 63) / 64) * QT * 128;   // bf16 P in 64-key SW128 blocks
-  static constexpr int kBuf = kQ + 2 * kKV;              // Q | K | V
-  static constexpr bool kPInQK = (kP <= kQ + kKV);       // P overwrites the dead Q|K tiles
+  // above 128 keys (S = 197 -> 224, r02): TWO CTAs per SM instead of one
+  // double-buffered CTA -- one CTA's softmax overlaps the other's loads and
+  // MMAs (r01 trace: 3.6 us per item, strictly serial load -> S -> softmax
+  // -> PV -> store).  To fit two 256-thread CTAs, P (64 KB) overwrites the
+  // dead Q | K tiles plus a pad placed before V: [Q | K | pad | V].
+  static constexpr bool kTwoPerSm = SKV > 128;
+  static constexpr int kPad = (kTwoPerSm && kP > kQ + kKV) ? kP - kQ - kKV : 0;
+  static constexpr int kVOff = kQ + kKV + kPad;          // V tile offset in a buffer
+  static constexpr int kBuf = kVOff + kKV;               // Q | K | (pad) | V
+  static constexpr bool kPInQK = (kP <= kQ + kKV + kPad);   // P overwrites the dead Q|K(|pad) tiles
   static constexpr int kExtra = 1024 + 64 + 2 * 2 * AThr<SKV>::KP * QT * 4;
 #ifdef E3_ATTN_SINGLE_BUF   // diagnostics: occupancy instead of double buffering
   static constexpr int kNBuf = 1;
 #else
-  static constexpr int kNBuf = (2 * kBuf + (kPInQK ? 0 : kP) + kExtra <= 232448) ? 2 : 1;   // double buffer if it fits
+  static constexpr int kNBuf = kTwoPerSm ? 1 : ((2 * kBuf + (kPInQK ? 0 : kP) + kExtra <= 232448) ? 2 : 1);
 #endif
   static constexpr int kSmem = kNBuf * kBuf + (kPInQK ? 0 : kP) + kExtra;
   static constexpr int kSCols = SKV <= 128 ? 128 : 256;      // one S (later O, 64 columns) accumulator
@@ -81,7 +91,7 @@ __device__ __forceinline__ void atrace(int j, int kind) {
 // kMask: S < SKV, keys >= S are masked; without it (S == SKV, BB) the
 // softmax loops carry no per-element compare / select
 template <int SKV, bool kMask>
-__global__ void __launch_bounds__(AThr<SKV>::kThreads, SKV == 128 ? 2 : 1)
+__global__ void __launch_bounds__(AThr<SKV>::kThreads, 2)
     attn_tc_kernel(const __grid_constant__ CUtensorMap tq, const __grid_constant__ CUtensorMap tkv,
                    const __grid_constant__ CUtensorMap tctx, int S, int H, int heads, int n_items) {
   using CF = ACfg<SKV>;
@@ -132,10 +142,10 @@ __global__ void __launch_bounds__(AThr<SKV>::kThreads, SKV == 128 ? 2 : 1)
     const int bh = item / qtiles, qt = item % qtiles;
     const int b = bh / heads, h = bh % heads;
     uint8_t *base = smem + buf * CF::kBuf;
-    mbar_expect_tx(&bar_load[buf], CF::kBuf);
+    mbar_expect_tx(&bar_load[buf], CF::kQ + 2 * CF::kKV);   // the pad is not loaded
     tma_load_3d(base, &tq, &bar_load[buf], h * D, qt * QT, b);
     tma_load_3d(base + CF::kQ, &tkv, &bar_load[buf], H + h * D, 0, b);
-    tma_load_3d(base + CF::kQ + CF::kKV, &tkv, &bar_load[buf], 2 * H + h * D, 0, b);
+    tma_load_3d(base + CF::kVOff, &tkv, &bar_load[buf], 2 * H + h * D, 0, b);
   };
 
   uint32_t load_phases = 0;                               // bit i: parity of bar_load[i] (thread 0)
@@ -164,7 +174,7 @@ __global__ void __launch_bounds__(AThr<SKV>::kThreads, SKV == 128 ? 2 : 1)
     const int buf = (CF::kNBuf == 2) ? (j & 1) : 0;
     uint8_t *sQ = smem + buf * CF::kBuf;
     uint8_t *sK = sQ + CF::kQ;
-    uint8_t *sV = sK + CF::kKV;
+    uint8_t *sV = sQ + CF::kVOff;
     uint8_t *sP = CF::kPInQK ? sQ : pbuf_sep;
     const int bh = item / qtiles, qt = item % qtiles;
     const int b = bh / heads, h = bh % heads;
