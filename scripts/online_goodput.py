@@ -63,7 +63,10 @@ def main():
         if os.path.exists(os.path.join(ROOT, "profiles", "r02_planner_profile_bb.json")) else \
         planner.Profile.load(os.path.join(ROOT, "profiles", "r01_planner_profile_bb.json"))
     est = online.BatchProfileEstimator(cfg.n_ramps, p=2, d=1)
-    rp = online.Replanner(cfg.ramp_layers, lambda s: planner.plan_dp(cfg.ramp_layers, s, prof, args.plan_gpus)[0])
+    # two stages forced (with free transfers pure replication is always optimal on identical GPUs,
+    # so the cut position is what the drifting profile moves)
+    rp = online.Replanner(cfg.ramp_layers, lambda s: planner.plan_dp(cfg.ramp_layers, s, prof, args.plan_gpus,
+                                                                       n_stages=2)[0])
     batcher = online.SloBatcher(args.batch, args.slo, 0.2)
     xbuf = torch.empty((args.batch, cfg.seq, cfg.hidden), dtype=torch.bfloat16, device=dev)
     ex = api.ExitBuffers(args.batch, cfg.classes, cfg.n_ramps, dev, logits=False)
