@@ -1,0 +1,21 @@
+# Round-2 measurement pass (on the GPU box, from the repo root): smoke, bench
+# lines for every config, the multi-step decode and PABEE lines, the device
+# timeline of a BB split run, the online goodput run, the ncu launch list of
+# the BB bench command and one --set full capture of a BB split run.
+mkdir -p gpurun_out
+timeout 600 python -c "import __graft_entry__ as g; g.smoke()" > gpurun_out/smoke.txt 2>&1; echo smoke=$?
+timeout 900 python bench.py > gpurun_out/r02_bench_bb.json 2> gpurun_out/r02_bench_bb.err; echo bb=$?
+timeout 600 python bench.py --impl reference --steps 2 --warmup 1 > gpurun_out/r02_bench_ref.json 2> gpurun_out/r02_bench_ref.err
+for c in tiny bl vt; do timeout 900 python bench.py --config $c > gpurun_out/r02_bench_$c.json 2> gpurun_out/r02_bench_$c.err; echo $c=$?; done
+timeout 1200 python bench.py --config lm > gpurun_out/r02_bench_lm.json 2> gpurun_out/r02_bench_lm.err; echo lm=$?
+timeout 900 python bench.py --config lm --decode-steps 4 --steps 3 --no-cpu > gpurun_out/r02_bench_lm_decode4.json 2> gpurun_out/r02_bench_lm_decode4.err
+timeout 600 python bench.py --config bbp --no-cpu > gpurun_out/r02_bench_bbp.json 2> gpurun_out/r02_bench_bbp.err
+timeout 600 python bench.py --plan cut6 --no-cpu > gpurun_out/r02_bench_bb_cut6.json 2> gpurun_out/r02_bench_bb_cut6.err
+timeout 300 python scripts/timeline.py bb 1 3 > gpurun_out/r02_timeline_bb_layer.txt 2>&1
+timeout 900 python scripts/online_goodput.py > gpurun_out/online.log 2>&1; echo online=$?
+timeout 900 ncu --metrics gpu__time_duration.sum,dram__bytes_read.sum,dram__bytes_write.sum --clock-control none --csv \
+  --log-file gpurun_out/launches_bb.csv python bench.py --steps 1 --warmup 1 --no-cpu --no-e2e > gpurun_out/ncu_bench.log 2>&1; echo ncu1=$?
+timeout 1200 ncu --set full --clock-control none --import-source on \
+  -k regex:"gemm_bf16|attn_tc|ramp_bert|ln_compact|layernorm_kernel|gemm_ln" -c 10 \
+  -o gpurun_out/layer_full python scripts/layer_time.py 1 > gpurun_out/ncu_full.log 2>&1; echo ncu2=$?
+for f in gpurun_out/r02_bench_*.json; do python -c "import json,sys; d=json.loads(open('$f').read().strip().splitlines()[-1]); print('$f', d.get('value'), d.get('unit'), d.get('ms_per_step'), (d.get('roofline') or {}).get('frac'), (d.get('clocks') or {}).get('sm_mhz'))" 2>/dev/null; done
