@@ -172,6 +172,10 @@ typedef struct e3_exits {
   void *hidden;        /* LLAMA: [capacity, H] (activation dtype) -- the hidden row each
                           token exited with (e3_decode_run fills the skipped layers'
                           K/V from it); NULL: not recorded                             */
+  float *ramp_metric;  /* [capacity, ramp_metric_stride]: the exit metric of EVERY ramp a
+                          row is evaluated at (model ramp index), exiting or not -- the
+                          profile the exit-wrapper's ramp choice needs (planner); NULL: off */
+  int32_t ramp_metric_stride;
 } e3_exits;
 
 typedef struct e3_split e3_split;

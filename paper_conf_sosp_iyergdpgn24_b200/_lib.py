@@ -69,7 +69,8 @@ class Weights(C.Structure):
 
 class Exits(C.Structure):
     _fields_ = [("exit_layer", P), ("label", P), ("conf", P), ("logits", P), ("capacity", I64),
-                ("n_exit", P), ("ramp_count", P), ("state", P), ("hidden", P)]
+                ("n_exit", P), ("ramp_count", P), ("state", P), ("hidden", P), ("ramp_metric", P),
+                ("ramp_metric_stride", I32)]
 
 
 class Plan(C.Structure):

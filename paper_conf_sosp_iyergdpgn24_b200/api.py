@@ -130,9 +130,11 @@ class ExitBuffers:
     """Exit records indexed by input id (e3_exits)."""
 
     def __init__(self, capacity: int, classes: int, n_ramps: int, device, logits=True, hidden=0,
-                 hidden_dtype=torch.bfloat16):
+                 hidden_dtype=torch.bfloat16, ramp_metrics=False):
         """hidden > 0: also record each token's exit hidden row ([capacity,
-        hidden], the activation dtype) -- needed by Pipeline.decode."""
+        hidden], the activation dtype) -- needed by Pipeline.decode.
+        ramp_metrics: also record the exit metric of every ramp a row is
+        evaluated at ([capacity, n_ramps], NaN where not evaluated)."""
         dev = torch.device(device)
         self.capacity = capacity
         self.exit_layer = torch.full((capacity,), -1, dtype=torch.int32, device=dev)
@@ -144,10 +146,13 @@ class ExitBuffers:
         # dependent exits (E3_TEST_PATIENCE): per-input counter state, zero per job
         self.state = torch.zeros((capacity,), dtype=torch.int32, device=dev)
         self.hidden = torch.zeros((capacity, hidden), dtype=hidden_dtype, device=dev) if hidden else None
+        self.ramp_metric = torch.full((capacity, max(n_ramps, 1)), float("nan"), dtype=torch.float32,
+                                      device=dev) if ramp_metrics else None
         self.c = _lib.Exits(self.exit_layer.data_ptr(), self.label.data_ptr(), self.conf.data_ptr(),
                             None if self.logits is None else self.logits.data_ptr(), capacity,
                             self.n_exit.data_ptr(), self.ramp_count.data_ptr(), self.state.data_ptr(),
-                            None if self.hidden is None else self.hidden.data_ptr())
+                            None if self.hidden is None else self.hidden.data_ptr(),
+                            None if self.ramp_metric is None else self.ramp_metric.data_ptr(), max(n_ramps, 1))
 
     def reset(self):
         self.exit_layer.fill_(-1)
@@ -158,6 +163,8 @@ class ExitBuffers:
         self.n_exit.zero_()
         self.ramp_count.zero_()
         self.state.zero_()
+        if self.ramp_metric is not None:
+            self.ramp_metric.fill_(float("nan"))
 
 
 class Split:

@@ -309,6 +309,8 @@ __global__ void __launch_bounds__(kRT) f32_ramp_kernel(RampArgs a) {
       pass = metric < a.tau;
     }
     const bool exit_now = pass || a.final_ramp;
+    if (a.ex.ramp_metric && a.id[b] >= 0 && a.id[b] < a.ex.capacity)
+      a.ex.ramp_metric[a.id[b] * a.ex.ramp_metric_stride + a.ramp_index] = metric;
     const int64_t id = a.id[b];
     const bool rec = exit_now && id >= 0 && id < a.ex.capacity;
     if (rec) {

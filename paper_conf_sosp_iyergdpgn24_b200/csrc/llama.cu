@@ -252,6 +252,8 @@ __global__ void __launch_bounds__(128) lm_decide_kernel(RampArgs a) {
     pass = metric < a.tau;
   }
   const bool exit_now = pass || a.final_ramp;
+  if (lane == 0 && a.ex.ramp_metric && a.id[b] >= 0 && a.id[b] < a.ex.capacity)
+    a.ex.ramp_metric[a.id[b] * a.ex.ramp_metric_stride + a.ramp_index] = metric;
   const int64_t id = a.id[b];
   if (exit_now && id >= 0 && id < a.ex.capacity) {
     if (lane == 0) {

@@ -298,6 +298,8 @@ __global__ void __launch_bounds__(kRThreads, 1) ramp_bert_kernel(RampArgs a) {
       pass = metric < a.tau;
     }
     exit_now = pass || a.final_ramp;
+    if (a.ex.ramp_metric && row_id >= 0 && row_id < a.ex.capacity)
+      a.ex.ramp_metric[row_id * a.ex.ramp_metric_stride + a.ramp_index] = metric;
     tlB = tl_now();
     if (exit_now) {
       const int64_t id = row_id;
@@ -520,6 +522,8 @@ __global__ void __launch_bounds__(kVitKQ * 2 * CB) ramp_vit_kernel(RampArgs a, i
           pass = metric < a.tau;
         }
         exit_now = pass || a.final_ramp;
+        if (a.ex.ramp_metric && a.id[b] >= 0 && a.id[b] < a.ex.capacity)
+          a.ex.ramp_metric[a.id[b] * a.ex.ramp_metric_stride + a.ramp_index] = metric;
         const int64_t id = a.id[b];
         if (exit_now && id >= 0 && id < a.ex.capacity) {
           if (a.ex.exit_layer) a.ex.exit_layer[id] = a.layer;
@@ -817,6 +821,8 @@ __global__ void __launch_bounds__(kVtcThreads, 1) ramp_vit_tc_kernel(RampArgs a,
           pass = metric < a.tau;
         }
         exit_now = pass || a.final_ramp;
+        if (a.ex.ramp_metric && a.id[b] >= 0 && a.id[b] < a.ex.capacity)
+          a.ex.ramp_metric[a.id[b] * a.ex.ramp_metric_stride + a.ramp_index] = metric;
         const int64_t id = a.id[b];
         if (exit_now && id >= 0 && id < a.ex.capacity) {
           if (a.ex.exit_layer) a.ex.exit_layer[id] = a.layer;

@@ -277,6 +277,8 @@ struct RampSlice {
           pass = metric < a.tau;
         }
         exit_now = pass || a.final_ramp;
+        if (a.ex.ramp_metric && a.id[b] >= 0 && a.id[b] < a.ex.capacity)
+          a.ex.ramp_metric[a.id[b] * a.ex.ramp_metric_stride + a.ramp_index] = metric;
         if (exit_now) {
           const int64_t id = a.id[b];
           if (id >= 0 && id < a.ex.capacity) {

@@ -151,3 +151,60 @@ def brute_force_plan(ramp_layers: Sequence[int], survival: Callable[[int], float
 def throughput(bottleneck_us_per_input: float) -> float:
     """Inputs per second of a pipeline whose slowest stage costs `bottleneck`."""
     return 1e6 / bottleneck_us_per_input
+
+
+# ---------------------------------------------------------------------------
+# Exit-wrapper ramp control (SURVEY §8(f) NEXT-4; §3.4 PAPER.md:985-1017 "A
+# simple use-case here is to disable ramps that are not useful", §5.8.6
+# PAPER.md:2648-2654: disabling the exits inside a split "(except the last one
+# which is required)" gains up to 16 % "by avoiding exit-checking overheads").
+# Given every input's exit metric at every ramp (recorded on the GPU,
+# e3_exits.ramp_metric, in a profiling run whose thresholds never pass) the
+# choice of enabled ramps E changes where inputs exit; the cost per input of
+# a single-GPU chain cut at the enabled ramps is
+#     sum_l S_E(l) t_layer[l] + sum_{r in E} S_E(layer_r) t_ramp     (/ B)
+# with S_E(l) the fraction alive entering layer l.  Exhaustive over the
+# subsets of the non-final ramps (2^11 for EE-BERT-base).
+
+def exits_with(M, tau, test: str, enabled: Sequence[int], last: int):
+    """Exit ramp index of every input (rows of M [n, R]) when only the ramps
+    in `enabled` (plus the last) are evaluated; strict tests (R12)."""
+    import numpy as np
+    M = np.asarray(M, dtype=np.float64)
+    n = M.shape[0]
+    out = np.full(n, last, dtype=np.int64)
+    undecided = np.ones(n, dtype=bool)
+    for r in sorted(set(enabled) - {last}):
+        t = np.float64(np.float32(tau[r]))
+        ok = (M[:, r] > t) if test == "maxprob" else (M[:, r] < t)
+        hit = undecided & ok
+        out[hit] = r
+        undecided &= ~hit
+    return out
+
+
+def ramp_plan_cost(exit_ramp, ramp_layers: Sequence[int], enabled: Sequence[int], prof: Profile) -> float:
+    """Expected GPU time per input (us) of the chain with `enabled` ramps."""
+    import numpy as np
+    L = ramp_layers[-1] + 1
+    exit_layer = np.asarray(ramp_layers)[exit_ramp]
+    alive = [float(np.mean(exit_layer >= l)) for l in range(L)]        # entering layer l
+    work = sum(alive[l] * prof.t_layer[l] for l in range(L))
+    ramps = sum(alive[ramp_layers[r]] * prof.t_ramp for r in set(enabled) | {len(ramp_layers) - 1})
+    return (work + ramps) / prof.batch
+
+
+def choose_ramps(M, tau, test: str, ramp_layers: Sequence[int], prof: Profile):
+    """Enabled ramp set (ascending, always with the last) of least cost;
+    returns (enabled, cost_us_per_input, exit ramp per profiled input)."""
+    R = len(ramp_layers)
+    last = R - 1
+    best = None
+    for mask in range(1 << (R - 1)):
+        en = tuple(r for r in range(R - 1) if (mask >> r) & 1) + (last,)
+        ex = exits_with(M, tau, test, en, last)
+        c = ramp_plan_cost(ex, ramp_layers, en, prof)
+        key = (round(c, 9), -len(en))                 # ties: keep more ramps (earlier answers)
+        if best is None or key < best[0]:
+            best = (key, en, c, ex)
+    return best[1], best[2], best[3]

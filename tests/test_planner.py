@@ -89,3 +89,32 @@ def test_bert_base_stage_cuts_match_the_survival_balance():
     assert lay.bounds == (0, 4, 12) and lay.replicas == (1, 1)
     lay, _ = plan_dp(ramps, surv, prof, 4, n_stages=4)
     assert lay.bounds == (0, 2, 4, 7, 12) and lay.replicas == (1, 1, 1, 1)
+
+
+def test_choose_ramps_extremes_and_hand_case():
+    import numpy as np
+    from paper_conf_sosp_iyergdpgn24_b200 import planner as pl
+    # 4 ramps after layers 0..3, max-prob metrics of 4 inputs, tau 0.5
+    M = np.array([[0.9, 0.1, 0.1, 0.1],      # exits at ramp 0 if enabled
+                  [0.1, 0.9, 0.1, 0.1],      # ramp 1
+                  [0.1, 0.1, 0.9, 0.1],      # ramp 2
+                  [0.1, 0.1, 0.1, 0.1]])     # last
+    tau = [0.5] * 4
+    rl = (0, 1, 2, 3)
+    assert pl.exits_with(M, tau, "maxprob", (0, 1, 2, 3), 3).tolist() == [0, 1, 2, 3]
+    assert pl.exits_with(M, tau, "maxprob", (1, 3), 3).tolist() == [3, 1, 3, 3]
+    free = pl.Profile((1.0,) * 4, 0.0, 0.0, 1)
+    en, cost, _ = pl.choose_ramps(M, tau, "maxprob", rl, free)
+    assert en == (0, 1, 2, 3)                              # free ramps: keep every one
+    # hand cost with t_layer 1, t_ramp 10: all ramps -> layers 1 + .75 + .5 + .25 = 2.5, ramps 10 (1 + .75
+    # + .5 + .25) = 25 -> 27.5; only the last -> layers 4, its ramp sees every input: 10 -> 14
+    dear = pl.Profile((1.0,) * 4, 10.0, 0.0, 1)
+    assert pl.ramp_plan_cost(pl.exits_with(M, tau, "maxprob", (0, 1, 2, 3), 3), rl, (0, 1, 2, 3), dear) == 27.5
+    en, cost, _ = pl.choose_ramps(M, tau, "maxprob", rl, dear)
+    assert en == (3,) and cost == 14.0
+    # moderate ramp cost: a ramp pays when it removes enough downstream work
+    mid = pl.Profile((1.0,) * 4, 0.2, 0.0, 1)
+    en, cost, _ = pl.choose_ramps(M, tau, "maxprob", rl, mid)
+    brute = min(pl.ramp_plan_cost(pl.exits_with(M, tau, "maxprob", e, 3), rl, e, mid)
+                for e in [tuple(r for r in range(3) if m >> r & 1) + (3,) for m in range(8)])
+    assert cost == pytest.approx(brute)
