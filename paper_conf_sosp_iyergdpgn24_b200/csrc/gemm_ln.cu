@@ -169,19 +169,6 @@ __global__ void __cluster_dims__(2, 1, 1) __launch_bounds__(kLThreads, 1)
     pdl_wait();
     pdl_trigger();
   }
-  // r02: the epilogue thread's residual slice (its row, its NH/2 columns) is
-  // loaded into registers while the mainloop runs, instead of a TMA of the
-  // whole tile after it (one L2 round trip less on the critical path)
-  constexpr int kRV = NH / 2 / 8;                 // uint4 per epilogue thread
-  constexpr bool kRegRes = kRV <= 24;
-  uint4 rres[kRegRes ? kRV : 1];
-  if (kRegRes && warp >= 4) {
-    const int rq = warp & 3, rh = (warp - 4) >> 2;
-    const int rm = m0 + rq * 32 + lane_id();
-    const uint4 *rp = reinterpret_cast<const uint4 *>(a.R + (size_t)rm * a.N + n0 + rh * (NH / 2));
-#pragma unroll
-    for (int j = 0; j < (kRegRes ? kRV : 1); ++j) rres[j] = rm < a.M ? __ldg(rp + j) : make_uint4(0, 0, 0, 0);
-  }
   __syncwarp();
   asm volatile("barrier.cluster.wait.aligned;" ::: "memory");   // the peer CTA is running
 
@@ -195,16 +182,16 @@ __global__ void __cluster_dims__(2, 1, 1) __launch_bounds__(kLThreads, 1)
   if (epi) {
     mbar_wait(tfull, 0);                          // all MMAs done: the stage buffers are drained
     tc_fence_after();
-    // the residual tile: prefetched into registers (kRegRes), else it lands by
-    // TMA exactly where y1 will be written (same 128-byte-swizzled layout)
-    if (!kRegRes && warp == 4 && lane == 0) {
+    // the residual tile lands, by TMA, exactly where y1 will be written
+    // (same 128-byte-swizzled block layout): one round trip for the whole tile
+    if (warp == 4 && lane == 0) {
       mbar_expect_tx(rbar, LM * NH * 2);
       for (int blk = 0; blk < NH / 64; ++blk) tma_load_2d(sY + blk * (LM * 128), &tmR, rbar, n0 + blk * 64, m0);
     }
     epi_bar256();                                 // sPar written by every epilogue thread
-    if (!kRegRes) mbar_wait(rbar, 0);
+    mbar_wait(rbar, 0);
     const uint32_t taddr = tmem_base + ((uint32_t)(q * 32) << 16);
-#pragma unroll
+#pragma unroll 1
     for (int c = 0; c < HC; c += 32) {
       const int col = h * HC + c;                 // within this CTA's NH columns
       uint32_t r[32];
@@ -214,8 +201,7 @@ __global__ void __cluster_dims__(2, 1, 1) __launch_bounds__(kLThreads, 1)
       uint4 rv[4], bv[4];
 #pragma unroll
       for (int j = 0; j < 4; ++j) {
-        rv[j] = kRegRes ? rres[kRegRes ? (c / 8 + j) : 0]
-                        : *reinterpret_cast<const uint4 *>(blk + (((ch0 + j) ^ (row & 7)) << 4));
+        rv[j] = *reinterpret_cast<const uint4 *>(blk + (((ch0 + j) ^ (row & 7)) << 4));
         bv[j] = reinterpret_cast<const uint4 *>(sPar + col)[j];
       }
       tmem_wait_ld();
