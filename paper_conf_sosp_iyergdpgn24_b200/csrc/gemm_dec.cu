@@ -53,7 +53,7 @@ struct DCfg {
   static constexpr int kXAtom = T * DK * 2;
   static constexpr int kWBytes = 2 * kWAtom;
   static constexpr int kXBytes = 2 * kXAtom;
-  static constexpr int kXStages = 2;
+  static constexpr int kXStages = T <= 64 ? 3 : 2;   // the third X stage is free at T <= 64 (same 4 W stages)
   static constexpr int kEBytes = DM * (T + 1) * 4;          // fp32 epilogue tile
   static constexpr int kStages = (kSmemMax - kEBytes - 1024 - 3072 - kXStages * kXBytes) / kWBytes;
   static constexpr int kTmemCols = (2 * T <= 32) ? 32 : (2 * T <= 64) ? 64 : (2 * T <= 128) ? 128 : 256;

@@ -79,9 +79,12 @@ struct RecvLink {
   std::unique_ptr<e3::Link> link;
   uint8_t *buf[kInbox] = {};
   cudaEvent_t appended_ev[kInbox] = {};
-  int64_t appended = 0;   // appends enqueued (messages 0 .. appended-1)
+  // message numbers are the link's (they continue across jobs): this job's
+  // first message is `base`, its inbox slot (no - base) % kInbox
+  int64_t base = 0;
+  int64_t appended = 0;   // appends enqueued (messages base .. appended-1)
   int64_t applied = 0;    // appends whose outcome the host has read
-  int64_t eos_at = -1;    // message index of the end-of-stream message (-1: not yet)
+  int64_t eos_at = -1;    // message number of the end-of-stream message (-1: not yet)
 };
 
 }  // namespace
@@ -298,7 +301,7 @@ struct Runner {
     for (int i = 0; i < nl; ++i) {
       RecvLink &R = pl->in[i];
       while (R.applied < R.appended) {
-        const int slot = (int)(R.applied % kInbox);
+        const int slot = (int)((R.applied - R.base) % kInbox);
         const cudaError_t qe = cudaEventQuery(R.appended_ev[slot]);
         if (qe == cudaErrorNotReady) {
           cudaGetLastError();
@@ -336,7 +339,7 @@ struct Runner {
         e3_status r = R.link->query(R.appended, &done, &rev);
         if (r != E3_OK) return r;
         if (!done) break;
-        const int slot = (int)(R.appended % kInbox);
+        const int slot = (int)((R.appended - R.base) % kInbox);
         E3_CUDA_TRY(cudaStreamWaitEvent(pl->append_stream, rev, 0));
         RingDst dst{};
         dst.rows = Q.rows;
@@ -405,7 +408,24 @@ struct Runner {
     }
     const double idle = std::chrono::duration<double>(std::chrono::steady_clock::now() - last_progress).count();
     if (idle > comm_timeout_s()) {
-      set_error("inter-stage transfer made no progress for E3_COMM_TIMEOUT_S seconds");
+      std::string m = "inter-stage transfer made no progress for E3_COMM_TIMEOUT_S seconds (rank " +
+                      std::to_string(pl->rank) + ", splits [" + std::to_string(pl->s_lo) + "," +
+                      std::to_string(pl->s_hi) + "), pending runs " + std::to_string(pending.size());
+      for (size_t i = 0; i < pl->in.size(); ++i) {
+        const RecvLink &R = pl->in[i];
+        m += "; in[" + std::to_string(i) + "] posted " + std::to_string(R.link->posted) + " appended " +
+             std::to_string(R.appended) + " applied " + std::to_string(R.applied) + " eos " + std::to_string(R.eos_at);
+      }
+      for (size_t i = 0; i < pl->out.size(); ++i) {
+        m += "; out[" + std::to_string(i) + "] posted " + std::to_string(pl->out[i].link->posted) + " in flight";
+        for (int k = 0; k < kOutSlots; ++k) m += " " + std::to_string(pl->out[i].msg_of[k]);
+      }
+      if (pl->s_lo > 0 && pl->s_lo < (int)pl->q.size()) {
+        const DevQueue &Q = pl->q[pl->s_lo];
+        m += "; q[s_lo] known " + std::to_string(Q.known) + " head " + std::to_string(Q.head) + " head_done " +
+             std::to_string(Q.head_done) + " inflight " + std::to_string(Q.inflight) + " cap " + std::to_string(Q.cap);
+      }
+      set_error(m + ")");
       return E3_ENCCL;
     }
     return E3_OK;
@@ -964,7 +984,7 @@ static e3_status pipeline_run_impl(e3_pipeline *pl, void *stream, const void *x,
   for (auto &L : pl->out)
     for (auto &m : L.msg_of) m = -1;
   for (auto &Rl : pl->in) {
-    Rl.appended = Rl.applied = 0;
+    Rl.base = Rl.appended = Rl.applied = Rl.link->posted;
     Rl.eos_at = -1;
   }
   pl->sent_data = 0;

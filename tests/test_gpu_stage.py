@@ -31,8 +31,10 @@ def api():
 
 
 def _run_ranks(api, model, cfg, bounds, tau, placement, inputs, world, deterministic=True, trace=False,
-               dtype="bf16"):
-    """One thread per rank; inputs[rank] = (x, ids) or None.  Returns per-rank
+               dtype="bf16", jobs=1):
+    """One thread per rank; inputs[rank] = (x, ids) or None.  `jobs` runs of
+    the same job back to back on the same pipelines and links (the link's
+    message numbers continue across jobs).  Returns the last job's per-rank
     (exit buffers, stats, trace)."""
     comms = api.Comm.loopback(world, 0)
     N = max(int(ids.max()) + 1 for v in inputs.values() if v is not None for _, ids in [v])
@@ -48,8 +50,10 @@ def _run_ranks(api, model, cfg, bounds, tau, placement, inputs, world, determini
             ex = api.ExitBuffers(N, cfg.classes, cfg.n_ramps, DEV)
             s = torch.cuda.Stream(DEV)
             x, ids = inputs.get(r) or (None, None)
-            st = pipes[r].run(x, ids, ex, stream=s)
-            torch.cuda.synchronize()
+            for _ in range(jobs):
+                ex.reset()
+                st = pipes[r].run(x, ids, ex, stream=s)
+                torch.cuda.synchronize()
             res[r] = (ex, st, pipes[r].trace() if trace else None)
         except Exception as e:  # surfaced in the main thread
             errs.append((r, e))
@@ -147,17 +151,19 @@ def test_replicated_stage_loopback_deterministic(api):
 def test_four_stage_loopback_bert_base(api):
     """EE-BERT-base per-ramp splits grouped into the 4 stages of SURVEY §8(e)
     ({L1-2, L3-4, L5-7, L8-12}), one rank each, 512 inputs: bitwise equal to
-    the single-rank 12-split pipeline; each split flushes at most once."""
+    the single-rank 12-split pipeline; each split flushes at most once.  Three
+    jobs back to back on the same links (a ragged 1000-input job), the last
+    one checked."""
     cfg = e3data.get("bb")
     tau = e3data.tau_for(cfg)
     W = e3data.make_weights(cfg)
     model = api.DeviceModel(cfg, W, DEV)
-    N = 512
+    N = 1000
     X = bf16_tensor(e3data.make_inputs(cfg, range(N)))
     ids = torch.arange(N, dtype=torch.int64, device=DEV)
     bounds = tuple(range(13))
     stage_of = [0, 0, 1, 1, 2, 2, 2, 3, 3, 3, 3, 3]
-    res = _run_ranks(api, model, cfg, bounds, tau, [[g] for g in stage_of], {0: (X, ids)}, 4)
+    res = _run_ranks(api, model, cfg, bounds, tau, [[g] for g in stage_of], {0: (X, ids)}, 4, jobs=3)
     el, lg = _merge(res, N, cfg.classes)
     el1, lg1 = _single(api, model, cfg, bounds, tau, X)
     assert (el >= 0).all()
