@@ -103,13 +103,19 @@ struct e3_pipeline {
   int64_t *tails = nullptr;           // device [2 * n_splits]
   int *overflow = nullptr;            // device flag
   uint8_t *staging = nullptr;         // [B, row] wrapped / flush pops
-  int64_t *staging_ids = nullptr;
+  int64_t *staging_ids = nullptr;     // [2, B]: by run parity (read by the run's tail)
   uint8_t *sink = nullptr;            // [B, row] output of the last split (empty)
   int64_t *out_tails = nullptr;       // device [2]: tail slots of the caller's output buffer
   int64_t *sink_ids = nullptr;
   volatile int *mailbox = nullptr;    // host-mapped [kSlots]
   int *mailbox_dev = nullptr;
-  cudaEvent_t ev[kSlots] = {};
+  cudaEvent_t ev[kSlots] = {};        // run done (recorded on tail_stream)
+  // the last ramp + compaction of a run overlap the next run's layers
+  // (split_run_to's tail stream; higher priority, so its few CTAs are placed
+  // first as the layer kernels' CTAs retire)
+  cudaStream_t tail_stream = nullptr;
+  cudaEvent_t fork[kSlots] = {};
+  cudaEvent_t joined = nullptr;
   // host-input staging
   uint8_t *in_rows = nullptr;         // [kInSlots, B, row]
   int64_t *in_ids = nullptr;
@@ -170,6 +176,10 @@ struct e3_pipeline {
       if (in_free[i]) cudaEventDestroy(in_free[i]);
     }
     if (copy_stream) cudaStreamDestroy(copy_stream);
+    for (auto &e : fork)
+      if (e) cudaEventDestroy(e);
+    if (joined) cudaEventDestroy(joined);
+    if (tail_stream) cudaStreamDestroy(tail_stream);
   }
 };
 
@@ -480,6 +490,12 @@ struct Runner {
     const int64_t *idin;
     int in_slot = -1;
     e3_status r;
+    const int par = (int)(run_no & 1);
+    const int slot = (int)(run_no % kSlots);
+    int64_t *const stg_ids = pl->staging_ids + (size_t)par * B;   // read until the run's tail ends
+    cudaStream_t tst = pl->tail_stream;
+    if (run_no >= 2)   // run_no - 2's tail still reads the parity buffers this run writes
+      E3_CUDA_TRY(cudaStreamWaitEvent(st, pl->ev[(run_no - 2) % kSlots], 0));
     // destination of the survivors first (a send link may have to free a buffer)
     RingDst dst{};
     SendLink *SL = nullptr;
@@ -531,10 +547,10 @@ struct Runner {
           idin = sid;
         } else {
           ProfScope ps(PK_COPY, st, 0, 2.0 * B * rb);
-          r = ring_pop_copy(src, sid, (int64_t)1 << 40, 0, nv, B, rb, pl->staging, pl->staging_ids, pl->sms, st);
+          r = ring_pop_copy(src, sid, (int64_t)1 << 40, 0, nv, B, rb, pl->staging, stg_ids, pl->sms, st);
           if (r != E3_OK) return r;
           xin = pl->staging;
-          idin = pl->staging_ids;
+          idin = stg_ids;
         }
       } else if (nv == B) {
         xin = x + cursor * rb;
@@ -542,10 +558,10 @@ struct Runner {
       } else {
         ProfScope ps(PK_COPY, st, 0, 2.0 * B * rb);
         r = ring_pop_copy(x + cursor * rb, ids + cursor, (int64_t)1 << 40, 0, nv, B, rb, pl->staging,
-                          pl->staging_ids, pl->sms, st);
+                          stg_ids, pl->sms, st);
         if (r != E3_OK) return r;
         xin = pl->staging;
-        idin = pl->staging_ids;
+        idin = stg_ids;
       }
       cursor += nv;
     } else {
@@ -556,23 +572,23 @@ struct Runner {
         idin = Q.ids + pos;
       } else {
         ProfScope ps(PK_COPY, st, 0, 2.0 * B * rb);
-        r = ring_pop_copy(Q.rows, Q.ids, Q.cap, Q.head, nv, B, rb, pl->staging, pl->staging_ids, pl->sms, st);
+        r = ring_pop_copy(Q.rows, Q.ids, Q.cap, Q.head, nv, B, rb, pl->staging, stg_ids, pl->sms, st);
         if (r != E3_OK) return r;
         xin = pl->staging;
-        idin = pl->staging_ids;
+        idin = stg_ids;
       }
       Q.head += nv;
     }
-    const int slot = (int)(run_no % kSlots);
     dst.overflow_dev = pl->overflow;
     dst.mailbox = pl->mailbox_dev ? reinterpret_cast<volatile int *>(pl->mailbox_dev + slot) : nullptr;
     int32_t *n_surv_dev = SL ? reinterpret_cast<int32_t *>(SL->buf[out_slot]) : nullptr;
-    r = split_run_to(pl->splits[s], st, xin, idin, nullptr, nv, dst, n_surv_dev, ex);
+    r = split_run_to(pl->splits[s], st, xin, idin, nullptr, nv, dst, n_surv_dev, ex, tst, par, pl->fork[slot]);
     if (r != E3_OK) return r;
-    if (in_slot >= 0) E3_CUDA_TRY(cudaEventRecord(pl->in_free[in_slot], st));
-    E3_CUDA_TRY(cudaEventRecord(pl->ev[slot], st));
+    // the run ends on the tail stream (its ids are read there)
+    if (in_slot >= 0) E3_CUDA_TRY(cudaEventRecord(pl->in_free[in_slot], tst));
+    E3_CUDA_TRY(cudaEventRecord(pl->ev[slot], tst));
     if (SL) {   // ship the message once the run has written it
-      E3_CUDA_TRY(cudaEventRecord(SL->ready[out_slot], st));
+      E3_CUDA_TRY(cudaEventRecord(SL->ready[out_slot], tst));
       r = SL->link->post(SL->buf[out_slot], (size_t)pl->msg.bytes, SL->ready[out_slot]);
       if (r != E3_OK) return r;
       SL->msg_of[out_slot] = SL->link->posted - 1;
@@ -900,7 +916,7 @@ e3_status e3_pipeline_create(const e3_plan *p, const e3_weights *w, int device, 
   e = cudaMalloc(&pl->overflow, sizeof(int));
   if (e == cudaSuccess) e = cudaMemset(pl->overflow, 0, sizeof(int));
   if (e == cudaSuccess) e = cudaMalloc(&pl->staging, (size_t)pl->B * pl->row_bytes);
-  if (e == cudaSuccess) e = cudaMalloc(&pl->staging_ids, (size_t)pl->B * 8);
+  if (e == cudaSuccess) e = cudaMalloc(&pl->staging_ids, 2 * (size_t)pl->B * 8);
   if (e == cudaSuccess) e = cudaMalloc(&pl->sink, (size_t)pl->B * pl->row_bytes);
   if (e == cudaSuccess) e = cudaMalloc(&pl->out_tails, 2 * sizeof(int64_t));
   if (e == cudaSuccess) e = cudaMalloc(&pl->sink_ids, (size_t)pl->B * 8);
@@ -920,6 +936,12 @@ e3_status e3_pipeline_create(const e3_plan *p, const e3_weights *w, int device, 
     if (e == cudaSuccess) e = cudaEventCreateWithFlags(&pl->in_free[i], cudaEventDisableTiming);
   }
   if (e == cudaSuccess) e = cudaStreamCreateWithFlags(&pl->copy_stream, cudaStreamNonBlocking);
+  int prio_lo = 0, prio_hi = 0;
+  if (e == cudaSuccess) e = cudaDeviceGetStreamPriorityRange(&prio_lo, &prio_hi);
+  if (e == cudaSuccess) e = cudaStreamCreateWithPriority(&pl->tail_stream, cudaStreamNonBlocking, prio_hi);
+  for (int i = 0; i < kSlots && e == cudaSuccess; ++i)
+    e = cudaEventCreateWithFlags(&pl->fork[i], cudaEventDisableTiming);
+  if (e == cudaSuccess) e = cudaEventCreateWithFlags(&pl->joined, cudaEventDisableTiming);
   if (e != cudaSuccess) return fail(e, "e3_pipeline_create");
   *out = pl;
   return E3_OK;
@@ -988,6 +1010,7 @@ static e3_status pipeline_run_impl(e3_pipeline *pl, void *stream, const void *x,
     Rl.eos_at = -1;
   }
   pl->sent_data = 0;
+  E3_CUDA_TRY(cudaStreamWaitEvent(R.st, pl->joined, 0));   // the previous job's tails (any stream)
   E3_CUDA_TRY(cudaMemsetAsync(pl->tails, 0, 2 * sizeof(int64_t) * pl->plan.n_splits, R.st));
   E3_CUDA_TRY(cudaStreamSynchronize(R.st));   // tails reset before any append-stream work
   if (R.host_in) {
@@ -995,6 +1018,14 @@ static e3_status pipeline_run_impl(e3_pipeline *pl, void *stream, const void *x,
     for (int i = 0; i < kInSlots; ++i) E3_CUDA_TRY(cudaEventRecord(pl->in_free[i], R.st));
   }
   e3_status r = R.run();
+  {   // join: the caller's stream waits for the last tails
+    const cudaError_t je = cudaEventRecord(pl->joined, pl->tail_stream);
+    if (je == cudaSuccess) cudaStreamWaitEvent(R.st, pl->joined, 0);
+    if (je != cudaSuccess && r == E3_OK) {
+      set_error("join of the tail stream failed");
+      r = E3_ECUDA;
+    }
+  }
   if (r == E3_OK) {
     int ovf = 0, derr = 0;
     E3_CUDA_TRY(cudaMemcpyAsync(&ovf, pl->overflow, sizeof(int), cudaMemcpyDeviceToHost, R.st));

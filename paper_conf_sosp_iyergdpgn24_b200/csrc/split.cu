@@ -44,7 +44,7 @@ Workspace::~Workspace() {
   int prev = 0;
   cudaGetDevice(&prev);
   cudaSetDevice(device);
-  void *bufs[] = {qkv, ctx, y, x1, h, xa, xb, pool, alive, ctr, err, lm_stats, dec_part, dec_tickets, rope};
+  void *bufs[] = {qkv, ctx, y, x1, h, xa, xb, yt, alive_t, pool, alive, ctr, err, lm_stats, dec_part, dec_tickets, rope};
   for (void *p : bufs)
     if (p) cudaFree(p);
   cudaSetDevice(prev);
@@ -101,6 +101,11 @@ e3_status Workspace::create(int device, int B, int S, int H, int F, int elem, st
   E3_CUDA_TRY(cudaMalloc(&ws->xb, M * H * e));
   E3_CUDA_TRY(cudaMalloc(&ws->pool, (size_t)B * H * 4));
   E3_CUDA_TRY(cudaMalloc(&ws->alive, (size_t)B));
+  if (elem == 2) {   // parity-1 tail buffers (bf16 encoder runs only)
+    E3_CUDA_TRY(cudaMalloc(&ws->yt, M * H * e));
+    E3_CUDA_TRY(cudaMalloc(&ws->alive_t, (size_t)B));
+    E3_CUDA_TRY(cudaMemset(ws->alive_t, 0, (size_t)B));
+  }
   E3_CUDA_TRY(cudaMalloc(&ws->ctr, kCtrWords * sizeof(unsigned)));
   E3_CUDA_TRY(cudaMemset(ws->ctr, 0, kCtrWords * sizeof(unsigned)));
   E3_CUDA_TRY(cudaMemset(ws->alive, 0, (size_t)B));
@@ -346,6 +351,7 @@ e3_status split_create_shared(const e3_split_desc *d, const e3_weights *w, int d
                          vit ? ws->y : nullptr, ws->x1, M, H, H);
     if (st == E3_OK) st = gemm_tmaps(&m.f1, ws->x1, H, s->L[i].w_1, ws->h, M, F, H, s->bn_f1);
     if (st == E3_OK) st = gemm_tmaps(&m.f2, ws->h, F, s->L[i].w_2, vit ? out : ws->y, M, H, F, s->bn_f2);
+    if (st == E3_OK && i == nl - 1) st = gemm_tmaps(&m.f2t, ws->h, F, s->L[i].w_2, ws->yt, M, H, F, s->bn_f2);
   }
   if (st == E3_OK) st = attn_tmaps(&s->attn, ws->qkv, ws->ctx, B, S, H);
   if (st != E3_OK) {
@@ -716,12 +722,42 @@ static LnGemmArgs oln_args(const void *bias, const void *R, const void *g, const
   return a;
 }
 
+bool split_tail_overlap(const e3_split *s) {
+  static const bool off = getenv("E3_NO_TAIL_OVERLAP") != nullptr;
+  const e3_split_desc &d = s->d;
+  return !off && d.dtype == E3_DTYPE_BF16 && d.arch != E3_ARCH_LLAMA_DECODE && d.n_ramps >= 1 &&
+         (d.n_ramps == 1 || d.inner == E3_INNER_DISABLED) && d.ramp_layer[d.n_ramps - 1] == d.layer_end - 1;
+}
+
+static e3_status split_run_body(e3_split *s, cudaStream_t st, const void *x_in, const int64_t *id_in,
+                                const int32_t *n_valid_dev, int n_valid_host, const RingDst &dst,
+                                int32_t *n_surv_dev, const e3_exits *ex, cudaStream_t tail_st, int par,
+                                cudaEvent_t fork);
+
 e3_status split_run_to(e3_split *s, cudaStream_t st, const void *x_in, const int64_t *id_in,
                        const int32_t *n_valid_dev, int n_valid_host, const RingDst &dst, int32_t *n_surv_dev,
-                       const e3_exits *ex) {
-  if (s->d.dtype == E3_DTYPE_FP32) return f32_run(s, st, x_in, id_in, n_valid_dev, n_valid_host, dst, n_surv_dev, ex);
-  if (s->d.arch == E3_ARCH_LLAMA_DECODE)
-    return llama_run(s, st, x_in, id_in, n_valid_dev, n_valid_host, dst, n_surv_dev, ex);
+                       const e3_exits *ex, cudaStream_t tail_st, int par, cudaEvent_t fork) {
+  const bool ovl = tail_st && tail_st != st && fork && split_tail_overlap(s);
+  e3_status r;
+  if (s->d.dtype == E3_DTYPE_FP32)
+    r = f32_run(s, st, x_in, id_in, n_valid_dev, n_valid_host, dst, n_surv_dev, ex);
+  else if (s->d.arch == E3_ARCH_LLAMA_DECODE)
+    r = llama_run(s, st, x_in, id_in, n_valid_dev, n_valid_host, dst, n_surv_dev, ex);
+  else
+    r = split_run_body(s, st, x_in, id_in, n_valid_dev, n_valid_host, dst, n_surv_dev, ex, ovl ? tail_st : st,
+                       ovl ? (par & 1) : 0, fork);
+  if (r == E3_OK && !ovl && tail_st && tail_st != st) {   // the run ends on tail_st all the same
+    E3_CHECK_ARG(fork, "split_run_to: tail stream without a fork event");
+    E3_CUDA_TRY(cudaEventRecord(fork, st));
+    E3_CUDA_TRY(cudaStreamWaitEvent(tail_st, fork, 0));
+  }
+  return r;
+}
+
+static e3_status split_run_body(e3_split *s, cudaStream_t st, const void *x_in, const int64_t *id_in,
+                                const int32_t *n_valid_dev, int n_valid_host, const RingDst &dst,
+                                int32_t *n_surv_dev, const e3_exits *ex, cudaStream_t tst, int par,
+                                cudaEvent_t fork) {
   const e3_split_desc &d = s->d;
   Workspace &ws = *s->ws;
   const int B = d.batch, S = d.seq_len, H = d.hidden, F = d.ffn, M = B * S;
@@ -743,6 +779,10 @@ e3_status split_run_to(e3_split *s, cudaStream_t st, const void *x_in, const int
   const double f_att = 4.0 * n_valid_host * (double)S * S * H, b_ln = 2.0 * nvS * H * 2;
   const bool vit = d.arch == E3_ARCH_VIT;
   bool compacted = false;   // the last ramp's fused kernel also compacted the survivors
+  // tst != st: the last ramp and the compaction run on tst (split_run_to)
+  const bool ovl = tst != st;
+  void *const y_last = par ? ws.yt : ws.y;        // BERT: the last layer's pre-LN2 output
+  uint8_t *const alive = par ? ws.alive_t : ws.alive;
   for (int i = 0; i < nl; ++i) {
     const int l = d.layer_begin + i;
     const e3_layer_weights &L = s->L[i];
@@ -783,9 +823,9 @@ e3_status split_run_to(e3_split *s, cudaStream_t st, const void *x_in, const int
       }
       {
         ProfScope ps(PK_GEMM_FFN2, st, f_1, 0);
-        E3_RUN(gemm_run(m.f2, L.b_2, ws.y, M, H, F, E3_EPI_BIAS_RESID, s->sms, st));
+        E3_RUN(gemm_run(last_layer && par ? m.f2t : m.f2, L.b_2, ws.y, M, H, F, E3_EPI_BIAS_RESID, s->sms, st));
       }
-      cur = out;
+      cur = last_layer && par ? ws.yt : out;
     } else {
     {
       ProfScope ps(PK_GEMM_QKV, st, f_qkv, 0);
@@ -820,7 +860,8 @@ e3_status split_run_to(e3_split *s, cudaStream_t st, const void *x_in, const int
     }
     {
       ProfScope ps(PK_GEMM_FFN2, st, f_1, 0);
-      if (!skip(PK_GEMM_FFN2)) E3_RUN(gemm_run(m.f2, L.b_2, ws.x1, M, H, F, E3_EPI_BIAS_RESID, s->sms, st));
+      if (!skip(PK_GEMM_FFN2))
+        E3_RUN(gemm_run(last_layer && par ? m.f2t : m.f2, L.b_2, ws.x1, M, H, F, E3_EPI_BIAS_RESID, s->sms, st));
     }
     // The split's last layer never materialises LN2: its ramp normalises the
     // CLS rows itself and the fused LN2 + compaction normalises only the
@@ -831,13 +872,18 @@ e3_status split_run_to(e3_split *s, cudaStream_t st, const void *x_in, const int
       cur = out;
     }
     }
+    if (ovl && last_layer) {   // fork: the tail waits for the last layer only
+      E3_CUDA_TRY(cudaEventRecord(fork, st));
+      E3_CUDA_TRY(cudaStreamWaitEvent(tst, fork, 0));
+    }
     while (ri < d.n_ramps && d.ramp_layer[ri] == l) {
       const bool last = (ri == d.n_ramps - 1);
+      cudaStream_t rst = last ? tst : st;
       if (last || d.inner == E3_INNER_EXACT) {
         RampArgs a{};
         a.arch = d.arch;
         const bool pre_ln_rows = last_layer && !vit;   // BERT: the ramp applies LN2 itself
-        a.x = pre_ln_rows ? ws.y : cur;
+        a.x = pre_ln_rows ? y_last : cur;
         a.ln_g = pre_ln_rows ? L.ln2_g : nullptr;
         a.ln_b = pre_ln_rows ? L.ln2_b : nullptr;
         a.id = id_in;
@@ -852,7 +898,7 @@ e3_status split_run_to(e3_split *s, cudaStream_t st, const void *x_in, const int
         a.layer = l;
         a.ramp_index = d.ramp_index[ri];
         a.eps = d.norm_eps;
-        a.alive = ws.alive;
+        a.alive = alive;
         a.init_alive = first_ramp;
         a.n_valid_dev = n_valid_dev;
         a.n_valid_host = n_valid_host;
@@ -862,15 +908,15 @@ e3_status split_run_to(e3_split *s, cudaStream_t st, const void *x_in, const int
         {
           // pooler weights + CLS rows + classifier weights (bytes); 2H^2 + 2HC per row (flops)
           const double hh = vit ? 0.0 : 2.0 * H * H;
-          ProfScope ps(PK_RAMP, st, (double)n_valid_host * (hh + 2.0 * H * d.num_labels),
+          ProfScope ps(PK_RAMP, rst, (double)n_valid_host * (hh + 2.0 * H * d.num_labels),
                        hh + 2.0 * n_valid_host * H + 2.0 * d.num_labels * H);
           if (last && pre_ln_rows && !skip(PK_RAMP)) {
             // the split's last ramp and the LN2 + compaction of its survivors in one launch
             bool fused = false;
-            E3_RUN(ramp_compact_run(a, ws.ctr, dst, n_surv_dev, s->sms, st, &fused));
+            E3_RUN(ramp_compact_run(a, ws.ctr, dst, n_surv_dev, s->sms, rst, &fused));
             compacted = fused;
           }
-          if (!compacted && !skip(PK_RAMP)) E3_RUN(ramp_run(a, st));
+          if (!compacted && !skip(PK_RAMP)) E3_RUN(ramp_run(a, rst));
         }
         first_ramp = false;
       }
@@ -881,14 +927,14 @@ e3_status split_run_to(e3_split *s, cudaStream_t st, const void *x_in, const int
     // survivors: LN2 of the last layer fused with the stable compaction
     // (bytes added once n_surv is known, in the pipeline)
     const e3_layer_weights &L = s->L[nl - 1];
-    ProfScope ps(PK_COMPACT, st, 0, 0);
+    ProfScope ps(PK_COMPACT, tst, 0, 0);
     if (skip(PK_COMPACT)) return E3_OK;
     if (vit)   // pre-LN: the layer output is final, survivors are copied
-      E3_RUN(ln_compact_run(cur, id_in, ws.alive, B, S, H, nullptr, nullptr, d.norm_eps, dst, n_surv_dev, s->sms,
-                            st));
+      E3_RUN(ln_compact_run(cur, id_in, alive, B, S, H, nullptr, nullptr, d.norm_eps, dst, n_surv_dev, s->sms,
+                            tst));
     else
-      E3_RUN(ln_compact_run(ws.y, id_in, ws.alive, B, S, H, L.ln2_g, L.ln2_b, d.norm_eps, dst, n_surv_dev, s->sms,
-                            st));
+      E3_RUN(ln_compact_run(y_last, id_in, alive, B, S, H, L.ln2_g, L.ln2_b, d.norm_eps, dst, n_surv_dev, s->sms,
+                            tst));
   }
 #undef E3_RUN
   return E3_OK;

@@ -19,6 +19,11 @@ struct Workspace {
   int B = 0, S = 0, H = 0, F = 0;
   int elem = 2;                   // bytes per activation element: 2 (BF16) or 4 (FP32)
   void *qkv = nullptr, *ctx = nullptr, *y = nullptr, *x1 = nullptr, *h = nullptr, *xa = nullptr, *xb = nullptr;
+  // the split's last layer output and alive flags of runs with parity 1 (the
+  // last ramp + compaction of run j overlaps run j+1 on a second stream:
+  // split_run_to's tail_st)
+  void *yt = nullptr;
+  uint8_t *alive_t = nullptr;
   float *pool = nullptr;
   uint8_t *alive = nullptr;
   unsigned *ctr = nullptr;        // [kCtrWords]: compaction ticket, ramp row-group tickets
@@ -49,6 +54,7 @@ struct e3_split {
   std::shared_ptr<e3::Workspace> ws;
   struct LayerMaps {
     e3::GemmMaps qkv, o, f1, f2;
+    e3::GemmMaps f2t;     // last layer: FFN2 writing Workspace::yt (runs with parity 1)
     e3::LnGemmMaps oln;   // fused O projection + residual + LayerNorm (when use_oln)
   };
   bool use_oln = false;
@@ -72,9 +78,17 @@ e3_status split_validate(const e3_split_desc *d, const e3_weights *w);
 e3_status split_create_shared(const e3_split_desc *d, const e3_weights *w, int device,
                               std::shared_ptr<Workspace> ws, e3_split **out);
 // Runs the split; survivors go to `dst` (contiguous or a queue ring).
+// tail_st (optional): the stream the run ENDS on.  Where the split allows it
+// (bf16 encoder, one active ramp: split_tail_overlap) the last ramp and the
+// compaction run there, forked from `st` by `fork` after the last layer, and
+// read the parity-`par` copies of the last layer output and alive flags, so
+// they overlap the next run's layers on `st`; otherwise `tail_st` just waits
+// for `st`.  The caller orders run j's start on `st` after run j-2's tail
+// (the parity buffers are reused) and reads dst / id_in until the tail ends.
 e3_status split_run_to(e3_split *s, cudaStream_t st, const void *x_in, const int64_t *id_in,
                        const int32_t *n_valid_dev, int n_valid_host, const RingDst &dst, int32_t *n_surv_dev,
-                       const e3_exits *ex);
+                       const e3_exits *ex, cudaStream_t tail_st = nullptr, int par = 0, cudaEvent_t fork = nullptr);
+bool split_tail_overlap(const e3_split *s);
 // multi-step decode: K/V of layer l (in this split) for the chunk's tokens exited before l
 e3_status llama_fill_layer(e3_split *s, int l, cudaStream_t st, const int64_t *ids_in, int nv, const e3_exits &ex,
                            int64_t *ids_buf);

@@ -33,7 +33,6 @@ sys.path.insert(0, ROOT)
 
 import e3data  # noqa: E402
 from paper_conf_sosp_iyergdpgn24_b200 import api, online, planner  # noqa: E402
-from oracle.pipeline_sim import Plan  # noqa: E402
 
 
 def main():
@@ -50,7 +49,7 @@ def main():
     cfg = e3data.get("bb")
     tau = e3data.tau_for(cfg)
     model = api.DeviceModel(cfg, e3data.make_weights(cfg), dev)
-    pipe = api.Pipeline(model, api.make_plan(cfg, Plan.per_ramp(cfg.ramp_layers).bounds, tau))
+    pipe = api.Pipeline(model, api.make_plan(cfg, (0,) + tuple(l + 1 for l in cfg.ramp_layers), tau))
     # pools: calibration-seed inputs classified by where they exit
     Xp = api.to_bf16(e3data.make_inputs(cfg, range(args.pool), seed=2), dev)
     exp = api.ExitBuffers(args.pool, cfg.classes, cfg.n_ramps, dev, logits=False)

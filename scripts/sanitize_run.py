@@ -26,8 +26,7 @@ def enc(name, dtype, n=96):
     X = torch.from_numpy(e3data.make_inputs(cfg, range(n))).to(DEV)
     X = X.to(torch.bfloat16) if dtype == "bf16" else X
     ex = api.ExitBuffers(n, cfg.classes, cfg.n_ramps, DEV)
-    from oracle.pipeline_sim import Plan
-    api.Pipeline(model, api.make_plan(cfg, Plan.per_ramp(cfg.ramp_layers).bounds, cfg.tau, dtype=dtype)).run(
+    api.Pipeline(model, api.make_plan(cfg, (0,) + tuple(l + 1 for l in cfg.ramp_layers), cfg.tau, dtype=dtype)).run(
         X, torch.arange(n, dtype=torch.int64, device=DEV), ex)
     torch.cuda.synchronize()
     assert int(ex.n_exit.item()) == n

@@ -1,7 +1,7 @@
 """Whole-job parity helpers (GPU pipeline from seeded inputs vs the oracle).
 
 Shared by the -m gpu tests (tests/test_gpu_e2e.py) and the measurement
-script scripts/parity_stats.py that writes profiles/r02_parity_*.json.
+script tests/tools/parity_stats.py that writes profiles/r02_parity_*.json.
 Nothing here computes the method: the GPU side goes through the C ABI
 (paper_conf_sosp_iyergdpgn24_b200.api), the expected side through oracle/.
 """

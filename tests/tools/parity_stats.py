@@ -1,7 +1,7 @@
 """Whole-job parity measurement: the GPU pipeline from seeded inputs vs the
 oracle, every input compared (VERDICT r01 "what to do" 1(b)).
 
-    python scripts/parity_stats.py [--dtype bf16|fp32] [--configs t,tv,bb,bl,vt,tl,lm] [--out FILE]
+    python tests/tools/parity_stats.py [--dtype bf16|fp32] [--configs t,tv,bb,bl,vt,tl,lm] [--out FILE]
 
 Per config: the per-ramp plan through e3_pipeline_run on N inputs (tiny 256,
 tiny-vit 200, BB 128, BL 32, VT 32, tiny-llama 90, Llama-7B shape 16 tokens
@@ -17,7 +17,7 @@ import time
 
 import numpy as np
 
-ROOT = os.path.dirname(os.path.dirname(os.path.abspath(__file__)))
+ROOT = os.path.dirname(os.path.dirname(os.path.dirname(os.path.abspath(__file__))))
 sys.path.insert(0, ROOT)
 
 import e3data  # noqa: E402
