@@ -99,7 +99,9 @@ __global__ void __launch_bounds__(AThr<SKV>::kThreads, 2)
   constexpr int NCH = SKV / 32;     // 32-key chunks; key part p takes chunks [p NCHP, (p + 1) NCHP)
   constexpr int NCHP = (NCH + KP - 1) / KP;
   extern __shared__ uint8_t smem_raw[];
-  uint8_t *smem = reinterpret_cast<uint8_t *>((reinterpret_cast<uintptr_t>(smem_raw) + 1023) & ~uintptr_t(1023));
+  // 1024-B aligned by offset arithmetic on the __shared__ array, so the
+  // compiler keeps the shared address space (LDS / STS, not generic LD / ST)
+  uint8_t *smem = smem_raw + ((1024u - (smem_u32(smem_raw) & 1023u)) & 1023u);
   uint8_t *pbuf_sep = smem + CF::kNBuf * CF::kBuf;      // only when !kPInQK
   float *xch = reinterpret_cast<float *>(smem + CF::kNBuf * CF::kBuf + (CF::kPInQK ? 0 : CF::kP));  // [2][2][KP][QT]
   uint64_t *bars = reinterpret_cast<uint64_t *>(xch + 2 * 2 * KP * QT);

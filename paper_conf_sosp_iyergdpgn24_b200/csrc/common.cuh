@@ -377,7 +377,7 @@ __device__ __forceinline__ int lane_id() { return threadIdx.x & 31; }
 
 // ---- diagnostics: kernel timeline (e3_debug_timeline).  When a device buffer
 // is set (per translation unit: tl_set_<file>), thread 0 of every CTA of the
-// instrumented kernels appends {kernel id | blockIdx.x << 16, entry, released
+// instrumented kernels appends {kernel id | blockIdx.x << 16 | smid << 48, entry, released
 // (after griddepcontrol.wait), end} globaltimer stamps; buf[0] is the count.
 namespace {
 __device__ unsigned long long *g_tl = nullptr;
@@ -395,7 +395,9 @@ __device__ __forceinline__ void tl_rec(unsigned long long *b, int kid, unsigned 
   const unsigned long long t2 = tl_now();
   const unsigned long long i = atomicAdd(b, 1ull);
   if (i >= (unsigned long long)kTlCap) return;
-  b[1 + 4 * i] = (unsigned long long)kid | ((unsigned long long)blockIdx.x << 16);
+  unsigned smid;
+  asm volatile("mov.u32 %0, %%smid;" : "=r"(smid));
+  b[1 + 4 * i] = (unsigned long long)kid | ((unsigned long long)blockIdx.x << 16) | ((unsigned long long)smid << 48);
   b[2 + 4 * i] = t0;
   b[3 + 4 * i] = t1;
   b[4 + 4 * i] = t2;

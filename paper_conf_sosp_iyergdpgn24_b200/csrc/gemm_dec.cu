@@ -106,7 +106,9 @@ __global__ void __launch_bounds__(kDThreads, 1)
   const unsigned long long tl0 = tl_now();
   unsigned long long *const tlb = g_tl;
   extern __shared__ uint8_t smem_raw[];
-  uint8_t *smem = reinterpret_cast<uint8_t *>((reinterpret_cast<uintptr_t>(smem_raw) + 1023) & ~uintptr_t(1023));
+  // 1024-B aligned by offset arithmetic on the __shared__ array, so the
+  // compiler keeps the shared address space (LDS / STS, not generic LD / ST)
+  uint8_t *smem = smem_raw + ((1024u - (smem_u32(smem_raw) & 1023u)) & 1023u);
   constexpr int XS = CF::kXStages;
   uint8_t *sW = smem;
   uint8_t *sX = smem + S * CF::kWBytes;
@@ -311,6 +313,49 @@ __global__ void __launch_bounds__(kDThreads, 1)
       const long seg_end = min(my1, t1i);
       const bool whole = (i == t0i) && (seg_end == t1i);
       i = seg_end;
+      // Early fetch (T <= 64, two contributors): while this segment's MMAs
+      // still run, look whether the tile's other contributor already
+      // published its partial (the usual case for a CTA's last segment: the
+      // head of a tile whose tail the next CTA computed first).  If so this
+      // CTA is the tile's last arrival; the other partial is loaded into
+      // registers now, so the reduction after the accumulator lands costs no
+      // memory round trip on the kernel's critical path.
+      bool early = false;
+      int early_slot = 0;
+      if (T <= 64 && !whole) {
+        const int c_first = sk.owner(t0i), c_last = sk.owner(t1i - 1);
+        if (c_last - c_first == 1) {
+          const int slot = (int)blockIdx.x - c_first;
+          if (et == 0) {
+            const unsigned seen = *reinterpret_cast<volatile unsigned *>(&a.tickets[tile]);
+            *s_last = (seen == 1u) ? 3 : 0;
+            if (seen == 1u) a.tickets[tile] = 0;   // both contributors accounted for: ready for the next launch
+          }
+          epi_bar();
+          early = *s_last == 3;
+          early_slot = slot;
+          if (early) {
+            // the other partial goes to sE (free: the previous segment's
+            // epilogue has finished with it); the accumulator is added below
+            __threadfence();
+            const float4 *op = reinterpret_cast<const float4 *>(a.part) +
+                               ((size_t)tile * a.max_contrib + (1 - slot)) * (T / 4) * DM + r;
+#pragma unroll 1
+            for (int k0 = 0; k0 < T / 4; k0 += 8) {   // 8 vectors in flight (registers)
+              float4 pv[8];
+#pragma unroll
+              for (int k = 0; k < 8; ++k) pv[k] = __ldcg(op + (size_t)(k0 + k) * DM);
+#pragma unroll
+              for (int k = 0; k < 8; ++k) {
+                sE[r * P + 4 * (k0 + k)] = pv[k].x;
+                sE[r * P + 4 * (k0 + k) + 1] = pv[k].y;
+                sE[r * P + 4 * (k0 + k) + 2] = pv[k].z;
+                sE[r * P + 4 * (k0 + k) + 3] = pv[k].w;
+              }
+            }
+          }
+        }
+      }
       mbar_wait(&tfull[acc], acc_phase);
       tc_fence_after();
       tlm = tl_now();
@@ -321,8 +366,16 @@ __global__ void __launch_bounds__(kDThreads, 1)
         uint32_t v[32];
         tmem_ld32(taddr + c * 32, v);
         tmem_wait_ld();
+        if (early) {   // contributor order: acc = (0 + p0) + p1, as the reduction below
 #pragma unroll
-        for (int j = 0; j < 32; ++j) sE[r * P + c * 32 + j] = __uint_as_float(v[j]);
+          for (int j = 0; j < 32; ++j) {
+            const float own = __uint_as_float(v[j]), oth = sE[r * P + c * 32 + j];
+            sE[r * P + c * 32 + j] = early_slot == 0 ? (0.f + own) + oth : (0.f + oth) + own;
+          }
+        } else {
+#pragma unroll
+          for (int j = 0; j < 32; ++j) sE[r * P + c * 32 + j] = __uint_as_float(v[j]);
+        }
       }
       tc_fence_before();
       __syncwarp();
@@ -331,7 +384,10 @@ __global__ void __launch_bounds__(kDThreads, 1)
       epi_bar();
       if (CSK > 1) break;               // one segment; reduced across the cluster below
 
-      if (!whole) {
+      unsigned long long tl_tk = 0, tl_rd = 0;
+      if (early) {
+        tl_rd = tl_now();   // reduced while the accumulator was read (each thread its own row)
+      } else if (!whole) {
         // shared tile: publish this contributor's partial; the tile's last
         // arrival sums the contributors' partials in contributor order
         const int c_first = sk.owner(t0i), c_last = sk.owner(t1i - 1);
@@ -340,19 +396,37 @@ __global__ void __launch_bounds__(kDThreads, 1)
         // thread moves its row's T values as 16-byte vectors and a warp's
         // access is 512 contiguous bytes
         float4 *part = reinterpret_cast<float4 *>(a.part) + ((size_t)tile * a.max_contrib + slot) * (T / 4) * DM + r;
-#pragma unroll
-        for (int i = 0; i < T / 4; ++i)
-          part[(size_t)i * DM] =
-              make_float4(sE[r * P + 4 * i], sE[r * P + 4 * i + 1], sE[r * P + 4 * i + 2], sE[r * P + 4 * i + 3]);
-        __threadfence();
-        epi_bar();
+        // every other contributor already arrived (the usual case for a
+        // CTA's last segment, the head of a tile whose tail the next CTA
+        // computed first): this CTA is the last, its partial stays in sE and
+        // is summed in its contributor position below -- no write, fence and
+        // ticket round trips on the kernel's critical path
         if (et == 0) {
-          const unsigned prev = atomicAdd(&a.tickets[tile], 1u);
-          *s_last = (prev == (unsigned)(ncon - 1));
-          if (*s_last) a.tickets[tile] = 0;   // ready for the next launch
+          const unsigned seen = *reinterpret_cast<volatile unsigned *>(&a.tickets[tile]);
+          *s_last = (seen == (unsigned)(ncon - 1)) ? 2 : 0;
+          if (*s_last) a.tickets[tile] = 0;   // every contributor arrived: ready for the next launch
         }
         epi_bar();
-        if (!*s_last) continue;
+        const bool own_in_smem = *s_last == 2;
+        if (!own_in_smem) {
+#pragma unroll
+          for (int i = 0; i < T / 4; ++i)
+            part[(size_t)i * DM] =
+                make_float4(sE[r * P + 4 * i], sE[r * P + 4 * i + 1], sE[r * P + 4 * i + 2], sE[r * P + 4 * i + 3]);
+          __threadfence();
+          epi_bar();
+          if (et == 0) {
+            const unsigned prev = atomicAdd(&a.tickets[tile], 1u);
+            *s_last = (prev == (unsigned)(ncon - 1));
+            if (*s_last) a.tickets[tile] = 0;   // ready for the next launch
+          }
+          epi_bar();
+        }
+        tl_tk = tl_now();
+        if (!*s_last) {
+          if (threadIdx.x == 64) tl_rec(tlb, 8300 + EPI, tlm, tl_tk);   // segment: acc ready, ticket, (no reduction)
+          continue;
+        }
         const unsigned long long tlr0 = tl_now();
         __threadfence();
         // sum the contributors' partials in contributor order; contributor
@@ -361,20 +435,28 @@ __global__ void __launch_bounds__(kDThreads, 1)
         const float4 *base = reinterpret_cast<const float4 *>(a.part) + (size_t)tile * a.max_contrib * (T / 4) * DM + r;
         const size_t cstride = (size_t)DM * T / 4;   // float4s between contributors
 #pragma unroll 1
-        for (int h = 0; h < T / 64 + (T % 64 ? 1 : 0); ++h) {
-          constexpr int NV = (T < 64 ? T : 64) / 4;
+        for (int h = 0; h < T / 32 + (T % 32 ? 1 : 0); ++h) {   // 32 tokens per pass (registers)
+          constexpr int NV = (T < 32 ? T : 32) / 4;
           float4 acc4[NV], cur[NV], nxt[NV];
+          // contributor j's values: its partial in global memory, or this
+          // CTA's own accumulator in sE when it skipped publishing it
+          auto fetch = [&](int j, float4 *dst) {
 #pragma unroll
-          for (int i = 0; i < NV; ++i) {
-            acc4[i] = make_float4(0.f, 0.f, 0.f, 0.f);
-            cur[i] = __ldcg(base + (size_t)(h * NV + i) * DM);
-          }
+            for (int i = 0; i < NV; ++i) {
+              if (own_in_smem && j == slot) {
+                const int t = h * 32 + 4 * i;
+                dst[i] = make_float4(sE[r * P + t], sE[r * P + t + 1], sE[r * P + t + 2], sE[r * P + t + 3]);
+              } else {
+                dst[i] = __ldcg(base + j * cstride + (size_t)(h * NV + i) * DM);
+              }
+            }
+          };
+#pragma unroll
+          for (int i = 0; i < NV; ++i) acc4[i] = make_float4(0.f, 0.f, 0.f, 0.f);
+          fetch(0, cur);
 #pragma unroll 1
           for (int j = 0; j < ncon; ++j) {
-            if (j + 1 < ncon) {
-#pragma unroll
-              for (int i = 0; i < NV; ++i) nxt[i] = __ldcg(base + (j + 1) * cstride + (size_t)(h * NV + i) * DM);
-            }
+            if (j + 1 < ncon) fetch(j + 1, nxt);
 #pragma unroll
             for (int i = 0; i < NV; ++i) {
               acc4[i].x += cur[i].x;
@@ -386,7 +468,7 @@ __global__ void __launch_bounds__(kDThreads, 1)
           }
 #pragma unroll
           for (int i = 0; i < NV; ++i) {
-            const int t = h * 64 + 4 * i;
+            const int t = h * 32 + 4 * i;
             sE[r * P + t] = acc4[i].x;
             sE[r * P + t + 1] = acc4[i].y;
             sE[r * P + t + 2] = acc4[i].z;
@@ -395,6 +477,7 @@ __global__ void __launch_bounds__(kDThreads, 1)
         }
         epi_bar();
         if (threadIdx.x == 64) tl_rec(tlb, 8200 + EPI, tlr0, tlr0);   // reduction: start, end
+        tl_rd = tl_now();
       }
 
       // ---------------------------------------------------- final epilogue
@@ -446,7 +529,10 @@ __global__ void __launch_bounds__(kDThreads, 1)
 #pragma unroll
           for (int j = 0; j < 8; ++j) {
             const float gv = sE[(8 * g + j) * P + t], up = sE[(64 + 8 * g + j) * P + t];
-            o[j] = gv / (1.0f + expf(-gv)) * up;
+            // SiLU(g) * u (bf16 output); __fdividef has no slow path when
+            // e^-g overflows (IEEE division / __frcp_rn took ~5 us per tile
+            // on |g| > 88)
+            o[j] = gv * __fdividef(1.0f, 1.0f + __expf(-gv)) * up;
           }
           *reinterpret_cast<uint4 *>(a.Y + (size_t)t * a.ldo + f) =
               make_uint4(pack_bf16(o[0], o[1]), pack_bf16(o[2], o[3]), pack_bf16(o[4], o[5]), pack_bf16(o[6], o[7]));
@@ -588,6 +674,7 @@ __global__ void __launch_bounds__(kDThreads, 1)
         }
       }
       epi_bar();                        // sE is reused by the next unit
+      if (threadIdx.x == 64) tl_rec(tlb, tl_rd ? 8400 + EPI : 8500 + EPI, tlm, tl_rd ? tl_rd : tlm);   // segment: acc ready, reduced, end
     }
     if (threadIdx.x == 64) {
       tl_rec(tlb, 8100 + EPI, tl0, tl1);
@@ -598,19 +685,42 @@ __global__ void __launch_bounds__(kDThreads, 1)
     constexpr int RPC = DM / CSK;       // rows reduced and stored by this CTA
     const int cr = (int)cluster_ctarank();
     const int tile = blockIdx.x / CSK;
+    const unsigned long long tc0 = tl_now();
     cluster_sync();                     // every CTA's partial tile is in its smem
+    const unsigned long long tc1 = tl_now();
     if (warp >= 2 && warp <= 5) {
+      // every remote value of a batch of elements is loaded before the first
+      // add (one load -> add chain per element and rank serialised ~48 DSMEM
+      // round trips per thread: ~5 us after the mainloop, r02 llama_timeline)
       const int et = threadIdx.x - 64;
-      for (int e = et; e < RPC * T; e += 128) {
-        const int row = cr * RPC + e / T, t = e % T;
-        const uint32_t off = smem_u32(&sE[row * P + t]);
-        float acc = 0.f;
+      constexpr int EB = 8;             // elements per batch
+      static_assert((RPC * T) % (128 * EB) == 0, "CSK reduction batches");
+#pragma unroll 1
+      for (int e0 = et; e0 < RPC * T; e0 += 128 * EB) {
+        float v[EB][CSK];
 #pragma unroll
-        for (int q = 0; q < CSK; ++q) acc += (q == cr) ? sE[row * P + t] : ld_dsmem_f32(mapa_shared(off, (uint32_t)q));
-        sE[row * P + t] = acc;          // only this CTA reads its own rows from here on
+        for (int u = 0; u < EB; ++u) {
+          const int e = e0 + 128 * u;
+          const int row = cr * RPC + e / T, t = e % T;
+          const uint32_t off = smem_u32(&sE[row * P + t]);
+#pragma unroll
+          for (int q = 0; q < CSK; ++q) v[u][q] = (q == cr) ? sE[row * P + t] : ld_dsmem_f32(mapa_shared(off, (uint32_t)q));
+        }
+#pragma unroll
+        for (int u = 0; u < EB; ++u) {
+          const int e = e0 + 128 * u;
+          const int row = cr * RPC + e / T, t = e % T;
+          float acc = 0.f;
+#pragma unroll
+          for (int q = 0; q < CSK; ++q) acc += v[u][q];   // rank order
+          sE[row * P + t] = acc;        // only this CTA reads its own rows from here on
+        }
       }
     }
+    const unsigned long long tc2 = tl_now();
     cluster_sync();                     // no CTA leaves while a peer may still read its smem
+    if (threadIdx.x == 64) tl_rec(tlb, 8800 + EPI, tc0, tc1);   // CSK tail: before / after sync 1, reduced
+    if (threadIdx.x == 64) tl_rec(tlb, 8900 + EPI, tc2, tl_now());   // reduced, after sync 2, (stored: below)
     if (warp >= 2 && warp <= 5 && (EPI == E3_DEC_STORE || EPI == E3_DEC_RESID)) {
       const int et = threadIdx.x - 64;
       constexpr int NG = RPC / 8, TP = 128 / NG;   // 8-row groups, tokens per pass
@@ -642,6 +752,7 @@ __global__ void __launch_bounds__(kDThreads, 1)
       }
     }
   }
+  if (CSK > 1 && threadIdx.x == 64) tl_rec(tlb, 8950 + EPI, tl0, tl0);   // CSK tail: stored
   tc_fence_before();
   __syncthreads();
   tc_fence_after();

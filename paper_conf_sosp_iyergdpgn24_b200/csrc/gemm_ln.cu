@@ -64,7 +64,9 @@ __global__ void __cluster_dims__(2, 1, 1) __launch_bounds__(kLThreads, 1)
   const unsigned long long tl0 = tl_now();
   unsigned long long *const tlb = g_tl;
   extern __shared__ uint8_t smem_raw[];
-  uint8_t *smem = reinterpret_cast<uint8_t *>((reinterpret_cast<uintptr_t>(smem_raw) + 1023) & ~uintptr_t(1023));
+  // 1024-B aligned by offset arithmetic on the __shared__ array, so the
+  // compiler keeps the shared address space (LDS / STS, not generic LD / ST)
+  uint8_t *smem = smem_raw + ((1024u - (smem_u32(smem_raw) & 1023u)) & 1023u);
   uint8_t *sA = smem;
   uint8_t *sW = smem + S * CF::kA;
   uint8_t *sY = smem;                                   // after the mainloop: y / LN tile
@@ -348,7 +350,9 @@ __global__ void __cluster_dims__(4, 1, 1) __launch_bounds__(kLThreads, 1)
   const unsigned long long tl0 = tl_now();
   unsigned long long *const tlb = g_tl;
   extern __shared__ uint8_t smem_raw[];
-  uint8_t *smem = reinterpret_cast<uint8_t *>((reinterpret_cast<uintptr_t>(smem_raw) + 1023) & ~uintptr_t(1023));
+  // 1024-B aligned by offset arithmetic on the __shared__ array, so the
+  // compiler keeps the shared address space (LDS / STS, not generic LD / ST)
+  uint8_t *smem = smem_raw + ((1024u - (smem_u32(smem_raw) & 1023u)) & 1023u);
   uint8_t *sA = smem;
   uint8_t *sW = smem + S * CF::kA;
   uint8_t *sY = smem;                                   // after the mainloop: y / LN tile

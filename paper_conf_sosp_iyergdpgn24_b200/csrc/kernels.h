@@ -28,6 +28,7 @@ e3_status tl_set_ramp(void *buf);
 e3_status tl_set_compact(void *buf);
 e3_status tl_set_gemm_ln(void *buf);
 e3_status tl_set_dec(void *buf);
+e3_status tl_set_llama(void *buf);
 e3_status gemm_tmaps(GemmMaps *g, const void *A, int64_t lda, const void *W, const void *C, int M, int N, int K,
                      int bn);
 e3_status gemm_run(const GemmMaps &g, const void *bias, const void *R, int M, int N, int K, int epi, int sms,

@@ -40,8 +40,11 @@ __global__ void __launch_bounds__(256) rmsnorm_kernel(const __nv_bfloat16 *__res
     const int k = lane + 32 * i;
     gv[i] = (k < nvec) ? __ldg(reinterpret_cast<const uint4 *>(g) + k) : make_uint4(0, 0, 0, 0);
   }
+  const unsigned long long tl0 = tl_now();
+  unsigned long long *const tlb = g_tl;
   pdl_wait();
   pdl_trigger();
+  const unsigned long long tl1 = tl_now();
   if (row >= rows) return;
   const uint4 *xr = reinterpret_cast<const uint4 *>(x + (size_t)row * H);
   uint4 v[VPL];
@@ -70,6 +73,7 @@ __global__ void __launch_bounds__(256) rmsnorm_kernel(const __nv_bfloat16 *__res
       o[e] = pack_bf16(bf_lo(w[e]) * rinv * bf_lo(gw[e]), bf_hi(w[e]) * rinv * bf_hi(gw[e]));
     yr[k] = make_uint4(o[0], o[1], o[2], o[3]);
   }
+  if (threadIdx.x == 0) tl_rec(tlb, 8700, tl0, tl1);
 }
 
 constexpr int kAttnThreads = 256;
@@ -128,8 +132,11 @@ __global__ void __launch_bounds__(kAttnThreads)
   const int h = blockIdx.x, t = blockIdx.y;
   const int tid = threadIdx.x, warp = warp_id(), lane = lane_id();
   const int H = nh * kHd;
+  const unsigned long long tl0 = tl_now();
+  unsigned long long *const tlb = g_tl;
   pdl_wait();
   pdl_trigger();
+  const unsigned long long tl1 = tl_now();
   const int nv = n_valid_dev ? *n_valid_dev : n_valid_host;
   const int64_t id = ids[t];
   __nv_bfloat16 *out = ctx + (size_t)t * H + h * kHd;
@@ -217,6 +224,7 @@ __global__ void __launch_bounds__(kAttnThreads)
     o.y = pack_bf16(s4.z * il, s4.w * il);
     reinterpret_cast<uint2 *>(out)[lane] = o;
   }
+  if (tid == 0) tl_rec(tlb, 8600, tl0, tl1);
 }
 
 __global__ void __launch_bounds__(128) lm_decide_kernel(RampArgs a) {
@@ -323,6 +331,8 @@ __global__ void decode_advance_kernel(const int64_t *__restrict__ ids, int64_t n
 
 }  // namespace
 
+E3_TL_SETTER(tl_set_llama)
+
 e3_status fill_prep_run(const int64_t *ids, int nv, int B, const void *hidden, int64_t cap, const int32_t *exit_layer,
                         int layer, int64_t row_bytes, void *x, int64_t *ids_out, uint8_t *mask, cudaStream_t st) {
   fill_prep_kernel<<<B, 128, 0, st>>>(ids, nv, B, reinterpret_cast<const uint8_t *>(hidden), cap, exit_layer, layer,
@@ -355,6 +365,8 @@ __global__ void __launch_bounds__(256) rmsnorm_cta_kernel(const __nv_bfloat16 *_
                                                           const __nv_bfloat16 *__restrict__ g,
                                                           __nv_bfloat16 *__restrict__ y, int rows, int H, float eps) {
   __shared__ float red[8];
+  const unsigned long long tl0 = tl_now();
+  unsigned long long *const tlb = g_tl;
   const int row = blockIdx.x, t = threadIdx.x, warp = warp_id(), lane = lane_id();
   const int nvec = H / 8;
   uint4 gv[VPT];
@@ -365,6 +377,7 @@ __global__ void __launch_bounds__(256) rmsnorm_cta_kernel(const __nv_bfloat16 *_
   }
   pdl_wait();
   pdl_trigger();
+  const unsigned long long tl1 = tl_now();
   if (row >= rows) return;
   const uint4 *xr = reinterpret_cast<const uint4 *>(x + (size_t)row * H);
   uint4 v[VPT];
@@ -398,6 +411,7 @@ __global__ void __launch_bounds__(256) rmsnorm_cta_kernel(const __nv_bfloat16 *_
       o[e] = pack_bf16(bf_lo(w[e]) * rinv * bf_lo(gw[e]), bf_hi(w[e]) * rinv * bf_hi(gw[e]));
     yr[k] = make_uint4(o[0], o[1], o[2], o[3]);
   }
+  if (threadIdx.x == 0) tl_rec(tlb, 8700, tl0, tl1);
 }
 
 e3_status rmsnorm_run(const void *x, const void *g, void *y, int rows, int H, float eps, cudaStream_t st) {

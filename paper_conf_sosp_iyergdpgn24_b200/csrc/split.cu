@@ -17,6 +17,7 @@
 // x_in is never written.
 #include <cstdlib>
 #include <cstring>
+#include <mutex>
 #include <new>
 
 #include "common.cuh"
@@ -1009,6 +1010,7 @@ e3_status e3_debug_timeline(void *dev_buf) {
   if (r == E3_OK) r = tl_set_compact(dev_buf);
   if (r == E3_OK) r = tl_set_gemm_ln(dev_buf);
   if (r == E3_OK) r = tl_set_dec(dev_buf);
+  if (r == E3_OK) r = tl_set_llama(dev_buf);
   if (r == E3_OK) r = tl_set_rampc(dev_buf);
   return r;
 }
@@ -1038,11 +1040,41 @@ e3_status e3_op_dec_gemm(void *stream, const void *X, int32_t T, const void *W, 
   e3_status r = dec_tmaps(&m, X, T, K, W, W2, N, epi);
   if (r != E3_OK) return r;
   const int tiles = dec_tiles(N, epi), mc = dec_max_contrib(N, K, epi, sms);
-  float *part = nullptr;
-  unsigned *tick = nullptr;
-  E3_CUDA_TRY(cudaMallocAsync(reinterpret_cast<void **>(&part), (size_t)tiles * mc * T * 128 * 4, st));
-  E3_CUDA_TRY(cudaMallocAsync(reinterpret_cast<void **>(&tick), (size_t)tiles * 4, st));
-  E3_CUDA_TRY(cudaMemsetAsync(tick, 0, (size_t)tiles * 4, st));
+  // stream-K scratch kept per device across calls (the tickets reset
+  // themselves at the end of every launch), so back-to-back calls are
+  // kernel-to-kernel like the split path's: an allocation + memset + free
+  // per call put ~6-10 us of graph nodes between the kernels.  Calls on one
+  // device must not run concurrently on different streams.
+  struct Scratch {
+    float *part = nullptr;
+    unsigned *tick = nullptr;
+    size_t part_elems = 0, tick_elems = 0;
+  };
+  static std::mutex mu;
+  static Scratch scr[64];
+  E3_CHECK_ARG(dev >= 0 && dev < 64, "device index");
+  std::lock_guard<std::mutex> lock(mu);
+  Scratch &sc = scr[dev];
+  const size_t pe = (size_t)tiles * mc * T * 128, te = (size_t)tiles;
+  if (pe > sc.part_elems) {
+    E3_CUDA_TRY(cudaStreamSynchronize(st));
+    if (sc.part) cudaFree(sc.part);
+    sc.part = nullptr;
+    sc.part_elems = 0;
+    E3_CUDA_TRY(cudaMalloc(reinterpret_cast<void **>(&sc.part), pe * 4));
+    sc.part_elems = pe;
+  }
+  if (te > sc.tick_elems) {
+    E3_CUDA_TRY(cudaStreamSynchronize(st));
+    if (sc.tick) cudaFree(sc.tick);
+    sc.tick = nullptr;
+    sc.tick_elems = 0;
+    E3_CUDA_TRY(cudaMalloc(reinterpret_cast<void **>(&sc.tick), te * 4));
+    E3_CUDA_TRY(cudaMemset(sc.tick, 0, te * 4));
+    sc.tick_elems = te;
+  }
+  float *part = sc.part;
+  unsigned *tick = sc.tick;
   DecArgs a{};
   a.T = T;
   a.N = N;
@@ -1054,10 +1086,7 @@ e3_status e3_op_dec_gemm(void *stream, const void *X, int32_t T, const void *W, 
   a.ldo = N;
   a.part = part;
   a.tickets = tick;
-  r = dec_run(m, a, sms, st);
-  cudaFreeAsync(part, st);
-  cudaFreeAsync(tick, st);
-  return r;
+  return dec_run(m, a, sms, st);
 }
 
 e3_status e3_op_gemm_ln(void *stream, const void *A, const void *W, const void *bias, const void *R, const void *g,

@@ -52,7 +52,7 @@ for name, N, K, epi in shapes:
         print(f"         {len(red)} tile reductions: start {f(red[:, 0])}  end {f(red[:, 2])}  "
               f"duration median {np.median(red[:, 2] - red[:, 0]) / 1000:.2f} us")
     if name == "o" or "-v" in sys.argv:
-        bid = (r[:, 0] >> 16).astype(int)
+        bid = ((r[:, 0] >> 16) & 0xFFFFFFFF).astype(int)
         mm = (kid >= 8000) & (kid < 8100)
         order = np.argsort(-t[mm][:, 2])[:8]
         rb = bid[kid >= 8200]
