@@ -30,54 +30,51 @@ namespace {
 
 constexpr int D = 64;          // head dim
 constexpr int QT = 128;        // query rows per item
-// KP threads per query row (warps w, w+4, ... own TMEM lane quarter w % 4 and
-// one of KP key ranges): 2 for S <= 128 (256 threads, 2 CTAs per SM), 4 above
-// (512 threads, one CTA per SM: each thread keeps its <= 64 scores in
-// registers instead of re-reading TMEM, and twice the warps hide the MUFU
-// and TMEM latencies)
+// KP = 2 threads per query row: warps w and w+4 own TMEM lane quarter w % 4
+// and one of two key ranges each (256 threads, two CTAs per SM)
 template <int SKV>
 struct AThr {
-  // r02: 2 threads per query row at every SKV (above 128 keys the second CTA
-  // per SM, below, replaces the r01 layout of 4 threads per row in one CTA)
   static constexpr int KP = 2;
   static constexpr int kThreads = 128 * KP;
 };
 
 // SKV = keys per tile: S rounded up to 128 or, above 128, to a multiple of 32
-// (S = 197 -> 224: 12 % fewer masked exponentials than 256 and small enough
-// K/V tiles to double-buffer the next item's loads)
+// (S = 197 -> 224: 12 % fewer masked exponentials than 256).
+//
+// r02: P lives in TMEM (tcgen05.st over the thread's own dead S columns) and
+// MMA2 reads it as its A operand (tcgen05.mma [d], [a_tmem], b_desc), so the
+// smem holds only Q, K and V: above 128 keys the next item's Q | K land
+// during this item's softmax (Q | K are dead once MMA1 completed) and V is
+// double-buffered; at 128 keys whole Q | K | V buffers are double-buffered.
+// Before (P in smem over the dead Q | K): the next item's loads could only
+// start after MMA2, 2.3 us exposed per item at S = 197 (attn_trace).
 template <int SKV>
 struct ACfg {
   static constexpr int kQ = QT * D * 2;                  // 16 KB
   static constexpr int kKV = SKV * D * 2;                // 16 .. 32 KB
-  static constexpr int kP = ((SKV + 63) / 64) * QT * 128;   // bf16 P in 64-key SW128 blocks
-  // above 128 keys (S = 197 -> 224, r02): TWO CTAs per SM instead of one
-  // double-buffered CTA -- one CTA's softmax overlaps the other's loads and
-  // MMAs (r01 trace: 3.6 us per item, strictly serial load -> S -> softmax
-  // -> PV -> store).  To fit two 256-thread CTAs, P (64 KB) overwrites the
-  // dead Q | K tiles plus a pad placed before V: [Q | K | pad | V].
-  static constexpr bool kTwoPerSm = SKV > 128;
-  static constexpr int kPad = (kTwoPerSm && kP > kQ + kKV) ? kP - kQ - kKV : 0;
-  static constexpr int kVOff = kQ + kKV + kPad;          // V tile offset in a buffer
-  static constexpr int kBuf = kVOff + kKV;               // Q | K | (pad) | V
-  static constexpr bool kPInQK = (kP <= kQ + kKV + kPad);   // P overwrites the dead Q|K(|pad) tiles
-  static constexpr int kExtra = 1024 + 64 + 2 * 2 * AThr<SKV>::KP * QT * 4;
-#ifdef E3_ATTN_SINGLE_BUF   // diagnostics: occupancy instead of double buffering
-  static constexpr int kNBuf = 1;
-#else
-  static constexpr int kNBuf = kTwoPerSm ? 1 : ((2 * kBuf + (kPInQK ? 0 : kP) + kExtra <= 232448) ? 2 : 1);
-#endif
-  static constexpr int kSmem = kNBuf * kBuf + (kPInQK ? 0 : kP) + kExtra;
-  static constexpr int kSCols = SKV <= 128 ? 128 : 256;      // one S (later O, 64 columns) accumulator
-  // above 128 keys (one CTA per SM) two accumulators: MMA1 of item j+1 runs
-  // while item j's output is written
-  static constexpr bool kPipe = SKV > 128 && kNBuf == 2;
-  static constexpr int kTmemCols = kPipe ? 2 * kSCols : kSCols;
+  static constexpr int kExtra = 1024 + 128 + 2 * 2 * AThr<SKV>::KP * QT * 4;
+  static constexpr int kSmemMax = 232448 / 2 - 2048;     // two CTAs per SM
+  // slots: Q|K pairs and V tiles
+  static constexpr int kNQK = SKV <= 128 ? 2 : 1;
+  static constexpr int kNV = (kNQK * (kQ + kKV) + 2 * kKV + kExtra <= kSmemMax) ? 2 : 1;
+  static constexpr int kQKBytes = kNQK * (kQ + kKV);
+  static constexpr int kSmem = kQKBytes + kNV * kKV + kExtra;
+  static_assert(kSmem <= kSmemMax + 2048, "attention smem");
+  static constexpr int NCH = SKV / 32;                   // 32-key chunks
+  static constexpr int NCH0 = (NCH + 1) / 2;             // chunks of key part 0
+  static constexpr int kBeginB = NCH0 * 32;              // first key of part 1
+  // TMEM: S at columns [0, SKV); P of key k of part p at column
+  // begin_p + (k - begin_p) / 2 (two bf16 per column, inside the part's own
+  // S columns, already read); O (64 columns) past S, or between the parts
+  static constexpr int kTmemCols = 256;
+  static constexpr int kOCol = (((SKV + 31) / 32) * 32 + 64 <= kTmemCols) ? ((SKV + 31) / 32) * 32 : NCH0 * 16;
+  static_assert(kOCol + 64 <= kTmemCols, "O columns");
+  static_assert(kOCol >= SKV || kOCol + 64 <= kBeginB, "O overlaps part 1's P");
 };
 
 // Diagnostics (e3_debug_gemm_trace): per CTA and item (<= 8), globaltimer
-// stamps: [0] loads landed, [1] S in TMEM, [2] P in smem (MMA2 issued),
-// [3] O in TMEM, [4] output staged (store issued)
+// stamps: [0] MMA1 issued (Q | K landed), [1] S in TMEM, [2] P in TMEM
+// (MMA2 issued), [3] O in TMEM, [4] output staged (store issued)
 __device__ unsigned long long *g_attn_trace = nullptr;
 __device__ __forceinline__ void atrace(int j, int kind) {
   unsigned long long *b = g_attn_trace;
@@ -96,19 +93,20 @@ __global__ void __launch_bounds__(AThr<SKV>::kThreads, 2)
                    const __grid_constant__ CUtensorMap tctx, int S, int H, int heads, int n_items) {
   using CF = ACfg<SKV>;
   constexpr int KP = AThr<SKV>::KP;
-  constexpr int NCH = SKV / 32;     // 32-key chunks; key part p takes chunks [p NCHP, (p + 1) NCHP)
-  constexpr int NCHP = (NCH + KP - 1) / KP;
+  constexpr int NCH = CF::NCH;
+  constexpr int NCH0 = CF::NCH0;
   extern __shared__ uint8_t smem_raw[];
   // 1024-B aligned by offset arithmetic on the __shared__ array, so the
   // compiler keeps the shared address space (LDS / STS, not generic LD / ST)
   uint8_t *smem = smem_raw + ((1024u - (smem_u32(smem_raw) & 1023u)) & 1023u);
-  uint8_t *pbuf_sep = smem + CF::kNBuf * CF::kBuf;      // only when !kPInQK
-  float *xch = reinterpret_cast<float *>(smem + CF::kNBuf * CF::kBuf + (CF::kPInQK ? 0 : CF::kP));  // [2][2][KP][QT]
+  uint8_t *sVbase = smem + CF::kQKBytes;
+  float *xch = reinterpret_cast<float *>(sVbase + CF::kNV * CF::kKV);   // [2][2][KP][QT]
   uint64_t *bars = reinterpret_cast<uint64_t *>(xch + 2 * 2 * KP * QT);
-  uint64_t *bar_load = bars;        // [2]
-  uint64_t *bar_s = bars + 2;
-  uint64_t *bar_o = bars + 3;
-  uint32_t *tslot = reinterpret_cast<uint32_t *>(bars + 4);
+  uint64_t *bar_qk = bars;          // [2]
+  uint64_t *bar_v = bars + 2;       // [2]
+  uint64_t *bar_s = bars + 4;
+  uint64_t *bar_o = bars + 5;
+  uint32_t *tslot = reinterpret_cast<uint32_t *>(bars + 6);
 
   const int warp = warp_id(), lane = lane_id();
   const int tid = threadIdx.x;
@@ -116,7 +114,7 @@ __global__ void __launch_bounds__(AThr<SKV>::kThreads, 2)
   unsigned long long *const tlb = g_tl;
   const int qtiles = (S + QT - 1) / QT;
   const int quarter = warp & 3;
-  const int khalf = warp >> 2;                            // which key part (and, for parts 0-1, half of D)
+  const int khalf = warp >> 2;                            // which key part (and half of D for the output)
   const int row = quarter * 32 + lane;                    // query row within tile == TMEM lane
   const uint32_t lane_off = (uint32_t)(quarter * 32) << 16;
   const float sl2 = 1.4426950408889634f * 0.125f;         // log2(e) / sqrt(64)
@@ -125,10 +123,7 @@ __global__ void __launch_bounds__(AThr<SKV>::kThreads, 2)
     tma_prefetch(&tq);
     tma_prefetch(&tkv);
     tma_prefetch(&tctx);
-    mbar_init(&bar_load[0], 1);
-    mbar_init(&bar_load[1], 1);
-    mbar_init(bar_s, 1);
-    mbar_init(bar_o, 1);
+    for (int i = 0; i < 6; ++i) mbar_init(&bars[i], 1);
     fence_barrier_init();
   }
   if (warp == 0) tmem_alloc(tslot, CF::kTmemCols);
@@ -140,59 +135,66 @@ __global__ void __launch_bounds__(AThr<SKV>::kThreads, 2)
   pdl_trigger();
   const unsigned long long tl1 = tl_now();
 
-  auto issue_load = [&](int item, int buf) {
-    const int bh = item / qtiles, qt = item % qtiles;
-    const int b = bh / heads, h = bh % heads;
-    uint8_t *base = smem + buf * CF::kBuf;
-    mbar_expect_tx(&bar_load[buf], CF::kQ + 2 * CF::kKV);   // the pad is not loaded
-    tma_load_3d(base, &tq, &bar_load[buf], h * D, qt * QT, b);
-    tma_load_3d(base + CF::kQ, &tkv, &bar_load[buf], H + h * D, 0, b);
-    tma_load_3d(base + CF::kVOff, &tkv, &bar_load[buf], 2 * H + h * D, 0, b);
+  auto coords = [&](int it, int &b, int &h, int &qt) {
+    const int bh = it / qtiles;
+    qt = it % qtiles;
+    b = bh / heads;
+    h = bh % heads;
   };
-
-  uint32_t load_phases = 0;                               // bit i: parity of bar_load[i] (thread 0)
-  // S = Q K^T of the item in buffer `bf` into S accumulator `acc`
-  auto issue_mma1 = [&](int bf, int acc) {
-    mbar_wait(&bar_load[bf], (load_phases >> bf) & 1u);
-    load_phases ^= 1u << bf;
-    tc_fence_after();
-    uint8_t *q = smem + bf * CF::kBuf;
-    const uint32_t idesc = idesc_bf16_f32(QT, SKV, 0);
-    const uint64_t dq = smem_desc_sw128(smem_u32(q), 16, 1024);
-    const uint64_t dk = smem_desc_sw128(smem_u32(q + CF::kQ), 16, 1024);
-#pragma unroll
-    for (int k = 0; k < D / 16; ++k) tc_mma_f16(tbase + acc * CF::kSCols, dq + 2 * k, dk + 2 * k, idesc, k != 0);
-    tc_commit(bar_s);
+  auto issue_qk = [&](int it, int slot) {
+    int b, h, qt;
+    coords(it, b, h, qt);
+    uint8_t *base = smem + slot * (CF::kQ + CF::kKV);
+    mbar_expect_tx(&bar_qk[slot], CF::kQ + CF::kKV);
+    tma_load_3d(base, &tq, &bar_qk[slot], h * D, qt * QT, b);
+    tma_load_3d(base + CF::kQ, &tkv, &bar_qk[slot], H + h * D, 0, b);
+  };
+  auto issue_v = [&](int it, int slot) {
+    int b, h, qt;
+    coords(it, b, h, qt);
+    mbar_expect_tx(&bar_v[slot], CF::kKV);
+    tma_load_3d(sVbase + slot * CF::kKV, &tkv, &bar_v[slot], 2 * H + h * D, 0, b);
+  };
+  uint32_t phases = 0;                                    // bit i: parity of bars[i] (thread 0)
+  auto wait_bar = [&](int i) {
+    mbar_wait(&bars[i], (phases >> i) & 1u);
+    phases ^= 1u << i;
   };
 
   int item = blockIdx.x;
   if (tid == 0 && item < n_items) {
-    issue_load(item, 0);
-    if (CF::kPipe) issue_mma1(0, 0);
+    issue_qk(item, 0);
+    issue_v(item, 0);
   }
   uint32_t sphase = 0, ophase = 0;
 
   for (int j = 0; item < n_items; ++j, item += gridDim.x) {
-    const int buf = (CF::kNBuf == 2) ? (j & 1) : 0;
-    uint8_t *sQ = smem + buf * CF::kBuf;
-    uint8_t *sK = sQ + CF::kQ;
-    uint8_t *sV = sQ + CF::kVOff;
-    uint8_t *sP = CF::kPInQK ? sQ : pbuf_sep;
-    const int bh = item / qtiles, qt = item % qtiles;
-    const int b = bh / heads, h = bh % heads;
+    const int qs = (CF::kNQK == 2) ? (j & 1) : 0;
+    const int vs = (CF::kNV == 2) ? (j & 1) : 0;
+    uint8_t *sQ = smem + qs * (CF::kQ + CF::kKV);
+    uint8_t *sV = sVbase + vs * CF::kKV;
+    int b, h, qt;
+    coords(item, b, h, qt);
     const int q0 = qt * QT;
     const int next = item + gridDim.x;
 
-    const uint32_t tS = tbase + (CF::kPipe ? (j & 1) * CF::kSCols : 0);   // this item's S, later O
-    (void)sK;
     if (tid == 0) {
-      if (!CF::kPipe) issue_mma1(buf, 0);               // kPipe: issued during the previous item
+      // MMA1: S = Q K^T
+      wait_bar(qs);
+      tc_fence_after();
       atrace(j, 0);
-      if (CF::kNBuf == 2 && next < n_items) {
-        // the other buffer's last readers: MMA2 of item j-1 (done: waited before
-        // its epilogue) and the TMA store of its output from the V tile
+      const uint32_t idesc = idesc_bf16_f32(QT, SKV, 0);
+      const uint64_t dq = smem_desc_sw128(smem_u32(sQ), 16, 1024);
+      const uint64_t dk = smem_desc_sw128(smem_u32(sQ + CF::kQ), 16, 1024);
+#pragma unroll
+      for (int k = 0; k < D / 16; ++k) tc_mma_f16(tbase, dq + 2 * k, dk + 2 * k, idesc, k != 0);
+      tc_commit(bar_s);
+      if (next < n_items) {
+        // the other slots' last readers: MMA1 / MMA2 of item j-1 (done: waited
+        // before its output) and the TMA store of its output from its V tile
         bulk_wait_read<0>();
-        issue_load(next, buf ^ 1);
+        if (CF::kNQK == 2) issue_qk(next, qs ^ 1);
+        if (CF::kNV == 2) issue_v(next, vs ^ 1);
       }
     }
     __syncwarp();
@@ -201,11 +203,13 @@ __global__ void __launch_bounds__(AThr<SKV>::kThreads, 2)
     mbar_wait(bar_s, sphase);
     sphase ^= 1;
     tc_fence_after();
-    if (tid == 0) atrace(j, 1);
+    if (tid == 0) {
+      atrace(j, 1);
+      if (CF::kNQK == 1 && next < n_items) issue_qk(next, 0);   // Q | K dead once MMA1 completed
+    }
     // S = 128: S is read from TMEM once, this thread's 64 keys stay in
     // registers between the max pass and the exponentiation pass (-6 %);
     // longer rows would spill, so they are read twice
-    constexpr int NCH0 = NCHP;                            // chunks per key part (the last may have fewer)
     constexpr bool kKeep = NCH0 <= 2;                     // <= 64 registers; longer rows reload
     const int c_begin = khalf * NCH0 * 32;
     // a lane quarter whose 32 query rows all lie past S (the second query
@@ -220,7 +224,7 @@ __global__ void __launch_bounds__(AThr<SKV>::kThreads, 2)
       if (ci < nch) {
         const int c = c_begin + ci * 32;
         uint32_t r[32];
-        tmem_ld32(tS + lane_off + c, r);
+        tmem_ld32(tbase + lane_off + c, r);
         tmem_wait_ld();
         float m4[4] = {-INFINITY, -INFINITY, -INFINITY, -INFINITY};
         if (kMask && c + 32 > S) {        // the chunk holding key S: masked keys become -inf (p = 0)
@@ -250,14 +254,13 @@ __global__ void __launch_bounds__(AThr<SKV>::kThreads, 2)
     for (int q = 1; q < KP; ++q) mx = fmaxf(mx, xmax[q * QT + row]);
     const float mb = mx * sl2;
     float l4[4] = {0.f, 0.f, 0.f, 0.f};
-    uint8_t *prow = sP + row * 128;
 #pragma unroll
     for (int ci = 0; ci < NCH0; ++ci) {
       if (ci < nch) {
         const int c = c_begin + ci * 32;
         if (!kKeep) {
           uint32_t r[32];
-          tmem_ld32(tS + lane_off + c, r);
+          tmem_ld32(tbase + lane_off + c, r);
           tmem_wait_ld();
 #pragma unroll
           for (int jj = 0; jj < 32; ++jj) sv[jj] = __uint_as_float(r[jj]);
@@ -286,38 +289,34 @@ __global__ void __launch_bounds__(AThr<SKV>::kThreads, 2)
           l4[2] = a1.x;
           l4[3] = a1.y;
         }
-        // columns c..c+31 -> block c/64, 16-byte chunks (c%64)/8 .. +3, XOR-swizzled by row%8
-        uint8_t *blk = prow + (c / 64) * (QT * 128);
-        const int ch0 = (c % 64) / 8;
+        // bf16(p) of keys c..c+31 -> 16 TMEM columns of this row, inside this
+        // part's own S columns (keys <= c + 15: already read)
+        uint32_t pk[16];
 #pragma unroll
-        for (int jj = 0; jj < 4; ++jj) {
-          uint4 o;
-          o.x = pack_bf16(p[8 * jj + 0], p[8 * jj + 1]);
-          o.y = pack_bf16(p[8 * jj + 2], p[8 * jj + 3]);
-          o.z = pack_bf16(p[8 * jj + 4], p[8 * jj + 5]);
-          o.w = pack_bf16(p[8 * jj + 6], p[8 * jj + 7]);
-          *reinterpret_cast<uint4 *>(blk + (((ch0 + jj) ^ (row & 7)) << 4)) = o;
-        }
+        for (int jj = 0; jj < 16; ++jj) pk[jj] = pack_bf16(p[2 * jj], p[2 * jj + 1]);
+        tmem_st16(tbase + lane_off + c_begin + (c - c_begin) / 2, pk);
       }
     }
     const float lpart = (l4[0] + l4[1]) + (l4[2] + l4[3]);
     xsum[khalf * QT + row] = lpart;
-    fence_proxy_async_smem();     // generic-proxy smem writes -> visible to the tensor core
-    tc_fence_before();            // S fully read before MMA2 overwrites it with O
+    tmem_wait_st();
+    tc_fence_before();            // P in TMEM before MMA2 reads it
     __syncthreads();
 
     if (tid == 0) {
+      wait_bar(2 + vs);           // this item's V
       tc_fence_after();
       atrace(j, 2);
-      const uint32_t idesc = idesc_bf16_f32(QT, D, 1);   // B (= V) is MN-major
+      const uint32_t idesc = idesc_bf16_f32(QT, D, 1);   // B (= V) is MN-major, A (= P) K-major in TMEM
 #pragma unroll
       for (int kk = 0; kk < SKV / 16; ++kk) {
-        const uint64_t dp = smem_desc_sw128(smem_u32(sP + (kk / 4) * (QT * 128) + (kk % 4) * 32), 16, 1024);
+        const int k = kk * 16;
+        const int cb = k < CF::kBeginB ? 0 : CF::kBeginB;
+        const uint32_t ap = tbase + (uint32_t)(cb + (k - cb) / 2);
         const uint64_t dv = smem_desc_sw128(smem_u32(sV + kk * 16 * 128), SKV * 128, 1024);
-        tc_mma_f16(tS, dp, dv, idesc, kk != 0);
+        tc_mma_f16_ts(tbase + CF::kOCol, ap, dv, idesc, kk != 0);
       }
       tc_commit(bar_o);
-      if (CF::kPipe && next < n_items) issue_mma1(buf ^ 1, (j + 1) & 1);   // overlaps this item's output
     }
     __syncwarp();
     mbar_wait(bar_o, ophase);     // MMA2 done: V tile is dead -> output staging
@@ -328,9 +327,9 @@ __global__ void __launch_bounds__(AThr<SKV>::kThreads, 2)
 #pragma unroll
     for (int q = 1; q < KP; ++q) l += xsum[q * QT + row];
     const float inv_l = 1.0f / l;
-    if (khalf < 2 && qvalid) {    // parts 0 and 1 write the 2 x 32 output columns
+    if (qvalid) {                 // part k writes output columns 32k .. 32k + 31
       uint32_t r[32];
-      tmem_ld32(tS + lane_off + khalf * 32, r);           // this thread's 32 of the 64 d columns
+      tmem_ld32(tbase + lane_off + CF::kOCol + khalf * 32, r);   // this thread's 32 of the 64 d columns
       tmem_wait_ld();
       uint8_t *orow = sV + row * 128;                     // [128 q x 128 B], 128B swizzle
 #pragma unroll
@@ -344,15 +343,15 @@ __global__ void __launch_bounds__(AThr<SKV>::kThreads, 2)
       }
     }
     fence_proxy_async_smem();
-    tc_fence_before();            // O read before the next MMA1 overwrites TMEM
+    tc_fence_before();            // O read before the next MMA1 / P writes reuse TMEM
     __syncthreads();
     if (tid == 0) {
       atrace(j, 4);
       tma_store_3d(&tctx, sV, h * D, q0, b);
       bulk_commit();
-      if (CF::kNBuf == 1 && next < n_items) {
+      if (CF::kNV == 1 && next < n_items) {               // the store reads the only V tile first
         bulk_wait_read<0>();
-        issue_load(next, 0);
+        issue_v(next, 0);
       }
     }
   }
