@@ -355,7 +355,7 @@ __global__ void __launch_bounds__(AThr<SKV>::kThreads, 2)
       }
     }
   }
-  if (tid == 0) bulk_wait<0>();
+  if (tid == 0) bulk_wait_read<0>();   // smem read before exit; the global writes complete with the grid
   __syncthreads();
   if (warp == 0) tmem_dealloc(tbase, CF::kTmemCols);
   if (tid == 0) tl_rec(tlb, 2000 + SKV + (kMask ? 500 : 0), tl0, tl1);

@@ -43,7 +43,7 @@ struct LCfg {
   static constexpr int kA = LM * LBK * 2;            // 16 KB
   static constexpr int kW = NH * LBK * 2;
   static constexpr int kStage = kA + kW;
-  static constexpr int kExtra = 1024 + 512 + 4 * 2 * LM * 4 + 3 * NH * 2;   // align, barriers, partials, params
+  static constexpr int kExtra = 1024 + 512 + (2 * 3 + 4) * LM * 4 + 3 * NH * 2;   // align, barriers, partials, params
   static constexpr int kStages = (kLSmemMax - kExtra) / kStage;
   static constexpr int kY = LM * NH * 2;             // bf16 y tile, [NH/64 blocks][128 rows][128 B]
   static_assert(kStages >= 2, "pipeline too shallow");
@@ -53,6 +53,8 @@ struct LCfg {
 };
 
 __device__ __forceinline__ void epi_bar256() { asm volatile("bar.sync 1, 256;" ::: "memory"); }
+template <int NT>
+__device__ __forceinline__ void epi_bar_n() { asm volatile("bar.sync 1, %0;" ::"n"(NT) : "memory"); }
 
 template <int NH>
 __global__ void __cluster_dims__(2, 1, 1) __launch_bounds__(kLThreads, 1)
@@ -70,9 +72,14 @@ __global__ void __cluster_dims__(2, 1, 1) __launch_bounds__(kLThreads, 1)
   uint8_t *sA = smem;
   uint8_t *sW = smem + S * CF::kA;
   uint8_t *sY = smem;                                   // after the mainloop: y / LN tile
-  float *xs = reinterpret_cast<float *>(smem + S * CF::kStage);    // [2 halves][128] local sums
-  float *xr2 = xs + 2 * LM;                                        // [2 halves][128] local squares
-  float *xr1 = xr2 + 2 * LM;                                       // [2 ranks][128][2] exchange
+  // epilogue warps: all 12 where NH splits into three 32-column-aligned
+  // parts (BB's 384), else warps 4-11 (two parts); the producer, MMA and
+  // allocator warps are idle once the accumulator is complete
+  constexpr int EW = (NH % 96 == 0) ? 12 : 8;
+  constexpr int NPART = EW / 4;                                    // column parts per row
+  float *xs = reinterpret_cast<float *>(smem + S * CF::kStage);    // [NPART][128] local sums
+  float *xr2 = xs + NPART * LM;                                    // [NPART][128] local squares
+  float *xr1 = xr2 + NPART * LM;                                   // [2 ranks][128][2] exchange
   __nv_bfloat16 *sPar = reinterpret_cast<__nv_bfloat16 *>(xr1 + 4 * LM);   // [3][NH]: bias, gamma, beta
   uint64_t *full = reinterpret_cast<uint64_t *>(sPar + 3 * NH);
   uint64_t *empty = full + S;
@@ -175,22 +182,24 @@ __global__ void __cluster_dims__(2, 1, 1) __launch_bounds__(kLThreads, 1)
   asm volatile("barrier.cluster.wait.aligned;" ::: "memory");   // the peer CTA is running
 
   // ---------------------------------------------------------------- epilogue
-  const bool epi = warp >= 4;
-  const int q = warp & 3, h = (warp - 4) >> 2;   // lane quarter, column half of this CTA's NH
+  const bool epi = EW == 12 || warp >= 4;
+  const int q = warp & 3, h = EW == 12 ? (warp >> 2) : ((warp - 4) >> 2);   // lane quarter, column part
   const int row = q * 32 + lane;
   const int m = m0 + row;
-  constexpr int HC = NH / 2;                      // columns per epilogue thread
+  constexpr int HC = NH / NPART;                  // columns per epilogue thread
   float2 sum2 = make_float2(0.f, 0.f), sq2 = make_float2(0.f, 0.f);   // row sum, sum of squares
+  unsigned long long tlA = 0, tlB = 0;
   if (epi) {
     mbar_wait(tfull, 0);                          // all MMAs done: the stage buffers are drained
     tc_fence_after();
+    tlA = tl_now();
     // the residual tile lands, by TMA, exactly where y1 will be written
     // (same 128-byte-swizzled block layout): one round trip for the whole tile
     if (warp == 4 && lane == 0) {
       mbar_expect_tx(rbar, LM * NH * 2);
       for (int blk = 0; blk < NH / 64; ++blk) tma_load_2d(sY + blk * (LM * 128), &tmR, rbar, n0 + blk * 64, m0);
     }
-    epi_bar256();                                 // sPar written by every epilogue thread
+    epi_bar_n<EW * 32>();                                 // sPar written by every epilogue thread
     mbar_wait(rbar, 0);
     const uint32_t taddr = tmem_base + ((uint32_t)(q * 32) << 16);
 #pragma unroll 1
@@ -231,9 +240,14 @@ __global__ void __cluster_dims__(2, 1, 1) __launch_bounds__(kLThreads, 1)
     // moment about 0 is exact enough in fp32 for LayerNorm inputs of O(1))
     xs[h * LM + row] = sum2.x + sum2.y;
     xr2[h * LM + row] = sq2.x + sq2.y;
-    epi_bar256();
+    epi_bar_n<EW * 32>();
     if (h == 0) {
-      const float s1 = xs[row] + xs[LM + row], s2 = xr2[row] + xr2[LM + row];
+      float s1 = xs[row], s2 = xr2[row];
+#pragma unroll
+      for (int pp = 1; pp < NPART; ++pp) {        // parts in order
+        s1 += xs[pp * LM + row];
+        s2 += xr2[pp * LM + row];
+      }
       xr1[2 * rank * LM + 2 * row] = s1;          // xr1 here: [2 ranks][128 rows][2]
       xr1[2 * rank * LM + 2 * row + 1] = s2;
       const uint32_t dst = mapa_shared(smem_u32(&xr1[2 * rank * LM + 2 * row]), rank ^ 1);
@@ -243,7 +257,7 @@ __global__ void __cluster_dims__(2, 1, 1) __launch_bounds__(kLThreads, 1)
   // y1 (the residual stream, ViT) is an output too: stored before the tile is
   // normalised in place (every thread's y1 writes were fenced above)
   if (a.store_pre) {
-    if (epi) epi_bar256();
+    if (epi) epi_bar_n<EW * 32>();
     if (warp == 4 && lane == 0) {
       for (int blk = 0; blk < NH / 64; ++blk) tma_store_2d(&tmPre, sY + blk * (LM * 128), n0 + blk * 64, m0);
       bulk_commit();
@@ -251,6 +265,7 @@ __global__ void __cluster_dims__(2, 1, 1) __launch_bounds__(kLThreads, 1)
   }
   cluster_sync();                                 // both CTAs' row statistics visible
   if (epi) {
+    tlB = tl_now();
     const float s1 = xr1[2 * row] + xr1[2 * LM + 2 * row], s2 = xr1[2 * row + 1] + xr1[2 * LM + 2 * row + 1];
     const float mean = s1 / (float)a.N;
     const float var = fmaxf(s2 / (float)a.N - mean * mean, 0.f);
@@ -258,7 +273,7 @@ __global__ void __cluster_dims__(2, 1, 1) __launch_bounds__(kLThreads, 1)
     const float2 nmean2 = make_float2(-mean, -mean), rstd2 = make_float2(rstd, rstd);
     if (a.store_pre) {                            // the y1 stores must have read the tile
       if (warp == 4 && lane == 0) bulk_wait_read<0>();
-      epi_bar256();
+      epi_bar_n<EW * 32>();
     }
 #pragma unroll 1
     for (int c = 0; c < HC; c += 8) {
@@ -282,11 +297,12 @@ __global__ void __cluster_dims__(2, 1, 1) __launch_bounds__(kLThreads, 1)
       *p = make_uint4(o[0], o[1], o[2], o[3]);
     }
     fence_proxy_async_smem();
-    epi_bar256();
+    epi_bar_n<EW * 32>();
     if (warp == 4 && lane == 0) {
       for (int blk = 0; blk < NH / 64; ++blk) tma_store_2d(&tmOut, sY + blk * (LM * 128), n0 + blk * 64, m0);
       bulk_commit();
-      bulk_wait<0>();
+      bulk_wait_read<0>();                        // smem read before exit; the global writes complete with the grid
+      tl_rec(tlb, 77, tlA, tlB);                  // mainloop done, statistics exchanged, stored
     }
   }
   tc_fence_before();
@@ -569,7 +585,7 @@ __global__ void __cluster_dims__(4, 1, 1) __launch_bounds__(kLThreads, 1)
     if (warp == 4 && lane == 0) {
       for (int blk = 0; blk < NH / 64; ++blk) tma_store_2d(&tmOut, sY + blk * (LM * 128), n0 + blk * 64, m0);
       bulk_commit();
-      bulk_wait<0>();
+      bulk_wait_read<0>();                        // smem read before exit; the global writes complete with the grid
     }
   }
   tc_fence_before();

@@ -357,7 +357,7 @@ __global__ void __cluster_dims__(2, 1, 1) __launch_bounds__(Cfg<BN, EPI>::kThrea
       if (lane == 0 && (warp == 4 || warp == 11)) trace(tl, warp == 4 ? 3 : 5);
       if (++acc == CF::kNAcc) { acc = 0; acc_phase ^= 1; }
     }
-    if (lane == 0) bulk_wait<0>();
+    if (lane == 0) bulk_wait_read<0>();   // smem read before exit; the global writes complete with the grid
   }
   tc_fence_before();
   cluster_sync();                  // no CTA leaves while its peer may still signal it
