@@ -12,9 +12,14 @@ timeout 900 python bench.py --config lm --decode-steps 4 --steps 3 --no-cpu > gp
 timeout 600 python bench.py --config bbp --no-cpu > gpurun_out/r02_bench_bbp.json 2> gpurun_out/r02_bench_bbp.err
 timeout 600 python bench.py --plan cut6 --no-cpu > gpurun_out/r02_bench_bb_cut6.json 2> gpurun_out/r02_bench_bb_cut6.err
 timeout 300 python scripts/timeline.py bb 1 3 > gpurun_out/r02_timeline_bb_layer.txt 2>&1
+timeout 300 python scripts/pipeline_timeline.py bb 4096 10 4 > gpurun_out/r02_pipeline_timeline_bb.txt 2>&1
+timeout 300 python scripts/llama_timeline.py 4 > gpurun_out/r02_timeline_llama_layers.txt 2>&1
+timeout 300 python scripts/dec_bench.py > gpurun_out/r02_dec_bench.txt 2>&1
+(timeout 120 python scripts/attn_bench.py; timeout 120 python scripts/attn_bench.py 256 197 768 12) > gpurun_out/r02_attn_bench.txt 2>&1
+timeout 600 python scripts/stage_loopback_bench.py > gpurun_out/stage_loopback.log 2>&1; echo loopback=$?
 timeout 900 python scripts/online_goodput.py > gpurun_out/online.log 2>&1; echo online=$?
 timeout 900 ncu --metrics gpu__time_duration.sum,dram__bytes_read.sum,dram__bytes_write.sum --clock-control none --csv \
-  --log-file gpurun_out/launches_bb.csv python bench.py --steps 1 --warmup 1 --no-cpu --no-e2e > gpurun_out/ncu_bench.log 2>&1; echo ncu1=$?
+  --log-file gpurun_out/launches_bb.csv python bench.py --steps 1 --warmup 1 --no-cpu --no-e2e --inputs-per-gpu 2048 > gpurun_out/ncu_bench.log 2>&1; echo ncu1=$?
 timeout 1200 ncu --set full --clock-control none --import-source on \
   -k regex:"gemm_bf16|attn_tc|ramp_bert|ln_compact|layernorm_kernel|gemm_ln" -c 10 \
   -o gpurun_out/layer_full python scripts/layer_time.py 1 > gpurun_out/ncu_full.log 2>&1; echo ncu2=$?
