@@ -817,8 +817,15 @@ e3_status dec_launch_epi(const DecMaps &m, const DecArgs &a, int grid, int csk, 
 
 int dec_tiles(int N, int epi) { return epi == E3_DEC_SWIGLU ? N / 64 : (N + DM - 1) / DM; }
 
+// Stream-K grid: every SM.  E3_DEC_MAXGRID caps it (diagnostics): one whole
+// tile per CTA (Llama-7B QKV, 96 tiles) is faster standalone (30.8 -> 23.0
+// us, scripts/dec_bench.py) and in a graph-replayed split (llama_timeline:
+// 893 -> 859 us per 4 layers) but 0.3 % slower in the LM bench's pipeline
+// (same box, A/B twice), so it is not the default.
 static int dec_grid(int N, int K, int epi, int sms) {
   const long total = (long)dec_tiles(N, epi) * (K / DKS);
+  static const int cap = getenv("E3_DEC_MAXGRID") ? atoi(getenv("E3_DEC_MAXGRID")) : 0;   // diagnostics
+  if (cap > 0 && cap < sms) sms = cap;
   return (int)(total < sms ? total : sms);
 }
 
