@@ -141,6 +141,24 @@ __global__ void __cluster_dims__(2, 1, 1) __launch_bounds__(kLThreads, 1)
           tma_load_2d(sW + stage * CF::kW + s * CF::NSUB * 128, &tmW, &full[stage], kb * LBK, n0 + s * CF::NSUB);
         if (++stage == S) { stage = 0; phase ^= 1; }
       }
+      // The residual tile lands, by TMA, exactly where y1 will be written (the
+      // same 128-byte-swizzled 64-column blocks, over the drained stages):
+      // block b is issued as soon as the last MMA reading any stage region it
+      // overlaps has completed, so most of it arrives during the last k-blocks
+      // instead of one round trip after the mainloop (~2 us, r02 timeline)
+      mbar_expect_tx(rbar, LM * NH * 2);
+      for (int blk = 0; blk < NH / 64; ++blk) {
+        const int lo = blk * LM * 128, hi = lo + LM * 128;
+        int last = -1;                            // latest k-block reading an overlapped region
+        for (int s2 = 0; s2 < S && s2 < nkb; ++s2) {
+          const int alo = s2 * CF::kA, wlo = S * CF::kA + s2 * CF::kW;
+          const bool ov = (lo < alo + CF::kA && hi > alo) || (lo < wlo + CF::kW && hi > wlo);
+          const int kl = s2 + ((nkb - 1 - s2) / S) * S;   // the stage's final k-block
+          if (ov && kl > last) last = kl;
+        }
+        if (last >= 0) mbar_wait(&empty[last % S], (uint32_t)((last / S) & 1));   // no later phase exists
+        tma_load_2d(sY + lo, &tmR, rbar, n0 + blk * 64, m0);
+      }
     }
   } else if (warp == 1) {
     // ------------------------------------------------------------ MMA issuer
@@ -188,19 +206,15 @@ __global__ void __cluster_dims__(2, 1, 1) __launch_bounds__(kLThreads, 1)
   const int m = m0 + row;
   constexpr int HC = NH / NPART;                  // columns per epilogue thread
   float2 sum2 = make_float2(0.f, 0.f), sq2 = make_float2(0.f, 0.f);   // row sum, sum of squares
-  unsigned long long tlA = 0, tlB = 0;
+  unsigned long long tlA = 0, tlB = 0, tlR = 0, tlP = 0, tlX = 0;
   if (epi) {
     mbar_wait(tfull, 0);                          // all MMAs done: the stage buffers are drained
     tc_fence_after();
     tlA = tl_now();
-    // the residual tile lands, by TMA, exactly where y1 will be written
-    // (same 128-byte-swizzled block layout): one round trip for the whole tile
-    if (warp == 4 && lane == 0) {
-      mbar_expect_tx(rbar, LM * NH * 2);
-      for (int blk = 0; blk < NH / 64; ++blk) tma_load_2d(sY + blk * (LM * 128), &tmR, rbar, n0 + blk * 64, m0);
-    }
+    // (the residual tile was issued by the producer as the stages drained)
     epi_bar_n<EW * 32>();                                 // sPar written by every epilogue thread
     mbar_wait(rbar, 0);
+    tlR = tl_now();
     const uint32_t taddr = tmem_base + ((uint32_t)(q * 32) << 16);
 #pragma unroll 1
     for (int c = 0; c < HC; c += 32) {
@@ -238,6 +252,7 @@ __global__ void __cluster_dims__(2, 1, 1) __launch_bounds__(kLThreads, 1)
     // this CTA's (sum, sum of squares) of the row (fixed order: half 0 +
     // half 1) -> both CTAs' slot [rank]; one exchange round (the second
     // moment about 0 is exact enough in fp32 for LayerNorm inputs of O(1))
+    tlP = tl_now();
     xs[h * LM + row] = sum2.x + sum2.y;
     xr2[h * LM + row] = sq2.x + sq2.y;
     epi_bar_n<EW * 32>();
@@ -263,6 +278,7 @@ __global__ void __cluster_dims__(2, 1, 1) __launch_bounds__(kLThreads, 1)
       bulk_commit();
     }
   }
+  tlX = tl_now();
   cluster_sync();                                 // both CTAs' row statistics visible
   if (epi) {
     tlB = tl_now();
@@ -303,6 +319,8 @@ __global__ void __cluster_dims__(2, 1, 1) __launch_bounds__(kLThreads, 1)
       bulk_commit();
       bulk_wait_read<0>();                        // smem read before exit; the global writes complete with the grid
       tl_rec(tlb, 77, tlA, tlB);                  // mainloop done, statistics exchanged, stored
+      tl_rec(tlb, 78, tlR, tlP);                  // residual landed, pass 1 done, (before cluster sync)
+      tl_rec(tlb, 79, tlX, tlX);
     }
   }
   tc_fence_before();

@@ -17,7 +17,7 @@ sys.path.insert(0, ".")
 import e3data  # noqa: E402
 from paper_conf_sosp_iyergdpgn24_b200 import _lib, api  # noqa: E402
 
-NAMES = {77: "O+LN: tfull|stats|stored", 9: "ramp_vit", 91: "vit ramp: ln|cls|end", 3: "layernorm", 4: "ramp(all CTAs)", 5: "ramp decision", 6: "ln_compact", 7: "gemm_ln (O+LN1)", 40: "ramp: cls ready|partials|sync", 41: "decide: synced|computed|tl5", 60: "compact: scan done", 70: "ramp+compact (fused)", 71: "fused: pdl|decided|end", 72: "fused slice: rel|rows|computed", 73: "fused decider start", 74: "ramp2", 75: "ramp2 slice: rel|computed|end", 76: "ramp2 decider: rel|computed|end"}
+NAMES = {77: "O+LN: tfull|stats|stored", 78: "O+LN: resid|pass1|rec", 79: "O+LN: pre-sync|.|rec", 9: "ramp_vit", 91: "vit ramp: ln|cls|end", 3: "layernorm", 4: "ramp(all CTAs)", 5: "ramp decision", 6: "ln_compact", 7: "gemm_ln (O+LN1)", 40: "ramp: cls ready|partials|sync", 41: "decide: synced|computed|tl5", 60: "compact: scan done", 70: "ramp+compact (fused)", 71: "fused: pdl|decided|end", 72: "fused slice: rel|rows|computed", 73: "fused decider start", 74: "ramp2", 75: "ramp2 slice: rel|computed|end", 76: "ramp2 decider: rel|computed|end"}
 
 
 def name(kid):
