@@ -493,7 +493,7 @@ struct Runner {
     const int par = (int)(run_no & 1);
     const int slot = (int)(run_no % kSlots);
     int64_t *const stg_ids = pl->staging_ids + (size_t)par * B;   // read until the run's tail ends
-    cudaStream_t tst = pl->tail_stream;
+    cudaStream_t tst = prof_enabled() ? st : pl->tail_stream;   // profiled step: serial, clean intervals
     if (run_no >= 2)   // run_no - 2's tail still reads the parity buffers this run writes
       E3_CUDA_TRY(cudaStreamWaitEvent(st, pl->ev[(run_no - 2) % kSlots], 0));
     // destination of the survivors first (a send link may have to free a buffer)

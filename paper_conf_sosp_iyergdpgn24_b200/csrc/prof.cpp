@@ -94,6 +94,8 @@ ProfScope::~ProfScope() {
   cudaEventRecord(P.pending[slot].b, st);
 }
 
+bool prof_enabled() { return g_enabled.load() != 0; }
+
 }  // namespace e3
 
 extern "C" {

@@ -21,6 +21,10 @@ enum ProfKind {
 };
 
 void count_launch();
+// per-kernel profiling on (its events bracket each launch; the pipeline then
+// runs a split's tail on the main stream, so no interval includes waiting for
+// SMs held by an overlapping kernel)
+bool prof_enabled();
 // add algorithmic bytes to a kind after the fact (e.g. compaction: n_surv is
 // only known once the run completed)
 void prof_add_bytes(int kind, double bytes);
