@@ -718,7 +718,10 @@ __global__ void __launch_bounds__(kDThreads, 1)
       }
     }
     const unsigned long long tc2 = tl_now();
-    cluster_sync();                     // no CTA leaves while a peer may still read its smem
+    // done reading the peers' smem; the matching wait is just before exit, so
+    // the stores below overlap the barrier (no CTA leaves while a peer may
+    // still read its smem)
+    asm volatile("barrier.cluster.arrive.release.aligned;" ::: "memory");
     if (threadIdx.x == 64) tl_rec(tlb, 8800 + EPI, tc0, tc1);   // CSK tail: before / after sync 1, reduced
     if (threadIdx.x == 64) tl_rec(tlb, 8900 + EPI, tc2, tl_now());   // reduced, after sync 2, (stored: below)
     if (warp >= 2 && warp <= 5 && (EPI == E3_DEC_STORE || EPI == E3_DEC_RESID)) {
@@ -758,6 +761,7 @@ __global__ void __launch_bounds__(kDThreads, 1)
   tc_fence_after();
   if (a.late_trigger) pdl_trigger();
   if (warp == 2) tmem_dealloc(tmem_base, CF::kTmemCols);
+  if (CSK > 1) asm volatile("barrier.cluster.wait.acquire.aligned;" ::: "memory");
 }
 
 }  // namespace
