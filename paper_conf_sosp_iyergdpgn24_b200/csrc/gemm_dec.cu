@@ -127,6 +127,7 @@ __global__ void __launch_bounds__(kDThreads, 1)
 
   const int warp = warp_id(), lane = lane_id();
   const int tiles = (EPI == E3_DEC_SWIGLU) ? a.N / 64 : (a.N + DM - 1) / DM;
+  constexpr bool kCluster = CSK > 1 && EPI != E3_DEC_PARTIAL;
   SK sk;
   sk.nkb = a.K / DKS;
   sk.total = (long)tiles * sk.nkb;
@@ -681,7 +682,18 @@ __global__ void __launch_bounds__(kDThreads, 1)
       tl_rec(tlb, 8000 + EPI, tlf, tlm);
     }
   }
-  if (CSK > 1) {
+  if (EPI == E3_DEC_PARTIAL && warp >= 2 && warp <= 5) {
+    // this CTA's fp32 partial tile -> part_out[k][t][n] (k = its K quarter):
+    // per token a warp writes 32 consecutive features (128 B)
+    const int kq = blockIdx.x % CSK, tile = blockIdx.x / CSK;
+    const int r = (warp & 3) * 32 + lane_id(), n = tile * DM + r;
+    if (n < a.N) {
+      float *po = a.part_out + (size_t)kq * a.T * a.N + n;
+#pragma unroll 8
+      for (int t = 0; t < T; ++t) po[(size_t)t * a.N] = sE[r * (T + 1) + t];
+    }
+  }
+  if (kCluster) {
     constexpr int RPC = DM / CSK;       // rows reduced and stored by this CTA
     const int cr = (int)cluster_ctarank();
     const int tile = blockIdx.x / CSK;
@@ -755,13 +767,13 @@ __global__ void __launch_bounds__(kDThreads, 1)
       }
     }
   }
-  if (CSK > 1 && threadIdx.x == 64) tl_rec(tlb, 8950 + EPI, tl0, tl0);   // CSK tail: stored
+  if (kCluster && threadIdx.x == 64) tl_rec(tlb, 8950 + EPI, tl0, tl0);   // CSK tail: stored
   tc_fence_before();
   __syncthreads();
   tc_fence_after();
   if (a.late_trigger) pdl_trigger();
   if (warp == 2) tmem_dealloc(tmem_base, CF::kTmemCols);
-  if (CSK > 1) asm volatile("barrier.cluster.wait.acquire.aligned;" ::: "memory");
+  if (kCluster) asm volatile("barrier.cluster.wait.acquire.aligned;" ::: "memory");
 }
 
 }  // namespace
@@ -778,7 +790,7 @@ e3_status dec_launch(const DecMaps &m, const DecArgs &a, int grid, cudaStream_t 
     E3_CUDA_TRY(cudaFuncSetAttribute(kern, cudaFuncAttributeMaxDynamicSharedMemorySize, DCfg<T>::kSmem));
     attr_done = true;
   }
-  if (CSK > 1) {
+  if (CSK > 1 && EPI != E3_DEC_PARTIAL) {
     cudaLaunchConfig_t cfg = {};
     cfg.gridDim = dim3(grid);
     cfg.blockDim = dim3(kDThreads);
@@ -812,6 +824,7 @@ e3_status dec_launch_epi(const DecMaps &m, const DecArgs &a, int grid, int csk, 
     case E3_DEC_SWIGLU: return dec_launch<T, E3_DEC_SWIGLU, 1>(m, a, grid, st);
     case E3_DEC_QKV_ROPE: return dec_launch<T, E3_DEC_QKV_ROPE, 1>(m, a, grid, st);
     case E3_DEC_LOGITS: return dec_launch<T, E3_DEC_LOGITS, 1>(m, a, grid, st);
+    case E3_DEC_PARTIAL: return dec_launch<T, E3_DEC_PARTIAL, 4>(m, a, grid, st);
   }
   set_error("bad decode epilogue");
   return E3_EINVAL;
@@ -854,7 +867,13 @@ e3_status dec_tmaps(DecMaps *m, const void *X, int T, int K, const void *W, cons
 // of the SMs (W_o, W_down of Llama-7B: 32 tiles -> 128 CTAs) and the
 // epilogue is a plain / residual store with 16-byte vectors; E3_DEC_STREAMK
 // forces stream-K everywhere (diagnostics)
+bool dec_partial_ok(int N, int K, int sms) {
+  static const bool off = getenv("E3_DEC_NO_PARTIAL") != nullptr;   // diagnostics: cluster split-K + rmsnorm
+  return !off && N % 8 == 0 && 4 * dec_tiles(N, E3_DEC_RESID) <= sms && K / DKS >= 4;
+}
+
 static int dec_csk(const DecArgs &a, int sms) {
+  if (a.epi == E3_DEC_PARTIAL) return 4;
   static const bool off = getenv("E3_DEC_STREAMK") != nullptr;
   if (off || (a.epi != E3_DEC_STORE && a.epi != E3_DEC_RESID)) return 1;
   const int tiles = dec_tiles(a.N, a.epi);

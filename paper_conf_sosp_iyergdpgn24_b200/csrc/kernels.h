@@ -111,7 +111,10 @@ e3_status ramp_compact_run(const RampArgs &a, unsigned *ctr_words, const struct 
 e3_status tl_set_rampc(void *buf);
 
 // ---- K7 decode GEMM (gemm_dec.cu): Y[T,N] = epi(X[T,K] W[N,K]^T), swap-AB tcgen05
-enum { E3_DEC_STORE = 0, E3_DEC_RESID = 1, E3_DEC_SWIGLU = 2, E3_DEC_QKV_ROPE = 3, E3_DEC_LOGITS = 4 };
+// PARTIAL: split-K by 4 (CSK) without a cluster; each CTA writes its fp32
+// partial tile to part_out[k][t][n] and the reduction (+ residual, + the
+// following RMSNorm) is done by reduce_rmsnorm_run
+enum { E3_DEC_STORE = 0, E3_DEC_RESID = 1, E3_DEC_SWIGLU = 2, E3_DEC_QKV_ROPE = 3, E3_DEC_LOGITS = 4, E3_DEC_PARTIAL = 5 };
 struct DecMaps {
   CUtensorMap w;    // W [N,K], box 128 (SWIGLU: 64) x 64, 128-B swizzle
   CUtensorMap w2;   // SWIGLU: W_up, same box
@@ -142,6 +145,7 @@ struct DecArgs {
   int n_slots;              // QKV_ROPE: slots of the cache; slot / pos outside it -> *err, row skipped
   int *err;                 // device error flag (E3_EINVAL reported by the pipeline), may be NULL
   int late_trigger;         // PDL trigger at the end instead of after the dependency wait
+  float *part_out;          // PARTIAL: [4][T][N] fp32 split-K partials
 };
 int dec_tiles(int N, int epi);
 int dec_max_contrib(int N, int K, int epi, int sms);
@@ -151,6 +155,14 @@ e3_status rope_table(int max_ctx, int head_dim, double theta, float2 **out);
 
 // ---- K8 LLaMA decode helpers (llama.cu)
 e3_status rmsnorm_run(const void *x, const void *g, void *y, int rows, int H, float eps, cudaStream_t st);
+// h = bf16((((0 + p0) + p1) + p2) + p3 + resid) from 4 split-K partials
+// [4][rows][H] (the cluster split-K's rank-order sum + RESID epilogue, bit for
+// bit), stored to h_out; then y = RMSNorm(h) * g exactly as rmsnorm_run
+// (g == nullptr: no norm)
+e3_status reduce_rmsnorm_run(const float *part, const void *resid, void *h_out, const void *g, void *y, int rows,
+                             int H, float eps, cudaStream_t st);
+// the split-K-by-4 partial mode is available for this GEMM shape (else RESID + rmsnorm_run)
+bool dec_partial_ok(int N, int K, int sms);
 // ctx[t, h*128 + :] = softmax(q_t,h . K[slot, g(h), 0..pos]^T / sqrt 128) V[...]
 e3_status attn_dec_run(const void *q, void *ctx, const void *kc, const void *vc, const int64_t *ids,
                        const int32_t *n_valid_dev, int n_valid_host, const int32_t *slot_of_id, int64_t id_cap,

@@ -414,6 +414,116 @@ __global__ void __launch_bounds__(256) rmsnorm_cta_kernel(const __nv_bfloat16 *_
   if (threadIdx.x == 0) tl_rec(tlb, 8700, tl0, tl1);
 }
 
+// The split-K-by-4 decode GEMM's reduction + residual epilogue fused with the
+// RMSNorm that follows it (O -> RMSNorm2, down -> the next RMSNorm1 or the LM
+// ramp's final norm): h = bf16((((0 + p0) + p1) + p2) + p3 + r), the same sum
+// order and rounding as the cluster split-K kernel's DSMEM reduction and
+// RESID epilogue, stored; then the rmsnorm_cta_kernel arithmetic on the
+// rounded h.  Replaces the cluster's two barriers, the DSMEM reduction and the
+// separate RMSNorm launch (~6 us per GEMM + norm pair, r02 llama_timeline).
+template <int VPT>
+__global__ void __launch_bounds__(256) reduce_rmsnorm_kernel(const float *__restrict__ part,
+                                                             const __nv_bfloat16 *__restrict__ resid,
+                                                             __nv_bfloat16 *__restrict__ h_out,
+                                                             const __nv_bfloat16 *__restrict__ g,
+                                                             __nv_bfloat16 *__restrict__ y, int rows, int H,
+                                                             float eps) {
+  __shared__ float red[8];
+  const unsigned long long tl0 = tl_now();
+  unsigned long long *const tlb = g_tl;
+  const int row = blockIdx.x, t = threadIdx.x, warp = warp_id(), lane = lane_id();
+  const int nvec = H / 8;
+  const size_t qstride = (size_t)rows * H;
+  uint4 gv[VPT];
+#pragma unroll
+  for (int i = 0; i < VPT; ++i) {
+    const int k = t + 256 * i;
+    gv[i] = (g && k < nvec) ? __ldg(reinterpret_cast<const uint4 *>(g) + k) : make_uint4(0, 0, 0, 0);
+  }
+  pdl_wait();
+  pdl_trigger();
+  const unsigned long long tl1 = tl_now();
+  if (row >= rows) return;
+  uint4 v[VPT];
+  float ss = 0.f;
+#pragma unroll
+  for (int i = 0; i < VPT; ++i) {
+    const int k = t + 256 * i;
+    if (k >= nvec) {
+      v[i] = make_uint4(0, 0, 0, 0);
+      continue;
+    }
+    const float4 *p = reinterpret_cast<const float4 *>(part + (size_t)row * H + 8 * k);
+    float4 a0[4], a1[4];
+#pragma unroll
+    for (int q = 0; q < 4; ++q) {
+      a0[q] = __ldcg(p + q * (qstride / 4));
+      a1[q] = __ldcg(p + q * (qstride / 4) + 1);
+    }
+    const uint4 rv = __ldg(reinterpret_cast<const uint4 *>(resid + (size_t)row * H) + k);
+    float acc[8];
+#pragma unroll
+    for (int e = 0; e < 8; ++e) acc[e] = 0.f;
+#pragma unroll
+    for (int q = 0; q < 4; ++q) {   // rank order
+      acc[0] += a0[q].x; acc[1] += a0[q].y; acc[2] += a0[q].z; acc[3] += a0[q].w;
+      acc[4] += a1[q].x; acc[5] += a1[q].y; acc[6] += a1[q].z; acc[7] += a1[q].w;
+    }
+    const uint32_t rw[4] = {rv.x, rv.y, rv.z, rv.w};
+    uint32_t o[4];
+#pragma unroll
+    for (int e = 0; e < 4; ++e) o[e] = pack_bf16(acc[2 * e] + bf_lo(rw[e]), acc[2 * e + 1] + bf_hi(rw[e]));
+    v[i] = make_uint4(o[0], o[1], o[2], o[3]);
+    reinterpret_cast<uint4 *>(h_out + (size_t)row * H)[k] = v[i];
+#pragma unroll
+    for (int e = 0; e < 4; ++e) ss += bf_lo(o[e]) * bf_lo(o[e]) + bf_hi(o[e]) * bf_hi(o[e]);
+  }
+  if (!g) {
+    if (t == 0) tl_rec(tlb, 8710, tl0, tl1);
+    return;
+  }
+#pragma unroll
+  for (int o = 16; o; o >>= 1) ss += __shfl_xor_sync(0xffffffffu, ss, o);
+  if (lane == 0) red[warp] = ss;
+  __syncthreads();
+  float tot = red[0];
+#pragma unroll
+  for (int w = 1; w < 8; ++w) tot += red[w];
+  const float rinv = 1.0f / sqrtf(tot / (float)H + eps);
+  uint4 *yr = reinterpret_cast<uint4 *>(y + (size_t)row * H);
+#pragma unroll
+  for (int i = 0; i < VPT; ++i) {
+    const int k = t + 256 * i;
+    if (k >= nvec) continue;
+    const uint32_t w[4] = {v[i].x, v[i].y, v[i].z, v[i].w};
+    const uint32_t gw[4] = {gv[i].x, gv[i].y, gv[i].z, gv[i].w};
+    uint32_t o[4];
+#pragma unroll
+    for (int e = 0; e < 4; ++e)
+      o[e] = pack_bf16(bf_lo(w[e]) * rinv * bf_lo(gw[e]), bf_hi(w[e]) * rinv * bf_hi(gw[e]));
+    yr[k] = make_uint4(o[0], o[1], o[2], o[3]);
+  }
+  if (t == 0) tl_rec(tlb, 8710, tl0, tl1);
+}
+
+e3_status reduce_rmsnorm_run(const float *part, const void *resid, void *h_out, const void *g, void *y, int rows,
+                             int H, float eps, cudaStream_t st) {
+  if (H % 8 || H > 8192 || (g && !y)) {
+    set_error("reduce_rmsnorm: need H % 8 == 0, H <= 8192");
+    return E3_EUNSUPPORTED;
+  }
+  auto *rp = reinterpret_cast<const __nv_bfloat16 *>(resid);
+  auto *hp = reinterpret_cast<__nv_bfloat16 *>(h_out);
+  auto *gp = reinterpret_cast<const __nv_bfloat16 *>(g);
+  auto *yp = reinterpret_cast<__nv_bfloat16 *>(y);
+  const int vpt = (H / 8 + 255) / 256;
+  if (vpt <= 2) E3_CUDA_TRY(launch_k(reduce_rmsnorm_kernel<2>, dim3(rows), dim3(256), 0, st, part, rp, hp, gp, yp, rows, H, eps));
+  else E3_CUDA_TRY(launch_k(reduce_rmsnorm_kernel<4>, dim3(rows), dim3(256), 0, st, part, rp, hp, gp, yp, rows, H, eps));
+  E3_CUDA_TRY(cudaGetLastError());
+  count_launch();
+  return E3_OK;
+}
+
 e3_status rmsnorm_run(const void *x, const void *g, void *y, int rows, int H, float eps, cudaStream_t st) {
   if (H % 8 || H > 8192) {
     set_error("rmsnorm: need H % 8 == 0, H <= 8192");

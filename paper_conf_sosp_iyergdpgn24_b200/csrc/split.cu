@@ -258,6 +258,7 @@ static e3_status llama_create(e3_split *s, const e3_weights *w) {
   need(F, s->mc_gu, E3_DEC_SWIGLU);
   need(H, s->mc_down, E3_DEC_RESID);
   need(V, s->mc_lm, E3_DEC_LOGITS);
+  if ((size_t)4 * B * H > part) part = (size_t)4 * B * H;   // split-K-by-4 partials (E3_DEC_PARTIAL), reused
   e3_status st = ws.ensure_llama(V, part, tickets, w->kv->max_ctx, 128, 10000.0);
   if (st != E3_OK) return st;
   const int nl = d.layer_end - d.layer_begin;
@@ -401,15 +402,24 @@ static e3_status llama_run(e3_split *s, cudaStream_t st, const void *x_in, const
   base.T = B;
   base.part = ws.dec_part;
   base.tickets = ws.dec_tickets;
+  // O and down as split-K-by-4 partials reduced by the RMSNorm that follows
+  // (reduce_rmsnorm_run), where the cluster split-K would run and the
+  // following norm is the one-CTA-per-row kernel (bitwise the same results)
+  const bool cta_norm = H >= 2048 && B <= 256;
+  const bool fuse_o = cta_norm && dec_partial_ok(H, H, s->sms);
+  const bool fuse_down = cta_norm && dec_partial_ok(H, F, s->sms);
+  bool n1_ready = false;     // ws.x1 already holds this layer's RMSNorm1 (fused into the previous down)
+  bool rnorm_ready = false;  // ws.x1 already holds the ramp's final norm of this layer's output
   for (int i = 0; i < nl; ++i) {
     const int l = d.layer_begin + i;
     const e3_layer_weights &L = s->L[i];
     auto &m = s->dmaps[i];
     void *out = (i % 2 == 0) ? ws.xa : ws.xb;
-    {
+    if (!n1_ready) {
       ProfScope ps(PK_LN, st, 0, nv * H * 2 * b2);
       E3_RUN(rmsnorm_run(cur, L.ln1_g, ws.x1, B, H, d.norm_eps, st));
     }
+    n1_ready = false;
     {
       DecArgs a = base;
       a.N = nqkv;
@@ -449,7 +459,8 @@ static e3_status llama_run(e3_split *s, cudaStream_t st, const void *x_in, const
       a.N = H;
       a.K = H;
       a.max_contrib = s->mc_o;
-      a.epi = E3_DEC_RESID;
+      a.epi = fuse_o ? E3_DEC_PARTIAL : E3_DEC_RESID;
+      a.part_out = ws.dec_part;
       a.R = reinterpret_cast<const __nv_bfloat16 *>(cur);
       a.Y = reinterpret_cast<__nv_bfloat16 *>(ws.y);
       a.ldo = H;
@@ -458,7 +469,8 @@ static e3_status llama_run(e3_split *s, cudaStream_t st, const void *x_in, const
     }
     {
       ProfScope ps(PK_LN, st, 0, nv * H * 2 * b2);
-      E3_RUN(rmsnorm_run(ws.y, L.ln2_g, ws.x1, B, H, d.norm_eps, st));
+      if (fuse_o) E3_RUN(reduce_rmsnorm_run(ws.dec_part, cur, ws.y, L.ln2_g, ws.x1, B, H, d.norm_eps, st));
+      else E3_RUN(rmsnorm_run(ws.y, L.ln2_g, ws.x1, B, H, d.norm_eps, st));
     }
     {
       DecArgs a = base;
@@ -476,19 +488,38 @@ static e3_status llama_run(e3_split *s, cudaStream_t st, const void *x_in, const
       a.N = H;
       a.K = F;
       a.max_contrib = s->mc_down;
-      a.epi = E3_DEC_RESID;
+      a.epi = fuse_down ? E3_DEC_PARTIAL : E3_DEC_RESID;
+      a.part_out = ws.dec_part;
       a.R = reinterpret_cast<const __nv_bfloat16 *>(ws.y);
       a.Y = reinterpret_cast<__nv_bfloat16 *>(out);
       a.ldo = H;
       ProfScope ps(PK_GEMM_FFN2, st, 0, (double)F * H * b2 + nv * (F + 2 * H) * b2);
       E3_RUN(dec_run(m.down, a, s->sms, st));
     }
+    if (fuse_down) {
+      // the first norm that reads this layer's output: the ramp's final norm
+      // (an evaluated ramp after layer l), else the next layer's RMSNorm1
+      const void *g = nullptr;
+      for (int rj = ri; rj < d.n_ramps && d.ramp_layer[rj] == l; ++rj)
+        if (rj == d.n_ramps - 1 || d.inner == E3_INNER_EXACT) {
+          g = s->R[rj].ln_g;
+          rnorm_ready = true;
+          break;
+        }
+      if (!g && i + 1 < nl) {
+        g = s->L[i + 1].ln1_g;
+        n1_ready = true;
+      }
+      ProfScope ps(PK_LN, st, 0, nv * H * 2 * b2);
+      E3_RUN(reduce_rmsnorm_run(ws.dec_part, ws.y, out, g, ws.x1, B, H, d.norm_eps, st));
+    }
     cur = out;
     while (ri < d.n_ramps && d.ramp_layer[ri] == l) {
       const bool last = (ri == d.n_ramps - 1);
       if (last || d.inner == E3_INNER_EXACT) {
         ProfScope ps(PK_RAMP, st, 0, (double)V * H * b2 + nv * (H * b2 + V * 4.0));
-        E3_RUN(rmsnorm_run(cur, s->R[ri].ln_g, ws.x1, B, H, d.norm_eps, st));
+        if (!rnorm_ready) E3_RUN(rmsnorm_run(cur, s->R[ri].ln_g, ws.x1, B, H, d.norm_eps, st));
+        rnorm_ready = false;
         DecArgs a = base;
         a.N = V;
         a.K = H;

@@ -60,10 +60,10 @@ n = min(int(b[0]), 32768)
 r = b[1:1 + 4 * n].reshape(n, 4)
 kid = (r[:, 0] & 0xFFFF).astype(int)
 t = r[:, 1:].astype(np.float64)
-keep = (kid == 8600) | (kid == 8700) | ((kid >= 8100) & (kid < 8200))
+keep = (kid == 8600) | (kid == 8700) | (kid == 8710) | ((kid >= 8100) & (kid < 8200))
 kid, t = kid[keep], t[keep]
 t = (t - t.min()) / 1000.0
-NAMES = {8600: "attn_dec", 8700: "rmsnorm", 8100: "gemm STORE", 8101: "gemm RESID (O/down)", 8102: "gemm SWIGLU",
+NAMES = {8600: "attn_dec", 8700: "rmsnorm", 8710: "reduce+rmsnorm", 8105: "gemm PARTIAL (O/down)", 8100: "gemm STORE", 8101: "gemm RESID (O/down)", 8102: "gemm SWIGLU",
          8103: "gemm QKV+RoPE", 8104: "gemm LM head"}
 inst = []
 for k in np.unique(kid):
