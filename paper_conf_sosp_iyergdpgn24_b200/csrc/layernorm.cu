@@ -33,19 +33,38 @@ __global__ void __launch_bounds__(256)
   pdl_trigger();
   const unsigned long long tl1 = tl_now();
   // persistent: the grid is at most one wave; each warp walks its rows RPW at
-  // a time (loads of a batch first)
-  for (int base = row0; base < rows; base += RPW * warps) {
+  // a time (loads of a batch first).  RPW == 1: the next row's loads are
+  // issued before the current row is normalised (VT, H = 768: 3.37 -> 4.16
+  // TB/s, VT 37.7 -> 38.2 k inputs/s; at H = 1024 two rows per warp without
+  // the prefetch stay ahead: 3.36 vs 3.22 TB/s)
+  const int stride = RPW * warps;
+  if (RPW == 1) {
+    uint4 w[VPL];
+    int base = row0;
+    if (base < rows) ln_load_row<VPL>(v[0], x + (size_t)base * H, H, lane);
+    while (base < rows) {
+      const int nb = base + stride;
+      if (nb < rows) ln_load_row<VPL>(w, x + (size_t)nb * H, H, lane);
+      ln_apply<VPL>(v[0], p, H, eps, lane);
+      ln_store_row<VPL>(v[0], y + (size_t)base * H, H, lane);
 #pragma unroll
-    for (int j = 0; j < RPW; ++j) {
-      const int row = base + j * warps;
-      if (row < rows) ln_load_row<VPL>(v[j], x + (size_t)row * H, H, lane);
+      for (int i = 0; i < VPL; ++i) v[0][i] = w[i];
+      base = nb;
     }
+  } else {
+    for (int base = row0; base < rows; base += stride) {
 #pragma unroll
-    for (int j = 0; j < RPW; ++j) {
-      const int row = base + j * warps;
-      if (row < rows) {
-        ln_apply<VPL>(v[j], p, H, eps, lane);
-        ln_store_row<VPL>(v[j], y + (size_t)row * H, H, lane);
+      for (int j = 0; j < RPW; ++j) {
+        const int row = base + j * warps;
+        if (row < rows) ln_load_row<VPL>(v[j], x + (size_t)row * H, H, lane);
+      }
+#pragma unroll
+      for (int j = 0; j < RPW; ++j) {
+        const int row = base + j * warps;
+        if (row < rows) {
+          ln_apply<VPL>(v[j], p, H, eps, lane);
+          ln_store_row<VPL>(v[j], y + (size_t)row * H, H, lane);
+        }
       }
     }
   }
@@ -71,7 +90,9 @@ e3_status layernorm_run(const void *x, const void *g, const void *b, void *y, in
     set_error("LayerNorm: H > 4096 unsupported");
     return E3_EUNSUPPORTED;
   }
-  const bool two = rows > 8 * 4 * sms && H <= 1024;   // registers: 2 rows of <= 4 vectors per lane
+  // rows per warp: 1 with the next row prefetched up to H = 768, else 2
+  // when one row per warp would exceed one wave of resident CTAs
+  const bool two = rows > 8 * 4 * sms && H <= 1024 && H > 768;   // registers: 2 rows of <= 4 vectors per lane
   using Kern = void (*)(const __nv_bfloat16 *, const __nv_bfloat16 *, const __nv_bfloat16 *, __nv_bfloat16 *, int,
                         int, float);
   const int vi = vpl <= 1 ? 0 : vpl <= 3 ? 1 : vpl <= 4 ? 2 : vpl <= 8 ? 3 : 4;
