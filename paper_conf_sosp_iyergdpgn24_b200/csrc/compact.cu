@@ -257,23 +257,64 @@ __global__ void __launch_bounds__(kThreads, VPL <= 3 ? 2 : 1)
       }
     }
   }
-  for (int u0 = blockIdx.x * (kThreads / 32) + warp; !spec && u0 < units; u0 += kRowsInFlight * stride) {
+  // gather by destination, software-pipelined: the rows are walked in
+  // batches of kRowsInFlight / 2 and the next batch's loads are issued before
+  // the current batch is normalised and stored, so every warp always has
+  // loads in flight (VT, 50 k token rows per run: the load -> store -> load
+  // rhythm of whole batches left the HBM idle between them)
+  if (!spec && kLn) {   // LayerNorm-ing gathers: batches of kRowsInFlight (the pipelined form spills here)
+    for (int u0 = blockIdx.x * (kThreads / 32) + warp; u0 < units; u0 += kRowsInFlight * stride) {
 #pragma unroll
-    for (int j = 0; j < kRowsInFlight; ++j) {
-      const int u = u0 + j * stride;
-      if (u < units) {
-        const int k = u / S, t = u - k * S;
-        ln_load_row<VPL>(v[j], y + (size_t)src_of[k] * row_elems + (size_t)t * H, H, lane);
+      for (int j = 0; j < kRowsInFlight; ++j) {
+        const int u = u0 + j * stride;
+        if (u < units) {
+          const int k = u / S, t = u - k * S;
+          ln_load_row<VPL>(v[j], y + (size_t)src_of[k] * row_elems + (size_t)t * H, H, lane);
+        }
+      }
+#pragma unroll
+      for (int j = 0; j < kRowsInFlight; ++j) {
+        const int u = u0 + j * stride;
+        if (u < units) {
+          const int k = u / S, t = u - k * S;
+          ln_apply<VPL>(v[j], p, H, eps, lane);
+          ln_store_row<VPL>(v[j], ring + ((tail + k) % dst.cap) * row_elems + (size_t)t * H, H, lane);
+        }
       }
     }
+  } else if (!spec) {
+    constexpr int HB = kRowsInFlight / 2;
+    auto load_batch = [&](int u0, int half) {
 #pragma unroll
-    for (int j = 0; j < kRowsInFlight; ++j) {
-      const int u = u0 + j * stride;
-      if (u < units) {
-        const int k = u / S, t = u - k * S;
-        if (kLn) ln_apply<VPL>(v[j], p, H, eps, lane);
-        ln_store_row<VPL>(v[j], ring + ((tail + k) % dst.cap) * row_elems + (size_t)t * H, H, lane);
+      for (int j = 0; j < HB; ++j) {
+        const int u = u0 + j * stride;
+        if (u < units) {
+          const int k = u / S, t = u - k * S;
+          ln_load_row<VPL>(v[half * HB + j], y + (size_t)src_of[k] * row_elems + (size_t)t * H, H, lane);
+        }
       }
+    };
+    auto store_batch = [&](int u0, int half) {
+#pragma unroll
+      for (int j = 0; j < HB; ++j) {
+        const int u = u0 + j * stride;
+        if (u < units) {
+          const int k = u / S, t = u - k * S;
+          if (kLn) ln_apply<VPL>(v[half * HB + j], p, H, eps, lane);
+          ln_store_row<VPL>(v[half * HB + j], ring + ((tail + k) % dst.cap) * row_elems + (size_t)t * H, H, lane);
+        }
+      }
+    };
+    int u0 = blockIdx.x * (kThreads / 32) + warp;
+    if (u0 < units) load_batch(u0, 0);
+    while (u0 < units) {   // two batches per trip: the register halves stay compile-time indices
+      if (u0 + HB * stride < units) load_batch(u0 + HB * stride, 1);
+      store_batch(u0, 0);
+      u0 += HB * stride;
+      if (u0 >= units) break;
+      if (u0 + HB * stride < units) load_batch(u0 + HB * stride, 0);
+      store_batch(u0, 1);
+      u0 += HB * stride;
     }
   }
   if (blockIdx.x == 0)
