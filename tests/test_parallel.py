@@ -85,7 +85,7 @@ def _run(bounds, replicas):
     procs = [ctx.Process(target=_worker, args=(r, world, port, bounds, replicas, q)) for r in range(world)]
     for p in procs:
         p.start()
-    res = q.get(timeout=120)
+    res = q.get(timeout=600)
     for p in procs:
         p.join(timeout=60)
         assert p.exitcode == 0
