@@ -276,6 +276,18 @@ __device__ __forceinline__ void tma_load_2d_2sm(void *dst, const CUtensorMap *m,
       "l"(reinterpret_cast<uint64_t>(m)), "r"(mbar_cluster), "r"(c0), "r"(c1)
       : "memory");
 }
+// 2-SM TMA multicast: the box lands at the same smem offset in every CTA of
+// cta_mask; each destination's completion bytes go to the barrier at this
+// offset in the LEADER of the destination's pair (peer bit of the address
+// cleared, as the sm_100 2-SM multicast form requires)
+__device__ __forceinline__ void tma_load_2d_2sm_mc(void *dst, const CUtensorMap *m, uint32_t mbar_local, int c0,
+                                                   int c1, uint16_t cta_mask) {
+  asm volatile(
+      "cp.async.bulk.tensor.2d.cta_group::2.shared::cluster.global.mbarrier::complete_tx::bytes.multicast::cluster"
+      " [%0], [%1, {%3, %4}], [%2], %5;" ::"r"(smem_u32(dst)),
+      "l"(reinterpret_cast<uint64_t>(m)), "r"(mbar_local & 0xFEFFFFFFu), "r"(c0), "r"(c1), "h"(cta_mask)
+      : "memory");
+}
 __device__ __forceinline__ void tmem_alloc2(uint32_t *dst_smem, uint32_t ncols) {
   asm volatile("tcgen05.alloc.cta_group::2.sync.aligned.shared::cta.b32 [%0], %1;" ::"r"(smem_u32(dst_smem)),
                "r"(ncols)

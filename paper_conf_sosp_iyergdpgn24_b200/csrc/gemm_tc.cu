@@ -93,8 +93,17 @@ struct Cfg {
 // 64-byte swizzle of a [32 rows x 64 B] box: 16-byte chunk j of row r
 __device__ __forceinline__ uint32_t sw64(int r, int j) { return r * 64 + ((j ^ ((r >> 1) & 3)) << 4); }
 
-template <int BN, int EPI>
-__global__ void __cluster_dims__(2, 1, 1) __launch_bounds__(Cfg<BN, EPI>::kThreads, 1)
+// MC (GEMM_MC_*): with multicast the cluster is two CTA pairs (ranks 0-1 and
+// 2-3) walking 2-tile units in lockstep; the operand they share is loaded
+// half by each pair and multicast to the same smem offset in both, so each
+// CTA fetches (128 + BN/2) - 64 (A shared) or - BN/4 (W shared) rows per K
+// element instead of 128 + BN/2 (ncu: 385 MB of L2 traffic per BB FFN1 at
+// 31 % of the lts peak; cuBLAS's 2x2-cluster kernel moves 242 MB in the same
+// time).  A stage is freed only when BOTH pairs' MMAs have read it (empty
+// barriers count two commits, multicast to all four CTAs).  Off by default
+// (E3_GEMM_MC): same results bit for bit, no faster (gemm_pick_bn).
+template <int BN, int EPI, int MC>
+__global__ void __cluster_dims__(MC ? 4 : 2, 1, 1) __launch_bounds__(Cfg<BN, EPI>::kThreads, 1)
     gemm_bf16_tc_kernel(const __grid_constant__ CUtensorMap tmA, const __grid_constant__ CUtensorMap tmB,
                         const __grid_constant__ CUtensorMap tmC, const __nv_bfloat16 *__restrict__ bias,
                         const __nv_bfloat16 *__restrict__ R, int M, int N, int K) {
@@ -118,13 +127,22 @@ __global__ void __cluster_dims__(2, 1, 1) __launch_bounds__(Cfg<BN, EPI>::kThrea
 
   const int warp = warp_id();
   const int lane = lane_id();
+  constexpr int CL = MC ? 4 : 2;                 // CTAs per cluster
   const uint32_t rank = cluster_ctarank();
-  const bool leader = rank == 0;
-  const int pair = blockIdx.x >> 1;
-  const int num_pairs = gridDim.x >> 1;
+  const uint32_t rp = rank & 1;                  // rank within the pair
+  const int pi = (int)(rank >> 1);               // pair within the cluster
+  const bool leader = rp == 0;
+  const uint32_t lead_rank = rank & ~1u;
+  const int pair = blockIdx.x / CL;              // cluster index (one pair per cluster without MC)
+  const int num_pairs = gridDim.x / CL;
   const int num_m = (M + 2 * BM - 1) / (2 * BM);
   const int num_n = N / BN;
-  const int num_tiles = num_m * num_n;
+  // work units: one pair tile (MC == 0) or two neighbouring tiles, one per pair
+  const int num_tiles = MC == GEMM_MC_A ? num_m * (num_n / 2) : MC == GEMM_MC_B ? ((num_m + 1) / 2) * num_n
+                                                                               : num_m * num_n;
+  auto tile_m = [&](int t) { return MC == GEMM_MC_A ? t / (num_n / 2) : MC == GEMM_MC_B ? 2 * (t / num_n) + pi : t / num_n; };
+  auto tile_n = [&](int t) { return MC == GEMM_MC_A ? 2 * (t % (num_n / 2)) + pi : t % num_n; };
+  const uint16_t mc_mask = (uint16_t)((1u << rp) | (1u << (rp + 2)));   // this CTA's twin in the other pair
   const int num_kb = K / (BK * CF::kKsub);
 
   if (warp == 0 && lane == 0) {
@@ -135,7 +153,7 @@ __global__ void __cluster_dims__(2, 1, 1) __launch_bounds__(Cfg<BN, EPI>::kThrea
   if (warp == 1 && lane == 0) {
     for (int i = 0; i < S; ++i) {
       mbar_init(&full[i], 1);      // leader's arrive.expect_tx (bytes of both CTAs)
-      mbar_init(&empty[i], 1);     // multicast tcgen05.commit
+      mbar_init(&empty[i], MC ? 2 : 1);   // multicast tcgen05.commit of each pair's leader
     }
     for (int i = 0; i < 2; ++i) {
       mbar_init(&tfull[i], 1);     // multicast tcgen05.commit
@@ -163,14 +181,19 @@ __global__ void __cluster_dims__(2, 1, 1) __launch_bounds__(Cfg<BN, EPI>::kThrea
       // W rows of CTA r for MMA m: [n0 + m * BN / kNMma + r * kBox, + kBox),
       // so that D's columns map linearly onto the tile's N range
       auto load_w = [&](int st, int t, int kb) {
-        const uint32_t fb = mapa_shared(smem_u32(&full[st]), 0);
+        const uint32_t fb = mapa_shared(smem_u32(&full[st]), lead_rank);
 #pragma unroll
         for (int ks = 0; ks < CF::kKsub; ++ks)
 #pragma unroll
-          for (int m = 0; m < CF::kNMma; ++m)
-            tma_load_2d_2sm(sB + st * CF::kBBytes + ks * CF::kBSub + m * CF::kBox * 128, &tmB, fb,
-                            (kb * CF::kKsub + ks) * BK,
-                            (t % num_n) * BN + m * (BN / CF::kNMma) + (int)rank * CF::kBox);
+          for (int m = 0; m < CF::kNMma; ++m) {
+            const int wrow = tile_n(t) * BN + m * (BN / CF::kNMma) + (int)rp * CF::kBox;
+            uint8_t *dst = sB + st * CF::kBBytes + ks * CF::kBSub + m * CF::kBox * 128;
+            if (MC == GEMM_MC_B)   // half of the box from each pair, multicast to both
+              tma_load_2d_2sm_mc(dst + pi * (CF::kBox / 2) * 128, &tmB, smem_u32(&full[st]),
+                                 (kb * CF::kKsub + ks) * BK, wrow + pi * (CF::kBox / 2), mc_mask);
+            else
+              tma_load_2d_2sm(dst, &tmB, fb, (kb * CF::kKsub + ks) * BK, wrow);
+          }
       };
       int npre = 0;
       for (int t = pair; t < num_tiles && npre < S; t += num_pairs) {
@@ -184,18 +207,23 @@ __global__ void __cluster_dims__(2, 1, 1) __launch_bounds__(Cfg<BN, EPI>::kThrea
       int stage = 0, it = 0;
       uint32_t phase = 0;
       for (int t = pair; t < num_tiles; t += num_pairs) {
-        const int m_blk = t / num_n;
-        const int am = m_blk * 2 * BM + (int)rank * BM;
+        const int m_blk = tile_m(t);
+        const int am = m_blk * 2 * BM + (int)rp * BM;
         for (int kb = 0; kb < num_kb; ++kb, ++it) {
-          const uint32_t fb = mapa_shared(smem_u32(&full[stage]), 0);
+          const uint32_t fb = mapa_shared(smem_u32(&full[stage]), lead_rank);
           const bool pre = it < npre;
           if (!pre) {
             mbar_wait(&empty[stage], phase ^ 1);
             if (leader) mbar_expect_tx(&full[stage], 2 * CF::kStageBytes);
           }
 #pragma unroll
-          for (int ks = 0; ks < CF::kKsub; ++ks)
-            tma_load_2d_2sm(sA + stage * CF::kABytes + ks * CF::kASub, &tmA, fb, (kb * CF::kKsub + ks) * BK, am);
+          for (int ks = 0; ks < CF::kKsub; ++ks) {
+            if (MC == GEMM_MC_A)   // rows [64 pi, +64) of the block from this pair, multicast to both
+              tma_load_2d_2sm_mc(sA + stage * CF::kABytes + ks * CF::kASub + pi * (BM / 2) * 128, &tmA,
+                                 smem_u32(&full[stage]), (kb * CF::kKsub + ks) * BK, am + pi * (BM / 2), mc_mask);
+            else
+              tma_load_2d_2sm(sA + stage * CF::kABytes + ks * CF::kASub, &tmA, fb, (kb * CF::kKsub + ks) * BK, am);
+          }
           if (!pre) load_w(stage, t, kb);
           if (++stage == S) { stage = 0; phase ^= 1; }
         }
@@ -234,10 +262,10 @@ __global__ void __cluster_dims__(2, 1, 1) __launch_bounds__(Cfg<BN, EPI>::kThrea
                             (kb | ks | k) != 0);
             }
           }
-          tc_commit2_mc(&empty[stage], 0x3);
+          tc_commit2_mc(&empty[stage], MC ? 0xF : 0x3);   // both pairs' stages (MC: they share it)
           if (++stage == S) { stage = 0; phase ^= 1; }
         }
-        tc_commit2_mc(&tfull[acc], 0x3);
+        tc_commit2_mc(&tfull[acc], (uint16_t)(0x3u << (2 * pi)));
         trace(tl, 1);
         if (++acc == CF::kNAcc) { acc = 0; acc_phase ^= 1; }
       }
@@ -248,15 +276,15 @@ __global__ void __cluster_dims__(2, 1, 1) __launch_bounds__(Cfg<BN, EPI>::kThrea
     const int q = warp & 3;              // TMEM lane quarter this warp may access
     const int part = (warp - 4) >> 2;    // which CW-column part of the tile
     uint8_t *ebuf = sE + (warp - 4) * 2 * kEpiBuf;
-    const uint32_t tempty_leader0 = mapa_shared(smem_u32(&tempty[0]), 0);
-    const uint32_t tempty_leader1 = mapa_shared(smem_u32(&tempty[1]), 0);
+    const uint32_t tempty_leader0 = mapa_shared(smem_u32(&tempty[0]), lead_rank);
+    const uint32_t tempty_leader1 = mapa_shared(smem_u32(&tempty[1]), lead_rank);
     int acc = 0;
     uint32_t acc_phase = 0;
     int ci = 0;                          // chunk counter (selects the staging buffer)
     int tl = 0;
     for (int t = pair; t < num_tiles; t += num_pairs, ++tl) {
-      const int m_blk = t / num_n, n_blk = t % num_n;
-      const int m0 = m_blk * 2 * BM + (int)rank * BM + q * 32;   // this warp's first row
+      const int m_blk = tile_m(t), n_blk = tile_n(t);
+      const int m0 = m_blk * 2 * BM + (int)rp * BM + q * 32;     // this warp's first row
       const int m = m0 + lane;
       const int nw0 = n_blk * BN + part * CW;                     // this warp's first column
       const uint32_t taddr = tmem_base + ((uint32_t)(q * 32) << 16) + acc * BN + part * CW;
@@ -366,39 +394,63 @@ __global__ void __cluster_dims__(2, 1, 1) __launch_bounds__(Cfg<BN, EPI>::kThrea
   if (threadIdx.x == 0) tl_rec(tlb, 1000 + BN + EPI, tl0, tl1);
 }
 
-template <int BN, int EPI>
+template <int BN, int EPI, int MC>
 e3_status launch(const GemmMaps &g, const __nv_bfloat16 *bias, const __nv_bfloat16 *R, int M, int N, int K, int sms,
                  cudaStream_t st) {
-  auto kern = gemm_bf16_tc_kernel<BN, EPI>;
+  auto kern = gemm_bf16_tc_kernel<BN, EPI, MC>;
   using CF = Cfg<BN, EPI>;
-  static bool attr_done = false;   // per instantiation
-  if (!attr_done) {
+  constexpr int CL = MC ? 4 : 2;
+  static int max_clusters = 0;     // per instantiation: clusters of CL CTAs resident at once
+  if (!max_clusters) {
     E3_CUDA_TRY(cudaFuncSetAttribute(kern, cudaFuncAttributeMaxDynamicSharedMemorySize, CF::kSmem));
-    attr_done = true;
+    cudaLaunchConfig_t cfg = {};
+    cfg.gridDim = dim3(CL * 64);
+    cfg.blockDim = dim3(CF::kThreads);
+    cfg.dynamicSmemBytes = CF::kSmem;
+    int n = 0;
+    if (cudaOccupancyMaxActiveClusters(&n, kern, &cfg) != cudaSuccess || n <= 0) {
+      cudaGetLastError();
+      n = sms / CL;
+    }
+    max_clusters = n < sms / CL ? n : sms / CL;
   }
-  const int tiles = ((M + 2 * BM - 1) / (2 * BM)) * (N / BN);
-  const int pairs = tiles < sms / 2 ? tiles : sms / 2;
-  E3_CUDA_TRY(launch_k(kern, dim3(2 * pairs), dim3(CF::kThreads), CF::kSmem, st, g.a, g.b, g.c, bias, R, M, N, K));
+  const int num_m = (M + 2 * BM - 1) / (2 * BM), num_n = N / BN;
+  const int units = MC == GEMM_MC_A ? num_m * (num_n / 2) : MC == GEMM_MC_B ? ((num_m + 1) / 2) * num_n : num_m * num_n;
+  const int clusters = units < max_clusters ? units : max_clusters;
+  E3_CUDA_TRY(launch_k(kern, dim3(CL * clusters), dim3(CF::kThreads), CF::kSmem, st, g.a, g.b, g.c, bias, R, M, N, K));
   E3_CUDA_TRY(cudaGetLastError());
   count_launch();
   return E3_OK;
 }
 
-template <int BN>
+template <int BN, int MC>
 e3_status launch_epi(int epi, const GemmMaps &g, const __nv_bfloat16 *bias, const __nv_bfloat16 *R, int M, int N,
                      int K, int sms, cudaStream_t st) {
   if (BN > 256) {   // 384: bias / residual epilogues only
-    if (epi == E3_EPI_BIAS) return launch<(BN > 256 ? BN : 384), E3_EPI_BIAS>(g, bias, R, M, N, K, sms, st);
-    if (epi == E3_EPI_BIAS_RESID) return launch<(BN > 256 ? BN : 384), E3_EPI_BIAS_RESID>(g, bias, R, M, N, K, sms, st);
+    if (epi == E3_EPI_BIAS) return launch<(BN > 256 ? BN : 384), E3_EPI_BIAS, MC>(g, bias, R, M, N, K, sms, st);
+    if (epi == E3_EPI_BIAS_RESID)
+      return launch<(BN > 256 ? BN : 384), E3_EPI_BIAS_RESID, MC>(g, bias, R, M, N, K, sms, st);
     set_error("GEMM: N tile 384 has no GELU epilogue");
     return E3_EUNSUPPORTED;
   }
   switch (epi) {
-    case E3_EPI_BIAS: return launch<BN, E3_EPI_BIAS>(g, bias, R, M, N, K, sms, st);
-    case E3_EPI_BIAS_GELU: return launch<BN, E3_EPI_BIAS_GELU>(g, bias, R, M, N, K, sms, st);
-    case E3_EPI_BIAS_RESID: return launch<BN, E3_EPI_BIAS_RESID>(g, bias, R, M, N, K, sms, st);
+    case E3_EPI_BIAS: return launch<BN, E3_EPI_BIAS, MC>(g, bias, R, M, N, K, sms, st);
+    case E3_EPI_BIAS_GELU: return launch<BN, E3_EPI_BIAS_GELU, MC>(g, bias, R, M, N, K, sms, st);
+    case E3_EPI_BIAS_RESID: return launch<BN, E3_EPI_BIAS_RESID, MC>(g, bias, R, M, N, K, sms, st);
   }
   set_error("bad epilogue");
+  return E3_EINVAL;
+}
+
+template <int BN>
+e3_status launch_mc(int mc, int epi, const GemmMaps &g, const __nv_bfloat16 *bias, const __nv_bfloat16 *R, int M,
+                    int N, int K, int sms, cudaStream_t st) {
+  switch (mc) {
+    case GEMM_MC_NONE: return launch_epi<BN, GEMM_MC_NONE>(epi, g, bias, R, M, N, K, sms, st);
+    case GEMM_MC_A: return launch_epi<BN, GEMM_MC_A>(epi, g, bias, R, M, N, K, sms, st);
+    case GEMM_MC_B: return launch_epi<BN, GEMM_MC_B>(epi, g, bias, R, M, N, K, sms, st);
+  }
+  set_error("bad GEMM multicast mode");
   return E3_EINVAL;
 }
 
@@ -412,15 +464,22 @@ e3_status gemm_set_trace(void *buf) {
 }
 
 int gemm_pick_bn(int M, int N, int K, int sms, int epi) {
-  // diagnostics: E3_GEMM_BN forces the N tile where it divides N
+  // diagnostics: E3_GEMM_BN forces the N tile where it divides N, E3_GEMM_MC
+  // the multicast mode (0 none, 1 A, 2 W) where it applies
   static const int forced = [] {
     const char *e = getenv("E3_GEMM_BN");
     return e ? atoi(e) : 0;
   }();
-  if (forced && N % forced == 0) return forced;
+  static const int forced_mc = [] {
+    const char *e = getenv("E3_GEMM_MC");
+    return e ? atoi(e) : -1;
+  }();
   // Minimise waves x per-tile cost over the pair tiles (256 x BN), in units
-  // of one row of TMA fill per K element: the mainloop moves 256 + BN rows per
-  // K step (it is fill-bound), the issue-bound GELU epilogue adds ~ BN / 2 per
+  // of one row of TMA fill per K element.  The mainloop is bound by the L2 ->
+  // SM fill (the chip-wide LTS cap, ~42 B/clk per SM) or by the MMA (BN / 32
+  // clk per K element per pair = 1.31 BN fill rows), whichever is slower: a
+  // pair fetches 256 + BN rows per K element, 128 + BN with A multicast, 256 +
+  // BN / 2 with W multicast.  The issue-bound GELU epilogue adds ~ BN / 2 per
   // K step, and BN = 384 (one TMEM accumulator: nothing to overlap its
   // epilogue with) pays ~ 1720 x BN for the exposed epilogue.  Calibrated on
   // scripts/gemm_bn_sweep*.sh: BL N = 1024 FFN2 102 us at BN 256 (120 at 128);
@@ -430,25 +489,49 @@ int gemm_pick_bn(int M, int N, int K, int sms, int epi) {
   long long best_cost = 0;
   const int cands[5] = {384, 256, 192, 128, 64};
   const int pairs = sms / 2;
+  const int num_m = (M + 2 * BM - 1) / (2 * BM);
   for (int i = 0; i < 5; ++i) {
     const int bn = cands[i];
     if (N % bn || (bn == 384 && epi == E3_EPI_BIAS_GELU)) continue;
-    const long long tiles = (long long)((M + 2 * BM - 1) / (2 * BM)) * (N / bn);
-    const long long waves = (tiles + pairs - 1) / pairs;
-    const long long tile = (long long)K * (2 * BM + bn) + (epi == E3_EPI_BIAS_GELU ? (long long)K * bn / 2 : 0) +
-                           (bn > 256 ? 1720LL * bn : 0);
-    const long long cost = waves * tile;
-    if (best == 0 || cost < best_cost) { best = bn; best_cost = cost; }
+    if (forced && bn != forced) continue;
+    const int num_n = N / bn;
+    // multicast only on request: measured bitwise-equal but not faster on the
+    // B200 (scripts/gemm_mc_check.py: BB FFN1 + GELU 34.9 us unicast, 36.8 A
+    // multicast, 37.1 W multicast; FFN2 31.4 / 30.7 / 31.1; QKV 23.0 / - /
+    // 24.8): the mainloop is bound by the bytes one SM keeps in flight (three
+    // 56 KB stages beside the epilogue staging), not by the chip's L2 output
+    for (int mc = 0; mc < (forced_mc > 0 ? 3 : 1); ++mc) {
+      if (forced_mc >= 0 && mc != forced_mc) continue;
+      if (mc == GEMM_MC_A && num_n % 2) continue;
+      if (mc == GEMM_MC_B && num_m < 2) continue;
+      const long long units = mc == GEMM_MC_A   ? (long long)num_m * (num_n / 2)
+                              : mc == GEMM_MC_B ? (long long)((num_m + 1) / 2) * num_n
+                                                : (long long)num_m * num_n;
+      const long long slots = mc ? pairs / 2 : pairs;
+      const long long waves = (units + slots - 1) / slots;
+      const long long fill = (mc == GEMM_MC_A ? 128 : 256) + (mc == GEMM_MC_B ? bn / 2 : bn);
+      const long long mma = (long long)bn * 21 / 16;
+      const long long tile = (long long)K * (fill > mma ? fill : mma) +
+                             (epi == E3_EPI_BIAS_GELU ? (long long)K * bn / 2 : 0) + (bn > 256 ? 1720LL * bn : 0);
+      const long long cost = waves * tile;
+      if (best == 0 || cost < best_cost) { best = bn | (mc << 12); best_cost = cost; }
+    }
+  }
+  if (!best) {   // a forced combination that does not apply: the first N tile that divides N
+    for (int i = 0; i < 5 && !best; ++i)
+      if (N % cands[i] == 0 && !(cands[i] == 384 && epi == E3_EPI_BIAS_GELU)) best = cands[i];
   }
   return best;
 }
 
 e3_status gemm_tmaps(GemmMaps *g, const void *A, int64_t lda, const void *W, const void *C, int M, int N, int K,
-                     int bn) {
-  e3_status s = make_tmap_2d(&g->a, A, (uint64_t)M, (uint64_t)K, (uint64_t)lda, BM, BK);
-  if (s == E3_OK) s = make_tmap_2d(&g->b, W, (uint64_t)N, (uint64_t)K, (uint64_t)K, (uint32_t)(bn > 256 ? bn / 4 : bn / 2), BK);
+                     int code) {
+  const int bn = code & 0xFFF, mc = code >> 12;
+  const uint32_t wbox = (uint32_t)(bn > 256 ? bn / 4 : bn / 2) / (mc == GEMM_MC_B ? 2 : 1);
+  e3_status s = make_tmap_2d(&g->a, A, (uint64_t)M, (uint64_t)K, (uint64_t)lda, mc == GEMM_MC_A ? BM / 2 : BM, BK);
+  if (s == E3_OK) s = make_tmap_2d(&g->b, W, (uint64_t)N, (uint64_t)K, (uint64_t)K, wbox, BK);
   if (s == E3_OK) s = make_tmap_2d_sw64(&g->c, C, (uint64_t)M, (uint64_t)N, (uint64_t)N, 32, 32);
-  g->bn = bn;
+  g->bn = code;
   return s;
 }
 
@@ -456,12 +539,13 @@ e3_status gemm_run(const GemmMaps &g, const void *bias, const void *R, int M, in
                    cudaStream_t st) {
   auto *b = reinterpret_cast<const __nv_bfloat16 *>(bias);
   auto *r = reinterpret_cast<const __nv_bfloat16 *>(R);
-  switch (g.bn) {
-    case 384: return launch_epi<384>(epi, g, b, r, M, N, K, sms, st);
-    case 256: return launch_epi<256>(epi, g, b, r, M, N, K, sms, st);
-    case 192: return launch_epi<192>(epi, g, b, r, M, N, K, sms, st);
-    case 128: return launch_epi<128>(epi, g, b, r, M, N, K, sms, st);
-    case 64: return launch_epi<64>(epi, g, b, r, M, N, K, sms, st);
+  const int bn = g.bn & 0xFFF, mc = g.bn >> 12;
+  switch (bn) {
+    case 384: return launch_mc<384>(mc, epi, g, b, r, M, N, K, sms, st);
+    case 256: return launch_mc<256>(mc, epi, g, b, r, M, N, K, sms, st);
+    case 192: return launch_mc<192>(mc, epi, g, b, r, M, N, K, sms, st);
+    case 128: return launch_mc<128>(mc, epi, g, b, r, M, N, K, sms, st);
+    case 64: return launch_mc<64>(mc, epi, g, b, r, M, N, K, sms, st);
   }
   set_error("unsupported GEMM N tile");
   return E3_EUNSUPPORTED;

@@ -12,11 +12,18 @@ namespace e3 {
 
 // ---- K1 layer GEMM (gemm_tc.cu)
 struct GemmMaps {
-  CUtensorMap a;   // A [M,K], box 128 x 64, 128-B swizzle
-  CUtensorMap b;   // W [N,K], box BN/2 x 64, 128-B swizzle
+  CUtensorMap a;   // A [M,K], box 128 (64 when A is multicast) x 64, 128-B swizzle
+  CUtensorMap b;   // W [N,K], box BN/2 (/2 again when W is multicast) x 64, 128-B swizzle
   CUtensorMap c;   // C [M,N], box 32 x 32, 64-B swizzle (epilogue TMA store)
-  int bn;
+  int bn;          // tile code: N tile | multicast mode << 12 (gemm_pick_bn)
 };
+// Multicast modes of the layer GEMM (a cluster of two CTA pairs):
+//   GEMM_MC_NONE  one pair per cluster
+//   GEMM_MC_A     the pairs own N-neighbour tiles of one M block: each A box is
+//                 loaded half by each pair and multicast to both
+//   GEMM_MC_B     the pairs own M-neighbour tiles of one N block: W multicast
+enum { GEMM_MC_NONE = 0, GEMM_MC_A = 1, GEMM_MC_B = 2 };
+// returns a tile code (N tile | mode << 12) for gemm_tmaps / gemm_run
 int gemm_pick_bn(int M, int N, int K, int sms, int epi);
 e3_status gemm_set_trace(void *buf);   // diagnostics (e3_debug_gemm_trace)
 e3_status attn_set_trace(void *buf);   // diagnostics (e3_debug_gemm_trace)
