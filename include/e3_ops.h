@@ -48,7 +48,9 @@ e3_status e3_op_gemm_ln(void *stream, const void *A, const void *W, const void *
 /* Self-attention (a2) on tcgen05: qkv [B*S, 3H] (q | k | v, head h owning
  * columns h*64..h*64+63 of each third) -> ctx [B*S, H].  head_dim 64,
  * S <= 256, no mask.  softmax(q k^T / sqrt(64)) v with the rounding contract
- * p_bf16 = bf16(exp(s - max)), ctx = bf16((p_bf16 v) / sum(exp(s - max))). */
+ * p_bf16 = bf16(exp(s - max)), ctx = bf16((p_bf16 v) / sum(exp(s - max))).
+ * Work items are handed out through one device counter per GPU (allocated on
+ * the first call): calls on one device must be ordered on one stream. */
 e3_status e3_op_attention(void *stream, const void *qkv, void *ctx, int32_t B, int32_t S, int32_t H,
                           int32_t heads);
 

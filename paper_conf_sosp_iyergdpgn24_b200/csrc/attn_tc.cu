@@ -90,7 +90,8 @@ __device__ __forceinline__ void atrace(int j, int kind) {
 template <int SKV, bool kMask>
 __global__ void __launch_bounds__(AThr<SKV>::kThreads, 2)
     attn_tc_kernel(const __grid_constant__ CUtensorMap tq, const __grid_constant__ CUtensorMap tkv,
-                   const __grid_constant__ CUtensorMap tctx, int S, int H, int heads, int n_items) {
+                   const __grid_constant__ CUtensorMap tctx, int S, int H, int heads, int n_items,
+                   unsigned *__restrict__ ctr) {
   using CF = ACfg<SKV>;
   constexpr int KP = AThr<SKV>::KP;
   constexpr int NCH = CF::NCH;
@@ -125,6 +126,25 @@ __global__ void __launch_bounds__(AThr<SKV>::kThreads, 2)
     tma_prefetch(&tctx);
     for (int i = 0; i < 6; ++i) mbar_init(&bars[i], 1);
     fence_barrier_init();
+  }
+  // Items are handed out by an atomic counter (ctr[0]) instead of a static
+  // stride: a CTA that becomes resident late (the SMs held by the previous
+  // run's ramp and compaction on the tail stream) takes only what is left,
+  // instead of its fixed share finishing last.  The last CTA to leave
+  // (ctr[1]) zeroes both words for the next launch.  Every item is computed
+  // the same way wherever it runs, so results do not depend on the schedule.
+  // The counter is taken before the PDL wait: consecutive launches on one
+  // counter set alternate between its two pairs (attn_run), and the launch
+  // that last used (and zeroed) this pair completed before the previous
+  // kernel in the stream -- the other pair's launch -- passed its own wait.
+  // Thread 0 holds one ticket ahead (nreg), so the atomic's round trip is
+  // off the critical path: the ticket taken in iteration j is used in j + 1.
+  // (ctr == NULL: the static stride, E3_ATTN_STATIC=1 diagnostics)
+  __shared__ int s_item[2];
+  int nreg = 0;
+  if (tid == 0) {
+    s_item[0] = ctr ? (int)atomicAdd(&ctr[0], 1u) : (int)blockIdx.x;
+    if (s_item[0] < n_items) nreg = ctr ? (int)atomicAdd(&ctr[0], 1u) : s_item[0] + (int)gridDim.x;
   }
   if (warp == 0) tmem_alloc(tslot, CF::kTmemCols);
   tc_fence_before();
@@ -161,14 +181,14 @@ __global__ void __launch_bounds__(AThr<SKV>::kThreads, 2)
     phases ^= 1u << i;
   };
 
-  int item = blockIdx.x;
+  int item = s_item[0];
   if (tid == 0 && item < n_items) {
     issue_qk(item, 0);
     issue_v(item, 0);
   }
   uint32_t sphase = 0, ophase = 0;
 
-  for (int j = 0; item < n_items; ++j, item += gridDim.x) {
+  for (int j = 0; item < n_items; ++j) {
     const int qs = (CF::kNQK == 2) ? (j & 1) : 0;
     const int vs = (CF::kNV == 2) ? (j & 1) : 0;
     uint8_t *sQ = smem + qs * (CF::kQ + CF::kKV);
@@ -176,7 +196,12 @@ __global__ void __launch_bounds__(AThr<SKV>::kThreads, 2)
     int b, h, qt;
     coords(item, b, h, qt);
     const int q0 = qt * QT;
-    const int next = item + gridDim.x;
+    int next = n_items;
+    if (tid == 0) {                 // read by the other threads after the softmax exchange barrier
+      next = nreg;
+      s_item[(j + 1) & 1] = next;
+      if (next < n_items) nreg = ctr ? (int)atomicAdd(&ctr[0], 1u) : next + (int)gridDim.x;
+    }
 
     if (tid == 0) {
       // MMA1: S = Q K^T
@@ -354,6 +379,14 @@ __global__ void __launch_bounds__(AThr<SKV>::kThreads, 2)
         issue_v(next, 0);
       }
     }
+    item = s_item[(j + 1) & 1];   // written by thread 0 before this iteration's first barrier
+  }
+  if (tid == 0 && ctr) {
+    __threadfence();
+    if (atomicAdd(&ctr[1], 1u) == gridDim.x - 1) {   // every CTA has taken its last item
+      atomicExch(&ctr[0], 0u);
+      atomicExch(&ctr[1], 0u);
+    }
   }
   if (tid == 0) bulk_wait_read<0>();   // smem read before exit; the global writes complete with the grid
   __syncthreads();
@@ -362,7 +395,7 @@ __global__ void __launch_bounds__(AThr<SKV>::kThreads, 2)
 }
 
 template <int SKV, bool kMask>
-e3_status launch_attn(const AttnMaps &m, int B, int S, int H, int heads, cudaStream_t st) {
+e3_status launch_attn(const AttnMaps &m, int B, int S, int H, int heads, unsigned *ctr, cudaStream_t st) {
   auto kern = attn_tc_kernel<SKV, kMask>;
   static bool attr_done = false;
   static int sms = 0, per_sm = 0;
@@ -389,8 +422,10 @@ e3_status launch_attn(const AttnMaps &m, int B, int S, int H, int heads, cudaStr
   }
   const int n_items = B * heads * ((S + QT - 1) / QT);
   const int grid = n_items < per_sm * sms ? n_items : per_sm * sms;
+  static const bool stat = getenv("E3_ATTN_STATIC") != nullptr;
+  if (stat) ctr = nullptr;
   E3_CUDA_TRY(launch_k(kern, dim3(grid), dim3(AThr<SKV>::kThreads), ACfg<SKV>::kSmem, st, m.q, m.kv, m.ctx, S, H, heads,
-                       n_items));
+                       n_items, ctr));
   E3_CUDA_TRY(cudaGetLastError());
   count_launch();
   return E3_OK;
@@ -415,13 +450,16 @@ e3_status attn_tmaps(AttnMaps *m, const void *qkv, const void *ctx, int B, int S
   return s;
 }
 
-e3_status attn_run(const AttnMaps &m, int B, int S, int H, int heads, cudaStream_t st) {
+e3_status attn_run(const AttnMaps &m, int B, int S, int H, int heads, unsigned *ctr4, int *parity,
+                   cudaStream_t st) {
+  unsigned *ctr = ctr4 + 2 * (*parity & 1);
+  *parity ^= 1;
   switch (m.skv) {
-    case 128: return S == 128 ? launch_attn<128, false>(m, B, S, H, heads, st) : launch_attn<128, true>(m, B, S, H, heads, st);
-    case 160: return S == 160 ? launch_attn<160, false>(m, B, S, H, heads, st) : launch_attn<160, true>(m, B, S, H, heads, st);
-    case 192: return S == 192 ? launch_attn<192, false>(m, B, S, H, heads, st) : launch_attn<192, true>(m, B, S, H, heads, st);
-    case 224: return S == 224 ? launch_attn<224, false>(m, B, S, H, heads, st) : launch_attn<224, true>(m, B, S, H, heads, st);
-    case 256: return S == 256 ? launch_attn<256, false>(m, B, S, H, heads, st) : launch_attn<256, true>(m, B, S, H, heads, st);
+    case 128: return S == 128 ? launch_attn<128, false>(m, B, S, H, heads, ctr, st) : launch_attn<128, true>(m, B, S, H, heads, ctr, st);
+    case 160: return S == 160 ? launch_attn<160, false>(m, B, S, H, heads, ctr, st) : launch_attn<160, true>(m, B, S, H, heads, ctr, st);
+    case 192: return S == 192 ? launch_attn<192, false>(m, B, S, H, heads, ctr, st) : launch_attn<192, true>(m, B, S, H, heads, ctr, st);
+    case 224: return S == 224 ? launch_attn<224, false>(m, B, S, H, heads, ctr, st) : launch_attn<224, true>(m, B, S, H, heads, ctr, st);
+    case 256: return S == 256 ? launch_attn<256, false>(m, B, S, H, heads, ctr, st) : launch_attn<256, true>(m, B, S, H, heads, ctr, st);
   }
   set_error("attention: S > 256");
   return E3_EUNSUPPORTED;

@@ -66,7 +66,11 @@ struct AttnMaps {
   int skv;
 };
 e3_status attn_tmaps(AttnMaps *m, const void *qkv, const void *ctx, int B, int S, int H);
-e3_status attn_run(const AttnMaps &m, int B, int S, int H, int heads, cudaStream_t st);
+// ctr: four device words, zero before the first launch (the kernel leaves
+// them zero): two (item counter, CTA exit count) pairs, used alternately by
+// consecutive launches (*parity flips per call), so a launch never takes
+// items from the pair its still-running predecessor uses
+e3_status attn_run(const AttnMaps &m, int B, int S, int H, int heads, unsigned *ctr, int *parity, cudaStream_t st);
 
 // ---- K3 LayerNorm (layernorm.cu)
 e3_status layernorm_run(const void *x, const void *g, const void *b, void *y, int rows, int H, float eps,
@@ -78,7 +82,8 @@ constexpr int kRampRowsPerCta = 16;   // rows per ramp row group (one ticket eac
 // tickets, then the fused ramp + compaction's decision and exit counters
 constexpr int kRampCtrGroupsDone = 1 + 4096 / kRampRowsPerCta;
 constexpr int kRampCtrExit = kRampCtrGroupsDone + 1;
-constexpr int kCtrWordsAll = kRampCtrExit + 1;
+constexpr int kAttnCtr = kRampCtrExit + 1;   // [2][2]: attention item counter, CTA exits (two pairs)
+constexpr int kCtrWordsAll = kAttnCtr + 4;
 struct RampArgs {
   int arch;
   const void *x;            // [B,S,H] bf16 (pre-LN rows when ln_g != NULL)

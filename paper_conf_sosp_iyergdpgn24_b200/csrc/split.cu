@@ -834,7 +834,7 @@ static e3_status split_run_body(e3_split *s, cudaStream_t st, const void *x_in, 
       }
       {
         ProfScope ps(PK_ATTN, st, f_att, 0);
-        E3_RUN(attn_run(s->attn, B, S, H, d.heads, st));
+        E3_RUN(attn_run(s->attn, B, S, H, d.heads, ws.ctr + kAttnCtr, &ws.attn_parity, st));
       }
       if (s->use_oln) {
         LnGemmMaps lm = m.oln;
@@ -871,7 +871,7 @@ static e3_status split_run_body(e3_split *s, cudaStream_t st, const void *x_in, 
     }
     {
       ProfScope ps(PK_ATTN, st, f_att, 0);
-      if (!skip(PK_ATTN)) E3_RUN(attn_run(s->attn, B, S, H, d.heads, st));
+      if (!skip(PK_ATTN)) E3_RUN(attn_run(s->attn, B, S, H, d.heads, ws.ctr + kAttnCtr, &ws.attn_parity, st));
     }
     if (s->use_oln) {
       LnGemmMaps lm = m.oln;
@@ -1145,7 +1145,18 @@ e3_status e3_op_attention(void *stream, const void *qkv, void *ctx, int32_t B, i
   AttnMaps m;
   e3_status r = attn_tmaps(&m, qkv, ctx, B, S, H);
   if (r != E3_OK) return r;
-  return attn_run(m, B, S, H, heads, reinterpret_cast<cudaStream_t>(stream));
+  // the item counter: one per device, zeroed once (every launch leaves it
+  // zero), so launches of this op on one device must be stream-ordered
+  int dev = 0;
+  E3_CUDA_TRY(cudaGetDevice(&dev));
+  static unsigned *ctr_of[64] = {};
+  static int par_of[64] = {};
+  if (dev < 0 || dev >= 64) return E3_EINVAL;
+  if (!ctr_of[dev]) {
+    E3_CUDA_TRY(cudaMalloc(reinterpret_cast<void **>(&ctr_of[dev]), 4 * sizeof(unsigned)));
+    E3_CUDA_TRY(cudaMemset(ctr_of[dev], 0, 4 * sizeof(unsigned)));
+  }
+  return attn_run(m, B, S, H, heads, ctr_of[dev], &par_of[dev], reinterpret_cast<cudaStream_t>(stream));
 }
 
 e3_status e3_op_layernorm(void *stream, const void *x, const void *g, const void *b, void *y, int32_t rows, int32_t H,

@@ -26,7 +26,8 @@ struct Workspace {
   uint8_t *alive_t = nullptr;
   float *pool = nullptr;
   uint8_t *alive = nullptr;
-  unsigned *ctr = nullptr;        // [kCtrWords]: compaction ticket, ramp row-group tickets
+  unsigned *ctr = nullptr;        // [kCtrWords]: compaction ticket, ramp row-group tickets, attention items
+  int attn_parity = 0;            // which attention counter pair the next launch uses (attn_run)
   int *err = nullptr;             // device error flag: a kernel saw an argument outside its range
   // LLAMA decode (allocated by ensure_llama): LM-head tile statistics,
   // stream-K partials and tickets of the decode GEMMs, RoPE cos/sin table

@@ -37,14 +37,21 @@ if os.environ.get("_GEMM_MC_CHILD"):
     sys.exit(0)
 
 os.makedirs("gpurun_out", exist_ok=True)
-for case in sys.argv[1:]:
+args = sys.argv[1:]
+libs = [None]
+if args and args[0].startswith("--libs="):   # A/B of library builds (scripts/build_variant.py), unicast only
+    libs = args[0][len("--libs="):].split(",")
+    args = args[1:]
+for case in args:
     f = case.split(",")
     M, N, K, epi = int(f[0]), int(f[1]), int(f[2]), f[3]
     bns = [int(f[4])] if len(f) > 4 else [0]
     base = None
     for bn in bns:
-        for mc in (0, 1, 2):
+        for mc, lib in ([(0, x) for x in libs] if libs[0] else [(m, None) for m in (0, 1, 2)]):
             env = dict(os.environ, _GEMM_MC_CHILD="1", E3_GEMM_MC=str(mc))
+            if lib:
+                env["E3_LIB_PATH"] = os.path.abspath(lib)
             if bn:
                 env["E3_GEMM_BN"] = str(bn)
             out = f"gpurun_out/_mc_{mc}.pt"
@@ -60,4 +67,4 @@ for case in sys.argv[1:]:
                 base = C
             fl = 2 * M * N * K
             print(f"M={M} N={N} K={K} {epi:10s} bn={bn or 'auto'} mc={mc}: {float(t):7.2f} us "
-                  f"({fl / float(t) / 1e6:6.0f} TF/s) max|err| {err} {same}", flush=True)
+                  f"({fl / float(t) / 1e6:6.0f} TF/s) max|err| {err} {same} {lib or ''}", flush=True)

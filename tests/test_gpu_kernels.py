@@ -87,6 +87,42 @@ def test_attention_matches_oracle(api, B, S, H, heads):
     _assert_bf16_close(got, ref, ulps=2.0, atol=2e-3, min_exact=0.9)
 
 
+@pytest.mark.parametrize("B,S,H,heads", [(64, 128, 768, 12), (40, 197, 768, 12)])
+def test_attention_back_to_back_launches(api, B, S, H, heads):
+    """Work items come from a device counter that each launch leaves zeroed
+    (two counter pairs alternate): launches queued back to back under PDL --
+    eagerly, and 5 per CUDA graph replayed twice -- must each reproduce the
+    isolated launch bit for bit (a launch taking items from its still-running
+    predecessor's counter recomputes or skips items)."""
+    g = torch.Generator(device=DEV).manual_seed(S)
+    xs = [torch.randn(B * S, 3 * H, device=DEV, generator=g).to(torch.bfloat16) for _ in range(3)]
+    ref = []
+    for x in xs:
+        ref.append(api.ops.attention(x, B, S, H, heads).clone())
+        torch.cuda.synchronize()
+    outs = [torch.empty(B * S, H, device=DEV, dtype=torch.bfloat16) for _ in range(7)]
+    for i, o in enumerate(outs):
+        api.ops.attention(xs[i % 3], B, S, H, heads, out=o)
+    torch.cuda.synchronize()
+    for i, o in enumerate(outs):
+        assert torch.equal(o, ref[i % 3]), i
+    st = torch.cuda.Stream()
+    with torch.cuda.stream(st):
+        api.ops.attention(xs[0], B, S, H, heads, out=outs[0], stream=st)   # warm-up outside capture
+        st.synchronize()
+        graph = torch.cuda.CUDAGraph()
+        with torch.cuda.graph(graph, stream=st):
+            for i in range(5):
+                api.ops.attention(xs[i % 3], B, S, H, heads, out=outs[i], stream=st)
+    for _ in range(2):
+        for o in outs[:5]:
+            o.fill_(0)
+        graph.replay()
+        torch.cuda.synchronize()
+        for i in range(5):
+            assert torch.equal(outs[i], ref[i % 3]), i
+
+
 @pytest.mark.parametrize("rows,H,eps", [(37, 128, 1e-12), (1000, 768, 1e-12), (64, 1024, 1e-6), (5, 64, 1e-5)])
 def test_layernorm_matches_oracle(api, rows, H, eps):
     from oracle.encoder import layer_norm
