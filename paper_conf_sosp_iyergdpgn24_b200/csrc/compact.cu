@@ -341,6 +341,10 @@ e3_status ln_compact_run(const void *y, const int64_t *id, const uint8_t *alive,
   auto *gp = reinterpret_cast<const __nv_bfloat16 *>(g);
   auto *bp = reinterpret_cast<const __nv_bfloat16 *>(b);
   const int vpl = (H / 8 + 31) / 32;
+  static const int cap_env = [] {   // diagnostics: E3_COMPACT_GRID caps the CTAs
+    const char *e = getenv("E3_COMPACT_GRID");
+    return e ? atoi(e) : 0;
+  }();
 #define E3_LNC(V)                                                                                          \
   do {                                                                                                     \
     auto kern = gp ? ln_compact_kernel<V, true> : ln_compact_kernel<V, false>;                             \
@@ -349,6 +353,7 @@ e3_status ln_compact_run(const void *y, const int64_t *id, const uint8_t *alive,
     if (!occ) E3_CUDA_TRY(cudaOccupancyMaxActiveBlocksPerMultiprocessor(&occ, kern, kThreads, 0));        \
     if (occ < 1) occ = 1;                                                                                  \
     if (grid > (int64_t)occ * sms) grid = (int64_t)occ * sms;                                              \
+    if (cap_env > 0 && grid > cap_env) grid = cap_env;                                                     \
     if (grid < 1) grid = 1;                                                                                \
     E3_CUDA_TRY(launch_k(kern, dim3((unsigned)grid), dim3(kThreads), 0, st, yp, id, alive, B, S, H, gp, bp, \
                          eps, dst, n_surv_dev));                                                           \

@@ -839,11 +839,36 @@ int dec_tiles(int N, int epi) { return epi == E3_DEC_SWIGLU ? N / 64 : (N + DM -
 // us, scripts/dec_bench.py) and in a graph-replayed split (llama_timeline:
 // 893 -> 859 us per 4 layers) but 0.3 % slower in the LM bench's pipeline
 // (same box, A/B twice), so it is not the default.
+// Most contributors any tile has when `total` iterations (tiles of nkb) are cut
+// into G ranges start(c) = c total / G (the kernel's SK split).
+static int sk_max_contrib(long total, int nkb, long G) {
+  int worst = 0;
+  long c = 0;   // first range touching the current tile
+  for (long t0 = 0; t0 < total; t0 += nkb) {
+    while (c + 1 < G && (c + 1) * total / G <= t0) ++c;
+    long e = c;
+    while (e + 1 < G && (e + 1) * total / G < t0 + nkb) ++e;
+    if ((int)(e - c + 1) > worst) worst = (int)(e - c + 1);
+  }
+  return worst;
+}
+
+// Stream-K grid: one CTA per SM, except that a few SMs are left out when that
+// bounds every tile at two contributors (Llama-7B QKV: 96 tiles x 32 k-blocks
+// on 148 CTAs gives tiles of three contributors, whose last one pays the
+// global fixup; 144 CTAs = 3 ranges per 2 tiles, two contributors each, and
+// the second contributor fetches the first's partial while its MMAs run)
 static int dec_grid(int N, int K, int epi, int sms) {
-  const long total = (long)dec_tiles(N, epi) * (K / DKS);
+  const int nkb = K / DKS;
+  const long total = (long)dec_tiles(N, epi) * nkb;
   static const int cap = getenv("E3_DEC_MAXGRID") ? atoi(getenv("E3_DEC_MAXGRID")) : 0;   // diagnostics
+  static const bool any3 = getenv("E3_DEC_ANY_CONTRIB") != nullptr;                      // diagnostics: old grid
   if (cap > 0 && cap < sms) sms = cap;
-  return (int)(total < sms ? total : sms);
+  if (total <= sms) return (int)total;
+  if (!any3 && sk_max_contrib(total, nkb, sms) > 2)
+    for (int g = sms - 1; g >= (sms * 15) / 16; --g)
+      if (sk_max_contrib(total, nkb, g) <= 2) return g;
+  return sms;
 }
 
 int dec_max_contrib(int N, int K, int epi, int sms) {
