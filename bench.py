@@ -63,6 +63,7 @@ def parse():
                     help="llama: one step = e3_decode_run of this many greedy tokens per sequence (NEXT-2: "
                          "skipped layers' K/V filled from the exit state); 0 = one token (e3_pipeline_run)")
     ap.add_argument("--plan", default="per-ramp", choices=["per-ramp", "cut6"])
+    ap.add_argument("--lag", type=int, default=1, help="host look-behind of the stage loop (runs in flight)")
     ap.add_argument("--no-e2e", action="store_true")
     ap.add_argument("--no-cpu", action="store_true")
     ap.add_argument("--cpu-inputs", type=int, default=32)
@@ -281,7 +282,7 @@ def main():
         total = n * world
         lo, hi = par.input_share(layout, rank, total)
         comm = par.make_comm(rank, world, local)
-        plan = api.make_plan(cfg, bounds, tau, lag=1, placement=par.placement(layout, bounds), transport="nccl")
+        plan = api.make_plan(cfg, bounds, tau, lag=args.lag, placement=par.placement(layout, bounds), transport="nccl")
         pipe = api.Pipeline(model, plan, comm)
         ex = api.ExitBuffers(total, cfg.classes, cfg.n_ramps, dev)
         plan_name = f"stages {list(layout.bounds)} replicas {list(layout.replicas)} (per-ramp splits inside)"
@@ -299,7 +300,7 @@ def main():
         ids_dev = torch.arange(0, n, dtype=torch.int64, device=dev)   # local ids index the exit arrays
         ids_host = torch.arange(0, n, dtype=torch.int64).pin_memory()
         ex = api.ExitBuffers(n, cfg.classes, cfg.n_ramps, dev, hidden=cfg.hidden if dsteps else 0)
-        pipe = api.Pipeline(model, api.make_plan(cfg, bounds, tau, lag=1))
+        pipe = api.Pipeline(model, api.make_plan(cfg, bounds, tau, lag=args.lag))
         if dsteps:
             x_dec = torch.empty_like(x_dev[:, 0, :])
 
@@ -389,7 +390,7 @@ def main():
         del Xr
         idr = torch.arange(0, n, dtype=torch.int64, device=dev)
         exr = api.ExitBuffers(n, cfg.classes, cfg.n_ramps, dev)
-        rpipe = api.Pipeline(model, api.make_plan(cfg, bounds, tau, lag=1))
+        rpipe = api.Pipeline(model, api.make_plan(cfg, bounds, tau, lag=args.lag))
 
         def rstep():
             with torch.cuda.stream(stream):

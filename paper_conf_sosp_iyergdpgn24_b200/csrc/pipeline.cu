@@ -938,7 +938,9 @@ e3_status e3_pipeline_create(const e3_plan *p, const e3_weights *w, int device, 
   if (e == cudaSuccess) e = cudaStreamCreateWithFlags(&pl->copy_stream, cudaStreamNonBlocking);
   int prio_lo = 0, prio_hi = 0;
   if (e == cudaSuccess) e = cudaDeviceGetStreamPriorityRange(&prio_lo, &prio_hi);
-  if (e == cudaSuccess) e = cudaStreamCreateWithPriority(&pl->tail_stream, cudaStreamNonBlocking, prio_hi);
+  static const bool tail_lo = getenv("E3_TAIL_PRIO_LOW") != nullptr;   // diagnostics: tail at the main stream's priority
+  if (e == cudaSuccess)
+    e = cudaStreamCreateWithPriority(&pl->tail_stream, cudaStreamNonBlocking, tail_lo ? prio_lo : prio_hi);
   for (int i = 0; i < kSlots && e == cudaSuccess; ++i)
     e = cudaEventCreateWithFlags(&pl->fork[i], cudaEventDisableTiming);
   if (e == cudaSuccess) e = cudaEventCreateWithFlags(&pl->joined, cudaEventDisableTiming);
