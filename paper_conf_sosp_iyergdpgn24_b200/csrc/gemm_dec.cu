@@ -37,6 +37,9 @@ namespace e3 {
 
 namespace {
 
+#ifndef E3_DEC_NO_LL
+#define E3_DEC_NO_LL 0                // diagnostics builds: last-arrival reduction for every shared tile
+#endif
 constexpr int DM = 128;            // weight rows per tile (MMA M)
 constexpr int DK = 64;             // K per 128-byte swizzle atom / TMA box
 constexpr int DKS = 2 * DK;        // K per pipeline stage: two atoms, so the two 128-byte
@@ -323,12 +326,28 @@ __global__ void __launch_bounds__(kDThreads, 1)
       // memory round trip on the kernel's critical path.
       bool early = false;
       int early_slot = 0;
+      // Two contributors whose ranges BOTH end in this tile (with 3 ranges per
+      // 2 tiles, every other tile): fixed roles instead of "last arrival
+      // reduces" -- the head (slot 0) publishes its partial without reading
+      // the ticket first, the tail (slot 1, this tile is its whole range)
+      // waits for it and adds it as in the early fetch.  Before, both often
+      // arrived together and each paid ticket read + partial write + fence +
+      // atomic before either could reduce (~4.6 us, dec_segments).  The tail
+      // waits only on the head's mainloop, which depends on nothing else.
+      bool ll = false;
       if (T <= 64 && !whole) {
         const int c_first = sk.owner(t0i), c_last = sk.owner(t1i - 1);
-        if (c_last - c_first == 1) {
+        ll = !E3_DEC_NO_LL && c_last - c_first == 1 && sk.start(c_last + 1) == t1i;
+        if (c_last - c_first == 1 && !(ll && blockIdx.x == c_first)) {
           const int slot = (int)blockIdx.x - c_first;
           if (et == 0) {
-            const unsigned seen = *reinterpret_cast<volatile unsigned *>(&a.tickets[tile]);
+            volatile unsigned *tk = &a.tickets[tile];
+            unsigned seen = *tk;
+            if (ll)
+              while (seen != 1u) {
+                __nanosleep(100);
+                seen = *tk;
+              }
             *s_last = (seen == 1u) ? 3 : 0;
             if (seen == 1u) a.tickets[tile] = 0;   // both contributors accounted for: ready for the next launch
           }
@@ -403,9 +422,13 @@ __global__ void __launch_bounds__(kDThreads, 1)
         // is summed in its contributor position below -- no write, fence and
         // ticket round trips on the kernel's critical path
         if (et == 0) {
-          const unsigned seen = *reinterpret_cast<volatile unsigned *>(&a.tickets[tile]);
-          *s_last = (seen == (unsigned)(ncon - 1)) ? 2 : 0;
-          if (*s_last) a.tickets[tile] = 0;   // every contributor arrived: ready for the next launch
+          if (ll) {
+            *s_last = 0;                        // the head of a two-late tile always publishes
+          } else {
+            const unsigned seen = *reinterpret_cast<volatile unsigned *>(&a.tickets[tile]);
+            *s_last = (seen == (unsigned)(ncon - 1)) ? 2 : 0;
+            if (*s_last) a.tickets[tile] = 0;   // every contributor arrived: ready for the next launch
+          }
         }
         epi_bar();
         const bool own_in_smem = *s_last == 2;
