@@ -230,6 +230,33 @@ def test_two_stage_nccl_two_gpus(api):
     assert np.array_equal(el, el1)
 
 
+def test_nccl_single_rank_communicator_runs_the_pipeline(api):
+    """The NCCL transport's setup on the one GPU this pod has: the library
+    resolves libnccl (the copy torch loaded) at run time, creates a unique id
+    and a world-size-1 communicator, validates a transport=NCCL plan and runs
+    it (every split on rank 0: no links) -- bitwise the single-rank pipeline
+    without a communicator.  The two-rank data path is
+    test_two_stage_nccl_two_gpus (two GPUs) and the LOOPBACK tests above."""
+    cfg = e3data.get("tiny")
+    N = 160
+    model = api.DeviceModel(cfg, e3data.make_weights(cfg), DEV)
+    uid = api.Comm.unique_id()
+    assert len(uid) == 128 and any(uid)
+    comm = api.Comm.nccl(uid, 0, 1, 0)
+    assert comm.rank_world() == (0, 1)
+    X = bf16_tensor(e3data.make_inputs(cfg, range(N)))
+    ex = api.ExitBuffers(N, cfg.classes, cfg.n_ramps, DEV)
+    plan = api.make_plan(cfg, (0, 2, 4), cfg.tau, placement=[[0], [0]], transport="nccl")
+    pipe = api.Pipeline(model, plan, comm)
+    pipe.run(X, torch.arange(N, dtype=torch.int64, device=DEV), ex)
+    torch.cuda.synchronize()
+    el1, lg1 = _single(api, model, cfg, (0, 2, 4), cfg.tau, X)
+    assert np.array_equal(ex.exit_layer.cpu().numpy(), el1)
+    assert np.array_equal(ex.logits.cpu().numpy(), lg1)
+    del pipe
+    comm.close()
+
+
 def test_dp_planned_layout_runs_through_the_library(api):
     """NEXT-1 end to end: planner.plan_dp on the measured r02 profile chooses
     cuts and replicas for 4 GPUs (forced to 3 stages so that transfers
