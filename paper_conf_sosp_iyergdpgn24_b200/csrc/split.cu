@@ -45,7 +45,7 @@ Workspace::~Workspace() {
   int prev = 0;
   cudaGetDevice(&prev);
   cudaSetDevice(device);
-  void *bufs[] = {qkv, ctx, y, x1, h, xa, xb, yt, alive_t, pool, alive, ctr, err, lm_stats, dec_part, dec_tickets, rope};
+  void *bufs[] = {qkv, ctx, y, x1, h, xa, xb, yt, yt0, alive_t, pool, alive, ctr, err, lm_stats, dec_part, dec_tickets, rope};
   for (void *p : bufs)
     if (p) cudaFree(p);
   cudaSetDevice(prev);
@@ -102,8 +102,9 @@ e3_status Workspace::create(int device, int B, int S, int H, int F, int elem, st
   E3_CUDA_TRY(cudaMalloc(&ws->xb, M * H * e));
   E3_CUDA_TRY(cudaMalloc(&ws->pool, (size_t)B * H * 4));
   E3_CUDA_TRY(cudaMalloc(&ws->alive, (size_t)B));
-  if (elem == 2) {   // parity-1 tail buffers (bf16 encoder runs only)
+  if (elem == 2) {   // tail buffers (bf16 encoder runs only)
     E3_CUDA_TRY(cudaMalloc(&ws->yt, M * H * e));
+    E3_CUDA_TRY(cudaMalloc(&ws->yt0, M * H * e));
     E3_CUDA_TRY(cudaMalloc(&ws->alive_t, (size_t)B));
     E3_CUDA_TRY(cudaMemset(ws->alive_t, 0, (size_t)B));
   }
@@ -354,6 +355,7 @@ e3_status split_create_shared(const e3_split_desc *d, const e3_weights *w, int d
     if (st == E3_OK) st = gemm_tmaps(&m.f1, ws->x1, H, s->L[i].w_1, ws->h, M, F, H, s->bn_f1);
     if (st == E3_OK) st = gemm_tmaps(&m.f2, ws->h, F, s->L[i].w_2, vit ? out : ws->y, M, H, F, s->bn_f2);
     if (st == E3_OK && i == nl - 1) st = gemm_tmaps(&m.f2t, ws->h, F, s->L[i].w_2, ws->yt, M, H, F, s->bn_f2);
+    if (st == E3_OK && i == nl - 1) st = gemm_tmaps(&m.f2t0, ws->h, F, s->L[i].w_2, ws->yt0, M, H, F, s->bn_f2);
   }
   if (st == E3_OK) st = attn_tmaps(&s->attn, ws->qkv, ws->ctx, B, S, H);
   if (st != E3_OK) {
@@ -813,7 +815,12 @@ static e3_status split_run_body(e3_split *s, cudaStream_t st, const void *x_in, 
   bool compacted = false;   // the last ramp's fused kernel also compacted the survivors
   // tst != st: the last ramp and the compaction run on tst (split_run_to)
   const bool ovl = tst != st;
-  void *const y_last = par ? ws.yt : ws.y;        // BERT: the last layer's pre-LN2 output
+  // The split's last layer writes a buffer of its own per run parity: the
+  // run's tail (last ramp + compaction, on tst) still reads it while the next
+  // run's layers execute, and a multi-layer split's earlier layers write
+  // ws.y / xa / xb (BERT: every FFN2 writes ws.y -- a parity-0 tail reading
+  // ws.y raced the next run's first FFN2: EE-BERT-large, 4-layer splits)
+  void *const y_last = par ? ws.yt : ws.yt0;      // BERT: the last layer's pre-LN2 output
   uint8_t *const alive = par ? ws.alive_t : ws.alive;
   for (int i = 0; i < nl; ++i) {
     const int l = d.layer_begin + i;
@@ -855,9 +862,10 @@ static e3_status split_run_body(e3_split *s, cudaStream_t st, const void *x_in, 
       }
       {
         ProfScope ps(PK_GEMM_FFN2, st, f_1, 0);
-        E3_RUN(gemm_run(last_layer && par ? m.f2t : m.f2, L.b_2, ws.y, M, H, F, E3_EPI_BIAS_RESID, s->sms, st));
+        E3_RUN(gemm_run(last_layer ? (par ? m.f2t : m.f2t0) : m.f2, L.b_2, ws.y, M, H, F, E3_EPI_BIAS_RESID, s->sms,
+                        st));
       }
-      cur = last_layer && par ? ws.yt : out;
+      cur = last_layer ? y_last : out;
     } else {
     {
       ProfScope ps(PK_GEMM_QKV, st, f_qkv, 0);
@@ -893,7 +901,8 @@ static e3_status split_run_body(e3_split *s, cudaStream_t st, const void *x_in, 
     {
       ProfScope ps(PK_GEMM_FFN2, st, f_1, 0);
       if (!skip(PK_GEMM_FFN2))
-        E3_RUN(gemm_run(last_layer && par ? m.f2t : m.f2, L.b_2, ws.x1, M, H, F, E3_EPI_BIAS_RESID, s->sms, st));
+        E3_RUN(gemm_run(last_layer ? (par ? m.f2t : m.f2t0) : m.f2, L.b_2, ws.x1, M, H, F, E3_EPI_BIAS_RESID, s->sms,
+                        st));
     }
     // The split's last layer never materialises LN2: its ramp normalises the
     // CLS rows itself and the fused LN2 + compaction normalises only the

@@ -23,6 +23,7 @@ struct Workspace {
   // last ramp + compaction of run j overlaps run j+1 on a second stream:
   // split_run_to's tail_st)
   void *yt = nullptr;
+  void *yt0 = nullptr;            // the same for runs with parity 0 (never a non-last layer's output)
   uint8_t *alive_t = nullptr;
   float *pool = nullptr;
   uint8_t *alive = nullptr;
@@ -56,6 +57,7 @@ struct e3_split {
   struct LayerMaps {
     e3::GemmMaps qkv, o, f1, f2;
     e3::GemmMaps f2t;     // last layer: FFN2 writing Workspace::yt (runs with parity 1)
+    e3::GemmMaps f2t0;    // last layer: FFN2 writing Workspace::yt0 (runs with parity 0)
     e3::LnGemmMaps oln;   // fused O projection + residual + LayerNorm (when use_oln)
   };
   bool use_oln = false;

@@ -382,6 +382,28 @@ def test_bert_large_pipeline_full_size_sampled(api, bert_large):
     _compare_records(recs, ex, sample, cfg, E2E_MARGIN, E2E_LOGIT_TOL)
 
 
+def test_bert_large_pipeline_repeats_bitwise(api, bert_large):
+    """The same EE-BERT-large job (4-layer splits, the tail stream overlapping
+    the next run's layers) five times: exit records bit for bit equal.  A
+    run's tail reads its last layer's output while the next run executes; when
+    that output shared ws.y with every layer's FFN2, 2 of 8 repeats differed
+    (79 exit layers) -- the last layer now writes a per-parity buffer."""
+    cfg, tau, W, model = bert_large
+    N = 768
+    X = bf16_tensor(e3data.make_inputs(cfg, range(N)))
+    pipe = api.Pipeline(model, api.make_plan(cfg, Plan.per_ramp(cfg.ramp_layers).bounds, tau))
+    base = None
+    for rep in range(5):
+        ex = api.ExitBuffers(N, cfg.classes, cfg.n_ramps, DEV)
+        pipe.run(X, torch.arange(N, dtype=torch.int64, device=DEV), ex)
+        torch.cuda.synchronize()
+        got = (ex.exit_layer.cpu().numpy(), ex.logits.cpu().numpy())
+        if base is None:
+            base = got
+        else:
+            assert np.array_equal(got[0], base[0]) and np.array_equal(got[1], base[1]), rep
+
+
 @pytest.fixture(scope="module")
 def vit_base(api):
     cfg = e3data.get("vt")
