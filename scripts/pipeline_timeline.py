@@ -72,8 +72,8 @@ for k in np.unique(kid):
             inst.append((k, sel[start:i]))
             start = i
 inst.sort(key=lambda p: np.max(t[p[1], 1]))
-qkv = [i for i, (k, _) in enumerate(inst) if 1000 <= k < 2000 and (k - 1000) // 64 * 64 in (192, 256, 384)
-       and i + 1 < len(inst) and 2000 <= inst[i + 1][0] < 3000]
+# the QKV GEMM is the encoder layer's only bias-only (epilogue 0) GEMM
+qkv = [i for i, (k, _) in enumerate(inst) if 1000 <= k < 2000 and (k - 1000) % 64 == 0 and len(_) >= 64]
 if len(qkv) < first + nruns + 1:
     first = max(0, len(qkv) - nruns - 1)
 lo, hi = qkv[first], qkv[min(first + nruns, len(qkv) - 1)]
