@@ -343,11 +343,17 @@ __global__ void __launch_bounds__(kDThreads, 1)
           if (et == 0) {
             volatile unsigned *tk = &a.tickets[tile];
             unsigned seen = *tk;
-            if (ll)
+            if (ll) {
+              // the head CTA is resident (the grid never exceeds the SMs, and
+              // no dependent grid launches before every CTA has triggered);
+              // a bound turns a broken invariant into an error, not a hang
+              long spins = 0;
               while (seen != 1u) {
                 __nanosleep(100);
                 seen = *tk;
+                if (++spins > (1L << 24)) __trap();
               }
+            }
             *s_last = (seen == 1u) ? 3 : 0;
             if (seen == 1u) a.tickets[tile] = 0;   // both contributors accounted for: ready for the next launch
           }
