@@ -56,6 +56,8 @@ MODEL_NAME = {"ee-bert-base": "EE-BERT-base", "ee-bert-large": "EE-BERT-large", 
 
 def metric_of(cfg):
     if cfg.arch == "llama":
+        if cfg.name == "ee-llama3-8b-decode":
+            return METRIC_LM.replace("Llama-7B shape", "Llama-3.1-8B shape, GQA 8 KV heads, V 128256")
         return METRIC_LM
     return METRIC.replace("EE-BERT-base", MODEL_NAME.get(cfg.name, cfg.name))
 

@@ -110,6 +110,16 @@ LLAMA_7B = ModelConfig(
     kv_heads=32, ctx=512, cls_gain=8.0,
 )
 
+# Llama-3.1-8B shape (SURVEY §8(f) NEXT-2's variant): grouped-query attention
+# (32 query heads over 8 KV heads), F 14336, V = 128256, RoPE theta 5e5; the
+# same four ramps and exit profile as the Llama-2-7B case
+LLAMA3_8B = ModelConfig(
+    name="ee-llama3-8b-decode", arch="llama", layers=32, hidden=4096, heads=32,
+    ffn=14336, seq=1, classes=128256, norm_eps=1e-5, ramp_layers=(7, 15, 23, 31),
+    batch=64, test="maxprob", exit_profile=(0.05, 0.10, 0.35, 0.50),
+    kv_heads=8, ctx=512, cls_gain=8.0, rope_theta=500000.0,
+)
+
 # Dependent exits (NEXT-4; PABEE): the counter-based criterion
 # with patience t (DESIGN R26).  TINY_PABEE: tiny dims, a ramp after every
 # layer; BERT_BASE_PABEE: EE-BERT-base's shape and weights, patience 2.
@@ -125,10 +135,11 @@ BERT_BASE_PABEE = ModelConfig(
     test="patience", tau=(2.0,) * 12,
 )
 
-CONFIGS = {c.name: c for c in (TINY, TINY_VIT, BERT_BASE, BERT_LARGE, VIT_BASE, TINY_LLAMA, LLAMA_7B,
+CONFIGS = {c.name: c for c in (TINY, TINY_VIT, BERT_BASE, BERT_LARGE, VIT_BASE, TINY_LLAMA, LLAMA_7B, LLAMA3_8B,
                                TINY_PABEE, BERT_BASE_PABEE)}
 ALIASES = {"t": "tiny", "tv": "tiny-vit", "tl": "tiny-llama", "bb": "ee-bert-base", "bl": "ee-bert-large",
-           "vt": "ee-vit-b16", "lm": "ee-llama-7b-decode", "tp": "tiny-pabee", "bbp": "ee-bert-base-pabee"}
+           "vt": "ee-vit-b16", "lm": "ee-llama-7b-decode", "l8": "ee-llama3-8b-decode", "tp": "tiny-pabee",
+           "bbp": "ee-bert-base-pabee"}
 
 
 def get(name: str) -> ModelConfig:

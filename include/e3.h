@@ -106,6 +106,8 @@ typedef struct e3_split_desc {
   int32_t final_ramp;
   int32_t inner;       /* e3_inner                                              */
   int32_t batch;       /* constant batch B (rows per run)                       */
+  float rope_theta;    /* LLAMA: RoPE base (Llama-2 10000, Llama-3 500000);
+                          <= 0 means 10000                                      */
 } e3_split_desc;
 
 typedef struct e3_layer_weights {

@@ -45,7 +45,7 @@ class SplitDesc(C.Structure):
                 ("norm_eps", C.c_float), ("layer_begin", I32), ("layer_end", I32), ("n_ramps", I32),
                 ("ramp_layer", I32 * E3_MAX_RAMPS), ("ramp_index", I32 * E3_MAX_RAMPS),
                 ("tau", C.c_float * E3_MAX_RAMPS), ("test", I32), ("final_ramp", I32),
-                ("inner", I32), ("batch", I32)]
+                ("inner", I32), ("batch", I32), ("rope_theta", C.c_float)]
 
 
 class LayerWeights(C.Structure):

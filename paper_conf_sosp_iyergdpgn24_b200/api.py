@@ -123,6 +123,7 @@ def split_desc(cfg, begin: int, end: int, tau, batch: Optional[int] = None,
     d.final_ramp = int(bool(rs) and rs[-1][0] == cfg.n_ramps - 1)
     d.inner = _lib.INNER[inner]
     d.batch = cfg.batch if batch is None else batch
+    d.rope_theta = float(getattr(cfg, "rope_theta", 10000.0))
     return d
 
 

@@ -242,7 +242,7 @@ static e3_status llama_create(e3_split *s, const e3_weights *w) {
     s->kv_v.push_back(w->kv->v[l]);
   }
   if (d.dtype == E3_DTYPE_FP32)   // SIMT fp32 kernels: only the RoPE table
-    return ws.ensure_llama(V, 0, 0, w->kv->max_ctx, 128, 10000.0);
+    return ws.ensure_llama(V, 0, 0, w->kv->max_ctx, 128, d.rope_theta > 0.f ? d.rope_theta : 10000.0);
   s->mc_qkv = dec_max_contrib(nqkv, H, E3_DEC_QKV_ROPE, s->sms);
   s->mc_o = dec_max_contrib(H, H, E3_DEC_RESID, s->sms);
   s->mc_gu = dec_max_contrib(F, H, E3_DEC_SWIGLU, s->sms);
@@ -260,7 +260,7 @@ static e3_status llama_create(e3_split *s, const e3_weights *w) {
   need(H, s->mc_down, E3_DEC_RESID);
   need(V, s->mc_lm, E3_DEC_LOGITS);
   if ((size_t)4 * B * H > part) part = (size_t)4 * B * H;   // split-K-by-4 partials (E3_DEC_PARTIAL), reused
-  e3_status st = ws.ensure_llama(V, part, tickets, w->kv->max_ctx, 128, 10000.0);
+  e3_status st = ws.ensure_llama(V, part, tickets, w->kv->max_ctx, 128, d.rope_theta > 0.f ? d.rope_theta : 10000.0);
   if (st != E3_OK) return st;
   const int nl = d.layer_end - d.layer_begin;
   s->dmaps.resize(nl);

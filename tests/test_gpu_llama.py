@@ -154,11 +154,14 @@ class _LazyLayers:
         return self.n
 
 
-def test_llama7b_shape_split_parity_sampled(api):
+@pytest.mark.parametrize("name", ["lm", "l8"])
+def test_llama7b_shape_split_parity_sampled(api, name):
     """Llama-2-7B layer shapes (H 4096, 32 heads x 128, F 11008, V 32000,
-    513 cache positions, B = 64) on a 2-layer model (ramps after both):
-    split [0,1) on a full batch, sampled tokens vs the oracle."""
-    cfg = dataclasses.replace(e3data.get("lm"), layers=2, ramp_layers=(0, 1), exit_profile=None, tau=(0.2, 0.2))
+    513 cache positions, B = 64) -- and the Llama-3.1-8B variant (32 query
+    heads over 8 KV heads, F 14336, V 128256, RoPE base 5e5) -- on a 2-layer
+    model (ramps after both): split [0,1) on a full batch, sampled tokens vs
+    the oracle."""
+    cfg = dataclasses.replace(e3data.get(name), layers=2, ramp_layers=(0, 1), exit_profile=None, tau=(0.2, 0.2))
     B = cfg.batch
     slot_of = {i: i for i in range(B)}
     pos_of = {s: cfg.ctx for s in range(B)}
