@@ -202,7 +202,9 @@ __global__ void __launch_bounds__(kRT) f32_ramp_kernel(RampArgs a) {
   const int H = a.H, C = a.C;
   float *c = rs;          // [H] CLS row (ViT: normalised)
   float *p = c + H;       // [H] pooler output (BERT)
-  float *z = p + H;       // [C] logits
+  // [C] logits: shared memory, or this row's slice of a global scratch
+  // (a.pool_ws, [B][C]) when C does not fit (Llama-3 vocabulary, 128256)
+  float *z = a.pool_ws ? a.pool_ws + (size_t)blockIdx.x * C : p + H;
   __shared__ double red[kRT / 32][3];
   __shared__ int redi[kRT / 32];
   const int b = blockIdx.x, tid = threadIdx.x, warp = warp_id(), lane = lane_id();
@@ -539,7 +541,8 @@ e3_status f32_ln_run(const float *x, const void *g, const void *b, float *y, int
 }
 
 e3_status f32_ramp_run(const RampArgs &a, cudaStream_t st) {
-  const size_t smem = (2 * (size_t)a.H + a.C) * sizeof(float);
+  // a.pool_ws: global [B][C] logits scratch (large vocabularies), else shared memory
+  const size_t smem = (2 * (size_t)a.H + (a.pool_ws ? 0 : a.C)) * sizeof(float);
   static size_t attr = 0;
   if (smem > 48 * 1024 && smem > attr) {
     E3_CUDA_TRY(cudaFuncSetAttribute(f32_ramp_kernel, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem));

@@ -93,7 +93,8 @@ e3_status Workspace::create(int device, int B, int S, int H, int F, int elem, st
   ws->F = F;
   ws->elem = elem;
   const size_t M = (size_t)B * S, e = (size_t)elem;
-  E3_CUDA_TRY(cudaMalloc(&ws->qkv, M * 3 * H * e));
+  // qkv [M, 3H]; also the FP32 LLaMA decode's SwiGLU gate [M, F] (Llama-3: F = 3.5 H)
+  E3_CUDA_TRY(cudaMalloc(&ws->qkv, M * (size_t)(3 * H > F ? 3 * H : F) * e));
   E3_CUDA_TRY(cudaMalloc(&ws->ctx, M * H * e));
   E3_CUDA_TRY(cudaMalloc(&ws->y, M * H * e));
   E3_CUDA_TRY(cudaMalloc(&ws->x1, M * H * e));
@@ -124,10 +125,6 @@ static bool aligned16(const void *p) { return (reinterpret_cast<uintptr_t>(p) & 
 static e3_status llama_validate(const e3_split_desc *d, const e3_weights *w) {
   if (d->dtype != E3_DTYPE_BF16 && d->dtype != E3_DTYPE_FP32) {
     set_error("e3_split_create (LLAMA): dtype must be BF16 or FP32");
-    return E3_EUNSUPPORTED;
-  }
-  if (d->dtype == E3_DTYPE_FP32 && d->ffn > 3 * d->hidden) {
-    set_error("e3_split_create (LLAMA FP32): need F <= 3 H");
     return E3_EUNSUPPORTED;
   }
   const int kvh = d->kv_heads > 0 ? d->kv_heads : d->heads;
@@ -241,8 +238,8 @@ static e3_status llama_create(e3_split *s, const e3_weights *w) {
     s->kv_k.push_back(w->kv->k[l]);
     s->kv_v.push_back(w->kv->v[l]);
   }
-  if (d.dtype == E3_DTYPE_FP32)   // SIMT fp32 kernels: only the RoPE table
-    return ws.ensure_llama(V, 0, 0, w->kv->max_ctx, 128, d.rope_theta > 0.f ? d.rope_theta : 10000.0);
+  if (d.dtype == E3_DTYPE_FP32)   // SIMT fp32 kernels: the RoPE table, and a [B][V] logits scratch for the ramp
+    return ws.ensure_llama(V, (size_t)B * V, 0, w->kv->max_ctx, 128, d.rope_theta > 0.f ? d.rope_theta : 10000.0);
   s->mc_qkv = dec_max_contrib(nqkv, H, E3_DEC_QKV_ROPE, s->sms);
   s->mc_o = dec_max_contrib(H, H, E3_DEC_RESID, s->sms);
   s->mc_gu = dec_max_contrib(F, H, E3_DEC_SWIGLU, s->sms);
@@ -672,6 +669,15 @@ static e3_status f32_run(e3_split *s, cudaStream_t st, const void *x_in, const i
         a.n_valid_dev = n_valid_dev;
         a.n_valid_host = n_valid_host;
         a.ex = exits;
+        // logits that do not fit shared memory next to two H rows: the
+        // decode GEMMs' partial scratch, sized [B][C] for FP32 (llama_create)
+        if ((2 * (size_t)H + a.C) * 4 > 200 * 1024) {
+          if (!ws.dec_part || ws.part_elems < (size_t)B * a.C) {
+            set_error("FP32 ramp: no logits scratch for C classes");
+            return E3_EUNSUPPORTED;
+          }
+          a.pool_ws = ws.dec_part;
+        }
         E3_RUN(f32_ramp_run(a, st));
         first_ramp = false;
       }

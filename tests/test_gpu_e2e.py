@@ -57,18 +57,24 @@ def test_bf16_whole_job_every_input(api, name):
     assert set(gpu["exit_layer"].tolist()) <= set(cfg.ramp_layers)
 
 
-def test_bf16_llama7b_calibrated_32_layer_chain(api):
+@pytest.mark.parametrize("name", ["lm", "l8"])
+def test_bf16_llama7b_calibrated_32_layer_chain(api, name):
     """Llama-7B shape, all 32 layers in the calibrated 4-split chain (ramps
     after layers 8/16/24/32, B = 64), 16 tokens at different positions.
     bf16 over 32 decode layers: measured r02 logit error p50 0.67, max 0.90
     (vs the emulator; emulator vs fp64 is of the same size) and one decision
     flip at margin > 1e-3 among 16 tokens -- the chaotic drift of a 32-layer
-    residual stream; the same chain is held to 1e-4 in FP32 mode."""
-    cfg = e3data.get("lm")
+    residual stream; the same chain is held to 1e-4 in FP32 mode.  l8: the
+    Llama-3.1-8B shape (GQA 32 / 8 heads, V 128256, RoPE base 5e5), measured
+    on B200: 3 flips among 16 tokens vs the bf16 emulator (1 vs fp64), logit
+    error p50 0.73, max 0.95 -- the same drift; its FP32 chain meets 1e-4
+    (tests/test_gpu_fp32.py)."""
+    cfg = e3data.get(name)
     gpu, recs = pu.llama_job(api, cfg, 16, "bf16", ("bf16",))
     st = pu.compare(gpu, recs["bf16"])
-    assert st["flips"] <= 1, st
-    assert st["same_layer"] >= 14
+    max_flips = {"lm": 1, "l8": 3}[name]
+    assert st["flips"] <= max_flips, st
+    assert st["same_layer"] >= 16 - max_flips - 1
     assert st["logit_err"]["p50"] < 1.0 and st["logit_err"]["max"] < 1.5
     assert set(gpu["exit_layer"].tolist()) <= set(cfg.ramp_layers)
 

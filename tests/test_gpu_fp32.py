@@ -132,11 +132,13 @@ def test_fp32_tiny_llama_pipeline(api):
     _assert_job(gpu, recs["fp64"])
 
 
-def test_fp32_llama7b_calibrated_32_layer_chain(api):
+@pytest.mark.parametrize("name", ["lm", "l8"])
+def test_fp32_llama7b_calibrated_32_layer_chain(api, name):
     """Llama-7B shape: 16 tokens through the calibrated 4-split, 32-layer
     chain (ramps after layers 8/16/24/32, V = 32000) in FP32 vs the fp64
-    oracle: decisions exact at margin > 1e-3, logits within 1e-4."""
-    cfg = e3data.get("lm")
+    oracle: decisions exact at margin > 1e-3, logits within 1e-4.  l8: the
+    Llama-3.1-8B shape (GQA 32 / 8 heads, V 128256, RoPE base 5e5)."""
+    cfg = e3data.get(name)
     gpu, recs = pu.llama_job(api, cfg, 16, "fp32", ("fp64",))
     st = pu.compare(gpu, recs["fp64"], MARGIN)
     assert st["flips"] == 0, st
