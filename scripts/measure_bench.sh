@@ -7,6 +7,7 @@ timeout 900 python bench.py > gpurun_out/r02_bench_bb.json 2> gpurun_out/r02_ben
 timeout 600 python bench.py --impl reference --steps 2 --warmup 1 > gpurun_out/r02_bench_ref.json 2> gpurun_out/r02_bench_ref.err
 for c in tiny bl vt; do timeout 900 python bench.py --config $c > gpurun_out/r02_bench_$c.json 2> gpurun_out/r02_bench_$c.err; echo $c=$?; done
 timeout 1200 python bench.py --config lm > gpurun_out/r02_bench_lm.json 2> gpurun_out/r02_bench_lm.err; echo lm=$?
+timeout 1200 python bench.py --config l8 > gpurun_out/r02_bench_l8.json 2> gpurun_out/r02_bench_l8.err; echo l8=$?
 timeout 900 python bench.py --config lm --decode-steps 4 --steps 3 --no-cpu > gpurun_out/r02_bench_lm_decode4.json 2> gpurun_out/r02_bench_lm_decode4.err
 timeout 600 python bench.py --config bbp --no-cpu > gpurun_out/r02_bench_bbp.json 2> gpurun_out/r02_bench_bbp.err
 timeout 600 python bench.py --plan cut6 --no-cpu > gpurun_out/r02_bench_bb_cut6.json 2> gpurun_out/r02_bench_bb_cut6.err
