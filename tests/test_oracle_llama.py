@@ -26,11 +26,15 @@ def _rand_layer(cfg, rng):
             "ln1_g": 1 + 0.1 * rng.standard_normal(H), "ln2_g": 1 + 0.1 * rng.standard_normal(H)}
 
 
-@pytest.mark.parametrize("kvh", [2, 1])
-def test_decode_layer_matches_transformers_llama_layer(kvh):
+@pytest.mark.parametrize("nh,kvh,theta", [(2, 2, None), (2, 1, None), (4, 1, 500000.0)])
+def test_decode_layer_matches_transformers_llama_layer(nh, kvh, theta):
+    """(4, 1, 5e5): a group of four query heads per KV head and the Llama-3
+    RoPE base, as in the Llama-3.1-8B-shaped config (e3data l8)."""
     from transformers import DynamicCache, LlamaConfig
     from transformers.models.llama import modeling_llama as ml
-    cfg = _cfg(kvh=kvh)
+    cfg = _cfg(H=32 * nh, nh=nh, kvh=kvh)
+    if theta is not None:
+        cfg = dataclasses.replace(cfg, rope_theta=theta)
     H, nh, d, T = cfg.hidden, cfg.heads, cfg.head_dim, 7
     rng = np.random.default_rng(kvh)
     W = _rand_layer(cfg, rng)
